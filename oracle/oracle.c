@@ -1,0 +1,435 @@
+/*
+ * GROPHECY++ CPU ORACLE — TEST INFRASTRUCTURE ONLY (see oracle.h).
+ * Plain C11; build: gcc -O2 -std=c11 -ffp-contract=off -fno-fast-math -fPIC -shared -pthread
+ * Every function cites the PAPER.md passage (P:Lnnn) or DESIGN.md reading it follows.
+ */
+#include "oracle.h"
+
+#include <math.h>
+#include <pthread.h>
+#include <stdlib.h>
+#include <string.h>
+
+#define OR_INF_K 0x7fffffff   /* "no kernel" = +infinity for fr / fw */
+
+/* min(a, b) = a < b ? a : b  (N1; never fmin) */
+static double dmin(double a, double b) { return a < b ? a : b; }
+static int64_t imin64(int64_t a, int64_t b) { return a < b ? a : b; }
+static int64_t imax64(int64_t a, int64_t b) { return a > b ? a : b; }
+static uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+
+/* ------------------------------------------------------------------------ */
+/* PCIe model — §III-C.  Eq. (1): T(d) = alpha + beta*d.           */
+/* Fit: alpha = t_S (1-byte transfer), beta = t_L / s_L.            */
+/* ------------------------------------------------------------------------ */
+int oracle_fit_pcie(double t_small, double t_large, uint64_t large_bytes, or_link *out)
+{
+    if (!out || !isfinite(t_small) || !isfinite(t_large) || t_small < 0.0 ||
+        t_large <= 0.0 || large_bytes == 0)
+        return -1;
+    out->alpha = t_small;
+    out->beta = t_large / (double)large_bytes;
+    return 0;
+}
+
+/* Eq. (1); a zero-byte "transfer" is no transfer (reading 9). */
+double oracle_pcie_time(const or_link *l, uint64_t bytes)
+{
+    if (bytes == 0) return 0.0;
+    return l->alpha + l->beta * (double)bytes;
+}
+
+/* Size-affine value (N2): c0 + floor((c1 nx + c2 ny + c3 nx ny) / 8). */
+int64_t oracle_affine8(const or_affine8 *a, int64_t nx, int64_t ny)
+{
+    int64_t num = (int64_t)a->c1 * nx + (int64_t)a->c2 * ny + (int64_t)a->c3 * nx * ny;
+    int64_t q = num / 8;
+    if (num % 8 != 0 && num < 0) q -= 1;   /* floor, not truncation */
+    return (int64_t)a->c0 + q;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Data usage — §III-B, N4.                            */
+/* ------------------------------------------------------------------------ */
+
+/* The BRS of one region instantiated at (nx, ny), clamped to the array. */
+static void region_box(const or_region *g, int64_t R, int64_t C, int64_t nx, int64_t ny,
+                       int64_t *r0, int64_t *r1, int64_t *c0, int64_t *c1)
+{
+    if (g->whole) {                     /* irregular: whole array */
+        *r0 = 0; *r1 = R; *c0 = 0; *c1 = C;
+        return;
+    }
+    *r0 = imin64(imax64(oracle_affine8(&g->r0, nx, ny), 0), R);
+    *r1 = imin64(imax64(oracle_affine8(&g->r1, nx, ny), 0), R);
+    *c0 = imin64(imax64(oracle_affine8(&g->c0, nx, ny), 0), C);
+    *c1 = imin64(imax64(oracle_affine8(&g->c1, nx, ny), 0), C);
+}
+
+static int cmp_i64(const void *a, const void *b)
+{
+    int64_t x = *(const int64_t *)a, y = *(const int64_t *)b;
+    return (x > y) - (x < y);
+}
+
+static int sort_unique(int64_t *v, int n)
+{
+    qsort(v, (size_t)n, sizeof(int64_t), cmp_i64);
+    int m = 0;
+    for (int i = 0; i < n; i++)
+        if (m == 0 || v[i] != v[m - 1]) v[m++] = v[i];
+    return m;
+}
+
+/*
+ * For every element e of array a:  fr(e) = first kernel reading e,
+ * fw(e) = first kernel writing e (program order).
+ *   H2D_a = elem_bytes * |{e : fr(e) < inf and fr(e) <= fw(e)}|
+ *           ("read but not previously written"; a kernel's reads see the
+ *            state before its own writes, reading 7)
+ *   D2H_a = [live-out] * elem_bytes * |{e : fw(e) < inf}|
+ *           ("union of all written BRSs", minus temporaries)
+ * Cell method: the row/column breakpoints of all boxes cut the array into
+ * cells that every box either contains or misses; fr/fw are constant per cell.
+ */
+void oracle_usage(const or_skeleton *s, int64_t nx, int64_t ny,
+                  uint64_t *h2d_per_array, uint64_t *d2h_per_array)
+{
+    int nreg = (int)s->n_regions;
+    int64_t *rb = (int64_t *)malloc(sizeof(int64_t) * (size_t)(2 * nreg + 2));
+    int64_t *cb = (int64_t *)malloc(sizeof(int64_t) * (size_t)(2 * nreg + 2));
+    int64_t *box = (int64_t *)malloc(sizeof(int64_t) * (size_t)(4 * nreg + 4));
+    for (uint32_t a = 0; a < s->n_arrays; a++) {
+        const or_array *A = &s->arrays[a];
+        int64_t R = imax64(0, oracle_affine8(&A->rows, nx, ny));
+        int64_t C = imax64(0, oracle_affine8(&A->cols, nx, ny));
+        int nr = 0, nc = 0;
+        rb[nr++] = 0; rb[nr++] = R;
+        cb[nc++] = 0; cb[nc++] = C;
+        for (int j = 0; j < nreg; j++) {
+            const or_region *g = &s->regions[j];
+            if (g->array != a) continue;
+            region_box(g, R, C, nx, ny, &box[4 * j], &box[4 * j + 1], &box[4 * j + 2], &box[4 * j + 3]);
+            rb[nr++] = box[4 * j]; rb[nr++] = box[4 * j + 1];
+            cb[nc++] = box[4 * j + 2]; cb[nc++] = box[4 * j + 3];
+        }
+        nr = sort_unique(rb, nr);
+        nc = sort_unique(cb, nc);
+        uint64_t h = 0, d = 0;
+        for (int i = 0; i + 1 < nr; i++) {
+            for (int jj = 0; jj + 1 < nc; jj++) {
+                int64_t y0 = rb[i], y1 = rb[i + 1], x0 = cb[jj], x1 = cb[jj + 1];
+                int fr = OR_INF_K, fw = OR_INF_K;
+                for (int j = 0; j < nreg; j++) {
+                    const or_region *g = &s->regions[j];
+                    if (g->array != a) continue;
+                    const int64_t *b = &box[4 * j];
+                    if (b[0] <= y0 && y1 <= b[1] && b[2] <= x0 && x1 <= b[3]) {
+                        if ((g->mode & 1u) && (int)g->kernel < fr) fr = (int)g->kernel;
+                        if ((g->mode & 2u) && (int)g->kernel < fw) fw = (int)g->kernel;
+                    }
+                }
+                uint64_t area = (uint64_t)(y1 - y0) * (uint64_t)(x1 - x0);
+                if (fr != OR_INF_K && fr <= fw) h += area;
+                if (fw != OR_INF_K) d += area;
+            }
+        }
+        h2d_per_array[a] = h * A->elem_bytes;
+        d2h_per_array[a] = A->liveout ? d * A->elem_bytes : 0;
+    }
+    free(rb); free(cb); free(box);
+}
+
+/* The literal per-element definition (test-only; R*C <= 2^20 per array). */
+int oracle_bitmap_usage(const or_skeleton *s, int64_t nx, int64_t ny,
+                        uint64_t *h2d_per_array, uint64_t *d2h_per_array)
+{
+    for (uint32_t a = 0; a < s->n_arrays; a++) {
+        const or_array *A = &s->arrays[a];
+        int64_t R = imax64(0, oracle_affine8(&A->rows, nx, ny));
+        int64_t C = imax64(0, oracle_affine8(&A->cols, nx, ny));
+        if (R * C > (1 << 20)) return -1;
+        uint64_t h = 0, d = 0;
+        for (int64_t r = 0; r < R; r++) {
+            for (int64_t c = 0; c < C; c++) {
+                int fr = OR_INF_K, fw = OR_INF_K;
+                for (uint32_t j = 0; j < s->n_regions; j++) {
+                    const or_region *g = &s->regions[j];
+                    if (g->array != a) continue;
+                    int64_t r0, r1, c0, c1;
+                    region_box(g, R, C, nx, ny, &r0, &r1, &c0, &c1);
+                    if (r0 <= r && r < r1 && c0 <= c && c < c1) {
+                        if ((g->mode & 1u) && (int)g->kernel < fr) fr = (int)g->kernel;
+                        if ((g->mode & 2u) && (int)g->kernel < fw) fw = (int)g->kernel;
+                    }
+                }
+                if (fr != OR_INF_K && fr <= fw) h += 1;
+                if (fw != OR_INF_K) d += 1;
+            }
+        }
+        h2d_per_array[a] = h * A->elem_bytes;
+        d2h_per_array[a] = A->liveout ? d * A->elem_bytes : 0;
+    }
+    return 0;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Kernel-time projection.  The paper defers to GROPHECY [15] (P:L13, L67,   */
+/* L123) whose GPU model is Hong & Kim's MWP/CWP model [6].   */
+/* The formula is absent from PAPER.md; DESIGN.md §3 N5 writes down the      */
+/* reading implemented here, step by step, in H&K's notation.               */
+/* regime: 0 = no work, 1/2/3 = H&K case, 4 = no memory insts, -1 = infeasible */
+/* ------------------------------------------------------------------------ */
+double oracle_kernel_time(const or_skeleton *s, const or_gpu *g, uint32_t xform,
+                          uint32_t k, int64_t nx, int64_t ny, int *regime)
+{
+    const or_kx *c = &s->kx[(size_t)xform * s->n_kernels + k];
+    int dummy;
+    if (!regime) regime = &dummy;
+
+    /* occupancy: active blocks per SM (no allocation granularity) */
+    uint64_t occ;
+    if (c->tpb > g->max_tpb) {
+        occ = 0;
+    } else {
+        occ = umin64(g->max_bps, g->max_tps / c->tpb);
+        if (c->regs > 0) occ = umin64(occ, g->regs_sm / ((uint64_t)c->regs * c->tpb));
+        if (c->smem > 0) occ = umin64(occ, g->smem_sm / c->smem);
+    }
+    uint64_t wpb = c->tpb / g->warp_size + (c->tpb % g->warp_size != 0);
+    uint64_t ipb = (uint64_t)c->tpb * c->ipt;
+    double mem = c->coal + c->uncoal;                   /* #Mem_insts */
+    double comp = g->issue * c->total;                  /* Comp_cycles */
+
+    int64_t Wi = oracle_affine8(&s->kernels[k].work, nx, ny);
+    uint64_t W = Wi > 0 ? (uint64_t)Wi : 0;             /* work items */
+    if (occ == 0) { *regime = -1; return INFINITY; }
+    uint64_t blocks = W / ipb + (W % ipb != 0);
+    if (blocks == 0) { *regime = 0; return 0.0; }
+    uint64_t asm_ = umin64(g->n_sm, blocks);            /* #Active_SMs */
+    uint64_t abps = umin64(occ, blocks / asm_ + (blocks % asm_ != 0)); /* active blocks/SM */
+    double N = (double)(abps * wpb);                    /* active warps per SM */
+    double rep = (double)blocks / (double)(abps * asm_);/* #Rep */
+    double cyc;
+    if (mem == 0.0) {
+        cyc = comp * N * rep;
+        *regime = 4;
+    } else {
+        double mlu = g->mem_ld + (c->upm - 1.0) * g->dd_uncoal;   /* Mem_L_Uncoal */
+        double mlc = g->mem_ld;                                   /* Mem_L_Coal */
+        double wu = c->uncoal / mem;
+        double wc = c->coal / mem;
+        double ml = mlu * wu + mlc * wc;                          /* Mem_L */
+        double dd = (g->dd_uncoal * c->upm) * wu + g->dd_coal * wc; /* Departure_delay */
+        double mwp0 = ml / dd;                                    /* MWP_Without_BW */
+        double bwpw = g->freq * c->lbpw / ml;                     /* BW_per_warp */
+        double bwr = g->mem_bw / bwpw;
+        double mpk = bwr / (double)asm_;                          /* MWP_peak_BW */
+        double memc = mlu * c->uncoal + mlc * c->coal;            /* Mem_cycles */
+        double cwpf = (memc + comp) / comp;                       /* CWP_full */
+        double cpm = comp / mem;
+        double mwp = dmin(dmin(mwp0, mpk), N);
+        double cwp = dmin(cwpf, N);
+        if (mwp == N && cwp == N) {
+            cyc = (memc + comp + cpm * (mwp - 1.0)) * rep;
+            *regime = 1;
+        } else if (cwp >= mwp || comp > memc) {
+            cyc = (memc * N / mwp + cpm * (mwp - 1.0)) * rep;
+            *regime = 2;
+        } else {
+            cyc = (ml + comp * N) * rep;
+            *regime = 3;
+        }
+        cyc = cyc + dd * (mwp - 1.0) * c->synch * (double)abps * rep;  /* Synch_cost */
+    }
+    return cyc / g->freq;
+}
+
+/* ------------------------------------------------------------------------ */
+/* One candidate: total GPU time = kernels + transfers;        */
+/* transfers happen once, per-iteration kernels repeat.            */
+/* ------------------------------------------------------------------------ */
+int oracle_eval_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                    const or_link *h2d_link, const or_link *d2h_link,
+                    uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters,
+                    uint64_t *h2d, uint64_t *d2h, double *t)
+{
+    uint32_t skel = skx >> 16, xform = skx & 0xffffu;
+    if (skel >= n_skels || xform >= skels[skel].n_xforms || nx < 1 || nx > (1u << 20) ||
+        ny < 1 || ny > (1u << 20) || iters < 1) {
+        *h2d = 0; *d2h = 0; *t = NAN;
+        return 0;
+    }
+    const or_skeleton *s = &skels[skel];
+    uint64_t hpa[64], dpa[64];
+    oracle_usage(s, nx, ny, hpa, dpa);
+
+    double t_iter = 0.0, t_once = 0.0;
+    for (uint32_t k = 0; k < s->n_kernels; k++) {
+        double tk = oracle_kernel_time(s, g, xform, k, nx, ny, NULL);
+        if (s->kernels[k].per_iter) t_iter = t_iter + tk;
+        else t_once = t_once + tk;
+    }
+    double t_kern = t_once + (double)iters * t_iter;
+
+    /* each array is transferred separately */
+    double t_h = 0.0, t_d = 0.0;
+    uint64_t H = 0, D = 0;
+    for (uint32_t a = 0; a < s->n_arrays; a++) {
+        if (hpa[a] > 0) t_h = t_h + oracle_pcie_time(h2d_link, hpa[a]);
+        H += hpa[a];
+    }
+    for (uint32_t a = 0; a < s->n_arrays; a++) {
+        if (dpa[a] > 0) t_d = t_d + oracle_pcie_time(d2h_link, dpa[a]);
+        D += dpa[a];
+    }
+    *h2d = H;
+    *d2h = D;
+    *t = (t_kern + t_h) + t_d;
+    return 1;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Batch drivers: a static partition over host threads (plain loop inside). */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+    const or_skeleton *skels; uint32_t n_skels; const or_gpu *g;
+    const or_link *hl, *dl;
+    const uint32_t *skx, *nx, *ny, *iters;
+    uint64_t lo, hi, index_base;
+    uint64_t *h2d, *d2h; double *t;         /* eval mode (may be NULL) */
+    or_best best;                           /* best mode partial */
+} or_job;
+
+static void *eval_worker(void *p)
+{
+    or_job *j = (or_job *)p;
+    for (uint64_t i = j->lo; i < j->hi; i++)
+        oracle_eval_one(j->skels, j->n_skels, j->g, j->hl, j->dl, j->skx[i], j->nx[i],
+                        j->ny[i], j->iters[i], &j->h2d[i], &j->d2h[i], &j->t[i]);
+    return NULL;
+}
+
+/* (t, index) lexicographic: is (ta, ia) < (tb, ib)?  (the best) */
+static int better(double ta, uint64_t ia, double tb, uint64_t ib)
+{
+    return ta < tb || (ta == tb && ia < ib);
+}
+
+static void *best_worker(void *p)
+{
+    or_job *j = (or_job *)p;
+    or_best b = {INFINITY, UINT64_MAX, 0, 0, 0, 0};
+    for (uint64_t i = j->lo; i < j->hi; i++) {
+        uint64_t h, d; double t;
+        if (!oracle_eval_one(j->skels, j->n_skels, j->g, j->hl, j->dl, j->skx[i], j->nx[i],
+                             j->ny[i], j->iters[i], &h, &d, &t)) {
+            b.n_invalid++;
+            continue;
+        }
+        b.n_valid++;
+        if (!isfinite(t)) continue;
+        uint64_t gi = j->index_base + i;
+        if (b.index == UINT64_MAX || better(t, gi, b.t_total_s, b.index)) {
+            b.t_total_s = t; b.index = gi; b.h2d_bytes = h; b.d2h_bytes = d;
+        }
+    }
+    j->best = b;
+    return NULL;
+}
+
+static void run_jobs(or_job *jobs, int nthreads, void *(*fn)(void *))
+{
+    if (nthreads <= 1) { fn(&jobs[0]); return; }
+    pthread_t *th = (pthread_t *)malloc(sizeof(pthread_t) * (size_t)nthreads);
+    for (int i = 0; i < nthreads; i++) pthread_create(&th[i], NULL, fn, &jobs[i]);
+    for (int i = 0; i < nthreads; i++) pthread_join(th[i], NULL);
+    free(th);
+}
+
+static or_job *make_jobs(int nthreads, uint64_t n, or_job proto)
+{
+    or_job *jobs = (or_job *)malloc(sizeof(or_job) * (size_t)nthreads);
+    for (int i = 0; i < nthreads; i++) {
+        jobs[i] = proto;
+        jobs[i].lo = n * (uint64_t)i / (uint64_t)nthreads;
+        jobs[i].hi = n * (uint64_t)(i + 1) / (uint64_t)nthreads;
+    }
+    return jobs;
+}
+
+void oracle_eval(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                 const or_link *h2d_link, const or_link *d2h_link,
+                 const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                 const uint32_t *iters, uint64_t n, int nthreads,
+                 uint64_t *h2d, uint64_t *d2h, double *t)
+{
+    if (nthreads < 1) nthreads = 1;
+    or_job proto;
+    memset(&proto, 0, sizeof proto);
+    proto.skels = skels; proto.n_skels = n_skels; proto.g = g;
+    proto.hl = h2d_link; proto.dl = d2h_link;
+    proto.skx = skx; proto.nx = nx; proto.ny = ny; proto.iters = iters;
+    proto.h2d = h2d; proto.d2h = d2h; proto.t = t;
+    or_job *jobs = make_jobs(nthreads, n, proto);
+    run_jobs(jobs, nthreads, eval_worker);
+    free(jobs);
+}
+
+int oracle_best(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                const or_link *h2d_link, const or_link *d2h_link,
+                const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                const uint32_t *iters, uint64_t n, uint64_t index_base,
+                int nthreads, or_best *out)
+{
+    if (nthreads < 1) nthreads = 1;
+    or_job proto;
+    memset(&proto, 0, sizeof proto);
+    proto.skels = skels; proto.n_skels = n_skels; proto.g = g;
+    proto.hl = h2d_link; proto.dl = d2h_link;
+    proto.skx = skx; proto.nx = nx; proto.ny = ny; proto.iters = iters;
+    proto.index_base = index_base;
+    or_job *jobs = make_jobs(nthreads, n, proto);
+    run_jobs(jobs, nthreads, best_worker);
+    or_best b = {INFINITY, UINT64_MAX, 0, 0, 0, 0};
+    for (int i = 0; i < nthreads; i++) {
+        or_best *p = &jobs[i].best;
+        b.n_invalid += p->n_invalid;
+        b.n_valid += p->n_valid;
+        if (p->index != UINT64_MAX &&
+            (b.index == UINT64_MAX || better(p->t_total_s, p->index, b.t_total_s, b.index))) {
+            b.t_total_s = p->t_total_s; b.index = p->index;
+            b.h2d_bytes = p->h2d_bytes; b.d2h_bytes = p->d2h_bytes;
+        }
+    }
+    free(jobs);
+    *out = b;
+    return b.index == UINT64_MAX ? -1 : 0;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Validation helpers.                                                       */
+/* ------------------------------------------------------------------------ */
+/* "error magnitude ... absolute value of the percent difference between the
+ * predicted and measured values" — returned as a fraction. */
+double oracle_error_magnitude(double predicted, double measured)
+{
+    return fabs(predicted - measured) / measured;
+}
+
+/* arithmetic mean */
+double oracle_mean(const double *v, uint64_t n)
+{
+    double s = 0.0;
+    for (uint64_t i = 0; i < n; i++) s = s + v[i];
+    return s / (double)n;
+}
+
+/* "The GPU speedup is the total CPU time divided by the total GPU time" */
+double oracle_speedup(double t_cpu, double t_gpu) { return t_cpu / t_gpu; }
+
+/* Error magnitude of a predicted speedup (Table II). */
+double oracle_speedup_error(double s_pred, double s_meas)
+{
+    return oracle_error_magnitude(s_pred, s_meas);
+}

@@ -1,0 +1,110 @@
+/*
+ * GROPHECY++ CPU ORACLE — TEST INFRASTRUCTURE ONLY.
+ *
+ * A plain, slow, obviously-correct CPU implementation of the projection the
+ * CUDA path computes.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load it.  It shares no code,
+ * header or table with paper_conf_ipps_boyermk13_b200/ (the product), and
+ * the product never loads it.
+ *
+ * Source of truth: /root/reference/PAPER.md ("P:Lnnn" = line nnn) and the
+ * readings recorded in DESIGN.md §3.
+ *
+ * Arithmetic (N1): byte counts are exact 64-bit integers; times are IEEE-754
+ * binary64 evaluated in exactly the written order (compiled with
+ * -ffp-contract=off, no fast-math).
+ *
+ * Parity status per function:
+ *   oracle_fit_pcie / oracle_pcie_time ... pinned (Eq. 1 closed form)
+ *   oracle_usage ......................... pinned (bitmap brute force, Table I sizes,
+ *                                           invariants)
+ *   oracle_bitmap_usage .................. pinned (hand-counted tiny cases)
+ *   oracle_kernel_time ................... pinned only to hand-derived closed forms
+ *                                           of OUR reading (H&K MWP/CWP): the paper
+ *                                           prints no kernel-model formula
+ *                                           ("parity unpinned" by the paper itself)
+ *   oracle_eval_one / oracle_best ........ pinned (composition identities, brute-force min)
+ *   validation helpers ................... pinned (Table II arithmetic)
+ */
+#ifndef GROPHECY_ORACLE_H
+#define GROPHECY_ORACLE_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct { int32_t c0, c1, c2, c3; } or_affine8;   /* c0 + floor((c1 nx + c2 ny + c3 nx ny)/8) */
+
+typedef struct { or_affine8 rows, cols; uint32_t elem_bytes, liveout; } or_array;
+/* mode: bit0 = read, bit1 = write.  whole != 0: the region is the whole array. */
+typedef struct { uint32_t kernel, array, mode, whole; or_affine8 r0, r1, c0, c1; } or_region;
+typedef struct { or_affine8 work; uint32_t per_iter; } or_kernel;
+typedef struct {
+    uint32_t tpb, ipt, regs, smem;
+    double total, coal, uncoal, upm, lbpw, synch;
+} or_kx;
+typedef struct {
+    uint32_t n_kernels, n_arrays, n_regions, n_xforms;
+    const or_kernel *kernels;
+    const or_array *arrays;
+    const or_region *regions;
+    const or_kx *kx;               /* [n_xforms][n_kernels] */
+} or_skeleton;
+typedef struct {
+    uint32_t n_sm, warp_size, max_tpb, max_bps, max_tps, regs_sm, smem_sm;
+    double freq, mem_bw, mem_ld, dd_coal, dd_uncoal, issue;
+} or_gpu;
+typedef struct { double alpha, beta; } or_link;
+
+/* §III-C, Eq. (1) and P:L113 */
+int     oracle_fit_pcie(double t_small, double t_large, uint64_t large_bytes, or_link *out);
+double  oracle_pcie_time(const or_link *l, uint64_t bytes);
+
+int64_t oracle_affine8(const or_affine8 *a, int64_t nx, int64_t ny);
+
+/* §III-B: per-array H2D / D2H bytes, cell method and literal bitmap. */
+void oracle_usage(const or_skeleton *s, int64_t nx, int64_t ny,
+                  uint64_t *h2d_per_array, uint64_t *d2h_per_array);
+int  oracle_bitmap_usage(const or_skeleton *s, int64_t nx, int64_t ny,
+                         uint64_t *h2d_per_array, uint64_t *d2h_per_array);
+
+/* Kernel-time projection (GROPHECY [15] / Hong & Kim [6] reading). */
+double oracle_kernel_time(const or_skeleton *s, const or_gpu *g, uint32_t xform,
+                          uint32_t k, int64_t nx, int64_t ny, int *regime);
+
+/* One candidate.  Returns 1 if the record is valid. */
+int oracle_eval_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                    const or_link *h2d_link, const or_link *d2h_link,
+                    uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters,
+                    uint64_t *h2d, uint64_t *d2h, double *t);
+
+void oracle_eval(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                 const or_link *h2d_link, const or_link *d2h_link,
+                 const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                 const uint32_t *iters, uint64_t n, int nthreads,
+                 uint64_t *h2d, uint64_t *d2h, double *t);
+
+typedef struct {
+    double t_total_s;
+    uint64_t index, h2d_bytes, d2h_bytes, n_invalid, n_valid;
+} or_best;
+
+/* argmin over valid, finite records of (t, index_base + i).
+ * Returns 0 if a best exists, -1 if none (index = UINT64_MAX). */
+int oracle_best(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                const or_link *h2d_link, const or_link *d2h_link,
+                const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                const uint32_t *iters, uint64_t n, uint64_t index_base,
+                int nthreads, or_best *out);
+
+/* Validation helpers (Table II). */
+double oracle_error_magnitude(double predicted, double measured);
+double oracle_mean(const double *v, uint64_t n);
+double oracle_speedup(double t_cpu, double t_gpu);
+double oracle_speedup_error(double s_pred, double s_meas);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
