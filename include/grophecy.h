@@ -1,0 +1,270 @@
+/*
+ * grophecy.h — C ABI of the B200-native GROPHECY++ projection engine.
+ *
+ * The engine is the data-parallel hot path of GROPHECY++ (Boyer, Meng,
+ * Kumaran, "Improving GPU Performance Prediction with Data Transfer
+ * Modeling", IPDPS 2013; /root/reference/PAPER.md, cited as P:Lnnn):
+ * for every candidate (code skeleton x transformation x problem size) it
+ *   1. analyses data usage across the kernel sequence to find the bytes that
+ *      must cross PCIe in each direction           (§III-B),
+ *   2. prices each per-array transfer with the two-measurement linear PCIe
+ *      model T(d) = alpha + beta*d                  (§III-C, Eq. (1)),
+ *   3. projects every kernel's GPU time with an MWP/CWP model (GROPHECY [15],
+ *      Hong & Kim [6]; P:L13, L67, L123 — formula read in DESIGN.md §3 N5),
+ * sums them and selects the fastest candidate.
+ *
+ * Conventions
+ *  - extern "C", plain pointers and sizes; no exceptions cross the ABI.
+ *  - Every call returns a grophecy_status (0 = OK) unless it returns a value;
+ *    grophecy_last_error() returns a thread-local message for the last
+ *    non-OK status on the calling thread.
+ *  - Bytes are uint64; times are double seconds (IEEE-754 binary64, evaluated
+ *    in the fixed order of DESIGN.md §3 — results are bitwise reproducible
+ *    and bitwise equal to the CPU oracle's).
+ *  - "DEVICE" pointers are CUDA global-memory pointers on the space's device;
+ *    "HOST" pointers are host memory (pinned where stated for speed).
+ *  - cuda_stream is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  Asynchronous calls return the LAUNCH status only.
+ *  - A grophecy_space is not thread-safe and its best-mode scratch is shared:
+ *    use one space per host thread / per concurrently-used stream.
+ */
+#ifndef GROPHECY_H
+#define GROPHECY_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GROPHECY_ABI_VERSION 1
+
+typedef enum {
+    GROPHECY_OK = 0,
+    GROPHECY_EINVAL = -1,       /* bad argument / malformed descriptor */
+    GROPHECY_ELIMIT = -2,       /* a documented size limit is exceeded */
+    GROPHECY_ECUDA = -3,        /* CUDA runtime error (message has details) */
+    GROPHECY_ENOFEASIBLE = -5,  /* best: no valid candidate with finite time */
+    GROPHECY_EBADCAND = -6      /* some records were invalid (see n_invalid) */
+} grophecy_status;
+
+/* ---------------------------------------------------------------------- */
+/* PCIe model — §III-C                                                     */
+/* ---------------------------------------------------------------------- */
+
+/* T(d) = alpha + beta*d for d > 0 bytes; T(0) = 0 (no transfer).  Eq. (1). */
+typedef struct { double alpha_s, beta_s_per_byte; } grophecy_link;
+/* Separate links per direction (Figs. 2/4 measure each direction). */
+typedef struct { grophecy_link h2d, d2h; } grophecy_pcie;
+
+/* The paper's two-measurement fit: alpha = t_small (time of a 1-byte
+ * transfer), beta = t_large / large_bytes (paper: 512 MB, read as 2^29 B).
+ * Pure host function.  EINVAL if out == NULL, t_small < 0, t_large <= 0,
+ * large_bytes == 0, or either time is not finite. */
+int grophecy_fit_pcie(double t_small_s, double t_large_s, uint64_t large_bytes,
+                      grophecy_link *out);
+
+/* Eq. (1) on the host: 0 for bytes == 0, else alpha + beta*(double)bytes. */
+double grophecy_pcie_time(const grophecy_link *link, uint64_t bytes);
+
+/* ---------------------------------------------------------------------- */
+/* Design-space description                                                */
+/* ---------------------------------------------------------------------- */
+
+/* A size-affine integer: v = c0 + floor((c1*nx + c2*ny + c3*nx*ny) / 8),
+ * evaluated in int64 (eighths keep halves/quarters of a dimension integral).
+ * |c1|,|c2|,|c3| <= 2^15. */
+typedef struct { int32_t c0, c1, c2, c3; } grophecy_affine8;
+
+enum { GROPHECY_ARRAY_LIVEOUT = 1u };   /* written data goes back to the CPU;
+                                           clear = "temporary" hint */
+enum { GROPHECY_R = 1u, GROPHECY_W = 2u };   /* region mode bits; R|W = read-modify-write */
+enum { GROPHECY_REGION_WHOLE = 1u };    /* irregular read: the whole array may be
+                                           referenced; only with mode == R */
+enum { GROPHECY_KERNEL_PER_ITER = 1u }; /* runs every iteration; else once */
+
+/* A 2-D array of rows x cols elements (row-major), extents clamped at 0. */
+typedef struct { grophecy_affine8 rows, cols; uint32_t elem_bytes, flags; } grophecy_array_desc;
+
+/* A bounded regular section: the box [r0, r1) x [c0, c1) of `array`
+ * accessed by `kernel` (program order index).  Bounds are clamped to the
+ * array; lo >= hi is empty. */
+typedef struct {
+    uint8_t kernel, array, mode, flags;
+    grophecy_affine8 r0, r1, c0, c1;
+} grophecy_region_desc;
+
+typedef struct { grophecy_affine8 work_items; uint32_t flags; } grophecy_kernel_desc;
+
+/* Characteristics of one kernel under one transformation, as GROPHECY's
+ * characteristic synthesis would supply them (DESIGN.md §3 N5):
+ * threads per block, work items per thread, registers per thread, shared
+ * memory per block, and per-thread instruction counts (total, coalesced /
+ * uncoalesced memory, uncoalesced transactions per memory warp, bytes per
+ * warp load, synchronisations). */
+typedef struct {
+    uint32_t tpb, ipt, regs_per_thread, smem_per_block;
+    double total_insts, coal_insts, uncoal_insts, uncoal_per_mw, load_bytes_per_warp,
+        synch_insts;
+} grophecy_kx_desc;
+
+/* One code skeleton: a kernel sequence, its arrays and access regions, and
+ * the characteristics table kx[x * n_kernels + k] for n_xforms transformations. */
+typedef struct {
+    uint32_t n_kernels, n_arrays, n_regions, n_xforms;
+    const grophecy_kernel_desc *kernels;
+    const grophecy_array_desc *arrays;
+    const grophecy_region_desc *regions;
+    const grophecy_kx_desc *kx;
+} grophecy_skeleton_desc;
+
+/* The modelled GPU ("configured to reflect different GPU architectures"). */
+typedef struct {
+    uint32_t n_sm, warp_size, max_threads_per_block, max_blocks_per_sm, max_threads_per_sm,
+        regs_per_sm, smem_per_sm;
+    double freq_hz, mem_bw_Bps, mem_ld_cycles, dep_del_coal, dep_del_uncoal, issue_cycles;
+} grophecy_gpu_model;
+
+/* Limits checked by grophecy_space_validate / _create (ELIMIT / EINVAL):
+ *   1 <= n_skels <= 65536; 1 <= n_xforms <= 65536; 1 <= n_kernels <= 32;
+ *   n_arrays <= 16; n_regions <= 256; <= 32 regions per array;
+ *   region.kernel < n_kernels, region.array < n_arrays, mode in {R, W, R|W},
+ *   REGION_WHOLE only with mode R (irregular writes: DESIGN.md reading 10);
+ *   1 <= tpb <= 65536, 1 <= ipt <= 65536; instruction counts finite, >= 0,
+ *   total >= coal + uncoal, uncoal_per_mw >= 1, load_bytes_per_warp > 0;
+ *   GPU integers >= 1 and GPU doubles finite and > 0; elem_bytes >= 1. */
+#define GROPHECY_MAX_SKELS 65536u
+#define GROPHECY_MAX_XFORMS 65536u
+#define GROPHECY_MAX_KERNELS 32u
+#define GROPHECY_MAX_ARRAYS 16u
+#define GROPHECY_MAX_REGIONS 256u
+#define GROPHECY_MAX_REGIONS_PER_ARRAY 32u
+#define GROPHECY_MAX_DIM (1u << 20)
+
+/* Pure host validation of a design space (no CUDA). */
+int grophecy_space_validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
+                            const grophecy_gpu_model *gpu);
+
+typedef struct grophecy_space grophecy_space;   /* opaque; owns device tables + scratch */
+
+/* Validate, precompute per-(kernel, transformation) constants on the host and
+ * upload the tables to `device`.  Copies its inputs: the caller may free
+ * them on return.  On error *out is NULL. */
+int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
+                          const grophecy_gpu_model *gpu, int device, grophecy_space **out);
+void grophecy_space_destroy(grophecy_space *space);
+
+/* ---------------------------------------------------------------------- */
+/* Candidate batches                                                       */
+/* ---------------------------------------------------------------------- */
+
+/* Struct-of-arrays candidate records, DEVICE pointers, length n, 16-byte
+ * aligned.  skx = (skeleton << 16) | transformation.  Global index of
+ * record i is index_base + i (used for tie-breaking and reported by best).
+ * A record is valid iff skeleton < n_skels, transformation < that
+ * skeleton's n_xforms, 1 <= nx, ny <= 2^20 and iters >= 1. */
+typedef struct {
+    const uint32_t *skx, *nx, *ny, *iters;
+    uint64_t n, index_base;
+} grophecy_batch;
+
+/* Project every candidate.  Outputs are DEVICE arrays of length n owned by
+ * the caller: h2d_bytes[i], d2h_bytes[i] (exact), t_total_s[i] (+inf when a
+ * transformation cannot run: zero occupancy).  Invalid records produce
+ * (0, 0, NaN) and are counted in the space's invalid counter.  Async. */
+int grophecy_eval(const grophecy_space *space, const grophecy_pcie *pcie,
+                  const grophecy_batch *batch, uint64_t *h2d_bytes, uint64_t *d2h_bytes,
+                  double *t_total_s, void *cuda_stream);
+
+/* Synchronise the stream, return the number of invalid records seen by
+ * grophecy_eval on this space since the last call, and reset the counter. */
+int grophecy_invalid_count(grophecy_space *space, uint64_t *count, void *cuda_stream);
+
+/* The selected candidate: minimum (t_total_s, index) over valid records with
+ * finite time, ties to the lowest global index.  48 bytes. */
+typedef struct {
+    double t_total_s;      /* +inf when none */
+    uint64_t index;        /* global index; UINT64_MAX when none */
+    uint64_t h2d_bytes, d2h_bytes;   /* of the selected candidate */
+    uint64_t n_invalid;    /* invalid records in the batch */
+    uint64_t n_valid;      /* valid records (finite or not) */
+} grophecy_best_result;
+
+/* Fused projection + argmin; writes one result to HOST memory and
+ * synchronises the stream.  Returns ENOFEASIBLE if nothing qualifies
+ * (result still filled), EBADCAND if n_invalid > 0 (result still filled). */
+int grophecy_best(grophecy_space *space, const grophecy_pcie *pcie,
+                  const grophecy_batch *batch, grophecy_best_result *host_out,
+                  void *cuda_stream);
+
+/* Asynchronous variant: one launch; the result lands in DEVICE memory.
+ * If accumulate != 0 the batch's result is merged (min-loc, counters summed)
+ * into the existing *device_out instead of overwriting it. */
+int grophecy_best_async(grophecy_space *space, const grophecy_pcie *pcie,
+                        const grophecy_batch *batch, grophecy_best_result *device_out,
+                        int accumulate, void *cuda_stream);
+
+/* Min-loc combine of `count` results (e.g. one per rank after an all-gather):
+ * device_in and device_out are DEVICE pointers; one tiny launch. */
+int grophecy_best_combine(const grophecy_best_result *device_in, uint32_t count,
+                          grophecy_best_result *device_out, void *cuda_stream);
+/* The same combine on the host (pure C, no CUDA). */
+int grophecy_best_combine_host(const grophecy_best_result *in, uint32_t count,
+                               grophecy_best_result *out);
+
+/* End-to-end entry point with HOST record arrays (pinned for full speed):
+ * streams the records to the device in chunks, overlapping copies with the
+ * fused projection + argmin, and returns the result in host memory.
+ * Synchronous.  Same status rules as grophecy_best. */
+int grophecy_best_host(grophecy_space *space, const grophecy_pcie *pcie,
+                       const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                       const uint32_t *iters, uint64_t n, uint64_t index_base,
+                       grophecy_best_result *host_out, void *cuda_stream);
+
+/* ---------------------------------------------------------------------- */
+/* PCIe calibration / validation subsystem      */
+/* ---------------------------------------------------------------------- */
+
+enum { GROPHECY_DIR_H2D = 0, GROPHECY_DIR_D2H = 1 };
+
+/* Time `reps` pinned cudaMemcpyAsync transfers of `bytes` in one direction on
+ * `device` (after `warmup` discarded ones).  Each transfer is issued and
+ * waited for individually.  mean_wall_s: mean host steady-clock time per
+ * transfer (what a program sees); mean_event_s: mean CUDA-event time (may be
+ * NULL).  bytes <= 2^31. */
+int grophecy_measure_transfer(int device, int direction, uint64_t bytes, int reps,
+                              int warmup, double *mean_wall_s, double *mean_event_s);
+
+/* The paper's automatic calibration: per direction, t_S = mean
+ * of `reps` 1-byte transfers and t_L = mean of `reps` transfers of
+ * large_bytes (paper: 512 MB = 2^29 B), then grophecy_fit_pcie. */
+int grophecy_calibrate(int device, int reps, uint64_t large_bytes, grophecy_pcie *out);
+
+/* ---------------------------------------------------------------------- */
+/* Synthetic workloads (bench / tests) — not part of the method             */
+/* ---------------------------------------------------------------------- */
+
+/* Per-skeleton size rule for the counter-based generator (synth/records.py
+ * documents the closed form; this is an independent CUDA implementation). */
+typedef struct { uint32_t kind, lo, hi, it_lo, it_hi, pad; } grophecy_synth_rule;
+enum { GROPHECY_SYNTH_SQUARE = 0, GROPHECY_SYNTH_INDEP = 1, GROPHECY_SYNTH_ONED = 2,
+       GROPHECY_SYNTH_FIXED = 3 };
+
+/* Generate records [start, start + count) of an n_total-record workload into
+ * DEVICE arrays.  rules is a HOST array of n_rules entries.  Async. */
+int grophecy_synth_records(const grophecy_synth_rule *rules, uint32_t n_rules,
+                           uint64_t n_total, uint32_t n_xforms, uint64_t seed, uint64_t start,
+                           uint64_t count, uint32_t *skx, uint32_t *nx, uint32_t *ny,
+                           uint32_t *iters, void *cuda_stream);
+
+/* Number of CUDA kernel launches issued by this library since load (for
+ * the bench's gpu_launches count). */
+uint64_t grophecy_launch_count(void);
+
+const char *grophecy_last_error(void);
+int grophecy_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GROPHECY_H */

@@ -1,0 +1,94 @@
+// Internal layout of a grophecy_space (host + device).  Product code only.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "grophecy.h"
+
+namespace grophecy {
+
+// Per (skeleton, kernel, transformation) constants, precomputed on the host in
+// the exact operation order of DESIGN.md §3 N5.  Stored struct-of-arrays by
+// field pair (index kxi = skel.kx_base + k * n_xforms + x) so the 16 lanes of
+// a candidate group read 16 consecutive 16-byte entries.
+//
+// "Saturated" grid: blocks >= sat_blocks  <=>  #Active_SMs == n_sm and
+// active blocks/SM == occ; then N, MWP, CWP and the H&K case are constants
+// and cyc = E*rep + S*rep with rep = blocks / D (D = occ * n_sm).
+struct KxES { double E, S; };         // case expression, synch factor
+struct KxD  { double D, rD; };        // rep denominator and RN(1/D)
+struct KxI  { uint64_t magic; uint64_t sat_blocks; };  // ceil(2^64/ipb) (0 if ipb==1)
+struct KxJ  { uint32_t ipb, occ, wpb, flags; };        // flags: KXF_*
+enum : uint32_t { KXF_INFEASIBLE = 1u, KXF_NOMEM = 2u };
+
+// General-grid constants (small grids / huge W), read only off the fast path.
+struct KxG {
+    double comp, mwp0, bwr, memc, cwpf, cpm, ml, dd, synch, pad;
+};
+
+struct SkelInfo {
+    uint32_t n_kernels, n_arrays, n_xforms, n_regions;
+    uint32_t k_base;   // into kern_work / kern_flags
+    uint32_t a_base;   // into arrays
+    uint32_t kx_base;  // into kx tables
+    uint32_t pad;
+};
+
+struct ArrayDev {
+    int4 rows, cols;
+    uint32_t elem_bytes, liveout, r_base, r_count;   // regions [r_base, r_base+r_count)
+};
+
+// Regions are stored grouped by array and sorted by kernel within an array,
+// so "first writer" = lowest set bit of a mask and upto = mask of regions of
+// the same array whose kernel <= this region's kernel.
+struct RegionDev {
+    int4 r0, r1, c0, c1;
+    uint32_t mode, whole, upto, kernel;
+};
+
+struct SpaceDev {
+    const SkelInfo *skel;
+    const int4 *kern_work;
+    const uint32_t *kern_flags;
+    const ArrayDev *arrays;
+    const RegionDev *regions;
+    const KxES *kx_es;
+    const KxD *kx_d;
+    const KxI *kx_i;
+    const KxJ *kx_j;
+    const KxG *kx_g;
+    uint32_t n_skels;
+    uint32_t n_sm;
+    double freq, rfreq;
+    unsigned long long *invalid_counter;
+};
+
+}  // namespace grophecy
+
+struct grophecy_space {
+    int device;
+    grophecy::SpaceDev dev;
+    void *blob;                          // one device allocation for all tables
+    size_t blob_bytes;
+    grophecy_best_result *partials;      // best-mode per-block partials
+    unsigned int *ticket;                // best-mode last-block counter
+    unsigned long long *invalid_counter;
+    uint32_t max_partials;
+    int grid_best, grid_eval;            // persistent grid sizes
+    // e2e host path staging
+    void *stage[2];
+    size_t stage_bytes;
+    cudaStream_t copy_stream;
+    cudaEvent_t ev_copied[2], ev_done[2];
+};
+
+namespace grophecy {
+void set_error(const std::string &msg);
+int cuda_fail(cudaError_t e, const char *what);
+void count_launch(uint64_t n = 1);
+int launch_best(grophecy_space *s, const grophecy_pcie *pcie, const grophecy_batch *b,
+                grophecy_best_result *dout, int accumulate, cudaStream_t st);
+}  // namespace grophecy

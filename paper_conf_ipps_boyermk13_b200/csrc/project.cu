@@ -1,0 +1,723 @@
+// The projection hot path for sm_100a: grophecy_eval / grophecy_best[_async]
+// / grophecy_best_combine / grophecy_best_host.
+//
+// One fused kernel per call.  Each warp takes tiles of 32 consecutive records
+// (coalesced 32-bit SoA loads).  Data usage depends only on (skeleton, nx, ny)
+// (reading 11), so the warp deduplicates keys with ballots and
+// computes the usage of each distinct key cooperatively (lanes over regions,
+// then over coordinate-compressed cells), broadcasting the result to every
+// lane with that key.  The kernel-time model then runs per lane (one
+// candidate per lane) from per-(kernel, transformation) constants that the
+// host precomputed in the definition's operation order; on saturated grids
+// the two remaining IEEE divisions use Markstein's correction
+// (q = a*rb; r = fma(-q, b, a); q' = fma(r, rb, q)), which is correctly
+// rounded when rb = RN(1/b) — bitwise the result of a / b.
+//
+// Compiled with -fmad=false: no contraction anywhere; FMAs appear only as the
+// explicit __fma_rn of the Markstein step.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+#include <cmath>
+
+#include "grophecy.h"
+#include "internal.h"
+
+namespace grophecy {
+
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int THREADS = 256;
+constexpr int WARPS = THREADS / 32;
+constexpr long long BIG = 0x7fffffffffffffffLL;
+
+__device__ __forceinline__ long long aff8(int4 c, long long nx, long long ny)
+{
+    long long num = (long long)c.y * nx + (long long)c.z * ny + (long long)c.w * nx * ny;
+    return (long long)c.x + (num >> 3);   // arithmetic shift: floor(num / 8)
+}
+
+__device__ __forceinline__ long long clampll(long long v, long long hi)
+{
+    return v < 0 ? 0 : (v > hi ? hi : v);
+}
+
+__device__ __forceinline__ double dmin(double a, double b) { return a < b ? a : b; }
+
+// Correctly rounded a / b given rb = RN(1/b) (Markstein).
+__device__ __forceinline__ double div_rn(double a, double b, double rb)
+{
+    double q = __dmul_rn(a, rb);
+    double r = __fma_rn(-q, b, a);
+    return __fma_rn(r, rb, q);
+}
+
+struct WarpScratch {
+    long long box[32][4];
+    long long rs_h[64];
+    long long cs_w[64];
+    unsigned rs_m[64];
+    unsigned cs_m[64];
+    unsigned upto[32];
+};
+
+struct Usage {
+    unsigned long long h, d;
+    double th, td;
+};
+
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+    return v;
+}
+
+// Data usage of one (skeleton, nx, ny) key, computed by the whole warp
+// (DESIGN.md §3 N4; §III-B), plus the per-array PCIe
+// transfer times in array order (Eq. (1), one transfer per array).
+__device__ Usage warp_usage(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
+                            const grophecy_pcie &pc, WarpScratch &ws, int lane)
+{
+    Usage o = {0ull, 0ull, 0.0, 0.0};
+    const unsigned lt = (1u << lane) - 1u;
+    for (uint32_t a = 0; a < I.n_arrays; a++) {
+        const ArrayDev A = S.arrays[I.a_base + a];
+        long long R = aff8(A.rows, nx, ny);
+        long long C = aff8(A.cols, nx, ny);
+        R = R > 0 ? R : 0;
+        C = C > 0 ? C : 0;
+        const int n = (int)A.r_count;
+        unsigned long long h = 0, d = 0;
+        if (n > 0 && R > 0 && C > 0) {
+            long long r0 = 0, r1 = 0, c0 = 0, c1 = 0;
+            bool valid = false;
+            unsigned mode = 0, up = 0;
+            if (lane < n) {
+                const RegionDev &g = S.regions[A.r_base + lane];
+                if (g.whole) {
+                    r1 = R;
+                    c1 = C;
+                } else {
+                    r0 = clampll(aff8(g.r0, nx, ny), R);
+                    r1 = clampll(aff8(g.r1, nx, ny), R);
+                    c0 = clampll(aff8(g.c0, nx, ny), C);
+                    c1 = clampll(aff8(g.c1, nx, ny), C);
+                }
+                valid = r0 < r1 && c0 < c1;
+                mode = g.mode;
+                up = g.upto;
+            }
+            const unsigned vm = __ballot_sync(FULL, valid);
+            const unsigned Rm = __ballot_sync(FULL, valid && (mode & GROPHECY_R));
+            const unsigned Wm = __ballot_sync(FULL, valid && (mode & GROPHECY_W));
+            if (vm) {
+                const bool full = valid && r0 == 0 && r1 == R && c0 == 0 && c1 == C;
+                const unsigned fm = __ballot_sync(FULL, full);
+                if (fm == vm) {
+                    // every access covers the whole array: one cell
+                    const int fwl = Wm ? __ffs(Wm) - 1 : 0;
+                    const unsigned upw = __shfl_sync(FULL, up, fwl);
+                    const unsigned long long area = (unsigned long long)R * (unsigned long long)C;
+                    if (Rm && (!Wm || (Rm & upw))) h = area;
+                    if (Wm) d = area;
+                } else {
+                    if (lane < n) {
+                        ws.box[lane][0] = r0;
+                        ws.box[lane][1] = r1;
+                        ws.box[lane][2] = c0;
+                        ws.box[lane][3] = c1;
+                        ws.upto[lane] = up;
+                    }
+                    __syncwarp();
+                    // elementary slabs: for each breakpoint value, is it the
+                    // first occurrence, the next larger breakpoint, and which
+                    // boxes cover [value, next)
+                    long long rn0 = BIG, rn1 = BIG, cn0 = BIG, cn1 = BIG;
+                    bool rd0 = false, rd1 = false, cd0 = false, cd1 = false;
+                    unsigned rm0 = 0, rm1 = 0, cm0 = 0, cm1 = 0;
+                    for (int i = 0; i < n; i++) {
+                        if (!((vm >> i) & 1u)) continue;
+                        const long long b0 = ws.box[i][0], b1 = ws.box[i][1];
+                        const long long b2 = ws.box[i][2], b3 = ws.box[i][3];
+                        const bool before = i < lane;
+                        rd0 |= before && (b0 == r0 || b1 == r0);
+                        rd1 |= (i <= lane && b0 == r1) || (before && b1 == r1);
+                        cd0 |= before && (b2 == c0 || b3 == c0);
+                        cd1 |= (i <= lane && b2 == c1) || (before && b3 == c1);
+                        if (b0 > r0 && b0 < rn0) rn0 = b0;
+                        if (b1 > r0 && b1 < rn0) rn0 = b1;
+                        if (b0 > r1 && b0 < rn1) rn1 = b0;
+                        if (b1 > r1 && b1 < rn1) rn1 = b1;
+                        if (b2 > c0 && b2 < cn0) cn0 = b2;
+                        if (b3 > c0 && b3 < cn0) cn0 = b3;
+                        if (b2 > c1 && b2 < cn1) cn1 = b2;
+                        if (b3 > c1 && b3 < cn1) cn1 = b3;
+                        const unsigned bit = 1u << i;
+                        if (b0 <= r0 && r0 < b1) rm0 |= bit;
+                        if (b0 <= r1 && r1 < b1) rm1 |= bit;
+                        if (b2 <= c0 && c0 < b3) cm0 |= bit;
+                        if (b2 <= c1 && c1 < b3) cm1 |= bit;
+                    }
+                    const bool sr0 = valid && !rd0 && rn0 != BIG;
+                    const bool sr1 = valid && !rd1 && rn1 != BIG;
+                    const bool sc0 = valid && !cd0 && cn0 != BIG;
+                    const bool sc1 = valid && !cd1 && cn1 != BIG;
+                    const unsigned br0 = __ballot_sync(FULL, sr0), br1 = __ballot_sync(FULL, sr1);
+                    const unsigned bc0 = __ballot_sync(FULL, sc0), bc1 = __ballot_sync(FULL, sc1);
+                    __syncwarp();
+                    if (sr0) {
+                        int p = __popc(br0 & lt);
+                        ws.rs_h[p] = rn0 - r0;
+                        ws.rs_m[p] = rm0;
+                    }
+                    if (sr1) {
+                        int p = __popc(br0) + __popc(br1 & lt);
+                        ws.rs_h[p] = rn1 - r1;
+                        ws.rs_m[p] = rm1;
+                    }
+                    if (sc0) {
+                        int p = __popc(bc0 & lt);
+                        ws.cs_w[p] = cn0 - c0;
+                        ws.cs_m[p] = cm0;
+                    }
+                    if (sc1) {
+                        int p = __popc(bc0) + __popc(bc1 & lt);
+                        ws.cs_w[p] = cn1 - c1;
+                        ws.cs_m[p] = cm1;
+                    }
+                    __syncwarp();
+                    const int Sr = __popc(br0) + __popc(br1);
+                    const int Sc = __popc(bc0) + __popc(bc1);
+                    for (int i = 0; i < Sr; i++) {
+                        const unsigned rm = ws.rs_m[i];
+                        if (!rm) continue;
+                        const unsigned long long hg = (unsigned long long)ws.rs_h[i];
+                        for (int j = lane; j < Sc; j += 32) {
+                            const unsigned m = rm & ws.cs_m[j];
+                            if (m) {
+                                const unsigned mr = m & Rm, mw = m & Wm;
+                                const unsigned long long area = hg * (unsigned long long)ws.cs_w[j];
+                                if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) h += area;
+                                if (mw) d += area;
+                            }
+                        }
+                    }
+                    h = warp_sum_u64(h);
+                    d = warp_sum_u64(d);
+                    __syncwarp();
+                }
+            }
+        }
+        const unsigned long long ha = h * (unsigned long long)A.elem_bytes;
+        const unsigned long long da = A.liveout ? d * (unsigned long long)A.elem_bytes : 0ull;
+        if (ha) o.th = __dadd_rn(o.th, __dadd_rn(pc.h2d.alpha_s,
+                                                 __dmul_rn(pc.h2d.beta_s_per_byte, (double)ha)));
+        if (da) o.td = __dadd_rn(o.td, __dadd_rn(pc.d2h.alpha_s,
+                                                 __dmul_rn(pc.d2h.beta_s_per_byte, (double)da)));
+        o.h += ha;
+        o.d += da;
+    }
+    return o;
+}
+
+// Kernel time of kernel k of skeleton I under transformation x (DESIGN.md §3 N5).
+__device__ __forceinline__ double kernel_time(const SpaceDev &S, const SkelInfo &I, uint32_t k,
+                                              uint32_t x, long long nx, long long ny)
+{
+    const long long Wi = aff8(__ldg(&S.kern_work[I.k_base + k]), nx, ny);
+    const unsigned long long W = Wi > 0 ? (unsigned long long)Wi : 0ull;
+    const uint32_t kxi = I.kx_base + k * I.n_xforms + x;
+    const KxJ J = S.kx_j[kxi];
+    if (J.flags & KXF_INFEASIBLE) return __longlong_as_double(0x7ff0000000000000LL);
+    const KxI II = S.kx_i[kxi];
+    unsigned long long blocks;
+    if (W < (1ull << 32)) {
+        const unsigned long long q = II.magic ? __umul64hi(II.magic, W) : W;
+        blocks = q + (q * J.ipb != W);
+    } else {
+        blocks = W / J.ipb + (W % J.ipb != 0);
+    }
+    if (blocks == 0) return 0.0;
+    if (blocks >= II.sat_blocks) {
+        const KxES es = S.kx_es[kxi];
+        const KxD dd = S.kx_d[kxi];
+        const double rep = div_rn(__ull2double_rn(blocks), dd.D, dd.rD);
+        const double cyc = __dadd_rn(__dmul_rn(es.E, rep), __dmul_rn(es.S, rep));
+        return div_rn(cyc, S.freq, S.rfreq);
+    }
+    // general (small) grid: the definition step by step
+    const KxG G = S.kx_g[kxi];
+    const unsigned long long nsm = S.n_sm;
+    const unsigned long long asm_ = nsm < blocks ? nsm : blocks;
+    unsigned long long abps = blocks / asm_ + (blocks % asm_ != 0);
+    if ((unsigned long long)J.occ < abps) abps = J.occ;
+    const double N = __ull2double_rn(abps * (unsigned long long)J.wpb);
+    const double rep = __ddiv_rn(__ull2double_rn(blocks), __ull2double_rn(abps * asm_));
+    double cyc;
+    if (J.flags & KXF_NOMEM) {
+        cyc = __dmul_rn(__dmul_rn(G.comp, N), rep);
+    } else {
+        const double mpk = __ddiv_rn(G.bwr, __ull2double_rn(asm_));
+        const double mwp = dmin(dmin(G.mwp0, mpk), N);
+        const double cwp = dmin(G.cwpf, N);
+        const double cpm_term = __dmul_rn(G.cpm, __dsub_rn(mwp, 1.0));
+        if (mwp == N && cwp == N)
+            cyc = __dmul_rn(__dadd_rn(__dadd_rn(G.memc, G.comp), cpm_term), rep);
+        else if (cwp >= mwp || G.comp > G.memc)
+            cyc = __dmul_rn(__dadd_rn(__ddiv_rn(__dmul_rn(G.memc, N), mwp), cpm_term), rep);
+        else
+            cyc = __dmul_rn(__dadd_rn(G.ml, __dmul_rn(G.comp, N)), rep);
+        const double sync = __dmul_rn(
+            __dmul_rn(__dmul_rn(__dmul_rn(G.dd, __dsub_rn(mwp, 1.0)), G.synch),
+                      __ull2double_rn(abps)),
+            rep);
+        cyc = __dadd_rn(cyc, sync);
+    }
+    return __ddiv_rn(cyc, S.freq);
+}
+
+struct Best {
+    double t;
+    unsigned long long i, h, d, ninv, nval;
+};
+
+__device__ __forceinline__ bool better(double ta, unsigned long long ia, double tb,
+                                       unsigned long long ib)
+{
+    return ta < tb || (ta == tb && ia < ib);
+}
+
+__device__ __forceinline__ void merge(Best &a, const Best &b)
+{
+    if (better(b.t, b.i, a.t, a.i)) {
+        a.t = b.t;
+        a.i = b.i;
+        a.h = b.h;
+        a.d = b.d;
+    }
+    a.ninv += b.ninv;
+    a.nval += b.nval;
+}
+
+__device__ __forceinline__ Best shfl_best(const Best &b, int src_xor)
+{
+    Best o;
+    o.t = __shfl_xor_sync(FULL, b.t, src_xor);
+    o.i = __shfl_xor_sync(FULL, b.i, src_xor);
+    o.h = __shfl_xor_sync(FULL, b.h, src_xor);
+    o.d = __shfl_xor_sync(FULL, b.d, src_xor);
+    o.ninv = __shfl_xor_sync(FULL, b.ninv, src_xor);
+    o.nval = __shfl_xor_sync(FULL, b.nval, src_xor);
+    return o;
+}
+
+__device__ __forceinline__ Best warp_best(Best b)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) merge(b, shfl_best(b, o));
+    return b;
+}
+
+__device__ __forceinline__ Best none_best()
+{
+    Best b;
+    b.t = __longlong_as_double(0x7ff0000000000000LL);
+    b.i = ~0ull;
+    b.h = b.d = b.ninv = b.nval = 0;
+    return b;
+}
+
+__device__ __forceinline__ Best from_result(const grophecy_best_result &r)
+{
+    Best b;
+    b.t = r.t_total_s;
+    b.i = r.index;
+    b.h = r.h2d_bytes;
+    b.d = r.d2h_bytes;
+    b.ninv = r.n_invalid;
+    b.nval = r.n_valid;
+    return b;
+}
+
+__device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b)
+{
+    r.t_total_s = b.t;
+    r.index = b.i;
+    r.h2d_bytes = b.h;
+    r.d2h_bytes = b.d;
+    r.n_invalid = b.ninv;
+    r.n_valid = b.nval;
+}
+
+struct Params {
+    SpaceDev S;
+    grophecy_pcie pc;
+    const uint32_t *skx, *nx, *ny, *iters;
+    unsigned long long n, base;
+    unsigned long long *h2d;
+    unsigned long long *d2h;
+    double *t;
+    grophecy_best_result *partials;
+    unsigned int *ticket;
+    grophecy_best_result *out;
+    int accumulate;
+};
+
+template <bool BEST>
+__global__ void __launch_bounds__(THREADS) project_kernel(const Params P)
+{
+    __shared__ WarpScratch scratch[WARPS];
+    __shared__ Best wbest[WARPS];
+    __shared__ bool am_last;
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    WarpScratch &ws = scratch[warp];
+    const SpaceDev &S = P.S;
+
+    Best mine = none_best();
+    const unsigned long long ntiles = (P.n + 31) >> 5;
+    const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
+    for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
+         tile += wstride) {
+        const unsigned long long i = (tile << 5) + lane;
+        const bool has = i < P.n;
+        uint32_t skx = 0, nx = 0, ny = 0, it = 0;
+        if (has) {
+            skx = __ldcs(P.skx + i);
+            nx = __ldcs(P.nx + i);
+            ny = __ldcs(P.ny + i);
+            it = __ldcs(P.iters + i);
+        }
+        const uint32_t skel = skx >> 16, x = skx & 0xffffu;
+        bool valid = has && skel < S.n_skels && nx >= 1 && nx <= GROPHECY_MAX_DIM && ny >= 1 &&
+                     ny <= GROPHECY_MAX_DIM && it >= 1;
+        SkelInfo I = {0, 0, 0, 0, 0, 0, 0, 0};
+        if (valid) {
+            I = S.skel[skel];
+            valid = x < I.n_xforms;
+        }
+        const unsigned long long key =
+            valid ? ((unsigned long long)skel << 42) | ((unsigned long long)nx << 21) | ny : ~0ull;
+        unsigned pending = __ballot_sync(FULL, valid);
+        Usage u = {0ull, 0ull, 0.0, 0.0};
+        while (pending) {
+            const int L = __ffs(pending) - 1;
+            const unsigned long long kL = __shfl_sync(FULL, key, L);
+            const unsigned same = __ballot_sync(FULL, key == kL);
+            const uint32_t sL = (uint32_t)(kL >> 42);
+            const long long nxL = (long long)((kL >> 21) & 0x1fffffull);
+            const long long nyL = (long long)(kL & 0x1fffffull);
+            const SkelInfo IL = S.skel[sL];
+            const Usage r = warp_usage(S, IL, nxL, nyL, P.pc, ws, lane);
+            if (key == kL) u = r;
+            pending &= ~same;
+        }
+        double t = __longlong_as_double(0x7ff8000000000000LL);   // NaN for invalid
+        if (valid) {
+            double t_iter = 0.0, t_once = 0.0;
+            for (uint32_t k = 0; k < I.n_kernels; k++) {
+                const double tk = kernel_time(S, I, k, x, nx, ny);
+                if (__ldg(&S.kern_flags[I.k_base + k]) & GROPHECY_KERNEL_PER_ITER)
+                    t_iter = __dadd_rn(t_iter, tk);
+                else
+                    t_once = __dadd_rn(t_once, tk);
+            }
+            const double t_kern = __dadd_rn(t_once, __dmul_rn((double)it, t_iter));
+            t = __dadd_rn(__dadd_rn(t_kern, u.th), u.td);
+        }
+        if (!BEST) {
+            if (has) {
+                __stcs(P.h2d + i, valid ? u.h : 0ull);
+                __stcs(P.d2h + i, valid ? u.d : 0ull);
+                __stcs(P.t + i, t);
+            }
+            const unsigned inv = __ballot_sync(FULL, has && !valid);
+            if (lane == 0 && inv) atomicAdd(S.invalid_counter, (unsigned long long)__popc(inv));
+        } else {
+            if (has) {
+                if (!valid) {
+                    mine.ninv++;
+                } else {
+                    mine.nval++;
+                    if (t < __longlong_as_double(0x7ff0000000000000LL) &&
+                        better(t, P.base + i, mine.t, mine.i)) {
+                        mine.t = t;
+                        mine.i = P.base + i;
+                        mine.h = u.h;
+                        mine.d = u.d;
+                    }
+                }
+            }
+        }
+    }
+    if (!BEST) return;
+
+    // ---- argmin: warp -> CTA -> grid (last-block pattern) ----
+    mine = warp_best(mine);
+    if (lane == 0) wbest[warp] = mine;
+    __syncthreads();
+    if (warp == 0) {
+        Best b = lane < WARPS ? wbest[lane] : none_best();
+        b = warp_best(b);
+        if (lane == 0) {
+            to_result(P.partials[blockIdx.x], b);
+            __threadfence();
+            const unsigned prev = atomicAdd(P.ticket, 1u);
+            am_last = prev == gridDim.x - 1;
+        }
+    }
+    __syncthreads();
+    if (!am_last) return;
+    __threadfence();
+    if (warp == 0) {
+        Best b = none_best();
+        for (unsigned j = lane; j < gridDim.x; j += 32) {
+            grophecy_best_result r;
+            const volatile grophecy_best_result *pr = P.partials + j;
+            r.t_total_s = pr->t_total_s;
+            r.index = pr->index;
+            r.h2d_bytes = pr->h2d_bytes;
+            r.d2h_bytes = pr->d2h_bytes;
+            r.n_invalid = pr->n_invalid;
+            r.n_valid = pr->n_valid;
+            merge(b, from_result(r));
+        }
+        b = warp_best(b);
+        if (lane == 0) {
+            if (P.accumulate) {
+                Best prev = from_result(*P.out);
+                merge(prev, b);
+                b = prev;
+            }
+            to_result(*P.out, b);
+            *P.ticket = 0u;
+        }
+    }
+}
+
+__global__ void combine_kernel(const grophecy_best_result *in, uint32_t count,
+                               grophecy_best_result *out)
+{
+    const int lane = threadIdx.x & 31;
+    Best b = none_best();
+    for (uint32_t j = lane; j < count; j += 32) merge(b, from_result(in[j]));
+    b = warp_best(b);
+    if (lane == 0) to_result(*out, b);
+}
+
+static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_cap)
+{
+    static int occ_best = 0, occ_eval = 0;
+    (void)occ_eval;
+    if (!occ_best) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_best, project_kernel<true>, THREADS, 0);
+        if (occ_best < 1) occ_best = 1;
+    }
+    const unsigned long long tiles = (n + 31) / 32;
+    unsigned long long want = (tiles + WARPS - 1) / WARPS;
+    unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ_best, per_sm_cap);
+    if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
+    return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
+}
+
+static int check_batch(const grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b)
+{
+    if (!s || !pc || !b) {
+        set_error("null argument");
+        return GROPHECY_EINVAL;
+    }
+    if (b->n && (!b->skx || !b->nx || !b->ny || !b->iters)) {
+        set_error("null record array");
+        return GROPHECY_EINVAL;
+    }
+    return GROPHECY_OK;
+}
+
+static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b)
+{
+    Params P;
+    P.S = s->dev;
+    P.pc = *pc;
+    P.skx = b->skx;
+    P.nx = b->nx;
+    P.ny = b->ny;
+    P.iters = b->iters;
+    P.n = b->n;
+    P.base = b->index_base;
+    P.h2d = nullptr;
+    P.d2h = nullptr;
+    P.t = nullptr;
+    P.partials = s->partials;
+    P.ticket = s->ticket;
+    P.out = nullptr;
+    P.accumulate = 0;
+    return P;
+}
+
+int launch_best(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
+                grophecy_best_result *dout, int accumulate, cudaStream_t st)
+{
+    Params P = make_params(s, pc, b);
+    P.out = dout;
+    P.accumulate = accumulate;
+    const int grid = grid_for(s, b->n, 32);
+    project_kernel<true><<<grid, THREADS, 0, st>>>(P);
+    count_launch();
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "project_kernel<best> launch");
+    return GROPHECY_OK;
+}
+
+}  // namespace grophecy
+
+using namespace grophecy;
+
+extern "C" {
+
+int grophecy_eval(const grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
+                  uint64_t *h2d, uint64_t *d2h, double *t, void *stream)
+{
+    int rc = check_batch(s, pc, b);
+    if (rc) return rc;
+    if (b->n == 0) return GROPHECY_OK;
+    if (!h2d || !d2h || !t) {
+        set_error("null output array");
+        return GROPHECY_EINVAL;
+    }
+    Params P = make_params(s, pc, b);
+    P.h2d = (unsigned long long *)h2d;
+    P.d2h = (unsigned long long *)d2h;
+    P.t = t;
+    const int grid = grid_for(s, b->n, 32);
+    project_kernel<false><<<grid, THREADS, 0, (cudaStream_t)stream>>>(P);
+    count_launch();
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "project_kernel<eval> launch");
+    return GROPHECY_OK;
+}
+
+int grophecy_best_async(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
+                        grophecy_best_result *dout, int accumulate, void *stream)
+{
+    int rc = check_batch(s, pc, b);
+    if (rc) return rc;
+    if (!dout) {
+        set_error("null device_out");
+        return GROPHECY_EINVAL;
+    }
+    return launch_best(s, pc, b, dout, accumulate, (cudaStream_t)stream);
+}
+
+static int status_of(const grophecy_best_result &r)
+{
+    if (r.index == ~0ull) {
+        set_error("no valid candidate with finite projected time");
+        return GROPHECY_ENOFEASIBLE;
+    }
+    if (r.n_invalid) {
+        set_error("batch contains invalid records");
+        return GROPHECY_EBADCAND;
+    }
+    return GROPHECY_OK;
+}
+
+int grophecy_best(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
+                  grophecy_best_result *host_out, void *stream)
+{
+    int rc = check_batch(s, pc, b);
+    if (rc) return rc;
+    if (!host_out) {
+        set_error("null host_out");
+        return GROPHECY_EINVAL;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    // the result slot lives in the space's scratch, after the partials
+    grophecy_best_result *dres = s->partials + (s->max_partials - 1);
+    rc = launch_best(s, pc, b, dres, 0, st);
+    if (rc) return rc;
+    cudaError_t e = cudaMemcpyAsync(host_out, dres, sizeof *host_out, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_fail(e, "grophecy_best");
+    return status_of(*host_out);
+}
+
+int grophecy_best_combine(const grophecy_best_result *din, uint32_t count,
+                          grophecy_best_result *dout, void *stream)
+{
+    if (!dout || (count && !din)) {
+        set_error("null argument");
+        return GROPHECY_EINVAL;
+    }
+    combine_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(din, count, dout);
+    count_launch();
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "combine_kernel launch");
+    return GROPHECY_OK;
+}
+
+// End-to-end path with host records: chunked H2D copies on a copy stream,
+// double-buffered, overlapped with the fused kernel on the caller's stream;
+// one accumulating result slot; one D2H of 48 bytes at the end.
+int grophecy_best_host(grophecy_space *s, const grophecy_pcie *pc, const uint32_t *skx,
+                       const uint32_t *nx, const uint32_t *ny, const uint32_t *iters,
+                       uint64_t n, uint64_t index_base, grophecy_best_result *host_out,
+                       void *stream)
+{
+    if (!s || !pc || !host_out || (n && (!skx || !nx || !ny || !iters))) {
+        set_error("null argument");
+        return GROPHECY_EINVAL;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    cudaError_t e;
+    const uint64_t CHUNK = 1ull << 23;   // records per chunk (128 MiB of records)
+    const size_t need = (size_t)CHUNK * 16;
+    if (!s->copy_stream) {
+        if ((e = cudaStreamCreateWithFlags(&s->copy_stream, cudaStreamNonBlocking)) != cudaSuccess)
+            return cuda_fail(e, "cudaStreamCreate");
+        for (int i = 0; i < 2; i++) {
+            cudaEventCreateWithFlags(&s->ev_copied[i], cudaEventDisableTiming);
+            cudaEventCreateWithFlags(&s->ev_done[i], cudaEventDisableTiming);
+        }
+    }
+    if (s->stage_bytes < need) {
+        for (int i = 0; i < 2; i++) {
+            if (s->stage[i]) cudaFree(s->stage[i]);
+            s->stage[i] = nullptr;
+            if ((e = cudaMalloc(&s->stage[i], need)) != cudaSuccess) return cuda_fail(e, "cudaMalloc(stage)");
+        }
+        s->stage_bytes = need;
+    }
+    grophecy_best_result *dres = s->partials + (s->max_partials - 1);
+    grophecy_best_result init;
+    grophecy_best_combine_host(nullptr, 0, &init);
+    if ((e = cudaMemcpyAsync(dres, &init, sizeof init, cudaMemcpyHostToDevice, st)) != cudaSuccess)
+        return cuda_fail(e, "init result");
+    // copies of chunk c may start once the kernel of chunk c-2 finished
+    cudaEventRecord(s->ev_done[0], st);
+    cudaEventRecord(s->ev_done[1], st);
+    for (uint64_t off = 0, c = 0; off < n; off += CHUNK, c++) {
+        const uint64_t m = std::min<uint64_t>(CHUNK, n - off);
+        const int slot = (int)(c & 1);
+        uint32_t *buf = (uint32_t *)s->stage[slot];
+        cudaStreamWaitEvent(s->copy_stream, s->ev_done[slot], 0);
+        const uint32_t *src[4] = {skx, nx, ny, iters};
+        for (int f = 0; f < 4; f++) {
+            e = cudaMemcpyAsync(buf + (size_t)f * CHUNK, src[f] + off, m * 4, cudaMemcpyHostToDevice,
+                                s->copy_stream);
+            if (e != cudaSuccess) return cuda_fail(e, "H2D chunk");
+        }
+        cudaEventRecord(s->ev_copied[slot], s->copy_stream);
+        cudaStreamWaitEvent(st, s->ev_copied[slot], 0);
+        grophecy_batch b = {buf, buf + CHUNK, buf + 2 * CHUNK, buf + 3 * CHUNK, m, index_base + off};
+        int rc = launch_best(s, pc, &b, dres, 1, st);
+        if (rc) return rc;
+        cudaEventRecord(s->ev_done[slot], st);
+    }
+    e = cudaMemcpyAsync(host_out, dres, sizeof *host_out, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_fail(e, "grophecy_best_host");
+    return status_of(*host_out);
+}
+
+}  // extern "C"

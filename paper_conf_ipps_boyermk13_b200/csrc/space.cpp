@@ -1,0 +1,445 @@
+// Host side of the C ABI: PCIe fit, design-space validation, per-(kernel,
+// transformation) constant precompute and device upload.
+//
+// Compiled with -ffp-contract=off: every double expression below is evaluated
+// exactly as written (DESIGN.md §3 N1) so that the constants the GPU consumes
+// are bitwise the values the definition produces.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "grophecy.h"
+#include "internal.h"
+
+namespace grophecy {
+
+static thread_local std::string g_err;
+static std::atomic<uint64_t> g_launches{0};
+
+void set_error(const std::string &msg) { g_err = msg; }
+
+int cuda_fail(cudaError_t e, const char *what)
+{
+    set_error(std::string(what) + ": " + cudaGetErrorString(e));
+    return GROPHECY_ECUDA;
+}
+
+void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+static int fail(int code, const std::string &msg)
+{
+    set_error(msg);
+    return code;
+}
+
+static double dmin(double a, double b) { return a < b ? a : b; }
+
+static bool fin_nonneg(double v) { return std::isfinite(v) && v >= 0.0; }
+
+static bool coef_ok(const grophecy_affine8 &a)
+{
+    const int32_t L = 1 << 15;
+    return a.c1 >= -L && a.c1 <= L && a.c2 >= -L && a.c2 <= L && a.c3 >= -L && a.c3 <= L;
+}
+
+static int validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
+                    const grophecy_gpu_model *g)
+{
+    if (!skels || !g) return fail(GROPHECY_EINVAL, "null skeleton array or gpu model");
+    if (n_skels < 1) return fail(GROPHECY_EINVAL, "n_skels must be >= 1");
+    if (n_skels > GROPHECY_MAX_SKELS) return fail(GROPHECY_ELIMIT, "too many skeletons");
+    if (g->n_sm < 1 || g->warp_size < 1 || g->max_threads_per_block < 1 ||
+        g->max_blocks_per_sm < 1 || g->max_threads_per_sm < 1 || g->regs_per_sm < 1 ||
+        g->smem_per_sm < 1)
+        return fail(GROPHECY_EINVAL, "gpu model integers must be >= 1");
+    const double gd[] = {g->freq_hz, g->mem_bw_Bps, g->mem_ld_cycles, g->dep_del_coal,
+                         g->dep_del_uncoal, g->issue_cycles};
+    for (double v : gd)
+        if (!std::isfinite(v) || !(v > 0.0))
+            return fail(GROPHECY_EINVAL, "gpu model doubles must be finite and > 0");
+    for (uint32_t s = 0; s < n_skels; s++) {
+        const grophecy_skeleton_desc &S = skels[s];
+        char where[64];
+        snprintf(where, sizeof where, "skeleton %u: ", s);
+        if (S.n_kernels < 1 || S.n_xforms < 1)
+            return fail(GROPHECY_EINVAL, std::string(where) + "needs >= 1 kernel and transformation");
+        if (S.n_kernels > GROPHECY_MAX_KERNELS) return fail(GROPHECY_ELIMIT, std::string(where) + "too many kernels");
+        if (S.n_arrays > GROPHECY_MAX_ARRAYS) return fail(GROPHECY_ELIMIT, std::string(where) + "too many arrays");
+        if (S.n_regions > GROPHECY_MAX_REGIONS) return fail(GROPHECY_ELIMIT, std::string(where) + "too many regions");
+        if (S.n_xforms > GROPHECY_MAX_XFORMS) return fail(GROPHECY_ELIMIT, std::string(where) + "too many transformations");
+        if (!S.kernels || !S.kx || (S.n_arrays && !S.arrays) || (S.n_regions && !S.regions))
+            return fail(GROPHECY_EINVAL, std::string(where) + "null table");
+        for (uint32_t k = 0; k < S.n_kernels; k++)
+            if (!coef_ok(S.kernels[k].work_items))
+                return fail(GROPHECY_ELIMIT, std::string(where) + "work coefficient out of range");
+        for (uint32_t a = 0; a < S.n_arrays; a++) {
+            if (!coef_ok(S.arrays[a].rows) || !coef_ok(S.arrays[a].cols))
+                return fail(GROPHECY_ELIMIT, std::string(where) + "extent coefficient out of range");
+            if (S.arrays[a].elem_bytes < 1)
+                return fail(GROPHECY_EINVAL, std::string(where) + "elem_bytes must be >= 1");
+        }
+        std::vector<uint32_t> per_array(S.n_arrays, 0);
+        for (uint32_t j = 0; j < S.n_regions; j++) {
+            const grophecy_region_desc &r = S.regions[j];
+            if (r.kernel >= S.n_kernels || r.array >= S.n_arrays)
+                return fail(GROPHECY_EINVAL, std::string(where) + "region kernel/array index out of range");
+            if (r.mode < 1 || r.mode > 3)
+                return fail(GROPHECY_EINVAL, std::string(where) + "region mode must be R, W or R|W");
+            if ((r.flags & GROPHECY_REGION_WHOLE) && r.mode != GROPHECY_R)
+                return fail(GROPHECY_EINVAL, std::string(where) + "irregular (WHOLE) regions must be read-only");
+            if (!coef_ok(r.r0) || !coef_ok(r.r1) || !coef_ok(r.c0) || !coef_ok(r.c1))
+                return fail(GROPHECY_ELIMIT, std::string(where) + "region coefficient out of range");
+            if (++per_array[r.array] > GROPHECY_MAX_REGIONS_PER_ARRAY)
+                return fail(GROPHECY_ELIMIT, std::string(where) + "more than 32 regions on one array");
+        }
+        for (uint64_t i = 0; i < (uint64_t)S.n_xforms * S.n_kernels; i++) {
+            const grophecy_kx_desc &c = S.kx[i];
+            if (c.tpb < 1 || c.ipt < 1 || c.tpb > 65536u || c.ipt > 65536u ||
+                (uint64_t)c.tpb * c.ipt > 0xffffffffull)
+                return fail(GROPHECY_ELIMIT, std::string(where) + "tpb/ipt out of range");
+            if (!fin_nonneg(c.total_insts) || !fin_nonneg(c.coal_insts) ||
+                !fin_nonneg(c.uncoal_insts) || !fin_nonneg(c.synch_insts) ||
+                !std::isfinite(c.uncoal_per_mw) || !std::isfinite(c.load_bytes_per_warp))
+                return fail(GROPHECY_EINVAL, std::string(where) + "instruction counts must be finite and >= 0");
+            if (c.total_insts < c.coal_insts + c.uncoal_insts)
+                return fail(GROPHECY_EINVAL, std::string(where) + "total_insts < coal + uncoal");
+            if (!(c.uncoal_per_mw >= 1.0) || !(c.load_bytes_per_warp > 0.0))
+                return fail(GROPHECY_EINVAL, std::string(where) + "uncoal_per_mw must be >= 1, load_bytes_per_warp > 0");
+        }
+    }
+    return GROPHECY_OK;
+}
+
+// Per-(kernel, transformation) constants — DESIGN.md §3 N5 part A, plus the
+// saturated-grid reduction of part B.  Same operation order as the definition.
+static void precompute(const grophecy_kx_desc &c, const grophecy_gpu_model &g, KxES &es,
+                       KxD &dd_, KxI &ii, KxJ &jj, KxG &gg)
+{
+    uint64_t occ;
+    if (c.tpb > g.max_threads_per_block) {
+        occ = 0;
+    } else {
+        occ = std::min<uint64_t>(g.max_blocks_per_sm, g.max_threads_per_sm / c.tpb);
+        if (c.regs_per_thread > 0)
+            occ = std::min<uint64_t>(occ, g.regs_per_sm / ((uint64_t)c.regs_per_thread * c.tpb));
+        if (c.smem_per_block > 0) occ = std::min<uint64_t>(occ, g.smem_per_sm / c.smem_per_block);
+    }
+    uint64_t wpb = c.tpb / g.warp_size + (c.tpb % g.warp_size != 0);
+    uint64_t ipb = (uint64_t)c.tpb * c.ipt;
+    double mem = c.coal_insts + c.uncoal_insts;
+    double comp = g.issue_cycles * c.total_insts;
+
+    std::memset(&gg, 0, sizeof gg);
+    gg.comp = comp;
+    gg.synch = c.synch_insts;
+    jj.ipb = (uint32_t)ipb;
+    jj.occ = (uint32_t)occ;
+    jj.wpb = (uint32_t)wpb;
+    jj.flags = (occ == 0 ? KXF_INFEASIBLE : 0u) | (mem == 0.0 ? KXF_NOMEM : 0u);
+    ii.magic = ipb == 1 ? 0 : (~0ull) / ipb + 1;   // ceil(2^64 / ipb)
+    if (mem != 0.0) {
+        double mlu = g.mem_ld_cycles + (c.uncoal_per_mw - 1.0) * g.dep_del_uncoal;
+        double mlc = g.mem_ld_cycles;
+        double wu = c.uncoal_insts / mem;
+        double wc = c.coal_insts / mem;
+        double ml = mlu * wu + mlc * wc;
+        double dd = (g.dep_del_uncoal * c.uncoal_per_mw) * wu + g.dep_del_coal * wc;
+        double mwp0 = ml / dd;
+        double bwpw = g.freq_hz * c.load_bytes_per_warp / ml;
+        double bwr = g.mem_bw_Bps / bwpw;
+        double memc = mlu * c.uncoal_insts + mlc * c.coal_insts;
+        double cwpf = (memc + comp) / comp;
+        double cpm = comp / mem;
+        gg.mwp0 = mwp0; gg.bwr = bwr; gg.memc = memc; gg.cwpf = cwpf; gg.cpm = cpm;
+        gg.ml = ml; gg.dd = dd;
+    }
+    if (occ == 0) {
+        es = {0.0, 0.0};
+        dd_ = {1.0, 1.0};
+        ii.sat_blocks = ~0ull;
+        return;
+    }
+    // Saturated grid: blocks >= n_sm and ceil(blocks / n_sm) >= occ.
+    uint64_t nsm = g.n_sm;
+    ii.sat_blocks = std::max<uint64_t>(nsm, (occ - 1) * nsm + 1);
+    double N = (double)(occ * wpb);
+    double D = (double)(occ * nsm);
+    dd_.D = D;
+    dd_.rD = 1.0 / D;
+    if (mem == 0.0) {
+        es.E = comp * N;
+        es.S = 0.0;
+        return;
+    }
+    double mpk = gg.bwr / (double)nsm;
+    double mwp = dmin(dmin(gg.mwp0, mpk), N);
+    double cwp = dmin(gg.cwpf, N);
+    if (mwp == N && cwp == N)
+        es.E = gg.memc + comp + gg.cpm * (mwp - 1.0);
+    else if (cwp >= mwp || comp > gg.memc)
+        es.E = gg.memc * N / mwp + gg.cpm * (mwp - 1.0);
+    else
+        es.E = gg.ml + comp * N;
+    es.S = gg.dd * (mwp - 1.0) * c.synch_insts * (double)occ;
+}
+
+}  // namespace grophecy
+
+using namespace grophecy;
+
+extern "C" {
+
+int grophecy_abi_version(void) { return GROPHECY_ABI_VERSION; }
+
+const char *grophecy_last_error(void) { return g_err.c_str(); }
+
+uint64_t grophecy_launch_count(void) { return g_launches.load(); }
+
+int grophecy_fit_pcie(double t_small_s, double t_large_s, uint64_t large_bytes,
+                      grophecy_link *out)
+{
+    if (!out) return fail(GROPHECY_EINVAL, "out is NULL");
+    if (!std::isfinite(t_small_s) || !std::isfinite(t_large_s) || t_small_s < 0.0 ||
+        !(t_large_s > 0.0) || large_bytes == 0)
+        return fail(GROPHECY_EINVAL, "need finite t_small >= 0, t_large > 0, large_bytes > 0");
+    out->alpha_s = t_small_s;
+    out->beta_s_per_byte = t_large_s / (double)large_bytes;
+    return GROPHECY_OK;
+}
+
+double grophecy_pcie_time(const grophecy_link *link, uint64_t bytes)
+{
+    if (!link || bytes == 0) return 0.0;
+    return link->alpha_s + link->beta_s_per_byte * (double)bytes;
+}
+
+int grophecy_space_validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
+                            const grophecy_gpu_model *gpu)
+{
+    return validate(skels, n_skels, gpu);
+}
+
+static size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
+                          const grophecy_gpu_model *gpu, int device, grophecy_space **out)
+{
+    if (!out) return fail(GROPHECY_EINVAL, "out is NULL");
+    *out = nullptr;
+    int rc = validate(skels, n_skels, gpu);
+    if (rc) return rc;
+
+    // ---- host tables ----
+    std::vector<SkelInfo> info(n_skels);
+    std::vector<int4> kwork;
+    std::vector<uint32_t> kflags;
+    std::vector<ArrayDev> arrays;
+    std::vector<RegionDev> regions;
+    std::vector<KxES> kes;
+    std::vector<KxD> kd;
+    std::vector<KxI> ki;
+    std::vector<KxJ> kj;
+    std::vector<KxG> kg;
+    auto a4 = [](const grophecy_affine8 &a) { return make_int4(a.c0, a.c1, a.c2, a.c3); };
+    for (uint32_t s = 0; s < n_skels; s++) {
+        const grophecy_skeleton_desc &S = skels[s];
+        SkelInfo &I = info[s];
+        I.n_kernels = S.n_kernels;
+        I.n_arrays = S.n_arrays;
+        I.n_xforms = S.n_xforms;
+        I.n_regions = S.n_regions;
+        I.k_base = (uint32_t)kwork.size();
+        I.a_base = (uint32_t)arrays.size();
+        I.kx_base = (uint32_t)kes.size();
+        I.pad = 0;
+        for (uint32_t k = 0; k < S.n_kernels; k++) {
+            kwork.push_back(a4(S.kernels[k].work_items));
+            kflags.push_back(S.kernels[k].flags);
+        }
+        for (uint32_t a = 0; a < S.n_arrays; a++) {
+            ArrayDev A;
+            A.rows = a4(S.arrays[a].rows);
+            A.cols = a4(S.arrays[a].cols);
+            A.elem_bytes = S.arrays[a].elem_bytes;
+            A.liveout = (S.arrays[a].flags & GROPHECY_ARRAY_LIVEOUT) ? 1u : 0u;
+            A.r_base = (uint32_t)regions.size();
+            // regions of this array, stably sorted by kernel (order within a
+            // kernel is irrelevant: usage does not depend on region order)
+            std::vector<const grophecy_region_desc *> rs;
+            for (uint32_t j = 0; j < S.n_regions; j++)
+                if (S.regions[j].array == a) rs.push_back(&S.regions[j]);
+            std::stable_sort(rs.begin(), rs.end(), [](const grophecy_region_desc *x,
+                                                      const grophecy_region_desc *y) {
+                return x->kernel < y->kernel;
+            });
+            A.r_count = (uint32_t)rs.size();
+            for (size_t j = 0; j < rs.size(); j++) {
+                RegionDev R;
+                R.r0 = a4(rs[j]->r0); R.r1 = a4(rs[j]->r1);
+                R.c0 = a4(rs[j]->c0); R.c1 = a4(rs[j]->c1);
+                R.mode = rs[j]->mode;
+                R.whole = (rs[j]->flags & GROPHECY_REGION_WHOLE) ? 1u : 0u;
+                R.kernel = rs[j]->kernel;
+                uint32_t upto = 0;
+                for (size_t q = 0; q < rs.size(); q++)
+                    if (rs[q]->kernel <= rs[j]->kernel) upto |= 1u << q;
+                R.upto = upto;
+                regions.push_back(R);
+            }
+            arrays.push_back(A);
+        }
+        for (uint32_t k = 0; k < S.n_kernels; k++)
+            for (uint32_t x = 0; x < S.n_xforms; x++) {
+                KxES es; KxD d; KxI i; KxJ j; KxG g;
+                precompute(S.kx[(size_t)x * S.n_kernels + k], *gpu, es, d, i, j, g);
+                kes.push_back(es); kd.push_back(d); ki.push_back(i); kj.push_back(j);
+                kg.push_back(g);
+            }
+    }
+
+    // ---- one device blob ----
+    struct Part { const void *src; size_t bytes; size_t off; };
+    std::vector<Part> parts = {
+        {info.data(), info.size() * sizeof(SkelInfo), 0},
+        {kwork.data(), kwork.size() * sizeof(int4), 0},
+        {kflags.data(), kflags.size() * sizeof(uint32_t), 0},
+        {arrays.data(), arrays.size() * sizeof(ArrayDev), 0},
+        {regions.data(), regions.size() * sizeof(RegionDev), 0},
+        {kes.data(), kes.size() * sizeof(KxES), 0},
+        {kd.data(), kd.size() * sizeof(KxD), 0},
+        {ki.data(), ki.size() * sizeof(KxI), 0},
+        {kj.data(), kj.size() * sizeof(KxJ), 0},
+        {kg.data(), kg.size() * sizeof(KxG), 0},
+    };
+    size_t total = 0;
+    for (auto &p : parts) {
+        p.off = total;
+        total = align_up(total + p.bytes, 256);
+    }
+    std::vector<unsigned char> host(total, 0);
+    for (auto &p : parts)
+        if (p.bytes) std::memcpy(host.data() + p.off, p.src, p.bytes);
+
+    int prev = 0;
+    cudaError_t e = cudaGetDevice(&prev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    if ((e = cudaSetDevice(device)) != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+
+    grophecy_space *sp = new grophecy_space();
+    std::memset(sp, 0, sizeof *sp);
+    sp->device = device;
+    auto bail = [&](cudaError_t err, const char *what) {
+        if (sp->blob) cudaFree(sp->blob);
+        delete sp;
+        cudaSetDevice(prev);
+        return cuda_fail(err, what);
+    };
+    int nsm = 0;
+    if ((e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device)) != cudaSuccess)
+        return bail(e, "cudaDeviceGetAttribute");
+    sp->max_partials = (uint32_t)nsm * 32u;
+    size_t scratch_off = align_up(total, 256);
+    size_t part_bytes = sizeof(grophecy_best_result) * sp->max_partials;
+    size_t blob = scratch_off + align_up(part_bytes, 256) + 256;
+    if ((e = cudaMalloc(&sp->blob, blob)) != cudaSuccess) return bail(e, "cudaMalloc(space)");
+    sp->blob_bytes = blob;
+    if ((e = cudaMemcpy(sp->blob, host.data(), total, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return bail(e, "cudaMemcpy(space)");
+    unsigned char *base = (unsigned char *)sp->blob;
+    sp->partials = (grophecy_best_result *)(base + scratch_off);
+    unsigned char *ctr = base + scratch_off + align_up(part_bytes, 256);
+    sp->ticket = (unsigned int *)ctr;
+    sp->invalid_counter = (unsigned long long *)(ctr + 64);
+    if ((e = cudaMemset(ctr, 0, 256)) != cudaSuccess) return bail(e, "cudaMemset(space)");
+
+    SpaceDev &D = sp->dev;
+    D.skel = (const SkelInfo *)(base + parts[0].off);
+    D.kern_work = (const int4 *)(base + parts[1].off);
+    D.kern_flags = (const uint32_t *)(base + parts[2].off);
+    D.arrays = (const ArrayDev *)(base + parts[3].off);
+    D.regions = (const RegionDev *)(base + parts[4].off);
+    D.kx_es = (const KxES *)(base + parts[5].off);
+    D.kx_d = (const KxD *)(base + parts[6].off);
+    D.kx_i = (const KxI *)(base + parts[7].off);
+    D.kx_j = (const KxJ *)(base + parts[8].off);
+    D.kx_g = (const KxG *)(base + parts[9].off);
+    D.n_skels = n_skels;
+    D.n_sm = gpu->n_sm;
+    D.freq = gpu->freq_hz;
+    D.rfreq = 1.0 / gpu->freq_hz;
+    D.invalid_counter = sp->invalid_counter;
+    sp->grid_best = nsm;
+    sp->grid_eval = nsm;
+    cudaSetDevice(prev);
+    *out = sp;
+    return GROPHECY_OK;
+}
+
+void grophecy_space_destroy(grophecy_space *sp)
+{
+    if (!sp) return;
+    int prev = 0;
+    cudaGetDevice(&prev);
+    cudaSetDevice(sp->device);
+    if (sp->copy_stream) {
+        cudaStreamSynchronize(sp->copy_stream);
+        cudaStreamDestroy(sp->copy_stream);
+        for (int i = 0; i < 2; i++) {
+            cudaEventDestroy(sp->ev_copied[i]);
+            cudaEventDestroy(sp->ev_done[i]);
+        }
+    }
+    for (int i = 0; i < 2; i++)
+        if (sp->stage[i]) cudaFree(sp->stage[i]);
+    if (sp->blob) cudaFree(sp->blob);
+    cudaSetDevice(prev);
+    delete sp;
+}
+
+int grophecy_invalid_count(grophecy_space *sp, uint64_t *count, void *stream)
+{
+    if (!sp || !count) return fail(GROPHECY_EINVAL, "null argument");
+    cudaStream_t st = (cudaStream_t)stream;
+    unsigned long long v = 0;
+    cudaError_t e = cudaMemcpyAsync(&v, sp->invalid_counter, sizeof v, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(sp->invalid_counter, 0, sizeof v, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_fail(e, "grophecy_invalid_count");
+    *count = v;
+    return GROPHECY_OK;
+}
+
+// (t, index) lexicographic min-loc with counter sums; "none" = index UINT64_MAX.
+int grophecy_best_combine_host(const grophecy_best_result *in, uint32_t count,
+                               grophecy_best_result *out)
+{
+    if (!out || (count && !in)) return fail(GROPHECY_EINVAL, "null argument");
+    grophecy_best_result b;
+    b.t_total_s = INFINITY;
+    b.index = ~0ull;
+    b.h2d_bytes = b.d2h_bytes = 0;
+    b.n_invalid = b.n_valid = 0;
+    for (uint32_t i = 0; i < count; i++) {
+        const grophecy_best_result &r = in[i];
+        b.n_invalid += r.n_invalid;
+        b.n_valid += r.n_valid;
+        if (r.index == ~0ull) continue;
+        if (b.index == ~0ull || r.t_total_s < b.t_total_s ||
+            (r.t_total_s == b.t_total_s && r.index < b.index)) {
+            b.t_total_s = r.t_total_s;
+            b.index = r.index;
+            b.h2d_bytes = r.h2d_bytes;
+            b.d2h_bytes = r.d2h_bytes;
+        }
+    }
+    *out = b;
+    return GROPHECY_OK;
+}
+
+}  // extern "C"

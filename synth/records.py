@@ -33,12 +33,17 @@ def make_rule(kind, lo, hi, it_lo=1, it_hi=1024):
 
 def gen_records(cfg, start=0, stop=None):
     """Records [start, stop) of config ``cfg`` as four uint32 numpy arrays."""
-    N, X, seed, rules = cfg["n"], cfg["n_xforms"], cfg["seed"], cfg["rules"]
     if stop is None:
-        stop = N
+        stop = cfg["n"]
+    return gen_records_at(cfg, np.arange(start, stop, dtype=np.uint64))
+
+
+def gen_records_at(cfg, i):
+    """Records at arbitrary global indices ``i`` (uint64 array)."""
+    N, X, seed, rules = cfg["n"], cfg["n_xforms"], cfg["seed"], cfg["rules"]
     S = len(rules)
     G = (N + X - 1) // X
-    i = np.arange(start, stop, dtype=np.uint64)
+    i = np.asarray(i, dtype=np.uint64)
     g = i // np.uint64(X)
     x = (i % np.uint64(X)).astype(np.uint32)
     skel = ((g * np.uint64(S)) // np.uint64(G)).astype(np.int64)

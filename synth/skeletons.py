@@ -287,3 +287,10 @@ FX5600 = {"n_sm": 16, "warp_size": 32, "max_threads_per_block": 512, "max_blocks
 PAPER_TS = 1e-5
 PAPER_TL = 0.2147483648
 PAPER_SL = 1 << 29
+
+# A second, modern preset (B200-class numbers) to exercise other regimes.
+B200_LIKE = {"n_sm": 148, "warp_size": 32, "max_threads_per_block": 1024,
+             "max_blocks_per_sm": 32, "max_threads_per_sm": 2048, "regs_per_sm": 65536,
+             "smem_per_sm": 233472, "freq_hz": 1.965e9, "mem_bw_Bps": 7.7e12,
+             "mem_ld_cycles": 600.0, "dep_del_coal": 4.0, "dep_del_uncoal": 20.0,
+             "issue_cycles": 1.0}

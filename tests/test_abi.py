@@ -1,0 +1,136 @@
+"""The C-ABI boundary on CPU: the library loads, exports every symbol
+include/grophecy.h declares, and its host-only entry points behave
+(no compute calls need a GPU here)."""
+import math
+import os
+import re
+
+import numpy as np
+import pytest
+
+from synth import records as R
+from synth import skeletons as S
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def G():
+    from paper_conf_ipps_boyermk13_b200 import build
+    build.build()
+    from paper_conf_ipps_boyermk13_b200 import grophecy
+    return grophecy
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "grophecy.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(grophecy_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_every_declared_symbol_is_exported(G):
+    import ctypes
+    lib = ctypes.CDLL(G.LIB_PATH)
+    names = header_functions()
+    assert len(names) >= 18
+    for n in names:
+        assert hasattr(lib, n), n
+    assert set(names) == set(G.EXPORTED)
+
+
+def test_abi_version(G):
+    assert G.lib().grophecy_abi_version() == 1
+
+
+def test_fit_pcie_matches_oracle_bitwise(G, O):
+    rng = np.random.default_rng(5)
+    for _ in range(2000):
+        tS = float(rng.uniform(0, 1e-3))
+        tL = float(rng.uniform(1e-4, 1.0))
+        sL = int(rng.integers(1, 1 << 40))
+        a = G.fit_pcie(tS, tL, sL)
+        rc, b = O.fit_pcie(tS, tL, sL)
+        assert rc == 0 and a.alpha_s == b.alpha and a.beta_s_per_byte == b.beta
+        for d in (0, 1, int(rng.integers(1, 1 << 45))):
+            assert G.pcie_time(a, d) == O.pcie_time(b, d)
+
+
+@pytest.mark.parametrize("args", [(-1e-6, 1.0, 10), (1e-6, 0.0, 10), (1e-6, 1.0, 0),
+                                  (math.nan, 1.0, 10), (1e-6, math.inf, 10)])
+def test_fit_pcie_rejects(G, args):
+    with pytest.raises(G.GrophecyError) as e:
+        G.fit_pcie(*args)
+    assert e.value.code == G.EINVAL
+
+
+def test_validate_accepts_library(G):
+    for c in ("c1", "c2", "c3", "c4"):
+        assert G.validate(R.config(c)["skeletons"], S.FX5600) == G.OK
+
+
+def _s0():
+    return S.s0_stencil2()
+
+
+@pytest.mark.parametrize("mutate,code", [
+    (lambda s: s["kernels"].clear(), -1),
+    (lambda s: s["regions"].append(dict(s["regions"][0], kernel=5)), -1),
+    (lambda s: s["regions"].append(dict(s["regions"][0], array=7)), -1),
+    (lambda s: s["regions"].append(dict(s["regions"][0], mode="W", whole=True)), -1),
+    (lambda s: s["regions"].extend([dict(s["regions"][1])] * 40), -2),
+    (lambda s: s["arrays"].extend([dict(s["arrays"][0])] * 20), -2),
+    (lambda s: s["kernels"].__setitem__(0, dict(s["kernels"][0], work=(0, 1 << 16, 0, 0))), -2),
+    (lambda s: s["kx"][0].__setitem__(0, dict(s["kx"][0][0], total=1.0)), -1),
+    (lambda s: s["kx"][0].__setitem__(0, dict(s["kx"][0][0], tpb=0)), -2),
+    (lambda s: s["kx"][0].__setitem__(0, dict(s["kx"][0][0], upm=0.5)), -1),
+    (lambda s: s["kx"][0].__setitem__(0, dict(s["kx"][0][0], coal=math.nan)), -1),
+])
+def test_validate_rejects(G, mutate, code):
+    s = _s0()
+    mutate(s)
+    assert G.validate([s], S.FX5600) == code
+
+
+def test_validate_rejects_bad_gpu(G):
+    g = dict(S.FX5600, freq_hz=0.0)
+    assert G.validate([_s0()], g) == G.EINVAL
+    g = dict(S.FX5600, n_sm=0)
+    assert G.validate([_s0()], g) == G.EINVAL
+
+
+def test_combine_host_is_minloc(G):
+    rng = np.random.default_rng(9)
+    for _ in range(300):
+        k = int(rng.integers(0, 9))
+        res = []
+        for _ in range(k):
+            if rng.random() < 0.2:
+                res.append(G.BestResult(math.inf, G.UINT64_MAX, 0, 0, int(rng.integers(0, 5)),
+                                        int(rng.integers(0, 5))))
+            else:
+                t = float(rng.choice([1.0, 2.0, 0.5, 3.25]))
+                res.append(G.BestResult(t, int(rng.integers(0, 100)), int(rng.integers(0, 9)),
+                                        int(rng.integers(0, 9)), int(rng.integers(0, 5)),
+                                        int(rng.integers(1, 5))))
+        out = G.best_combine_host(res)
+        valid = [(r.t_total_s, r.index, r.h2d_bytes, r.d2h_bytes) for r in res
+                 if r.index != G.UINT64_MAX]
+        assert out.n_invalid == sum(r.n_invalid for r in res)
+        assert out.n_valid == sum(r.n_valid for r in res)
+        if not valid:
+            assert out.index == G.UINT64_MAX and math.isinf(out.t_total_s)
+        else:
+            best = min(valid, key=lambda v: (v[0], v[1]))
+            assert (out.t_total_s, out.index) == best[:2]
+            # the winner's byte counts travel with it (first occurrence of the min)
+            cand = [v for v in valid if (v[0], v[1]) == best[:2]]
+            assert (out.h2d_bytes, out.d2h_bytes) in [(v[2], v[3]) for v in cand]
+
+
+def test_no_gpu_fails_loudly(G):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(G.GrophecyError) as e:
+        G.Space([_s0()], S.FX5600, device=0)
+    assert e.value.code == G.ECUDA
