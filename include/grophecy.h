@@ -257,6 +257,16 @@ int grophecy_synth_records(const grophecy_synth_rule *rules, uint32_t n_rules,
                            uint64_t count, uint32_t *skx, uint32_t *nx, uint32_t *ny,
                            uint32_t *iters, void *cuda_stream);
 
+/* Diagnostic: evaluate on the HOST the usage plan that grophecy_space_create
+ * compiles for `skel` (the closed-form band programs the kernel runs for
+ * sizes inside the plan's domain nx >= *plan_tx, ny >= *plan_ty).  Fills
+ * per-array H2D / D2H bytes (arrays of skel->n_arrays).  Returns ELIMIT if
+ * the skeleton has no plan or (nx, ny) is outside its domain (the kernel then
+ * uses the general cell sweep).  Pure host function. */
+int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int64_t nx, int64_t ny,
+                             uint64_t *h2d_per_array, uint64_t *d2h_per_array,
+                             uint32_t *plan_tx, uint32_t *plan_ty);
+
 /* Number of CUDA kernel launches issued by this library since load (for
  * the bench's gpu_launches count). */
 uint64_t grophecy_launch_count(void);

@@ -4,6 +4,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <vector>
 
 #include "grophecy.h"
 
@@ -34,11 +35,25 @@ struct SkelInfo {
     uint32_t a_base;   // into arrays
     uint32_t kx_base;  // into kx tables
     uint32_t pad;
+    // usage plan (plan.cpp): valid for nx >= plan_tx and ny >= plan_ty
+    uint32_t plan_tx, plan_ty, expr_base, n_expr;
 };
 
 struct ArrayDev {
     int4 rows, cols;
     uint32_t elem_bytes, liveout, r_base, r_count;   // regions [r_base, r_base+r_count)
+    uint32_t h_prog, d_prog, pad0, pad1;             // plan band programs (u16 offsets)
+};
+
+constexpr uint32_t PLAN_MAX_EXPR = 128;
+
+// Host-side result of compiling one skeleton's usage plan.
+struct SkelPlanHost {
+    bool ok = false;
+    uint32_t tx = 0, ty = 0;
+    std::vector<int4> exprs;
+    std::vector<uint16_t> prog;
+    std::vector<uint32_t> h_off, d_off;   // per array, into prog
 };
 
 // Regions are stored grouped by array and sorted by kernel within an array,
@@ -60,6 +75,8 @@ struct SpaceDev {
     const KxI *kx_i;
     const KxJ *kx_j;
     const KxG *kx_g;
+    const int4 *plan_expr;
+    const uint16_t *plan_prog;
     uint32_t n_skels;
     uint32_t n_sm;
     double freq, rfreq;
@@ -86,6 +103,7 @@ struct grophecy_space {
 };
 
 namespace grophecy {
+bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out);
 void set_error(const std::string &msg);
 int cuda_fail(cudaError_t e, const char *what);
 void count_launch(uint64_t n = 1);

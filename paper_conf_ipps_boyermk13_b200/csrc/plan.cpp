@@ -1,0 +1,323 @@
+// Usage plans: the data-usage analysis of one skeleton "compiled" at space
+// creation into closed-form band programs valid on a size domain.
+//
+// For one array the H2D / D2H element counts are areas of unions of cells of
+// the grid cut by the region bounds (§III-B; DESIGN.md §3
+// N4).  The bounds are size-affine expressions v = c0 + floor(L(nx, ny) / 8).
+// On a domain D = [tx, 2^20] x [ty, 2^20] where every pairwise order between
+// the bounds (and 0 and the array extent) is FIXED, the cell structure, the
+// clamping and the first-reader / first-writer of every cell are the same for
+// all sizes in D, so
+//     count = sum_bands (row[e] - row[s]) * sum_runs (col[e'] - col[s'])
+// with row/col values the (unclamped-by-construction) bound expressions.
+// Equal values at some sizes only produce zero-height slabs, so a fixed
+// non-strict order suffices.
+//
+// u <= v on D is proven exactly: floor(a) - floor(b) >= (a - b) - 7/8 for
+// a, b in Z/8, so  8(v0 - u0) - 7 + (Lv - Lu)(nx, ny) >= 0  on D  implies
+// v - u >= 0 on D; the left side is bilinear in (nx, ny), hence its minimum
+// over the box D is at a corner.
+//
+// Keys outside the domain (or skeletons without a plan) take the general
+// cooperative sweep on the device.
+#include <algorithm>
+#include <cstdint>
+#include <vector>
+
+#include "grophecy.h"
+#include "internal.h"
+
+namespace grophecy {
+
+namespace {
+
+struct Ex {
+    int64_t c0, c1, c2, c3;
+    bool operator==(const Ex &o) const { return c0 == o.c0 && c1 == o.c1 && c2 == o.c2 && c3 == o.c3; }
+};
+
+Ex ex_of(const grophecy_affine8 &a) { return {a.c0, a.c1, a.c2, a.c3}; }
+const Ex ZERO = {0, 0, 0, 0};
+
+struct Dom {
+    int64_t x0, x1, y0, y1;
+};
+
+bool nonneg_on(int64_t a, int64_t b, int64_t c, int64_t d, const Dom &D)
+{
+    const int64_t xs[2] = {D.x0, D.x1}, ys[2] = {D.y0, D.y1};
+    for (int64_t x : xs)
+        for (int64_t y : ys)
+            if (a + b * x + c * y + d * x * y < 0) return false;
+    return true;
+}
+
+// proven u <= v at every size of D
+bool le(const Ex &u, const Ex &v, const Dom &D)
+{
+    if (u == v) return true;
+    return nonneg_on(8 * (v.c0 - u.c0) - 7, v.c1 - u.c1, v.c2 - u.c2, v.c3 - u.c3, D);
+}
+
+enum Ord { LT, GT, EQ, UNK };
+
+Ord order(const Ex &u, const Ex &v, const Dom &D)
+{
+    if (u == v) return EQ;
+    const bool a = le(u, v, D), b = le(v, u, D);
+    if (a && b) return EQ;   // cannot happen for distinct coefficients (slack), kept for safety
+    if (a) return LT;
+    if (b) return GT;
+    return UNK;
+}
+
+// clamp(x, 0, E) resolved symbolically on D; false if the branch varies.
+bool clamp_sym(const Ex &x, const Ex &E, const Dom &D, Ex &out)
+{
+    if (le(x, ZERO, D)) { out = ZERO; return true; }
+    if (le(E, x, D)) { out = E; return true; }
+    if (le(ZERO, x, D) && le(x, E, D)) { out = x; return true; }
+    return false;
+}
+
+// Sort expression list into classes of a fixed order on D.  pos[i] = class of
+// vals[i]; reps = one representative per class, ascending.
+bool classify(const std::vector<Ex> &vals, const Dom &D, std::vector<int> &pos, std::vector<Ex> &reps)
+{
+    const size_t m = vals.size();
+    std::vector<int> idx(m);
+    for (size_t i = 0; i < m; i++) idx[i] = (int)i;
+    for (size_t i = 0; i < m; i++)
+        for (size_t j = i + 1; j < m; j++)
+            if (order(vals[i], vals[j], D) == UNK) return false;
+    std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) { return order(vals[a], vals[b], D) == LT; });
+    pos.assign(m, 0);
+    reps.clear();
+    for (size_t k = 0; k < m; k++) {
+        const int i = idx[k];
+        if (k == 0 || order(vals[idx[k - 1]], vals[i], D) != EQ) reps.push_back(vals[i]);
+        pos[i] = (int)reps.size() - 1;
+    }
+    return true;
+}
+
+struct ArrayProg {
+    std::vector<Ex> rowv, colv;                 // class representatives
+    std::vector<std::vector<uint8_t>> hcell, dcell;   // [row slab][col slab]
+};
+
+// Compile one array on domain D.  regs: the array's regions (any order).
+bool compile_array(const grophecy_array_desc &A, const std::vector<const grophecy_region_desc *> &regs,
+                   const Dom &D, ArrayProg &P)
+{
+    P = ArrayProg();
+    Ex Er = ex_of(A.rows), Ec = ex_of(A.cols);
+    // extents R = max(0, rows), C = max(0, cols)
+    Ex R, C;
+    if (le(Er, ZERO, D)) R = ZERO;
+    else if (le(ZERO, Er, D)) R = Er;
+    else return false;
+    if (le(Ec, ZERO, D)) C = ZERO;
+    else if (le(ZERO, Ec, D)) C = Ec;
+    else return false;
+    if (R == ZERO || C == ZERO) return true;    // empty array: no cells
+
+    struct Box { Ex r0, r1, c0, c1; uint32_t kernel, mode; };
+    std::vector<Box> boxes;
+    for (const grophecy_region_desc *g : regs) {
+        Box b;
+        b.kernel = g->kernel;
+        b.mode = g->mode;
+        if (g->flags & GROPHECY_REGION_WHOLE) {
+            b.r0 = ZERO; b.r1 = R; b.c0 = ZERO; b.c1 = C;
+        } else {
+            if (!clamp_sym(ex_of(g->r0), R, D, b.r0) || !clamp_sym(ex_of(g->r1), R, D, b.r1) ||
+                !clamp_sym(ex_of(g->c0), C, D, b.c0) || !clamp_sym(ex_of(g->c1), C, D, b.c1))
+                return false;
+        }
+        // always empty on D?
+        if (le(b.r1, b.r0, D) || le(b.c1, b.c0, D)) continue;
+        if (!le(b.r0, b.r1, D) || !le(b.c0, b.c1, D)) return false;
+        boxes.push_back(b);
+    }
+    std::vector<Ex> rv = {ZERO, R}, cv = {ZERO, C};
+    for (const Box &b : boxes) {
+        rv.push_back(b.r0); rv.push_back(b.r1);
+        cv.push_back(b.c0); cv.push_back(b.c1);
+    }
+    std::vector<int> rp, cp;
+    if (!classify(rv, D, rp, P.rowv) || !classify(cv, D, cp, P.colv)) return false;
+    const int nr = (int)P.rowv.size() - 1, nc = (int)P.colv.size() - 1;
+    if (nr <= 0 || nc <= 0) return true;
+    P.hcell.assign(nr, std::vector<uint8_t>(nc, 0));
+    P.dcell.assign(nr, std::vector<uint8_t>(nc, 0));
+    const uint32_t INF = 0xffffffffu;
+    for (int i = 0; i < nr; i++)
+        for (int j = 0; j < nc; j++) {
+            uint32_t fr = INF, fw = INF;
+            for (size_t q = 0; q < boxes.size(); q++) {
+                const int r0 = rp[2 + 2 * q], r1 = rp[3 + 2 * q];
+                const int c0 = cp[2 + 2 * q], c1 = cp[3 + 2 * q];
+                if (r0 <= i && i + 1 <= r1 && c0 <= j && j + 1 <= c1) {
+                    if ((boxes[q].mode & GROPHECY_R) && boxes[q].kernel < fr) fr = boxes[q].kernel;
+                    if ((boxes[q].mode & GROPHECY_W) && boxes[q].kernel < fw) fw = boxes[q].kernel;
+                }
+            }
+            P.hcell[i][j] = fr != INF && fr <= fw;
+            P.dcell[i][j] = fw != INF;
+        }
+    return true;
+}
+
+// Emit band program for one cell matrix; expression indices via idx().
+template <class F>
+void emit(const std::vector<std::vector<uint8_t>> &cell, const std::vector<Ex> &rowv,
+          const std::vector<Ex> &colv, F idx, std::vector<uint16_t> &out)
+{
+    const size_t at = out.size();
+    out.push_back(0);
+    uint16_t nb = 0;
+    const int nr = (int)cell.size();
+    int i = 0;
+    while (i < nr) {
+        bool any = false;
+        for (uint8_t v : cell[i]) any |= v != 0;
+        if (!any) { i++; continue; }
+        int e = i + 1;
+        while (e < nr && cell[e] == cell[i]) e++;
+        // band rows [i, e): from rowv[i] to rowv[e]
+        std::vector<std::pair<int, int>> runs;
+        const int nc = (int)cell[i].size();
+        for (int j = 0; j < nc;) {
+            if (!cell[i][j]) { j++; continue; }
+            int k = j + 1;
+            while (k < nc && cell[i][k]) k++;
+            runs.push_back({j, k});
+            j = k;
+        }
+        out.push_back(idx(rowv[i]));
+        out.push_back(idx(rowv[e]));
+        out.push_back((uint16_t)runs.size());
+        for (auto &r : runs) {
+            out.push_back(idx(colv[r.first]));
+            out.push_back(idx(colv[r.second]));
+        }
+        nb++;
+        i = e;
+    }
+    out[at] = nb;
+}
+
+}  // namespace
+
+bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out)
+{
+    out = SkelPlanHost();
+    std::vector<std::vector<const grophecy_region_desc *>> regs(S.n_arrays);
+    for (uint32_t j = 0; j < S.n_regions; j++) regs[S.regions[j].array].push_back(&S.regions[j]);
+
+    auto try_dom = [&](int64_t tx, int64_t ty, std::vector<ArrayProg> &progs) {
+        const Dom D = {tx, (int64_t)GROPHECY_MAX_DIM, ty, (int64_t)GROPHECY_MAX_DIM};
+        progs.assign(S.n_arrays, ArrayProg());
+        for (uint32_t a = 0; a < S.n_arrays; a++)
+            if (!compile_array(S.arrays[a], regs[a], D, progs[a])) return false;
+        return true;
+    };
+    // smallest domain corner (tx, ty) over powers of two, minimising log tx + log ty
+    int best_l = -1, best_tx = 0, best_ty = 0;
+    std::vector<ArrayProg> progs;
+    for (int ly = 0; ly <= 20; ly++) {
+        int lo = 0, hi = 21;   // find minimal lx in [0, 20] that works (21 = none)
+        while (lo < hi) {
+            const int mid = (lo + hi) / 2;
+            if (try_dom(1ll << mid, 1ll << ly, progs)) hi = mid;
+            else lo = mid + 1;
+        }
+        if (lo <= 20 && (best_l < 0 || lo + ly < best_l)) {
+            best_l = lo + ly;
+            best_tx = lo;
+            best_ty = ly;
+        }
+        if (best_l >= 0 && ly >= best_l) break;
+    }
+    if (best_l < 0) return false;
+    if (!try_dom(1ll << best_tx, 1ll << best_ty, progs)) return false;
+
+    std::vector<Ex> table;
+    auto idx = [&](const Ex &e) -> uint16_t {
+        for (size_t i = 0; i < table.size(); i++)
+            if (table[i] == e) return (uint16_t)i;
+        table.push_back(e);
+        return (uint16_t)(table.size() - 1);
+    };
+    for (uint32_t a = 0; a < S.n_arrays; a++) {
+        out.h_off.push_back((uint32_t)out.prog.size());
+        emit(progs[a].hcell, progs[a].rowv, progs[a].colv, idx, out.prog);
+        out.d_off.push_back((uint32_t)out.prog.size());
+        emit(progs[a].dcell, progs[a].rowv, progs[a].colv, idx, out.prog);
+    }
+    if (table.size() > PLAN_MAX_EXPR) return false;
+    for (const Ex &e : table)
+        out.exprs.push_back(make_int4((int)e.c0, (int)e.c1, (int)e.c2, (int)e.c3));
+    out.tx = 1u << best_tx;
+    out.ty = 1u << best_ty;
+    out.ok = true;
+    return true;
+}
+
+}  // namespace grophecy
+
+// ---- host evaluation of a plan (diagnostic entry point, mirrors the device) ----
+namespace {
+int64_t aff8_host(const int4 &c, int64_t nx, int64_t ny)
+{
+    const int64_t num = (int64_t)c.y * nx + (int64_t)c.z * ny + (int64_t)c.w * nx * ny;
+    return (int64_t)c.x + (num >> 3);
+}
+}  // namespace
+
+using namespace grophecy;
+
+extern "C" int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int64_t nx, int64_t ny,
+                                        uint64_t *h2d_per_array, uint64_t *d2h_per_array,
+                                        uint32_t *plan_tx, uint32_t *plan_ty)
+{
+    if (!skel || !h2d_per_array || !d2h_per_array) {
+        set_error("null argument");
+        return GROPHECY_EINVAL;
+    }
+    SkelPlanHost P;
+    if (!compile_plan(*skel, P)) {
+        if (plan_tx) *plan_tx = 0xffffffffu;
+        if (plan_ty) *plan_ty = 0xffffffffu;
+        set_error("skeleton has no usage plan");
+        return GROPHECY_ELIMIT;
+    }
+    if (plan_tx) *plan_tx = P.tx;
+    if (plan_ty) *plan_ty = P.ty;
+    if (nx < (int64_t)P.tx || ny < (int64_t)P.ty) {
+        set_error("size outside the plan's domain");
+        return GROPHECY_ELIMIT;
+    }
+    std::vector<int64_t> val(P.exprs.size());
+    for (size_t e = 0; e < P.exprs.size(); e++) val[e] = aff8_host(P.exprs[e], nx, ny);
+    for (uint32_t a = 0; a < skel->n_arrays; a++) {
+        for (int which = 0; which < 2; which++) {
+            const uint16_t *p = P.prog.data() + (which ? P.d_off[a] : P.h_off[a]);
+            const uint32_t nb = *p++;
+            uint64_t cnt = 0;
+            for (uint32_t b = 0; b < nb; b++) {
+                const int64_t rh = val[p[1]] - val[p[0]];
+                const uint32_t nr = p[2];
+                p += 3;
+                int64_t w = 0;
+                for (uint32_t q = 0; q < nr; q++, p += 2) w += val[p[1]] - val[p[0]];
+                cnt += (uint64_t)(rh * w);
+            }
+            const uint64_t eb = skel->arrays[a].elem_bytes;
+            if (which == 0) h2d_per_array[a] = cnt * eb;
+            else d2h_per_array[a] = (skel->arrays[a].flags & GROPHECY_ARRAY_LIVEOUT) ? cnt * eb : 0;
+        }
+    }
+    return GROPHECY_OK;
+}

@@ -52,13 +52,18 @@ __device__ __forceinline__ double div_rn(double a, double b, double rb)
     return __fma_rn(r, rb, q);
 }
 
-struct WarpScratch {
+struct SweepScratch {
     long long box[32][4];
     long long rs_h[64];
     long long cs_w[64];
     unsigned rs_m[64];
     unsigned cs_m[64];
     unsigned upto[32];
+};
+
+union WarpScratch {
+    SweepScratch sw;                 // general cell sweep
+    long long val[PLAN_MAX_EXPR];    // usage plan: expression values of one key
 };
 
 struct Usage {
@@ -73,12 +78,62 @@ __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v)
     return v;
 }
 
+// Per-array byte counts -> totals and per-array PCIe times in array order
+// (Eq. (1), one transfer per array).  Warp-uniform.
+__device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned long long h,
+                                          unsigned long long d, const grophecy_pcie &pc)
+{
+    const unsigned long long ha = h * (unsigned long long)A.elem_bytes;
+    const unsigned long long da = A.liveout ? d * (unsigned long long)A.elem_bytes : 0ull;
+    if (ha) o.th = __dadd_rn(o.th, __dadd_rn(pc.h2d.alpha_s,
+                                             __dmul_rn(pc.h2d.beta_s_per_byte, (double)ha)));
+    if (da) o.td = __dadd_rn(o.td, __dadd_rn(pc.d2h.alpha_s,
+                                             __dmul_rn(pc.d2h.beta_s_per_byte, (double)da)));
+    o.h += ha;
+    o.d += da;
+}
+
+// Usage of one key from the skeleton's compiled plan (plan.cpp): lanes over
+// the plan's expressions, then lanes over (array, H|D) band programs.
+__device__ Usage warp_usage_plan(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
+                                 const grophecy_pcie &pc, WarpScratch &ws, int lane)
+{
+    for (uint32_t e = lane; e < I.n_expr; e += 32)
+        ws.val[e] = aff8(__ldg(&S.plan_expr[I.expr_base + e]), nx, ny);
+    __syncwarp();
+    unsigned long long cnt = 0;
+    if ((uint32_t)lane < 2 * I.n_arrays) {
+        const ArrayDev &A = S.arrays[I.a_base + (lane >> 1)];
+        const uint16_t *p = S.plan_prog + ((lane & 1) ? A.d_prog : A.h_prog);
+        const uint32_t nb = __ldg(p++);
+        for (uint32_t b = 0; b < nb; b++) {
+            const long long rh = ws.val[__ldg(p + 1)] - ws.val[__ldg(p)];
+            const uint32_t nr = __ldg(p + 2);
+            p += 3;
+            long long w = 0;
+            for (uint32_t q = 0; q < nr; q++, p += 2) w += ws.val[__ldg(p + 1)] - ws.val[__ldg(p)];
+            cnt += (unsigned long long)(rh * w);
+        }
+    }
+    Usage o = {0ull, 0ull, 0.0, 0.0};
+    for (uint32_t a = 0; a < I.n_arrays; a++) {
+        const unsigned long long h = __shfl_sync(FULL, cnt, 2 * a);
+        const unsigned long long d = __shfl_sync(FULL, cnt, 2 * a + 1);
+        add_array(o, S.arrays[I.a_base + a], h, d, pc);
+    }
+    __syncwarp();
+    return o;
+}
+
 // Data usage of one (skeleton, nx, ny) key, computed by the whole warp
 // (DESIGN.md §3 N4; §III-B), plus the per-array PCIe
-// transfer times in array order (Eq. (1), one transfer per array).
+// transfer times in array order.  General coordinate-compressed sweep; the
+// compiled plan is used instead whenever it covers the key.
 __device__ Usage warp_usage(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
-                            const grophecy_pcie &pc, WarpScratch &ws, int lane)
+                            const grophecy_pcie &pc, WarpScratch &wsu, int lane)
 {
+    if (nx >= I.plan_tx && ny >= I.plan_ty) return warp_usage_plan(S, I, nx, ny, pc, wsu, lane);
+    SweepScratch &ws = wsu.sw;
     Usage o = {0ull, 0ull, 0.0, 0.0};
     const unsigned lt = (1u << lane) - 1u;
     for (uint32_t a = 0; a < I.n_arrays; a++) {
@@ -209,14 +264,7 @@ __device__ Usage warp_usage(const SpaceDev &S, const SkelInfo &I, long long nx, 
                 }
             }
         }
-        const unsigned long long ha = h * (unsigned long long)A.elem_bytes;
-        const unsigned long long da = A.liveout ? d * (unsigned long long)A.elem_bytes : 0ull;
-        if (ha) o.th = __dadd_rn(o.th, __dadd_rn(pc.h2d.alpha_s,
-                                                 __dmul_rn(pc.h2d.beta_s_per_byte, (double)ha)));
-        if (da) o.td = __dadd_rn(o.td, __dadd_rn(pc.d2h.alpha_s,
-                                                 __dmul_rn(pc.d2h.beta_s_per_byte, (double)da)));
-        o.h += ha;
-        o.d += da;
+        add_array(o, A, h, d, pc);
     }
     return o;
 }
@@ -365,7 +413,7 @@ struct Params {
 };
 
 template <bool BEST>
-__global__ void __launch_bounds__(THREADS) project_kernel(const Params P)
+__global__ void __launch_bounds__(THREADS, 3) project_kernel(const Params P)
 {
     __shared__ WarpScratch scratch[WARPS];
     __shared__ Best wbest[WARPS];
@@ -392,7 +440,7 @@ __global__ void __launch_bounds__(THREADS) project_kernel(const Params P)
         const uint32_t skel = skx >> 16, x = skx & 0xffffu;
         bool valid = has && skel < S.n_skels && nx >= 1 && nx <= GROPHECY_MAX_DIM && ny >= 1 &&
                      ny <= GROPHECY_MAX_DIM && it >= 1;
-        SkelInfo I = {0, 0, 0, 0, 0, 0, 0, 0};
+        SkelInfo I = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
         if (valid) {
             I = S.skel[skel];
             valid = x < I.n_xforms;

@@ -246,6 +246,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxI> ki;
     std::vector<KxJ> kj;
     std::vector<KxG> kg;
+    std::vector<int4> pexpr;
+    std::vector<uint16_t> pprog;
     auto a4 = [](const grophecy_affine8 &a) { return make_int4(a.c0, a.c1, a.c2, a.c3); };
     for (uint32_t s = 0; s < n_skels; s++) {
         const grophecy_skeleton_desc &S = skels[s];
@@ -258,6 +260,19 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         I.a_base = (uint32_t)arrays.size();
         I.kx_base = (uint32_t)kes.size();
         I.pad = 0;
+        SkelPlanHost plan;
+        if (compile_plan(S, plan)) {
+            I.plan_tx = plan.tx;
+            I.plan_ty = plan.ty;
+            I.expr_base = (uint32_t)pexpr.size();
+            I.n_expr = (uint32_t)plan.exprs.size();
+            pexpr.insert(pexpr.end(), plan.exprs.begin(), plan.exprs.end());
+        } else {
+            I.plan_tx = I.plan_ty = 0xffffffffu;   // never applicable
+            I.expr_base = I.n_expr = 0;
+        }
+        const uint32_t prog_base = (uint32_t)pprog.size();
+        if (plan.ok) pprog.insert(pprog.end(), plan.prog.begin(), plan.prog.end());
         for (uint32_t k = 0; k < S.n_kernels; k++) {
             kwork.push_back(a4(S.kernels[k].work_items));
             kflags.push_back(S.kernels[k].flags);
@@ -269,6 +284,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             A.elem_bytes = S.arrays[a].elem_bytes;
             A.liveout = (S.arrays[a].flags & GROPHECY_ARRAY_LIVEOUT) ? 1u : 0u;
             A.r_base = (uint32_t)regions.size();
+            A.h_prog = plan.ok ? prog_base + plan.h_off[a] : 0;
+            A.d_prog = plan.ok ? prog_base + plan.d_off[a] : 0;
+            A.pad0 = A.pad1 = 0;
             // regions of this array, stably sorted by kernel (order within a
             // kernel is irrelevant: usage does not depend on region order)
             std::vector<const grophecy_region_desc *> rs;
@@ -316,6 +334,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {ki.data(), ki.size() * sizeof(KxI), 0},
         {kj.data(), kj.size() * sizeof(KxJ), 0},
         {kg.data(), kg.size() * sizeof(KxG), 0},
+        {pexpr.data(), pexpr.size() * sizeof(int4), 0},
+        {pprog.data(), pprog.size() * sizeof(uint16_t), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -369,6 +389,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.kx_i = (const KxI *)(base + parts[7].off);
     D.kx_j = (const KxJ *)(base + parts[8].off);
     D.kx_g = (const KxG *)(base + parts[9].off);
+    D.plan_expr = (const int4 *)(base + parts[10].off);
+    D.plan_prog = (const uint16_t *)(base + parts[11].off);
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;
     D.freq = gpu->freq_hz;

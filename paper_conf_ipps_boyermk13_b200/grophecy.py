@@ -130,6 +130,9 @@ _sig = {
     "grophecy_synth_records": (C.c_int, [C.POINTER(SynthRule), C.c_uint32, C.c_uint64, C.c_uint32,
                                          C.c_uint64, C.c_uint64, C.c_uint64, _vp, _vp, _vp, _vp,
                                          _vp]),
+    "grophecy_plan_usage_host": (C.c_int, [C.POINTER(SkeletonDesc), C.c_int64, C.c_int64,
+                                           C.POINTER(C.c_uint64), C.POINTER(C.c_uint64),
+                                           C.POINTER(C.c_uint32), C.POINTER(C.c_uint32)]),
     "grophecy_launch_count": (C.c_uint64, []),
     "grophecy_last_error": (C.c_char_p, []),
     "grophecy_abi_version": (C.c_int, []),
@@ -381,6 +384,18 @@ def calibrate(device=0, reps=10, large_bytes=1 << 29):
     out = PCIe()
     _check(_L.grophecy_calibrate(device, reps, large_bytes, C.byref(out)), "calibrate")
     return out
+
+
+def plan_usage_host(skel, nx, ny):
+    """Host evaluation of the compiled usage plan: (rc, h2d[], d2h[], tx, ty)."""
+    sd = Skeletons([skel])
+    na = max(1, len(skel["arrays"]))
+    h = (C.c_uint64 * na)()
+    d = (C.c_uint64 * na)()
+    tx, ty = C.c_uint32(), C.c_uint32()
+    rc = _L.grophecy_plan_usage_host(sd.arr, nx, ny, h, d, C.byref(tx), C.byref(ty))
+    n = len(skel["arrays"])
+    return rc, list(h)[:n], list(d)[:n], tx.value, ty.value
 
 
 def launch_count():

@@ -134,3 +134,43 @@ def test_no_gpu_fails_loudly(G):
     with pytest.raises(G.GrophecyError) as e:
         G.Space([_s0()], S.FX5600, device=0)
     assert e.value.code == G.ECUDA
+
+
+def _check_plan(G, O, s, sizes):
+    covered = 0
+    for nx, ny in sizes:
+        rc, h, d, tx, ty = G.plan_usage_host(s, nx, ny)
+        if rc != G.OK:
+            assert rc == G.ELIMIT and (nx < tx or ny < ty or tx == 0xFFFFFFFF)
+            continue
+        covered += 1
+        oh, od = O.usage(s, nx, ny)
+        assert list(h) == [int(v) for v in oh], (s["name"], nx, ny)
+        assert list(d) == [int(v) for v in od], (s["name"], nx, ny)
+    return covered
+
+
+def test_usage_plans_match_oracle_library(G, O):
+    """The compiled usage plans (closed-form band programs the kernel runs)
+    reproduce the oracle's data usage at every size of their domain."""
+    r = np.random.default_rng(17)
+    sizes = [(int(a), int(b)) for a, b in zip(np.exp2(r.uniform(0, 20, 120)).astype(int),
+                                                 np.exp2(r.uniform(0, 20, 120)).astype(int))]
+    sizes += [(1, 1), (2, 2), (3, 5), (1 << 20, 1 << 20), (1 << 20, 1), (1, 1 << 20)]
+    skels = [f() for f in S.LIBRARY] + S.random_skeletons(0x5EED0003, 20)
+    tot = 0
+    for s in skels:
+        tot += _check_plan(G, O, s, sizes)
+    assert tot > 0.5 * len(sizes) * len(skels)
+
+
+def test_usage_plans_match_oracle_random_tiny(G, O):
+    from tests.tiny import random_tiny_skeleton, rng
+    r = rng(555)
+    tot = 0
+    for _ in range(400):
+        s, _, _ = random_tiny_skeleton(r)
+        sizes = [(int(r.integers(1, 2000)), int(r.integers(1, 2000))) for _ in range(6)]
+        sizes += [(1 << 20, 1 << 20), (int(r.integers(1, 64)), 1 << 20)]
+        tot += _check_plan(G, O, s, sizes)
+    assert tot > 500

@@ -349,3 +349,17 @@ def test_c3_full_size_sampled(G, O, pc):
 
 def test_c4_full_size_sampled(G, O, pc):
     _full_size_check(G, O, pc, "c4", n_sample=30_000)
+
+
+def test_random_tiny_skeletons_large_sizes(G, O, pc):
+    """Tiny random skeletons at log-uniform sizes up to 2^20: keys inside and
+    outside each skeleton's compiled usage-plan domain, in the same warps."""
+    r = rng(4242)
+    for trial in range(20):
+        skels = [random_tiny_skeleton(r, n_xforms=2)[0] for _ in range(6)]
+        n = 4096
+        rec = {"skx": ((r.integers(0, 6, n) << 16) | r.integers(0, 2, n)).astype(np.uint32),
+               "nx": np.exp2(r.uniform(0, 20, n)).astype(np.uint32),
+               "ny": np.exp2(r.uniform(0, 20, n)).astype(np.uint32),
+               "iters": r.integers(1, 50, n).astype(np.uint32)}
+        run_parity(G, O, pc, skels, rec)
