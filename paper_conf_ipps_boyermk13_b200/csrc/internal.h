@@ -22,7 +22,7 @@ struct KxES { double E, S; };         // case expression, synch factor
 struct KxD  { double D, rD; };        // rep denominator and RN(1/D)
 struct KxI  { uint64_t magic; uint64_t sat_blocks; };  // ceil(2^64/ipb) (0 if ipb==1)
 struct KxJ  { uint32_t ipb, occ, wpb, flags; };        // flags: KXF_*
-enum : uint32_t { KXF_INFEASIBLE = 1u, KXF_NOMEM = 2u };
+enum : uint32_t { KXF_INFEASIBLE = 1u, KXF_NOMEM = 2u, KXF_PER_ITER = 4u };
 
 // General-grid constants (small grids / huge W), read only off the fast path.
 struct KxG {
@@ -42,7 +42,7 @@ struct SkelInfo {
 struct ArrayDev {
     int4 rows, cols;
     uint32_t elem_bytes, liveout, r_base, r_count;   // regions [r_base, r_base+r_count)
-    uint32_t h_prog, d_prog, pad0, pad1;             // plan band programs (u16 offsets)
+    uint32_t h_prog, d_prog, pad0, pad1;             // plan band programs (u32 word offsets)
 };
 
 constexpr uint32_t PLAN_MAX_EXPR = 128;
@@ -52,7 +52,7 @@ struct SkelPlanHost {
     bool ok = false;
     uint32_t tx = 0, ty = 0;
     std::vector<int4> exprs;
-    std::vector<uint16_t> prog;
+    std::vector<uint32_t> prog;           // band programs (see plan.cpp)
     std::vector<uint32_t> h_off, d_off;   // per array, into prog
 };
 
@@ -76,7 +76,7 @@ struct SpaceDev {
     const KxJ *kx_j;
     const KxG *kx_g;
     const int4 *plan_expr;
-    const uint16_t *plan_prog;
+    const uint32_t *plan_prog;
     uint32_t n_skels;
     uint32_t n_sm;
     double freq, rfreq;

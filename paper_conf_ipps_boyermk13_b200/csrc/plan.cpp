@@ -169,14 +169,17 @@ bool compile_array(const grophecy_array_desc &A, const std::vector<const grophec
     return true;
 }
 
-// Emit band program for one cell matrix; expression indices via idx().
+// Emit the band program of one cell matrix as u32 words:
+//   [n_bands] then per band [rs | re << 16, n_runs, (cs | ce << 16) x n_runs]
+// (indices into the skeleton's expression table): count =
+//   sum_bands (val[re] - val[rs]) * sum_runs (val[ce] - val[cs]).
 template <class F>
 void emit(const std::vector<std::vector<uint8_t>> &cell, const std::vector<Ex> &rowv,
-          const std::vector<Ex> &colv, F idx, std::vector<uint16_t> &out)
+          const std::vector<Ex> &colv, F idx, std::vector<uint32_t> &out)
 {
     const size_t at = out.size();
     out.push_back(0);
-    uint16_t nb = 0;
+    uint32_t nb = 0;
     const int nr = (int)cell.size();
     int i = 0;
     while (i < nr) {
@@ -195,13 +198,10 @@ void emit(const std::vector<std::vector<uint8_t>> &cell, const std::vector<Ex> &
             runs.push_back({j, k});
             j = k;
         }
-        out.push_back(idx(rowv[i]));
-        out.push_back(idx(rowv[e]));
-        out.push_back((uint16_t)runs.size());
-        for (auto &r : runs) {
-            out.push_back(idx(colv[r.first]));
-            out.push_back(idx(colv[r.second]));
-        }
+        out.push_back((uint32_t)idx(rowv[i]) | ((uint32_t)idx(rowv[e]) << 16));
+        out.push_back((uint32_t)runs.size());
+        for (auto &r : runs)
+            out.push_back((uint32_t)idx(colv[r.first]) | ((uint32_t)idx(colv[r.second]) << 16));
         nb++;
         i = e;
     }
@@ -243,7 +243,10 @@ bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out)
     if (best_l < 0) return false;
     if (!try_dom(1ll << best_tx, 1ll << best_ty, progs)) return false;
 
+    // table: kernel work expressions first (entry k = kernel k, read by the
+    // model), then the usage expressions
     std::vector<Ex> table;
+    for (uint32_t k = 0; k < S.n_kernels; k++) table.push_back(ex_of(S.kernels[k].work_items));
     auto idx = [&](const Ex &e) -> uint16_t {
         for (size_t i = 0; i < table.size(); i++)
             if (table[i] == e) return (uint16_t)i;
@@ -303,15 +306,15 @@ extern "C" int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int6
     for (size_t e = 0; e < P.exprs.size(); e++) val[e] = aff8_host(P.exprs[e], nx, ny);
     for (uint32_t a = 0; a < skel->n_arrays; a++) {
         for (int which = 0; which < 2; which++) {
-            const uint16_t *p = P.prog.data() + (which ? P.d_off[a] : P.h_off[a]);
+            const uint32_t *p = P.prog.data() + (which ? P.d_off[a] : P.h_off[a]);
             const uint32_t nb = *p++;
             uint64_t cnt = 0;
             for (uint32_t b = 0; b < nb; b++) {
-                const int64_t rh = val[p[1]] - val[p[0]];
-                const uint32_t nr = p[2];
-                p += 3;
+                const int64_t rh = val[p[0] >> 16] - val[p[0] & 0xffff];
+                const uint32_t nr = p[1];
+                p += 2;
                 int64_t w = 0;
-                for (uint32_t q = 0; q < nr; q++, p += 2) w += val[p[1]] - val[p[0]];
+                for (uint32_t q = 0; q < nr; q++, p++) w += val[*p >> 16] - val[*p & 0xffff];
                 cnt += (uint64_t)(rh * w);
             }
             const uint64_t eb = skel->arrays[a].elem_bytes;

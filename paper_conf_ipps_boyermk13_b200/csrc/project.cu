@@ -62,8 +62,8 @@ struct SweepScratch {
 };
 
 union WarpScratch {
-    SweepScratch sw;                 // general cell sweep
-    long long val[PLAN_MAX_EXPR];    // usage plan: expression values of one key
+    SweepScratch sw;                    // general cell sweep
+    long long val[2][PLAN_MAX_EXPR];    // usage plans: expression values of up to two keys
 };
 
 struct Usage {
@@ -93,46 +93,65 @@ __device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned 
     o.d += da;
 }
 
-// Usage of one key from the skeleton's compiled plan (plan.cpp): lanes over
-// the plan's expressions, then lanes over (array, H|D) band programs.
-__device__ Usage warp_usage_plan(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
-                                 const grophecy_pcie &pc, WarpScratch &ws, int lane)
+// Usage of one key from its skeleton's compiled plan (plan.cpp), by a segment
+// of L lanes (L = 16: two keys per warp, one per half; L = 32: one key).
+// Lanes first evaluate the plan's expressions (entries 0..K-1 are the
+// kernels' work-item counts, kept for the model), then lane 2a / 2a+1 of the
+// segment runs the H2D / D2H band program of array a and prices its transfer
+// with Eq. (1); byte totals are an integer tree sum, transfer times an
+// ordered (array-order) floating-point sum.
+__device__ __forceinline__ Usage plan_usage(const SpaceDev &S, uint32_t s, long long nx,
+                                            long long ny, const grophecy_pcie &pc, long long *val,
+                                            int sl, int L, int base, uint32_t max_arrays)
 {
-    for (uint32_t e = lane; e < I.n_expr; e += 32)
-        ws.val[e] = aff8(__ldg(&S.plan_expr[I.expr_base + e]), nx, ny);
+    const SkelInfo &I = S.skel[s];
+    const uint32_t n_expr = I.n_expr, n_arrays = I.n_arrays, e0 = I.expr_base, a0 = I.a_base;
+    for (uint32_t e = sl; e < n_expr; e += L) val[e] = aff8(__ldg(&S.plan_expr[e0 + e]), nx, ny);
     __syncwarp();
-    unsigned long long cnt = 0;
-    if ((uint32_t)lane < 2 * I.n_arrays) {
-        const ArrayDev &A = S.arrays[I.a_base + (lane >> 1)];
-        const uint16_t *p = S.plan_prog + ((lane & 1) ? A.d_prog : A.h_prog);
+    double T = 0.0;
+    unsigned long long bytes = 0;
+    if ((uint32_t)sl < 2 * n_arrays) {
+        const ArrayDev &A = S.arrays[a0 + (sl >> 1)];
+        const bool dir_d2h = sl & 1;
+        const uint32_t *p = S.plan_prog + (dir_d2h ? A.d_prog : A.h_prog);
         const uint32_t nb = __ldg(p++);
+        unsigned long long cnt = 0;
         for (uint32_t b = 0; b < nb; b++) {
-            const long long rh = ws.val[__ldg(p + 1)] - ws.val[__ldg(p)];
-            const uint32_t nr = __ldg(p + 2);
-            p += 3;
+            const uint32_t w0 = __ldg(p), nr = __ldg(p + 1);
+            p += 2;
+            const long long rh = val[w0 >> 16] - val[w0 & 0xffffu];
             long long w = 0;
-            for (uint32_t q = 0; q < nr; q++, p += 2) w += ws.val[__ldg(p + 1)] - ws.val[__ldg(p)];
+            for (uint32_t q = 0; q < nr; q++) {
+                const uint32_t wq = __ldg(p++);
+                w += val[wq >> 16] - val[wq & 0xffffu];
+            }
             cnt += (unsigned long long)(rh * w);
         }
+        bytes = (dir_d2h && !A.liveout) ? 0ull : cnt * (unsigned long long)A.elem_bytes;
+        const grophecy_link lk = dir_d2h ? pc.d2h : pc.h2d;
+        if (bytes) T = __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte, __ull2double_rn(bytes)));
     }
-    Usage o = {0ull, 0ull, 0.0, 0.0};
-    for (uint32_t a = 0; a < I.n_arrays; a++) {
-        const unsigned long long h = __shfl_sync(FULL, cnt, 2 * a);
-        const unsigned long long d = __shfl_sync(FULL, cnt, 2 * a + 1);
-        add_array(o, S.arrays[I.a_base + a], h, d, pc);
+    Usage o;
+    for (int off = 2; off < L; off <<= 1) bytes += __shfl_xor_sync(FULL, bytes, off);
+    o.h = __shfl_sync(FULL, bytes, base);
+    o.d = __shfl_sync(FULL, bytes, base + 1);
+    double th = 0.0, td = 0.0;
+    for (uint32_t a = 0; a < max_arrays; a++) {   // arrays without transfer add +0.0
+        th = __dadd_rn(th, __shfl_sync(FULL, T, base + 2 * a));
+        td = __dadd_rn(td, __shfl_sync(FULL, T, base + 2 * a + 1));
     }
-    __syncwarp();
+    o.th = th;
+    o.td = td;
     return o;
 }
 
-// Data usage of one (skeleton, nx, ny) key, computed by the whole warp
-// (DESIGN.md §3 N4; §III-B), plus the per-array PCIe
-// transfer times in array order.  General coordinate-compressed sweep; the
-// compiled plan is used instead whenever it covers the key.
-__device__ Usage warp_usage(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
-                            const grophecy_pcie &pc, WarpScratch &wsu, int lane)
+// Data usage of one (skeleton, nx, ny) key by the general coordinate-compressed
+// sweep over the whole warp (DESIGN.md §3 N4; §III-B), plus
+// the per-array PCIe transfer times in array order.  Used for keys outside
+// their skeleton's plan domain.
+__device__ Usage warp_usage_sweep(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
+                                  const grophecy_pcie &pc, WarpScratch &wsu, int lane)
 {
-    if (nx >= I.plan_tx && ny >= I.plan_ty) return warp_usage_plan(S, I, nx, ny, pc, wsu, lane);
     SweepScratch &ws = wsu.sw;
     Usage o = {0ull, 0ull, 0.0, 0.0};
     const unsigned lt = (1u << lane) - 1u;
@@ -269,14 +288,12 @@ __device__ Usage warp_usage(const SpaceDev &S, const SkelInfo &I, long long nx, 
     return o;
 }
 
-// Kernel time of kernel k of skeleton I under transformation x (DESIGN.md §3 N5).
-__device__ __forceinline__ double kernel_time(const SpaceDev &S, const SkelInfo &I, uint32_t k,
-                                              uint32_t x, long long nx, long long ny)
+// Kernel time of one kernel (DESIGN.md §3 N5) from its work-item count Wi and
+// its (kernel, transformation) constants J / kxi.
+__device__ __forceinline__ double kernel_time(const SpaceDev &S, long long Wi, const KxJ &J,
+                                              uint32_t kxi)
 {
-    const long long Wi = aff8(__ldg(&S.kern_work[I.k_base + k]), nx, ny);
     const unsigned long long W = Wi > 0 ? (unsigned long long)Wi : 0ull;
-    const uint32_t kxi = I.kx_base + k * I.n_xforms + x;
-    const KxJ J = S.kx_j[kxi];
     if (J.flags & KXF_INFEASIBLE) return __longlong_as_double(0x7ff0000000000000LL);
     const KxI II = S.kx_i[kxi];
     unsigned long long blocks;
@@ -323,6 +340,28 @@ __device__ __forceinline__ double kernel_time(const SpaceDev &S, const SkelInfo 
         cyc = __dadd_rn(cyc, sync);
     }
     return __ddiv_rn(cyc, S.freq);
+}
+
+// Total projected time of one candidate: kernels (run-once
+// plus iters x per-iteration) + transfers.  val = the key's plan values
+// (work counts at 0..K-1) or NULL to evaluate the work expressions here.
+__device__ __forceinline__ double candidate_time(const SpaceDev &S, uint32_t s, uint32_t x,
+                                                 long long nx, long long ny, uint32_t it,
+                                                 const long long *val, const Usage &u)
+{
+    const SkelInfo &I = S.skel[s];
+    const uint32_t K = I.n_kernels, X = I.n_xforms, kb = I.k_base;
+    uint32_t kxi = I.kx_base + x;
+    double t_iter = 0.0, t_once = 0.0;
+    for (uint32_t k = 0; k < K; k++, kxi += X) {
+        const long long Wi = val ? val[k] : aff8(__ldg(&S.kern_work[kb + k]), nx, ny);
+        const KxJ J = S.kx_j[kxi];
+        const double tk = kernel_time(S, Wi, J, kxi);
+        if (J.flags & KXF_PER_ITER) t_iter = __dadd_rn(t_iter, tk);
+        else t_once = __dadd_rn(t_once, tk);
+    }
+    const double t_kern = __dadd_rn(t_once, __dmul_rn((double)it, t_iter));
+    return __dadd_rn(__dadd_rn(t_kern, u.th), u.td);
 }
 
 struct Best {
@@ -426,53 +465,88 @@ __global__ void __launch_bounds__(THREADS, 3) project_kernel(const Params P)
     Best mine = none_best();
     const unsigned long long ntiles = (P.n + 31) >> 5;
     const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
-    for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
-         tile += wstride) {
+    unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp;
+    // software pipeline: records of the next tile are loaded while this one computes
+    uint32_t c_skx = 0, c_nx = 0, c_ny = 0, c_it = 0;
+    {
+        const unsigned long long i = (tile << 5) + lane;
+        if (tile < ntiles && i < P.n) {
+            c_skx = __ldcs(P.skx + i); c_nx = __ldcs(P.nx + i);
+            c_ny = __ldcs(P.ny + i); c_it = __ldcs(P.iters + i);
+        }
+    }
+    for (; tile < ntiles; tile += wstride) {
         const unsigned long long i = (tile << 5) + lane;
         const bool has = i < P.n;
-        uint32_t skx = 0, nx = 0, ny = 0, it = 0;
-        if (has) {
-            skx = __ldcs(P.skx + i);
-            nx = __ldcs(P.nx + i);
-            ny = __ldcs(P.ny + i);
-            it = __ldcs(P.iters + i);
+        const uint32_t skx = c_skx, nx = c_nx, ny = c_ny, it = c_it;
+        {
+            const unsigned long long nt = tile + wstride, ni = (nt << 5) + lane;
+            c_skx = c_nx = c_ny = c_it = 0;
+            if (nt < ntiles && ni < P.n) {
+                c_skx = __ldcs(P.skx + ni); c_nx = __ldcs(P.nx + ni);
+                c_ny = __ldcs(P.ny + ni); c_it = __ldcs(P.iters + ni);
+            }
         }
         const uint32_t skel = skx >> 16, x = skx & 0xffffu;
         bool valid = has && skel < S.n_skels && nx >= 1 && nx <= GROPHECY_MAX_DIM && ny >= 1 &&
                      ny <= GROPHECY_MAX_DIM && it >= 1;
-        SkelInfo I = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
-        if (valid) {
-            I = S.skel[skel];
-            valid = x < I.n_xforms;
-        }
+        if (valid) valid = x < S.skel[skel].n_xforms;
         const unsigned long long key =
             valid ? ((unsigned long long)skel << 42) | ((unsigned long long)nx << 21) | ny : ~0ull;
         unsigned pending = __ballot_sync(FULL, valid);
-        Usage u = {0ull, 0ull, 0.0, 0.0};
-        while (pending) {
-            const int L = __ffs(pending) - 1;
-            const unsigned long long kL = __shfl_sync(FULL, key, L);
-            const unsigned same = __ballot_sync(FULL, key == kL);
-            const uint32_t sL = (uint32_t)(kL >> 42);
-            const long long nxL = (long long)((kL >> 21) & 0x1fffffull);
-            const long long nyL = (long long)(kL & 0x1fffffull);
-            const SkelInfo IL = S.skel[sL];
-            const Usage r = warp_usage(S, IL, nxL, nyL, P.pc, ws, lane);
-            if (key == kL) u = r;
-            pending &= ~same;
-        }
         double t = __longlong_as_double(0x7ff8000000000000LL);   // NaN for invalid
-        if (valid) {
-            double t_iter = 0.0, t_once = 0.0;
-            for (uint32_t k = 0; k < I.n_kernels; k++) {
-                const double tk = kernel_time(S, I, k, x, nx, ny);
-                if (__ldg(&S.kern_flags[I.k_base + k]) & GROPHECY_KERNEL_PER_ITER)
-                    t_iter = __dadd_rn(t_iter, tk);
-                else
-                    t_once = __dadd_rn(t_once, tk);
+        Usage u = {0ull, 0ull, 0.0, 0.0};
+        // rounds of one or two distinct keys (usage is shared by every lane
+        // with the same key; the model then runs per lane)
+        while (pending) {
+            const int LA = __ffs(pending) - 1;
+            const unsigned long long kA = __shfl_sync(FULL, key, LA);
+            const unsigned sameA = __ballot_sync(FULL, key == kA);
+            const uint32_t sA = (uint32_t)(kA >> 42);
+            const long long nxA = (long long)((kA >> 21) & 0x1fffffull);
+            const long long nyA = (long long)(kA & 0x1fffffull);
+            const SkelInfo &IA = S.skel[sA];
+            const bool planA = nxA >= IA.plan_tx && nyA >= IA.plan_ty;
+            const uint32_t naA = IA.n_arrays;
+            const unsigned rest = pending & ~sameA;
+            bool two = false;
+            unsigned long long kB = ~0ull;
+            if (planA && naA <= 8 && rest) {
+                kB = __shfl_sync(FULL, key, __ffs(rest) - 1);
+                const SkelInfo &IB = S.skel[(uint32_t)(kB >> 42)];
+                two = (long long)((kB >> 21) & 0x1fffffull) >= IB.plan_tx &&
+                      (long long)(kB & 0x1fffffull) >= IB.plan_ty && IB.n_arrays <= 8;
             }
-            const double t_kern = __dadd_rn(t_once, __dmul_rn((double)it, t_iter));
-            t = __dadd_rn(__dadd_rn(t_kern, u.th), u.td);
+            const long long *myval = nullptr;
+            Usage r;
+            if (two) {
+                const unsigned sameB = __ballot_sync(FULL, key == kB);
+                const int h = lane >> 4;
+                const unsigned long long kh = h ? kB : kA;
+                const uint32_t naB = S.skel[(uint32_t)(kB >> 42)].n_arrays;
+                r = plan_usage(S, (uint32_t)(kh >> 42), (long long)((kh >> 21) & 0x1fffffull),
+                               (long long)(kh & 0x1fffffull), P.pc, ws.val[h], lane & 15, 16,
+                               lane & 16, naA > naB ? naA : naB);
+                const int src = key == kB ? 16 : 0;
+                r.h = __shfl_sync(FULL, r.h, src);
+                r.d = __shfl_sync(FULL, r.d, src);
+                r.th = __shfl_sync(FULL, r.th, src);
+                r.td = __shfl_sync(FULL, r.td, src);
+                myval = ws.val[key == kB ? 1 : 0];
+                pending &= ~(sameA | sameB);
+            } else if (planA) {
+                r = plan_usage(S, sA, nxA, nyA, P.pc, ws.val[0], lane, 32, 0, naA);
+                myval = ws.val[0];
+                pending &= ~sameA;
+            } else {
+                r = warp_usage_sweep(S, IA, nxA, nyA, P.pc, ws, lane);
+                pending &= ~sameA;
+            }
+            if (key == kA || (two && key == kB)) {
+                u = r;
+                t = candidate_time(S, skel, x, nx, ny, it, myval, u);
+            }
+            __syncwarp();   // scratch is reused by the next round
         }
         if (!BEST) {
             if (has) {

@@ -247,7 +247,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxJ> kj;
     std::vector<KxG> kg;
     std::vector<int4> pexpr;
-    std::vector<uint16_t> pprog;
+    std::vector<uint32_t> pprog;
     auto a4 = [](const grophecy_affine8 &a) { return make_int4(a.c0, a.c1, a.c2, a.c3); };
     for (uint32_t s = 0; s < n_skels; s++) {
         const grophecy_skeleton_desc &S = skels[s];
@@ -316,6 +316,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             for (uint32_t x = 0; x < S.n_xforms; x++) {
                 KxES es; KxD d; KxI i; KxJ j; KxG g;
                 precompute(S.kx[(size_t)x * S.n_kernels + k], *gpu, es, d, i, j, g);
+                if (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) j.flags |= KXF_PER_ITER;
                 kes.push_back(es); kd.push_back(d); ki.push_back(i); kj.push_back(j);
                 kg.push_back(g);
             }
@@ -335,7 +336,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {kj.data(), kj.size() * sizeof(KxJ), 0},
         {kg.data(), kg.size() * sizeof(KxG), 0},
         {pexpr.data(), pexpr.size() * sizeof(int4), 0},
-        {pprog.data(), pprog.size() * sizeof(uint16_t), 0},
+        {pprog.data(), pprog.size() * sizeof(uint32_t), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -390,7 +391,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.kx_j = (const KxJ *)(base + parts[8].off);
     D.kx_g = (const KxG *)(base + parts[9].off);
     D.plan_expr = (const int4 *)(base + parts[10].off);
-    D.plan_prog = (const uint16_t *)(base + parts[11].off);
+    D.plan_prog = (const uint32_t *)(base + parts[11].off);
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;
     D.freq = gpu->freq_hz;
