@@ -1,17 +1,20 @@
 // The projection hot path for sm_100a: grophecy_eval / grophecy_best[_async]
 // / grophecy_best_combine / grophecy_best_host.
 //
-// One fused kernel per call.  Each warp takes tiles of 32 consecutive records
-// (coalesced 32-bit SoA loads).  Data usage depends only on (skeleton, nx, ny)
-// (reading 11), so the warp deduplicates keys with ballots and
-// computes the usage of each distinct key cooperatively (lanes over regions,
-// then over coordinate-compressed cells), broadcasting the result to every
-// lane with that key.  The kernel-time model then runs per lane (one
-// candidate per lane) from per-(kernel, transformation) constants that the
-// host precomputed in the definition's operation order; on saturated grids
-// the two remaining IEEE divisions use Markstein's correction
-// (q = a*rb; r = fma(-q, b, a); q' = fma(r, rb, q)), which is correctly
-// rounded when rb = RN(1/b) — bitwise the result of a / b.
+// One fused, persistent kernel per call.  A CTA (256 threads) takes a tile of
+// 1024 consecutive candidate records: each thread loads 4 records with one
+// 16-byte load per SoA array.  Data usage depends only on the key
+// (skeleton, nx, ny) (reading 11), so the CTA finds the runs of equal
+// keys with a block scan, computes the usage of every distinct key ONCE — from
+// the skeleton's compiled usage plan (plan.cpp) with several keys per warp, or
+// with the general coordinate-compressed sweep for keys outside the plan
+// domain — and keeps the results in shared memory.  The kernel-time model then
+// runs per candidate from per-(kernel, transformation) constants the host
+// precomputed in the definition's operation order; on saturated grids the two
+// remaining IEEE divisions use Markstein's correction
+// (q = a*rb; r = fma(-q, b, a); q' = fma(r, rb, q)), correctly rounded when
+// rb = RN(1/b), i.e. bitwise a / b.  Best mode fuses the argmin
+// (thread -> warp -> CTA -> grid, last-block pattern).
 //
 // Compiled with -fmad=false: no contraction anywhere; FMAs appear only as the
 // explicit __fma_rn of the Markstein step.
@@ -29,7 +32,14 @@ namespace grophecy {
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int THREADS = 256;
 constexpr int WARPS = THREADS / 32;
+constexpr int RPT = 4;                       // records per thread
+constexpr int TILE = THREADS * RPT;          // records per CTA tile
+constexpr int SLOT_CAP = 256;                // distinct keys resident per chunk
+constexpr int VAL_PER_WARP = 256;            // plan expression values per warp
 constexpr long long BIG = 0x7fffffffffffffffLL;
+#ifndef GROPHECY_MINB
+#define GROPHECY_MINB 3
+#endif
 
 __device__ __forceinline__ long long aff8(int4 c, long long nx, long long ny)
 {
@@ -62,8 +72,8 @@ struct SweepScratch {
 };
 
 union WarpScratch {
-    SweepScratch sw;                    // general cell sweep
-    long long val[2][PLAN_MAX_EXPR];    // usage plans: expression values of up to two keys
+    SweepScratch sw;                    // general cell sweep (one key per warp)
+    long long val[VAL_PER_WARP];        // usage plans: expression values of G keys
 };
 
 struct Usage {
@@ -94,18 +104,25 @@ __device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned 
 }
 
 // Usage of one key from its skeleton's compiled plan (plan.cpp), by a segment
-// of L lanes (L = 16: two keys per warp, one per half; L = 32: one key).
-// Lanes first evaluate the plan's expressions (entries 0..K-1 are the
-// kernels' work-item counts, kept for the model), then lane 2a / 2a+1 of the
-// segment runs the H2D / D2H band program of array a and prices its transfer
-// with Eq. (1); byte totals are an integer tree sum, transfer times an
-// ordered (array-order) floating-point sum.
-__device__ __forceinline__ Usage plan_usage(const SpaceDev &S, uint32_t s, long long nx,
-                                            long long ny, const grophecy_pcie &pc, long long *val,
-                                            int sl, int L, int base, uint32_t max_arrays)
+// of L lanes [base, base+L) (several keys per warp).  Lanes first evaluate the
+// plan's expressions (entries 0..K-1 are the kernels' work-item counts), then
+// lane 2a / 2a+1 of the segment runs the H2D / D2H band program of array a
+// and prices its transfer with Eq. (1) (requires 2 * n_arrays <= L); byte
+// totals are an integer tree sum, transfer times an ordered (array-order)
+// floating-point sum.  Inactive segments (active == false) contribute nothing
+// but take part in the shuffles.
+__device__ __forceinline__ Usage plan_usage(const SpaceDev &S, bool active, unsigned long long key,
+                                            const grophecy_pcie &pc, long long *val, int sl, int L,
+                                            int base, uint32_t max_arrays)
 {
-    const SkelInfo &I = S.skel[s];
-    const uint32_t n_expr = I.n_expr, n_arrays = I.n_arrays, e0 = I.expr_base, a0 = I.a_base;
+    uint32_t n_expr = 0, n_arrays = 0, e0 = 0, a0 = 0;
+    long long nx = 0, ny = 0;
+    if (active) {
+        const SkelInfo &I = S.skel[(uint32_t)(key >> 42)];
+        n_expr = I.n_expr; n_arrays = I.n_arrays; e0 = I.expr_base; a0 = I.a_base;
+        nx = (long long)((key >> 21) & 0x1fffffull);
+        ny = (long long)(key & 0x1fffffull);
+    }
     for (uint32_t e = sl; e < n_expr; e += L) val[e] = aff8(__ldg(&S.plan_expr[e0 + e]), nx, ny);
     __syncwarp();
     double T = 0.0;
@@ -449,128 +466,198 @@ struct Params {
     unsigned int *ticket;
     grophecy_best_result *out;
     int accumulate;
+    int aligned;    // record arrays 16-byte aligned -> vector loads
 };
 
+__device__ __forceinline__ unsigned long long key_of(const SpaceDev &S, uint32_t skx, uint32_t nx,
+                                                     uint32_t ny, uint32_t it, bool has)
+{
+    const uint32_t skel = skx >> 16, x = skx & 0xffffu;
+    bool valid = has && skel < S.n_skels && nx >= 1 && nx <= GROPHECY_MAX_DIM && ny >= 1 &&
+                 ny <= GROPHECY_MAX_DIM && it >= 1;
+    if (valid) valid = x < S.skel[skel].n_xforms;
+    return valid ? ((unsigned long long)skel << 42) | ((unsigned long long)nx << 21) | ny : ~0ull;
+}
+
 template <bool BEST>
-__global__ void __launch_bounds__(THREADS, 3) project_kernel(const Params P)
+__global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const Params P)
 {
     __shared__ WarpScratch scratch[WARPS];
+    __shared__ unsigned long long slot_key[SLOT_CAP];
+    __shared__ Usage res[SLOT_CAP];
+    __shared__ unsigned long long last_key[WARPS];
+    __shared__ unsigned wsum[WARPS];
     __shared__ Best wbest[WARPS];
     __shared__ bool am_last;
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    WarpScratch &ws = scratch[warp];
     const SpaceDev &S = P.S;
 
     Best mine = none_best();
-    const unsigned long long ntiles = (P.n + 31) >> 5;
-    const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
-    unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp;
-    // software pipeline: records of the next tile are loaded while this one computes
-    uint32_t c_skx = 0, c_nx = 0, c_ny = 0, c_it = 0;
-    {
-        const unsigned long long i = (tile << 5) + lane;
-        if (tile < ntiles && i < P.n) {
-            c_skx = __ldcs(P.skx + i); c_nx = __ldcs(P.nx + i);
-            c_ny = __ldcs(P.ny + i); c_it = __ldcs(P.iters + i);
-        }
-    }
-    for (; tile < ntiles; tile += wstride) {
-        const unsigned long long i = (tile << 5) + lane;
-        const bool has = i < P.n;
-        const uint32_t skx = c_skx, nx = c_nx, ny = c_ny, it = c_it;
-        {
-            const unsigned long long nt = tile + wstride, ni = (nt << 5) + lane;
-            c_skx = c_nx = c_ny = c_it = 0;
-            if (nt < ntiles && ni < P.n) {
-                c_skx = __ldcs(P.skx + ni); c_nx = __ldcs(P.nx + ni);
-                c_ny = __ldcs(P.ny + ni); c_it = __ldcs(P.iters + ni);
-            }
-        }
-        const uint32_t skel = skx >> 16, x = skx & 0xffffu;
-        bool valid = has && skel < S.n_skels && nx >= 1 && nx <= GROPHECY_MAX_DIM && ny >= 1 &&
-                     ny <= GROPHECY_MAX_DIM && it >= 1;
-        if (valid) valid = x < S.skel[skel].n_xforms;
-        const unsigned long long key =
-            valid ? ((unsigned long long)skel << 42) | ((unsigned long long)nx << 21) | ny : ~0ull;
-        unsigned pending = __ballot_sync(FULL, valid);
-        double t = __longlong_as_double(0x7ff8000000000000LL);   // NaN for invalid
-        Usage u = {0ull, 0ull, 0.0, 0.0};
-        // rounds of one or two distinct keys (usage is shared by every lane
-        // with the same key; the model then runs per lane)
-        while (pending) {
-            const int LA = __ffs(pending) - 1;
-            const unsigned long long kA = __shfl_sync(FULL, key, LA);
-            const unsigned sameA = __ballot_sync(FULL, key == kA);
-            const uint32_t sA = (uint32_t)(kA >> 42);
-            const long long nxA = (long long)((kA >> 21) & 0x1fffffull);
-            const long long nyA = (long long)(kA & 0x1fffffull);
-            const SkelInfo &IA = S.skel[sA];
-            const bool planA = nxA >= IA.plan_tx && nyA >= IA.plan_ty;
-            const uint32_t naA = IA.n_arrays;
-            const unsigned rest = pending & ~sameA;
-            bool two = false;
-            unsigned long long kB = ~0ull;
-            if (planA && naA <= 8 && rest) {
-                kB = __shfl_sync(FULL, key, __ffs(rest) - 1);
-                const SkelInfo &IB = S.skel[(uint32_t)(kB >> 42)];
-                two = (long long)((kB >> 21) & 0x1fffffull) >= IB.plan_tx &&
-                      (long long)(kB & 0x1fffffull) >= IB.plan_ty && IB.n_arrays <= 8;
-            }
-            const long long *myval = nullptr;
-            Usage r;
-            if (two) {
-                const unsigned sameB = __ballot_sync(FULL, key == kB);
-                const int h = lane >> 4;
-                const unsigned long long kh = h ? kB : kA;
-                const uint32_t naB = S.skel[(uint32_t)(kB >> 42)].n_arrays;
-                r = plan_usage(S, (uint32_t)(kh >> 42), (long long)((kh >> 21) & 0x1fffffull),
-                               (long long)(kh & 0x1fffffull), P.pc, ws.val[h], lane & 15, 16,
-                               lane & 16, naA > naB ? naA : naB);
-                const int src = key == kB ? 16 : 0;
-                r.h = __shfl_sync(FULL, r.h, src);
-                r.d = __shfl_sync(FULL, r.d, src);
-                r.th = __shfl_sync(FULL, r.th, src);
-                r.td = __shfl_sync(FULL, r.td, src);
-                myval = ws.val[key == kB ? 1 : 0];
-                pending &= ~(sameA | sameB);
-            } else if (planA) {
-                r = plan_usage(S, sA, nxA, nyA, P.pc, ws.val[0], lane, 32, 0, naA);
-                myval = ws.val[0];
-                pending &= ~sameA;
-            } else {
-                r = warp_usage_sweep(S, IA, nxA, nyA, P.pc, ws, lane);
-                pending &= ~sameA;
-            }
-            if (key == kA || (two && key == kB)) {
-                u = r;
-                t = candidate_time(S, skel, x, nx, ny, it, myval, u);
-            }
-            __syncwarp();   // scratch is reused by the next round
-        }
-        if (!BEST) {
-            if (has) {
-                __stcs(P.h2d + i, valid ? u.h : 0ull);
-                __stcs(P.d2h + i, valid ? u.d : 0ull);
-                __stcs(P.t + i, t);
-            }
-            const unsigned inv = __ballot_sync(FULL, has && !valid);
-            if (lane == 0 && inv) atomicAdd(S.invalid_counter, (unsigned long long)__popc(inv));
+    const unsigned long long ntiles = (P.n + TILE - 1) / TILE;
+    for (unsigned long long tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        // ---- A: load 4 consecutive records per thread, keys, run heads ----
+        const unsigned long long r0 = tile * TILE + (unsigned long long)threadIdx.x * RPT;
+        uint32_t skx[RPT], nx[RPT], ny[RPT], it[RPT];
+        if (P.aligned && r0 + RPT <= P.n) {
+            const uint4 a = __ldcs((const uint4 *)(P.skx + r0));
+            const uint4 b = __ldcs((const uint4 *)(P.nx + r0));
+            const uint4 c = __ldcs((const uint4 *)(P.ny + r0));
+            const uint4 d = __ldcs((const uint4 *)(P.iters + r0));
+            skx[0] = a.x; skx[1] = a.y; skx[2] = a.z; skx[3] = a.w;
+            nx[0] = b.x; nx[1] = b.y; nx[2] = b.z; nx[3] = b.w;
+            ny[0] = c.x; ny[1] = c.y; ny[2] = c.z; ny[3] = c.w;
+            it[0] = d.x; it[1] = d.y; it[2] = d.z; it[3] = d.w;
         } else {
-            if (has) {
-                if (!valid) {
-                    mine.ninv++;
-                } else {
-                    mine.nval++;
-                    if (t < __longlong_as_double(0x7ff0000000000000LL) &&
-                        better(t, P.base + i, mine.t, mine.i)) {
-                        mine.t = t;
-                        mine.i = P.base + i;
-                        mine.h = u.h;
-                        mine.d = u.d;
-                    }
+#pragma unroll
+            for (int j = 0; j < RPT; j++) {
+                const bool h = r0 + j < P.n;
+                skx[j] = h ? __ldcs(P.skx + r0 + j) : 0u;
+                nx[j] = h ? __ldcs(P.nx + r0 + j) : 0u;
+                ny[j] = h ? __ldcs(P.ny + r0 + j) : 0u;
+                it[j] = h ? __ldcs(P.iters + r0 + j) : 0u;
+            }
+        }
+        unsigned long long key[RPT];
+#pragma unroll
+        for (int j = 0; j < RPT; j++) key[j] = key_of(S, skx[j], nx[j], ny[j], it[j], r0 + j < P.n);
+        if (lane == 31) last_key[warp] = key[RPT - 1];
+        __syncthreads();
+        unsigned long long prev = __shfl_up_sync(FULL, key[RPT - 1], 1);
+        if (lane == 0) prev = warp ? last_key[warp - 1] : ~0ull;
+        unsigned head = 0;   // bit j: record j starts a run of a valid key
+#pragma unroll
+        for (int j = 0; j < RPT; j++) {
+            const unsigned long long pk = j ? key[j - 1] : prev;
+            if (key[j] != ~0ull && key[j] != pk) head |= 1u << j;
+        }
+        // block exclusive scan of head counts -> slot ids
+        const unsigned cnt = __popc(head);
+        unsigned inc = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned v = __shfl_up_sync(FULL, inc, o);
+            if (lane >= o) inc += v;
+        }
+        if (lane == 31) wsum[warp] = inc;
+        __syncthreads();
+        unsigned before = 0, nslots = 0;
+#pragma unroll
+        for (int w = 0; w < WARPS; w++) {
+            const unsigned v = wsum[w];
+            before += w < warp ? v : 0u;
+            nslots += v;
+        }
+        const unsigned excl = before + inc - cnt;
+        int slot[RPT];
+        {
+            unsigned s = excl;
+#pragma unroll
+            for (int j = 0; j < RPT; j++) {
+                if ((head >> j) & 1u) s++;
+                slot[j] = key[j] == ~0ull ? -1 : (int)s - 1;
+            }
+        }
+
+        for (unsigned c0 = 0; c0 < nslots; c0 += SLOT_CAP) {
+            const unsigned c1 = min(nslots, c0 + SLOT_CAP);
+#pragma unroll
+            for (int j = 0; j < RPT; j++)
+                if (((head >> j) & 1u) && (unsigned)slot[j] >= c0 && (unsigned)slot[j] < c1)
+                    slot_key[slot[j] - c0] = ((unsigned long long)(skx[j] >> 16) << 42) |
+                                             ((unsigned long long)nx[j] << 21) | ny[j];
+            __syncthreads();
+            // ---- B: usage of every distinct key of the chunk, once ----
+            for (unsigned g0 = c0 + warp * 8; g0 < c1; g0 += WARPS * 8) {
+                const unsigned gcnt = min(8u, c1 - g0);
+                const bool mv = (unsigned)lane < gcnt;
+                const unsigned long long mk = mv ? slot_key[g0 - c0 + lane] : 0ull;
+                bool mplan = false;
+                uint32_t mna = 0, mne = 0;
+                if (mv) {
+                    const SkelInfo &I = S.skel[(uint32_t)(mk >> 42)];
+                    mplan = (long long)((mk >> 21) & 0x1fffffull) >= I.plan_tx &&
+                            (long long)(mk & 0x1fffffull) >= I.plan_ty;
+                    mna = I.n_arrays;
+                    mne = I.n_expr;
+                }
+                unsigned todo = __ballot_sync(FULL, mv && mplan);
+                unsigned sweep = __ballot_sync(FULL, mv && !mplan);
+                const uint32_t max_na = __reduce_max_sync(FULL, mplan ? mna : 0u);
+                const uint32_t max_ne = __reduce_max_sync(FULL, mplan ? mne : 0u);
+                int L = 2;
+                while (L < 2 * (int)max_na) L <<= 1;
+                while ((32 / L) * (int)max_ne > VAL_PER_WARP) L <<= 1;
+                const int G = 32 / L, seg = lane / L, sl = lane % L;
+                while (todo) {
+                    const unsigned pos = __fns(todo, 0, seg + 1);
+                    const bool act = pos < 32u;
+                    const unsigned long long k = __shfl_sync(FULL, mk, act ? pos : 0);
+                    const Usage r = plan_usage(S, act, k, P.pc,
+                                               scratch[warp].val + seg * (VAL_PER_WARP / G), sl, L,
+                                               seg * L, max_na);
+                    if (act && sl == 0) res[g0 - c0 + pos] = r;
+                    for (int q = 0; q < G && todo; q++) todo &= todo - 1;
+                    __syncwarp();
+                }
+                while (sweep) {
+                    const int pos = __ffs(sweep) - 1;
+                    const unsigned long long k = __shfl_sync(FULL, mk, pos);
+                    const Usage r = warp_usage_sweep(S, S.skel[(uint32_t)(k >> 42)],
+                                                     (long long)((k >> 21) & 0x1fffffull),
+                                                     (long long)(k & 0x1fffffull), P.pc,
+                                                     scratch[warp], lane);
+                    if (lane == 0) res[g0 - c0 + pos] = r;
+                    sweep &= sweep - 1;
+                    __syncwarp();
                 }
             }
+            __syncthreads();
+            // ---- C: per-candidate model + output / argmin ----
+#pragma unroll
+            for (int j = 0; j < RPT; j++) {
+                const unsigned long long i = r0 + j;
+                if (slot[j] < (int)c0 || slot[j] >= (int)c1) continue;
+                const Usage u = res[slot[j] - c0];
+                const double t = candidate_time(S, skx[j] >> 16, skx[j] & 0xffffu, nx[j], ny[j],
+                                                it[j], nullptr, u);
+                if (!BEST) {
+                    __stcs(P.h2d + i, u.h);
+                    __stcs(P.d2h + i, u.d);
+                    __stcs(P.t + i, t);
+                } else if (t < __longlong_as_double(0x7ff0000000000000LL) &&
+                           better(t, P.base + i, mine.t, mine.i)) {
+                    mine.t = t;
+                    mine.i = P.base + i;
+                    mine.h = u.h;
+                    mine.d = u.d;
+                }
+            }
+            __syncthreads();
+        }
+        // invalid records (no slot) and counters
+        unsigned ninv = 0, nval = 0;
+#pragma unroll
+        for (int j = 0; j < RPT; j++) {
+            const unsigned long long i = r0 + j;
+            if (i >= P.n) continue;
+            if (slot[j] < 0) {
+                ninv++;
+                if (!BEST) {
+                    __stcs(P.h2d + i, 0ull);
+                    __stcs(P.d2h + i, 0ull);
+                    __stcs(P.t + i, __longlong_as_double(0x7ff8000000000000LL));
+                }
+            } else {
+                nval++;
+            }
+        }
+        if (BEST) {
+            mine.ninv += ninv;
+            mine.nval += nval;
+        } else {
+            const unsigned tot = __reduce_add_sync(FULL, ninv);
+            if (lane == 0 && tot) atomicAdd(S.invalid_counter, (unsigned long long)tot);
         }
     }
     if (!BEST) return;
@@ -630,14 +717,12 @@ __global__ void combine_kernel(const grophecy_best_result *in, uint32_t count,
 
 static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_cap)
 {
-    static int occ_best = 0, occ_eval = 0;
-    (void)occ_eval;
+    static int occ_best = 0;
     if (!occ_best) {
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_best, project_kernel<true>, THREADS, 0);
         if (occ_best < 1) occ_best = 1;
     }
-    const unsigned long long tiles = (n + 31) / 32;
-    unsigned long long want = (tiles + WARPS - 1) / WARPS;
+    const unsigned long long want = (n + TILE - 1) / TILE;
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ_best, per_sm_cap);
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
@@ -674,6 +759,8 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
     P.ticket = s->ticket;
     P.out = nullptr;
     P.accumulate = 0;
+    const uintptr_t m = (uintptr_t)b->skx | (uintptr_t)b->nx | (uintptr_t)b->ny | (uintptr_t)b->iters;
+    P.aligned = (m & 15u) == 0;
     return P;
 }
 
