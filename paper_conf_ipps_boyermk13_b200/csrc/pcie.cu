@@ -30,7 +30,7 @@ struct XferBuffers {
 };
 constexpr int MAX_DEV = 64;
 XferBuffers g_buf[MAX_DEV];
-std::mutex g_mu;
+std::mutex g_mu[MAX_DEV];   // one per device: concurrent mode measures all GPUs at once
 
 int ensure(int device, size_t bytes, XferBuffers *&out)
 {
@@ -78,7 +78,11 @@ int grophecy_measure_transfer(int device, int direction, uint64_t bytes, int rep
         set_error("grophecy_measure_transfer: bad arguments");
         return GROPHECY_EINVAL;
     }
-    std::lock_guard<std::mutex> lock(g_mu);
+    if (device < 0 || device >= MAX_DEV) {
+        set_error("device index out of range");
+        return GROPHECY_EINVAL;
+    }
+    std::lock_guard<std::mutex> lock(g_mu[device]);
     int prev = 0;
     cudaGetDevice(&prev);
     cudaError_t e = cudaSetDevice(device);
