@@ -121,14 +121,13 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-def profile_traffic():
-    """Per-launch DRAM traffic of the best kernel from the committed ncu
-    capture (profiles/ncu_best_summary.json), if present."""
+def profile_summary():
+    """Per-launch DRAM traffic and executed warp instructions of the best
+    kernel from the committed ncu capture (profiles/ncu_best_summary.json)."""
     p = os.path.join(ROOT, "profiles", "ncu_best_summary.json")
     if not os.path.exists(p):
-        return None, None
-    d = json.load(open(p))
-    return d.get("dram_bytes_per_launch"), d.get("n_candidates")
+        return {}
+    return json.load(open(p))
 
 
 # ---------------------------------------------------------------- oracle legs
@@ -285,9 +284,10 @@ def main():
     value = N * args.steps / (ms_max * 1e-3)
     peak, peak_src = measured_peaks()
     achieved = 16.0 * n_local / (kern_avg_max * 1e-3) / 1e9
-    traffic, traffic_n = profile_traffic()
-    if traffic is not None and traffic_n:
-        traffic = traffic * n_local / traffic_n
+    prof = profile_summary()
+    traffic, prof_n = prof.get("dram_bytes_per_launch"), prof.get("n_candidates")
+    if traffic is not None and prof_n:
+        traffic = traffic * n_local / prof_n
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": achieved / peak, "traffic": traffic,
             "kernel": "project_kernel<best> (fused projection + argmin)",
@@ -295,6 +295,20 @@ def main():
             "kernel_ms_avg": kern_avg_max, "peak_source": peak_src,
             "note": "16 B/candidate record read (DESIGN.md §5); kernel duration from CUDA "
                     "events around each launch on its stream"}
+    # the binding resource: instruction issue (executed warp instructions per
+    # candidate from the committed ncu capture x this run's candidates / time)
+    roof_issue = None
+    if prof.get("warp_inst_per_launch") and prof_n:
+        sm_mhz = (clocks or {}).get("sm_mhz") or 1965.0
+        props = torch.cuda.get_device_properties(local_rank)
+        peak_issue = props.multi_processor_count * 4 * sm_mhz * 1e6
+        ach = prof["warp_inst_per_launch"] / prof_n * n_local / (kern_avg_max * 1e-3)
+        roof_issue = {"bound": "alu", "achieved": ach, "peak": peak_issue,
+                      "unit": "warp-inst/s", "frac": ach / peak_issue,
+                      "warp_inst_per_candidate": prof["warp_inst_per_launch"] / prof_n,
+                      "note": "executed (not algorithmic) warp instructions from "
+                              + prof.get("source", "profiles/") + "; peak = SMs x 4 "
+                              "schedulers x 1 inst/clk x measured SM clock"}
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         threads = cpu_cores()
@@ -314,7 +328,7 @@ def main():
                        "gpu_model": "Quadro FX 5600 preset (paper's GPU, P:L149)",
                        "pcie": "alpha=1e-5 s, 1/beta=2.5 GB/s (paper magnitudes, P:L111)",
                        "l2": "inputs 16 B x shard >> 126 MB L2; no flush needed"},
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "roofline": roof, "roofline_issue": roof_issue, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
             "gpu_launches": launches,
             "best": {"index": best.index, "t_total_s": best.t_total_s,
                      "h2d_bytes": best.h2d_bytes, "d2h_bytes": best.d2h_bytes}}
