@@ -18,11 +18,20 @@ namespace grophecy {
 // "Saturated" grid: blocks >= sat_blocks  <=>  #Active_SMs == n_sm and
 // active blocks/SM == occ; then N, MWP, CWP and the H&K case are constants
 // and cyc = E*rep + S*rep with rep = blocks / D (D = occ * n_sm).
-struct KxES { double E, S; };         // case expression, synch factor
-struct KxD  { double D, rD; };        // rep denominator and RN(1/D)
-struct KxI  { uint64_t magic; uint64_t sat_blocks; };  // ceil(2^64/ipb) (0 if ipb==1)
-struct KxJ  { uint32_t ipb, occ, wpb, flags; };        // flags: KXF_*
+struct __align__(16) KxES { double E, S; };         // case expression, synch factor
+struct __align__(16) KxD  { double D, rD; };        // rep denominator and RN(1/D)
+struct __align__(16) KxI  { uint64_t magic; uint64_t sat_blocks; };  // ceil(2^64/ipb) (0 if ipb==1)
+struct __align__(16) KxJ  { uint32_t ipb, occ, wpb, flags; };        // flags: KXF_*
 enum : uint32_t { KXF_INFEASIBLE = 1u, KXF_NOMEM = 2u, KXF_PER_ITER = 4u };
+
+// Packed fast-path record (48 B, one address per (kernel, transformation)):
+// blocks = ceil(W / ipb) from q = hi32(magic_hi*W + hi32(magic_lo*W)) for
+// W < 2^32 - 1 (magic = ceil(2^64/ipb), or 2^64-1 when ipb == 1); saturated
+// iff blocks >= sat32; infeasible (occupancy 0) <=> E == +inf.
+struct __align__(16) KxFast {
+    double E, S, D, rD;
+    uint32_t magic_lo, magic_hi, sat32, ipb;
+};
 
 // General-grid constants (small grids / huge W), read only off the fast path.
 struct KxG {
@@ -75,6 +84,7 @@ struct SpaceDev {
     const KxI *kx_i;
     const KxJ *kx_j;
     const KxG *kx_g;
+    const KxFast *kx_f;
     const int4 *plan_expr;
     const uint32_t *plan_prog;
     uint32_t n_skels;

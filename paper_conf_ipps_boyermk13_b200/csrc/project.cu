@@ -34,8 +34,9 @@ constexpr int THREADS = 256;
 constexpr int WARPS = THREADS / 32;
 constexpr int RPT = 4;                       // records per thread
 constexpr int TILE = THREADS * RPT;          // records per CTA tile
-constexpr int SLOT_CAP = 256;                // distinct keys resident per chunk
+constexpr int SLOT_CAP = 64;                 // distinct keys resident per chunk
 constexpr int VAL_PER_WARP = 256;            // plan expression values per warp
+constexpr int MAXK = GROPHECY_MAX_KERNELS;   // kernels per skeleton
 constexpr long long BIG = 0x7fffffffffffffffLL;
 #ifndef GROPHECY_MINB
 #define GROPHECY_MINB 3
@@ -454,6 +455,66 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
     r.n_valid = b.nval;
 }
 
+// Model of NJ records of one skeleton at once (NJ independent dependency
+// chains per thread).  W[j] = the work-item counts of record j's key (shared
+// memory, one row per distinct key).  The saturated-grid formula is computed
+// branch-free for every record; the rare general-grid / >= 2^32-item cases
+// are recomputed by kernel_time.
+template <int NJ>
+__device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uint32_t *x,
+                                        const uint32_t *it, const uint32_t *const *W,
+                                        const uint32_t *nx, const uint32_t *ny,
+                                        const Usage *const *u, double *t)
+{
+    const SkelInfo &I = S.skel[s];
+    const uint32_t K = I.n_kernels, X = I.n_xforms;
+    double ti[NJ], to[NJ];
+#pragma unroll
+    for (int j = 0; j < NJ; j++) ti[j] = to[j] = 0.0;
+    uint32_t kb = I.kx_base;
+    for (uint32_t k = 0; k < K; k++, kb += X) {
+        double tk[NJ];
+        bool gen[NJ];
+#pragma unroll
+        for (int j = 0; j < NJ; j++) {
+            const KxFast F = S.kx_f[kb + x[j]];
+            const uint32_t w = W[j][k];   // saturated at 2^32 - 1
+            const unsigned long long lo = (unsigned long long)F.magic_lo * w;
+            const uint32_t q = (uint32_t)(((unsigned long long)F.magic_hi * w + (lo >> 32)) >> 32);
+            const uint32_t blocks = q + (q * F.ipb != w);
+            const double rep = div_rn(__uint2double_rn(blocks), F.D, F.rD);
+            const double cyc = __dadd_rn(__dmul_rn(F.E, rep), __dmul_rn(F.S, rep));
+            const double v = div_rn(cyc, S.freq, S.rfreq);
+            const bool inf = isinf(F.E);
+            gen[j] = !inf && blocks != 0 && (w == 0xffffffffu || blocks < F.sat32);
+            tk[j] = inf ? __longlong_as_double(0x7ff0000000000000LL) : (blocks == 0 ? 0.0 : v);
+        }
+#pragma unroll
+        for (int j = 0; j < NJ; j++)
+            if (gen[j]) {
+                const long long Wi = aff8(__ldg(&S.kern_work[I.k_base + k]), nx[j], ny[j]);
+                tk[j] = kernel_time(S, Wi, S.kx_j[kb + x[j]], kb + x[j]);
+            }
+        if (__ldg(&S.kern_flags[I.k_base + k]) & GROPHECY_KERNEL_PER_ITER) {
+#pragma unroll
+            for (int j = 0; j < NJ; j++) ti[j] = __dadd_rn(ti[j], tk[j]);
+        } else {
+#pragma unroll
+            for (int j = 0; j < NJ; j++) to[j] = __dadd_rn(to[j], tk[j]);
+        }
+    }
+#pragma unroll
+    for (int j = 0; j < NJ; j++) {
+        const double t_kern = __dadd_rn(to[j], __dmul_rn((double)it[j], ti[j]));
+        t[j] = __dadd_rn(__dadd_rn(t_kern, u[j]->th), u[j]->td);
+    }
+}
+
+__device__ __forceinline__ uint32_t sat_u32(long long w)
+{
+    return w <= 0 ? 0u : (w >= 0xffffffffLL ? 0xffffffffu : (uint32_t)w);
+}
+
 struct Params {
     SpaceDev S;
     grophecy_pcie pc;
@@ -485,6 +546,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
     __shared__ WarpScratch scratch[WARPS];
     __shared__ unsigned long long slot_key[SLOT_CAP];
     __shared__ Usage res[SLOT_CAP];
+    __shared__ uint32_t slot_w[SLOT_CAP][MAXK];    // work-item counts per distinct key (saturated)
     __shared__ unsigned long long last_key[WARPS];
     __shared__ unsigned wsum[WARPS];
     __shared__ Best wbest[WARPS];
@@ -593,10 +655,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     const unsigned pos = __fns(todo, 0, seg + 1);
                     const bool act = pos < 32u;
                     const unsigned long long k = __shfl_sync(FULL, mk, act ? pos : 0);
-                    const Usage r = plan_usage(S, act, k, P.pc,
-                                               scratch[warp].val + seg * (VAL_PER_WARP / G), sl, L,
-                                               seg * L, max_na);
-                    if (act && sl == 0) res[g0 - c0 + pos] = r;
+                    long long *v = scratch[warp].val + seg * (VAL_PER_WARP / G);
+                    const Usage r = plan_usage(S, act, k, P.pc, v, sl, L, seg * L, max_na);
+                    if (act) {
+                        if (sl == 0) res[g0 - c0 + pos] = r;
+                        const uint32_t K = S.skel[(uint32_t)(k >> 42)].n_kernels;
+                        for (uint32_t q = sl; q < K; q += L) slot_w[g0 - c0 + pos][q] = sat_u32(v[q]);
+                    }
                     for (int q = 0; q < G && todo; q++) todo &= todo - 1;
                     __syncwarp();
                 }
@@ -608,29 +673,57 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                                                      (long long)(k & 0x1fffffull), P.pc,
                                                      scratch[warp], lane);
                     if (lane == 0) res[g0 - c0 + pos] = r;
+                    {
+                        const SkelInfo &I = S.skel[(uint32_t)(k >> 42)];
+                        if ((uint32_t)lane < I.n_kernels)
+                            slot_w[g0 - c0 + pos][lane] = sat_u32(
+                                aff8(__ldg(&S.kern_work[I.k_base + lane]),
+                                     (long long)((k >> 21) & 0x1fffffull), (long long)(k & 0x1fffffull)));
+                    }
                     sweep &= sweep - 1;
                     __syncwarp();
                 }
             }
             __syncthreads();
             // ---- C: per-candidate model + output / argmin ----
+            bool inj[RPT];
+            uint32_t xs[RPT];
+            const uint32_t *wp[RPT];
+            const Usage *up[RPT];
+            double tt[RPT];
+            bool all = true;
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
+                inj[j] = slot[j] >= (int)c0 && slot[j] < (int)c1;
+                const int ls = inj[j] ? slot[j] - (int)c0 : 0;
+                xs[j] = skx[j] & 0xffffu;
+                wp[j] = slot_w[ls];
+                up[j] = &res[ls];
+                all = all && inj[j] && (skx[j] >> 16) == (skx[0] >> 16);
+            }
+            if (all) {
+                model_n<RPT>(S, skx[0] >> 16, xs, it, wp, nx, ny, up, tt);
+            } else {
+#pragma unroll
+                for (int j = 0; j < RPT; j++)
+                    if (inj[j])
+                        model_n<1>(S, skx[j] >> 16, xs + j, it + j, wp + j, nx + j, ny + j, up + j, tt + j);
+            }
+#pragma unroll
+            for (int j = 0; j < RPT; j++) {
+                if (!inj[j]) continue;
                 const unsigned long long i = r0 + j;
-                if (slot[j] < (int)c0 || slot[j] >= (int)c1) continue;
-                const Usage u = res[slot[j] - c0];
-                const double t = candidate_time(S, skx[j] >> 16, skx[j] & 0xffffu, nx[j], ny[j],
-                                                it[j], nullptr, u);
+                const double t = tt[j];
                 if (!BEST) {
-                    __stcs(P.h2d + i, u.h);
-                    __stcs(P.d2h + i, u.d);
+                    __stcs(P.h2d + i, up[j]->h);
+                    __stcs(P.d2h + i, up[j]->d);
                     __stcs(P.t + i, t);
                 } else if (t < __longlong_as_double(0x7ff0000000000000LL) &&
                            better(t, P.base + i, mine.t, mine.i)) {
                     mine.t = t;
                     mine.i = P.base + i;
-                    mine.h = u.h;
-                    mine.d = u.d;
+                    mine.h = up[j]->h;
+                    mine.d = up[j]->d;
                 }
             }
             __syncthreads();

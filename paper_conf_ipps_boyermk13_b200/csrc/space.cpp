@@ -246,6 +246,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxI> ki;
     std::vector<KxJ> kj;
     std::vector<KxG> kg;
+    std::vector<KxFast> kf;
     std::vector<int4> pexpr;
     std::vector<uint32_t> pprog;
     auto a4 = [](const grophecy_affine8 &a) { return make_int4(a.c0, a.c1, a.c2, a.c3); };
@@ -319,6 +320,18 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 if (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) j.flags |= KXF_PER_ITER;
                 kes.push_back(es); kd.push_back(d); ki.push_back(i); kj.push_back(j);
                 kg.push_back(g);
+                KxFast f;
+                if (j.flags & KXF_INFEASIBLE) {
+                    f.E = INFINITY; f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0;
+                } else {
+                    f.E = es.E; f.S = es.S; f.D = d.D; f.rD = d.rD;
+                    f.sat32 = i.sat_blocks > 0xffffffffull ? 0xffffffffu : (uint32_t)i.sat_blocks;
+                }
+                const uint64_t m = j.ipb == 1 ? ~0ull : i.magic;
+                f.magic_lo = (uint32_t)m;
+                f.magic_hi = (uint32_t)(m >> 32);
+                f.ipb = j.ipb;
+                kf.push_back(f);
             }
     }
 
@@ -337,6 +350,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {kg.data(), kg.size() * sizeof(KxG), 0},
         {pexpr.data(), pexpr.size() * sizeof(int4), 0},
         {pprog.data(), pprog.size() * sizeof(uint32_t), 0},
+        {kf.data(), kf.size() * sizeof(KxFast), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -392,6 +406,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.kx_g = (const KxG *)(base + parts[9].off);
     D.plan_expr = (const int4 *)(base + parts[10].off);
     D.plan_prog = (const uint32_t *)(base + parts[11].off);
+    D.kx_f = (const KxFast *)(base + parts[12].off);
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;
     D.freq = gpu->freq_hz;
