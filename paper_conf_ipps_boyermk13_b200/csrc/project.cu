@@ -460,7 +460,7 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
 // memory, one row per distinct key).  The saturated-grid formula is computed
 // branch-free for every record; the rare general-grid / >= 2^32-item cases
 // are recomputed by kernel_time.
-template <int NJ>
+template <int NJ, bool SAMEX>
 __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uint32_t *x,
                                         const uint32_t *it, const uint32_t *const *W,
                                         const uint32_t *nx, const uint32_t *ny,
@@ -475,9 +475,11 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
     for (uint32_t k = 0; k < K; k++, kb += X) {
         double tk[NJ];
         bool gen[NJ];
+        KxFast F0;
+        if (SAMEX) F0 = S.kx_f[kb + x[0]];   // one constant load shared by the NJ records
 #pragma unroll
         for (int j = 0; j < NJ; j++) {
-            const KxFast F = S.kx_f[kb + x[j]];
+            const KxFast F = SAMEX ? F0 : S.kx_f[kb + x[j]];
             const uint32_t w = W[j][k];   // saturated at 2^32 - 1
             const unsigned long long lo = (unsigned long long)F.magic_lo * w;
             const uint32_t q = (uint32_t)(((unsigned long long)F.magic_hi * w + (lo >> 32)) >> 32);
@@ -547,6 +549,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
     __shared__ unsigned long long slot_key[SLOT_CAP];
     __shared__ Usage res[SLOT_CAP];
     __shared__ uint32_t slot_w[SLOT_CAP][MAXK];    // work-item counts per distinct key (saturated)
+    __shared__ uint32_t rec_skx[TILE], rec_it[TILE];   // the tile's records for the strided model
+    __shared__ int rec_slot[TILE];
     __shared__ unsigned long long last_key[WARPS];
     __shared__ unsigned wsum[WARPS];
     __shared__ Best wbest[WARPS];
@@ -618,6 +622,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             for (int j = 0; j < RPT; j++) {
                 if ((head >> j) & 1u) s++;
                 slot[j] = key[j] == ~0ull ? -1 : (int)s - 1;
+                rec_skx[threadIdx.x * RPT + j] = skx[j];
+                rec_it[threadIdx.x * RPT + j] = it[j];
+                rec_slot[threadIdx.x * RPT + j] = slot[j];
             }
         }
 
@@ -686,33 +693,44 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             }
             __syncthreads();
             // ---- C: per-candidate model + output / argmin ----
+            // strided mapping: thread t takes records t + 256 j, which share the
+            // transformation when candidates come in groups of 16 (or 256/2^k)
             bool inj[RPT];
-            uint32_t xs[RPT];
+            uint32_t xs[RPT], its[RPT], nxs[RPT], nys[RPT];
             const uint32_t *wp[RPT];
             const Usage *up[RPT];
             double tt[RPT];
-            bool all = true;
+            const uint32_t skx0 = rec_skx[threadIdx.x];
+            bool same = true;
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
-                inj[j] = slot[j] >= (int)c0 && slot[j] < (int)c1;
-                const int ls = inj[j] ? slot[j] - (int)c0 : 0;
-                xs[j] = skx[j] & 0xffffu;
+                const int q = threadIdx.x + THREADS * j;
+                const int sj = rec_slot[q];
+                const uint32_t sk = rec_skx[q];
+                inj[j] = sj >= (int)c0 && sj < (int)c1;
+                const int ls = inj[j] ? sj - (int)c0 : 0;
+                xs[j] = sk & 0xffffu;
+                its[j] = rec_it[q];
                 wp[j] = slot_w[ls];
                 up[j] = &res[ls];
-                all = all && inj[j] && (skx[j] >> 16) == (skx[0] >> 16);
+                const unsigned long long kk = slot_key[ls];
+                nxs[j] = (uint32_t)((kk >> 21) & 0x1fffffull);
+                nys[j] = (uint32_t)(kk & 0x1fffffull);
+                same = same && inj[j] && sk == skx0;
             }
-            if (all) {
-                model_n<RPT>(S, skx[0] >> 16, xs, it, wp, nx, ny, up, tt);
+            if (same) {
+                model_n<RPT, true>(S, skx0 >> 16, xs, its, wp, nxs, nys, up, tt);
             } else {
 #pragma unroll
                 for (int j = 0; j < RPT; j++)
                     if (inj[j])
-                        model_n<1>(S, skx[j] >> 16, xs + j, it + j, wp + j, nx + j, ny + j, up + j, tt + j);
+                        model_n<1, false>(S, rec_skx[threadIdx.x + THREADS * j] >> 16, xs + j,
+                                          its + j, wp + j, nxs + j, nys + j, up + j, tt + j);
             }
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
                 if (!inj[j]) continue;
-                const unsigned long long i = r0 + j;
+                const unsigned long long i = tile * TILE + threadIdx.x + THREADS * j;
                 const double t = tt[j];
                 if (!BEST) {
                     __stcs(P.h2d + i, up[j]->h);
