@@ -267,6 +267,12 @@ int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int64_t nx, int
                              uint64_t *h2d_per_array, uint64_t *d2h_per_array,
                              uint32_t *plan_tx, uint32_t *plan_ty);
 
+/* Diagnostic: size of the usage plan compiled for `skel`: stats[0] =
+ * expressions, [1] = program words, [2] = terms, [3] = terms, [4] = max terms
+ * of one array program, [5] = max words of one program.  ELIMIT if the
+ * skeleton has no plan.  Pure host function. */
+int grophecy_plan_stats(const grophecy_skeleton_desc *skel, uint32_t *stats);
+
 /* Number of CUDA kernel launches issued by this library since load (for
  * the bench's gpu_launches count). */
 uint64_t grophecy_launch_count(void);

@@ -54,7 +54,7 @@ struct ArrayDev {
     uint32_t h_prog, d_prog, pad0, pad1;             // plan band programs (u32 word offsets)
 };
 
-constexpr uint32_t PLAN_MAX_EXPR = 128;
+constexpr uint32_t PLAN_MAX_EXPR = 128;   // < 256: programs pack u8 indices
 
 // Host-side result of compiling one skeleton's usage plan.
 struct SkelPlanHost {

@@ -169,17 +169,19 @@ bool compile_array(const grophecy_array_desc &A, const std::vector<const grophec
     return true;
 }
 
-// Emit the band program of one cell matrix as u32 words:
-//   [n_bands] then per band [rs | re << 16, n_runs, (cs | ce << 16) x n_runs]
-// (indices into the skeleton's expression table): count =
-//   sum_bands (val[re] - val[rs]) * sum_runs (val[ce] - val[cs]).
+// Emit the program of one cell matrix as u32 words: [n_terms] then one word
+// per (band, run) term packing four expression indices (u8 each):
+//   rs | re << 8 | cs << 16 | ce << 24,
+//   count = sum_terms (val[re] - val[rs]) * (val[ce] - val[cs]).
+// Bands merge consecutive row slabs with identical column patterns; runs are
+// maximal column runs of a band.
 template <class F>
 void emit(const std::vector<std::vector<uint8_t>> &cell, const std::vector<Ex> &rowv,
           const std::vector<Ex> &colv, F idx, std::vector<uint32_t> &out)
 {
     const size_t at = out.size();
     out.push_back(0);
-    uint32_t nb = 0;
+    uint32_t nt = 0;
     const int nr = (int)cell.size();
     int i = 0;
     while (i < nr) {
@@ -188,24 +190,19 @@ void emit(const std::vector<std::vector<uint8_t>> &cell, const std::vector<Ex> &
         if (!any) { i++; continue; }
         int e = i + 1;
         while (e < nr && cell[e] == cell[i]) e++;
-        // band rows [i, e): from rowv[i] to rowv[e]
-        std::vector<std::pair<int, int>> runs;
         const int nc = (int)cell[i].size();
         for (int j = 0; j < nc;) {
             if (!cell[i][j]) { j++; continue; }
             int k = j + 1;
             while (k < nc && cell[i][k]) k++;
-            runs.push_back({j, k});
+            out.push_back((uint32_t)idx(rowv[i]) | ((uint32_t)idx(rowv[e]) << 8) |
+                          ((uint32_t)idx(colv[j]) << 16) | ((uint32_t)idx(colv[k]) << 24));
+            nt++;
             j = k;
         }
-        out.push_back((uint32_t)idx(rowv[i]) | ((uint32_t)idx(rowv[e]) << 16));
-        out.push_back((uint32_t)runs.size());
-        for (auto &r : runs)
-            out.push_back((uint32_t)idx(colv[r.first]) | ((uint32_t)idx(colv[r.second]) << 16));
-        nb++;
         i = e;
     }
-    out[at] = nb;
+    out[at] = nt;
 }
 
 }  // namespace
@@ -307,20 +304,42 @@ extern "C" int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int6
     for (uint32_t a = 0; a < skel->n_arrays; a++) {
         for (int which = 0; which < 2; which++) {
             const uint32_t *p = P.prog.data() + (which ? P.d_off[a] : P.h_off[a]);
-            const uint32_t nb = *p++;
+            const uint32_t nt = *p++;
             uint64_t cnt = 0;
-            for (uint32_t b = 0; b < nb; b++) {
-                const int64_t rh = val[p[0] >> 16] - val[p[0] & 0xffff];
-                const uint32_t nr = p[1];
-                p += 2;
-                int64_t w = 0;
-                for (uint32_t q = 0; q < nr; q++, p++) w += val[*p >> 16] - val[*p & 0xffff];
-                cnt += (uint64_t)(rh * w);
+            for (uint32_t t = 0; t < nt; t++, p++) {
+                const uint32_t w = *p;
+                cnt += (uint64_t)((val[(w >> 8) & 0xff] - val[w & 0xff]) *
+                                  (val[w >> 24] - val[(w >> 16) & 0xff]));
             }
             const uint64_t eb = skel->arrays[a].elem_bytes;
             if (which == 0) h2d_per_array[a] = cnt * eb;
             else d2h_per_array[a] = (skel->arrays[a].flags & GROPHECY_ARRAY_LIVEOUT) ? cnt * eb : 0;
         }
     }
+    return GROPHECY_OK;
+}
+
+// Diagnostic: size of the compiled plan of `skel` (expressions, program words,
+// bands and runs summed over arrays, max bands of one array).
+extern "C" int grophecy_plan_stats(const grophecy_skeleton_desc *skel, uint32_t *stats)
+{
+    if (!skel || !stats) return GROPHECY_EINVAL;
+    SkelPlanHost P;
+    if (!compile_plan(*skel, P)) return GROPHECY_ELIMIT;
+    uint32_t bands = 0, runs = 0, maxb = 0, maxw = 0;
+    for (uint32_t a = 0; a < skel->n_arrays; a++)
+        for (int which = 0; which < 2; which++) {
+            const uint32_t nt = P.prog[which ? P.d_off[a] : P.h_off[a]];
+            runs += nt;
+            bands += nt;
+            if (nt > maxb) maxb = nt;
+            if (nt + 1 > maxw) maxw = nt + 1;
+        }
+    stats[0] = (uint32_t)P.exprs.size();
+    stats[1] = (uint32_t)P.prog.size();
+    stats[2] = bands;
+    stats[3] = runs;
+    stats[4] = maxb;
+    stats[5] = maxw;
     return GROPHECY_OK;
 }

@@ -132,18 +132,12 @@ __device__ __forceinline__ Usage plan_usage(const SpaceDev &S, bool active, unsi
         const ArrayDev &A = S.arrays[a0 + (sl >> 1)];
         const bool dir_d2h = sl & 1;
         const uint32_t *p = S.plan_prog + (dir_d2h ? A.d_prog : A.h_prog);
-        const uint32_t nb = __ldg(p++);
+        const uint32_t nt = __ldg(p++);
         unsigned long long cnt = 0;
-        for (uint32_t b = 0; b < nb; b++) {
-            const uint32_t w0 = __ldg(p), nr = __ldg(p + 1);
-            p += 2;
-            const long long rh = val[w0 >> 16] - val[w0 & 0xffffu];
-            long long w = 0;
-            for (uint32_t q = 0; q < nr; q++) {
-                const uint32_t wq = __ldg(p++);
-                w += val[wq >> 16] - val[wq & 0xffffu];
-            }
-            cnt += (unsigned long long)(rh * w);
+        for (uint32_t t = 0; t < nt; t++) {
+            const uint32_t w = __ldg(p + t);   // rs | re << 8 | cs << 16 | ce << 24
+            cnt += (unsigned long long)((val[(w >> 8) & 0xffu] - val[w & 0xffu]) *
+                                        (val[w >> 24] - val[(w >> 16) & 0xffu]));
         }
         bytes = (dir_d2h && !A.liveout) ? 0ull : cnt * (unsigned long long)A.elem_bytes;
         const grophecy_link lk = dir_d2h ? pc.d2h : pc.h2d;

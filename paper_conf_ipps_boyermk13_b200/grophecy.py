@@ -133,6 +133,7 @@ _sig = {
     "grophecy_plan_usage_host": (C.c_int, [C.POINTER(SkeletonDesc), C.c_int64, C.c_int64,
                                            C.POINTER(C.c_uint64), C.POINTER(C.c_uint64),
                                            C.POINTER(C.c_uint32), C.POINTER(C.c_uint32)]),
+    "grophecy_plan_stats": (C.c_int, [C.POINTER(SkeletonDesc), C.POINTER(C.c_uint32)]),
     "grophecy_launch_count": (C.c_uint64, []),
     "grophecy_last_error": (C.c_char_p, []),
     "grophecy_abi_version": (C.c_int, []),
@@ -396,6 +397,13 @@ def plan_usage_host(skel, nx, ny):
     rc = _L.grophecy_plan_usage_host(sd.arr, nx, ny, h, d, C.byref(tx), C.byref(ty))
     n = len(skel["arrays"])
     return rc, list(h)[:n], list(d)[:n], tx.value, ty.value
+
+
+def plan_stats(skel):
+    sd = Skeletons([skel])
+    st = (C.c_uint32 * 6)()
+    rc = _L.grophecy_plan_stats(sd.arr, st)
+    return rc, list(st)
 
 
 def launch_count():
