@@ -72,9 +72,16 @@ struct SweepScratch {
     unsigned upto[32];
 };
 
+constexpr int MAX_SEG = 8;                   // keys per warp pass (plan path)
+
+struct PlanScratch {
+    long long val[VAL_PER_WARP];                 // expression values of the pass's keys
+    double T[MAX_SEG][2 * GROPHECY_MAX_ARRAYS];  // per-array transfer times
+};
+
 union WarpScratch {
     SweepScratch sw;                    // general cell sweep (one key per warp)
-    long long val[VAL_PER_WARP];        // usage plans: expression values of G keys
+    PlanScratch pl;                     // usage plans: up to MAX_SEG keys per pass
 };
 
 struct Usage {
@@ -105,56 +112,72 @@ __device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned 
 }
 
 // Usage of one key from its skeleton's compiled plan (plan.cpp), by a segment
-// of L lanes [base, base+L) (several keys per warp).  Lanes first evaluate the
-// plan's expressions (entries 0..K-1 are the kernels' work-item counts), then
-// lane 2a / 2a+1 of the segment runs the H2D / D2H band program of array a
-// and prices its transfer with Eq. (1) (requires 2 * n_arrays <= L); byte
-// totals are an integer tree sum, transfer times an ordered (array-order)
-// floating-point sum.  Inactive segments (active == false) contribute nothing
-// but take part in the shuffles.
-__device__ __forceinline__ Usage plan_usage(const SpaceDev &S, bool active, unsigned long long key,
-                                            const grophecy_pcie &pc, long long *val, int sl, int L,
-                                            int base, uint32_t max_arrays)
+// of L lanes (32/L keys per warp pass).  Lanes evaluate the plan's
+// expressions (entries 0..K-1 are the kernels' work-item counts), then lane sl
+// runs the H2D and D2H programs of arrays sl, sl+L, ... and prices each
+// transfer with Eq. (1) into T[2a + dir]; byte totals are an integer tree sum
+// over the segment, and the segment's lane 0 adds the transfer times in array
+// order.  Results: *res (segment lane 0) and the key's work counts in w_out.
+__device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsigned long long key,
+                                           const grophecy_pcie &pc, long long *val, double *T,
+                                           int sl, int L, Usage *res, uint32_t *w_out)
 {
-    uint32_t n_expr = 0, n_arrays = 0, e0 = 0, a0 = 0;
+    uint32_t n_expr = 0, n_arrays = 0, e0 = 0, a0 = 0, K = 0;
     long long nx = 0, ny = 0;
     if (active) {
         const SkelInfo &I = S.skel[(uint32_t)(key >> 42)];
         n_expr = I.n_expr; n_arrays = I.n_arrays; e0 = I.expr_base; a0 = I.a_base;
+        K = I.n_kernels;
         nx = (long long)((key >> 21) & 0x1fffffull);
         ny = (long long)(key & 0x1fffffull);
     }
     for (uint32_t e = sl; e < n_expr; e += L) val[e] = aff8(__ldg(&S.plan_expr[e0 + e]), nx, ny);
     __syncwarp();
-    double T = 0.0;
-    unsigned long long bytes = 0;
-    if ((uint32_t)sl < 2 * n_arrays) {
-        const ArrayDev &A = S.arrays[a0 + (sl >> 1)];
-        const bool dir_d2h = sl & 1;
-        const uint32_t *p = S.plan_prog + (dir_d2h ? A.d_prog : A.h_prog);
-        const uint32_t nt = __ldg(p++);
-        unsigned long long cnt = 0;
-        for (uint32_t t = 0; t < nt; t++) {
-            const uint32_t w = __ldg(p + t);   // rs | re << 8 | cs << 16 | ce << 24
-            cnt += (unsigned long long)((val[(w >> 8) & 0xffu] - val[w & 0xffu]) *
-                                        (val[w >> 24] - val[(w >> 16) & 0xffu]));
+    unsigned long long hs = 0, ds = 0;
+    for (uint32_t a = sl; a < n_arrays; a += L) {
+        const ArrayDev &A = S.arrays[a0 + a];
+        const uint32_t eb = A.elem_bytes;
+#pragma unroll
+        for (int dir = 0; dir < 2; dir++) {
+            const uint32_t *p = S.plan_prog + (dir ? A.d_prog : A.h_prog);
+            const uint32_t nt = __ldg(p++);
+            unsigned long long cnt = 0;
+#pragma unroll 1
+            for (uint32_t t = 0; t < nt; t++) {
+                const uint32_t w = __ldg(p + t);   // rs | re << 8 | cs << 16 | ce << 24
+                cnt += (unsigned long long)((val[(w >> 8) & 0xffu] - val[w & 0xffu]) *
+                                            (val[w >> 24] - val[(w >> 16) & 0xffu]));
+            }
+            const unsigned long long bytes = (dir && !A.liveout) ? 0ull : cnt * eb;
+            const grophecy_link lk = dir ? pc.d2h : pc.h2d;
+            T[2 * a + dir] = bytes ? __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte,
+                                                                    __ull2double_rn(bytes)))
+                                   : 0.0;
+            if (dir) ds += bytes; else hs += bytes;
         }
-        bytes = (dir_d2h && !A.liveout) ? 0ull : cnt * (unsigned long long)A.elem_bytes;
-        const grophecy_link lk = dir_d2h ? pc.d2h : pc.h2d;
-        if (bytes) T = __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte, __ull2double_rn(bytes)));
     }
-    Usage o;
-    for (int off = 2; off < L; off <<= 1) bytes += __shfl_xor_sync(FULL, bytes, off);
-    o.h = __shfl_sync(FULL, bytes, base);
-    o.d = __shfl_sync(FULL, bytes, base + 1);
-    double th = 0.0, td = 0.0;
-    for (uint32_t a = 0; a < max_arrays; a++) {   // arrays without transfer add +0.0
-        th = __dadd_rn(th, __shfl_sync(FULL, T, base + 2 * a));
-        td = __dadd_rn(td, __shfl_sync(FULL, T, base + 2 * a + 1));
+    for (uint32_t q = sl; q < K; q += L) {
+        const long long v = val[q];
+        w_out[q] = v <= 0 ? 0u : (v >= 0xffffffffLL ? 0xffffffffu : (uint32_t)v);
     }
-    o.th = th;
-    o.td = td;
-    return o;
+    for (int off = 1; off < L; off <<= 1) {
+        hs += __shfl_xor_sync(FULL, hs, off);
+        ds += __shfl_xor_sync(FULL, ds, off);
+    }
+    __syncwarp();
+    if (active && sl == 0) {
+        double th = 0.0, td = 0.0;   // arrays without transfer add +0.0
+        for (uint32_t a = 0; a < n_arrays; a++) {
+            th = __dadd_rn(th, T[2 * a]);
+            td = __dadd_rn(td, T[2 * a + 1]);
+        }
+        Usage o;
+        o.h = hs;
+        o.d = ds;
+        o.th = th;
+        o.td = td;
+        *res = o;
+    }
 }
 
 // Data usage of one (skeleton, nx, ny) key by the general coordinate-compressed
@@ -536,15 +559,27 @@ __device__ __forceinline__ unsigned long long key_of(const SpaceDev &S, uint32_t
     return valid ? ((unsigned long long)skel << 42) | ((unsigned long long)nx << 21) | ny : ~0ull;
 }
 
+// Dynamic shared memory of one CTA (> 48 KB: opt-in attribute at first launch).
+struct CtaSmem {
+    WarpScratch scratch[WARPS];
+    unsigned long long slot_key[SLOT_CAP];      // distinct keys of the chunk
+    Usage res[SLOT_CAP];                        // their usage
+    uint32_t slot_w[SLOT_CAP][MAXK];            // their work-item counts (saturated)
+    uint32_t rec_skx[TILE], rec_it[TILE];       // the tile's records for the strided model
+    int rec_slot[TILE];
+};
+
 template <bool BEST>
 __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const Params P)
 {
-    __shared__ WarpScratch scratch[WARPS];
-    __shared__ unsigned long long slot_key[SLOT_CAP];
-    __shared__ Usage res[SLOT_CAP];
-    __shared__ uint32_t slot_w[SLOT_CAP][MAXK];    // work-item counts per distinct key (saturated)
-    __shared__ uint32_t rec_skx[TILE], rec_it[TILE];   // the tile's records for the strided model
-    __shared__ int rec_slot[TILE];
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    CtaSmem &sm = *reinterpret_cast<CtaSmem *>(smem_raw);
+    WarpScratch *scratch = sm.scratch;
+    unsigned long long *slot_key = sm.slot_key;
+    Usage *res = sm.res;
+    uint32_t (*slot_w)[MAXK] = sm.slot_w;
+    uint32_t *rec_skx = sm.rec_skx, *rec_it = sm.rec_it;
+    int *rec_slot = sm.rec_slot;
     __shared__ unsigned long long last_key[WARPS];
     __shared__ unsigned wsum[WARPS];
     __shared__ Best wbest[WARPS];
@@ -646,23 +681,18 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                 }
                 unsigned todo = __ballot_sync(FULL, mv && mplan);
                 unsigned sweep = __ballot_sync(FULL, mv && !mplan);
-                const uint32_t max_na = __reduce_max_sync(FULL, mplan ? mna : 0u);
                 const uint32_t max_ne = __reduce_max_sync(FULL, mplan ? mne : 0u);
-                int L = 2;
-                while (L < 2 * (int)max_na) L <<= 1;
+                (void)mna;
+                int L = 32 / MAX_SEG;
                 while ((32 / L) * (int)max_ne > VAL_PER_WARP) L <<= 1;
                 const int G = 32 / L, seg = lane / L, sl = lane % L;
                 while (todo) {
                     const unsigned pos = __fns(todo, 0, seg + 1);
                     const bool act = pos < 32u;
                     const unsigned long long k = __shfl_sync(FULL, mk, act ? pos : 0);
-                    long long *v = scratch[warp].val + seg * (VAL_PER_WARP / G);
-                    const Usage r = plan_usage(S, act, k, P.pc, v, sl, L, seg * L, max_na);
-                    if (act) {
-                        if (sl == 0) res[g0 - c0 + pos] = r;
-                        const uint32_t K = S.skel[(uint32_t)(k >> 42)].n_kernels;
-                        for (uint32_t q = sl; q < K; q += L) slot_w[g0 - c0 + pos][q] = sat_u32(v[q]);
-                    }
+                    const unsigned ls = g0 - c0 + (act ? pos : 0);
+                    plan_usage(S, act, k, P.pc, scratch[warp].pl.val + seg * (VAL_PER_WARP / G),
+                               scratch[warp].pl.T[seg], sl, L, &res[ls], slot_w[ls]);
                     for (int q = 0; q < G && todo; q++) todo &= todo - 1;
                     __syncwarp();
                 }
@@ -820,11 +850,24 @@ __global__ void combine_kernel(const grophecy_best_result *in, uint32_t count,
     if (lane == 0) to_result(*out, b);
 }
 
+static void set_smem_attrs()
+{
+    static bool done = false;
+    if (done) return;
+    cudaFuncSetAttribute(project_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)sizeof(CtaSmem));
+    cudaFuncSetAttribute(project_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)sizeof(CtaSmem));
+    done = true;
+}
+
 static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_cap)
 {
     static int occ_best = 0;
+    set_smem_attrs();
     if (!occ_best) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_best, project_kernel<true>, THREADS, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_best, project_kernel<true>, THREADS,
+                                                      sizeof(CtaSmem));
         if (occ_best < 1) occ_best = 1;
     }
     const unsigned long long want = (n + TILE - 1) / TILE;
@@ -876,7 +919,7 @@ int launch_best(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch
     P.out = dout;
     P.accumulate = accumulate;
     const int grid = grid_for(s, b->n, 32);
-    project_kernel<true><<<grid, THREADS, 0, st>>>(P);
+    project_kernel<true><<<grid, THREADS, sizeof(CtaSmem), st>>>(P);
     count_launch();
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "project_kernel<best> launch");
@@ -904,7 +947,7 @@ int grophecy_eval(const grophecy_space *s, const grophecy_pcie *pc, const grophe
     P.d2h = (unsigned long long *)d2h;
     P.t = t;
     const int grid = grid_for(s, b->n, 32);
-    project_kernel<false><<<grid, THREADS, 0, (cudaStream_t)stream>>>(P);
+    project_kernel<false><<<grid, THREADS, sizeof(CtaSmem), (cudaStream_t)stream>>>(P);
     count_launch();
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "project_kernel<eval> launch");
