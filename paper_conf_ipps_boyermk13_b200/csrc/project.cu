@@ -32,14 +32,14 @@ namespace grophecy {
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int THREADS = 256;
 constexpr int WARPS = THREADS / 32;
-constexpr int RPT = 4;                       // records per thread
-constexpr int TILE = THREADS * RPT;          // records per CTA tile
-constexpr int SLOT_CAP = 64;                 // distinct keys resident per chunk
+constexpr int RPT = 4;                       // records per lane
+constexpr int WTILE = 32 * RPT;              // records per warp tile
+constexpr int SLOT_CAP = 16;                 // distinct keys resident per warp chunk
 constexpr int VAL_PER_WARP = 256;            // plan expression values per warp
 constexpr int MAXK = GROPHECY_MAX_KERNELS;   // kernels per skeleton
 constexpr long long BIG = 0x7fffffffffffffffLL;
 #ifndef GROPHECY_MINB
-#define GROPHECY_MINB 3
+#define GROPHECY_MINB 2
 #endif
 
 __device__ __forceinline__ long long aff8(int4 c, long long nx, long long ny)
@@ -559,42 +559,49 @@ __device__ __forceinline__ unsigned long long key_of(const SpaceDev &S, uint32_t
     return valid ? ((unsigned long long)skel << 42) | ((unsigned long long)nx << 21) | ny : ~0ull;
 }
 
-// Dynamic shared memory of one CTA (> 48 KB: opt-in attribute at first launch).
-struct CtaSmem {
-    WarpScratch scratch[WARPS];
+// Per-warp shared memory (dynamic; > 48 KB per CTA needs the opt-in attribute).
+struct WarpSmem {
+    WarpScratch scratch;                        // usage plans / general sweep
     unsigned long long slot_key[SLOT_CAP];      // distinct keys of the chunk
     Usage res[SLOT_CAP];                        // their usage
     uint32_t slot_w[SLOT_CAP][MAXK];            // their work-item counts (saturated)
-    uint32_t rec_skx[TILE], rec_it[TILE];       // the tile's records for the strided model
-    int rec_slot[TILE];
+    uint32_t rec_skx[WTILE], rec_it[WTILE];     // the tile's records, for the strided model
+    int rec_slot[WTILE];
+};
+struct CtaSmem {
+    WarpSmem w[WARPS];
 };
 
+// Persistent kernel; every warp works alone on tiles of 128 consecutive
+// records (no CTA barriers on the hot loop):
+//   A  lane l loads records 4l..4l+3 (one 16-byte load per SoA array), checks
+//      them, and run heads of equal keys get slot ids by a warp scan;
+//   B  usage of each distinct key once (plan: 32/L keys per pass; else sweep);
+//   C  lane l models records l, l+32, l+64, l+96 — the same transformation
+//      when candidates come in groups of 16 — sharing one constant load per
+//      kernel, then writes outputs / keeps its running argmin.
 template <bool BEST>
 __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const Params P)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    CtaSmem &sm = *reinterpret_cast<CtaSmem *>(smem_raw);
-    WarpScratch *scratch = sm.scratch;
-    unsigned long long *slot_key = sm.slot_key;
-    Usage *res = sm.res;
-    uint32_t (*slot_w)[MAXK] = sm.slot_w;
-    uint32_t *rec_skx = sm.rec_skx, *rec_it = sm.rec_it;
-    int *rec_slot = sm.rec_slot;
-    __shared__ unsigned long long last_key[WARPS];
-    __shared__ unsigned wsum[WARPS];
-    __shared__ Best wbest[WARPS];
-    __shared__ bool am_last;
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
+    WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
+    __shared__ Best wbest[WARPS];
+    __shared__ bool am_last;
     const SpaceDev &S = P.S;
+    const unsigned lt = (1u << lane) - 1u;
 
     Best mine = none_best();
-    const unsigned long long ntiles = (P.n + TILE - 1) / TILE;
-    for (unsigned long long tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        // ---- A: load 4 consecutive records per thread, keys, run heads ----
-        const unsigned long long r0 = tile * TILE + (unsigned long long)threadIdx.x * RPT;
+    const unsigned long long ntiles = (P.n + WTILE - 1) / WTILE;
+    const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
+    for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
+         tile += wstride) {
+        // ---- A: 4 consecutive records per lane, keys, run heads, slots ----
+        const unsigned long long tb = tile * WTILE;
+        const unsigned long long r0 = tb + (unsigned long long)lane * RPT;
         uint32_t skx[RPT], nx[RPT], ny[RPT], it[RPT];
-        if (P.aligned && r0 + RPT <= P.n) {
+        if (P.aligned && tb + WTILE <= P.n) {
             const uint4 a = __ldcs((const uint4 *)(P.skx + r0));
             const uint4 b = __ldcs((const uint4 *)(P.nx + r0));
             const uint4 c = __ldcs((const uint4 *)(P.ny + r0));
@@ -613,20 +620,30 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                 it[j] = h ? __ldcs(P.iters + r0 + j) : 0u;
             }
         }
+        // warm L2 with the records of this warp's next tile
+        if (lane < 4) {
+            const unsigned long long nt = tile + wstride;
+            if (nt < ntiles && P.aligned) {
+                const unsigned long long nb = nt * WTILE;
+                const unsigned long long cnt = min((unsigned long long)WTILE, P.n - nb);
+                const uint32_t *base = lane == 0 ? P.skx : lane == 1 ? P.nx : lane == 2 ? P.ny : P.iters;
+                const uint32_t bytes = (uint32_t)(cnt * 4) & ~15u;
+                if (bytes)
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;"
+                                 :: "l"(base + nb), "r"(bytes) : "memory");
+            }
+        }
         unsigned long long key[RPT];
 #pragma unroll
         for (int j = 0; j < RPT; j++) key[j] = key_of(S, skx[j], nx[j], ny[j], it[j], r0 + j < P.n);
-        if (lane == 31) last_key[warp] = key[RPT - 1];
-        __syncthreads();
         unsigned long long prev = __shfl_up_sync(FULL, key[RPT - 1], 1);
-        if (lane == 0) prev = warp ? last_key[warp - 1] : ~0ull;
+        if (lane == 0) prev = ~0ull;
         unsigned head = 0;   // bit j: record j starts a run of a valid key
 #pragma unroll
         for (int j = 0; j < RPT; j++) {
             const unsigned long long pk = j ? key[j - 1] : prev;
             if (key[j] != ~0ull && key[j] != pk) head |= 1u << j;
         }
-        // block exclusive scan of head counts -> slot ids
         const unsigned cnt = __popc(head);
         unsigned inc = cnt;
 #pragma unroll
@@ -634,55 +651,44 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             const unsigned v = __shfl_up_sync(FULL, inc, o);
             if (lane >= o) inc += v;
         }
-        if (lane == 31) wsum[warp] = inc;
-        __syncthreads();
-        unsigned before = 0, nslots = 0;
-#pragma unroll
-        for (int w = 0; w < WARPS; w++) {
-            const unsigned v = wsum[w];
-            before += w < warp ? v : 0u;
-            nslots += v;
-        }
-        const unsigned excl = before + inc - cnt;
+        const unsigned nslots = __shfl_sync(FULL, inc, 31);
         int slot[RPT];
         {
-            unsigned s = excl;
+            unsigned sidx = inc - cnt;
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
-                if ((head >> j) & 1u) s++;
-                slot[j] = key[j] == ~0ull ? -1 : (int)s - 1;
-                rec_skx[threadIdx.x * RPT + j] = skx[j];
-                rec_it[threadIdx.x * RPT + j] = it[j];
-                rec_slot[threadIdx.x * RPT + j] = slot[j];
+                if ((head >> j) & 1u) sidx++;
+                slot[j] = key[j] == ~0ull ? -1 : (int)sidx - 1;
+                ws.rec_skx[lane * RPT + j] = skx[j];
+                ws.rec_it[lane * RPT + j] = it[j];
+                ws.rec_slot[lane * RPT + j] = slot[j];
             }
         }
+        (void)lt;
 
         for (unsigned c0 = 0; c0 < nslots; c0 += SLOT_CAP) {
             const unsigned c1 = min(nslots, c0 + SLOT_CAP);
 #pragma unroll
             for (int j = 0; j < RPT; j++)
                 if (((head >> j) & 1u) && (unsigned)slot[j] >= c0 && (unsigned)slot[j] < c1)
-                    slot_key[slot[j] - c0] = ((unsigned long long)(skx[j] >> 16) << 42) |
-                                             ((unsigned long long)nx[j] << 21) | ny[j];
-            __syncthreads();
+                    ws.slot_key[slot[j] - c0] = key[j];
+            __syncwarp();
             // ---- B: usage of every distinct key of the chunk, once ----
-            for (unsigned g0 = c0 + warp * 8; g0 < c1; g0 += WARPS * 8) {
-                const unsigned gcnt = min(8u, c1 - g0);
+            for (unsigned g0 = c0; g0 < c1; g0 += MAX_SEG) {
+                const unsigned gcnt = min((unsigned)MAX_SEG, c1 - g0);
                 const bool mv = (unsigned)lane < gcnt;
-                const unsigned long long mk = mv ? slot_key[g0 - c0 + lane] : 0ull;
+                const unsigned long long mk = mv ? ws.slot_key[g0 - c0 + lane] : 0ull;
                 bool mplan = false;
-                uint32_t mna = 0, mne = 0;
+                uint32_t mne = 0;
                 if (mv) {
                     const SkelInfo &I = S.skel[(uint32_t)(mk >> 42)];
                     mplan = (long long)((mk >> 21) & 0x1fffffull) >= I.plan_tx &&
                             (long long)(mk & 0x1fffffull) >= I.plan_ty;
-                    mna = I.n_arrays;
                     mne = I.n_expr;
                 }
                 unsigned todo = __ballot_sync(FULL, mv && mplan);
                 unsigned sweep = __ballot_sync(FULL, mv && !mplan);
                 const uint32_t max_ne = __reduce_max_sync(FULL, mplan ? mne : 0u);
-                (void)mna;
                 int L = 32 / MAX_SEG;
                 while ((32 / L) * (int)max_ne > VAL_PER_WARP) L <<= 1;
                 const int G = 32 / L, seg = lane / L, sl = lane % L;
@@ -691,53 +697,47 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     const bool act = pos < 32u;
                     const unsigned long long k = __shfl_sync(FULL, mk, act ? pos : 0);
                     const unsigned ls = g0 - c0 + (act ? pos : 0);
-                    plan_usage(S, act, k, P.pc, scratch[warp].pl.val + seg * (VAL_PER_WARP / G),
-                               scratch[warp].pl.T[seg], sl, L, &res[ls], slot_w[ls]);
+                    plan_usage(S, act, k, P.pc, ws.scratch.pl.val + seg * (VAL_PER_WARP / G),
+                               ws.scratch.pl.T[seg], sl, L, &ws.res[ls], ws.slot_w[ls]);
                     for (int q = 0; q < G && todo; q++) todo &= todo - 1;
                     __syncwarp();
                 }
                 while (sweep) {
                     const int pos = __ffs(sweep) - 1;
                     const unsigned long long k = __shfl_sync(FULL, mk, pos);
-                    const Usage r = warp_usage_sweep(S, S.skel[(uint32_t)(k >> 42)],
-                                                     (long long)((k >> 21) & 0x1fffffull),
-                                                     (long long)(k & 0x1fffffull), P.pc,
-                                                     scratch[warp], lane);
-                    if (lane == 0) res[g0 - c0 + pos] = r;
-                    {
-                        const SkelInfo &I = S.skel[(uint32_t)(k >> 42)];
-                        if ((uint32_t)lane < I.n_kernels)
-                            slot_w[g0 - c0 + pos][lane] = sat_u32(
-                                aff8(__ldg(&S.kern_work[I.k_base + lane]),
-                                     (long long)((k >> 21) & 0x1fffffull), (long long)(k & 0x1fffffull)));
-                    }
+                    const SkelInfo &I = S.skel[(uint32_t)(k >> 42)];
+                    const long long kx_ = (long long)((k >> 21) & 0x1fffffull);
+                    const long long ky_ = (long long)(k & 0x1fffffull);
+                    const Usage r = warp_usage_sweep(S, I, kx_, ky_, P.pc, ws.scratch, lane);
+                    if (lane == 0) ws.res[g0 - c0 + pos] = r;
+                    if ((uint32_t)lane < I.n_kernels)
+                        ws.slot_w[g0 - c0 + pos][lane] =
+                            sat_u32(aff8(__ldg(&S.kern_work[I.k_base + lane]), kx_, ky_));
                     sweep &= sweep - 1;
                     __syncwarp();
                 }
             }
-            __syncthreads();
-            // ---- C: per-candidate model + output / argmin ----
-            // strided mapping: thread t takes records t + 256 j, which share the
-            // transformation when candidates come in groups of 16 (or 256/2^k)
+            __syncwarp();
+            // ---- C: per-candidate model + output / argmin (records lane + 32 j) ----
             bool inj[RPT];
             uint32_t xs[RPT], its[RPT], nxs[RPT], nys[RPT];
             const uint32_t *wp[RPT];
             const Usage *up[RPT];
             double tt[RPT];
-            const uint32_t skx0 = rec_skx[threadIdx.x];
+            const uint32_t skx0 = ws.rec_skx[lane];
             bool same = true;
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
-                const int q = threadIdx.x + THREADS * j;
-                const int sj = rec_slot[q];
-                const uint32_t sk = rec_skx[q];
+                const int q = lane + 32 * j;
+                const int sj = ws.rec_slot[q];
+                const uint32_t sk = ws.rec_skx[q];
                 inj[j] = sj >= (int)c0 && sj < (int)c1;
                 const int ls = inj[j] ? sj - (int)c0 : 0;
                 xs[j] = sk & 0xffffu;
-                its[j] = rec_it[q];
-                wp[j] = slot_w[ls];
-                up[j] = &res[ls];
-                const unsigned long long kk = slot_key[ls];
+                its[j] = ws.rec_it[q];
+                wp[j] = ws.slot_w[ls];
+                up[j] = &ws.res[ls];
+                const unsigned long long kk = ws.slot_key[ls];
                 nxs[j] = (uint32_t)((kk >> 21) & 0x1fffffull);
                 nys[j] = (uint32_t)(kk & 0x1fffffull);
                 same = same && inj[j] && sk == skx0;
@@ -748,13 +748,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
 #pragma unroll
                 for (int j = 0; j < RPT; j++)
                     if (inj[j])
-                        model_n<1, false>(S, rec_skx[threadIdx.x + THREADS * j] >> 16, xs + j,
-                                          its + j, wp + j, nxs + j, nys + j, up + j, tt + j);
+                        model_n<1, false>(S, ws.rec_skx[lane + 32 * j] >> 16, xs + j, its + j,
+                                          wp + j, nxs + j, nys + j, up + j, tt + j);
             }
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
                 if (!inj[j]) continue;
-                const unsigned long long i = tile * TILE + threadIdx.x + THREADS * j;
+                const unsigned long long i = tb + lane + 32 * j;
                 const double t = tt[j];
                 if (!BEST) {
                     __stcs(P.h2d + i, up[j]->h);
@@ -768,7 +768,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     mine.d = up[j]->d;
                 }
             }
-            __syncthreads();
+            __syncwarp();
         }
         // invalid records (no slot) and counters
         unsigned ninv = 0, nval = 0;
@@ -870,7 +870,7 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
                                                       sizeof(CtaSmem));
         if (occ_best < 1) occ_best = 1;
     }
-    const unsigned long long want = (n + TILE - 1) / TILE;
+    const unsigned long long want = (n + (unsigned long long)WTILE * WARPS - 1) / ((unsigned long long)WTILE * WARPS);
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ_best, per_sm_cap);
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
