@@ -35,17 +35,27 @@ constexpr int WARPS = THREADS / 32;
 constexpr int RPT = 4;                       // records per lane
 constexpr int WTILE = 32 * RPT;              // records per warp tile
 constexpr int SLOT_CAP = 16;                 // distinct keys resident per warp chunk
-constexpr int VAL_PER_WARP = 256;            // plan expression values per warp
+#ifndef GROPHECY_VAL
+#define GROPHECY_VAL 256
+#endif
+constexpr int VAL_PER_WARP = GROPHECY_VAL;   // plan expression values per warp pass
 constexpr int MAXK = GROPHECY_MAX_KERNELS;   // kernels per skeleton
 constexpr long long BIG = 0x7fffffffffffffffLL;
 #ifndef GROPHECY_MINB
 #define GROPHECY_MINB 2
 #endif
 
+// c0 + floor((c1 nx + c2 ny + c3 nx ny) / 8); nx, ny <= 2^20 (so the 32x32->64
+// products are exact), nxny = nx * ny precomputed.
+__device__ __forceinline__ long long aff8n(int4 c, int nx, int ny, long long nxny)
+{
+    const long long num = (long long)c.y * nx + (long long)c.z * ny + (long long)c.w * nxny;
+    return (long long)c.x + (num >> 3);   // arithmetic shift: floor(num / 8)
+}
+
 __device__ __forceinline__ long long aff8(int4 c, long long nx, long long ny)
 {
-    long long num = (long long)c.y * nx + (long long)c.z * ny + (long long)c.w * nx * ny;
-    return (long long)c.x + (num >> 3);   // arithmetic shift: floor(num / 8)
+    return aff8n(c, (int)nx, (int)ny, nx * ny);
 }
 
 __device__ __forceinline__ long long clampll(long long v, long long hi)
@@ -131,7 +141,12 @@ __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsig
         nx = (long long)((key >> 21) & 0x1fffffull);
         ny = (long long)(key & 0x1fffffull);
     }
-    for (uint32_t e = sl; e < n_expr; e += L) val[e] = aff8(__ldg(&S.plan_expr[e0 + e]), nx, ny);
+    {
+        const int ix = (int)nx, iy = (int)ny;
+        const long long nxny = (long long)((unsigned long long)(uint32_t)ix * (uint32_t)iy);
+        for (uint32_t e = sl; e < n_expr; e += L)
+            val[e] = aff8n(__ldg(&S.plan_expr[e0 + e]), ix, iy, nxny);
+    }
     __syncwarp();
     unsigned long long hs = 0, ds = 0;
     for (uint32_t a = sl; a < n_arrays; a += L) {
