@@ -487,6 +487,21 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
     r.n_valid = b.nval;
 }
 
+// Per-warp shared memory (dynamic; > 48 KB per CTA needs the opt-in attribute).
+struct WarpSmem {
+    WarpScratch scratch;                        // usage plans / general sweep
+    unsigned long long slot_key[SLOT_CAP];      // distinct keys of the chunk
+    Usage res[SLOT_CAP];                        // their usage
+    uint32_t slot_w[SLOT_CAP][MAXK];            // their work-item counts (saturated)
+    unsigned long long rec_key[WTILE];          // the tile's records after phase A
+    uint32_t rec_skx[WTILE], rec_it[WTILE];
+    int rec_slot[WTILE];
+    unsigned long long best_h[32], best_d[32];  // bytes of each lane's running best
+};
+struct CtaSmem {
+    WarpSmem w[WARPS];
+};
+
 // Model of NJ records of one skeleton at once (NJ independent dependency
 // chains per thread).  W[j] = the work-item counts of record j's key (shared
 // memory, one row per distinct key).  The saturated-grid formula is computed
@@ -494,9 +509,8 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
 // are recomputed by kernel_time.
 template <int NJ, bool SAMEX>
 __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uint32_t *x,
-                                        const uint32_t *it, const uint32_t *const *W,
-                                        const uint32_t *nx, const uint32_t *ny,
-                                        const Usage *const *u, double *t)
+                                        const int *ls, const WarpSmem &ws, double *t_iter,
+                                        double *t_once)
 {
     const SkelInfo &I = S.skel[s];
     const uint32_t K = I.n_kernels, X = I.n_xforms;
@@ -509,24 +523,51 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
         bool gen[NJ];
         KxFast F0;
         if (SAMEX) F0 = S.kx_f[kb + x[0]];   // one constant load shared by the NJ records
+        // staged so that the NJ independent dependency chains interleave
+        KxFast F[NJ];
+        uint32_t w[NJ], blocks[NJ];
+        double bb[NJ], q[NJ], rep[NJ], cyc[NJ];
 #pragma unroll
         for (int j = 0; j < NJ; j++) {
-            const KxFast F = SAMEX ? F0 : S.kx_f[kb + x[j]];
-            const uint32_t w = W[j][k];   // saturated at 2^32 - 1
-            const unsigned long long lo = (unsigned long long)F.magic_lo * w;
-            const uint32_t q = (uint32_t)(((unsigned long long)F.magic_hi * w + (lo >> 32)) >> 32);
-            const uint32_t blocks = q + (q * F.ipb != w);
-            const double rep = div_rn(__uint2double_rn(blocks), F.D, F.rD);
-            const double cyc = __dadd_rn(__dmul_rn(F.E, rep), __dmul_rn(F.S, rep));
-            const double v = div_rn(cyc, S.freq, S.rfreq);
-            const bool inf = isinf(F.E);
-            gen[j] = !inf && blocks != 0 && (w == 0xffffffffu || blocks < F.sat32);
-            tk[j] = inf ? __longlong_as_double(0x7ff0000000000000LL) : (blocks == 0 ? 0.0 : v);
+            F[j] = SAMEX ? F0 : S.kx_f[kb + x[j]];
+            w[j] = ws.slot_w[ls[j]][k];   // saturated at 2^32 - 1
+        }
+#pragma unroll
+        for (int j = 0; j < NJ; j++) {
+            const unsigned long long lo = (unsigned long long)F[j].magic_lo * w[j];
+            const uint32_t qq = (uint32_t)(((unsigned long long)F[j].magic_hi * w[j] + (lo >> 32)) >> 32);
+            blocks[j] = qq + (qq * F[j].ipb != w[j]);
+            bb[j] = __uint2double_rn(blocks[j]);
+        }
+        // rep = blocks / D  (Markstein, bitwise the IEEE quotient)
+#pragma unroll
+        for (int j = 0; j < NJ; j++) q[j] = __dmul_rn(bb[j], F[j].rD);
+#pragma unroll
+        for (int j = 0; j < NJ; j++) rep[j] = __fma_rn(-q[j], F[j].D, bb[j]);
+#pragma unroll
+        for (int j = 0; j < NJ; j++) rep[j] = __fma_rn(rep[j], F[j].rD, q[j]);
+        // cycles = E rep + S rep
+#pragma unroll
+        for (int j = 0; j < NJ; j++) cyc[j] = __dadd_rn(__dmul_rn(F[j].E, rep[j]), __dmul_rn(F[j].S, rep[j]));
+        // t = cycles / freq  (Markstein)
+#pragma unroll
+        for (int j = 0; j < NJ; j++) q[j] = __dmul_rn(cyc[j], S.rfreq);
+#pragma unroll
+        for (int j = 0; j < NJ; j++) rep[j] = __fma_rn(-q[j], S.freq, cyc[j]);
+#pragma unroll
+        for (int j = 0; j < NJ; j++) {
+            const double v = __fma_rn(rep[j], S.rfreq, q[j]);
+            const bool inf = isinf(F[j].E);
+            gen[j] = !inf && blocks[j] != 0 && (w[j] == 0xffffffffu || blocks[j] < F[j].sat32);
+            tk[j] = inf ? __longlong_as_double(0x7ff0000000000000LL) : (blocks[j] == 0 ? 0.0 : v);
         }
 #pragma unroll
         for (int j = 0; j < NJ; j++)
             if (gen[j]) {
-                const long long Wi = aff8(__ldg(&S.kern_work[I.k_base + k]), nx[j], ny[j]);
+                const unsigned long long kk = ws.slot_key[ls[j]];
+                const long long Wi = aff8(__ldg(&S.kern_work[I.k_base + k]),
+                                          (long long)((kk >> 21) & 0x1fffffull),
+                                          (long long)(kk & 0x1fffffull));
                 tk[j] = kernel_time(S, Wi, S.kx_j[kb + x[j]], kb + x[j]);
             }
         if (__ldg(&S.kern_flags[I.k_base + k]) & GROPHECY_KERNEL_PER_ITER) {
@@ -539,8 +580,8 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
     }
 #pragma unroll
     for (int j = 0; j < NJ; j++) {
-        const double t_kern = __dadd_rn(to[j], __dmul_rn((double)it[j], ti[j]));
-        t[j] = __dadd_rn(__dadd_rn(t_kern, u[j]->th), u[j]->td);
+        t_iter[j] = ti[j];
+        t_once[j] = to[j];
     }
 }
 
@@ -574,19 +615,6 @@ __device__ __forceinline__ unsigned long long key_of(const SpaceDev &S, uint32_t
     return valid ? ((unsigned long long)skel << 42) | ((unsigned long long)nx << 21) | ny : ~0ull;
 }
 
-// Per-warp shared memory (dynamic; > 48 KB per CTA needs the opt-in attribute).
-struct WarpSmem {
-    WarpScratch scratch;                        // usage plans / general sweep
-    unsigned long long slot_key[SLOT_CAP];      // distinct keys of the chunk
-    Usage res[SLOT_CAP];                        // their usage
-    uint32_t slot_w[SLOT_CAP][MAXK];            // their work-item counts (saturated)
-    uint32_t rec_skx[WTILE], rec_it[WTILE];     // the tile's records, for the strided model
-    int rec_slot[WTILE];
-};
-struct CtaSmem {
-    WarpSmem w[WARPS];
-};
-
 // Persistent kernel; every warp works alone on tiles of 128 consecutive
 // records (no CTA barriers on the hot loop):
 //   A  lane l loads records 4l..4l+3 (one 16-byte load per SoA array), checks
@@ -607,7 +635,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
     const SpaceDev &S = P.S;
     const unsigned lt = (1u << lane) - 1u;
 
-    Best mine = none_best();
+    // running argmin kept lean in registers: (t, index) + counters; the
+    // winner's byte counts go to shared memory (rarely updated)
+    double best_t = __longlong_as_double(0x7ff0000000000000LL);
+    unsigned long long best_i = ~0ull;
+    uint32_t cnt_inv = 0, cnt_val = 0;
+    ws.best_h[lane] = 0;
+    ws.best_d[lane] = 0;
     const unsigned long long ntiles = (P.n + WTILE - 1) / WTILE;
     const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
     for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
@@ -676,17 +710,24 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                 slot[j] = key[j] == ~0ull ? -1 : (int)sidx - 1;
                 ws.rec_skx[lane * RPT + j] = skx[j];
                 ws.rec_it[lane * RPT + j] = it[j];
-                ws.rec_slot[lane * RPT + j] = slot[j];
+                ws.rec_slot[lane * RPT + j] = ((head >> j) & 1u) ? -2 - slot[j] : slot[j];
+                ws.rec_key[lane * RPT + j] = key[j];
             }
         }
         (void)lt;
+        __syncwarp();
+        // from here on the tile lives in shared memory (keeps registers free
+        // for the model's independent dependency chains)
 
         for (unsigned c0 = 0; c0 < nslots; c0 += SLOT_CAP) {
             const unsigned c1 = min(nslots, c0 + SLOT_CAP);
 #pragma unroll
-            for (int j = 0; j < RPT; j++)
-                if (((head >> j) & 1u) && (unsigned)slot[j] >= c0 && (unsigned)slot[j] < c1)
-                    ws.slot_key[slot[j] - c0] = key[j];
+            for (int j = 0; j < RPT; j++) {
+                const int q = lane * RPT + j;
+                const int hs = ws.rec_slot[q];   // heads are encoded as -2 - slot
+                if (hs <= -2 && (unsigned)(-2 - hs) >= c0 && (unsigned)(-2 - hs) < c1)
+                    ws.slot_key[-2 - hs - c0] = ws.rec_key[q];
+            }
             __syncwarp();
             // ---- B: usage of every distinct key of the chunk, once ----
             for (unsigned g0 = c0; g0 < c1; g0 += MAX_SEG) {
@@ -734,53 +775,50 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             }
             __syncwarp();
             // ---- C: per-candidate model + output / argmin (records lane + 32 j) ----
+            int ls[RPT];
+            uint32_t xs[RPT];
             bool inj[RPT];
-            uint32_t xs[RPT], its[RPT], nxs[RPT], nys[RPT];
-            const uint32_t *wp[RPT];
-            const Usage *up[RPT];
-            double tt[RPT];
+            double ti[RPT], to[RPT];
             const uint32_t skx0 = ws.rec_skx[lane];
             bool same = true;
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
                 const int q = lane + 32 * j;
-                const int sj = ws.rec_slot[q];
+                int sj = ws.rec_slot[q];
+                if (sj <= -2) sj = -2 - sj;
                 const uint32_t sk = ws.rec_skx[q];
                 inj[j] = sj >= (int)c0 && sj < (int)c1;
-                const int ls = inj[j] ? sj - (int)c0 : 0;
+                ls[j] = inj[j] ? sj - (int)c0 : 0;
                 xs[j] = sk & 0xffffu;
-                its[j] = ws.rec_it[q];
-                wp[j] = ws.slot_w[ls];
-                up[j] = &ws.res[ls];
-                const unsigned long long kk = ws.slot_key[ls];
-                nxs[j] = (uint32_t)((kk >> 21) & 0x1fffffull);
-                nys[j] = (uint32_t)(kk & 0x1fffffull);
                 same = same && inj[j] && sk == skx0;
             }
             if (same) {
-                model_n<RPT, true>(S, skx0 >> 16, xs, its, wp, nxs, nys, up, tt);
+                model_n<RPT, true>(S, skx0 >> 16, xs, ls, ws, ti, to);
             } else {
 #pragma unroll
                 for (int j = 0; j < RPT; j++)
                     if (inj[j])
-                        model_n<1, false>(S, ws.rec_skx[lane + 32 * j] >> 16, xs + j, its + j,
-                                          wp + j, nxs + j, nys + j, up + j, tt + j);
+                        model_n<1, false>(S, ws.rec_skx[lane + 32 * j] >> 16, xs + j, ls + j, ws,
+                                          ti + j, to + j);
             }
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
                 if (!inj[j]) continue;
                 const unsigned long long i = tb + lane + 32 * j;
-                const double t = tt[j];
+                const Usage &u = ws.res[ls[j]];
+                // total: run-once + iters x per-iteration + transfers
+                const double t_kern = __dadd_rn(to[j], __dmul_rn((double)ws.rec_it[lane + 32 * j], ti[j]));
+                const double t = __dadd_rn(__dadd_rn(t_kern, u.th), u.td);
                 if (!BEST) {
-                    __stcs(P.h2d + i, up[j]->h);
-                    __stcs(P.d2h + i, up[j]->d);
+                    __stcs(P.h2d + i, u.h);
+                    __stcs(P.d2h + i, u.d);
                     __stcs(P.t + i, t);
                 } else if (t < __longlong_as_double(0x7ff0000000000000LL) &&
-                           better(t, P.base + i, mine.t, mine.i)) {
-                    mine.t = t;
-                    mine.i = P.base + i;
-                    mine.h = up[j]->h;
-                    mine.d = up[j]->d;
+                           better(t, P.base + i, best_t, best_i)) {
+                    best_t = t;
+                    best_i = P.base + i;
+                    ws.best_h[lane] = u.h;
+                    ws.best_d[lane] = u.d;
                 }
             }
             __syncwarp();
@@ -789,9 +827,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
         unsigned ninv = 0, nval = 0;
 #pragma unroll
         for (int j = 0; j < RPT; j++) {
-            const unsigned long long i = r0 + j;
+            const unsigned long long i = tb + lane * RPT + j;
             if (i >= P.n) continue;
-            if (slot[j] < 0) {
+            if (ws.rec_slot[lane * RPT + j] == -1) {
                 ninv++;
                 if (!BEST) {
                     __stcs(P.h2d + i, 0ull);
@@ -803,8 +841,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             }
         }
         if (BEST) {
-            mine.ninv += ninv;
-            mine.nval += nval;
+            cnt_inv += ninv;
+            cnt_val += nval;
         } else {
             const unsigned tot = __reduce_add_sync(FULL, ninv);
             if (lane == 0 && tot) atomicAdd(S.invalid_counter, (unsigned long long)tot);
@@ -813,6 +851,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
     if (!BEST) return;
 
     // ---- argmin: warp -> CTA -> grid (last-block pattern) ----
+    Best mine;
+    mine.t = best_t;
+    mine.i = best_i;
+    mine.h = ws.best_h[lane];
+    mine.d = ws.best_d[lane];
+    mine.ninv = cnt_inv;
+    mine.nval = cnt_val;
     mine = warp_best(mine);
     if (lane == 0) wbest[warp] = mine;
     __syncthreads();
