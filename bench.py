@@ -303,7 +303,9 @@ def main():
         props = torch.cuda.get_device_properties(local_rank)
         peak_issue = props.multi_processor_count * 4 * sm_mhz * 1e6
         ach = prof["warp_inst_per_launch"] / prof_n * n_local / (kern_avg_max * 1e-3)
-        roof_issue = {"bound": "alu", "achieved": ach, "peak": peak_issue,
+        if ach > 1.02 * peak_issue:   # committed capture is stale for this build
+            ach = None
+        roof_issue = None if ach is None else {"bound": "alu", "achieved": ach, "peak": peak_issue,
                       "unit": "warp-inst/s", "frac": ach / peak_issue,
                       "warp_inst_per_candidate": prof["warp_inst_per_launch"] / prof_n,
                       "note": "executed (not algorithmic) warp instructions from "
