@@ -46,6 +46,8 @@ struct SkelInfo {
     uint32_t pad;
     // usage plan (plan.cpp): valid for nx >= plan_tx and ny >= plan_ty
     uint32_t plan_tx, plan_ty, expr_base, n_expr;
+    // flat term list of all arrays / directions: {packed indices, 2*array + dir}
+    uint32_t term_base, n_terms, pad1, pad2;
 };
 
 struct ArrayDev {
@@ -87,6 +89,7 @@ struct SpaceDev {
     const KxFast *kx_f;
     const int4 *plan_expr;
     const uint32_t *plan_prog;
+    const uint2 *plan_terms;
     uint32_t n_skels;
     uint32_t n_sm;
     double freq, rfreq;

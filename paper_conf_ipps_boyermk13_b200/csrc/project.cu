@@ -132,38 +132,48 @@ __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsig
                                            const grophecy_pcie &pc, long long *val, double *T,
                                            int sl, int L, Usage *res, uint32_t *w_out)
 {
-    uint32_t n_expr = 0, n_arrays = 0, e0 = 0, a0 = 0, K = 0;
+    uint32_t n_expr = 0, n_arrays = 0, e0 = 0, a0 = 0, K = 0, tb = 0, nt = 0;
     long long nx = 0, ny = 0;
     if (active) {
         const SkelInfo &I = S.skel[(uint32_t)(key >> 42)];
         n_expr = I.n_expr; n_arrays = I.n_arrays; e0 = I.expr_base; a0 = I.a_base;
-        K = I.n_kernels;
+        K = I.n_kernels; tb = I.term_base; nt = I.n_terms;
         nx = (long long)((key >> 21) & 0x1fffffull);
         ny = (long long)(key & 0x1fffffull);
     }
+    unsigned long long *cnt = reinterpret_cast<unsigned long long *>(T);   // counts, then times
     {
         const int ix = (int)nx, iy = (int)ny;
         const long long nxny = (long long)((unsigned long long)(uint32_t)ix * (uint32_t)iy);
         for (uint32_t e = sl; e < n_expr; e += L)
             val[e] = aff8n(__ldg(&S.plan_expr[e0 + e]), ix, iy, nxny);
+        for (uint32_t i = sl; i < 2 * n_arrays; i += L) cnt[i] = 0ull;
+    }
+    __syncwarp();
+    // lanes over the skeleton's flat term list: count[2a + dir] += (row extent) x (column run)
+    for (uint32_t t = sl; t < nt; t += L) {
+        const uint2 tw = __ldg(&S.plan_terms[tb + t]);   // rs | re << 8 | cs << 16 | ce << 24
+        const unsigned long long prod =
+            (unsigned long long)((val[(tw.x >> 8) & 0xffu] - val[tw.x & 0xffu]) *
+                                 (val[tw.x >> 24] - val[(tw.x >> 16) & 0xffu]));
+        // exact 64-bit accumulate from native 32-bit shared atomics: the carry
+        // out of the low word is taken at each add
+        unsigned *c32 = reinterpret_cast<unsigned *>(&cnt[tw.y]);
+        const unsigned lo = (unsigned)prod;
+        unsigned hi = (unsigned)(prod >> 32);
+        const unsigned old = atomicAdd(c32, lo);
+        hi += (old + lo) < old;
+        if (hi) atomicAdd(c32 + 1, hi);
     }
     __syncwarp();
     unsigned long long hs = 0, ds = 0;
     for (uint32_t a = sl; a < n_arrays; a += L) {
         const ArrayDev &A = S.arrays[a0 + a];
-        const uint32_t eb = A.elem_bytes;
+        const unsigned long long eb = A.elem_bytes;
 #pragma unroll
         for (int dir = 0; dir < 2; dir++) {
-            const uint32_t *p = S.plan_prog + (dir ? A.d_prog : A.h_prog);
-            const uint32_t nt = __ldg(p++);
-            unsigned long long cnt = 0;
-#pragma unroll 1
-            for (uint32_t t = 0; t < nt; t++) {
-                const uint32_t w = __ldg(p + t);   // rs | re << 8 | cs << 16 | ce << 24
-                cnt += (unsigned long long)((val[(w >> 8) & 0xffu] - val[w & 0xffu]) *
-                                            (val[w >> 24] - val[(w >> 16) & 0xffu]));
-            }
-            const unsigned long long bytes = (dir && !A.liveout) ? 0ull : cnt * eb;
+            const unsigned long long c = cnt[2 * a + dir];
+            const unsigned long long bytes = (dir && !A.liveout) ? 0ull : c * eb;
             const grophecy_link lk = dir ? pc.d2h : pc.h2d;
             T[2 * a + dir] = bytes ? __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte,
                                                                     __ull2double_rn(bytes)))

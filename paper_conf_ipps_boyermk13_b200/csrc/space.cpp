@@ -249,10 +249,12 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxFast> kf;
     std::vector<int4> pexpr;
     std::vector<uint32_t> pprog;
+    std::vector<uint2> pterms;
     auto a4 = [](const grophecy_affine8 &a) { return make_int4(a.c0, a.c1, a.c2, a.c3); };
     for (uint32_t s = 0; s < n_skels; s++) {
         const grophecy_skeleton_desc &S = skels[s];
         SkelInfo &I = info[s];
+        std::memset(&I, 0, sizeof I);
         I.n_kernels = S.n_kernels;
         I.n_arrays = S.n_arrays;
         I.n_xforms = S.n_xforms;
@@ -274,6 +276,16 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         }
         const uint32_t prog_base = (uint32_t)pprog.size();
         if (plan.ok) pprog.insert(pprog.end(), plan.prog.begin(), plan.prog.end());
+        I.term_base = (uint32_t)pterms.size();
+        I.n_terms = 0;
+        I.pad1 = I.pad2 = 0;
+        if (plan.ok)
+            for (uint32_t a = 0; a < S.n_arrays; a++)
+                for (uint32_t dir = 0; dir < 2; dir++) {
+                    const uint32_t *p = plan.prog.data() + (dir ? plan.d_off[a] : plan.h_off[a]);
+                    for (uint32_t t = 0; t < p[0]; t++) pterms.push_back(make_uint2(p[1 + t], 2 * a + dir));
+                }
+        I.n_terms = (uint32_t)pterms.size() - I.term_base;
         for (uint32_t k = 0; k < S.n_kernels; k++) {
             kwork.push_back(a4(S.kernels[k].work_items));
             kflags.push_back(S.kernels[k].flags);
@@ -351,6 +363,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {pexpr.data(), pexpr.size() * sizeof(int4), 0},
         {pprog.data(), pprog.size() * sizeof(uint32_t), 0},
         {kf.data(), kf.size() * sizeof(KxFast), 0},
+        {pterms.data(), pterms.size() * sizeof(uint2), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -407,6 +420,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.plan_expr = (const int4 *)(base + parts[10].off);
     D.plan_prog = (const uint32_t *)(base + parts[11].off);
     D.kx_f = (const KxFast *)(base + parts[12].off);
+    D.plan_terms = (const uint2 *)(base + parts[13].off);
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;
     D.freq = gpu->freq_hz;
