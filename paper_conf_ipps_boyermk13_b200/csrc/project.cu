@@ -615,13 +615,14 @@ struct Params {
     int aligned;    // record arrays 16-byte aligned -> vector loads
 };
 
+// Record validity (include/grophecy.h) and its usage key (skeleton, nx, ny).
+// n_xf = the skeleton's n_xforms (looked up by the caller).
 __device__ __forceinline__ unsigned long long key_of(const SpaceDev &S, uint32_t skx, uint32_t nx,
-                                                     uint32_t ny, uint32_t it, bool has)
+                                                     uint32_t ny, uint32_t it, bool has, uint32_t n_xf)
 {
     const uint32_t skel = skx >> 16, x = skx & 0xffffu;
-    bool valid = has && skel < S.n_skels && nx >= 1 && nx <= GROPHECY_MAX_DIM && ny >= 1 &&
-                 ny <= GROPHECY_MAX_DIM && it >= 1;
-    if (valid) valid = x < S.skel[skel].n_xforms;
+    const bool valid = has && skel < S.n_skels && nx - 1u < GROPHECY_MAX_DIM &&
+                       ny - 1u < GROPHECY_MAX_DIM && it >= 1 && x < n_xf;
     return valid ? ((unsigned long long)skel << 42) | ((unsigned long long)nx << 21) | ny : ~0ull;
 }
 
@@ -694,7 +695,19 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
         }
         unsigned long long key[RPT];
 #pragma unroll
-        for (int j = 0; j < RPT; j++) key[j] = key_of(S, skx[j], nx[j], ny[j], it[j], r0 + j < P.n);
+        {
+            // one n_xforms lookup per distinct skeleton among the lane's records
+            uint32_t nxf = 0, last = 0xffffffffu;
+#pragma unroll
+            for (int j = 0; j < RPT; j++) {
+                const uint32_t sj = skx[j] >> 16;
+                if (sj != last && sj < S.n_skels) {
+                    nxf = S.skel[sj].n_xforms;
+                    last = sj;
+                }
+                key[j] = key_of(S, skx[j], nx[j], ny[j], it[j], r0 + j < P.n, sj == last ? nxf : 0u);
+            }
+        }
         unsigned long long prev = __shfl_up_sync(FULL, key[RPT - 1], 1);
         if (lane == 0) prev = ~0ull;
         unsigned head = 0;   // bit j: record j starts a run of a valid key
@@ -704,6 +717,14 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             if (key[j] != ~0ull && key[j] != pk) head |= 1u << j;
         }
         const unsigned cnt = __popc(head);
+        unsigned n_invalid = 0, n_valid = 0;
+#pragma unroll
+        for (int j = 0; j < RPT; j++) {
+            if (r0 + j < P.n) {
+                if (key[j] == ~0ull) n_invalid++;
+                else n_valid++;
+            }
+        }
         unsigned inc = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -755,8 +776,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                 unsigned todo = __ballot_sync(FULL, mv && mplan);
                 unsigned sweep = __ballot_sync(FULL, mv && !mplan);
                 const uint32_t max_ne = __reduce_max_sync(FULL, mplan ? mne : 0u);
-                int L = 32 / MAX_SEG;
-                while ((32 / L) * (int)max_ne > VAL_PER_WARP) L <<= 1;
+                // lanes per key: 4 (8 keys per pass) unless the values do not fit
+                const int L = max_ne * MAX_SEG <= VAL_PER_WARP ? 32 / MAX_SEG
+                            : max_ne * 4 <= VAL_PER_WARP ? 8
+                            : max_ne * 2 <= VAL_PER_WARP ? 16 : 32;
                 const int G = 32 / L, seg = lane / L, sl = lane % L;
                 while (todo) {
                     const unsigned pos = __fns(todo, 0, seg + 1);
@@ -765,7 +788,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     const unsigned ls = g0 - c0 + (act ? pos : 0);
                     plan_usage(S, act, k, P.pc, ws.scratch.pl.val + seg * (VAL_PER_WARP / G),
                                ws.scratch.pl.T[seg], sl, L, &ws.res[ls], ws.slot_w[ls]);
-                    for (int q = 0; q < G && todo; q++) todo &= todo - 1;
+                    {   // drop the G keys just processed (the lowest G set bits)
+                        const unsigned nxt = __fns(todo, 0, G + 1);
+                        todo = nxt < 32u ? todo & ~((1u << nxt) - 1u) : 0u;
+                    }
                     __syncwarp();
                 }
                 while (sweep) {
@@ -833,28 +859,23 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             }
             __syncwarp();
         }
-        // invalid records (no slot) and counters
-        unsigned ninv = 0, nval = 0;
-#pragma unroll
-        for (int j = 0; j < RPT; j++) {
-            const unsigned long long i = tb + lane * RPT + j;
-            if (i >= P.n) continue;
-            if (ws.rec_slot[lane * RPT + j] == -1) {
-                ninv++;
-                if (!BEST) {
-                    __stcs(P.h2d + i, 0ull);
-                    __stcs(P.d2h + i, 0ull);
-                    __stcs(P.t + i, __longlong_as_double(0x7ff8000000000000LL));
-                }
-            } else {
-                nval++;
-            }
-        }
+        // invalid records: (0, 0, NaN) outputs and counters
         if (BEST) {
-            cnt_inv += ninv;
-            cnt_val += nval;
+            cnt_inv += n_invalid;
+            cnt_val += n_valid;
         } else {
-            const unsigned tot = __reduce_add_sync(FULL, ninv);
+            if (n_invalid) {
+#pragma unroll
+                for (int j = 0; j < RPT; j++) {
+                    const unsigned long long i = tb + lane * RPT + j;
+                    if (i < P.n && ws.rec_slot[lane * RPT + j] == -1) {
+                        __stcs(P.h2d + i, 0ull);
+                        __stcs(P.d2h + i, 0ull);
+                        __stcs(P.t + i, __longlong_as_double(0x7ff8000000000000LL));
+                    }
+                }
+            }
+            const unsigned tot = __reduce_add_sync(FULL, n_invalid);
             if (lane == 0 && tot) atomicAdd(S.invalid_counter, (unsigned long long)tot);
         }
     }
