@@ -43,6 +43,8 @@ def build(force=False, verbose=False):
            "-I", INCLUDE, "-I", CSRC, "-o", LIB]
     if verbose:
         cmd += ["-Xptxas", "-v"]
+    if os.environ.get("GROPHECY_THREADS"):
+        cmd += [f"-DGROPHECY_THREADS={int(os.environ['GROPHECY_THREADS'])}"]
     if os.environ.get("GROPHECY_VAL"):
         cmd += [f"-DGROPHECY_VAL={int(os.environ['GROPHECY_VAL'])}"]
     if os.environ.get("GROPHECY_MINB"):

@@ -30,7 +30,10 @@
 namespace grophecy {
 
 constexpr unsigned FULL = 0xffffffffu;
-constexpr int THREADS = 256;
+#ifndef GROPHECY_THREADS
+#define GROPHECY_THREADS 256
+#endif
+constexpr int THREADS = GROPHECY_THREADS;
 constexpr int WARPS = THREADS / 32;
 constexpr int RPT = 4;                       // records per lane
 constexpr int WTILE = 32 * RPT;              // records per warp tile
@@ -85,8 +88,8 @@ struct SweepScratch {
 constexpr int MAX_SEG = 8;                   // keys per warp pass (plan path)
 
 struct PlanScratch {
-    long long val[VAL_PER_WARP];                 // expression values of the pass's keys
-    double T[MAX_SEG][2 * GROPHECY_MAX_ARRAYS];  // per-array transfer times
+    long long val[VAL_PER_WARP + 32];                // expression values of the pass's keys
+    double T[MAX_SEG][2 * GROPHECY_MAX_ARRAYS + 4];  // per-array counts, then transfer times
 };
 
 union WarpScratch {
@@ -502,7 +505,7 @@ struct WarpSmem {
     WarpScratch scratch;                        // usage plans / general sweep
     unsigned long long slot_key[SLOT_CAP];      // distinct keys of the chunk
     Usage res[SLOT_CAP];                        // their usage
-    uint32_t slot_w[SLOT_CAP][MAXK];            // their work-item counts (saturated)
+    uint32_t slot_w[SLOT_CAP][MAXK + 1];        // their work-item counts (saturated; padded row)
     unsigned long long rec_key[WTILE];          // the tile's records after phase A
     uint32_t rec_skx[WTILE], rec_it[WTILE];
     int rec_slot[WTILE];
@@ -657,28 +660,18 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
     const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
     for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
          tile += wstride) {
-        // ---- A: 4 consecutive records per lane, keys, run heads, slots ----
+        // ---- A: records q = lane + 32 j (coalesced 32-bit loads), keys, run
+        //      heads (ballots) and slot ids in record order ----
         const unsigned long long tb = tile * WTILE;
-        const unsigned long long r0 = tb + (unsigned long long)lane * RPT;
         uint32_t skx[RPT], nx[RPT], ny[RPT], it[RPT];
-        if (P.aligned && tb + WTILE <= P.n) {
-            const uint4 a = __ldcs((const uint4 *)(P.skx + r0));
-            const uint4 b = __ldcs((const uint4 *)(P.nx + r0));
-            const uint4 c = __ldcs((const uint4 *)(P.ny + r0));
-            const uint4 d = __ldcs((const uint4 *)(P.iters + r0));
-            skx[0] = a.x; skx[1] = a.y; skx[2] = a.z; skx[3] = a.w;
-            nx[0] = b.x; nx[1] = b.y; nx[2] = b.z; nx[3] = b.w;
-            ny[0] = c.x; ny[1] = c.y; ny[2] = c.z; ny[3] = c.w;
-            it[0] = d.x; it[1] = d.y; it[2] = d.z; it[3] = d.w;
-        } else {
 #pragma unroll
-            for (int j = 0; j < RPT; j++) {
-                const bool h = r0 + j < P.n;
-                skx[j] = h ? __ldcs(P.skx + r0 + j) : 0u;
-                nx[j] = h ? __ldcs(P.nx + r0 + j) : 0u;
-                ny[j] = h ? __ldcs(P.ny + r0 + j) : 0u;
-                it[j] = h ? __ldcs(P.iters + r0 + j) : 0u;
-            }
+        for (int j = 0; j < RPT; j++) {
+            const unsigned long long i = tb + lane + 32 * j;
+            const bool h = i < P.n;
+            skx[j] = h ? __ldcs(P.skx + i) : 0u;
+            nx[j] = h ? __ldcs(P.nx + i) : 0u;
+            ny[j] = h ? __ldcs(P.ny + i) : 0u;
+            it[j] = h ? __ldcs(P.iters + i) : 0u;
         }
         // warm L2 with the records of this warp's next tile
         if (lane < 4) {
@@ -694,7 +687,6 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             }
         }
         unsigned long long key[RPT];
-#pragma unroll
         {
             // one n_xforms lookup per distinct skeleton among the lane's records
             uint32_t nxf = 0, last = 0xffffffffu;
@@ -705,44 +697,31 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     nxf = S.skel[sj].n_xforms;
                     last = sj;
                 }
-                key[j] = key_of(S, skx[j], nx[j], ny[j], it[j], r0 + j < P.n, sj == last ? nxf : 0u);
+                key[j] = key_of(S, skx[j], nx[j], ny[j], it[j], tb + lane + 32 * j < P.n,
+                                sj == last ? nxf : 0u);
             }
         }
-        unsigned long long prev = __shfl_up_sync(FULL, key[RPT - 1], 1);
-        if (lane == 0) prev = ~0ull;
-        unsigned head = 0;   // bit j: record j starts a run of a valid key
-#pragma unroll
-        for (int j = 0; j < RPT; j++) {
-            const unsigned long long pk = j ? key[j - 1] : prev;
-            if (key[j] != ~0ull && key[j] != pk) head |= 1u << j;
-        }
-        const unsigned cnt = __popc(head);
         unsigned n_invalid = 0, n_valid = 0;
+        unsigned nslots = 0;
+        const unsigned le = (2u << lane) - 1u;   // lanes <= this one
 #pragma unroll
         for (int j = 0; j < RPT; j++) {
-            if (r0 + j < P.n) {
+            // predecessor of record lane + 32 j is lane - 1 (same j) or lane 31 of j - 1
+            unsigned long long prev = __shfl_up_sync(FULL, key[j], 1);
+            const unsigned long long last_prev = j ? __shfl_sync(FULL, key[j > 0 ? j - 1 : 0], 31) : ~0ull;
+            if (lane == 0) prev = last_prev;
+            const bool head = key[j] != ~0ull && key[j] != prev;
+            const unsigned hb = __ballot_sync(FULL, head);
+            const int slot = key[j] == ~0ull ? -1 : (int)(nslots + __popc(hb & le)) - 1;
+            nslots += __popc(hb);
+            const int q = lane + 32 * j;
+            ws.rec_skx[q] = skx[j];
+            ws.rec_it[q] = it[j];
+            ws.rec_slot[q] = head ? -2 - slot : slot;   // heads encoded as -2 - slot
+            ws.rec_key[q] = key[j];
+            if (tb + q < P.n) {
                 if (key[j] == ~0ull) n_invalid++;
                 else n_valid++;
-            }
-        }
-        unsigned inc = cnt;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const unsigned v = __shfl_up_sync(FULL, inc, o);
-            if (lane >= o) inc += v;
-        }
-        const unsigned nslots = __shfl_sync(FULL, inc, 31);
-        int slot[RPT];
-        {
-            unsigned sidx = inc - cnt;
-#pragma unroll
-            for (int j = 0; j < RPT; j++) {
-                if ((head >> j) & 1u) sidx++;
-                slot[j] = key[j] == ~0ull ? -1 : (int)sidx - 1;
-                ws.rec_skx[lane * RPT + j] = skx[j];
-                ws.rec_it[lane * RPT + j] = it[j];
-                ws.rec_slot[lane * RPT + j] = ((head >> j) & 1u) ? -2 - slot[j] : slot[j];
-                ws.rec_key[lane * RPT + j] = key[j];
             }
         }
         (void)lt;
@@ -754,7 +733,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             const unsigned c1 = min(nslots, c0 + SLOT_CAP);
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
-                const int q = lane * RPT + j;
+                const int q = lane + 32 * j;
                 const int hs = ws.rec_slot[q];   // heads are encoded as -2 - slot
                 if (hs <= -2 && (unsigned)(-2 - hs) >= c0 && (unsigned)(-2 - hs) < c1)
                     ws.slot_key[-2 - hs - c0] = ws.rec_key[q];
@@ -786,7 +765,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     const bool act = pos < 32u;
                     const unsigned long long k = __shfl_sync(FULL, mk, act ? pos : 0);
                     const unsigned ls = g0 - c0 + (act ? pos : 0);
-                    plan_usage(S, act, k, P.pc, ws.scratch.pl.val + seg * (VAL_PER_WARP / G),
+                    // segment stride VAL/G + L longs: the segments' lanes hit distinct banks
+                    plan_usage(S, act, k, P.pc, ws.scratch.pl.val + seg * (VAL_PER_WARP / G + L),
                                ws.scratch.pl.T[seg], sl, L, &ws.res[ls], ws.slot_w[ls]);
                     {   // drop the G keys just processed (the lowest G set bits)
                         const unsigned nxt = __fns(todo, 0, G + 1);
@@ -867,8 +847,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             if (n_invalid) {
 #pragma unroll
                 for (int j = 0; j < RPT; j++) {
-                    const unsigned long long i = tb + lane * RPT + j;
-                    if (i < P.n && ws.rec_slot[lane * RPT + j] == -1) {
+                    const unsigned long long i = tb + lane + 32 * j;
+                    if (i < P.n && ws.rec_slot[lane + 32 * j] == -1) {
                         __stcs(P.h2d + i, 0ull);
                         __stcs(P.d2h + i, 0ull);
                         __stcs(P.t + i, __longlong_as_double(0x7ff8000000000000LL));
