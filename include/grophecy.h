@@ -176,6 +176,21 @@ int grophecy_eval(const grophecy_space *space, const grophecy_pcie *pcie,
                   const grophecy_batch *batch, uint64_t *h2d_bytes, uint64_t *d2h_bytes,
                   double *t_total_s, void *cuda_stream);
 
+/* Components of each projected time (DEVICE arrays of length n, each may be
+ * NULL): t_iter_s = sum of per-iteration kernel times, t_once_s = sum of
+ * run-once kernel times, t_h2d_s / t_d2h_s = summed per-array transfer times,
+ * so that  t_total_s = ((t_once + iters * t_iter) + t_h2d) + t_d2h  exactly
+ * (P:L77, L147, L167).  "Kernel only" = t_once + iters * t_iter and
+ * "transfer only" = t_h2d + t_d2h are the paper's Table II predictors
+ * (P:L251); iteration sweeps follow in closed form (Figs. 8/10/12).
+ * Invalid records get NaN in every component. */
+typedef struct { double *t_iter_s, *t_once_s, *t_h2d_s, *t_d2h_s; } grophecy_parts;
+
+/* grophecy_eval plus the time components of every candidate.  Async. */
+int grophecy_eval_parts(const grophecy_space *space, const grophecy_pcie *pcie,
+                        const grophecy_batch *batch, uint64_t *h2d_bytes, uint64_t *d2h_bytes,
+                        double *t_total_s, const grophecy_parts *parts, void *cuda_stream);
+
 /* Synchronise the stream, return the number of invalid records seen by
  * grophecy_eval on this space since the last call, and reset the counter. */
 int grophecy_invalid_count(grophecy_space *space, uint64_t *count, void *cuda_stream);
@@ -211,6 +226,30 @@ int grophecy_best_combine(const grophecy_best_result *device_in, uint32_t count,
 /* The same combine on the host (pure C, no CUDA). */
 int grophecy_best_combine_host(const grophecy_best_result *in, uint32_t count,
                                grophecy_best_result *out);
+
+/* Best transformation per projection point (the predicted kernel time
+ * "is the predicted time of the best-performing version").  A group is a
+ * maximal run of consecutive records with equal (skeleton, nx, ny, iters);
+ * per group: first global index, size, and the argmin (t, index) over valid
+ * records with finite time (ties to the lowest index; best_index UINT64_MAX
+ * and best_t_s +inf when none) with that candidate's bytes.  48 bytes. */
+typedef struct {
+    double best_t_s;
+    uint64_t first, count, best_index, h2d_bytes, d2h_bytes;
+} grophecy_group_result;
+
+/* Groups of the batch into DEVICE array device_out (capacity entries, in
+ * record order); *n_groups (HOST) receives the number of groups.  ELIMIT if
+ * n_groups > capacity (the first `capacity` are written).  Synchronous. */
+int grophecy_group_best(grophecy_space *space, const grophecy_pcie *pcie,
+                        const grophecy_batch *batch, grophecy_group_result *device_out,
+                        uint64_t capacity, uint64_t *n_groups, void *cuda_stream);
+
+/* GPU speedup = total CPU time / total GPU time. */
+double grophecy_speedup(double t_cpu_s, double t_gpu_s);
+/* Error magnitude |predicted - measured| / measured (Table II applies
+ * it to predicted vs measured speedups).  Pure host functions. */
+double grophecy_error_magnitude(double predicted, double measured);
 
 /* End-to-end entry point with HOST record arrays (pinned for full speed):
  * streams the records to the device in chunks, overlapping copies with the

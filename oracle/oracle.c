@@ -289,6 +289,70 @@ int oracle_eval_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
     return 1;
 }
 
+/* The same computation, returning the four components. */
+int oracle_eval_parts_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                          const or_link *h2d_link, const or_link *d2h_link,
+                          uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters,
+                          double *t_iter, double *t_once, double *t_h2d, double *t_d2h)
+{
+    uint32_t skel = skx >> 16, xform = skx & 0xffffu;
+    if (skel >= n_skels || xform >= skels[skel].n_xforms || nx < 1 || nx > (1u << 20) ||
+        ny < 1 || ny > (1u << 20) || iters < 1) {
+        *t_iter = *t_once = *t_h2d = *t_d2h = NAN;
+        return 0;
+    }
+    const or_skeleton *s = &skels[skel];
+    uint64_t hpa[64], dpa[64];
+    oracle_usage(s, nx, ny, hpa, dpa);
+    double ti = 0.0, to = 0.0;
+    for (uint32_t k = 0; k < s->n_kernels; k++) {
+        double tk = oracle_kernel_time(s, g, xform, k, nx, ny, NULL);
+        if (s->kernels[k].per_iter) ti = ti + tk;
+        else to = to + tk;
+    }
+    double th = 0.0, td = 0.0;
+    for (uint32_t a = 0; a < s->n_arrays; a++)
+        if (hpa[a] > 0) th = th + oracle_pcie_time(h2d_link, hpa[a]);
+    for (uint32_t a = 0; a < s->n_arrays; a++)
+        if (dpa[a] > 0) td = td + oracle_pcie_time(d2h_link, dpa[a]);
+    *t_iter = ti; *t_once = to; *t_h2d = th; *t_d2h = td;
+    return 1;
+}
+
+/* Plain loop: runs of equal (skeleton, nx, ny, iters); per run the argmin of
+ * (t, index) over valid records with finite t ("the predicted time of the
+ * best-performing version"). */
+uint64_t oracle_group_best(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                           const or_link *h2d_link, const or_link *d2h_link,
+                           const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                           const uint32_t *iters, uint64_t n, uint64_t index_base,
+                           uint64_t capacity, uint64_t *first, uint64_t *count,
+                           uint64_t *best_index, double *best_t)
+{
+    uint64_t ng = 0, i = 0;
+    while (i < n) {
+        uint64_t j = i;
+        double bt = INFINITY;
+        uint64_t bi = UINT64_MAX;
+        while (j < n && (skx[j] >> 16) == (skx[i] >> 16) && nx[j] == nx[i] && ny[j] == ny[i] &&
+               iters[j] == iters[i]) {
+            uint64_t h, d; double t;
+            if (oracle_eval_one(skels, n_skels, g, h2d_link, d2h_link, skx[j], nx[j], ny[j],
+                                iters[j], &h, &d, &t) && isfinite(t)) {
+                if (bi == UINT64_MAX || t < bt) { bt = t; bi = index_base + j; }
+            }
+            j++;
+        }
+        if (ng < capacity) {
+            first[ng] = index_base + i; count[ng] = j - i;
+            best_index[ng] = bi; best_t[ng] = bt;
+        }
+        ng++;
+        i = j;
+    }
+    return ng;
+}
+
 /* ------------------------------------------------------------------------ */
 /* Batch drivers: a static partition over host threads (plain loop inside). */
 /* ------------------------------------------------------------------------ */

@@ -73,6 +73,26 @@ int  oracle_bitmap_usage(const or_skeleton *s, int64_t nx, int64_t ny,
 double oracle_kernel_time(const or_skeleton *s, const or_gpu *g, uint32_t xform,
                           uint32_t k, int64_t nx, int64_t ny, int *regime);
 
+/* Components of one candidate's time:
+ * t = ((t_once + iters * t_iter) + t_h2d) + t_d2h.  Returns 1 if valid
+ * (else all components NaN). */
+int oracle_eval_parts_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                          const or_link *h2d_link, const or_link *d2h_link,
+                          uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters,
+                          double *t_iter, double *t_once, double *t_h2d, double *t_d2h);
+
+/* Best transformation per group: groups are maximal runs of
+ * consecutive records with equal (skeleton, nx, ny, iters); per group the
+ * first index, the size, and the argmin (t, index) over valid records with
+ * finite t (best_index UINT64_MAX, best_t +inf when none).  Returns the number
+ * of groups (results beyond `capacity` are not written). */
+uint64_t oracle_group_best(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                           const or_link *h2d_link, const or_link *d2h_link,
+                           const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                           const uint32_t *iters, uint64_t n, uint64_t index_base,
+                           uint64_t capacity, uint64_t *first, uint64_t *count,
+                           uint64_t *best_index, double *best_t);
+
 /* One candidate.  Returns 1 if the record is valid. */
 int oracle_eval_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
                     const or_link *h2d_link, const or_link *d2h_link,

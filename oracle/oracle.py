@@ -108,6 +108,13 @@ def lib():
         L.oracle_best.argtypes = [SK, C.c_uint32, C.POINTER(GPU), C.POINTER(Link),
                                   C.POINTER(Link), u32p, u32p, u32p, u32p, C.c_uint64,
                                   C.c_uint64, C.c_int, C.POINTER(Best)]
+        L.oracle_eval_parts_one.argtypes = [SK, C.c_uint32, C.POINTER(GPU), C.POINTER(Link),
+                                            C.POINTER(Link), C.c_uint32, C.c_uint32, C.c_uint32,
+                                            C.c_uint32] + [C.POINTER(C.c_double)] * 4
+        L.oracle_group_best.argtypes = [SK, C.c_uint32, C.POINTER(GPU), C.POINTER(Link),
+                                        C.POINTER(Link), u32p, u32p, u32p, u32p, C.c_uint64,
+                                        C.c_uint64, C.c_uint64, u64p, u64p, u64p, f64p]
+        L.oracle_group_best.restype = C.c_uint64
         for name in ("oracle_error_magnitude", "oracle_speedup", "oracle_speedup_error"):
             getattr(L, name).argtypes = [C.c_double, C.c_double]
             getattr(L, name).restype = C.c_double
@@ -222,6 +229,25 @@ class Problem:
         lib().oracle_eval(self.ss.arr, self.ss.n, C.byref(self.gpu), C.byref(self.hl),
                           C.byref(self.dl), *a, n, nthreads, h, d, t)
         return h, d, t
+
+    def eval_parts_one(self, skx, nx, ny, iters):
+        v = [C.c_double() for _ in range(4)]
+        ok = lib().oracle_eval_parts_one(self.ss.arr, self.ss.n, C.byref(self.gpu),
+                                         C.byref(self.hl), C.byref(self.dl), skx, nx, ny, iters,
+                                         *[C.byref(x) for x in v])
+        return bool(ok), tuple(x.value for x in v)
+
+    def group_best(self, rec, index_base=0):
+        n = len(rec["skx"])
+        cap = max(1, n)
+        first = np.zeros(cap, np.uint64)
+        count = np.zeros(cap, np.uint64)
+        bi = np.zeros(cap, np.uint64)
+        bt = np.zeros(cap, np.float64)
+        a = [np.ascontiguousarray(rec[k], dtype=np.uint32) for k in ("skx", "nx", "ny", "iters")]
+        ng = lib().oracle_group_best(self.ss.arr, self.ss.n, C.byref(self.gpu), C.byref(self.hl),
+                                     C.byref(self.dl), *a, n, index_base, cap, first, count, bi, bt)
+        return first[:ng], count[:ng], bi[:ng], bt[:ng]
 
     def best(self, rec, index_base=0, nthreads=None):
         n = len(rec["skx"])

@@ -16,7 +16,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(HERE, "libgrophecy.so")
-SOURCES = ["space.cpp", "plan.cpp", "project.cu", "synth.cu", "pcie.cu"]
+SOURCES = ["space.cpp", "plan.cpp", "project.cu", "groups.cu", "synth.cu", "pcie.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

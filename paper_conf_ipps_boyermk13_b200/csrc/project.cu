@@ -611,6 +611,7 @@ struct Params {
     unsigned long long *h2d;
     unsigned long long *d2h;
     double *t;
+    double *p_iter, *p_once, *p_h2d, *p_d2h;   // optional component outputs (eval)
     grophecy_best_result *partials;
     unsigned int *ticket;
     grophecy_best_result *out;
@@ -829,6 +830,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     __stcs(P.h2d + i, u.h);
                     __stcs(P.d2h + i, u.d);
                     __stcs(P.t + i, t);
+                    if (P.p_iter) __stcs(P.p_iter + i, ti[j]);
+                    if (P.p_once) __stcs(P.p_once + i, to[j]);
+                    if (P.p_h2d) __stcs(P.p_h2d + i, u.th);
+                    if (P.p_d2h) __stcs(P.p_d2h + i, u.td);
                 } else if (t < __longlong_as_double(0x7ff0000000000000LL) &&
                            better(t, P.base + i, best_t, best_i)) {
                     best_t = t;
@@ -851,7 +856,12 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     if (i < P.n && ws.rec_slot[lane + 32 * j] == -1) {
                         __stcs(P.h2d + i, 0ull);
                         __stcs(P.d2h + i, 0ull);
-                        __stcs(P.t + i, __longlong_as_double(0x7ff8000000000000LL));
+                        const double nan = __longlong_as_double(0x7ff8000000000000LL);
+                        __stcs(P.t + i, nan);
+                        if (P.p_iter) __stcs(P.p_iter + i, nan);
+                        if (P.p_once) __stcs(P.p_once + i, nan);
+                        if (P.p_h2d) __stcs(P.p_h2d + i, nan);
+                        if (P.p_d2h) __stcs(P.p_d2h + i, nan);
                     }
                 }
             }
@@ -974,6 +984,7 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
     P.h2d = nullptr;
     P.d2h = nullptr;
     P.t = nullptr;
+    P.p_iter = P.p_once = P.p_h2d = P.p_d2h = nullptr;
     P.partials = s->partials;
     P.ticket = s->ticket;
     P.out = nullptr;
@@ -1003,8 +1014,9 @@ using namespace grophecy;
 
 extern "C" {
 
-int grophecy_eval(const grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
-                  uint64_t *h2d, uint64_t *d2h, double *t, void *stream)
+int grophecy_eval_parts(const grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
+                        uint64_t *h2d, uint64_t *d2h, double *t, const grophecy_parts *parts,
+                        void *stream)
 {
     int rc = check_batch(s, pc, b);
     if (rc) return rc;
@@ -1017,12 +1029,24 @@ int grophecy_eval(const grophecy_space *s, const grophecy_pcie *pc, const grophe
     P.h2d = (unsigned long long *)h2d;
     P.d2h = (unsigned long long *)d2h;
     P.t = t;
+    if (parts) {
+        P.p_iter = parts->t_iter_s;
+        P.p_once = parts->t_once_s;
+        P.p_h2d = parts->t_h2d_s;
+        P.p_d2h = parts->t_d2h_s;
+    }
     const int grid = grid_for(s, b->n, 32);
     project_kernel<false><<<grid, THREADS, sizeof(CtaSmem), (cudaStream_t)stream>>>(P);
     count_launch();
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "project_kernel<eval> launch");
     return GROPHECY_OK;
+}
+
+int grophecy_eval(const grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
+                  uint64_t *h2d, uint64_t *d2h, double *t, void *stream)
+{
+    return grophecy_eval_parts(s, pc, b, h2d, d2h, t, nullptr, stream);
 }
 
 int grophecy_best_async(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,

@@ -219,6 +219,13 @@ double grophecy_pcie_time(const grophecy_link *link, uint64_t bytes)
     return link->alpha_s + link->beta_s_per_byte * (double)bytes;
 }
 
+double grophecy_speedup(double t_cpu_s, double t_gpu_s) { return t_cpu_s / t_gpu_s; }
+
+double grophecy_error_magnitude(double predicted, double measured)
+{
+    return std::fabs(predicted - measured) / measured;
+}
+
 int grophecy_space_validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                             const grophecy_gpu_model *gpu)
 {

@@ -103,6 +103,16 @@ class BestResult(C.Structure):
 assert C.sizeof(BestResult) == 48 and C.sizeof(RegionDesc) == 68 and C.sizeof(KxDesc) == 64
 
 
+class Parts(C.Structure):
+    _fields_ = [("t_iter_s", C.c_void_p), ("t_once_s", C.c_void_p), ("t_h2d_s", C.c_void_p),
+                ("t_d2h_s", C.c_void_p)]
+
+
+class GroupResult(C.Structure):
+    _fields_ = [("best_t_s", C.c_double), ("first", C.c_uint64), ("count", C.c_uint64),
+                ("best_index", C.c_uint64), ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64)]
+
+
 class SynthRule(C.Structure):
     _fields_ = [("kind", C.c_uint32), ("lo", C.c_uint32), ("hi", C.c_uint32),
                 ("it_lo", C.c_uint32), ("it_hi", C.c_uint32), ("pad", C.c_uint32)]
@@ -118,6 +128,12 @@ _sig = {
     "grophecy_space_destroy": (None, [_vp]),
     "grophecy_eval": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, _vp, _vp, _vp]),
     "grophecy_invalid_count": (C.c_int, [_vp, C.POINTER(C.c_uint64), _vp]),
+    "grophecy_eval_parts": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, _vp, _vp,
+                                      C.POINTER(Parts), _vp]),
+    "grophecy_group_best": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, C.c_uint64,
+                                      C.POINTER(C.c_uint64), _vp]),
+    "grophecy_speedup": (C.c_double, [C.c_double, C.c_double]),
+    "grophecy_error_magnitude": (C.c_double, [C.c_double, C.c_double]),
     "grophecy_best": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), C.POINTER(BestResult), _vp]),
     "grophecy_best_async": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, C.c_int, _vp]),
     "grophecy_best_combine": (C.c_int, [_vp, C.c_uint32, _vp, _vp]),
@@ -320,6 +336,34 @@ class Space:
                                 _ptr(out[2]), _stream_ptr(stream)), "eval")
         return out
 
+    def eval_parts(self, pc, rec, index_base=0, stream=None):
+        """(h2d, d2h, t, t_iter, t_once, t_h2d, t_d2h) device tensors."""
+        torch = _torch()
+        n, dev = rec.n, rec.skx.device
+        h = torch.empty(n, dtype=torch.int64, device=dev)
+        d = torch.empty(n, dtype=torch.int64, device=dev)
+        ts = [torch.empty(n, dtype=torch.float64, device=dev) for _ in range(5)]
+        parts = Parts(*[t.data_ptr() for t in ts[1:]])
+        b = rec.batch(index_base)
+        _check(_L.grophecy_eval_parts(self.h, C.byref(pc), C.byref(b), _ptr(h), _ptr(d),
+                                      _ptr(ts[0]), C.byref(parts), _stream_ptr(stream)),
+               "eval_parts")
+        return (h, d, *ts)
+
+    def group_best(self, pc, rec, index_base=0, capacity=None, stream=None):
+        """List of GroupResult (best transformation per projection point)."""
+        torch = _torch()
+        cap = rec.n if capacity is None else capacity
+        out = torch.empty(max(1, cap) * 6, dtype=torch.int64, device=rec.skx.device)
+        ng = C.c_uint64()
+        b = rec.batch(index_base)
+        rc = _L.grophecy_group_best(self.h, C.byref(pc), C.byref(b), _ptr(out), cap,
+                                    C.byref(ng), _stream_ptr(stream))
+        _check(rc, "group_best", ok=(OK, ELIMIT))
+        raw = out.cpu().numpy().tobytes()
+        k = min(ng.value, cap)
+        return rc, ng.value, [GroupResult.from_buffer_copy(raw[48 * i:48 * (i + 1)]) for i in range(k)]
+
     def invalid_count(self, stream=None):
         v = C.c_uint64()
         _check(_L.grophecy_invalid_count(self.h, C.byref(v), _stream_ptr(stream)), "invalid_count")
@@ -404,6 +448,14 @@ def plan_stats(skel):
     st = (C.c_uint32 * 6)()
     rc = _L.grophecy_plan_stats(sd.arr, st)
     return rc, list(st)
+
+
+def speedup(t_cpu, t_gpu):
+    return _L.grophecy_speedup(t_cpu, t_gpu)
+
+
+def error_magnitude(pred, meas):
+    return _L.grophecy_error_magnitude(pred, meas)
 
 
 def launch_count():
