@@ -350,16 +350,22 @@ class Space:
                "eval_parts")
         return (h, d, *ts)
 
-    def group_best(self, pc, rec, index_base=0, capacity=None, stream=None):
-        """List of GroupResult (best transformation per projection point)."""
+    def group_best(self, pc, rec, index_base=0, capacity=None, stream=None, out=None,
+                   as_tensor=False):
+        """Best transformation per projection point: (rc, n_groups, results)
+        with results a list of GroupResult, or the raw device tensor (6 int64
+        per group) when as_tensor=True."""
         torch = _torch()
         cap = rec.n if capacity is None else capacity
-        out = torch.empty(max(1, cap) * 6, dtype=torch.int64, device=rec.skx.device)
+        if out is None:
+            out = torch.empty(max(1, cap) * 6, dtype=torch.int64, device=rec.skx.device)
         ng = C.c_uint64()
         b = rec.batch(index_base)
         rc = _L.grophecy_group_best(self.h, C.byref(pc), C.byref(b), _ptr(out), cap,
                                     C.byref(ng), _stream_ptr(stream))
         _check(rc, "group_best", ok=(OK, ELIMIT))
+        if as_tensor:
+            return rc, ng.value, out
         raw = out.cpu().numpy().tobytes()
         k = min(ng.value, cap)
         return rc, ng.value, [GroupResult.from_buffer_copy(raw[48 * i:48 * (i + 1)]) for i in range(k)]

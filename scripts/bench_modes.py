@@ -1,0 +1,99 @@
+"""Throughput of every projection entry point on the C4 workload (one GPU).
+
+    python scripts/bench_modes.py [n_records] [reps]
+
+One JSON line per mode: best (fused argmin), eval (SoA outputs), eval_parts
+(+ time components), group_best (best transformation per projection point),
+best_host (host records, PCIe-bound).  Candidates/s from CUDA events (or the
+host clock for the synchronous calls), algorithmic HBM bytes per candidate,
+and the fraction of MEASURED_PEAKS.json's HBM bandwidth.
+"""
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+from paper_conf_ipps_boyermk13_b200 import build  # noqa: E402
+
+build.build()
+from paper_conf_ipps_boyermk13_b200 import grophecy as G  # noqa: E402
+from synth import records as R  # noqa: E402
+from synth import skeletons as S  # noqa: E402
+
+
+def hbm_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    return json.load(open(p))["hbm_gbs"] if os.path.exists(p) else 6650.0
+
+
+def timed(fn, reps, events=True):
+    fn()
+    torch.cuda.synchronize()
+    if events:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(reps):
+            fn()
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / reps * 1e-3
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        fn()
+    torch.cuda.synchronize()
+    return (time.perf_counter() - t0) / reps
+
+
+def main():
+    n = int(sys.argv[1]) if len(sys.argv) > 1 else 1 << 27
+    reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
+    cfg = R.config("c4")
+    space = G.Space(cfg["skeletons"], S.FX5600)
+    pc = G.pcie(G.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL))
+    # an evenly spread sample of the 10^9 sweep: 16 slices (every skeleton)
+    per = n // 16
+    recs = [G.synth_records(cfg, k * (cfg["n"] // 16), per) for k in range(16)]
+    rec = G.Records(*[torch.cat([getattr(r, f) for r in recs]) for f in ("skx", "nx", "ny", "iters")])
+    n = rec.n
+    peak = hbm_peak()
+    out = torch.empty(6, dtype=torch.int64, device="cuda")
+    h = torch.empty(n, dtype=torch.int64, device="cuda")
+    d = torch.empty(n, dtype=torch.int64, device="cuda")
+    t = torch.empty(n, dtype=torch.float64, device="cuda")
+    parts = [torch.empty(n, dtype=torch.float64, device="cuda") for _ in range(4)]
+    b = rec.batch()
+    gout = torch.empty((n // 8) * 6, dtype=torch.int64, device="cuda")
+    P = G.Parts(*[x.data_ptr() for x in parts])
+    import ctypes as C
+    st = torch.cuda.current_stream().cuda_stream
+    modes = {
+        "best": (lambda: space.best_async(pc, b, out), 16, True),
+        "eval": (lambda: G.lib().grophecy_eval(space.h, C.byref(pc), C.byref(b), h.data_ptr(),
+                                               d.data_ptr(), t.data_ptr(), C.c_void_p(st)), 40, True),
+        "eval_parts": (lambda: G.lib().grophecy_eval_parts(space.h, C.byref(pc), C.byref(b),
+                                                           h.data_ptr(), d.data_ptr(), t.data_ptr(),
+                                                           C.byref(P), C.c_void_p(st)), 72, True),
+        "group_best": (lambda: space.group_best(pc, rec, capacity=n // 8, out=gout, as_tensor=True),
+                       16 + 24 + 24 + 16, False),
+    }
+    for name, (fn, bpc, ev) in modes.items():
+        sec = timed(fn, reps, ev)
+        gbs = bpc * n / sec / 1e9
+        print(json.dumps({"mode": name, "n": n, "cand_per_s": n / sec, "ms": sec * 1e3,
+                          "bytes_per_candidate": bpc, "hbm_GBps": gbs, "hbm_frac": gbs / peak,
+                          "timer": "cuda events" if ev else "host clock (synchronous call)"}),
+              flush=True)
+    host = {k: getattr(rec, k).cpu().pin_memory() for k in ("skx", "nx", "ny", "iters")}
+    sec = timed(lambda: space.best_host(pc, host), max(1, reps // 2), False)
+    print(json.dumps({"mode": "best_host", "n": n, "cand_per_s": n / sec, "ms": sec * 1e3,
+                      "h2d_bytes": 16 * n, "link_GBps": 16 * n / sec / 1e9,
+                      "timer": "host clock"}), flush=True)
+
+
+if __name__ == "__main__":
+    main()
