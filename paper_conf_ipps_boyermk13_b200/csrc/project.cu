@@ -510,6 +510,7 @@ struct WarpSmem {
     uint32_t rec_skx[WTILE], rec_it[WTILE];
     int rec_slot[WTILE];
     unsigned long long best_h[32], best_d[32];  // bytes of each lane's running best
+    uint8_t plan_pos[MAX_SEG];                  // plan keys of the current slot group
 };
 struct CtaSmem {
     WarpSmem w[WARPS];
@@ -761,18 +762,18 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                             : max_ne * 4 <= VAL_PER_WARP ? 8
                             : max_ne * 2 <= VAL_PER_WARP ? 16 : 32;
                 const int G = 32 / L, seg = lane / L, sl = lane % L;
-                while (todo) {
-                    const unsigned pos = __fns(todo, 0, seg + 1);
-                    const bool act = pos < 32u;
-                    const unsigned long long k = __shfl_sync(FULL, mk, act ? pos : 0);
-                    const unsigned ls = g0 - c0 + (act ? pos : 0);
+                // compact list of the plan keys' positions (rank -> slot lane)
+                if (mv && mplan) ws.plan_pos[__popc(todo & ((1u << lane) - 1u))] = (uint8_t)lane;
+                const int nplan = __popc(todo);
+                __syncwarp();
+                for (int p0 = 0; p0 < nplan; p0 += G) {
+                    const bool act = p0 + seg < nplan;
+                    const unsigned pos = act ? ws.plan_pos[p0 + seg] : 0u;
+                    const unsigned long long k = __shfl_sync(FULL, mk, pos);
+                    const unsigned ls = g0 - c0 + pos;
                     // segment stride VAL/G + L longs: the segments' lanes hit distinct banks
                     plan_usage(S, act, k, P.pc, ws.scratch.pl.val + seg * (VAL_PER_WARP / G + L),
                                ws.scratch.pl.T[seg], sl, L, &ws.res[ls], ws.slot_w[ls]);
-                    {   // drop the G keys just processed (the lowest G set bits)
-                        const unsigned nxt = __fns(todo, 0, G + 1);
-                        todo = nxt < 32u ? todo & ~((1u << nxt) - 1u) : 0u;
-                    }
                     __syncwarp();
                 }
                 while (sweep) {
@@ -818,28 +819,47 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                         model_n<1, false>(S, ws.rec_skx[lane + 32 * j] >> 16, xs + j, ls + j, ws,
                                           ti + j, to + j);
             }
+            double tt[RPT];
 #pragma unroll
             for (int j = 0; j < RPT; j++) {
-                if (!inj[j]) continue;
-                const unsigned long long i = tb + lane + 32 * j;
                 const Usage &u = ws.res[ls[j]];
                 // total: run-once + iters x per-iteration + transfers
                 const double t_kern = __dadd_rn(to[j], __dmul_rn((double)ws.rec_it[lane + 32 * j], ti[j]));
-                const double t = __dadd_rn(__dadd_rn(t_kern, u.th), u.td);
-                if (!BEST) {
+                tt[j] = __dadd_rn(__dadd_rn(t_kern, u.th), u.td);
+            }
+            if (!BEST) {
+#pragma unroll
+                for (int j = 0; j < RPT; j++) {
+                    if (!inj[j]) continue;
+                    const unsigned long long i = tb + lane + 32 * j;
+                    const Usage &u = ws.res[ls[j]];
                     __stcs(P.h2d + i, u.h);
                     __stcs(P.d2h + i, u.d);
-                    __stcs(P.t + i, t);
+                    __stcs(P.t + i, tt[j]);
                     if (P.p_iter) __stcs(P.p_iter + i, ti[j]);
                     if (P.p_once) __stcs(P.p_once + i, to[j]);
                     if (P.p_h2d) __stcs(P.p_h2d + i, u.th);
                     if (P.p_d2h) __stcs(P.p_d2h + i, u.td);
-                } else if (t < __longlong_as_double(0x7ff0000000000000LL) &&
-                           better(t, P.base + i, best_t, best_i)) {
-                    best_t = t;
-                    best_i = P.base + i;
-                    ws.best_h[lane] = u.h;
-                    ws.best_d[lane] = u.d;
+                }
+            } else {
+                // the lane's best of its (index-ordered) records, then one compare
+                double bt = __longlong_as_double(0x7ff0000000000000LL);
+                int bj = -1;
+#pragma unroll
+                for (int j = 0; j < RPT; j++)
+                    if (inj[j] && tt[j] < bt) {
+                        bt = tt[j];
+                        bj = j;
+                    }
+                if (bj >= 0) {
+                    const unsigned long long i = P.base + tb + lane + 32 * bj;
+                    if (better(bt, i, best_t, best_i)) {
+                        best_t = bt;
+                        best_i = i;
+                        const Usage &u = ws.res[ls[bj]];
+                        ws.best_h[lane] = u.h;
+                        ws.best_d[lane] = u.d;
+                    }
                 }
             }
             __syncwarp();
