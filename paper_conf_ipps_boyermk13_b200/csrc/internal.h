@@ -47,7 +47,7 @@ struct SkelInfo {
     // usage plan (plan.cpp): valid for nx >= plan_tx and ny >= plan_ty
     uint32_t plan_tx, plan_ty, expr_base, n_expr;
     // flat term list of all arrays / directions: {packed indices, 2*array + dir}
-    uint32_t term_base, n_terms, pad1, pad2;
+    uint32_t term_base, n_terms, per_iter_mask, pad2;   // per_iter_mask: bit k = kernel k per-iteration
 };
 
 struct ArrayDev {

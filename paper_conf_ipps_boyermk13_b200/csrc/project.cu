@@ -381,12 +381,15 @@ __device__ __forceinline__ double kernel_time(const SpaceDev &S, long long Wi, c
     unsigned long long abps = blocks / asm_ + (blocks % asm_ != 0);
     if ((unsigned long long)J.occ < abps) abps = J.occ;
     const double N = __ull2double_rn(abps * (unsigned long long)J.wpb);
-    const double rep = __ddiv_rn(__ull2double_rn(blocks), __ull2double_rn(abps * asm_));
+    // integer denominators: RN(1/d) by __drcp_rn, then Markstein's correction
+    const double dden = __ull2double_rn(abps * asm_);
+    const double rep = div_rn(__ull2double_rn(blocks), dden, __drcp_rn(dden));
     double cyc;
     if (J.flags & KXF_NOMEM) {
         cyc = __dmul_rn(__dmul_rn(G.comp, N), rep);
     } else {
-        const double mpk = __ddiv_rn(G.bwr, __ull2double_rn(asm_));
+        const double dasm = __ull2double_rn(asm_);
+        const double mpk = div_rn(G.bwr, dasm, __drcp_rn(dasm));
         const double mwp = dmin(dmin(G.mwp0, mpk), N);
         const double cwp = dmin(G.cwpf, N);
         const double cpm_term = __dmul_rn(G.cpm, __dsub_rn(mwp, 1.0));
@@ -402,7 +405,7 @@ __device__ __forceinline__ double kernel_time(const SpaceDev &S, long long Wi, c
             rep);
         cyc = __dadd_rn(cyc, sync);
     }
-    return __ddiv_rn(cyc, S.freq);
+    return div_rn(cyc, S.freq, S.rfreq);
 }
 
 // Total projected time of one candidate: kernels (run-once
@@ -527,7 +530,7 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
                                         double *t_once)
 {
     const SkelInfo &I = S.skel[s];
-    const uint32_t K = I.n_kernels, X = I.n_xforms;
+    const uint32_t K = I.n_kernels, X = I.n_xforms, pim = I.per_iter_mask;
     double ti[NJ], to[NJ];
 #pragma unroll
     for (int j = 0; j < NJ; j++) ti[j] = to[j] = 0.0;
@@ -571,9 +574,10 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
 #pragma unroll
         for (int j = 0; j < NJ; j++) {
             const double v = __fma_rn(rep[j], S.rfreq, q[j]);
-            const bool inf = isinf(F[j].E);
-            gen[j] = !inf && blocks[j] != 0 && (w[j] == 0xffffffffu || blocks[j] < F[j].sat32);
-            tk[j] = inf ? __longlong_as_double(0x7ff0000000000000LL) : (blocks[j] == 0 ? 0.0 : v);
+            // feasible: sat32 >= 1, so blocks == 0 and small grids take the
+            // general path; infeasible (E == +inf): sat32 == 0, t = +inf
+            gen[j] = w[j] == 0xffffffffu || blocks[j] < F[j].sat32;
+            tk[j] = isinf(F[j].E) ? __longlong_as_double(0x7ff0000000000000LL) : v;
         }
 #pragma unroll
         for (int j = 0; j < NJ; j++)
@@ -584,7 +588,7 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
                                           (long long)(kk & 0x1fffffull));
                 tk[j] = kernel_time(S, Wi, S.kx_j[kb + x[j]], kb + x[j]);
             }
-        if (__ldg(&S.kern_flags[I.k_base + k]) & GROPHECY_KERNEL_PER_ITER) {
+        if ((pim >> k) & 1u) {
 #pragma unroll
             for (int j = 0; j < NJ; j++) ti[j] = __dadd_rn(ti[j], tk[j]);
         } else {
@@ -721,10 +725,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             ws.rec_it[q] = it[j];
             ws.rec_slot[q] = head ? -2 - slot : slot;   // heads encoded as -2 - slot
             ws.rec_key[q] = key[j];
-            if (tb + q < P.n) {
-                if (key[j] == ~0ull) n_invalid++;
-                else n_valid++;
-            }
+            const bool has = tb + q < P.n;
+            n_invalid += has && key[j] == ~0ull;
+            n_valid += key[j] != ~0ull;
         }
         (void)lt;
         __syncwarp();
@@ -757,11 +760,12 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                 unsigned todo = __ballot_sync(FULL, mv && mplan);
                 unsigned sweep = __ballot_sync(FULL, mv && !mplan);
                 const uint32_t max_ne = __reduce_max_sync(FULL, mplan ? mne : 0u);
-                // lanes per key: 4 (8 keys per pass) unless the values do not fit
-                const int L = max_ne * MAX_SEG <= VAL_PER_WARP ? 32 / MAX_SEG
-                            : max_ne * 4 <= VAL_PER_WARP ? 8
-                            : max_ne * 2 <= VAL_PER_WARP ? 16 : 32;
-                const int G = 32 / L, seg = lane / L, sl = lane % L;
+                // lanes per key L = 2^lg: 4 (8 keys per pass) unless the values do not fit
+                const int lg = max_ne * MAX_SEG <= VAL_PER_WARP ? 2
+                             : max_ne * 4 <= VAL_PER_WARP ? 3
+                             : max_ne * 2 <= VAL_PER_WARP ? 4 : 5;
+                const int L = 1 << lg, G = 32 >> lg, seg = lane >> lg, sl = lane & (L - 1);
+                const int vstride = (VAL_PER_WARP >> (5 - lg)) + L;   // VAL/G + L
                 // compact list of the plan keys' positions (rank -> slot lane)
                 if (mv && mplan) ws.plan_pos[__popc(todo & ((1u << lane) - 1u))] = (uint8_t)lane;
                 const int nplan = __popc(todo);
@@ -772,7 +776,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     const unsigned long long k = __shfl_sync(FULL, mk, pos);
                     const unsigned ls = g0 - c0 + pos;
                     // segment stride VAL/G + L longs: the segments' lanes hit distinct banks
-                    plan_usage(S, act, k, P.pc, ws.scratch.pl.val + seg * (VAL_PER_WARP / G + L),
+                    plan_usage(S, act, k, P.pc, ws.scratch.pl.val + seg * vstride,
                                ws.scratch.pl.T[seg], sl, L, &ws.res[ls], ws.slot_w[ls]);
                     __syncwarp();
                 }

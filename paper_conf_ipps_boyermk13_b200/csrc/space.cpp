@@ -285,7 +285,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         if (plan.ok) pprog.insert(pprog.end(), plan.prog.begin(), plan.prog.end());
         I.term_base = (uint32_t)pterms.size();
         I.n_terms = 0;
-        I.pad1 = I.pad2 = 0;
+        I.per_iter_mask = I.pad2 = 0;
+        for (uint32_t k = 0; k < S.n_kernels; k++)
+            if (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) I.per_iter_mask |= 1u << k;
         if (plan.ok)
             for (uint32_t a = 0; a < S.n_arrays; a++)
                 for (uint32_t dir = 0; dir < 2; dir++) {
