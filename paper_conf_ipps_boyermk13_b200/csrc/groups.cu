@@ -154,20 +154,24 @@ extern "C" int grophecy_group_best(grophecy_space *s, const grophecy_pcie *pc,
     cudaStream_t st = (cudaStream_t)stream;
     const unsigned long long n = b->n;
     const unsigned long long nb = (n + G_BLOCK - 1) / G_BLOCK;
-    char *tmp = nullptr;
     const size_t bytes = n * 24 + (nb + 1) * 8;
-    cudaError_t e = cudaMallocAsync((void **)&tmp, bytes, st);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaMallocAsync(group scratch)");
+    cudaError_t e;
+    if (s->gscratch_bytes < bytes) {   // space-owned scratch, grown on demand
+        if (s->gscratch) cudaFree(s->gscratch);
+        s->gscratch = nullptr;
+        s->gscratch_bytes = 0;
+        if ((e = cudaMalloc(&s->gscratch, bytes)) != cudaSuccess)
+            return cuda_fail(e, "cudaMalloc(group scratch)");
+        s->gscratch_bytes = bytes;
+    }
+    char *tmp = (char *)s->gscratch;
     double *t = (double *)tmp;
     unsigned long long *h2d = (unsigned long long *)(tmp + n * 8);
     unsigned long long *d2h = (unsigned long long *)(tmp + n * 16);
     unsigned long long *counts = (unsigned long long *)(tmp + n * 24);
     unsigned long long *total = counts + nb;
     int rc = grophecy_eval(s, pc, b, (uint64_t *)h2d, (uint64_t *)d2h, t, stream);
-    if (rc) {
-        cudaFreeAsync(tmp, st);
-        return rc;
-    }
+    if (rc) return rc;
     group_count<<<(unsigned)nb, G_THREADS, 0, st>>>(*b, counts);
     group_scan<<<1, 1024, 0, st>>>(counts, nb, total);
     group_reduce<<<(unsigned)nb, G_THREADS, 0, st>>>(*b, counts, t, h2d, d2h, device_out, capacity);
@@ -175,7 +179,6 @@ extern "C" int grophecy_group_best(grophecy_space *s, const grophecy_pcie *pc,
     unsigned long long ng = 0;
     e = cudaGetLastError();
     if (e == cudaSuccess) e = cudaMemcpyAsync(&ng, total, 8, cudaMemcpyDeviceToHost, st);
-    if (e == cudaSuccess) e = cudaFreeAsync(tmp, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     if (e != cudaSuccess) return cuda_fail(e, "grophecy_group_best");
     *n_groups = ng;

@@ -108,6 +108,9 @@ struct grophecy_space {
     unsigned long long *invalid_counter;
     uint32_t max_partials;
     int grid_best, grid_eval;            // persistent grid sizes
+    // group_best scratch (grown on demand)
+    void *gscratch;
+    size_t gscratch_bytes;
     // e2e host path staging
     void *stage[2];
     size_t stage_bytes;
