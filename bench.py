@@ -209,9 +209,16 @@ def main():
     from synth import records as R
     from synth import skeletons as S
 
-    torch.cuda.set_device(local_rank)
+    # one process per GPU; GROPHECY_DIST_BACKEND=gloo exercises the multi-rank
+    # path with several ranks sharing a GPU (NCCL needs one GPU per rank)
+    backend = os.environ.get("GROPHECY_DIST_BACKEND", "nccl")
+    local_dev = local_rank % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(local_dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_dev))
+        else:
+            dist.init_process_group(backend)
     cfg = R.config(args.config)
     if args.n:
         cfg = R.with_n(cfg, args.n)
@@ -223,7 +230,7 @@ def main():
     stream = torch.cuda.current_stream()
     rec = G.synth_records(cfg, lo, n_local)          # shard generated in its own HBM
     batch = rec.batch(index_base=lo)
-    minloc = D.MinLoc(world)
+    minloc = D.MinLoc(world, backend=backend)
     host_res = torch.empty(6, dtype=torch.int64, pin_memory=True)
     torch.cuda.synchronize()
 
@@ -244,7 +251,7 @@ def main():
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    sampler = ClockSampler(local_rank) if rank == 0 else None
+    sampler = ClockSampler(local_dev) if rank == 0 else None
     if sampler:
         sampler.start()
         time.sleep(0.3)
@@ -265,7 +272,8 @@ def main():
     clocks = sampler.stop() if sampler else None
     ms = t0.elapsed_time(t1)
     kern_ms = [a.elapsed_time(b) for a, b in ev_k]
-    ms_t = torch.tensor([ms, statistics.mean(kern_ms)], dtype=torch.float64, device="cuda")
+    ms_t = torch.tensor([ms, statistics.mean(kern_ms)], dtype=torch.float64,
+                        device="cuda" if backend == "nccl" else "cpu")
     if world > 1:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
     ms_max, kern_avg_max = float(ms_t[0]), float(ms_t[1])
@@ -300,7 +308,7 @@ def main():
     roof_issue = None
     if prof.get("warp_inst_per_launch") and prof_n:
         sm_mhz = (clocks or {}).get("sm_mhz") or 1965.0
-        props = torch.cuda.get_device_properties(local_rank)
+        props = torch.cuda.get_device_properties(local_dev)
         peak_issue = props.multi_processor_count * 4 * sm_mhz * 1e6
         ach = prof["warp_inst_per_launch"] / prof_n * n_local / (kern_avg_max * 1e-3)
         if ach > 1.02 * peak_issue:   # committed capture is stale for this build
@@ -366,7 +374,8 @@ def run_e2e(G, torch, dist, space, pc, rec, lo, n_local, N, world, args):
     for _ in range(steps):
         space.best_host(pc, host, index_base=lo)
     dt = time.perf_counter() - t0
-    dt_t = torch.tensor([dt], dtype=torch.float64, device="cuda")
+    dt_t = torch.tensor([dt], dtype=torch.float64,
+                        device="cuda" if dist.is_initialized() and dist.get_backend() == "nccl" else "cpu")
     if world > 1:
         dist.all_reduce(dt_t, op=dist.ReduceOp.MAX)
     dt = float(dt_t[0])

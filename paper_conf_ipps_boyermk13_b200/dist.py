@@ -22,23 +22,37 @@ def shard_range(n, rank, world):
 
 class MinLoc:
     """Device buffers for one query: ``local`` (this rank's result, written by
-    grophecy_best_async), ``result`` (the global best after combine())."""
+    grophecy_best_async), ``result`` (the global best after combine()).
 
-    def __init__(self, world, device="cuda"):
+    NCCL (default): the 48-byte results are all-gathered device to device on
+    the compute stream, then the combine kernel runs on every rank.  With a
+    gloo process group (CPU collectives; used to exercise the multi-rank path
+    on a single GPU) the gather goes through host memory."""
+
+    def __init__(self, world, device="cuda", backend=None):
         from . import grophecy as G
         self.G = G
         self.world = world
+        self.backend = backend or (dist.get_backend() if world > 1 else "nccl")
         self.local = torch.empty(RESULT_WORDS, dtype=torch.int64, device=device)
         if world > 1:
             self.gathered = torch.empty(RESULT_WORDS * world, dtype=torch.int64, device=device)
             self.result = torch.empty(RESULT_WORDS, dtype=torch.int64, device=device)
+            if self.backend != "nccl":
+                self.h_local = torch.empty(RESULT_WORDS, dtype=torch.int64)
+                self.h_gathered = torch.empty(RESULT_WORDS * world, dtype=torch.int64)
         else:
             self.result = self.local
 
     def combine(self):
         if self.world == 1:
             return self.result
-        dist.all_gather_into_tensor(self.gathered, self.local)
+        if self.backend == "nccl":
+            dist.all_gather_into_tensor(self.gathered, self.local)
+        else:
+            self.h_local.copy_(self.local)
+            dist.all_gather_into_tensor(self.h_gathered, self.h_local)
+            self.gathered.copy_(self.h_gathered, non_blocking=True)
         self.G.best_combine(self.gathered, self.world, self.result)
         return self.result
 
