@@ -245,6 +245,41 @@ int grophecy_group_best(grophecy_space *space, const grophecy_pcie *pcie,
                         const grophecy_batch *batch, grophecy_group_result *device_out,
                         uint64_t capacity, uint64_t *n_groups, void *cuda_stream);
 
+/* Cross-batch fix-up of a group split between two consecutive batches (e.g.
+ * the last group of shard r and the first group of shard r + 1 when their
+ * boundary records share (skeleton, nx, ny, iters)): out = the group of both
+ * halves — first = a->first, count = a->count + b->count, the better
+ * (t, index) of the two bests with its bytes.  `a` must precede `b`.  out may
+ * alias a or b.  EINVAL on NULL or if a->first + a->count != b->first.  Pure
+ * host function. */
+int grophecy_group_merge_host(const grophecy_group_result *a, const grophecy_group_result *b,
+                              grophecy_group_result *out);
+
+/* Predicted speedup per group, S_g = t_cpu[g] / groups[g].best_t_s (P:L147:
+ * "the total CPU time divided by the total GPU time"), in DEVICE memory:
+ * groups (n entries), t_cpu (n doubles; the caller's CPU time of the group's
+ * projection point), out (n doubles).  Groups without a feasible candidate
+ * (best_t_s = +inf) give t_cpu / inf = 0.  Async, one launch. */
+int grophecy_group_speedup(const grophecy_group_result *groups, const double *t_cpu, uint64_t n,
+                           double *out, void *cuda_stream);
+
+/* Break-even iteration count per candidate (the
+ * iteration sweeps of P:L167, L215-239): with F = (t_once + t_h2d) + t_d2h
+ * (one-time GPU cost) and c = the CPU time of one iteration, the GPU run with
+ * `it` iterations, F + it * t_iter, beats the CPU run it * c iff
+ * it * (c - t_iter) > F, so
+ *     n_be      = F / (c - t_iter)        if c > t_iter, else +inf
+ *     iters_min = 1 if n_be < 1, floor(n_be) + 1 if finite, else UINT64_MAX
+ * (n_be in IEEE binary64 in that order; iters_min exact from n_be; NaN inputs
+ * — invalid records — give NaN / UINT64_MAX; iters_min saturates at
+ * UINT64_MAX for n_be >= 2^64).  Inputs: grophecy_eval_parts outputs (DEVICE,
+ * n each) and either t_cpu_iter (DEVICE, n doubles) or, if it is NULL, the
+ * scalar c for every candidate.  Outputs DEVICE n_be (may be NULL) and
+ * iters_min (may be NULL).  Async, one launch. */
+int grophecy_crossover(const double *t_iter, const double *t_once, const double *t_h2d,
+                       const double *t_d2h, const double *t_cpu_iter, double t_cpu_iter_scalar,
+                       uint64_t n, double *n_be, uint64_t *iters_min, void *cuda_stream);
+
 /* GPU speedup = total CPU time / total GPU time. */
 double grophecy_speedup(double t_cpu_s, double t_gpu_s);
 /* Error magnitude |predicted - measured| / measured (Table II applies

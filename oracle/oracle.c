@@ -497,3 +497,23 @@ double oracle_speedup_error(double s_pred, double s_meas)
 {
     return oracle_error_magnitude(s_pred, s_meas);
 }
+
+/* Break-even iteration count (oracle.h; N9), written as the
+ * definition. */
+void oracle_crossover(double t_iter, double t_once, double t_h2d, double t_d2h, double c,
+                      double *n_be, uint64_t *iters_min)
+{
+    double F = (t_once + t_h2d) + t_d2h;
+    double den = c - t_iter;
+    double v;
+    if (isnan(F) || isnan(den)) v = NAN;
+    else if (den > 0.0) v = F / den;
+    else v = INFINITY;
+    *n_be = v;
+    if (isnan(v) || v >= 18446744073709551616.0) {   /* also +inf */
+        *iters_min = UINT64_MAX;
+        return;
+    }
+    /* smallest integer it >= 1 with it > v: 1 if v < 1, else floor(v) + 1 */
+    *iters_min = v < 1.0 ? 1 : (uint64_t)floor(v) + 1;
+}

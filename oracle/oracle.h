@@ -124,6 +124,15 @@ double oracle_mean(const double *v, uint64_t n);
 double oracle_speedup(double t_cpu, double t_gpu);
 double oracle_speedup_error(double s_pred, double s_meas);
 
+/* Break-even iteration count (NEXT-2; "transfers once, kernels every
+ * iteration"; reading N9): the GPU run with `it` iterations costs
+ * F + it*t_iter with F = (t_once + t_h2d) + t_d2h, the CPU run it*c; the GPU
+ * wins iff it*(c - t_iter) > F.  *n_be = F/(c - t_iter) (c > t_iter) else
+ * +inf; *iters_min = smallest integer it >= 1 with it > *n_be (UINT64_MAX if
+ * none representable); NaN inputs give NaN / UINT64_MAX. */
+void oracle_crossover(double t_iter, double t_once, double t_h2d, double t_d2h, double c,
+                      double *n_be, uint64_t *iters_min);
+
 #ifdef __cplusplus
 }
 #endif

@@ -118,6 +118,8 @@ def lib():
         for name in ("oracle_error_magnitude", "oracle_speedup", "oracle_speedup_error"):
             getattr(L, name).argtypes = [C.c_double, C.c_double]
             getattr(L, name).restype = C.c_double
+        L.oracle_crossover.argtypes = [C.c_double] * 5 + [C.POINTER(C.c_double),
+                                                          C.POINTER(C.c_uint64)]
         L.oracle_mean.argtypes = [f64p, C.c_uint64]
         L.oracle_mean.restype = C.c_double
         _lib = L
@@ -274,3 +276,10 @@ def speedup(t_cpu, t_gpu):
 
 def speedup_error(s_pred, s_meas):
     return lib().oracle_speedup_error(s_pred, s_meas)
+
+
+def crossover(t_iter, t_once, t_h2d, t_d2h, c):
+    """(n_be, iters_min): break-even iteration count (oracle.h)."""
+    v, m = C.c_double(), C.c_uint64()
+    lib().oracle_crossover(t_iter, t_once, t_h2d, t_d2h, c, C.byref(v), C.byref(m))
+    return v.value, m.value

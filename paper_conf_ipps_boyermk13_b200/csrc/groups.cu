@@ -9,6 +9,8 @@
 //   3. group_scan:  exclusive scan of the block counts (one CTA) -> group ids;
 //   4. group_reduce: each head walks its run and writes the argmin
 //      (t, index) over valid finite records (ties: lowest index).
+// Also the other NEXT elementwise entry points: the predicted speedup per
+// group and the break-even iteration count (NEXT-2).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -137,9 +139,86 @@ __global__ void group_reduce(grophecy_batch B, const unsigned long long *offsets
     }
 }
 
+// S_g = t_cpu[g] / t_gpu[g]
+__global__ void speedup_kernel(const grophecy_group_result *g, const double *t_cpu,
+                               unsigned long long n, double *out)
+{
+    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+         i += (unsigned long long)gridDim.x * blockDim.x)
+        out[i] = __ddiv_rn(t_cpu[i], g[i].best_t_s);
+}
+
+// Break-even iteration count (include/grophecy.h grophecy_crossover)
+__global__ void crossover_kernel(const double *ti, const double *to, const double *th,
+                                 const double *td, const double *cv, double cs,
+                                 unsigned long long n, double *nbe, unsigned long long *imin)
+{
+    for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+         i += (unsigned long long)gridDim.x * blockDim.x) {
+        const double c = cv ? __ldcs(cv + i) : cs;
+        const double t_iter = __ldcs(ti + i);
+        const double F = __dadd_rn(__dadd_rn(__ldcs(to + i), __ldcs(th + i)), __ldcs(td + i));
+        const double den = __dsub_rn(c, t_iter);
+        double v;
+        if (isnan(F) || isnan(den)) v = __longlong_as_double(0x7ff8000000000000LL);
+        else v = den > 0.0 ? __ddiv_rn(F, den) : __longlong_as_double(0x7ff0000000000000LL);
+        unsigned long long m;
+        if (!(v < 18446744073709551616.0)) m = ~0ull;   // NaN, +inf, >= 2^64
+        else if (v < 1.0) m = 1ull;
+        else {
+            const unsigned long long f = (unsigned long long)floor(v);   // exact: v < 2^64
+            m = f == ~0ull ? ~0ull : f + 1ull;
+        }
+        if (nbe) __stcs(nbe + i, v);
+        if (imin) __stcs(imin + i, m);
+    }
+}
+
+unsigned elementwise_grid(unsigned long long n)
+{
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const unsigned long long want = (n + 255) / 256;
+    const unsigned long long cap = (unsigned long long)sms * 8;
+    return (unsigned)(want < cap ? (want ? want : 1) : cap);
+}
+
 }  // namespace grophecy
 
 using namespace grophecy;
+
+extern "C" int grophecy_group_speedup(const grophecy_group_result *groups, const double *t_cpu,
+                                      uint64_t n, double *out, void *stream)
+{
+    if (n && (!groups || !t_cpu || !out)) {
+        set_error("grophecy_group_speedup: null argument");
+        return GROPHECY_EINVAL;
+    }
+    if (!n) return GROPHECY_OK;
+    speedup_kernel<<<elementwise_grid(n), 256, 0, (cudaStream_t)stream>>>(groups, t_cpu, n, out);
+    count_launch();
+    const cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? GROPHECY_OK : cuda_fail(e, "grophecy_group_speedup");
+}
+
+extern "C" int grophecy_crossover(const double *t_iter, const double *t_once, const double *t_h2d,
+                                  const double *t_d2h, const double *t_cpu_iter,
+                                  double t_cpu_iter_scalar, uint64_t n, double *n_be,
+                                  uint64_t *iters_min, void *stream)
+{
+    if (n && (!t_iter || !t_once || !t_h2d || !t_d2h)) {
+        set_error("grophecy_crossover: null argument");
+        return GROPHECY_EINVAL;
+    }
+    if (!n || (!n_be && !iters_min)) return GROPHECY_OK;
+    crossover_kernel<<<elementwise_grid(n), 256, 0, (cudaStream_t)stream>>>(
+        t_iter, t_once, t_h2d, t_d2h, t_cpu_iter, t_cpu_iter_scalar, n, n_be,
+        (unsigned long long *)iters_min);
+    count_launch();
+    const cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? GROPHECY_OK : cuda_fail(e, "grophecy_crossover");
+}
 
 extern "C" int grophecy_group_best(grophecy_space *s, const grophecy_pcie *pc,
                                    const grophecy_batch *b, grophecy_group_result *device_out,

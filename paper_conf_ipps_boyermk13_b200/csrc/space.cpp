@@ -504,4 +504,26 @@ int grophecy_best_combine_host(const grophecy_best_result *in, uint32_t count,
     return GROPHECY_OK;
 }
 
+// One group split across two consecutive batches (NEXT-1 cross-shard fix-up).
+int grophecy_group_merge_host(const grophecy_group_result *a, const grophecy_group_result *b,
+                              grophecy_group_result *out)
+{
+    if (!a || !b || !out) return fail(GROPHECY_EINVAL, "null argument");
+    if (a->first + a->count != b->first)
+        return fail(GROPHECY_EINVAL, "group_merge: b does not follow a");
+    grophecy_group_result m = *a;
+    m.count = a->count + b->count;
+    // "none" has index UINT64_MAX and t = +inf, so it never wins
+    if (b->best_index != ~0ull &&
+        (a->best_index == ~0ull || b->best_t_s < a->best_t_s ||
+         (b->best_t_s == a->best_t_s && b->best_index < a->best_index))) {
+        m.best_t_s = b->best_t_s;
+        m.best_index = b->best_index;
+        m.h2d_bytes = b->h2d_bytes;
+        m.d2h_bytes = b->d2h_bytes;
+    }
+    *out = m;
+    return GROPHECY_OK;
+}
+
 }  // extern "C"

@@ -70,3 +70,79 @@ def minloc_host(local_result, group=None):
     dist.all_gather(out, t, group=group)
     res = [G.BestResult.from_buffer_copy(o.numpy().tobytes()) for o in out]
     return G.best_combine_host(res)
+
+
+# ---------------------------------------------------------------------------
+# Best transformation per group across shards ("cross-
+# shard groups need a neighbour fix-up").  A group (maximal run of equal
+# (skeleton, nx, ny, iters)) may straddle shard boundaries; the rank holding
+# its first record reports it, merged over every continuation, and the later
+# ranks drop their continuation pieces.  Only the boundary groups move: each
+# rank contributes (n, first key, last key, first group, last group, n_groups).
+def record_key(skx, nx, ny, iters):
+    """Group key of one record (skeleton, nx, ny, iters)."""
+    return (int(skx) >> 16, int(nx), int(ny), int(iters))
+
+
+def shard_group_fixups(infos):
+    """infos[r] = (n_records, first_key, last_key, first_group, last_group,
+    n_groups) of rank r in shard order (groups as GroupResult; keys None for
+    empty shards).  Returns per rank {"drop_first": bool, "last": GroupResult
+    or None (replacement of the rank's last group)}.  Pure host logic; the
+    merge itself is grophecy_group_merge_host."""
+    from . import grophecy as G
+    fix = [{"drop_first": False, "last": None} for _ in infos]
+    open_r, open_key, acc = None, None, None
+    for r, (n, fk, lk, fg, lg, ng) in enumerate(infos):
+        if n == 0 or ng == 0:
+            continue
+        if open_r is not None and fk == open_key:
+            acc = G.group_merge_host(acc, fg)
+            fix[r]["drop_first"] = True
+            fix[open_r]["last"] = acc
+            if ng == 1:
+                continue        # the whole shard continued the open group
+        open_r, open_key, acc = r, lk, lg
+    return fix
+
+
+def apply_group_fixup(groups, fix):
+    """Apply one rank's fix-up to its local list of GroupResult."""
+    groups = list(groups)
+    if fix["drop_first"]:
+        groups = groups[1:]
+    if fix["last"] is not None:
+        groups[-1] = fix["last"]
+    return groups
+
+
+def fix_shard_groups(groups, n, first_key, last_key, group=None):
+    """Collective (all ranks): exchange the boundary groups and return this
+    rank's fixed list.  `groups` = this shard's GroupResult list."""
+    from . import grophecy as G
+    ng = len(groups)
+    mine = (n, first_key, last_key, bytes(groups[0]) if ng else None,
+            bytes(groups[-1]) if ng else None, ng)
+    world = dist.get_world_size(group)
+    allinfo = [None] * world
+    dist.all_gather_object(allinfo, mine, group=group)
+    infos = []
+    for (nn, fk, lk, fg, lg, g) in allinfo:
+        infos.append((nn, fk, lk, G.GroupResult.from_buffer_copy(fg) if fg else None,
+                      G.GroupResult.from_buffer_copy(lg) if lg else None, g))
+    fix = shard_group_fixups(infos)
+    return apply_group_fixup(groups, fix[dist.get_rank(group)])
+
+
+def group_best_sharded(space, pc, rec, index_base, group=None):
+    """grophecy_group_best on this rank's shard (device records, global
+    index_base) plus the cross-shard fix-up.  Returns this rank's groups."""
+    rc, ng, groups = space.group_best(pc, rec, index_base=index_base)
+    n = rec.n
+    if n:
+        ends = [[int(getattr(rec, f)[i].item()) & 0xffffffff for f in ("skx", "nx", "ny", "iters")]
+                for i in (0, n - 1)]
+        fk, lk = record_key(*ends[0]), record_key(*ends[1])
+    else:
+        fk = lk = None
+    return fix_shard_groups(groups, n, fk, lk, group)

@@ -132,6 +132,11 @@ _sig = {
                                       C.POINTER(Parts), _vp]),
     "grophecy_group_best": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, C.c_uint64,
                                       C.POINTER(C.c_uint64), _vp]),
+    "grophecy_group_merge_host": (C.c_int, [C.POINTER(GroupResult), C.POINTER(GroupResult),
+                                            C.POINTER(GroupResult)]),
+    "grophecy_group_speedup": (C.c_int, [_vp, _vp, C.c_uint64, _vp, _vp]),
+    "grophecy_crossover": (C.c_int, [_vp, _vp, _vp, _vp, _vp, C.c_double, C.c_uint64, _vp, _vp,
+                                     _vp]),
     "grophecy_speedup": (C.c_double, [C.c_double, C.c_double]),
     "grophecy_error_magnitude": (C.c_double, [C.c_double, C.c_double]),
     "grophecy_best": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), C.POINTER(BestResult), _vp]),
@@ -454,6 +459,41 @@ def plan_stats(skel):
     st = (C.c_uint32 * 6)()
     rc = _L.grophecy_plan_stats(sd.arr, st)
     return rc, list(st)
+
+
+def group_merge_host(a, b):
+    """The group split across two consecutive batches, merged (a precedes b)."""
+    out = GroupResult()
+    _check(_L.grophecy_group_merge_host(C.byref(a), C.byref(b), C.byref(out)), "group_merge_host")
+    return out
+
+
+def group_speedup(groups, t_cpu, stream=None):
+    """Predicted speedup per group: groups = the int64 device tensor
+    of grophecy_group_best (6 words per group), t_cpu = float64 device tensor
+    (one CPU time per group).  Returns a float64 device tensor."""
+    torch = _torch()
+    n = t_cpu.numel()
+    out = torch.empty(n, dtype=torch.float64, device=t_cpu.device)
+    _check(_L.grophecy_group_speedup(_ptr(groups), _ptr(t_cpu), n, _ptr(out), _stream_ptr(stream)),
+           "group_speedup")
+    return out
+
+
+def crossover(t_iter, t_once, t_h2d, t_d2h, t_cpu_iter, stream=None):
+    """Break-even iteration counts (n_be float64, iters_min int64 holding
+    uint64 bits) from grophecy_eval_parts outputs; t_cpu_iter is a float64
+    device tensor (per candidate) or a Python float (every candidate)."""
+    torch = _torch()
+    n = t_iter.numel()
+    nbe = torch.empty(n, dtype=torch.float64, device=t_iter.device)
+    imin = torch.empty(n, dtype=torch.int64, device=t_iter.device)
+    vec = not isinstance(t_cpu_iter, (int, float))
+    _check(_L.grophecy_crossover(_ptr(t_iter), _ptr(t_once), _ptr(t_h2d), _ptr(t_d2h),
+                                 _ptr(t_cpu_iter) if vec else None,
+                                 0.0 if vec else float(t_cpu_iter), n, _ptr(nbe), _ptr(imin),
+                                 _stream_ptr(stream)), "crossover")
+    return nbe, imin
 
 
 def speedup(t_cpu, t_gpu):

@@ -174,3 +174,26 @@ def test_usage_plans_match_oracle_random_tiny(G, O):
         sizes += [(1 << 20, 1 << 20), (int(r.integers(1, 64)), 1 << 20)]
         tot += _check_plan(G, O, s, sizes)
     assert tot > 500
+
+
+def test_group_merge_host_rules():
+    from paper_conf_ipps_boyermk13_b200 import grophecy as G
+    NONE = 2**64 - 1
+    a = G.GroupResult(2.0, 10, 5, 12, 100, 50)
+    b = G.GroupResult(1.0, 15, 3, 16, 7, 8)
+    m = G.group_merge_host(a, b)
+    assert (m.best_t_s, m.first, m.count, m.best_index, m.h2d_bytes, m.d2h_bytes) == \
+        (1.0, 10, 8, 16, 7, 8)
+    # tie: the lower index (a's) wins
+    b2 = G.GroupResult(2.0, 15, 3, 16, 7, 8)
+    m = G.group_merge_host(a, b2)
+    assert (m.best_index, m.h2d_bytes) == (12, 100)
+    # "none" halves never win
+    na = G.GroupResult(float("inf"), 10, 5, NONE, 0, 0)
+    m = G.group_merge_host(na, b)
+    assert (m.best_index, m.count) == (16, 8)
+    m = G.group_merge_host(b, G.GroupResult(float("inf"), 18, 2, NONE, 0, 0))
+    assert (m.best_index, m.first, m.count) == (16, 15, 5)
+    # b must follow a
+    with pytest.raises(G.GrophecyError):
+        G.group_merge_host(a, G.GroupResult(1.0, 16, 3, 16, 7, 8))

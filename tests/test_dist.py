@@ -29,11 +29,19 @@ def _worker(rank, world, port, case, q):
         from oracle import oracle as O
         from paper_conf_ipps_boyermk13_b200 import dist as D
         from paper_conf_ipps_boyermk13_b200 import grophecy as G
-        skels, rec, n = case
+        skels, rec, n = case[:3]
         lo, hi = D.shard_range(n, rank, world)
         rc, link = O.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL)
         P = O.Problem(skels, S.FX5600, link)
         part = {k: v[lo:hi] for k, v in rec.items()}
+        if len(case) > 3 and case[3] == "groups":
+            groups = _oracle_groups(G, P, part, lo)
+            keys = [D.record_key(*[part[f][i] for f in ("skx", "nx", "ny", "iters")])
+                    for i in ((0, hi - lo - 1) if hi > lo else ())]
+            fixed = D.fix_shard_groups(groups, hi - lo, keys[0] if keys else None,
+                                       keys[-1] if keys else None)
+            q.put((rank, [_gtuple(g) for g in fixed]))
+            return
         _, ob = P.best(part, index_base=lo, nthreads=1)
         local = G.BestResult(ob.t_total_s, ob.index, ob.h2d_bytes, ob.d2h_bytes, ob.n_invalid,
                              ob.n_valid)
@@ -41,6 +49,17 @@ def _worker(rank, world, port, case, q):
         q.put((rank, out.as_tuple()))
     finally:
         dist.destroy_process_group()
+
+
+def _oracle_groups(G, P, rec, base):
+    """Per-shard groups from the oracle as GroupResult (bytes left 0)."""
+    f, cnt, bi, bt = P.group_best(rec, index_base=base)
+    return [G.GroupResult(float(bt[g]), int(f[g]), int(cnt[g]), int(bi[g]), 0, 0)
+            for g in range(len(f))]
+
+
+def _gtuple(g):
+    return (g.first, g.count, g.best_index, float(np.float64(g.best_t_s).view(np.uint64)))
 
 
 def _run(world, case):
@@ -114,3 +133,77 @@ def test_minloc_invalid_and_empty_shards(O):
     res = _run(2, case)
     want = _oracle_best(O, case)
     assert res[0] == res[1] == want and want[4] == 8
+
+
+def _group_case(n, seed, n_xf=16):
+    """Records with runs of 1..n/3 equal keys (some spanning several shards),
+    invalid runs and transformations out of order."""
+    rng = np.random.default_rng(seed)
+    skx, nx, ny, it = [], [], [], []
+    while len(skx) < n:
+        run = int(rng.integers(1, max(2, n // 3)))
+        s_, x_, y_, i_ = int(rng.integers(0, 3)), int(rng.integers(256, 4096)), 0, int(rng.integers(1, 50))
+        y_ = x_
+        if rng.random() < 0.1:
+            x_ = 0          # invalid run
+        for _ in range(run):
+            skx.append((s_ << 16) | int(rng.integers(0, n_xf)))
+            nx.append(x_)
+            ny.append(y_)
+            it.append(i_)
+    rec = {"skx": np.array(skx[:n], np.uint32), "nx": np.array(nx[:n], np.uint32),
+           "ny": np.array(ny[:n], np.uint32), "iters": np.array(it[:n], np.uint32)}
+    return rec
+
+
+def _full_groups(O, skels, rec):
+    rc, link = O.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL)
+    P = O.Problem(skels, S.FX5600, link)
+    f, cnt, bi, bt = P.group_best(rec)
+    return [(int(f[g]), int(cnt[g]), int(bi[g]), float(np.float64(bt[g]).view(np.uint64)))
+            for g in range(len(f))]
+
+
+def test_shard_group_fixups_pure(O):
+    """Every split of a record set into 1..6 contiguous shards: per-shard
+    groups + fix-up == the groups of the whole set (NEXT-1 cross-shard)."""
+    from paper_conf_ipps_boyermk13_b200 import dist as D
+    from paper_conf_ipps_boyermk13_b200 import grophecy as G
+    skels = R.config("c2")["skeletons"]
+    rc, link = O.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL)
+    P = O.Problem(skels, S.FX5600, link)
+    for seed in range(12):
+        n = 40 + 7 * seed
+        rec = _group_case(n, seed)
+        want = _full_groups(O, skels, rec)
+        rng = np.random.default_rng(100 + seed)
+        for world in (1, 2, 3, 4, 6):
+            cuts = sorted(rng.integers(0, n + 1, world - 1).tolist())   # empty shards allowed
+            bounds = [0] + cuts + [n]
+            infos, locals_ = [], []
+            for r in range(world):
+                lo, hi = bounds[r], bounds[r + 1]
+                part = {k: v[lo:hi] for k, v in rec.items()}
+                gs = _oracle_groups(G, P, part, lo) if hi > lo else []
+                keys = [D.record_key(*[part[f][i] for f in ("skx", "nx", "ny", "iters")])
+                        for i in ((0, hi - lo - 1) if hi > lo else ())]
+                infos.append((hi - lo, keys[0] if keys else None, keys[-1] if keys else None,
+                              gs[0] if gs else None, gs[-1] if gs else None, len(gs)))
+                locals_.append(gs)
+            fix = D.shard_group_fixups(infos)
+            got = []
+            for r in range(world):
+                got += [_gtuple(g) for g in D.apply_group_fixup(locals_[r], fix[r])]
+            assert got == want, (seed, world, bounds)
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_group_fixup_over_gloo(O, world):
+    skels = R.config("c2")["skeletons"]
+    rec = _group_case(45, 7)
+    want = _full_groups(O, skels, rec)
+    res = _run(world, (skels, rec, 45, "groups"))
+    got = []
+    for r in range(world):
+        got += res[r]
+    assert got == want

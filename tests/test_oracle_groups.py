@@ -104,3 +104,44 @@ def test_product_speedup_helpers_match_oracle(O):
         assert G.error_magnitude(a, b) == O.error_magnitude(a, b)
     # Table II, Stassuij
     assert round(100 * G.error_magnitude(1.10, 0.39)) == 182
+
+
+def _exact_first_win(ti, to, th, td, c, limit=10**6):
+    """Brute force over integer iteration counts in exact rational arithmetic:
+    the smallest it >= 1 with F + it * t_iter < it * c (GPU strictly faster)."""
+    from fractions import Fraction as Fr
+    F = Fr(to) + Fr(th) + Fr(td)
+    for it in range(1, limit):
+        if F + it * Fr(ti) < it * Fr(c):
+            return it
+    return None
+
+
+def test_crossover_closed_form_and_brute_force(O):
+    """NEXT-2 break-even iteration count: a hand case, then dyadic inputs
+    (every sum and the quotient exact) against a brute-force scan of the
+    definition in exact arithmetic."""
+    # F = (1 + 0.5) + 0.5 = 2, c - t_iter = 1: break-even at 2 iterations,
+    # GPU strictly faster from 3 on
+    assert O.crossover(1.0, 1.0, 0.5, 0.5, 2.0) == (2.0, 3)
+    # GPU never wins
+    assert O.crossover(2.0, 1.0, 0.0, 0.0, 2.0) == (math.inf, 2**64 - 1)
+    assert O.crossover(3.0, 0.0, 0.0, 0.0, 2.0) == (math.inf, 2**64 - 1)
+    # no one-time cost: the first iteration already wins
+    assert O.crossover(1.0, 0.0, 0.0, 0.0, 2.0) == (0.0, 1)
+    # invalid (NaN) inputs
+    v, m = O.crossover(math.nan, 1.0, 1.0, 1.0, 2.0)
+    assert math.isnan(v) and m == 2**64 - 1
+    rng = np.random.default_rng(5)
+    for _ in range(400):
+        ti = int(rng.integers(0, 64)) / 64.0
+        to, th, td = (int(rng.integers(0, 4096)) / 64.0 for _ in range(3))
+        c = ti + 2.0 ** -int(rng.integers(0, 6))          # c - t_iter a power of two: exact quotient
+        v, m = O.crossover(ti, to, th, td, c)
+        want = _exact_first_win(ti, to, th, td, c)
+        assert m == want, (ti, to, th, td, c, v)
+    # huge break-even counts saturate instead of wrapping
+    v, m = O.crossover(0.0, 2.0 ** 70, 0.0, 0.0, 1.0)
+    assert v == 2.0 ** 70 and m == 2**64 - 1
+    v, m = O.crossover(0.0, 2.0 ** 60, 0.0, 0.0, 1.0)
+    assert m == 2**60 + 1
