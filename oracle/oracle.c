@@ -66,6 +66,39 @@ static void region_box(const or_region *g, int64_t R, int64_t C, int64_t nx, int
     *c1 = imin64(imax64(oracle_affine8(&g->c1, nx, ny), 0), C);
 }
 
+/* Strides of a region (whole regions are dense). */
+static int64_t row_step(const or_region *g) { return (!g->whole && g->r_step > 1) ? g->r_step : 1; }
+static int64_t col_step(const or_region *g) { return (!g->whole && g->c_step > 1) ? g->c_step : 1; }
+
+/* Lattice anchors: the unclamped lower bounds (the section's l). */
+static int64_t row_anchor(const or_region *g, int64_t nx, int64_t ny)
+{
+    return g->whole ? 0 : oracle_affine8(&g->r0, nx, ny);
+}
+static int64_t col_anchor(const or_region *g, int64_t nx, int64_t ny)
+{
+    return g->whole ? 0 : oracle_affine8(&g->c0, nx, ny);
+}
+
+/* x mod m in [0, m) */
+static int64_t pmod(int64_t x, int64_t m) { return ((x % m) + m) % m; }
+
+/* Effective access mode: an irregular ("may") write needs the original data
+ * on the GPU and returns the whole array, i.e. it reads and writes every
+ * element (reading 10). */
+static uint32_t eff_mode(const or_region *g)
+{
+    return (g->whole && (g->mode & 2u)) ? (g->mode | 1u) : g->mode;
+}
+
+static int64_t gcd64(int64_t a, int64_t b)
+{
+    if (a < 0) a = -a;
+    if (b < 0) b = -b;
+    while (b) { int64_t t = a % b; a = b; b = t; }
+    return a;
+}
+
 static int cmp_i64(const void *a, const void *b)
 {
     int64_t x = *(const int64_t *)a, y = *(const int64_t *)b;
@@ -81,6 +114,13 @@ static int sort_unique(int64_t *v, int n)
     return m;
 }
 
+/* #{ r in [a, b) : r mod L == rho } */
+static int64_t count_residue(int64_t a, int64_t b, int64_t rho, int64_t L)
+{
+    int64_t first = a + pmod(rho - a, L);
+    return first < b ? (b - 1 - first) / L + 1 : 0;
+}
+
 /*
  * For every element e of array a:  fr(e) = first kernel reading e,
  * fw(e) = first kernel writing e (program order).
@@ -90,50 +130,74 @@ static int sort_unique(int64_t *v, int n)
  *   D2H_a = [live-out] * elem_bytes * |{e : fw(e) < inf}|
  *           ("union of all written BRSs", minus temporaries)
  * Cell method: the row/column breakpoints of all boxes cut the array into
- * cells that every box either contains or misses; fr/fw are constant per cell.
+ * slabs that every box either contains or misses; with strides, rows of a
+ * slab are further split by their residue modulo L = lcm of the row strides
+ * (a region with stride s covers row r of a slab it contains iff
+ * (r - l) mod s == 0, which depends on r mod L only).  fr / fw are constant
+ * per (row slab, row residue) x (column slab, column residue) cell.
  */
 void oracle_usage(const or_skeleton *s, int64_t nx, int64_t ny,
                   uint64_t *h2d_per_array, uint64_t *d2h_per_array)
 {
+    if (s->hull) {
+        oracle_usage_hull(s, nx, ny, h2d_per_array, d2h_per_array);
+        return;
+    }
     int nreg = (int)s->n_regions;
     int64_t *rb = (int64_t *)malloc(sizeof(int64_t) * (size_t)(2 * nreg + 2));
     int64_t *cb = (int64_t *)malloc(sizeof(int64_t) * (size_t)(2 * nreg + 2));
-    int64_t *box = (int64_t *)malloc(sizeof(int64_t) * (size_t)(4 * nreg + 4));
+    int64_t *box = (int64_t *)malloc(sizeof(int64_t) * (size_t)(6 * nreg + 6));
     for (uint32_t a = 0; a < s->n_arrays; a++) {
         const or_array *A = &s->arrays[a];
         int64_t R = imax64(0, oracle_affine8(&A->rows, nx, ny));
         int64_t C = imax64(0, oracle_affine8(&A->cols, nx, ny));
         int nr = 0, nc = 0;
+        int64_t Lr = 1, Lc = 1;
         rb[nr++] = 0; rb[nr++] = R;
         cb[nc++] = 0; cb[nc++] = C;
         for (int j = 0; j < nreg; j++) {
             const or_region *g = &s->regions[j];
             if (g->array != a) continue;
-            region_box(g, R, C, nx, ny, &box[4 * j], &box[4 * j + 1], &box[4 * j + 2], &box[4 * j + 3]);
-            rb[nr++] = box[4 * j]; rb[nr++] = box[4 * j + 1];
-            cb[nc++] = box[4 * j + 2]; cb[nc++] = box[4 * j + 3];
+            int64_t *b = &box[6 * j];
+            region_box(g, R, C, nx, ny, &b[0], &b[1], &b[2], &b[3]);
+            b[4] = row_anchor(g, nx, ny);
+            b[5] = col_anchor(g, nx, ny);
+            rb[nr++] = b[0]; rb[nr++] = b[1];
+            cb[nc++] = b[2]; cb[nc++] = b[3];
+            Lr = Lr / gcd64(Lr, row_step(g)) * row_step(g);
+            Lc = Lc / gcd64(Lc, col_step(g)) * col_step(g);
         }
         nr = sort_unique(rb, nr);
         nc = sort_unique(cb, nc);
         uint64_t h = 0, d = 0;
-        for (int i = 0; i + 1 < nr; i++) {
-            for (int jj = 0; jj + 1 < nc; jj++) {
-                int64_t y0 = rb[i], y1 = rb[i + 1], x0 = cb[jj], x1 = cb[jj + 1];
-                int fr = OR_INF_K, fw = OR_INF_K;
-                for (int j = 0; j < nreg; j++) {
-                    const or_region *g = &s->regions[j];
-                    if (g->array != a) continue;
-                    const int64_t *b = &box[4 * j];
-                    if (b[0] <= y0 && y1 <= b[1] && b[2] <= x0 && x1 <= b[3]) {
-                        if ((g->mode & 1u) && (int)g->kernel < fr) fr = (int)g->kernel;
-                        if ((g->mode & 2u) && (int)g->kernel < fw) fw = (int)g->kernel;
+        for (int i = 0; i + 1 < nr; i++)
+            for (int64_t rho = 0; rho < Lr; rho++) {
+                int64_t y0 = rb[i], y1 = rb[i + 1];
+                int64_t hgt = count_residue(y0, y1, rho, Lr);
+                if (hgt == 0) continue;
+                for (int jj = 0; jj + 1 < nc; jj++)
+                    for (int64_t sig = 0; sig < Lc; sig++) {
+                        int64_t x0 = cb[jj], x1 = cb[jj + 1];
+                        int64_t wid = count_residue(x0, x1, sig, Lc);
+                        if (wid == 0) continue;
+                        int fr = OR_INF_K, fw = OR_INF_K;
+                        for (int j = 0; j < nreg; j++) {
+                            const or_region *g = &s->regions[j];
+                            if (g->array != a) continue;
+                            const int64_t *b = &box[6 * j];
+                            if (b[0] <= y0 && y1 <= b[1] && b[2] <= x0 && x1 <= b[3] &&
+                                pmod(rho - b[4], row_step(g)) == 0 &&
+                                pmod(sig - b[5], col_step(g)) == 0) {
+                                uint32_t m = eff_mode(g);
+                                if ((m & 1u) && (int)g->kernel < fr) fr = (int)g->kernel;
+                                if ((m & 2u) && (int)g->kernel < fw) fw = (int)g->kernel;
+                            }
+                        }
+                        uint64_t area = (uint64_t)hgt * (uint64_t)wid;
+                        if (fr != OR_INF_K && fr <= fw) h += area;
+                        if (fw != OR_INF_K) d += area;
                     }
-                }
-                uint64_t area = (uint64_t)(y1 - y0) * (uint64_t)(x1 - x0);
-                if (fr != OR_INF_K && fr <= fw) h += area;
-                if (fw != OR_INF_K) d += area;
             }
-        }
         h2d_per_array[a] = h * A->elem_bytes;
         d2h_per_array[a] = A->liveout ? d * A->elem_bytes : 0;
     }
@@ -158,9 +222,12 @@ int oracle_bitmap_usage(const or_skeleton *s, int64_t nx, int64_t ny,
                     if (g->array != a) continue;
                     int64_t r0, r1, c0, c1;
                     region_box(g, R, C, nx, ny, &r0, &r1, &c0, &c1);
-                    if (r0 <= r && r < r1 && c0 <= c && c < c1) {
-                        if ((g->mode & 1u) && (int)g->kernel < fr) fr = (int)g->kernel;
-                        if ((g->mode & 2u) && (int)g->kernel < fw) fw = (int)g->kernel;
+                    if (r0 <= r && r < r1 && c0 <= c && c < c1 &&
+                        pmod(r - row_anchor(g, nx, ny), row_step(g)) == 0 &&
+                        pmod(c - col_anchor(g, nx, ny), col_step(g)) == 0) {
+                        uint32_t m = eff_mode(g);
+                        if ((m & 1u) && (int)g->kernel < fr) fr = (int)g->kernel;
+                        if ((m & 2u) && (int)g->kernel < fw) fw = (int)g->kernel;
                     }
                 }
                 if (fr != OR_INF_K && fr <= fw) h += 1;
@@ -171,6 +238,134 @@ int oracle_bitmap_usage(const or_skeleton *s, int64_t nx, int64_t ny,
         d2h_per_array[a] = A->liveout ? d * A->elem_bytes : 0;
     }
     return 0;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Approximate mode: BRS lists with the Havlak-Kennedy UNION ([5]; */
+/* SURVEY §8(f) NEXT-3; N4h).                                      */
+/* ------------------------------------------------------------------------ */
+
+/* One dimension of a section: {l, l+s, ..., u}; s == 0 iff l == u; empty iff l > u. */
+typedef struct { int64_t l, u, s; } or_sec1;
+/* A 2-D section (rows x columns); empty iff either dimension is. */
+typedef struct { or_sec1 r, c; } or_sec;
+
+static int sec1_empty(or_sec1 a) { return a.l > a.u; }
+
+/* The elements of the lattice anchor + i*step inside [lo, hi). */
+static or_sec1 sec1_make(int64_t lo, int64_t hi, int64_t anchor, int64_t step)
+{
+    or_sec1 v = {1, 0, 0};
+    int64_t first = lo + pmod(anchor - lo, step);
+    if (first >= hi) return v;
+    v.l = first;
+    v.u = first + ((hi - 1 - first) / step) * step;
+    v.s = v.l == v.u ? 0 : step;
+    return v;
+}
+
+/* HK UNION: [min l : max u : gcd(s_a, s_b, |l_a - l_b|)] */
+static or_sec1 sec1_union(or_sec1 a, or_sec1 b)
+{
+    if (sec1_empty(a)) return b;
+    if (sec1_empty(b)) return a;
+    or_sec1 v;
+    v.l = imin64(a.l, b.l);
+    v.u = imax64(a.u, b.u);
+    v.s = gcd64(gcd64(a.s, b.s), a.l - b.l);
+    if (v.l == v.u) v.s = 0;
+    return v;
+}
+
+/* every element of x is an element of w */
+static int sec1_contains(or_sec1 w, or_sec1 x)
+{
+    if (sec1_empty(x)) return 1;
+    if (sec1_empty(w)) return 0;
+    if (w.s == 0) return x.l == w.l && x.u == w.l;
+    return x.l >= w.l && x.u <= w.u && pmod(x.l - w.l, w.s) == 0 && x.s % w.s == 0;
+}
+
+static uint64_t sec1_count(or_sec1 a)
+{
+    if (sec1_empty(a)) return 0;
+    return a.s == 0 ? 1 : (uint64_t)((a.u - a.l) / a.s) + 1;
+}
+
+static int sec_empty(or_sec x) { return sec1_empty(x.r) || sec1_empty(x.c); }
+
+static or_sec sec_union(or_sec a, or_sec b)
+{
+    if (sec_empty(a)) return b;
+    if (sec_empty(b)) return a;
+    or_sec v = {sec1_union(a.r, b.r), sec1_union(a.c, b.c)};
+    return v;
+}
+
+static int sec_contains(or_sec w, or_sec x)
+{
+    if (sec_empty(x)) return 1;
+    if (sec_empty(w)) return 0;
+    return sec1_contains(w.r, x.r) && sec1_contains(w.c, x.c);
+}
+
+static uint64_t sec_count(or_sec a)
+{
+    return sec_empty(a) ? 0 : sec1_count(a.r) * sec1_count(a.c);
+}
+
+static or_sec region_sec(const or_region *g, int64_t R, int64_t C, int64_t nx, int64_t ny)
+{
+    int64_t r0, r1, c0, c1;
+    region_box(g, R, C, nx, ny, &r0, &r1, &c0, &c1);
+    or_sec v = {sec1_make(r0, r1, row_anchor(g, nx, ny), row_step(g)),
+                sec1_make(c0, c1, col_anchor(g, nx, ny), col_step(g))};
+    return v;
+}
+
+/*
+ * Per array, kernels in program order: "we maintain a list of
+ * BRSs that are read but are not previously written" — a read section of
+ * kernel k is dropped when ONE write section of a kernel < k contains it
+ * (reads see the state before the kernel's own writes, reading 7);
+ * "the UNION of all such BRSs is data that needs to be transferred to the
+ * GPU.  The UNION of all written BRSs is data that needs to be transferred
+ * back" — UNION = Havlak-Kennedy hull.  Bytes = elements of the hull.
+ */
+void oracle_usage_hull(const or_skeleton *s, int64_t nx, int64_t ny,
+                       uint64_t *h2d_per_array, uint64_t *d2h_per_array)
+{
+    or_sec *wl = (or_sec *)malloc(sizeof(or_sec) * (size_t)(s->n_regions + 1));
+    for (uint32_t a = 0; a < s->n_arrays; a++) {
+        const or_array *A = &s->arrays[a];
+        int64_t R = imax64(0, oracle_affine8(&A->rows, nx, ny));
+        int64_t C = imax64(0, oracle_affine8(&A->cols, nx, ny));
+        or_sec hr = {{1, 0, 0}, {1, 0, 0}}, hw = {{1, 0, 0}, {1, 0, 0}};
+        int nw = 0;                                   /* writes of kernels < k */
+        for (uint32_t k = 0; k < s->n_kernels; k++) {
+            for (uint32_t j = 0; j < s->n_regions; j++) {   /* reads of kernel k */
+                const or_region *g = &s->regions[j];
+                if (g->array != a || g->kernel != k || !(eff_mode(g) & 1u)) continue;
+                or_sec x = region_sec(g, R, C, nx, ny);
+                if (sec_empty(x)) continue;
+                int written = 0;
+                for (int q = 0; q < nw; q++)
+                    if (sec_contains(wl[q], x)) written = 1;
+                if (!written) hr = sec_union(hr, x);
+            }
+            for (uint32_t j = 0; j < s->n_regions; j++) {   /* then its writes */
+                const or_region *g = &s->regions[j];
+                if (g->array != a || g->kernel != k || !(eff_mode(g) & 2u)) continue;
+                or_sec x = region_sec(g, R, C, nx, ny);
+                if (sec_empty(x)) continue;
+                wl[nw++] = x;
+                hw = sec_union(hw, x);
+            }
+        }
+        h2d_per_array[a] = sec_count(hr) * A->elem_bytes;
+        d2h_per_array[a] = A->liveout ? sec_count(hw) * A->elem_bytes : 0;
+    }
+    free(wl);
 }
 
 /* ------------------------------------------------------------------------ */

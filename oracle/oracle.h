@@ -37,8 +37,17 @@ extern "C" {
 typedef struct { int32_t c0, c1, c2, c3; } or_affine8;   /* c0 + floor((c1 nx + c2 ny + c3 nx ny)/8) */
 
 typedef struct { or_affine8 rows, cols; uint32_t elem_bytes, liveout; } or_array;
-/* mode: bit0 = read, bit1 = write.  whole != 0: the region is the whole array. */
-typedef struct { uint32_t kernel, array, mode, whole; or_affine8 r0, r1, c0, c1; } or_region;
+/* mode: bit0 = read, bit1 = write.  whole != 0: irregular access, the whole
+ * array may be referenced; an irregular write is a "may-write" and
+ * counts as read + write of the whole array (reading 10).
+ * r_step / c_step: the strides of the bounded regular section [l:u:s]
+ * ([5]); 0 or 1 = dense.  A strided region covers rows r0 + i*r_step
+ * inside the clamped box (the lattice is anchored at the unclamped r0). */
+typedef struct {
+    uint32_t kernel, array, mode, whole;
+    or_affine8 r0, r1, c0, c1;
+    uint32_t r_step, c_step;
+} or_region;
 typedef struct { or_affine8 work; uint32_t per_iter; } or_kernel;
 typedef struct {
     uint32_t tpb, ipt, regs, smem;
@@ -50,6 +59,7 @@ typedef struct {
     const or_array *arrays;
     const or_region *regions;
     const or_kx *kx;               /* [n_xforms][n_kernels] */
+    uint32_t hull;                 /* 1: Havlak-Kennedy approximate UNION (N4h) */
 } or_skeleton;
 typedef struct {
     uint32_t n_sm, warp_size, max_tpb, max_bps, max_tps, regs_sm, smem_sm;
@@ -68,6 +78,12 @@ void oracle_usage(const or_skeleton *s, int64_t nx, int64_t ny,
                   uint64_t *h2d_per_array, uint64_t *d2h_per_array);
 int  oracle_bitmap_usage(const or_skeleton *s, int64_t nx, int64_t ny,
                          uint64_t *h2d_per_array, uint64_t *d2h_per_array);
+/* The approximate mode: BRS lists merged with the
+ * Havlak-Kennedy UNION (per dimension [min l : max u : gcd]); a read is
+ * "previously written" when one earlier write section contains it.
+ * oracle_usage dispatches here when s->hull != 0. */
+void oracle_usage_hull(const or_skeleton *s, int64_t nx, int64_t ny,
+                       uint64_t *h2d_per_array, uint64_t *d2h_per_array);
 
 /* Kernel-time projection (GROPHECY [15] / Hong & Kim [6] reading). */
 double oracle_kernel_time(const or_skeleton *s, const or_gpu *g, uint32_t xform,

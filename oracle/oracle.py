@@ -38,7 +38,7 @@ class Array(C.Structure):
 class Region(C.Structure):
     _fields_ = [("kernel", C.c_uint32), ("array", C.c_uint32), ("mode", C.c_uint32),
                 ("whole", C.c_uint32), ("r0", Affine8), ("r1", Affine8), ("c0", Affine8),
-                ("c1", Affine8)]
+                ("c1", Affine8), ("r_step", C.c_uint32), ("c_step", C.c_uint32)]
 
 
 class Kernel(C.Structure):
@@ -56,7 +56,7 @@ class Skeleton(C.Structure):
     _fields_ = [("n_kernels", C.c_uint32), ("n_arrays", C.c_uint32),
                 ("n_regions", C.c_uint32), ("n_xforms", C.c_uint32),
                 ("kernels", C.POINTER(Kernel)), ("arrays", C.POINTER(Array)),
-                ("regions", C.POINTER(Region)), ("kx", C.POINTER(KX))]
+                ("regions", C.POINTER(Region)), ("kx", C.POINTER(KX)), ("hull", C.c_uint32)]
 
 
 class GPU(C.Structure):
@@ -95,6 +95,7 @@ def lib():
         L.oracle_affine8.restype = C.c_int64
         L.oracle_usage.argtypes = [SK, C.c_int64, C.c_int64, u64p, u64p]
         L.oracle_bitmap_usage.argtypes = [SK, C.c_int64, C.c_int64, u64p, u64p]
+        L.oracle_usage_hull.argtypes = [SK, C.c_int64, C.c_int64, u64p, u64p]
         L.oracle_kernel_time.argtypes = [SK, C.POINTER(GPU), C.c_uint32, C.c_uint32,
                                          C.c_int64, C.c_int64, C.POINTER(C.c_int)]
         L.oracle_kernel_time.restype = C.c_double
@@ -147,7 +148,8 @@ class SkeletonSet:
                                                for a in s["arrays"]])
             rs = (Region * max(1, len(s["regions"])))(*[
                 Region(r["kernel"], r["array"], _MODES[r["mode"]], int(r["whole"]),
-                       _a8(r["r0"]), _a8(r["r1"]), _a8(r["c0"]), _a8(r["c1"]))
+                       _a8(r["r0"]), _a8(r["r1"]), _a8(r["c0"]), _a8(r["c1"]),
+                       int(r.get("r_step", 1)), int(r.get("c_step", 1)))
                 for r in s["regions"]])
             flat = [c for row in s["kx"] for c in row]
             kx = (KX * len(flat))(*[KX(c["tpb"], c["ipt"], c["regs"], c["smem"], c["total"],
@@ -155,7 +157,7 @@ class SkeletonSet:
                                     for c in flat])
             self._keep += [ks, ars, rs, kx]
             self.arr[i] = Skeleton(len(s["kernels"]), len(s["arrays"]), len(s["regions"]),
-                                   len(s["kx"]), ks, ars, rs, kx)
+                                   len(s["kx"]), ks, ars, rs, kx, int(bool(s.get("hull", False))))
         self.n = len(skels)
 
     def ptr(self, i=0):

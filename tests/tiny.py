@@ -15,7 +15,10 @@ def _a8_const(v):
     return (int(v), 0, 0, 0)
 
 
-def random_tiny_skeleton(rng, n_xforms=1, max_kernels=8, max_arrays=3, max_regions=12):
+def random_tiny_skeleton(rng, n_xforms=1, max_kernels=8, max_arrays=3, max_regions=12,
+                         strided=False, maywrite=False, hull=False):
+    """strided: BRS strides in {1, 2, 3, 4, 6} per dimension (lcm <= 12);
+    maywrite: irregular (WHOLE) writes too; hull: the approximate-UNION mode."""
     nx = int(rng.integers(1, 13))
     ny = int(rng.integers(1, 13))
     n_arr = int(rng.integers(1, max_arrays + 1))
@@ -38,7 +41,7 @@ def random_tiny_skeleton(rng, n_xforms=1, max_kernels=8, max_arrays=3, max_regio
     for _ in range(int(rng.integers(0, max_regions + 1))):
         a = int(rng.integers(0, n_arr))
         mode = ["R", "W", "RW"][int(rng.integers(0, 3))]
-        whole = mode == "R" and rng.random() < 0.15
+        whole = (mode == "R" or maywrite) and rng.random() < 0.15
 
         def bound():
             # mix constants and size-scaled terms, some negative / too large
@@ -47,12 +50,18 @@ def random_tiny_skeleton(rng, n_xforms=1, max_kernels=8, max_arrays=3, max_regio
             c2 = int(rng.integers(-4, 9)) if rng.random() < 0.5 else 0
             return (c0, c1, c2, 0)
 
-        regions.append({"kernel": int(rng.integers(0, K)), "array": a, "mode": mode,
-                        "whole": bool(whole), "r0": bound(), "r1": bound(),
-                        "c0": bound(), "c1": bound()})
+        reg = {"kernel": int(rng.integers(0, K)), "array": a, "mode": mode,
+               "whole": bool(whole), "r0": bound(), "r1": bound(),
+               "c0": bound(), "c1": bound()}
+        if strided:
+            reg["r_step"] = int(rng.choice([1, 1, 2, 3, 4, 6]))
+            reg["c_step"] = int(rng.choice([1, 1, 2, 3, 4, 6]))
+        regions.append(reg)
     kx = [[DUMMY_KX] * K] * n_xforms
-    return {"name": "tiny", "arrays": arrays, "kernels": kernels, "regions": regions,
-            "kx": kx}, nx, ny
+    sk = {"name": "tiny", "arrays": arrays, "kernels": kernels, "regions": regions, "kx": kx}
+    if hull:
+        sk["hull"] = True
+    return sk, nx, ny
 
 
 def rng(seed):
