@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define GROPHECY_ABI_VERSION 1
+#define GROPHECY_ABI_VERSION 2
 
 typedef enum {
     GROPHECY_OK = 0,
@@ -79,19 +79,28 @@ typedef struct { int32_t c0, c1, c2, c3; } grophecy_affine8;
 enum { GROPHECY_ARRAY_LIVEOUT = 1u };   /* written data goes back to the CPU;
                                            clear = "temporary" hint */
 enum { GROPHECY_R = 1u, GROPHECY_W = 2u };   /* region mode bits; R|W = read-modify-write */
-enum { GROPHECY_REGION_WHOLE = 1u };    /* irregular read: the whole array may be
-                                           referenced; only with mode == R */
+enum { GROPHECY_REGION_WHOLE = 1u };    /* irregular access: the whole array may be
+                                           referenced.  With W in the mode it
+                                           is a "may-write": the kernel may write any
+                                           element, so it counts as a whole-array read
+                                           + write (reading 10) */
 enum { GROPHECY_KERNEL_PER_ITER = 1u }; /* runs every iteration; else once */
 
 /* A 2-D array of rows x cols elements (row-major), extents clamped at 0. */
 typedef struct { grophecy_affine8 rows, cols; uint32_t elem_bytes, flags; } grophecy_array_desc;
 
-/* A bounded regular section: the box [r0, r1) x [c0, c1) of `array`
- * accessed by `kernel` (program order index).  Bounds are clamped to the
- * array; lo >= hi is empty. */
+/* A bounded regular section (Havlak-Kennedy [5]) of `array` accessed
+ * by `kernel` (program order index): rows r0, r0 + r_step, ... and columns
+ * c0, c0 + c_step, ... inside the box [r0, r1) x [c0, c1) clamped to the
+ * array (the lattice stays anchored at the unclamped r0 / c0; lo >= hi is
+ * empty).  r_step / c_step: 0 or 1 = dense, else <= GROPHECY_MAX_STEP and the
+ * least common multiple of one array's row (column) steps must be
+ * <= GROPHECY_MAX_STEP_LCM.  WHOLE regions ignore the box and the steps.
+ * 72 bytes. */
 typedef struct {
     uint8_t kernel, array, mode, flags;
     grophecy_affine8 r0, r1, c0, c1;
+    uint16_t r_step, c_step;
 } grophecy_region_desc;
 
 typedef struct { grophecy_affine8 work_items; uint32_t flags; } grophecy_kernel_desc;
@@ -108,14 +117,25 @@ typedef struct {
         synch_insts;
 } grophecy_kx_desc;
 
+/* Skeleton flags.  HULL: data usage by the approximate BRS algebra instead of
+ * exact element sets — per array, a read section is "previously written"
+ * when one write section of an earlier kernel contains it, and the UNIONs of
+ * the remaining read sections (-> H2D) and of all write sections (-> D2H) are
+ * Havlak-Kennedy hulls [min l : max u : gcd] per dimension ([5];
+ * DESIGN.md N4h).  Never smaller than the exact counts; equal for
+ * whole-array workloads. */
+enum { GROPHECY_SKEL_HULL = 1u };
+
 /* One code skeleton: a kernel sequence, its arrays and access regions, and
- * the characteristics table kx[x * n_kernels + k] for n_xforms transformations. */
+ * the characteristics table kx[x * n_kernels + k] for n_xforms
+ * transformations; flags: GROPHECY_SKEL_*; reserved must be 0. */
 typedef struct {
     uint32_t n_kernels, n_arrays, n_regions, n_xforms;
     const grophecy_kernel_desc *kernels;
     const grophecy_array_desc *arrays;
     const grophecy_region_desc *regions;
     const grophecy_kx_desc *kx;
+    uint32_t flags, reserved;
 } grophecy_skeleton_desc;
 
 /* The modelled GPU ("configured to reflect different GPU architectures"). */
@@ -129,7 +149,8 @@ typedef struct {
  *   1 <= n_skels <= 65536; 1 <= n_xforms <= 65536; 1 <= n_kernels <= 32;
  *   n_arrays <= 16; n_regions <= 256; <= 32 regions per array;
  *   region.kernel < n_kernels, region.array < n_arrays, mode in {R, W, R|W},
- *   REGION_WHOLE only with mode R (irregular writes: DESIGN.md reading 10);
+ *   region steps <= 64, lcm of one array's row (column) steps <= 64;
+ *   skeleton flags within GROPHECY_SKEL_HULL;
  *   1 <= tpb <= 65536, 1 <= ipt <= 65536; instruction counts finite, >= 0,
  *   total >= coal + uncoal, uncoal_per_mw >= 1, load_bytes_per_warp > 0;
  *   GPU integers >= 1 and GPU doubles finite and > 0; elem_bytes >= 1. */
@@ -140,6 +161,8 @@ typedef struct {
 #define GROPHECY_MAX_REGIONS 256u
 #define GROPHECY_MAX_REGIONS_PER_ARRAY 32u
 #define GROPHECY_MAX_DIM (1u << 20)
+#define GROPHECY_MAX_STEP 64u
+#define GROPHECY_MAX_STEP_LCM 64u
 
 /* Pure host validation of a design space (no CUDA). */
 int grophecy_space_validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,

@@ -43,7 +43,7 @@ struct SkelInfo {
     uint32_t k_base;   // into kern_work / kern_flags
     uint32_t a_base;   // into arrays
     uint32_t kx_base;  // into kx tables
-    uint32_t pad;
+    uint32_t flags;    // GROPHECY_SKEL_* (HULL) | SKF_STRIDED
     // usage plan (plan.cpp): valid for nx >= plan_tx and ny >= plan_ty
     uint32_t plan_tx, plan_ty, expr_base, n_expr;
     // flat term list of all arrays / directions: {packed indices, 2*array + dir}
@@ -53,8 +53,10 @@ struct SkelInfo {
 struct ArrayDev {
     int4 rows, cols;
     uint32_t elem_bytes, liveout, r_base, r_count;   // regions [r_base, r_base+r_count)
-    uint32_t h_prog, d_prog, pad0, pad1;             // plan band programs (u32 word offsets)
+    uint32_t h_prog, d_prog;                         // plan band programs (u32 word offsets)
+    uint32_t lr, lc;    // lcm of the regions' row / column steps (1 = dense array)
 };
+enum : uint32_t { SKF_STRIDED = 1u << 16 };   // some region has a step > 1
 
 constexpr uint32_t PLAN_MAX_EXPR = 128;   // < 256: programs pack u8 indices
 
@@ -70,9 +72,12 @@ struct SkelPlanHost {
 // Regions are stored grouped by array and sorted by kernel within an array,
 // so "first writer" = lowest set bit of a mask and upto = mask of regions of
 // the same array whose kernel <= this region's kernel.
+// mode is the effective mode: an irregular (WHOLE) write is a may-write and
+// carries R as well (reading 10).  rs / cs: steps (1 = dense).
 struct RegionDev {
     int4 r0, r1, c0, c1;
     uint32_t mode, whole, upto, kernel;
+    uint32_t rs, cs, pad0, pad1;
 };
 
 struct SpaceDev {
@@ -101,6 +106,7 @@ struct SpaceDev {
 struct grophecy_space {
     int device;
     grophecy::SpaceDev dev;
+    grophecy::SpaceDev *dev_copy;        // the same struct in device memory (rare paths)
     void *blob;                          // one device allocation for all tables
     size_t blob_bytes;
     grophecy_best_result *partials;      // best-mode per-block partials

@@ -18,8 +18,8 @@
 // v - u >= 0 on D; the left side is bilinear in (nx, ny), hence its minimum
 // over the box D is at a corner.
 //
-// Keys outside the domain (or skeletons without a plan) take the general
-// cooperative sweep on the device.
+// Keys outside the domain (or skeletons without a plan: strided sections,
+// the approximate hull mode) take the general cooperative paths on the device.
 #include <algorithm>
 #include <cstdint>
 #include <vector>
@@ -129,6 +129,7 @@ bool compile_array(const grophecy_array_desc &A, const std::vector<const grophec
         b.kernel = g->kernel;
         b.mode = g->mode;
         if (g->flags & GROPHECY_REGION_WHOLE) {
+            if (g->mode & GROPHECY_W) b.mode |= GROPHECY_R;   // may-write (reading 10)
             b.r0 = ZERO; b.r1 = R; b.c0 = ZERO; b.c1 = C;
         } else {
             if (!clamp_sym(ex_of(g->r0), R, D, b.r0) || !clamp_sym(ex_of(g->r1), R, D, b.r1) ||
@@ -210,6 +211,12 @@ void emit(const std::vector<std::vector<uint8_t>> &cell, const std::vector<Ex> &
 bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out)
 {
     out = SkelPlanHost();
+    // the approximate (hull) mode and strided sections take the general path
+    if (S.flags & GROPHECY_SKEL_HULL) return false;
+    for (uint32_t j = 0; j < S.n_regions; j++)
+        if (!(S.regions[j].flags & GROPHECY_REGION_WHOLE) &&
+            (S.regions[j].r_step > 1 || S.regions[j].c_step > 1))
+            return false;
     std::vector<std::vector<const grophecy_region_desc *>> regs(S.n_arrays);
     for (uint32_t j = 0; j < S.n_regions; j++) regs[S.regions[j].array].push_back(&S.regions[j]);
 

@@ -80,8 +80,12 @@ struct SweepScratch {
     long long box[32][4];
     long long rs_h[64];
     long long cs_w[64];
+    long long rs_a[64];         // slab starts (strided arrays)
+    long long cs_a[64];
     unsigned rs_m[64];
     unsigned cs_m[64];
+    unsigned pr_m[64];          // strided arrays: regions whose row lattice hits residue rho
+    unsigned pc_m[64];
     unsigned upto[32];
 };
 
@@ -208,11 +212,83 @@ __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsig
     }
 }
 
+__device__ __forceinline__ uint32_t sat_u32(long long w)
+{
+    return w <= 0 ? 0u : (w >= 0xffffffffLL ? 0xffffffffu : (uint32_t)w);
+}
+
+// x mod m in [0, m) for m >= 1
+__device__ __forceinline__ long long pmodll(long long x, long long m)
+{
+    const long long r = x % m;
+    return r < 0 ? r + m : r;
+}
+
+// #{ r in [a, a + len) : r mod L == rho }, a >= 0, 0 <= rho < L
+__device__ __forceinline__ unsigned long long count_residue(long long a, long long len, unsigned rho,
+                                                           unsigned L)
+{
+    if (L == 1) return (unsigned long long)len;
+    const long long first = a + pmodll((long long)rho - a, L);
+    const long long b = a + len;
+    return first < b ? (unsigned long long)((b - 1 - first) / L) + 1ull : 0ull;
+}
+
+// Strided arrays (BRS [l:u:s]): the slabs of the sweep
+// are split by row residue rho mod Lr and column residue sigma mod Lc (Lr, Lc
+// = lcm of the array's steps); a region covers a (slab, residue) unit iff it
+// covers the slab and its lattice hits the residue: (rho - l) mod step == 0.
+// The first-reader / first-writer rule per cell is the dense sweep's.
+__device__ __forceinline__ void strided_cells(SweepScratch &ws, unsigned Lr, unsigned Lc, int Sr, int Sc, int n,
+                              long long ar, long long ac, unsigned rs, unsigned cs, unsigned Rm,
+                              unsigned Wm, int lane, unsigned long long &h, unsigned long long &d)
+{
+    // residue masks: lanes over residues, regions' phases by shuffle
+    const unsigned pr = (unsigned)pmodll(ar, rs), pcp = (unsigned)pmodll(ac, cs);
+    for (unsigned rho0 = 0; rho0 < 64; rho0 += 32) {
+        const unsigned rho = rho0 + lane;
+        unsigned mr = 0, mc = 0;
+        for (int q = 0; q < n; q++) {
+            const unsigned sq = __shfl_sync(FULL, rs, q), phq = __shfl_sync(FULL, pr, q);
+            const unsigned tq = __shfl_sync(FULL, cs, q), pcq = __shfl_sync(FULL, pcp, q);
+            if (rho < Lr && (rho + sq - phq) % sq == 0) mr |= 1u << q;
+            if (rho < Lc && (rho + tq - pcq) % tq == 0) mc |= 1u << q;
+        }
+        if (rho < Lr) ws.pr_m[rho] = mr;
+        if (rho < Lc) ws.pc_m[rho] = mc;
+    }
+    __syncwarp();
+    const int Uc = Sc * (int)Lc;
+    for (int i = 0; i < Sr; i++) {
+        const unsigned sm = ws.rs_m[i];
+        if (!sm) continue;
+        const long long ra = ws.rs_a[i], rh = ws.rs_h[i];
+        for (unsigned rho = 0; rho < Lr; rho++) {
+            const unsigned rm = sm & ws.pr_m[rho];
+            if (!rm) continue;
+            const unsigned long long hg = count_residue(ra, rh, rho, Lr);
+            if (!hg) continue;
+            for (int u = lane; u < Uc; u += 32) {
+                const int j = u / (int)Lc;
+                const unsigned sig = (unsigned)(u - j * (int)Lc);
+                const unsigned m = rm & ws.cs_m[j] & ws.pc_m[sig];
+                if (m) {
+                    const unsigned long long area =
+                        hg * count_residue(ws.cs_a[j], ws.cs_w[j], sig, Lc);
+                    const unsigned mr = m & Rm, mw = m & Wm;
+                    if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) h += area;
+                    if (mw) d += area;
+                }
+            }
+        }
+    }
+}
+
 // Data usage of one (skeleton, nx, ny) key by the general coordinate-compressed
 // sweep over the whole warp (DESIGN.md §3 N4; §III-B), plus
 // the per-array PCIe transfer times in array order.  Used for keys outside
 // their skeleton's plan domain.
-__device__ Usage warp_usage_sweep(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
+__device__ __forceinline__ Usage warp_usage_sweep(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
                                   const grophecy_pcie &pc, WarpScratch &wsu, int lane)
 {
     SweepScratch &ws = wsu.sw;
@@ -228,28 +304,35 @@ __device__ Usage warp_usage_sweep(const SpaceDev &S, const SkelInfo &I, long lon
         unsigned long long h = 0, d = 0;
         if (n > 0 && R > 0 && C > 0) {
             long long r0 = 0, r1 = 0, c0 = 0, c1 = 0;
+            long long ar = 0, ac = 0;          // lattice anchors (unclamped lower bounds)
             bool valid = false;
-            unsigned mode = 0, up = 0;
+            unsigned mode = 0, up = 0, rs = 1, cs = 1;
             if (lane < n) {
                 const RegionDev &g = S.regions[A.r_base + lane];
                 if (g.whole) {
                     r1 = R;
                     c1 = C;
                 } else {
-                    r0 = clampll(aff8(g.r0, nx, ny), R);
+                    ar = aff8(g.r0, nx, ny);
+                    ac = aff8(g.c0, nx, ny);
+                    r0 = clampll(ar, R);
                     r1 = clampll(aff8(g.r1, nx, ny), R);
-                    c0 = clampll(aff8(g.c0, nx, ny), C);
+                    c0 = clampll(ac, C);
                     c1 = clampll(aff8(g.c1, nx, ny), C);
                 }
                 valid = r0 < r1 && c0 < c1;
                 mode = g.mode;
                 up = g.upto;
+                rs = g.rs;
+                cs = g.cs;
             }
+            const bool strided = A.lr > 1 || A.lc > 1;
             const unsigned vm = __ballot_sync(FULL, valid);
             const unsigned Rm = __ballot_sync(FULL, valid && (mode & GROPHECY_R));
             const unsigned Wm = __ballot_sync(FULL, valid && (mode & GROPHECY_W));
             if (vm) {
-                const bool full = valid && r0 == 0 && r1 == R && c0 == 0 && c1 == C;
+                const bool full = valid && r0 == 0 && r1 == R && c0 == 0 && c1 == C && rs == 1 &&
+                                  cs == 1;
                 const unsigned fm = __ballot_sync(FULL, full);
                 if (fm == vm) {
                     // every access covers the whole array: one cell
@@ -307,25 +390,32 @@ __device__ Usage warp_usage_sweep(const SpaceDev &S, const SkelInfo &I, long lon
                         int p = __popc(br0 & lt);
                         ws.rs_h[p] = rn0 - r0;
                         ws.rs_m[p] = rm0;
+                        ws.rs_a[p] = r0;
                     }
                     if (sr1) {
                         int p = __popc(br0) + __popc(br1 & lt);
                         ws.rs_h[p] = rn1 - r1;
                         ws.rs_m[p] = rm1;
+                        ws.rs_a[p] = r1;
                     }
                     if (sc0) {
                         int p = __popc(bc0 & lt);
                         ws.cs_w[p] = cn0 - c0;
                         ws.cs_m[p] = cm0;
+                        ws.cs_a[p] = c0;
                     }
                     if (sc1) {
                         int p = __popc(bc0) + __popc(bc1 & lt);
                         ws.cs_w[p] = cn1 - c1;
                         ws.cs_m[p] = cm1;
+                        ws.cs_a[p] = c1;
                     }
                     __syncwarp();
                     const int Sr = __popc(br0) + __popc(br1);
                     const int Sc = __popc(bc0) + __popc(bc1);
+                    if (strided) {
+                        strided_cells(ws, A.lr, A.lc, Sr, Sc, n, ar, ac, rs, cs, Rm, Wm, lane, h, d);
+                    } else
                     for (int i = 0; i < Sr; i++) {
                         const unsigned rm = ws.rs_m[i];
                         if (!rm) continue;
@@ -349,6 +439,146 @@ __device__ Usage warp_usage_sweep(const SpaceDev &S, const SkelInfo &I, long lon
         add_array(o, A, h, d, pc);
     }
     return o;
+}
+
+// ---- approximate mode: BRS algebra with the Havlak-Kennedy UNION ----------
+// ([5]; N4h).  One dimension of a
+// section {l, l+s, ..., u}: s == 0 iff one element, empty iff l > u.
+struct Sec1 {
+    long long l, u, s;
+};
+
+__device__ __forceinline__ bool sec1_empty(const Sec1 &a) { return a.l > a.u; }
+
+__device__ __forceinline__ long long gcdll(long long a, long long b)
+{
+    a = a < 0 ? -a : a;
+    b = b < 0 ? -b : b;
+    while (b) {
+        const long long t = a % b;
+        a = b;
+        b = t;
+    }
+    return a;
+}
+
+// lattice anchor + i*step inside [lo, hi)
+__device__ __forceinline__ Sec1 sec1_make(long long lo, long long hi, long long anchor, long long step)
+{
+    Sec1 v = {1, 0, 0};
+    const long long first = lo + pmodll(anchor - lo, step);
+    if (first >= hi) return v;
+    v.l = first;
+    v.u = first + ((hi - 1 - first) / step) * step;
+    v.s = v.l == v.u ? 0 : step;
+    return v;
+}
+
+__device__ __forceinline__ Sec1 sec1_union(const Sec1 &a, const Sec1 &b)
+{
+    if (sec1_empty(a)) return b;
+    if (sec1_empty(b)) return a;
+    Sec1 v;
+    v.l = a.l < b.l ? a.l : b.l;
+    v.u = a.u > b.u ? a.u : b.u;
+    v.s = gcdll(gcdll(a.s, b.s), a.l - b.l);
+    if (v.l == v.u) v.s = 0;
+    return v;
+}
+
+// every element of x (non-empty) is one of w (non-empty)
+__device__ __forceinline__ bool sec1_contains(const Sec1 &w, const Sec1 &x)
+{
+    if (w.s == 0) return x.l == w.l && x.u == w.l;
+    return x.l >= w.l && x.u <= w.u && pmodll(x.l - w.l, w.s) == 0 && x.s % w.s == 0;
+}
+
+__device__ __forceinline__ unsigned long long sec1_count(const Sec1 &a)
+{
+    if (sec1_empty(a)) return 0ull;
+    return a.s == 0 ? 1ull : (unsigned long long)((a.u - a.l) / a.s) + 1ull;
+}
+
+// One dimension (rows: dim 0, columns: dim 1) of a region's section.
+__device__ __forceinline__ Sec1 region_sec1(const RegionDev &g, int dim, long long nx, long long ny,
+                                            long long E)
+{
+    if (g.whole) return sec1_make(0, E, 0, 1);
+    const int4 lo = dim ? g.c0 : g.r0, hi = dim ? g.c1 : g.r1;
+    const long long an = aff8(lo, nx, ny);
+    return sec1_make(clampll(an, E), clampll(aff8(hi, nx, ny), E), an, dim ? g.cs : g.rs);
+}
+
+// Usage of one key in the approximate mode: lane a works on array a.  Its
+// regions are sorted by kernel, so the write sections of earlier kernels are
+// the write regions before the first region of the current kernel.  Pass 1
+// marks the kept reads (not inside one earlier write section, both
+// dimensions); the hulls are then built one dimension at a time (the HK
+// UNION works per dimension), which keeps the live state small.
+__device__ __forceinline__ Usage warp_usage_hull(const SpaceDev &S, const SkelInfo &I, long long nx,
+                                                 long long ny, const grophecy_pcie &pc, int lane)
+{
+    unsigned long long h = 0, d = 0;
+    if ((uint32_t)lane < I.n_arrays) {
+        const ArrayDev &A = S.arrays[I.a_base + lane];
+        long long E[2] = {aff8(A.rows, nx, ny), aff8(A.cols, nx, ny)};
+        E[0] = E[0] > 0 ? E[0] : 0;
+        E[1] = E[1] > 0 ? E[1] : 0;
+        const RegionDev *G = S.regions + A.r_base;
+        const uint32_t n = A.r_count;
+        uint32_t nonempty = 0, keep = 0, wmask = 0;
+        for (uint32_t j = 0; j < n; j++) {
+            const Sec1 xr = region_sec1(G[j], 0, nx, ny, E[0]);
+            const Sec1 xc = region_sec1(G[j], 1, nx, ny, E[1]);
+            if (sec1_empty(xr) || sec1_empty(xc)) continue;
+            nonempty |= 1u << j;
+            if (G[j].mode & GROPHECY_W) wmask |= 1u << j;
+            if (!(G[j].mode & GROPHECY_R)) continue;
+            bool written = false;
+            for (uint32_t q = 0; q < j && !written; q++) {
+                if (!((wmask >> q) & 1u) || G[q].kernel >= G[j].kernel) continue;
+                written = sec1_contains(region_sec1(G[q], 0, nx, ny, E[0]), xr) &&
+                          sec1_contains(region_sec1(G[q], 1, nx, ny, E[1]), xc);
+            }
+            if (!written) keep |= 1u << j;
+        }
+        unsigned long long cr = 1, cw = 1;
+        for (int dim = 0; dim < 2; dim++) {
+            Sec1 hr = {1, 0, 0}, hw = {1, 0, 0};
+            for (uint32_t j = 0; j < n; j++) {
+                if (!((nonempty >> j) & 1u)) continue;
+                const Sec1 x = region_sec1(G[j], dim, nx, ny, E[dim]);
+                if ((keep >> j) & 1u) hr = sec1_union(hr, x);
+                if ((wmask >> j) & 1u) hw = sec1_union(hw, x);
+            }
+            cr *= sec1_count(hr);
+            cw *= sec1_count(hw);
+        }
+        h = keep ? cr : 0ull;
+        d = wmask ? cw : 0ull;
+    }
+    Usage o = {0ull, 0ull, 0.0, 0.0};
+    for (uint32_t a = 0; a < I.n_arrays; a++) {   // transfer times in array order
+        const unsigned long long ha = __shfl_sync(FULL, h, a), da = __shfl_sync(FULL, d, a);
+        add_array(o, S.arrays[I.a_base + a], ha, da, pc);
+    }
+    return o;
+}
+
+// Usage of one key off the plan path (outside the plan's domain, strided
+// sections, the hull mode) and its kernels' work counts, by the whole warp.
+__device__ __forceinline__ void slow_usage(const SpaceDev *gS, unsigned long long k, grophecy_pcie pc,
+                                        WarpScratch *scr, Usage *res, uint32_t *w_out, int lane)
+{
+    const SpaceDev &S = *gS;
+    const SkelInfo &I = S.skel[(uint32_t)(k >> 42)];
+    const long long kx_ = (long long)((k >> 21) & 0x1fffffull);
+    const long long ky_ = (long long)(k & 0x1fffffull);
+    const Usage r = (I.flags & GROPHECY_SKEL_HULL) ? warp_usage_hull(S, I, kx_, ky_, pc, lane)
+                                                   : warp_usage_sweep(S, I, kx_, ky_, pc, *scr, lane);
+    if (lane == 0) *res = r;
+    if ((uint32_t)lane < I.n_kernels)
+        w_out[lane] = sat_u32(aff8(__ldg(&S.kern_work[I.k_base + lane]), kx_, ky_));
 }
 
 // Kernel time of one kernel (DESIGN.md §3 N5) from its work-item count Wi and
@@ -603,13 +833,10 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
     }
 }
 
-__device__ __forceinline__ uint32_t sat_u32(long long w)
-{
-    return w <= 0 ? 0u : (w >= 0xffffffffLL ? 0xffffffffu : (uint32_t)w);
-}
 
 struct Params {
     SpaceDev S;
+    const SpaceDev *gS;   // device copy of S (out-of-line paths)
     grophecy_pcie pc;
     const uint32_t *skx, *nx, *ny, *iters;
     unsigned long long n, base;
@@ -783,14 +1010,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                 while (sweep) {
                     const int pos = __ffs(sweep) - 1;
                     const unsigned long long k = __shfl_sync(FULL, mk, pos);
-                    const SkelInfo &I = S.skel[(uint32_t)(k >> 42)];
-                    const long long kx_ = (long long)((k >> 21) & 0x1fffffull);
-                    const long long ky_ = (long long)(k & 0x1fffffull);
-                    const Usage r = warp_usage_sweep(S, I, kx_, ky_, P.pc, ws.scratch, lane);
-                    if (lane == 0) ws.res[g0 - c0 + pos] = r;
-                    if ((uint32_t)lane < I.n_kernels)
-                        ws.slot_w[g0 - c0 + pos][lane] =
-                            sat_u32(aff8(__ldg(&S.kern_work[I.k_base + lane]), kx_, ky_));
+                    slow_usage(P.gS, k, P.pc, &ws.scratch, &ws.res[g0 - c0 + pos],
+                               ws.slot_w[g0 - c0 + pos], lane);
                     sweep &= sweep - 1;
                     __syncwarp();
                 }
@@ -848,19 +1069,20 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             } else {
                 // the lane's best of its (index-ordered) records, then one compare
                 double bt = __longlong_as_double(0x7ff0000000000000LL);
-                int bj = -1;
+                int bj = -1, bls = 0;
 #pragma unroll
                 for (int j = 0; j < RPT; j++)
                     if (inj[j] && tt[j] < bt) {
                         bt = tt[j];
                         bj = j;
+                        bls = ls[j];
                     }
                 if (bj >= 0) {
                     const unsigned long long i = P.base + tb + lane + 32 * bj;
                     if (better(bt, i, best_t, best_i)) {
                         best_t = bt;
                         best_i = i;
-                        const Usage &u = ws.res[ls[bj]];
+                        const Usage &u = ws.res[bls];
                         ws.best_h[lane] = u.h;
                         ws.best_d[lane] = u.d;
                     }
@@ -998,6 +1220,7 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
 {
     Params P;
     P.S = s->dev;
+    P.gS = s->dev_copy;
     P.pc = *pc;
     P.skx = b->skx;
     P.nx = b->nx;

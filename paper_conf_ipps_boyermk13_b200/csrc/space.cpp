@@ -48,6 +48,15 @@ static bool coef_ok(const grophecy_affine8 &a)
     return a.c1 >= -L && a.c1 <= L && a.c2 >= -L && a.c2 <= L && a.c3 >= -L && a.c3 <= L;
 }
 
+// lcm(l, step) with step 0 / 1 = dense
+static uint64_t lcm_step(uint64_t l, uint32_t step)
+{
+    const uint64_t s = step > 1 ? step : 1;
+    uint64_t a = l, b = s;
+    while (b) { const uint64_t t = a % b; a = b; b = t; }
+    return l / a * s;
+}
+
 static int validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                     const grophecy_gpu_model *g)
 {
@@ -91,12 +100,26 @@ static int validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 return fail(GROPHECY_EINVAL, std::string(where) + "region kernel/array index out of range");
             if (r.mode < 1 || r.mode > 3)
                 return fail(GROPHECY_EINVAL, std::string(where) + "region mode must be R, W or R|W");
-            if ((r.flags & GROPHECY_REGION_WHOLE) && r.mode != GROPHECY_R)
-                return fail(GROPHECY_EINVAL, std::string(where) + "irregular (WHOLE) regions must be read-only");
+            if (r.r_step > GROPHECY_MAX_STEP || r.c_step > GROPHECY_MAX_STEP)
+                return fail(GROPHECY_ELIMIT, std::string(where) + "region step > 64");
             if (!coef_ok(r.r0) || !coef_ok(r.r1) || !coef_ok(r.c0) || !coef_ok(r.c1))
                 return fail(GROPHECY_ELIMIT, std::string(where) + "region coefficient out of range");
             if (++per_array[r.array] > GROPHECY_MAX_REGIONS_PER_ARRAY)
                 return fail(GROPHECY_ELIMIT, std::string(where) + "more than 32 regions on one array");
+        }
+        if (S.flags & ~(uint32_t)GROPHECY_SKEL_HULL)
+            return fail(GROPHECY_EINVAL, std::string(where) + "unknown skeleton flags");
+        if (S.reserved) return fail(GROPHECY_EINVAL, std::string(where) + "reserved must be 0");
+        for (uint32_t a = 0; a < S.n_arrays; a++) {
+            uint64_t lr = 1, lc = 1;
+            for (uint32_t j = 0; j < S.n_regions; j++) {
+                const grophecy_region_desc &r = S.regions[j];
+                if (r.array != a || (r.flags & GROPHECY_REGION_WHOLE)) continue;
+                lr = lcm_step(lr, r.r_step);
+                lc = lcm_step(lc, r.c_step);
+            }
+            if (lr > GROPHECY_MAX_STEP_LCM || lc > GROPHECY_MAX_STEP_LCM)
+                return fail(GROPHECY_ELIMIT, std::string(where) + "lcm of an array's steps > 64");
         }
         for (uint64_t i = 0; i < (uint64_t)S.n_xforms * S.n_kernels; i++) {
             const grophecy_kx_desc &c = S.kx[i];
@@ -269,7 +292,11 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         I.k_base = (uint32_t)kwork.size();
         I.a_base = (uint32_t)arrays.size();
         I.kx_base = (uint32_t)kes.size();
-        I.pad = 0;
+        I.flags = S.flags & GROPHECY_SKEL_HULL;
+        for (uint32_t j = 0; j < S.n_regions; j++)
+            if (!(S.regions[j].flags & GROPHECY_REGION_WHOLE) &&
+                (S.regions[j].r_step > 1 || S.regions[j].c_step > 1))
+                I.flags |= SKF_STRIDED;
         SkelPlanHost plan;
         if (compile_plan(S, plan)) {
             I.plan_tx = plan.tx;
@@ -308,7 +335,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             A.r_base = (uint32_t)regions.size();
             A.h_prog = plan.ok ? prog_base + plan.h_off[a] : 0;
             A.d_prog = plan.ok ? prog_base + plan.d_off[a] : 0;
-            A.pad0 = A.pad1 = 0;
+            A.lr = A.lc = 1;
             // regions of this array, stably sorted by kernel (order within a
             // kernel is irrelevant: usage does not depend on region order)
             std::vector<const grophecy_region_desc *> rs;
@@ -323,8 +350,15 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 RegionDev R;
                 R.r0 = a4(rs[j]->r0); R.r1 = a4(rs[j]->r1);
                 R.c0 = a4(rs[j]->c0); R.c1 = a4(rs[j]->c1);
-                R.mode = rs[j]->mode;
                 R.whole = (rs[j]->flags & GROPHECY_REGION_WHOLE) ? 1u : 0u;
+                // an irregular write may write any element: whole read + write
+                R.mode = (R.whole && (rs[j]->mode & GROPHECY_W)) ? (rs[j]->mode | GROPHECY_R)
+                                                                  : rs[j]->mode;
+                R.rs = (!R.whole && rs[j]->r_step > 1) ? rs[j]->r_step : 1u;
+                R.cs = (!R.whole && rs[j]->c_step > 1) ? rs[j]->c_step : 1u;
+                R.pad0 = R.pad1 = 0;
+                A.lr = (uint32_t)lcm_step(A.lr, R.rs);
+                A.lc = (uint32_t)lcm_step(A.lc, R.cs);
                 R.kernel = rs[j]->kernel;
                 uint32_t upto = 0;
                 for (size_t q = 0; q < rs.size(); q++)
@@ -403,7 +437,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     sp->max_partials = (uint32_t)nsm * 32u;
     size_t scratch_off = align_up(total, 256);
     size_t part_bytes = sizeof(grophecy_best_result) * sp->max_partials;
-    size_t blob = scratch_off + align_up(part_bytes, 256) + 256;
+    size_t blob = scratch_off + align_up(part_bytes, 256) + 256 + align_up(sizeof(SpaceDev), 256);
     if ((e = cudaMalloc(&sp->blob, blob)) != cudaSuccess) return bail(e, "cudaMalloc(space)");
     sp->blob_bytes = blob;
     if ((e = cudaMemcpy(sp->blob, host.data(), total, cudaMemcpyHostToDevice)) != cudaSuccess)
@@ -435,6 +469,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.freq = gpu->freq_hz;
     D.rfreq = 1.0 / gpu->freq_hz;
     D.invalid_counter = sp->invalid_counter;
+    sp->dev_copy = (SpaceDev *)(ctr + 256);
+    if ((e = cudaMemcpy(sp->dev_copy, &D, sizeof D, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return bail(e, "cudaMemcpy(space header)");
     sp->grid_best = nsm;
     sp->grid_eval = nsm;
     cudaSetDevice(prev);

@@ -23,6 +23,7 @@ OK, EINVAL, ELIMIT, ECUDA, ENOFEASIBLE, EBADCAND = 0, -1, -2, -3, -5, -6
 ARRAY_LIVEOUT = 1
 R, W = 1, 2
 REGION_WHOLE = 1
+SKEL_HULL = 1
 KERNEL_PER_ITER = 1
 DIR_H2D, DIR_D2H = 0, 1
 UINT64_MAX = 2**64 - 1
@@ -55,7 +56,7 @@ class ArrayDesc(C.Structure):
 class RegionDesc(C.Structure):
     _fields_ = [("kernel", C.c_uint8), ("array", C.c_uint8), ("mode", C.c_uint8),
                 ("flags", C.c_uint8), ("r0", Affine8), ("r1", Affine8), ("c0", Affine8),
-                ("c1", Affine8)]
+                ("c1", Affine8), ("r_step", C.c_uint16), ("c_step", C.c_uint16)]
 
 
 class KernelDesc(C.Structure):
@@ -74,7 +75,7 @@ class SkeletonDesc(C.Structure):
     _fields_ = [("n_kernels", C.c_uint32), ("n_arrays", C.c_uint32), ("n_regions", C.c_uint32),
                 ("n_xforms", C.c_uint32), ("kernels", C.POINTER(KernelDesc)),
                 ("arrays", C.POINTER(ArrayDesc)), ("regions", C.POINTER(RegionDesc)),
-                ("kx", C.POINTER(KxDesc))]
+                ("kx", C.POINTER(KxDesc)), ("flags", C.c_uint32), ("reserved", C.c_uint32)]
 
 
 class GpuModel(C.Structure):
@@ -100,7 +101,8 @@ class BestResult(C.Structure):
                 self.n_valid)
 
 
-assert C.sizeof(BestResult) == 48 and C.sizeof(RegionDesc) == 68 and C.sizeof(KxDesc) == 64
+assert C.sizeof(BestResult) == 48 and C.sizeof(RegionDesc) == 72 and C.sizeof(KxDesc) == 64
+assert C.sizeof(SkeletonDesc) == 56
 
 
 class Parts(C.Structure):
@@ -217,14 +219,16 @@ class Skeletons:
             rs = (RegionDesc * max(1, len(s["regions"])))(*[
                 RegionDesc(r["kernel"], r["array"], _MODES[r["mode"]],
                            REGION_WHOLE if r["whole"] else 0, _a8(r["r0"]), _a8(r["r1"]),
-                           _a8(r["c0"]), _a8(r["c1"])) for r in s["regions"]])
+                           _a8(r["c0"]), _a8(r["c1"]), int(r.get("r_step", 1)),
+                           int(r.get("c_step", 1))) for r in s["regions"]])
             flat = [c for row in s["kx"] for c in row]
             kx = (KxDesc * len(flat))(*[
                 KxDesc(c["tpb"], c["ipt"], c["regs"], c["smem"], c["total"], c["coal"],
                        c["uncoal"], c["upm"], c["lbpw"], c["synch"]) for c in flat])
             self.keep += [ks, ars, rs, kx]
             self.arr[i] = SkeletonDesc(len(s["kernels"]), len(s["arrays"]), len(s["regions"]),
-                                       len(s["kx"]), ks, ars, rs, kx)
+                                       len(s["kx"]), ks, ars, rs, kx,
+                                       SKEL_HULL if s.get("hull", False) else 0, 0)
         self.n = len(skels)
 
 

@@ -97,6 +97,13 @@ def config(name):
                 rules.append(make_rule(SQUARE, 256, 8192))
         return {"name": "c4", "skeletons": skels, "rules": rules, "n": 10**9,
                 "n_xforms": 16, "seed": 0x5EED0004}
+    if name in ("c3s", "c3h"):
+        # NEXT-3 workloads (not BASELINE configs): C3's shape with strided
+        # sections and irregular writes; "c3h" in the approximate hull mode
+        skels = sk.random_skeletons(0x5EED0033, 64, brs=True, hull=name == "c3h")
+        rules = [make_rule(INDEP, 256, 8192)] * 64
+        return {"name": name, "skeletons": skels, "rules": rules, "n": 10**7,
+                "n_xforms": 16, "seed": 0x5EED0033}
     raise ValueError(name)
 
 

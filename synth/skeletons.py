@@ -221,7 +221,12 @@ LIBRARY = [s0_stencil2, s1_hotspot, s2_hotspot_pp2, s3_srad, s4_cfd, s5_vecadd, 
 
 
 # ---- Generator R: random multi-kernel skeletons (C3/C4) -----------------------
-def random_skeleton(st: Stream, n_xforms=16, name="R"):
+def random_skeleton(st: Stream, n_xforms=16, name="R", brs=False, hull=False):
+    """Generator R.  brs=True adds the full-BRS features of
+    SURVEY §8(f) NEXT-3: strides in {1, 2, 3, 4} on partial boxes and
+    irregular ("may") writes; hull=True marks the skeleton for the
+    approximate-UNION mode.  Both only add draws, so brs=False keeps the
+    original stream."""
     K = st.randint(4, 16)
     arrays = [{"name": f"a{i}", "rows": NY, "cols": NX,
                "elem_bytes": st.choice((4, 8)), "liveout": st.bernoulli(0.5)}
@@ -233,6 +238,8 @@ def random_skeleton(st: Stream, n_xforms=16, name="R"):
         if st.bernoulli(0.3):
             if mode == "R":
                 regions.append(whole_read(k, a, arrays))
+            elif brs and st.bernoulli(0.3):
+                regions.append(region(k, a, mode, arrays=arrays, whole=True))   # may-write
             else:
                 regions.append(full(k, a, mode, arrays))
             return
@@ -242,7 +249,11 @@ def random_skeleton(st: Stream, n_xforms=16, name="R"):
         q1 = st.randint(q0 + 1, 8)
         d0, d1, e0, e1 = (st.randint(0, 2) - 1 for _ in range(4))
         box = ((d0, 0, p0, 0), (d1, 0, p1, 0), (e0, q0, 0, 0), (e1, q1, 0, 0))
-        regions.append(region(k, a, mode, box=box))
+        reg = region(k, a, mode, box=box)
+        if brs:
+            reg["r_step"] = st.choice((1, 1, 2, 3, 4))
+            reg["c_step"] = st.choice((1, 1, 2, 4))
+        regions.append(reg)
 
     for k in range(K):
         q = st.randint(1, 8)
@@ -268,12 +279,16 @@ def random_skeleton(st: Stream, n_xforms=16, name="R"):
                         "total": total, "coal": coal, "uncoal": uncoal,
                         "upm": 32.0, "lbpw": 128.0, "synch": float(st.randint(0, 2))})
         kx.append(row)
-    return {"name": name, "arrays": arrays, "kernels": kernels, "regions": regions, "kx": kx}
+    out = {"name": name, "arrays": arrays, "kernels": kernels, "regions": regions, "kx": kx}
+    if hull:
+        out["hull"] = True
+    return out
 
 
-def random_skeletons(seed, count, n_xforms=16):
+def random_skeletons(seed, count, n_xforms=16, brs=False, hull=False):
     st = Stream(seed)
-    return [random_skeleton(st, n_xforms, name=f"R{seed:x}_{i}") for i in range(count)]
+    return [random_skeleton(st, n_xforms, name=f"R{seed:x}_{i}", brs=brs, hull=hull)
+            for i in range(count)]
 
 
 # ---- GPU model presets (CC 1.0 / Quadro FX 5600) --

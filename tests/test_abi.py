@@ -39,7 +39,7 @@ def test_every_declared_symbol_is_exported(G):
 
 
 def test_abi_version(G):
-    assert G.lib().grophecy_abi_version() == 1
+    assert G.lib().grophecy_abi_version() == 2
 
 
 def test_fit_pcie_matches_oracle_bitwise(G, O):
@@ -76,7 +76,9 @@ def _s0():
     (lambda s: s["kernels"].clear(), -1),
     (lambda s: s["regions"].append(dict(s["regions"][0], kernel=5)), -1),
     (lambda s: s["regions"].append(dict(s["regions"][0], array=7)), -1),
-    (lambda s: s["regions"].append(dict(s["regions"][0], mode="W", whole=True)), -1),
+    (lambda s: s["regions"].append(dict(s["regions"][0], r_step=65)), -2),
+    (lambda s: s["regions"].extend([dict(s["regions"][0], array=0, whole=False, c_step=7),
+                                    dict(s["regions"][0], array=0, whole=False, c_step=11)]), -2),
     (lambda s: s["regions"].extend([dict(s["regions"][1])] * 40), -2),
     (lambda s: s["arrays"].extend([dict(s["arrays"][0])] * 20), -2),
     (lambda s: s["kernels"].__setitem__(0, dict(s["kernels"][0], work=(0, 1 << 16, 0, 0))), -2),
@@ -197,3 +199,34 @@ def test_group_merge_host_rules():
     # b must follow a
     with pytest.raises(G.GrophecyError):
         G.group_merge_host(a, G.GroupResult(1.0, 16, 3, 16, 7, 8))
+
+
+def test_usage_plans_with_maywrites_match_oracle(G, O):
+    """Irregular writes (may-writes, reading 10) keep the plan path; its
+    closed forms reproduce the oracle."""
+    from tests.tiny import random_tiny_skeleton, rng
+    r = rng(556)
+    tot = 0
+    for _ in range(300):
+        s, _, _ = random_tiny_skeleton(r, maywrite=True)
+        sizes = [(int(r.integers(1, 2000)), int(r.integers(1, 2000))) for _ in range(6)]
+        tot += _check_plan(G, O, s, sizes)
+    assert tot > 200
+
+
+def test_strided_and_hull_skeletons_have_no_plan(G):
+    """Strided sections and the hull mode take the general device paths."""
+    from tests.tiny import random_tiny_skeleton, rng
+    r = rng(557)
+    n_str = 0
+    for _ in range(60):
+        s, nx, ny = random_tiny_skeleton(r, strided=True)
+        strided = any(g.get("r_step", 1) > 1 or g.get("c_step", 1) > 1
+                      for g in s["regions"] if not g["whole"])
+        rc, h, d, tx, ty = G.plan_usage_host(s, 64, 64)
+        if strided:
+            n_str += 1
+            assert rc == G.ELIMIT and tx == 0xFFFFFFFF
+        rc, h, d, tx, ty = G.plan_usage_host(dict(s, hull=True), 64, 64)
+        assert rc == G.ELIMIT and tx == 0xFFFFFFFF
+    assert n_str > 20
