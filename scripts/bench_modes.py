@@ -4,7 +4,9 @@
 
 One JSON line per mode: best (fused argmin), eval (SoA outputs), eval_parts
 (+ time components), group_best (best transformation per projection point),
-best_host (host records, PCIe-bound).  Candidates/s from CUDA events (or the
+crossover (break-even iterations from the components), best over the
+C3-shaped plan / strided / hull workloads, best_host (host records,
+PCIe-bound).  Candidates/s from CUDA events (or the
 host clock for the synchronous calls), algorithmic HBM bytes per candidate,
 and the fraction of MEASURED_PEAKS.json's HBM bandwidth.
 """
@@ -66,6 +68,7 @@ def main():
     d = torch.empty(n, dtype=torch.int64, device="cuda")
     t = torch.empty(n, dtype=torch.float64, device="cuda")
     parts = [torch.empty(n, dtype=torch.float64, device="cuda") for _ in range(4)]
+    # eval_parts fills them (t_iter, t_once, t_h2d, t_d2h) for the crossover line
     b = rec.batch()
     gout = torch.empty((n // 8) * 6, dtype=torch.int64, device="cuda")
     P = G.Parts(*[x.data_ptr() for x in parts])
@@ -88,6 +91,28 @@ def main():
                           "bytes_per_candidate": bpc, "hbm_GBps": gbs, "hbm_frac": gbs / peak,
                           "timer": "cuda events" if ev else "host clock (synchronous call)"}),
               flush=True)
+    # next-row workloads: crossover (NEXT-2) on eval_parts outputs
+    ti, to, th, td = parts
+    sec = timed(lambda: G.crossover(ti, to, th, td, 1e-3), reps, True)
+    gbs = 48 * n / sec / 1e9
+    print(json.dumps({"mode": "crossover", "n": n, "cand_per_s": n / sec, "ms": sec * 1e3,
+                      "bytes_per_candidate": 48, "hbm_GBps": gbs, "hbm_frac": gbs / peak,
+                      "timer": "cuda events"}), flush=True)
+    # C3-shaped workloads over the general paths (10^7 candidates, fused best):
+    # plans (c3), strided sections + may-writes (c3s), hull mode (c3h)
+    for wname in ("c3", "c3s", "c3h"):
+        wc = R.config(wname)
+        wsp = G.Space(wc["skeletons"], S.FX5600)
+        wrec = G.synth_records(wc)
+        wb = wrec.batch()
+        sec = timed(lambda: wsp.best_async(pc, wb, out), reps, True)
+        gbs = 16 * wrec.n / sec / 1e9
+        print(json.dumps({"mode": "best", "workload": wname, "n": wrec.n,
+                          "cand_per_s": wrec.n / sec, "ms": sec * 1e3, "bytes_per_candidate": 16,
+                          "hbm_GBps": gbs, "hbm_frac": gbs / peak, "timer": "cuda events"}),
+              flush=True)
+        wsp.close()
+        del wrec
     host = {k: getattr(rec, k).cpu().pin_memory() for k in ("skx", "nx", "ny", "iters")}
     sec = timed(lambda: space.best_host(pc, host), max(1, reps // 2), False)
     print(json.dumps({"mode": "best_host", "n": n, "cand_per_s": n / sec, "ms": sec * 1e3,
