@@ -45,7 +45,8 @@ typedef enum {
     GROPHECY_ELIMIT = -2,       /* a documented size limit is exceeded */
     GROPHECY_ECUDA = -3,        /* CUDA runtime error (message has details) */
     GROPHECY_ENOFEASIBLE = -5,  /* best: no valid candidate with finite time */
-    GROPHECY_EBADCAND = -6      /* some records were invalid (see n_invalid) */
+    GROPHECY_EBADCAND = -6,     /* some records were invalid (see n_invalid) */
+    GROPHECY_EINTERNAL = -7     /* internal consistency check failed (a bug) */
 } grophecy_status;
 
 /* ---------------------------------------------------------------------- */
@@ -355,19 +356,22 @@ int grophecy_synth_records(const grophecy_synth_rule *rules, uint32_t n_rules,
                            uint32_t *iters, void *cuda_stream);
 
 /* Diagnostic: evaluate on the HOST the usage plan that grophecy_space_create
- * compiles for `skel` (the closed-form band programs the kernel runs for
- * sizes inside the plan's domain nx >= *plan_tx, ny >= *plan_ty).  Fills
+ * compiles for `skel` (for sizes inside the plan's domain nx >= *plan_tx,
+ * ny >= *plan_ty: the residue-class byte polynomials the kernel evaluates,
+ * cross-checked against the band programs they are derived from).  Fills
  * per-array H2D / D2H bytes (arrays of skel->n_arrays).  Returns ELIMIT if
  * the skeleton has no plan or (nx, ny) is outside its domain (the kernel then
- * uses the general cell sweep).  Pure host function. */
+ * uses the general cell sweep), EINTERNAL if polynomial and program disagree.
+ * Pure host function. */
 int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int64_t nx, int64_t ny,
                              uint64_t *h2d_per_array, uint64_t *d2h_per_array,
                              uint32_t *plan_tx, uint32_t *plan_ty);
 
 /* Diagnostic: size of the usage plan compiled for `skel`: stats[0] =
  * expressions, [1] = program words, [2] = terms, [3] = terms, [4] = max terms
- * of one array program, [5] = max words of one program.  ELIMIT if the
- * skeleton has no plan.  Pure host function. */
+ * of one array program, [5] = max words of one program, [6] = coefficients
+ * per byte polynomial (4 bilinear, 10 otherwise).  `stats` holds 7 entries.
+ * ELIMIT if the skeleton has no plan.  Pure host function. */
 int grophecy_plan_stats(const grophecy_skeleton_desc *skel, uint32_t *stats);
 
 /* Number of CUDA kernel launches issued by this library since load (for

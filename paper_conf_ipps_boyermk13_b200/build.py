@@ -45,8 +45,6 @@ def build(force=False, verbose=False):
         cmd += ["-Xptxas", "-v"]
     if os.environ.get("GROPHECY_THREADS"):
         cmd += [f"-DGROPHECY_THREADS={int(os.environ['GROPHECY_THREADS'])}"]
-    if os.environ.get("GROPHECY_VAL"):
-        cmd += [f"-DGROPHECY_VAL={int(os.environ['GROPHECY_VAL'])}"]
     if os.environ.get("GROPHECY_MINB"):
         cmd += [f"-DGROPHECY_MINB={int(os.environ['GROPHECY_MINB'])}"]
     cmd += [os.path.join(CSRC, f) for f in SOURCES]

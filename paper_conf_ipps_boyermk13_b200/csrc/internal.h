@@ -44,17 +44,17 @@ struct SkelInfo {
     uint32_t a_base;   // into arrays
     uint32_t kx_base;  // into kx tables
     uint32_t flags;    // GROPHECY_SKEL_* (HULL) | SKF_STRIDED
-    // usage plan (plan.cpp): valid for nx >= plan_tx and ny >= plan_ty
-    uint32_t plan_tx, plan_ty, expr_base, n_expr;
-    // flat term list of all arrays / directions: {packed indices, 2*array + dir}
-    uint32_t term_base, n_terms, per_iter_mask, pad2;   // per_iter_mask: bit k = kernel k per-iteration
+    // usage plan (plan.cpp): valid for nx >= plan_tx and ny >= plan_ty; its
+    // byte polynomials at poly[poly_base + ...] (SkelPlanHost layout)
+    uint32_t plan_tx, plan_ty, poly_base, poly_stride;
+    uint32_t per_iter_mask, pad1, pad2, pad3;   // per_iter_mask: bit k = kernel k per-iteration
 };
 
 struct ArrayDev {
     int4 rows, cols;
     uint32_t elem_bytes, liveout, r_base, r_count;   // regions [r_base, r_base+r_count)
-    uint32_t h_prog, d_prog;                         // plan band programs (u32 word offsets)
     uint32_t lr, lc;    // lcm of the regions' row / column steps (1 = dense array)
+    uint32_t pad0, pad1;
 };
 enum : uint32_t { SKF_STRIDED = 1u << 16 };   // some region has a step > 1
 
@@ -67,7 +67,26 @@ struct SkelPlanHost {
     std::vector<int4> exprs;
     std::vector<uint32_t> prog;           // band programs (see plan.cpp)
     std::vector<uint32_t> h_off, d_off;   // per array, into prog
+    // Byte polynomials (plan.cpp, "residue-class polynomials"): for size class
+    // c = (nx mod 8) * 8 + (ny mod 8) and polynomial p = 2 * array + dir,
+    // poly[(c * n_polys + p) * poly_stride + m] = coefficient of monomial m in
+    // (a, b) = (nx div 8, ny div 8), monomials {1, a, b, ab, a^2, b^2, a^2 b,
+    // a b^2, a^2 b^2}; stride 4 when every skeleton term is bilinear, else 10
+    // (9 + pad).  Coefficients are mod 2^64 (wrapping); elem_bytes and the
+    // live-out flag are folded in, so P(a, b) = transfer bytes of the array.
+    std::vector<uint64_t> poly;
+    uint32_t poly_stride = 0;
 };
+constexpr uint32_t POLY_CLASSES = 64;
+
+// P(a, b) of one byte polynomial (host and device share the formula; device
+// copy in project.cu).  a, b < 2^18.
+inline uint64_t poly_eval_host(const uint64_t *c, uint32_t stride, uint64_t a, uint64_t b)
+{
+    uint64_t v = c[0] + c[1] * a + (c[2] + c[3] * a) * b;
+    if (stride > 4) v += a * (a * (c[4] + b * (c[6] + b * c[8]))) + b * (b * (c[5] + a * c[7]));
+    return v;
+}
 
 // Regions are stored grouped by array and sorted by kernel within an array,
 // so "first writer" = lowest set bit of a mask and upto = mask of regions of
@@ -92,9 +111,7 @@ struct SpaceDev {
     const KxJ *kx_j;
     const KxG *kx_g;
     const KxFast *kx_f;
-    const int4 *plan_expr;
-    const uint32_t *plan_prog;
-    const uint2 *plan_terms;
+    const unsigned long long *poly;   // usage byte polynomials (all skeletons)
     uint32_t n_skels;
     uint32_t n_sm;
     double freq, rfreq;

@@ -206,6 +206,77 @@ void emit(const std::vector<std::vector<uint8_t>> &cell, const std::vector<Ex> &
     out[at] = nt;
 }
 
+// Residue-class polynomials.  With nx = 8a + r, ny = 8b + s (0 <= r, s < 8):
+//   c1 nx + c2 ny + c3 nx ny = 8 (c1 a + c2 b + c3 (8ab + s a + r b)) + (c1 r + c2 s + c3 r s)
+// so every bound v = c0 + floor(L / 8) is EXACTLY bilinear in (a, b) on the
+// class (r, s):  v = k0 + k1 a + k2 b + k3 ab with
+//   k0 = c0 + floor((c1 r + c2 s + c3 r s) / 8), k1 = c1 + c3 s, k2 = c2 + c3 r, k3 = 8 c3.
+// A program term (row e - row s)(col e - col s) is a product of two such forms,
+// so each count = sum of terms is a polynomial of degree <= 2 in a and in b,
+// exact in wrapping 64-bit arithmetic (the true count fits).  Evaluating the 9
+// coefficients replaces evaluating every bound and every term per key.
+using u64 = uint64_t;
+struct Bil {
+    u64 k[4];
+};
+
+Bil bil_of(const Ex &e, int64_t r, int64_t s)
+{
+    Bil v;
+    const int64_t rem = e.c1 * r + e.c2 * s + e.c3 * r * s;
+    v.k[0] = (u64)(e.c0 + (rem >> 3));   // arithmetic shift: floor
+    v.k[1] = (u64)(e.c1 + e.c3 * s);
+    v.k[2] = (u64)(e.c2 + e.c3 * r);
+    v.k[3] = (u64)(8 * e.c3);
+    return v;
+}
+
+void compile_polys(const grophecy_skeleton_desc &S, const std::vector<Ex> &table, SkelPlanHost &out)
+{
+    const uint32_t np = 2 * S.n_arrays;
+    std::vector<u64> full((size_t)POLY_CLASSES * np * 9, 0);
+    bool biq = false;
+    for (uint32_t c = 0; c < POLY_CLASSES; c++) {
+        const int64_t r = c >> 3, s = c & 7;
+        std::vector<Bil> v(table.size());
+        for (size_t e = 0; e < table.size(); e++) v[e] = bil_of(table[e], r, s);
+        for (uint32_t a = 0; a < S.n_arrays; a++)
+            for (uint32_t dir = 0; dir < 2; dir++) {
+                u64 *m = &full[((size_t)c * np + 2 * a + dir) * 9];
+                const uint32_t *p = out.prog.data() + (dir ? out.d_off[a] : out.h_off[a]);
+                for (uint32_t t = 0; t < p[0]; t++) {
+                    const uint32_t w = p[1 + t];
+                    const Bil &rs = v[w & 0xff], &re = v[(w >> 8) & 0xff];
+                    const Bil &cs = v[(w >> 16) & 0xff], &ce = v[w >> 24];
+                    u64 D[4], C[4];
+                    for (int i = 0; i < 4; i++) {
+                        D[i] = re.k[i] - rs.k[i];
+                        C[i] = ce.k[i] - cs.k[i];
+                    }
+                    m[0] += D[0] * C[0];
+                    m[1] += D[0] * C[1] + D[1] * C[0];
+                    m[2] += D[0] * C[2] + D[2] * C[0];
+                    m[3] += D[0] * C[3] + D[3] * C[0] + D[1] * C[2] + D[2] * C[1];
+                    m[4] += D[1] * C[1];
+                    m[5] += D[2] * C[2];
+                    m[6] += D[1] * C[3] + D[3] * C[1];
+                    m[7] += D[2] * C[3] + D[3] * C[2];
+                    m[8] += D[3] * C[3];
+                }
+                const bool live = dir == 0 || (S.arrays[a].flags & GROPHECY_ARRAY_LIVEOUT);
+                const u64 eb = live ? S.arrays[a].elem_bytes : 0;
+                for (int i = 0; i < 9; i++) {
+                    m[i] *= eb;
+                    if (i >= 4 && m[i]) biq = true;
+                }
+            }
+    }
+    out.poly_stride = biq ? 10 : 4;
+    out.poly.assign((size_t)POLY_CLASSES * np * out.poly_stride, 0);
+    for (size_t q = 0; q < (size_t)POLY_CLASSES * np; q++)
+        for (uint32_t i = 0; i < (biq ? 9u : 4u); i++) out.poly[q * out.poly_stride + i] = full[q * 9 + i];
+}
+
 }  // namespace
 
 bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out)
@@ -266,6 +337,7 @@ bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out)
     if (table.size() > PLAN_MAX_EXPR) return false;
     for (const Ex &e : table)
         out.exprs.push_back(make_int4((int)e.c0, (int)e.c1, (int)e.c2, (int)e.c3));
+    compile_polys(S, table, out);
     out.tx = 1u << best_tx;
     out.ty = 1u << best_ty;
     out.ok = true;
@@ -306,8 +378,12 @@ extern "C" int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int6
         set_error("size outside the plan's domain");
         return GROPHECY_ELIMIT;
     }
+    // the device evaluates the residue-class byte polynomials; the band
+    // programs they were derived from are evaluated alongside as a check
     std::vector<int64_t> val(P.exprs.size());
     for (size_t e = 0; e < P.exprs.size(); e++) val[e] = aff8_host(P.exprs[e], nx, ny);
+    const uint32_t np = 2 * skel->n_arrays;
+    const uint32_t cls = (uint32_t)((nx & 7) * 8 + (ny & 7));
     for (uint32_t a = 0; a < skel->n_arrays; a++) {
         for (int which = 0; which < 2; which++) {
             const uint32_t *p = P.prog.data() + (which ? P.d_off[a] : P.h_off[a]);
@@ -319,8 +395,17 @@ extern "C" int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int6
                                   (val[w >> 24] - val[(w >> 16) & 0xff]));
             }
             const uint64_t eb = skel->arrays[a].elem_bytes;
-            if (which == 0) h2d_per_array[a] = cnt * eb;
-            else d2h_per_array[a] = (skel->arrays[a].flags & GROPHECY_ARRAY_LIVEOUT) ? cnt * eb : 0;
+            const bool live = which == 0 || (skel->arrays[a].flags & GROPHECY_ARRAY_LIVEOUT);
+            const uint64_t bytes = live ? cnt * eb : 0;
+            const uint64_t pb = poly_eval_host(
+                P.poly.data() + ((size_t)cls * np + 2 * a + which) * P.poly_stride, P.poly_stride,
+                (uint64_t)(nx >> 3), (uint64_t)(ny >> 3));
+            if (pb != bytes) {
+                set_error("usage polynomial disagrees with its band program");
+                return GROPHECY_EINTERNAL;
+            }
+            if (which == 0) h2d_per_array[a] = pb;
+            else d2h_per_array[a] = pb;
         }
     }
     return GROPHECY_OK;
@@ -348,5 +433,6 @@ extern "C" int grophecy_plan_stats(const grophecy_skeleton_desc *skel, uint32_t 
     stats[3] = runs;
     stats[4] = maxb;
     stats[5] = maxw;
+    stats[6] = P.poly_stride;
     return GROPHECY_OK;
 }

@@ -38,10 +38,6 @@ constexpr int WARPS = THREADS / 32;
 constexpr int RPT = 4;                       // records per lane
 constexpr int WTILE = 32 * RPT;              // records per warp tile
 constexpr int SLOT_CAP = 16;                 // distinct keys resident per warp chunk
-#ifndef GROPHECY_VAL
-#define GROPHECY_VAL 256
-#endif
-constexpr int VAL_PER_WARP = GROPHECY_VAL;   // plan expression values per warp pass
 constexpr int MAXK = GROPHECY_MAX_KERNELS;   // kernels per skeleton
 constexpr long long BIG = 0x7fffffffffffffffLL;
 #ifndef GROPHECY_MINB
@@ -92,8 +88,7 @@ struct SweepScratch {
 constexpr int MAX_SEG = 8;                   // keys per warp pass (plan path)
 
 struct PlanScratch {
-    long long val[VAL_PER_WARP + 32];                // expression values of the pass's keys
-    double T[MAX_SEG][2 * GROPHECY_MAX_ARRAYS + 4];  // per-array counts, then transfer times
+    alignas(16) double T[MAX_SEG][2 * GROPHECY_MAX_ARRAYS + 2];  // per-array transfer times of the pass's keys
 };
 
 union WarpScratch {
@@ -128,59 +123,62 @@ __device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned 
     o.d += da;
 }
 
-// Usage of one key from its skeleton's compiled plan (plan.cpp), by a segment
-// of L lanes (32/L keys per warp pass).  Lanes evaluate the plan's
-// expressions (entries 0..K-1 are the kernels' work-item counts), then lane sl
-// runs the H2D and D2H programs of arrays sl, sl+L, ... and prices each
-// transfer with Eq. (1) into T[2a + dir]; byte totals are an integer tree sum
-// over the segment, and the segment's lane 0 adds the transfer times in array
-// order.  Results: *res (segment lane 0) and the key's work counts in w_out.
-__device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsigned long long key,
-                                           const grophecy_pcie &pc, long long *val, double *T,
-                                           int sl, int L, Usage *res, uint32_t *w_out)
+__device__ __forceinline__ uint32_t sat_u32(long long w)
 {
-    uint32_t n_expr = 0, n_arrays = 0, e0 = 0, a0 = 0, K = 0, tb = 0, nt = 0;
-    long long nx = 0, ny = 0;
+    return w <= 0 ? 0u : (w >= 0xffffffffLL ? 0xffffffffu : (uint32_t)w);
+}
+
+// One residue-class byte polynomial P(a, b) (plan.cpp; internal.h layout),
+// wrapping 64-bit arithmetic; a, b < 2^18.
+template <bool BIQ>
+__device__ __forceinline__ unsigned long long poly_eval(const unsigned long long *c, uint32_t a,
+                                                        uint32_t b)
+{
+    const ulonglong2 c01 = __ldg(reinterpret_cast<const ulonglong2 *>(c));
+    const ulonglong2 c23 = __ldg(reinterpret_cast<const ulonglong2 *>(c) + 1);
+    unsigned long long v = c01.x + c01.y * a + (c23.x + c23.y * a) * b;
+    if (BIQ) {
+        const ulonglong2 c45 = __ldg(reinterpret_cast<const ulonglong2 *>(c) + 2);
+        const ulonglong2 c67 = __ldg(reinterpret_cast<const ulonglong2 *>(c) + 3);
+        const unsigned long long c8 = __ldg(c + 8);
+        v += (unsigned long long)a * (a * (c45.x + b * (c67.x + b * c8))) +
+             (unsigned long long)b * (b * (c45.y + a * c67.y));
+    }
+    return v;
+}
+
+// Usage of one key from its skeleton's residue-class byte polynomials
+// (plan.cpp), by a segment of L lanes (32/L keys per warp pass).  Lane sl
+// evaluates the H2D and D2H polynomials of arrays sl, sl+L, ... (bytes, with
+// elem_bytes and live-out folded in) and prices each transfer with Eq. (1)
+// into T[2a + dir]; byte totals are an integer tree sum over the segment, and
+// the segment's lane 0 adds the transfer times in array order (N6).  The
+// kernels' work-item counts go to w_out.  Results: *res (segment lane 0).
+__device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsigned long long key,
+                                           const grophecy_pcie &pc, double *T, int sl, int L,
+                                           Usage *res, uint32_t *w_out)
+{
+    uint32_t n_arrays = 0, K = 0, kb = 0, stride = 4;
+    uint32_t nx = 0, ny = 0;
+    const unsigned long long *P = S.poly;
     if (active) {
         const SkelInfo &I = S.skel[(uint32_t)(key >> 42)];
-        n_expr = I.n_expr; n_arrays = I.n_arrays; e0 = I.expr_base; a0 = I.a_base;
-        K = I.n_kernels; tb = I.term_base; nt = I.n_terms;
-        nx = (long long)((key >> 21) & 0x1fffffull);
-        ny = (long long)(key & 0x1fffffull);
+        n_arrays = I.n_arrays;
+        K = I.n_kernels;
+        kb = I.k_base;
+        stride = I.poly_stride;
+        nx = (uint32_t)((key >> 21) & 0x1fffffull);
+        ny = (uint32_t)(key & 0x1fffffull);
+        P += I.poly_base + (size_t)((nx & 7u) * 8u + (ny & 7u)) * (2u * n_arrays * stride);
     }
-    unsigned long long *cnt = reinterpret_cast<unsigned long long *>(T);   // counts, then times
-    {
-        const int ix = (int)nx, iy = (int)ny;
-        const long long nxny = (long long)((unsigned long long)(uint32_t)ix * (uint32_t)iy);
-        for (uint32_t e = sl; e < n_expr; e += L)
-            val[e] = aff8n(__ldg(&S.plan_expr[e0 + e]), ix, iy, nxny);
-        for (uint32_t i = sl; i < 2 * n_arrays; i += L) cnt[i] = 0ull;
-    }
-    __syncwarp();
-    // lanes over the skeleton's flat term list: count[2a + dir] += (row extent) x (column run)
-    for (uint32_t t = sl; t < nt; t += L) {
-        const uint2 tw = __ldg(&S.plan_terms[tb + t]);   // rs | re << 8 | cs << 16 | ce << 24
-        const unsigned long long prod =
-            (unsigned long long)((val[(tw.x >> 8) & 0xffu] - val[tw.x & 0xffu]) *
-                                 (val[tw.x >> 24] - val[(tw.x >> 16) & 0xffu]));
-        // exact 64-bit accumulate from native 32-bit shared atomics: the carry
-        // out of the low word is taken at each add
-        unsigned *c32 = reinterpret_cast<unsigned *>(&cnt[tw.y]);
-        const unsigned lo = (unsigned)prod;
-        unsigned hi = (unsigned)(prod >> 32);
-        const unsigned old = atomicAdd(c32, lo);
-        hi += (old + lo) < old;
-        if (hi) atomicAdd(c32 + 1, hi);
-    }
-    __syncwarp();
+    const uint32_t a8 = nx >> 3, b8 = ny >> 3;
     unsigned long long hs = 0, ds = 0;
     for (uint32_t a = sl; a < n_arrays; a += L) {
-        const ArrayDev &A = S.arrays[a0 + a];
-        const unsigned long long eb = A.elem_bytes;
 #pragma unroll
         for (int dir = 0; dir < 2; dir++) {
-            const unsigned long long c = cnt[2 * a + dir];
-            const unsigned long long bytes = (dir && !A.liveout) ? 0ull : c * eb;
+            const unsigned long long *c = P + (2 * a + dir) * stride;
+            const unsigned long long bytes = stride > 4 ? poly_eval<true>(c, a8, b8)
+                                                        : poly_eval<false>(c, a8, b8);
             const grophecy_link lk = dir ? pc.d2h : pc.h2d;
             T[2 * a + dir] = bytes ? __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte,
                                                                     __ull2double_rn(bytes)))
@@ -188,9 +186,10 @@ __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsig
             if (dir) ds += bytes; else hs += bytes;
         }
     }
-    for (uint32_t q = sl; q < K; q += L) {
-        const long long v = val[q];
-        w_out[q] = v <= 0 ? 0u : (v >= 0xffffffffLL ? 0xffffffffu : (uint32_t)v);
+    {
+        const long long nxny = (long long)((unsigned long long)nx * ny);
+        for (uint32_t q = sl; q < K; q += L)
+            w_out[q] = sat_u32(aff8n(__ldg(&S.kern_work[kb + q]), (int)nx, (int)ny, nxny));
     }
     for (int off = 1; off < L; off <<= 1) {
         hs += __shfl_xor_sync(FULL, hs, off);
@@ -200,8 +199,9 @@ __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsig
     if (active && sl == 0) {
         double th = 0.0, td = 0.0;   // arrays without transfer add +0.0
         for (uint32_t a = 0; a < n_arrays; a++) {
-            th = __dadd_rn(th, T[2 * a]);
-            td = __dadd_rn(td, T[2 * a + 1]);
+            const double2 t2 = *reinterpret_cast<const double2 *>(&T[2 * a]);
+            th = __dadd_rn(th, t2.x);
+            td = __dadd_rn(td, t2.y);
         }
         Usage o;
         o.h = hs;
@@ -212,10 +212,6 @@ __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsig
     }
 }
 
-__device__ __forceinline__ uint32_t sat_u32(long long w)
-{
-    return w <= 0 ? 0u : (w >= 0xffffffffLL ? 0xffffffffu : (uint32_t)w);
-}
 
 // x mod m in [0, m) for m >= 1
 __device__ __forceinline__ long long pmodll(long long x, long long m)
@@ -977,22 +973,16 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                 const bool mv = (unsigned)lane < gcnt;
                 const unsigned long long mk = mv ? ws.slot_key[g0 - c0 + lane] : 0ull;
                 bool mplan = false;
-                uint32_t mne = 0;
                 if (mv) {
                     const SkelInfo &I = S.skel[(uint32_t)(mk >> 42)];
                     mplan = (long long)((mk >> 21) & 0x1fffffull) >= I.plan_tx &&
                             (long long)(mk & 0x1fffffull) >= I.plan_ty;
-                    mne = I.n_expr;
                 }
                 unsigned todo = __ballot_sync(FULL, mv && mplan);
                 unsigned sweep = __ballot_sync(FULL, mv && !mplan);
-                const uint32_t max_ne = __reduce_max_sync(FULL, mplan ? mne : 0u);
-                // lanes per key L = 2^lg: 4 (8 keys per pass) unless the values do not fit
-                const int lg = max_ne * MAX_SEG <= VAL_PER_WARP ? 2
-                             : max_ne * 4 <= VAL_PER_WARP ? 3
-                             : max_ne * 2 <= VAL_PER_WARP ? 4 : 5;
-                const int L = 1 << lg, G = 32 >> lg, seg = lane >> lg, sl = lane & (L - 1);
-                const int vstride = (VAL_PER_WARP >> (5 - lg)) + L;   // VAL/G + L
+                // 4 lanes per key, 8 keys per pass
+                constexpr int L = 32 / MAX_SEG, G = MAX_SEG;
+                const int seg = lane / L, sl = lane % L;
                 // compact list of the plan keys' positions (rank -> slot lane)
                 if (mv && mplan) ws.plan_pos[__popc(todo & ((1u << lane) - 1u))] = (uint8_t)lane;
                 const int nplan = __popc(todo);
@@ -1002,9 +992,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
                     const unsigned pos = act ? ws.plan_pos[p0 + seg] : 0u;
                     const unsigned long long k = __shfl_sync(FULL, mk, pos);
                     const unsigned ls = g0 - c0 + pos;
-                    // segment stride VAL/G + L longs: the segments' lanes hit distinct banks
-                    plan_usage(S, act, k, P.pc, ws.scratch.pl.val + seg * vstride,
-                               ws.scratch.pl.T[seg], sl, L, &ws.res[ls], ws.slot_w[ls]);
+                    plan_usage(S, act, k, P.pc, ws.scratch.pl.T[seg], sl, L, &ws.res[ls],
+                               ws.slot_w[ls]);
                     __syncwarp();
                 }
                 while (sweep) {

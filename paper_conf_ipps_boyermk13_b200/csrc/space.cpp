@@ -277,9 +277,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxJ> kj;
     std::vector<KxG> kg;
     std::vector<KxFast> kf;
-    std::vector<int4> pexpr;
-    std::vector<uint32_t> pprog;
-    std::vector<uint2> pterms;
+    std::vector<unsigned long long> poly;
     auto a4 = [](const grophecy_affine8 &a) { return make_int4(a.c0, a.c1, a.c2, a.c3); };
     for (uint32_t s = 0; s < n_skels; s++) {
         const grophecy_skeleton_desc &S = skels[s];
@@ -301,27 +299,18 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         if (compile_plan(S, plan)) {
             I.plan_tx = plan.tx;
             I.plan_ty = plan.ty;
-            I.expr_base = (uint32_t)pexpr.size();
-            I.n_expr = (uint32_t)plan.exprs.size();
-            pexpr.insert(pexpr.end(), plan.exprs.begin(), plan.exprs.end());
+            // keep every skeleton's table 16-byte aligned (2 coefficients)
+            if (poly.size() & 1) poly.push_back(0);
+            I.poly_base = (uint32_t)poly.size();
+            I.poly_stride = plan.poly_stride;
+            poly.insert(poly.end(), plan.poly.begin(), plan.poly.end());
         } else {
             I.plan_tx = I.plan_ty = 0xffffffffu;   // never applicable
-            I.expr_base = I.n_expr = 0;
+            I.poly_base = I.poly_stride = 0;
         }
-        const uint32_t prog_base = (uint32_t)pprog.size();
-        if (plan.ok) pprog.insert(pprog.end(), plan.prog.begin(), plan.prog.end());
-        I.term_base = (uint32_t)pterms.size();
-        I.n_terms = 0;
-        I.per_iter_mask = I.pad2 = 0;
+        I.per_iter_mask = I.pad1 = I.pad2 = I.pad3 = 0;
         for (uint32_t k = 0; k < S.n_kernels; k++)
             if (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) I.per_iter_mask |= 1u << k;
-        if (plan.ok)
-            for (uint32_t a = 0; a < S.n_arrays; a++)
-                for (uint32_t dir = 0; dir < 2; dir++) {
-                    const uint32_t *p = plan.prog.data() + (dir ? plan.d_off[a] : plan.h_off[a]);
-                    for (uint32_t t = 0; t < p[0]; t++) pterms.push_back(make_uint2(p[1 + t], 2 * a + dir));
-                }
-        I.n_terms = (uint32_t)pterms.size() - I.term_base;
         for (uint32_t k = 0; k < S.n_kernels; k++) {
             kwork.push_back(a4(S.kernels[k].work_items));
             kflags.push_back(S.kernels[k].flags);
@@ -333,9 +322,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             A.elem_bytes = S.arrays[a].elem_bytes;
             A.liveout = (S.arrays[a].flags & GROPHECY_ARRAY_LIVEOUT) ? 1u : 0u;
             A.r_base = (uint32_t)regions.size();
-            A.h_prog = plan.ok ? prog_base + plan.h_off[a] : 0;
-            A.d_prog = plan.ok ? prog_base + plan.d_off[a] : 0;
             A.lr = A.lc = 1;
+            A.pad0 = A.pad1 = 0;
             // regions of this array, stably sorted by kernel (order within a
             // kernel is irrelevant: usage does not depend on region order)
             std::vector<const grophecy_region_desc *> rs;
@@ -403,10 +391,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {ki.data(), ki.size() * sizeof(KxI), 0},
         {kj.data(), kj.size() * sizeof(KxJ), 0},
         {kg.data(), kg.size() * sizeof(KxG), 0},
-        {pexpr.data(), pexpr.size() * sizeof(int4), 0},
-        {pprog.data(), pprog.size() * sizeof(uint32_t), 0},
+        {poly.data(), poly.size() * sizeof(unsigned long long), 0},
         {kf.data(), kf.size() * sizeof(KxFast), 0},
-        {pterms.data(), pterms.size() * sizeof(uint2), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -460,10 +446,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.kx_i = (const KxI *)(base + parts[7].off);
     D.kx_j = (const KxJ *)(base + parts[8].off);
     D.kx_g = (const KxG *)(base + parts[9].off);
-    D.plan_expr = (const int4 *)(base + parts[10].off);
-    D.plan_prog = (const uint32_t *)(base + parts[11].off);
-    D.kx_f = (const KxFast *)(base + parts[12].off);
-    D.plan_terms = (const uint2 *)(base + parts[13].off);
+    D.poly = (const unsigned long long *)(base + parts[10].off);
+    D.kx_f = (const KxFast *)(base + parts[11].off);
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;
     D.freq = gpu->freq_hz;
