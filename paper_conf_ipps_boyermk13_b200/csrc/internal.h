@@ -25,12 +25,15 @@ struct __align__(16) KxJ  { uint32_t ipb, occ, wpb, flags; };        // flags: K
 enum : uint32_t { KXF_INFEASIBLE = 1u, KXF_NOMEM = 2u, KXF_PER_ITER = 4u };
 
 // Packed fast-path record (48 B, one address per (kernel, transformation)):
-// blocks = ceil(W / ipb) from q = hi32(magic_hi*W + hi32(magic_lo*W)) for
-// W < 2^32 - 1 (magic = ceil(2^64/ipb), or 2^64-1 when ipb == 1); saturated
-// iff blocks >= sat32; infeasible (occupancy 0) <=> E == +inf.
+// for 0 < W < 2^31, blocks = ceil(W / ipb) = hi32(magic_hi*W' + hi32(magic_lo*W'))
+// with W' = W + addend (magic = ceil(2^64/ipb), addend = ipb - 1; ipb == 1:
+// magic = 2^64 - 1, addend = 1); the saturated formula holds iff
+// blocks >= sat32.  Infeasible (occupancy 0) or ipb > 2^31: sat32 = 2^32 - 1
+// (always the general path).  Work counts outside (0, 2^31) are stored as 0,
+// which also selects the general path (blocks = 0 < sat32).
 struct __align__(16) KxFast {
     double E, S, D, rD;
-    uint32_t magic_lo, magic_hi, sat32, ipb;
+    uint32_t magic_lo, magic_hi, sat32, addend;
 };
 
 // General-grid constants (small grids / huge W), read only off the fast path.

@@ -123,9 +123,12 @@ __device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned 
     o.d += da;
 }
 
-__device__ __forceinline__ uint32_t sat_u32(long long w)
+// Work-item count as stored for the model's fast path: W if 0 < W < 2^31,
+// else 0 (blocks = 0 < sat32 sends the record to the general path, which
+// recomputes W from the key).
+__device__ __forceinline__ uint32_t w_store(long long w)
 {
-    return w <= 0 ? 0u : (w >= 0xffffffffLL ? 0xffffffffu : (uint32_t)w);
+    return (w > 0 && w < 0x80000000LL) ? (uint32_t)w : 0u;
 }
 
 // One residue-class byte polynomial P(a, b) (plan.cpp; internal.h layout),
@@ -189,7 +192,7 @@ __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsig
     {
         const long long nxny = (long long)((unsigned long long)nx * ny);
         for (uint32_t q = sl; q < K; q += L)
-            w_out[q] = sat_u32(aff8n(__ldg(&S.kern_work[kb + q]), (int)nx, (int)ny, nxny));
+            w_out[q] = w_store(aff8n(__ldg(&S.kern_work[kb + q]), (int)nx, (int)ny, nxny));
     }
     for (int off = 1; off < L; off <<= 1) {
         hs += __shfl_xor_sync(FULL, hs, off);
@@ -573,8 +576,8 @@ __device__ __forceinline__ void slow_usage(const SpaceDev *gS, unsigned long lon
     const Usage r = (I.flags & GROPHECY_SKEL_HULL) ? warp_usage_hull(S, I, kx_, ky_, pc, lane)
                                                    : warp_usage_sweep(S, I, kx_, ky_, pc, *scr, lane);
     if (lane == 0) *res = r;
-    if ((uint32_t)lane < I.n_kernels)
-        w_out[lane] = sat_u32(aff8(__ldg(&S.kern_work[I.k_base + lane]), kx_, ky_));
+    if (w_out && (uint32_t)lane < I.n_kernels)
+        w_out[lane] = w_store(aff8(__ldg(&S.kern_work[I.k_base + lane]), kx_, ky_));
 }
 
 // Kernel time of one kernel (DESIGN.md §3 N5) from its work-item count Wi and
@@ -729,27 +732,61 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
     r.n_valid = b.nval;
 }
 
+// Canonical tiles: CX consecutive records per group (one group per lane),
+// XW transformations per model pass.
+constexpr int CX = 16;
+constexpr int CTILE = 32 * CX;
+constexpr int XW = 4;
+
 // Per-warp shared memory (dynamic; > 48 KB per CTA needs the opt-in attribute).
 struct WarpSmem {
-    WarpScratch scratch;                        // usage plans / general sweep
-    unsigned long long slot_key[SLOT_CAP];      // distinct keys of the chunk
-    Usage res[SLOT_CAP];                        // their usage
-    uint32_t slot_w[SLOT_CAP][MAXK + 1];        // their work-item counts (saturated; padded row)
-    unsigned long long rec_key[WTILE];          // the tile's records after phase A
-    uint32_t rec_skx[WTILE], rec_it[WTILE];
-    int rec_slot[WTILE];
-    unsigned long long best_h[32], best_d[32];  // bytes of each lane's running best
-    uint8_t plan_pos[MAX_SEG];                  // plan keys of the current slot group
+    WarpScratch scratch;                            // usage plans / general sweep
+    union {
+        struct {                                    // general tiles
+            unsigned long long slot_key[SLOT_CAP];  // distinct keys of the chunk
+            Usage res[SLOT_CAP];                    // their usage
+            uint32_t slot_w[SLOT_CAP][MAXK + 1];    // their work-item counts (w_store; padded row)
+            unsigned long long rec_key[WTILE];      // the tile's records after phase A
+            uint32_t rec_skx[WTILE], rec_it[WTILE];
+            int rec_slot[WTILE];
+            uint8_t plan_pos[MAX_SEG];              // plan keys of the current slot group
+        };
+        struct {                                    // canonical tiles
+            uint32_t cw[MAXK][32];                  // work counts (w_store), [kernel][lane]
+            Usage cres[32];                         // usage of keys off the plan path
+        };
+    };
+    unsigned long long best_h[32], best_d[32];      // bytes of each lane's running best
 };
 struct CtaSmem {
     WarpSmem w[WARPS];
 };
 
+// Saturated-grid kernel time (DESIGN.md §3 N5, saturated reduction) of one
+// (record, kernel) from the packed constants and the stored work count w
+// (w_store): cyc = E rep + S rep, rep = blocks / D, t = cyc / freq, both
+// divisions by Markstein's correction (bitwise the IEEE quotients).  gen is
+// set when the record must take the general path instead (small grid, huge
+// or zero work, infeasible) — the returned value is then meaningless.
+__device__ __forceinline__ double fast_time(const KxFast &f, uint32_t w, double freq, double rfreq,
+                                            bool &gen)
+{
+    const uint32_t w1 = w + f.addend;
+    const unsigned long long lo = (unsigned long long)f.magic_lo * w1;
+    const uint32_t blocks = (uint32_t)(((unsigned long long)f.magic_hi * w1 + (lo >> 32)) >> 32);
+    gen = blocks < f.sat32;
+    const double bb = __uint2double_rn(blocks);
+    const double q = __dmul_rn(bb, f.rD);
+    const double rep = __fma_rn(__fma_rn(-q, f.D, bb), f.rD, q);
+    const double cyc = __dadd_rn(__dmul_rn(f.E, rep), __dmul_rn(f.S, rep));
+    const double q2 = __dmul_rn(cyc, rfreq);
+    return __fma_rn(__fma_rn(-q2, freq, cyc), rfreq, q2);
+}
+
 // Model of NJ records of one skeleton at once (NJ independent dependency
 // chains per thread).  W[j] = the work-item counts of record j's key (shared
 // memory, one row per distinct key).  The saturated-grid formula is computed
-// branch-free for every record; the rare general-grid / >= 2^32-item cases
-// are recomputed by kernel_time.
+// for every record; the rare general-grid cases are recomputed by kernel_time.
 template <int NJ, bool SAMEX>
 __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uint32_t *x,
                                         const int *ls, const WarpSmem &ws, double *t_iter,
@@ -766,54 +803,25 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
         bool gen[NJ];
         KxFast F0;
         if (SAMEX) F0 = S.kx_f[kb + x[0]];   // one constant load shared by the NJ records
-        // staged so that the NJ independent dependency chains interleave
-        KxFast F[NJ];
-        uint32_t w[NJ], blocks[NJ];
-        double bb[NJ], q[NJ], rep[NJ], cyc[NJ];
 #pragma unroll
         for (int j = 0; j < NJ; j++) {
-            F[j] = SAMEX ? F0 : S.kx_f[kb + x[j]];
-            w[j] = ws.slot_w[ls[j]][k];   // saturated at 2^32 - 1
+            const KxFast F = SAMEX ? F0 : S.kx_f[kb + x[j]];
+            tk[j] = fast_time(F, ws.slot_w[ls[j]][k], S.freq, S.rfreq, gen[j]);
         }
+        bool any = false;
 #pragma unroll
-        for (int j = 0; j < NJ; j++) {
-            const unsigned long long lo = (unsigned long long)F[j].magic_lo * w[j];
-            const uint32_t qq = (uint32_t)(((unsigned long long)F[j].magic_hi * w[j] + (lo >> 32)) >> 32);
-            blocks[j] = qq + (qq * F[j].ipb != w[j]);
-            bb[j] = __uint2double_rn(blocks[j]);
+        for (int j = 0; j < NJ; j++) any |= gen[j];
+        if (any) {
+#pragma unroll
+            for (int j = 0; j < NJ; j++)
+                if (gen[j]) {
+                    const unsigned long long kk = ws.slot_key[ls[j]];
+                    const long long Wi = aff8(__ldg(&S.kern_work[I.k_base + k]),
+                                              (long long)((kk >> 21) & 0x1fffffull),
+                                              (long long)(kk & 0x1fffffull));
+                    tk[j] = kernel_time(S, Wi, S.kx_j[kb + x[j]], kb + x[j]);
+                }
         }
-        // rep = blocks / D  (Markstein, bitwise the IEEE quotient)
-#pragma unroll
-        for (int j = 0; j < NJ; j++) q[j] = __dmul_rn(bb[j], F[j].rD);
-#pragma unroll
-        for (int j = 0; j < NJ; j++) rep[j] = __fma_rn(-q[j], F[j].D, bb[j]);
-#pragma unroll
-        for (int j = 0; j < NJ; j++) rep[j] = __fma_rn(rep[j], F[j].rD, q[j]);
-        // cycles = E rep + S rep
-#pragma unroll
-        for (int j = 0; j < NJ; j++) cyc[j] = __dadd_rn(__dmul_rn(F[j].E, rep[j]), __dmul_rn(F[j].S, rep[j]));
-        // t = cycles / freq  (Markstein)
-#pragma unroll
-        for (int j = 0; j < NJ; j++) q[j] = __dmul_rn(cyc[j], S.rfreq);
-#pragma unroll
-        for (int j = 0; j < NJ; j++) rep[j] = __fma_rn(-q[j], S.freq, cyc[j]);
-#pragma unroll
-        for (int j = 0; j < NJ; j++) {
-            const double v = __fma_rn(rep[j], S.rfreq, q[j]);
-            // feasible: sat32 >= 1, so blocks == 0 and small grids take the
-            // general path; infeasible (E == +inf): sat32 == 0, t = +inf
-            gen[j] = w[j] == 0xffffffffu || blocks[j] < F[j].sat32;
-            tk[j] = isinf(F[j].E) ? __longlong_as_double(0x7ff0000000000000LL) : v;
-        }
-#pragma unroll
-        for (int j = 0; j < NJ; j++)
-            if (gen[j]) {
-                const unsigned long long kk = ws.slot_key[ls[j]];
-                const long long Wi = aff8(__ldg(&S.kern_work[I.k_base + k]),
-                                          (long long)((kk >> 21) & 0x1fffffull),
-                                          (long long)(kk & 0x1fffffull));
-                tk[j] = kernel_time(S, Wi, S.kx_j[kb + x[j]], kb + x[j]);
-            }
         if ((pim >> k) & 1u) {
 #pragma unroll
             for (int j = 0; j < NJ; j++) ti[j] = __dadd_rn(ti[j], tk[j]);
@@ -866,32 +874,23 @@ __device__ __forceinline__ unsigned long long key_of(const SpaceDev &S, uint32_t
 //   C  lane l models records l, l+32, l+64, l+96 — the same transformation
 //      when candidates come in groups of 16 — sharing one constant load per
 //      kernel, then writes outputs / keeps its running argmin.
+// One general tile: 128 consecutive records from tb (any layout, ragged
+// tail, invalid records), processed by one warp:
+//   A  lane l loads records l + 32 j, checks them, and run heads of equal
+//      keys get slot ids by a warp scan;
+//   B  usage of each distinct key once (plan: 8 keys per pass; else sweep);
+//   C  lane l models records l, l+32, l+64, l+96 — the same transformation
+//      when candidates come in groups of 16 — sharing one constant load per
+//      kernel, then writes outputs / keeps its running argmin.
 template <bool BEST>
-__global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const Params P)
+__device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsigned long long tb,
+                                             int lane, double &best_t, unsigned long long &best_i,
+                                             uint32_t &cnt_inv, uint32_t &cnt_val)
 {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int lane = threadIdx.x & 31;
-    const int warp = threadIdx.x >> 5;
-    WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
-    __shared__ Best wbest[WARPS];
-    __shared__ bool am_last;
     const SpaceDev &S = P.S;
     const unsigned lt = (1u << lane) - 1u;
-
-    // running argmin kept lean in registers: (t, index) + counters; the
-    // winner's byte counts go to shared memory (rarely updated)
-    double best_t = __longlong_as_double(0x7ff0000000000000LL);
-    unsigned long long best_i = ~0ull;
-    uint32_t cnt_inv = 0, cnt_val = 0;
-    ws.best_h[lane] = 0;
-    ws.best_d[lane] = 0;
-    const unsigned long long ntiles = (P.n + WTILE - 1) / WTILE;
-    const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
-    for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
-         tile += wstride) {
         // ---- A: records q = lane + 32 j (coalesced 32-bit loads), keys, run
         //      heads (ballots) and slot ids in record order ----
-        const unsigned long long tb = tile * WTILE;
         uint32_t skx[RPT], nx[RPT], ny[RPT], it[RPT];
 #pragma unroll
         for (int j = 0; j < RPT; j++) {
@@ -901,19 +900,6 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             nx[j] = h ? __ldcs(P.nx + i) : 0u;
             ny[j] = h ? __ldcs(P.ny + i) : 0u;
             it[j] = h ? __ldcs(P.iters + i) : 0u;
-        }
-        // warm L2 with the records of this warp's next tile
-        if (lane < 4) {
-            const unsigned long long nt = tile + wstride;
-            if (nt < ntiles && P.aligned) {
-                const unsigned long long nb = nt * WTILE;
-                const unsigned long long cnt = min((unsigned long long)WTILE, P.n - nb);
-                const uint32_t *base = lane == 0 ? P.skx : lane == 1 ? P.nx : lane == 2 ? P.ny : P.iters;
-                const uint32_t bytes = (uint32_t)(cnt * 4) & ~15u;
-                if (bytes)
-                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;"
-                                 :: "l"(base + nb), "r"(bytes) : "memory");
-            }
         }
         unsigned long long key[RPT];
         {
@@ -1103,6 +1089,227 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
             const unsigned tot = __reduce_add_sync(FULL, n_invalid);
             if (lane == 0 && tot) atomicAdd(S.invalid_counter, (unsigned long long)tot);
         }
+}
+
+// One canonical tile: CTILE records from tb where every group of CX
+// consecutive records (lane l: records tb + CX l ...) is one design point
+// (same skeleton, nx, ny, iters; xform = position in the group, the layout
+// of a skeleton x transformation x size sweep) and the whole tile has one
+// skeleton.  Returns false, having written nothing, if the tile is not
+// canonical (the caller then runs general tiles).  Lane l:
+//   A  loads its group with 16-byte loads and checks it;
+//   B  computes its key's usage from the byte polynomials (keys off the plan
+//      path: the warp-cooperative sweep) and the kernels' work counts;
+//   C  models its CX records, XW transformations per pass over the kernels
+//      (the constants of (kernel, xform) are warp-uniform: one broadcast
+//      load serves 32 records), then writes outputs / keeps its argmin.
+template <bool BEST>
+__device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsigned long long tb,
+                                           int lane, double &best_t, unsigned long long &best_i,
+                                           uint32_t &cnt_val)
+{
+    const SpaceDev &S = P.S;
+    const unsigned long long q0 = tb + (unsigned long long)lane * CX;
+    // ---- A ----
+    uint32_t acc = 0, s0, n0, m0, i0;
+    {
+        const uint4 *p = reinterpret_cast<const uint4 *>(P.skx + q0);
+        uint4 v[CX / 4];
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++) v[m] = __ldcs(p + m);
+        s0 = v[0].x;
+        acc = s0 & 0xffffu;   // transformation 0 first, so s0 + x == s0 ^ x
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++) {
+            acc |= (v[m].x ^ s0) ^ (uint32_t)(4 * m + 0);
+            acc |= (v[m].y ^ s0) ^ (uint32_t)(4 * m + 1);
+            acc |= (v[m].z ^ s0) ^ (uint32_t)(4 * m + 2);
+            acc |= (v[m].w ^ s0) ^ (uint32_t)(4 * m + 3);
+        }
+    }
+    auto same = [&](const uint32_t *arr, uint32_t &first) {
+        const uint4 *p = reinterpret_cast<const uint4 *>(arr + q0);
+        uint4 v[CX / 4];
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++) v[m] = __ldcs(p + m);
+        first = v[0].x;
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++)
+            acc |= (v[m].x ^ first) | (v[m].y ^ first) | (v[m].z ^ first) | (v[m].w ^ first);
+    };
+    same(P.nx, n0);
+    same(P.ny, m0);
+    same(P.iters, i0);
+    const uint32_t skel = s0 >> 16;
+    const uint32_t skel_l0 = __shfl_sync(FULL, skel, 0);   // (every lane: no short-circuit)
+    bool ok = acc == 0 && skel < S.n_skels && n0 - 1u < GROPHECY_MAX_DIM &&
+              m0 - 1u < GROPHECY_MAX_DIM && i0 >= 1 && skel == skel_l0;
+    if (ok) ok = S.skel[skel].n_xforms >= (uint32_t)CX;
+    if (!__all_sync(FULL, ok)) return false;
+
+    // ---- B ----
+    const SkelInfo &I = S.skel[skel];   // warp-uniform from here on
+    const uint32_t K = I.n_kernels, n_arrays = I.n_arrays;
+    const long long nxny = (long long)((unsigned long long)n0 * m0);
+    for (uint32_t k = 0; k < K; k++)
+        ws.cw[k][lane] = w_store(aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny));
+    const bool plan = n0 >= I.plan_tx && m0 >= I.plan_ty;
+    Usage u = {0ull, 0ull, 0.0, 0.0};
+    if (plan) {
+        const uint32_t stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
+        const unsigned long long *pp =
+            S.poly + I.poly_base + (size_t)((n0 & 7u) * 8u + (m0 & 7u)) * (2u * n_arrays * stride);
+        for (uint32_t a = 0; a < n_arrays; a++, pp += 2 * stride) {
+            const unsigned long long h = stride > 4 ? poly_eval<true>(pp, a8, b8)
+                                                    : poly_eval<false>(pp, a8, b8);
+            const unsigned long long d = stride > 4 ? poly_eval<true>(pp + stride, a8, b8)
+                                                    : poly_eval<false>(pp + stride, a8, b8);
+            // Eq. (1) per array, times added in array order (N6)
+            u.th = __dadd_rn(u.th, h ? __dadd_rn(P.pc.h2d.alpha_s,
+                                                 __dmul_rn(P.pc.h2d.beta_s_per_byte, __ull2double_rn(h)))
+                                     : 0.0);
+            u.td = __dadd_rn(u.td, d ? __dadd_rn(P.pc.d2h.alpha_s,
+                                                 __dmul_rn(P.pc.d2h.beta_s_per_byte, __ull2double_rn(d)))
+                                     : 0.0);
+            u.h += h;
+            u.d += d;
+        }
+    }
+    unsigned slow = __ballot_sync(FULL, !plan);
+    if (slow) {
+        while (slow) {
+            const int pos = __ffs(slow) - 1;
+            const unsigned long long k = ((unsigned long long)skel << 42) |
+                                         ((unsigned long long)__shfl_sync(FULL, n0, pos) << 21) |
+                                         __shfl_sync(FULL, m0, pos);
+            slow_usage(P.gS, k, P.pc, &ws.scratch, &ws.cres[pos], nullptr, lane);
+            slow &= slow - 1;
+            __syncwarp();
+        }
+        if (!plan) u = ws.cres[lane];
+    }
+    __syncwarp();
+
+    // ---- C ----
+    const uint32_t X = I.n_xforms, pim = I.per_iter_mask;
+    const double it = (double)i0;
+    const unsigned long long gi = P.base + q0;   // global index of the group's record 0
+    double bt = __longlong_as_double(0x7ff0000000000000LL);
+    int bx = -1;
+#pragma unroll 1
+    for (int x0 = 0; x0 < CX; x0 += XW) {
+        double ti[XW], to[XW];
+#pragma unroll
+        for (int j = 0; j < XW; j++) ti[j] = to[j] = 0.0;
+        const KxFast *F = S.kx_f + I.kx_base + x0;
+#pragma unroll 1
+        for (uint32_t k = 0; k < K; k++, F += X) {
+            const uint32_t w = ws.cw[k][lane];
+            double tk[XW];
+            bool gen[XW], any = false;
+#pragma unroll
+            for (int j = 0; j < XW; j++) {
+                tk[j] = fast_time(F[j], w, S.freq, S.rfreq, gen[j]);
+                any |= gen[j];
+            }
+            if (any) {
+                const long long Wi = aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny);
+                const uint32_t kxi = I.kx_base + k * X + x0;
+#pragma unroll
+                for (int j = 0; j < XW; j++)
+                    if (gen[j]) tk[j] = kernel_time(S, Wi, S.kx_j[kxi + j], kxi + j);
+            }
+            if ((pim >> k) & 1u) {
+#pragma unroll
+                for (int j = 0; j < XW; j++) ti[j] = __dadd_rn(ti[j], tk[j]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < XW; j++) to[j] = __dadd_rn(to[j], tk[j]);
+            }
+        }
+        // totals: run-once + iters x per-iteration + transfers
+        double tt[XW];
+#pragma unroll
+        for (int j = 0; j < XW; j++)
+            tt[j] = __dadd_rn(__dadd_rn(__dadd_rn(to[j], __dmul_rn(it, ti[j])), u.th), u.td);
+        if (BEST) {
+#pragma unroll
+            for (int j = 0; j < XW; j++)
+                if (tt[j] < bt) {   // records in index order: the first minimum stays
+                    bt = tt[j];
+                    bx = x0 + j;
+                }
+        } else {
+            const unsigned long long i = q0 + x0;
+#pragma unroll
+            for (int j = 0; j < XW; j++) {
+                __stcs(P.h2d + i + j, u.h);
+                __stcs(P.d2h + i + j, u.d);
+                __stcs(P.t + i + j, tt[j]);
+                if (P.p_iter) __stcs(P.p_iter + i + j, ti[j]);
+                if (P.p_once) __stcs(P.p_once + i + j, to[j]);
+                if (P.p_h2d) __stcs(P.p_h2d + i + j, u.th);
+                if (P.p_d2h) __stcs(P.p_d2h + i + j, u.td);
+            }
+        }
+    }
+    if (BEST) {
+        cnt_val += CX;
+        if (bx >= 0 && better(bt, gi + (unsigned)bx, best_t, best_i)) {
+            best_t = bt;
+            best_i = gi + (unsigned)bx;
+            ws.best_h[lane] = u.h;
+            ws.best_d[lane] = u.d;
+        }
+    }
+    __syncwarp();
+    return true;
+}
+template <bool BEST>
+__global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const Params P)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
+    __shared__ Best wbest[WARPS];
+    __shared__ bool am_last;
+
+    // running argmin kept lean in registers: (t, index) + counters; the
+    // winner's byte counts go to shared memory (rarely updated)
+    double best_t = __longlong_as_double(0x7ff0000000000000LL);
+    unsigned long long best_i = ~0ull;
+    uint32_t cnt_inv = 0, cnt_val = 0;
+    ws.best_h[lane] = 0;
+    ws.best_d[lane] = 0;
+    // tiles of CTILE records: canonical tiles take the one-group-per-lane
+    // path, the others four general 128-record tiles
+    const unsigned long long ntiles = (P.n + CTILE - 1) / CTILE;
+    const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
+    for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
+         tile += wstride) {
+        const unsigned long long tb = tile * CTILE;
+        // warm L2 with the records of this warp's next tile
+        if (lane < 4) {
+            const unsigned long long nt = tile + wstride;
+            if (nt < ntiles && P.aligned) {
+                const unsigned long long nb = nt * CTILE;
+                const unsigned long long cnt = min((unsigned long long)CTILE, P.n - nb);
+                const uint32_t *base = lane == 0 ? P.skx : lane == 1 ? P.nx : lane == 2 ? P.ny : P.iters;
+                const uint32_t bytes = (uint32_t)(cnt * 4) & ~15u;
+                if (bytes)
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;"
+                                 :: "l"(base + nb), "r"(bytes) : "memory");
+            }
+        }
+        if (P.aligned && tb + CTILE <= P.n &&
+            canon_tile<BEST>(P, ws, tb, lane, best_t, best_i, cnt_val))
+            continue;
+#pragma unroll 1
+        for (int sub = 0; sub < CTILE / WTILE; sub++) {
+            const unsigned long long t0 = tb + (unsigned long long)sub * WTILE;
+            if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
+        }
     }
     if (!BEST) return;
 
@@ -1186,7 +1393,7 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
                                                       sizeof(CtaSmem));
         if (occ_best < 1) occ_best = 1;
     }
-    const unsigned long long want = (n + (unsigned long long)WTILE * WARPS - 1) / ((unsigned long long)WTILE * WARPS);
+    const unsigned long long want = (n + (unsigned long long)CTILE * WARPS - 1) / ((unsigned long long)CTILE * WARPS);
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ_best, per_sm_cap);
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));

@@ -364,16 +364,20 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 kes.push_back(es); kd.push_back(d); ki.push_back(i); kj.push_back(j);
                 kg.push_back(g);
                 KxFast f;
-                if (j.flags & KXF_INFEASIBLE) {
-                    f.E = INFINITY; f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0;
+                // blocks = hi64(magic * (W + addend)) = ceil(W / ipb) for
+                // W < 2^31 (magic = ceil(2^64 / ipb), addend = ipb - 1; for
+                // ipb == 1: magic = 2^64 - 1, addend = 1).  Infeasible or huge
+                // ipb: sat32 = 2^32 - 1, so every record takes the general path.
+                const uint64_t m = j.ipb == 1 ? ~0ull : i.magic;
+                f.magic_lo = (uint32_t)m;
+                f.magic_hi = (uint32_t)(m >> 32);
+                f.addend = j.ipb == 1 ? 1u : j.ipb - 1u;
+                if ((j.flags & KXF_INFEASIBLE) || j.ipb > 0x80000000u) {
+                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0xffffffffu;
                 } else {
                     f.E = es.E; f.S = es.S; f.D = d.D; f.rD = d.rD;
                     f.sat32 = i.sat_blocks > 0xffffffffull ? 0xffffffffu : (uint32_t)i.sat_blocks;
                 }
-                const uint64_t m = j.ipb == 1 ? ~0ull : i.magic;
-                f.magic_lo = (uint32_t)m;
-                f.magic_hi = (uint32_t)(m >> 32);
-                f.ipb = j.ipb;
                 kf.push_back(f);
             }
     }
