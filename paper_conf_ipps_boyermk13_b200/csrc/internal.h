@@ -81,6 +81,8 @@ struct SkelPlanHost {
     uint32_t poly_stride = 0;
 };
 constexpr uint32_t POLY_CLASSES = 64;
+constexpr uint32_t SMALL_GRID_MAX = 1024;   // tabulated small grids per (kernel, xform)
+#define GROPHECY_TILE_CAP (1u << 21)        // tiles of 512 records per projection pass
 
 // P(a, b) of one byte polynomial (host and device share the formula; device
 // copy in project.cu).  a, b < 2^18.
@@ -115,6 +117,10 @@ struct SpaceDev {
     const KxG *kx_g;
     const KxFast *kx_f;
     const unsigned long long *poly;   // usage byte polynomials (all skeletons)
+    // small-grid kernel times: small_t[kxi * small_stride + blocks] for
+    // blocks < sat32 when sat32 <= small_stride (space.cpp small_grid_time)
+    const double *small_t;
+    uint32_t small_stride;
     uint32_t n_skels;
     uint32_t n_sm;
     double freq, rfreq;
@@ -130,6 +136,8 @@ struct grophecy_space {
     void *blob;                          // one device allocation for all tables
     size_t blob_bytes;
     grophecy_best_result *partials;      // best-mode per-block partials
+    uint32_t *tile_list;                 // pass 1 -> pass 2 tile list (GROPHECY_TILE_CAP)
+    unsigned int *tile_count;
     unsigned int *ticket;                // best-mode last-block counter
     unsigned long long *invalid_counter;
     uint32_t max_partials;

@@ -124,11 +124,12 @@ __device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned 
 }
 
 // Work-item count as stored for the model's fast path: W if 0 < W < 2^31,
-// else 0 (blocks = 0 < sat32 sends the record to the general path, which
-// recomputes W from the key).
+// 0 if W <= 0 (blocks = 0: the small-grid table gives t = 0), W_HUGE above
+// (the general path recomputes W from the key).
+constexpr uint32_t W_HUGE = 0xffffffffu;
 __device__ __forceinline__ uint32_t w_store(long long w)
 {
-    return (w > 0 && w < 0x80000000LL) ? (uint32_t)w : 0u;
+    return w <= 0 ? 0u : (w < 0x80000000LL ? (uint32_t)w : W_HUGE);
 }
 
 // One residue-class byte polynomial P(a, b) (plan.cpp; internal.h layout),
@@ -764,16 +765,16 @@ struct CtaSmem {
 
 // Saturated-grid kernel time (DESIGN.md §3 N5, saturated reduction) of one
 // (record, kernel) from the packed constants and the stored work count w
-// (w_store): cyc = E rep + S rep, rep = blocks / D, t = cyc / freq, both
-// divisions by Markstein's correction (bitwise the IEEE quotients).  gen is
-// set when the record must take the general path instead (small grid, huge
-// or zero work, infeasible) — the returned value is then meaningless.
+// (w_store, < 2^31 here): cyc = E rep + S rep, rep = blocks / D,
+// t = cyc / freq, both divisions by Markstein's correction (bitwise the IEEE
+// quotients).  gen is set when the grid is not saturated (or the pair is
+// infeasible) — the returned value is then meaningless and gen_time decides.
 __device__ __forceinline__ double fast_time(const KxFast &f, uint32_t w, double freq, double rfreq,
-                                            bool &gen)
+                                            bool &gen, uint32_t &blocks)
 {
     const uint32_t w1 = w + f.addend;
     const unsigned long long lo = (unsigned long long)f.magic_lo * w1;
-    const uint32_t blocks = (uint32_t)(((unsigned long long)f.magic_hi * w1 + (lo >> 32)) >> 32);
+    blocks = (uint32_t)(((unsigned long long)f.magic_hi * w1 + (lo >> 32)) >> 32);
     gen = blocks < f.sat32;
     const double bb = __uint2double_rn(blocks);
     const double q = __dmul_rn(bb, f.rD);
@@ -781,6 +782,18 @@ __device__ __forceinline__ double fast_time(const KxFast &f, uint32_t w, double 
     const double cyc = __dadd_rn(__dmul_rn(f.E, rep), __dmul_rn(f.S, rep));
     const double q2 = __dmul_rn(cyc, rfreq);
     return __fma_rn(__fma_rn(-q2, freq, cyc), rfreq, q2);
+}
+
+// Kernel time off the saturated path: the small-grid table when the pair is
+// tabulated (space.cpp), else the definition step by step (infeasible pairs,
+// grids beyond the table, huge work counts).  Wi() recomputes the work count.
+template <class WiF>
+__device__ __forceinline__ double gen_time(const SpaceDev &S, uint32_t kxi, uint32_t sat32,
+                                           uint32_t w, uint32_t blocks, WiF Wi)
+{
+    if (sat32 <= S.small_stride && w != W_HUGE)
+        return __ldg(&S.small_t[(size_t)kxi * S.small_stride + blocks]);
+    return kernel_time(S, Wi(), S.kx_j[kxi], kxi);
 }
 
 // Model of NJ records of one skeleton at once (NJ independent dependency
@@ -803,10 +816,14 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
         bool gen[NJ];
         KxFast F0;
         if (SAMEX) F0 = S.kx_f[kb + x[0]];   // one constant load shared by the NJ records
+        uint32_t w[NJ], blocks[NJ], sat[NJ];
 #pragma unroll
         for (int j = 0; j < NJ; j++) {
             const KxFast F = SAMEX ? F0 : S.kx_f[kb + x[j]];
-            tk[j] = fast_time(F, ws.slot_w[ls[j]][k], S.freq, S.rfreq, gen[j]);
+            w[j] = ws.slot_w[ls[j]][k];
+            tk[j] = fast_time(F, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
+            gen[j] |= w[j] == W_HUGE;
+            sat[j] = F.sat32;
         }
         bool any = false;
 #pragma unroll
@@ -816,10 +833,10 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
             for (int j = 0; j < NJ; j++)
                 if (gen[j]) {
                     const unsigned long long kk = ws.slot_key[ls[j]];
-                    const long long Wi = aff8(__ldg(&S.kern_work[I.k_base + k]),
-                                              (long long)((kk >> 21) & 0x1fffffull),
-                                              (long long)(kk & 0x1fffffull));
-                    tk[j] = kernel_time(S, Wi, S.kx_j[kb + x[j]], kb + x[j]);
+                    tk[j] = gen_time(S, kb + x[j], sat[j], w[j], blocks[j], [&] {
+                        return aff8(__ldg(&S.kern_work[I.k_base + k]),
+                                    (long long)((kk >> 21) & 0x1fffffull), (long long)(kk & 0x1fffffull));
+                    });
                 }
         }
         if ((pim >> k) & 1u) {
@@ -853,6 +870,8 @@ struct Params {
     grophecy_best_result *out;
     int accumulate;
     int aligned;    // record arrays 16-byte aligned -> vector loads
+    uint32_t *tile_list;      // pass 1 -> pass 2: tiles left to the general path
+    unsigned int *tile_count;
 };
 
 // Record validity (include/grophecy.h) and its usage key (skeleton, nx, ny).
@@ -1151,8 +1170,13 @@ __device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsign
     const SkelInfo &I = S.skel[skel];   // warp-uniform from here on
     const uint32_t K = I.n_kernels, n_arrays = I.n_arrays;
     const long long nxny = (long long)((unsigned long long)n0 * m0);
-    for (uint32_t k = 0; k < K; k++)
-        ws.cw[k][lane] = w_store(aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny));
+    bool huge = false;
+    for (uint32_t k = 0; k < K; k++) {
+        const uint32_t w = w_store(aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny));
+        ws.cw[k][lane] = w;
+        huge |= w == W_HUGE;
+    }
+    if (__any_sync(FULL, huge)) return false;   // (nothing written yet)
     const bool plan = n0 >= I.plan_tx && m0 >= I.plan_ty;
     Usage u = {0ull, 0ull, 0.0, 0.0};
     if (plan) {
@@ -1207,17 +1231,22 @@ __device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsign
             const uint32_t w = ws.cw[k][lane];
             double tk[XW];
             bool gen[XW], any = false;
+            uint32_t blocks[XW], sat[XW];
 #pragma unroll
             for (int j = 0; j < XW; j++) {
-                tk[j] = fast_time(F[j], w, S.freq, S.rfreq, gen[j]);
+                const KxFast f = F[j];
+                tk[j] = fast_time(f, w, S.freq, S.rfreq, gen[j], blocks[j]);
+                sat[j] = f.sat32;
                 any |= gen[j];
             }
             if (any) {
-                const long long Wi = aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny);
                 const uint32_t kxi = I.kx_base + k * X + x0;
 #pragma unroll
                 for (int j = 0; j < XW; j++)
-                    if (gen[j]) tk[j] = kernel_time(S, Wi, S.kx_j[kxi + j], kxi + j);
+                    if (gen[j])
+                        tk[j] = gen_time(S, kxi + j, sat[j], w, blocks[j], [&] {
+                            return aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny);
+                        });
             }
             if ((pim >> k) & 1u) {
 #pragma unroll
@@ -1265,54 +1294,14 @@ __device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsign
     __syncwarp();
     return true;
 }
-template <bool BEST>
-__global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const Params P)
+// Block-level epilogue of best mode: warp -> CTA -> grid argmin (last-block
+// pattern; the last block also resets the ticket for reuse).
+__device__ __forceinline__ void finish_best(const Params &P, WarpSmem &ws, int lane, int warp,
+                                            double best_t, unsigned long long best_i,
+                                            uint32_t cnt_inv, uint32_t cnt_val)
 {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int lane = threadIdx.x & 31;
-    const int warp = threadIdx.x >> 5;
-    WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
     __shared__ Best wbest[WARPS];
     __shared__ bool am_last;
-
-    // running argmin kept lean in registers: (t, index) + counters; the
-    // winner's byte counts go to shared memory (rarely updated)
-    double best_t = __longlong_as_double(0x7ff0000000000000LL);
-    unsigned long long best_i = ~0ull;
-    uint32_t cnt_inv = 0, cnt_val = 0;
-    ws.best_h[lane] = 0;
-    ws.best_d[lane] = 0;
-    // tiles of CTILE records: canonical tiles take the one-group-per-lane
-    // path, the others four general 128-record tiles
-    const unsigned long long ntiles = (P.n + CTILE - 1) / CTILE;
-    const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
-    for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
-         tile += wstride) {
-        const unsigned long long tb = tile * CTILE;
-        // warm L2 with the records of this warp's next tile
-        if (lane < 4) {
-            const unsigned long long nt = tile + wstride;
-            if (nt < ntiles && P.aligned) {
-                const unsigned long long nb = nt * CTILE;
-                const unsigned long long cnt = min((unsigned long long)CTILE, P.n - nb);
-                const uint32_t *base = lane == 0 ? P.skx : lane == 1 ? P.nx : lane == 2 ? P.ny : P.iters;
-                const uint32_t bytes = (uint32_t)(cnt * 4) & ~15u;
-                if (bytes)
-                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;"
-                                 :: "l"(base + nb), "r"(bytes) : "memory");
-            }
-        }
-        if (P.aligned && tb + CTILE <= P.n &&
-            canon_tile<BEST>(P, ws, tb, lane, best_t, best_i, cnt_val))
-            continue;
-#pragma unroll 1
-        for (int sub = 0; sub < CTILE / WTILE; sub++) {
-            const unsigned long long t0 = tb + (unsigned long long)sub * WTILE;
-            if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
-        }
-    }
-    if (!BEST) return;
-
     // ---- argmin: warp -> CTA -> grid (last-block pattern) ----
     Best mine;
     mine.t = best_t;
@@ -1363,6 +1352,75 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) project_kernel(const P
     }
 }
 
+// Pass 1 of a projection (persistent): every tile of CTILE records that is
+// canonical is projected here; the others (and the ragged tail) are appended
+// to the space's tile list for pass 2.
+template <bool BEST>
+__global__ void __launch_bounds__(THREADS, GROPHECY_MINB) canon_kernel(const Params P)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
+    // running argmin kept lean in registers: (t, index) + counters; the
+    // winner's byte counts go to shared memory (rarely updated)
+    double best_t = __longlong_as_double(0x7ff0000000000000LL);
+    unsigned long long best_i = ~0ull;
+    uint32_t cnt_val = 0;
+    ws.best_h[lane] = 0;
+    ws.best_d[lane] = 0;
+    const unsigned long long ntiles = (P.n + CTILE - 1) / CTILE;
+    const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
+    for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
+         tile += wstride) {
+        const unsigned long long tb = tile * CTILE;
+        // warm L2 with the records of this warp's next tile
+        if (lane < 4) {
+            const unsigned long long nt = tile + wstride;
+            if (nt < ntiles && P.aligned) {
+                const unsigned long long nb = nt * CTILE;
+                const unsigned long long cnt = min((unsigned long long)CTILE, P.n - nb);
+                const uint32_t *base = lane == 0 ? P.skx : lane == 1 ? P.nx : lane == 2 ? P.ny : P.iters;
+                const uint32_t bytes = (uint32_t)(cnt * 4) & ~15u;
+                if (bytes)
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;"
+                                 :: "l"(base + nb), "r"(bytes) : "memory");
+            }
+        }
+        if (!(P.aligned && tb + CTILE <= P.n &&
+              canon_tile<BEST>(P, ws, tb, lane, best_t, best_i, cnt_val)) &&
+            lane == 0)
+            P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)tile;
+    }
+    if (BEST) finish_best(P, ws, lane, warp, best_t, best_i, 0u, cnt_val);
+}
+
+// Pass 2: the listed tiles as general 128-record tiles (any layout).
+template <bool BEST>
+__global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const Params P)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
+    double best_t = __longlong_as_double(0x7ff0000000000000LL);
+    unsigned long long best_i = ~0ull;
+    uint32_t cnt_inv = 0, cnt_val = 0;
+    ws.best_h[lane] = 0;
+    ws.best_d[lane] = 0;
+    const unsigned count = *(volatile unsigned *)P.tile_count;
+    const unsigned wstride = gridDim.x * WARPS;
+    for (unsigned e = blockIdx.x * WARPS + warp; e < count; e += wstride) {
+        const unsigned long long tb = (unsigned long long)P.tile_list[e] * CTILE;
+#pragma unroll 1
+        for (int sub = 0; sub < CTILE / WTILE; sub++) {
+            const unsigned long long t0 = tb + (unsigned long long)sub * WTILE;
+            if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
+        }
+    }
+    if (BEST) finish_best(P, ws, lane, warp, best_t, best_i, cnt_inv, cnt_val);
+}
+
 __global__ void combine_kernel(const grophecy_best_result *in, uint32_t count,
                                grophecy_best_result *out)
 {
@@ -1377,10 +1435,11 @@ static void set_smem_attrs()
 {
     static bool done = false;
     if (done) return;
-    cudaFuncSetAttribute(project_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)sizeof(CtaSmem));
-    cudaFuncSetAttribute(project_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)sizeof(CtaSmem));
+    const int sm = (int)sizeof(CtaSmem);
+    cudaFuncSetAttribute(canon_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+    cudaFuncSetAttribute(canon_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+    cudaFuncSetAttribute(general_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+    cudaFuncSetAttribute(general_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     done = true;
 }
 
@@ -1389,7 +1448,7 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
     static int occ_best = 0;
     set_smem_attrs();
     if (!occ_best) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_best, project_kernel<true>, THREADS,
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_best, canon_kernel<true>, THREADS,
                                                       sizeof(CtaSmem));
         if (occ_best < 1) occ_best = 1;
     }
@@ -1397,6 +1456,43 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ_best, per_sm_cap);
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
+}
+
+// One projection = per chunk of at most GROPHECY_TILE_CAP tiles: reset the
+// tile list, pass 1 (canonical tiles), pass 2 (the listed tiles).  Best mode
+// accumulates the chunks into P.out.
+template <bool BEST>
+static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
+{
+    const unsigned long long cap = (unsigned long long)GROPHECY_TILE_CAP * CTILE;
+    const unsigned long long n = P.n;
+    unsigned long long off = 0;
+    do {
+        Params Q = P;
+        Q.n = std::min(cap, n - off);
+        Q.skx += off; Q.nx += off; Q.ny += off; Q.iters += off;
+        Q.base += off;
+        if (!BEST) {
+            Q.h2d += off; Q.d2h += off; Q.t += off;
+            if (Q.p_iter) Q.p_iter += off;
+            if (Q.p_once) Q.p_once += off;
+            if (Q.p_h2d) Q.p_h2d += off;
+            if (Q.p_d2h) Q.p_d2h += off;
+        } else if (off) {
+            Q.accumulate = 1;
+        }
+        cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, sizeof(unsigned int), st);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(tile count)");
+        const int grid = grid_for(s, Q.n, 32);
+        canon_kernel<BEST><<<grid, THREADS, sizeof(CtaSmem), st>>>(Q);
+        Q.accumulate = BEST ? 1 : 0;   // pass 2 merges into pass 1's result
+        general_kernel<BEST><<<grid, THREADS, sizeof(CtaSmem), st>>>(Q);
+        count_launch(2);
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_fail(e, BEST ? "projection (best) launch" : "projection (eval) launch");
+        off += Q.n;
+    } while (off < n);
+    return GROPHECY_OK;
 }
 
 static int check_batch(const grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b)
@@ -1432,6 +1528,8 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
     P.ticket = s->ticket;
     P.out = nullptr;
     P.accumulate = 0;
+    P.tile_list = s->tile_list;
+    P.tile_count = s->tile_count;
     const uintptr_t m = (uintptr_t)b->skx | (uintptr_t)b->nx | (uintptr_t)b->ny | (uintptr_t)b->iters;
     P.aligned = (m & 15u) == 0;
     return P;
@@ -1443,12 +1541,7 @@ int launch_best(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch
     Params P = make_params(s, pc, b);
     P.out = dout;
     P.accumulate = accumulate;
-    const int grid = grid_for(s, b->n, 32);
-    project_kernel<true><<<grid, THREADS, sizeof(CtaSmem), st>>>(P);
-    count_launch();
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_fail(e, "project_kernel<best> launch");
-    return GROPHECY_OK;
+    return launch_passes<true>(s, P, st);
 }
 
 }  // namespace grophecy
@@ -1478,12 +1571,7 @@ int grophecy_eval_parts(const grophecy_space *s, const grophecy_pcie *pc, const 
         P.p_h2d = parts->t_h2d_s;
         P.p_d2h = parts->t_d2h_s;
     }
-    const int grid = grid_for(s, b->n, 32);
-    project_kernel<false><<<grid, THREADS, sizeof(CtaSmem), (cudaStream_t)stream>>>(P);
-    count_launch();
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_fail(e, "project_kernel<eval> launch");
-    return GROPHECY_OK;
+    return launch_passes<false>(s, P, (cudaStream_t)stream);
 }
 
 int grophecy_eval(const grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,

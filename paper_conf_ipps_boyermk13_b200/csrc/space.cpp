@@ -212,6 +212,39 @@ static void precompute(const grophecy_kx_desc &c, const grophecy_gpu_model &g, K
     es.S = gg.dd * (mwp - 1.0) * c.synch_insts * (double)occ;
 }
 
+// Kernel time on a grid of `blocks` < sat_blocks blocks: the general branch of
+// DESIGN.md §3 N5 step by step, in the definition's operation order (the same
+// order as the device's kernel_time and the oracle).  Tabulated at space
+// creation: on such grids the time depends on (kernel, xform, blocks) only.
+static double small_grid_time(const KxJ &J, const KxG &G, uint64_t nsm, double freq,
+                              uint64_t blocks)
+{
+    if (blocks == 0) return 0.0;
+    const uint64_t asm_ = std::min<uint64_t>(nsm, blocks);
+    uint64_t abps = blocks / asm_ + (blocks % asm_ != 0);
+    if ((uint64_t)J.occ < abps) abps = J.occ;
+    const double N = (double)(abps * (uint64_t)J.wpb);
+    const double rep = (double)blocks / (double)(abps * asm_);
+    double cyc;
+    if (J.flags & KXF_NOMEM) {
+        cyc = G.comp * N * rep;
+    } else {
+        const double mpk = G.bwr / (double)asm_;
+        const double mwp = dmin(dmin(G.mwp0, mpk), N);
+        const double cwp = dmin(G.cwpf, N);
+        const double cpm_term = G.cpm * (mwp - 1.0);
+        if (mwp == N && cwp == N)
+            cyc = (G.memc + G.comp + cpm_term) * rep;
+        else if (cwp >= mwp || G.comp > G.memc)
+            cyc = (G.memc * N / mwp + cpm_term) * rep;
+        else
+            cyc = (G.ml + G.comp * N) * rep;
+        const double sync = G.dd * (mwp - 1.0) * G.synch * (double)abps * rep;
+        cyc = cyc + sync;
+    }
+    return cyc / freq;
+}
+
 }  // namespace grophecy
 
 using namespace grophecy;
@@ -382,6 +415,17 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             }
     }
 
+    // ---- small-grid table: t(kernel, xform, blocks) for blocks < sat32 ----
+    uint32_t max_sat = 0;
+    for (const KxFast &f : kf)
+        if (f.sat32 != 0xffffffffu) max_sat = std::max(max_sat, f.sat32);
+    const uint32_t small_stride = std::min<uint32_t>(max_sat, SMALL_GRID_MAX);
+    std::vector<double> small((size_t)kf.size() * small_stride, 0.0);
+    for (size_t q = 0; q < kf.size(); q++)
+        if (kf[q].sat32 <= small_stride)
+            for (uint32_t b = 0; b < kf[q].sat32; b++)
+                small[q * small_stride + b] = small_grid_time(kj[q], kg[q], gpu->n_sm, gpu->freq_hz, b);
+
     // ---- one device blob ----
     struct Part { const void *src; size_t bytes; size_t off; };
     std::vector<Part> parts = {
@@ -397,6 +441,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {kg.data(), kg.size() * sizeof(KxG), 0},
         {poly.data(), poly.size() * sizeof(unsigned long long), 0},
         {kf.data(), kf.size() * sizeof(KxFast), 0},
+        {small.data(), small.size() * sizeof(double), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -427,7 +472,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     sp->max_partials = (uint32_t)nsm * 32u;
     size_t scratch_off = align_up(total, 256);
     size_t part_bytes = sizeof(grophecy_best_result) * sp->max_partials;
-    size_t blob = scratch_off + align_up(part_bytes, 256) + 256 + align_up(sizeof(SpaceDev), 256);
+    const size_t list_bytes = (size_t)GROPHECY_TILE_CAP * sizeof(uint32_t);
+    size_t blob = scratch_off + align_up(part_bytes, 256) + 256 + align_up(sizeof(SpaceDev), 256) +
+                  list_bytes;
     if ((e = cudaMalloc(&sp->blob, blob)) != cudaSuccess) return bail(e, "cudaMalloc(space)");
     sp->blob_bytes = blob;
     if ((e = cudaMemcpy(sp->blob, host.data(), total, cudaMemcpyHostToDevice)) != cudaSuccess)
@@ -437,6 +484,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     unsigned char *ctr = base + scratch_off + align_up(part_bytes, 256);
     sp->ticket = (unsigned int *)ctr;
     sp->invalid_counter = (unsigned long long *)(ctr + 64);
+    sp->tile_count = (unsigned int *)(ctr + 128);
+    sp->tile_list = (uint32_t *)(ctr + 256 + align_up(sizeof(SpaceDev), 256));
     if ((e = cudaMemset(ctr, 0, 256)) != cudaSuccess) return bail(e, "cudaMemset(space)");
 
     SpaceDev &D = sp->dev;
@@ -452,6 +501,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.kx_g = (const KxG *)(base + parts[9].off);
     D.poly = (const unsigned long long *)(base + parts[10].off);
     D.kx_f = (const KxFast *)(base + parts[11].off);
+    D.small_t = (const double *)(base + parts[12].off);
+    D.small_stride = small_stride;
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;
     D.freq = gpu->freq_hz;
