@@ -32,8 +32,8 @@ enum : uint32_t { KXF_INFEASIBLE = 1u, KXF_NOMEM = 2u, KXF_PER_ITER = 4u };
 // (always the general path).  Work counts outside (0, 2^31) are stored as 0,
 // which also selects the general path (blocks = 0 < sat32).
 struct __align__(16) KxFast {
-    double E, S, D, rD;
-    uint32_t magic_lo, magic_hi, sat32, addend;
+    uint32_t magic_lo, magic_hi, sat32, addend;   // first: the chain starts with blocks
+    double D, rD, E, S;                           // E = +inf iff infeasible
 };
 
 // General-grid constants (small grids / huge W), read only off the fast path.
@@ -46,7 +46,7 @@ struct SkelInfo {
     uint32_t k_base;   // into kern_work / kern_flags
     uint32_t a_base;   // into arrays
     uint32_t kx_base;  // into kx tables
-    uint32_t flags;    // GROPHECY_SKEL_* (HULL) | SKF_STRIDED
+    uint32_t flags;    // GROPHECY_SKEL_* (HULL) | SKF_*
     // usage plan (plan.cpp): valid for nx >= plan_tx and ny >= plan_ty; its
     // byte polynomials at poly[poly_base + ...] (SkelPlanHost layout)
     uint32_t plan_tx, plan_ty, poly_base, poly_stride;
@@ -59,7 +59,11 @@ struct ArrayDev {
     uint32_t lr, lc;    // lcm of the regions' row / column steps (1 = dense array)
     uint32_t pad0, pad1;
 };
-enum : uint32_t { SKF_STRIDED = 1u << 16 };   // some region has a step > 1
+enum : uint32_t {
+    SKF_STRIDED = 1u << 16,     // some region has a step > 1
+    SKF_TABULATED = 1u << 17,   // every (kernel, xform) off the saturated path is in the
+                                // small-grid table or infeasible (canonical kernel eligible)
+};
 
 constexpr uint32_t PLAN_MAX_EXPR = 128;   // < 256: programs pack u8 indices
 

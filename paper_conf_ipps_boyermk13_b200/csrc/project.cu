@@ -737,30 +737,37 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
 // XW transformations per model pass.
 constexpr int CX = 16;
 constexpr int CTILE = 32 * CX;
-constexpr int XW = 4;
+#ifndef GROPHECY_XW
+#define GROPHECY_XW 4
+#endif
+constexpr int XW = GROPHECY_XW;
+#ifndef GROPHECY_CMINB
+#define GROPHECY_CMINB 2
+#endif
 
-// Per-warp shared memory (dynamic; > 48 KB per CTA needs the opt-in attribute).
+// Per-warp shared memory of the general kernel (dynamic; > 48 KB per CTA
+// needs the opt-in attribute).
 struct WarpSmem {
-    WarpScratch scratch;                            // usage plans / general sweep
-    union {
-        struct {                                    // general tiles
-            unsigned long long slot_key[SLOT_CAP];  // distinct keys of the chunk
-            Usage res[SLOT_CAP];                    // their usage
-            uint32_t slot_w[SLOT_CAP][MAXK + 1];    // their work-item counts (w_store; padded row)
-            unsigned long long rec_key[WTILE];      // the tile's records after phase A
-            uint32_t rec_skx[WTILE], rec_it[WTILE];
-            int rec_slot[WTILE];
-            uint8_t plan_pos[MAX_SEG];              // plan keys of the current slot group
-        };
-        struct {                                    // canonical tiles
-            uint32_t cw[MAXK][32];                  // work counts (w_store), [kernel][lane]
-            Usage cres[32];                         // usage of keys off the plan path
-        };
-    };
-    unsigned long long best_h[32], best_d[32];      // bytes of each lane's running best
+    WarpScratch scratch;                        // usage plans / general sweep
+    unsigned long long slot_key[SLOT_CAP];      // distinct keys of the chunk
+    Usage res[SLOT_CAP];                        // their usage
+    uint32_t slot_w[SLOT_CAP][MAXK + 1];        // their work-item counts (w_store; padded row)
+    unsigned long long rec_key[WTILE];          // the tile's records after phase A
+    uint32_t rec_skx[WTILE], rec_it[WTILE];
+    int rec_slot[WTILE];
+    uint8_t plan_pos[MAX_SEG];                  // plan keys of the current slot group
+    unsigned long long best_h[32], best_d[32];  // bytes of each lane's running best
+};
+// ... and of the canonical kernel.
+struct CanonSmem {
+    uint32_t cw[MAXK][32];                      // work counts (w_store), [kernel][lane]
+    unsigned long long best_h[32], best_d[32];
 };
 struct CtaSmem {
     WarpSmem w[WARPS];
+};
+struct CanonCtaSmem {
+    CanonSmem w[WARPS];
 };
 
 // Saturated-grid kernel time (DESIGN.md §3 N5, saturated reduction) of one
@@ -789,10 +796,11 @@ __device__ __forceinline__ double fast_time(const KxFast &f, uint32_t w, double 
 // grids beyond the table, huge work counts).  Wi() recomputes the work count.
 template <class WiF>
 __device__ __forceinline__ double gen_time(const SpaceDev &S, uint32_t kxi, uint32_t sat32,
-                                           uint32_t w, uint32_t blocks, WiF Wi)
+                                           double E, uint32_t w, uint32_t blocks, WiF Wi)
 {
     if (sat32 <= S.small_stride && w != W_HUGE)
         return __ldg(&S.small_t[(size_t)kxi * S.small_stride + blocks]);
+    if (E == __longlong_as_double(0x7ff0000000000000LL)) return E;   // infeasible: +inf
     return kernel_time(S, Wi(), S.kx_j[kxi], kxi);
 }
 
@@ -817,6 +825,7 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
         KxFast F0;
         if (SAMEX) F0 = S.kx_f[kb + x[0]];   // one constant load shared by the NJ records
         uint32_t w[NJ], blocks[NJ], sat[NJ];
+        double E[NJ];
 #pragma unroll
         for (int j = 0; j < NJ; j++) {
             const KxFast F = SAMEX ? F0 : S.kx_f[kb + x[j]];
@@ -824,6 +833,7 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
             tk[j] = fast_time(F, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
             gen[j] |= w[j] == W_HUGE;
             sat[j] = F.sat32;
+            E[j] = F.E;
         }
         bool any = false;
 #pragma unroll
@@ -833,7 +843,7 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
             for (int j = 0; j < NJ; j++)
                 if (gen[j]) {
                     const unsigned long long kk = ws.slot_key[ls[j]];
-                    tk[j] = gen_time(S, kb + x[j], sat[j], w[j], blocks[j], [&] {
+                    tk[j] = gen_time(S, kb + x[j], sat[j], E[j], w[j], blocks[j], [&] {
                         return aff8(__ldg(&S.kern_work[I.k_base + k]),
                                     (long long)((kk >> 21) & 0x1fffffull), (long long)(kk & 0x1fffffull));
                     });
@@ -1123,7 +1133,7 @@ __device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsi
 //      (the constants of (kernel, xform) are warp-uniform: one broadcast
 //      load serves 32 records), then writes outputs / keeps its argmin.
 template <bool BEST>
-__device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsigned long long tb,
+__device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsigned long long tb,
                                            int lane, double &best_t, unsigned long long &best_i,
                                            uint32_t &cnt_val)
 {
@@ -1163,7 +1173,7 @@ __device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsign
     const uint32_t skel_l0 = __shfl_sync(FULL, skel, 0);   // (every lane: no short-circuit)
     bool ok = acc == 0 && skel < S.n_skels && n0 - 1u < GROPHECY_MAX_DIM &&
               m0 - 1u < GROPHECY_MAX_DIM && i0 >= 1 && skel == skel_l0;
-    if (ok) ok = S.skel[skel].n_xforms >= (uint32_t)CX;
+    if (ok) ok = S.skel[skel].n_xforms >= (uint32_t)CX && (S.skel[skel].flags & SKF_TABULATED);
     if (!__all_sync(FULL, ok)) return false;
 
     // ---- B ----
@@ -1177,9 +1187,10 @@ __device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsign
         huge |= w == W_HUGE;
     }
     if (__any_sync(FULL, huge)) return false;   // (nothing written yet)
-    const bool plan = n0 >= I.plan_tx && m0 >= I.plan_ty;
+    // keys off the plan path (small sizes, strided, hull): general tiles
+    if (!__all_sync(FULL, n0 >= I.plan_tx && m0 >= I.plan_ty)) return false;
     Usage u = {0ull, 0ull, 0.0, 0.0};
-    if (plan) {
+    {
         const uint32_t stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
         const unsigned long long *pp =
             S.poly + I.poly_base + (size_t)((n0 & 7u) * 8u + (m0 & 7u)) * (2u * n_arrays * stride);
@@ -1199,21 +1210,6 @@ __device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsign
             u.d += d;
         }
     }
-    unsigned slow = __ballot_sync(FULL, !plan);
-    if (slow) {
-        while (slow) {
-            const int pos = __ffs(slow) - 1;
-            const unsigned long long k = ((unsigned long long)skel << 42) |
-                                         ((unsigned long long)__shfl_sync(FULL, n0, pos) << 21) |
-                                         __shfl_sync(FULL, m0, pos);
-            slow_usage(P.gS, k, P.pc, &ws.scratch, &ws.cres[pos], nullptr, lane);
-            slow &= slow - 1;
-            __syncwarp();
-        }
-        if (!plan) u = ws.cres[lane];
-    }
-    __syncwarp();
-
     // ---- C ----
     const uint32_t X = I.n_xforms, pim = I.per_iter_mask;
     const double it = (double)i0;
@@ -1232,21 +1228,24 @@ __device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsign
             double tk[XW];
             bool gen[XW], any = false;
             uint32_t blocks[XW], sat[XW];
+            double E[XW];
 #pragma unroll
             for (int j = 0; j < XW; j++) {
                 const KxFast f = F[j];
                 tk[j] = fast_time(f, w, S.freq, S.rfreq, gen[j], blocks[j]);
                 sat[j] = f.sat32;
+                E[j] = f.E;
                 any |= gen[j];
             }
             if (any) {
+                // off the saturated path: the small-grid table (SKF_TABULATED), or infeasible
                 const uint32_t kxi = I.kx_base + k * X + x0;
 #pragma unroll
                 for (int j = 0; j < XW; j++)
                     if (gen[j])
-                        tk[j] = gen_time(S, kxi + j, sat[j], w, blocks[j], [&] {
-                            return aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny);
-                        });
+                        tk[j] = sat[j] <= S.small_stride
+                                    ? __ldg(&S.small_t[(size_t)(kxi + j) * S.small_stride + blocks[j]])
+                                    : E[j];
             }
             if ((pim >> k) & 1u) {
 #pragma unroll
@@ -1296,7 +1295,8 @@ __device__ __forceinline__ bool canon_tile(const Params &P, WarpSmem &ws, unsign
 }
 // Block-level epilogue of best mode: warp -> CTA -> grid argmin (last-block
 // pattern; the last block also resets the ticket for reuse).
-__device__ __forceinline__ void finish_best(const Params &P, WarpSmem &ws, int lane, int warp,
+__device__ __forceinline__ void finish_best(const Params &P, const unsigned long long *best_h,
+                                            const unsigned long long *best_d, int lane, int warp,
                                             double best_t, unsigned long long best_i,
                                             uint32_t cnt_inv, uint32_t cnt_val)
 {
@@ -1306,8 +1306,8 @@ __device__ __forceinline__ void finish_best(const Params &P, WarpSmem &ws, int l
     Best mine;
     mine.t = best_t;
     mine.i = best_i;
-    mine.h = ws.best_h[lane];
-    mine.d = ws.best_d[lane];
+    mine.h = best_h[lane];
+    mine.d = best_d[lane];
     mine.ninv = cnt_inv;
     mine.nval = cnt_val;
     mine = warp_best(mine);
@@ -1356,12 +1356,12 @@ __device__ __forceinline__ void finish_best(const Params &P, WarpSmem &ws, int l
 // canonical is projected here; the others (and the ragged tail) are appended
 // to the space's tile list for pass 2.
 template <bool BEST>
-__global__ void __launch_bounds__(THREADS, GROPHECY_MINB) canon_kernel(const Params P)
+__global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Params P)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
+    CanonSmem &ws = reinterpret_cast<CanonCtaSmem *>(smem_raw)->w[warp];
     // running argmin kept lean in registers: (t, index) + counters; the
     // winner's byte counts go to shared memory (rarely updated)
     double best_t = __longlong_as_double(0x7ff0000000000000LL);
@@ -1392,7 +1392,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) canon_kernel(const Par
             lane == 0)
             P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)tile;
     }
-    if (BEST) finish_best(P, ws, lane, warp, best_t, best_i, 0u, cnt_val);
+    if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, 0u, cnt_val);
 }
 
 // Pass 2: the listed tiles as general 128-record tiles (any layout).
@@ -1418,7 +1418,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
             if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
         }
     }
-    if (BEST) finish_best(P, ws, lane, warp, best_t, best_i, cnt_inv, cnt_val);
+    if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, cnt_inv, cnt_val);
 }
 
 __global__ void combine_kernel(const grophecy_best_result *in, uint32_t count,
@@ -1435,25 +1435,29 @@ static void set_smem_attrs()
 {
     static bool done = false;
     if (done) return;
-    const int sm = (int)sizeof(CtaSmem);
-    cudaFuncSetAttribute(canon_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
-    cudaFuncSetAttribute(canon_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+    const int sm = (int)sizeof(CtaSmem), cs = (int)sizeof(CanonCtaSmem);
+    cudaFuncSetAttribute(canon_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
+    cudaFuncSetAttribute(canon_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
     cudaFuncSetAttribute(general_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     cudaFuncSetAttribute(general_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     done = true;
 }
 
-static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_cap)
+static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_cap, bool canon)
 {
-    static int occ_best = 0;
+    static int occ[2] = {0, 0};
     set_smem_attrs();
-    if (!occ_best) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_best, canon_kernel<true>, THREADS,
-                                                      sizeof(CtaSmem));
-        if (occ_best < 1) occ_best = 1;
+    if (!occ[canon]) {
+        if (canon)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], canon_kernel<true>, THREADS,
+                                                          sizeof(CanonCtaSmem));
+        else
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], general_kernel<true>, THREADS,
+                                                          sizeof(CtaSmem));
+        if (occ[canon] < 1) occ[canon] = 1;
     }
     const unsigned long long want = (n + (unsigned long long)CTILE * WARPS - 1) / ((unsigned long long)CTILE * WARPS);
-    unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ_best, per_sm_cap);
+    unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ[canon], per_sm_cap);
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
 }
@@ -1483,8 +1487,8 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         }
         cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, sizeof(unsigned int), st);
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(tile count)");
-        const int grid = grid_for(s, Q.n, 32);
-        canon_kernel<BEST><<<grid, THREADS, sizeof(CtaSmem), st>>>(Q);
+        const int grid = grid_for(s, Q.n, 32, false), grid_c = grid_for(s, Q.n, 32, true);
+        canon_kernel<BEST><<<grid_c, THREADS, sizeof(CanonCtaSmem), st>>>(Q);
         Q.accumulate = BEST ? 1 : 0;   // pass 2 merges into pass 1's result
         general_kernel<BEST><<<grid, THREADS, sizeof(CtaSmem), st>>>(Q);
         count_launch(2);

@@ -406,7 +406,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 f.magic_hi = (uint32_t)(m >> 32);
                 f.addend = j.ipb == 1 ? 1u : j.ipb - 1u;
                 if ((j.flags & KXF_INFEASIBLE) || j.ipb > 0x80000000u) {
-                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0xffffffffu;
+                    f.E = (j.flags & KXF_INFEASIBLE) ? INFINITY : 0.0;
+                    f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0xffffffffu;
                 } else {
                     f.E = es.E; f.S = es.S; f.D = d.D; f.rD = d.rD;
                     f.sat32 = i.sat_blocks > 0xffffffffull ? 0xffffffffu : (uint32_t)i.sat_blocks;
@@ -425,6 +426,14 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         if (kf[q].sat32 <= small_stride)
             for (uint32_t b = 0; b < kf[q].sat32; b++)
                 small[q * small_stride + b] = small_grid_time(kj[q], kg[q], gpu->n_sm, gpu->freq_hz, b);
+
+    for (uint32_t s = 0; s < n_skels; s++) {
+        bool tab = true;
+        const uint32_t nkx = skels[s].n_kernels * skels[s].n_xforms;
+        for (uint32_t q = info[s].kx_base; q < info[s].kx_base + nkx; q++)
+            tab = tab && (kf[q].sat32 <= small_stride || std::isinf(kf[q].E));
+        if (tab) info[s].flags |= SKF_TABULATED;
+    }
 
     // ---- one device blob ----
     struct Part { const void *src; size_t bytes; size_t off; };

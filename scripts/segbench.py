@@ -31,7 +31,10 @@ def main():
     out = G.best_result_tensor()
     rows = []
     Gn = (N + 15) // 16
+    only = os.environ.get("SEG_ONLY")
     for s in range(ns):
+        if only is not None and s not in [int(v) for v in only.split(",")]:
+            continue
         g0 = -(-s * Gn // ns)
         g1 = -(-(s + 1) * Gn // ns)
         lo, hi = g0 * 16, min(N, g1 * 16)
