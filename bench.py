@@ -298,7 +298,7 @@ def main():
         traffic = traffic * n_local / prof_n
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": achieved / peak, "traffic": traffic,
-            "kernel": "project_kernel<best> (fused projection + argmin)",
+            "kernel": "canon_kernel<best> + general_kernel<best> (fused projection + argmin; pass 1 is >99% of the step, profiles/)",
             "algorithmic_bytes_per_launch": 16 * n_local,
             "kernel_ms_avg": kern_avg_max, "peak_source": peak_src,
             "note": "16 B/candidate record read (DESIGN.md §5); kernel duration from CUDA "

@@ -23,13 +23,16 @@ struct __align__(16) KxD  { double D, rD; };        // rep denominator and RN(1/
 struct __align__(16) KxI  { uint64_t magic; uint64_t sat_blocks; };  // ceil(2^64/ipb) (0 if ipb==1)
 struct __align__(16) KxJ  { uint32_t ipb, occ, wpb, flags; };        // flags: KXF_*
 enum : uint32_t { KXF_INFEASIBLE = 1u, KXF_NOMEM = 2u, KXF_PER_ITER = 4u };
+enum : uint32_t { XINF_ITER = 1u, XINF_ONCE = 2u };
 
 // Packed fast-path record (48 B, one address per (kernel, transformation)):
 // for 0 < W < 2^31, blocks = ceil(W / ipb) = hi32(magic_hi*W' + hi32(magic_lo*W'))
 // with W' = W + addend (magic = ceil(2^64/ipb), addend = ipb - 1; ipb == 1:
 // magic = 2^64 - 1, addend = 1); the saturated formula holds iff
-// blocks >= sat32.  Infeasible (occupancy 0) or ipb > 2^31: sat32 = 2^32 - 1
-// (always the general path).  Work counts outside (0, 2^31) are stored as 0,
+// blocks >= sat32.  ipb > 2^31: sat32 = 2^32 - 1 (always the general path).
+// Infeasible (occupancy 0): E = S = 0, sat32 = 0 (a finite 0 from the fast
+// path, replaced by +inf through SpaceDev::xinf).  Work counts
+// outside (0, 2^31) are stored as 0,
 // which also selects the general path (blocks = 0 < sat32).
 struct __align__(16) KxFast {
     uint32_t magic_lo, magic_hi, sat32, addend;   // first: the chain starts with blocks
@@ -50,7 +53,9 @@ struct SkelInfo {
     // usage plan (plan.cpp): valid for nx >= plan_tx and ny >= plan_ty; its
     // byte polynomials at poly[poly_base + ...] (SkelPlanHost layout)
     uint32_t plan_tx, plan_ty, poly_base, poly_stride;
-    uint32_t per_iter_mask, pad1, pad2, pad3;   // per_iter_mask: bit k = kernel k per-iteration
+    uint32_t per_iter_mask;   // bit k = kernel k per-iteration
+    uint32_t poly_mask;       // bit 2a + dir: byte polynomial not zero in every size class
+    uint32_t pad2, pad3;
 };
 
 struct ArrayDev {
@@ -124,6 +129,9 @@ struct SpaceDev {
     // small-grid kernel times: small_t[kxi * small_stride + blocks] for
     // blocks < sat32 when sat32 <= small_stride (space.cpp small_grid_time)
     const double *small_t;
+    // per (skeleton, xform), at kx_base + x: some per-iteration (XINF_ITER) /
+    // run-once (XINF_ONCE) kernel is infeasible, so that sum is +inf
+    const uint32_t *xinf;
     uint32_t small_stride;
     uint32_t n_skels;
     uint32_t n_sm;

@@ -733,14 +733,16 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
     r.n_valid = b.nval;
 }
 
-// Canonical tiles: CX consecutive records per group (one group per lane),
-// XW transformations per model pass.
+// Canonical tiles: CX consecutive records per group, 32 groups per tile (one
+// group per lane in phases A/B).  Phase C maps lane = (transformation x,
+// half h): the lane models transformation x of groups h, h + 2, ..., CG
+// groups per pass, so one (kernel, x) constant load serves CG records.
 constexpr int CX = 16;
 constexpr int CTILE = 32 * CX;
-#ifndef GROPHECY_XW
-#define GROPHECY_XW 4
+#ifndef GROPHECY_CG
+#define GROPHECY_CG 8
 #endif
-constexpr int XW = GROPHECY_XW;
+constexpr int CG = GROPHECY_CG;   // groups per lane per model pass (divides 16)
 #ifndef GROPHECY_CMINB
 #define GROPHECY_CMINB 2
 #endif
@@ -758,9 +760,13 @@ struct WarpSmem {
     uint8_t plan_pos[MAX_SEG];                  // plan keys of the current slot group
     unsigned long long best_h[32], best_d[32];  // bytes of each lane's running best
 };
-// ... and of the canonical kernel.
+// ... and of the canonical kernel.  Per group g (= lane of phase A/B):
+// work counts at cw[k][g & 1][g >> 1] (a phase-C lane of half h reads its
+// groups h, h + 2, ... as consecutive words), usage and iterations at [g].
 struct CanonSmem {
-    uint32_t cw[MAXK][32];                      // work counts (w_store), [kernel][lane]
+    alignas(16) uint32_t cw[MAXK][2][16];       // work counts (w_store)
+    double th[32], td[32], it[32];              // transfer times, (double) iters
+    unsigned long long uh[32], ud[32];          // transfer bytes
     unsigned long long best_h[32], best_d[32];
 };
 struct CtaSmem {
@@ -857,10 +863,13 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
             for (int j = 0; j < NJ; j++) to[j] = __dadd_rn(to[j], tk[j]);
         }
     }
+    // infeasible kernels (fast path: a finite 0): that sum is +inf (xinf)
 #pragma unroll
     for (int j = 0; j < NJ; j++) {
-        t_iter[j] = ti[j];
-        t_once[j] = to[j];
+        const uint32_t xf = __ldg(&S.xinf[I.kx_base + x[j]]);
+        const double inf = __longlong_as_double(0x7ff0000000000000LL);
+        t_iter[j] = (xf & XINF_ITER) ? inf : ti[j];
+        t_once[j] = (xf & XINF_ONCE) ? inf : to[j];
     }
 }
 
@@ -1183,113 +1192,129 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
     bool huge = false;
     for (uint32_t k = 0; k < K; k++) {
         const uint32_t w = w_store(aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny));
-        ws.cw[k][lane] = w;
+        ws.cw[k][lane & 1][lane >> 1] = w;
         huge |= w == W_HUGE;
     }
     if (__any_sync(FULL, huge)) return false;   // (nothing written yet)
     // keys off the plan path (small sizes, strided, hull): general tiles
     if (!__all_sync(FULL, n0 >= I.plan_tx && m0 >= I.plan_ty)) return false;
-    Usage u = {0ull, 0ull, 0.0, 0.0};
     {
+        Usage u = {0ull, 0ull, 0.0, 0.0};
         const uint32_t stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
         const unsigned long long *pp =
             S.poly + I.poly_base + (size_t)((n0 & 7u) * 8u + (m0 & 7u)) * (2u * n_arrays * stride);
+        // skipped polynomials vanish in every class: their transfers add +0.0
+        // to a sum that is never -0.0, i.e. nothing (exact)
+        const uint32_t pm = I.poly_mask;
         for (uint32_t a = 0; a < n_arrays; a++, pp += 2 * stride) {
-            const unsigned long long h = stride > 4 ? poly_eval<true>(pp, a8, b8)
-                                                    : poly_eval<false>(pp, a8, b8);
-            const unsigned long long d = stride > 4 ? poly_eval<true>(pp + stride, a8, b8)
-                                                    : poly_eval<false>(pp + stride, a8, b8);
+            unsigned long long h = 0, d = 0;
+            if ((pm >> (2 * a)) & 1u)
+                h = stride > 4 ? poly_eval<true>(pp, a8, b8) : poly_eval<false>(pp, a8, b8);
+            if ((pm >> (2 * a + 1)) & 1u)
+                d = stride > 4 ? poly_eval<true>(pp + stride, a8, b8)
+                               : poly_eval<false>(pp + stride, a8, b8);
             // Eq. (1) per array, times added in array order (N6)
-            u.th = __dadd_rn(u.th, h ? __dadd_rn(P.pc.h2d.alpha_s,
-                                                 __dmul_rn(P.pc.h2d.beta_s_per_byte, __ull2double_rn(h)))
-                                     : 0.0);
-            u.td = __dadd_rn(u.td, d ? __dadd_rn(P.pc.d2h.alpha_s,
-                                                 __dmul_rn(P.pc.d2h.beta_s_per_byte, __ull2double_rn(d)))
-                                     : 0.0);
+            if (h) u.th = __dadd_rn(u.th, __dadd_rn(P.pc.h2d.alpha_s,
+                                                    __dmul_rn(P.pc.h2d.beta_s_per_byte, __ull2double_rn(h))));
+            if (d) u.td = __dadd_rn(u.td, __dadd_rn(P.pc.d2h.alpha_s,
+                                                    __dmul_rn(P.pc.d2h.beta_s_per_byte, __ull2double_rn(d))));
             u.h += h;
             u.d += d;
         }
+        ws.th[lane] = u.th;
+        ws.td[lane] = u.td;
+        ws.uh[lane] = u.h;
+        ws.ud[lane] = u.d;
+        ws.it[lane] = (double)i0;
     }
-    // ---- C ----
+    __syncwarp();
+    // ---- C: lane = (transformation x, half h); groups g = 2 i + h ----
     const uint32_t X = I.n_xforms, pim = I.per_iter_mask;
-    const double it = (double)i0;
-    const unsigned long long gi = P.base + q0;   // global index of the group's record 0
-    double bt = __longlong_as_double(0x7ff0000000000000LL);
-    int bx = -1;
+    const uint32_t x = (uint32_t)lane & (CX - 1), h = (uint32_t)lane / CX;
+    const KxFast *F0 = S.kx_f + I.kx_base + x;
+    const uint32_t xf = __ldg(&S.xinf[I.kx_base + x]);
 #pragma unroll 1
-    for (int x0 = 0; x0 < CX; x0 += XW) {
-        double ti[XW], to[XW];
+    for (int i0g = 0; i0g < 32 / 2; i0g += CG) {
+        double ti[CG], to[CG];
 #pragma unroll
-        for (int j = 0; j < XW; j++) ti[j] = to[j] = 0.0;
-        const KxFast *F = S.kx_f + I.kx_base + x0;
+        for (int j = 0; j < CG; j++) ti[j] = to[j] = 0.0;
+        const KxFast *F = F0;
+        uint32_t kxi = I.kx_base + x;
 #pragma unroll 1
-        for (uint32_t k = 0; k < K; k++, F += X) {
-            const uint32_t w = ws.cw[k][lane];
-            double tk[XW];
-            bool gen[XW], any = false;
-            uint32_t blocks[XW], sat[XW];
-            double E[XW];
+        for (uint32_t k = 0; k < K; k++, F += X, kxi += X) {
+            const KxFast f = *F;   // this lane's (kernel, transformation) constants
+            uint32_t w[CG];
 #pragma unroll
-            for (int j = 0; j < XW; j++) {
-                const KxFast f = F[j];
-                tk[j] = fast_time(f, w, S.freq, S.rfreq, gen[j], blocks[j]);
-                sat[j] = f.sat32;
-                E[j] = f.E;
+            for (int j = 0; j < CG; j += 4) {
+                const uint4 v = *reinterpret_cast<const uint4 *>(&ws.cw[k][h][i0g + j]);
+                w[j] = v.x;
+                w[j + 1] = v.y;
+                w[j + 2] = v.z;
+                w[j + 3] = v.w;
+            }
+            double tk[CG];
+            bool gen[CG], any = false;
+            uint32_t blocks[CG];
+#pragma unroll
+            for (int j = 0; j < CG; j++) {
+                tk[j] = fast_time(f, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
                 any |= gen[j];
             }
             if (any) {
-                // off the saturated path: the small-grid table (SKF_TABULATED), or infeasible
-                const uint32_t kxi = I.kx_base + k * X + x0;
+                // off the saturated path: the small-grid table (SKF_TABULATED:
+                // blocks < sat32 <= small_stride; infeasible pairs never get here)
+                const double *tab = S.small_t + (size_t)kxi * S.small_stride;
 #pragma unroll
-                for (int j = 0; j < XW; j++)
-                    if (gen[j])
-                        tk[j] = sat[j] <= S.small_stride
-                                    ? __ldg(&S.small_t[(size_t)(kxi + j) * S.small_stride + blocks[j]])
-                                    : E[j];
+                for (int j = 0; j < CG; j++)
+                    if (gen[j]) tk[j] = __ldg(tab + blocks[j]);
             }
             if ((pim >> k) & 1u) {
 #pragma unroll
-                for (int j = 0; j < XW; j++) ti[j] = __dadd_rn(ti[j], tk[j]);
+                for (int j = 0; j < CG; j++) ti[j] = __dadd_rn(ti[j], tk[j]);
             } else {
 #pragma unroll
-                for (int j = 0; j < XW; j++) to[j] = __dadd_rn(to[j], tk[j]);
+                for (int j = 0; j < CG; j++) to[j] = __dadd_rn(to[j], tk[j]);
             }
+        }
+        // infeasible kernels: that sum is +inf (exact, see xinf)
+        const double inf = __longlong_as_double(0x7ff0000000000000LL);
+        if (xf & XINF_ITER) {
+#pragma unroll
+            for (int j = 0; j < CG; j++) ti[j] = inf;
+        }
+        if (xf & XINF_ONCE) {
+#pragma unroll
+            for (int j = 0; j < CG; j++) to[j] = inf;
         }
         // totals: run-once + iters x per-iteration + transfers
-        double tt[XW];
 #pragma unroll
-        for (int j = 0; j < XW; j++)
-            tt[j] = __dadd_rn(__dadd_rn(__dadd_rn(to[j], __dmul_rn(it, ti[j])), u.th), u.td);
-        if (BEST) {
-#pragma unroll
-            for (int j = 0; j < XW; j++)
-                if (tt[j] < bt) {   // records in index order: the first minimum stays
-                    bt = tt[j];
-                    bx = x0 + j;
+        for (int j = 0; j < CG; j++) {
+            const uint32_t g = 2u * (uint32_t)(i0g + j) + h;
+            const double tt = __dadd_rn(__dadd_rn(__dadd_rn(to[j], __dmul_rn(ws.it[g], ti[j])),
+                                                  ws.th[g]), ws.td[g]);
+            const unsigned long long r = tb + (unsigned long long)g * CX + x;
+            if (BEST) {
+                // a lane meets its records in increasing index order (tiles,
+                // then groups): strict < keeps the lowest index among ties
+                const unsigned long long gi = P.base + r;
+                if (tt < best_t) {
+                    best_t = tt;
+                    best_i = gi;
+                    ws.best_h[lane] = ws.uh[g];
+                    ws.best_d[lane] = ws.ud[g];
                 }
-        } else {
-            const unsigned long long i = q0 + x0;
-#pragma unroll
-            for (int j = 0; j < XW; j++) {
-                __stcs(P.h2d + i + j, u.h);
-                __stcs(P.d2h + i + j, u.d);
-                __stcs(P.t + i + j, tt[j]);
-                if (P.p_iter) __stcs(P.p_iter + i + j, ti[j]);
-                if (P.p_once) __stcs(P.p_once + i + j, to[j]);
-                if (P.p_h2d) __stcs(P.p_h2d + i + j, u.th);
-                if (P.p_d2h) __stcs(P.p_d2h + i + j, u.td);
+            } else {
+                __stcs(P.h2d + r, ws.uh[g]);
+                __stcs(P.d2h + r, ws.ud[g]);
+                __stcs(P.t + r, tt);
+                if (P.p_iter) __stcs(P.p_iter + r, ti[j]);
+                if (P.p_once) __stcs(P.p_once + r, to[j]);
+                if (P.p_h2d) __stcs(P.p_h2d + r, ws.th[g]);
+                if (P.p_d2h) __stcs(P.p_d2h + r, ws.td[g]);
             }
         }
     }
-    if (BEST) {
-        cnt_val += CX;
-        if (bx >= 0 && better(bt, gi + (unsigned)bx, best_t, best_i)) {
-            best_t = bt;
-            best_i = gi + (unsigned)bx;
-            ws.best_h[lane] = u.h;
-            ws.best_d[lane] = u.d;
-        }
-    }
+    if (BEST) cnt_val += CX;
     __syncwarp();
     return true;
 }

@@ -310,6 +310,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxJ> kj;
     std::vector<KxG> kg;
     std::vector<KxFast> kf;
+    std::vector<uint32_t> xinf;   // per (skeleton, xform) at kx_base + x: XINF_* bits
     std::vector<unsigned long long> poly;
     auto a4 = [](const grophecy_affine8 &a) { return make_int4(a.c0, a.c1, a.c2, a.c3); };
     for (uint32_t s = 0; s < n_skels; s++) {
@@ -337,11 +338,20 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             I.poly_base = (uint32_t)poly.size();
             I.poly_stride = plan.poly_stride;
             poly.insert(poly.end(), plan.poly.begin(), plan.poly.end());
+            // polynomials that vanish in every size class price no transfer
+            // (Eq. (1) is applied only to non-zero bytes) and are skipped
+            I.poly_mask = 0;
+            const size_t np = 2 * (size_t)S.n_arrays, st = plan.poly_stride;
+            for (size_t c = 0; c < POLY_CLASSES; c++)
+                for (size_t q = 0; q < np; q++)
+                    for (size_t m = 0; m < st; m++)
+                        if (plan.poly[(c * np + q) * st + m]) I.poly_mask |= 1u << q;
         } else {
             I.plan_tx = I.plan_ty = 0xffffffffu;   // never applicable
             I.poly_base = I.poly_stride = 0;
+            I.poly_mask = 0;
         }
-        I.per_iter_mask = I.pad1 = I.pad2 = I.pad3 = 0;
+        I.per_iter_mask = I.pad2 = I.pad3 = 0;
         for (uint32_t k = 0; k < S.n_kernels; k++)
             if (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) I.per_iter_mask |= 1u << k;
         for (uint32_t k = 0; k < S.n_kernels; k++) {
@@ -389,6 +399,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             }
             arrays.push_back(A);
         }
+        const size_t kx0 = kf.size();   // this skeleton's kx_base
+        xinf.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, 0u);
         for (uint32_t k = 0; k < S.n_kernels; k++)
             for (uint32_t x = 0; x < S.n_xforms; x++) {
                 KxES es; KxD d; KxI i; KxJ j; KxG g;
@@ -405,9 +417,15 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 f.magic_lo = (uint32_t)m;
                 f.magic_hi = (uint32_t)(m >> 32);
                 f.addend = j.ipb == 1 ? 1u : j.ipb - 1u;
-                if ((j.flags & KXF_INFEASIBLE) || j.ipb > 0x80000000u) {
-                    f.E = (j.flags & KXF_INFEASIBLE) ? INFINITY : 0.0;
-                    f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0xffffffffu;
+                if (j.flags & KXF_INFEASIBLE) {
+                    // occupancy 0: t_k = +inf for every size (N5).  The fast
+                    // path yields a finite 0 here (sat32 = 0, never the general
+                    // branch) and the record's sum is set to +inf from xinf
+                    // (+inf + finite = +inf in any order: exact)
+                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0u;
+                    xinf[kx0 + x] |= (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) ? XINF_ITER : XINF_ONCE;
+                } else if (j.ipb > 0x80000000u) {
+                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0xffffffffu;
                 } else {
                     f.E = es.E; f.S = es.S; f.D = d.D; f.rD = d.rD;
                     f.sat32 = i.sat_blocks > 0xffffffffull ? 0xffffffffu : (uint32_t)i.sat_blocks;
@@ -431,7 +449,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         bool tab = true;
         const uint32_t nkx = skels[s].n_kernels * skels[s].n_xforms;
         for (uint32_t q = info[s].kx_base; q < info[s].kx_base + nkx; q++)
-            tab = tab && (kf[q].sat32 <= small_stride || std::isinf(kf[q].E));
+            tab = tab && kf[q].sat32 <= small_stride;
         if (tab) info[s].flags |= SKF_TABULATED;
     }
 
@@ -451,6 +469,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {poly.data(), poly.size() * sizeof(unsigned long long), 0},
         {kf.data(), kf.size() * sizeof(KxFast), 0},
         {small.data(), small.size() * sizeof(double), 0},
+        {xinf.data(), xinf.size() * sizeof(uint32_t), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -511,6 +530,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.poly = (const unsigned long long *)(base + parts[10].off);
     D.kx_f = (const KxFast *)(base + parts[11].off);
     D.small_t = (const double *)(base + parts[12].off);
+    D.xinf = (const uint32_t *)(base + parts[13].off);
     D.small_stride = small_stride;
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;

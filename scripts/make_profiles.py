@@ -76,8 +76,8 @@ def main(tag):
                 "smsp__inst_executed.sum", "dram__throughput.avg.pct_of_peak_sustained_elapsed"]
         summ = {}
         with open(os.path.join(PROF, f"{tag}_ncu_best.txt"), "w") as f:
-            f.write("ncu --set full --clock-control none -k regex:project_kernel (bench config, "
-                    "one 10^9-candidate best launch)\n")
+            f.write("ncu --set full --clock-control none -k regex:canon_kernel (bench config, "
+                    "pass 1 of one 10^9-candidate best projection)\n")
             for k in want:
                 if k in r:
                     f.write(f"{k:70s} {r[k]} {units.get(k, '')}\n")
