@@ -25,19 +25,24 @@ struct __align__(16) KxJ  { uint32_t ipb, occ, wpb, flags; };        // flags: K
 enum : uint32_t { KXF_INFEASIBLE = 1u, KXF_NOMEM = 2u, KXF_PER_ITER = 4u };
 enum : uint32_t { XINF_ITER = 1u, XINF_ONCE = 2u };
 
-// Packed fast-path record (48 B, one address per (kernel, transformation)):
-// for 0 < W < 2^31, blocks = ceil(W / ipb) = hi32(magic_hi*W' + hi32(magic_lo*W'))
-// with W' = W + addend (magic = ceil(2^64/ipb), addend = ipb - 1; ipb == 1:
-// magic = 2^64 - 1, addend = 1); the saturated formula holds iff
-// blocks >= sat32.  ipb > 2^31: sat32 = 2^32 - 1 (always the general path).
-// Infeasible (occupancy 0): E = S = 0, sat32 = 0 (a finite 0 from the fast
-// path, replaced by +inf through SpaceDev::xinf).  Work counts
-// outside (0, 2^31) are stored as 0,
-// which also selects the general path (blocks = 0 < sat32).
+// Packed fast-path record (48 B, one address per (kernel, transformation)).
+// Work counts are stored as w in [0, 2^30) (else W_HUGE: the general path).
+// blocks = ceil(w / ipb) = hi32(w * m + cc) >> sh: for ipb = d >= 2,
+// l = ceil(log2 d), m = ceil(2^(31 + l) / d) < 2^32, cc = (d - 1) m, sh = l - 1
+// (Granlund-Montgomery: floor(n m / 2^(31 + l)) = floor(n / d) for every
+// n = w + d - 1 < 2^31); d = 1: m = cc = 2^32 - 1, sh = 0.  satsh = sat |
+// sh << KXF_SAT_BITS; the saturated formula holds iff blocks >= sat.
+// Pairs the fast path cannot take (ipb > 2^30, sat >= KXF_SAT_MASK): m = cc =
+// 0 (blocks = 0) and sat = KXF_SAT_MASK, i.e. always the general path.
+// Infeasible (occupancy 0): E = S = 0, sat = 0 (a finite 0 from the fast
+// path, replaced by +inf through SpaceDev::xinf).
+constexpr uint32_t KXF_SAT_BITS = 27, KXF_SAT_MASK = (1u << KXF_SAT_BITS) - 1u;
 struct __align__(16) KxFast {
-    uint32_t magic_lo, magic_hi, sat32, addend;   // first: the chain starts with blocks
-    double D, rD, E, S;                           // E = +inf iff infeasible
+    uint32_t m, satsh;        // first: the chain starts with blocks
+    uint64_t cc;
+    double D, rD, E, S;
 };
+inline uint32_t kxf_sat(const KxFast &f) { return f.satsh & KXF_SAT_MASK; }
 
 // General-grid constants (small grids / huge W), read only off the fast path.
 struct KxG {

@@ -123,13 +123,13 @@ __device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned 
     o.d += da;
 }
 
-// Work-item count as stored for the model's fast path: W if 0 < W < 2^31,
+// Work-item count as stored for the model's fast path: W if 0 < W < 2^30,
 // 0 if W <= 0 (blocks = 0: the small-grid table gives t = 0), W_HUGE above
 // (the general path recomputes W from the key).
 constexpr uint32_t W_HUGE = 0xffffffffu;
 __device__ __forceinline__ uint32_t w_store(long long w)
 {
-    return w <= 0 ? 0u : (w < 0x80000000LL ? (uint32_t)w : W_HUGE);
+    return w <= 0 ? 0u : (w < 0x40000000LL ? (uint32_t)w : W_HUGE);
 }
 
 // One residue-class byte polynomial P(a, b) (plan.cpp; internal.h layout),
@@ -777,18 +777,18 @@ struct CanonCtaSmem {
 };
 
 // Saturated-grid kernel time (DESIGN.md §3 N5, saturated reduction) of one
-// (record, kernel) from the packed constants and the stored work count w
-// (w_store, < 2^31 here): cyc = E rep + S rep, rep = blocks / D,
-// t = cyc / freq, both divisions by Markstein's correction (bitwise the IEEE
-// quotients).  gen is set when the grid is not saturated (or the pair is
-// infeasible) — the returned value is then meaningless and gen_time decides.
-__device__ __forceinline__ double fast_time(const KxFast &f, uint32_t w, double freq, double rfreq,
-                                            bool &gen, uint32_t &blocks)
+// (record, kernel) from the packed constants (sat, sh = satsh fields) and
+// the stored work count w (w_store, < 2^30 here): blocks = ceil(w / ipb) by
+// one 32x32+64 multiply-add and a shift, cyc = E rep + S rep, rep = blocks /
+// D, t = cyc / freq, both divisions by Markstein's correction (bitwise the
+// IEEE quotients).  gen is set when the grid is not saturated — the returned
+// value is then meaningless and the general branch decides.
+__device__ __forceinline__ double fast_time(const KxFast &f, uint32_t sat, uint32_t sh, uint32_t w,
+                                            double freq, double rfreq, bool &gen, uint32_t &blocks)
 {
-    const uint32_t w1 = w + f.addend;
-    const unsigned long long lo = (unsigned long long)f.magic_lo * w1;
-    blocks = (uint32_t)(((unsigned long long)f.magic_hi * w1 + (lo >> 32)) >> 32);
-    gen = blocks < f.sat32;
+    const unsigned long long p = (unsigned long long)w * f.m + f.cc;
+    blocks = (uint32_t)(p >> 32) >> sh;
+    gen = blocks < sat;
     const double bb = __uint2double_rn(blocks);
     const double q = __dmul_rn(bb, f.rD);
     const double rep = __fma_rn(__fma_rn(-q, f.D, bb), f.rD, q);
@@ -836,9 +836,10 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
         for (int j = 0; j < NJ; j++) {
             const KxFast F = SAMEX ? F0 : S.kx_f[kb + x[j]];
             w[j] = ws.slot_w[ls[j]][k];
-            tk[j] = fast_time(F, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
+            sat[j] = F.satsh & KXF_SAT_MASK;
+            tk[j] = fast_time(F, sat[j], F.satsh >> KXF_SAT_BITS, w[j], S.freq, S.rfreq, gen[j],
+                              blocks[j]);
             gen[j] |= w[j] == W_HUGE;
-            sat[j] = F.sat32;
             E[j] = F.E;
         }
         bool any = false;
@@ -1240,9 +1241,12 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
         for (int j = 0; j < CG; j++) ti[j] = to[j] = 0.0;
         const KxFast *F = F0;
         uint32_t kxi = I.kx_base + x;
+        KxFast fn = *F0;   // K >= 1; the next kernel's constants load one step ahead
 #pragma unroll 1
         for (uint32_t k = 0; k < K; k++, F += X, kxi += X) {
-            const KxFast f = *F;   // this lane's (kernel, transformation) constants
+            const KxFast f = fn;   // this lane's (kernel, transformation) constants
+            if (k + 1 < K) fn = F[X];
+            const uint32_t sat = f.satsh & KXF_SAT_MASK, sh = f.satsh >> KXF_SAT_BITS;
             uint32_t w[CG];
 #pragma unroll
             for (int j = 0; j < CG; j += 4) {
@@ -1257,7 +1261,7 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
             uint32_t blocks[CG];
 #pragma unroll
             for (int j = 0; j < CG; j++) {
-                tk[j] = fast_time(f, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
+                tk[j] = fast_time(f, sat, sh, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
                 any |= gen[j];
             }
             if (any) {

@@ -409,27 +409,41 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 kes.push_back(es); kd.push_back(d); ki.push_back(i); kj.push_back(j);
                 kg.push_back(g);
                 KxFast f;
-                // blocks = hi64(magic * (W + addend)) = ceil(W / ipb) for
-                // W < 2^31 (magic = ceil(2^64 / ipb), addend = ipb - 1; for
-                // ipb == 1: magic = 2^64 - 1, addend = 1).  Infeasible or huge
-                // ipb: sat32 = 2^32 - 1, so every record takes the general path.
-                const uint64_t m = j.ipb == 1 ? ~0ull : i.magic;
-                f.magic_lo = (uint32_t)m;
-                f.magic_hi = (uint32_t)(m >> 32);
-                f.addend = j.ipb == 1 ? 1u : j.ipb - 1u;
+                // blocks = hi32(w m + cc) >> sh = ceil(w / ipb) for w < 2^30
+                // (internal.h); pairs off the fast path: blocks = 0 < sat
+                const uint32_t dv = j.ipb;
+                uint32_t sh = 0;
+                if (dv == 1) {
+                    f.m = 0xffffffffu;
+                    f.cc = 0xffffffffull;
+                } else if (dv <= (1u << 30)) {
+                    uint32_t l = 0;
+                    while ((1ull << l) < dv) l++;
+                    const uint64_t m = ((1ull << (31 + l)) + dv - 1) / dv;
+                    f.m = (uint32_t)m;
+                    f.cc = (uint64_t)(dv - 1) * m;
+                    sh = l - 1;
+                } else {
+                    f.m = 0;
+                    f.cc = 0;
+                }
+                uint32_t sat;
                 if (j.flags & KXF_INFEASIBLE) {
                     // occupancy 0: t_k = +inf for every size (N5).  The fast
-                    // path yields a finite 0 here (sat32 = 0, never the general
+                    // path yields a finite 0 here (sat = 0, never the general
                     // branch) and the record's sum is set to +inf from xinf
                     // (+inf + finite = +inf in any order: exact)
-                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0u;
+                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; sat = 0;
                     xinf[kx0 + x] |= (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) ? XINF_ITER : XINF_ONCE;
-                } else if (j.ipb > 0x80000000u) {
-                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; f.sat32 = 0xffffffffu;
+                } else if (dv > (1u << 30) || i.sat_blocks >= KXF_SAT_MASK) {
+                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; sat = KXF_SAT_MASK;
+                    f.m = 0;
+                    f.cc = 0;
                 } else {
                     f.E = es.E; f.S = es.S; f.D = d.D; f.rD = d.rD;
-                    f.sat32 = i.sat_blocks > 0xffffffffull ? 0xffffffffu : (uint32_t)i.sat_blocks;
+                    sat = (uint32_t)i.sat_blocks;
                 }
+                f.satsh = sat | sh << KXF_SAT_BITS;
                 kf.push_back(f);
             }
     }
@@ -437,19 +451,19 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     // ---- small-grid table: t(kernel, xform, blocks) for blocks < sat32 ----
     uint32_t max_sat = 0;
     for (const KxFast &f : kf)
-        if (f.sat32 != 0xffffffffu) max_sat = std::max(max_sat, f.sat32);
+        if (kxf_sat(f) != KXF_SAT_MASK) max_sat = std::max(max_sat, kxf_sat(f));
     const uint32_t small_stride = std::min<uint32_t>(max_sat, SMALL_GRID_MAX);
     std::vector<double> small((size_t)kf.size() * small_stride, 0.0);
     for (size_t q = 0; q < kf.size(); q++)
-        if (kf[q].sat32 <= small_stride)
-            for (uint32_t b = 0; b < kf[q].sat32; b++)
+        if (kxf_sat(kf[q]) <= small_stride)
+            for (uint32_t b = 0; b < kxf_sat(kf[q]); b++)
                 small[q * small_stride + b] = small_grid_time(kj[q], kg[q], gpu->n_sm, gpu->freq_hz, b);
 
     for (uint32_t s = 0; s < n_skels; s++) {
         bool tab = true;
         const uint32_t nkx = skels[s].n_kernels * skels[s].n_xforms;
         for (uint32_t q = info[s].kx_base; q < info[s].kx_base + nkx; q++)
-            tab = tab && kf[q].sat32 <= small_stride;
+            tab = tab && kxf_sat(kf[q]) <= small_stride;
         if (tab) info[s].flags |= SKF_TABULATED;
     }
 
