@@ -764,10 +764,12 @@ struct WarpSmem {
 // work counts at cw[k][g & 1][g >> 1] (a phase-C lane of half h reads its
 // groups h, h + 2, ... as consecutive words), usage and iterations at [g].
 struct CanonSmem {
+    alignas(128) uint32_t rec[4][CTILE];        // the tile's SoA records (TMA bulk copies)
     alignas(16) uint32_t cw[MAXK][2][16];       // work counts (w_store)
     double th[32], td[32], it[32];              // transfer times, (double) iters
     unsigned long long uh[32], ud[32];          // transfer bytes
     unsigned long long best_h[32], best_d[32];
+    unsigned long long mbar;                    // completion of the rec copies
 };
 struct CtaSmem {
     WarpSmem w[WARPS];
@@ -1130,6 +1132,48 @@ __device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsi
         }
 }
 
+// ---- 1-D bulk copies (TMA) global -> shared with mbarrier completion ----
+__device__ __forceinline__ uint32_t smem_u32(const void *p)
+{
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__device__ __forceinline__ void mbar_init(unsigned long long *bar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t phase)
+{
+    asm volatile(
+        "{\n .reg .pred p;\n"
+        "W%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra W%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(phase)
+        : "memory");
+}
+
+// Lane 0 of a warp: copy the CTILE records of the tile at tb (full, 16-byte
+// aligned) into ws.rec, completing on ws.mbar.  Earlier generic-proxy reads of
+// ws.rec are ordered before the async-proxy writes by the fence.
+__device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, unsigned long long tb)
+{
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    const uint32_t bar = smem_u32(&ws.mbar);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
+                 "r"((uint32_t)(4 * CTILE * sizeof(uint32_t)))
+                 : "memory");
+    const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
+#pragma unroll
+    for (int a = 0; a < 4; a++)
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                smem_u32(ws.rec[a])),
+            "l"(src[a] + tb), "r"((uint32_t)(CTILE * sizeof(uint32_t))), "r"(bar)
+            : "memory");
+}
+
 // One canonical tile: CTILE records from tb where every group of CX
 // consecutive records (lane l: records tb + CX l ...) is one design point
 // (same skeleton, nx, ny, iters; xform = position in the group, the layout
@@ -1144,41 +1188,51 @@ __device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsi
 //      load serves 32 records), then writes outputs / keeps its argmin.
 template <bool BEST>
 __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsigned long long tb,
-                                           int lane, double &best_t, unsigned long long &best_i,
-                                           uint32_t &cnt_val)
+                                           unsigned long long next_tb, int lane, double &best_t,
+                                           unsigned long long &best_i, uint32_t &cnt_val)
 {
     const SpaceDev &S = P.S;
     const unsigned long long q0 = tb + (unsigned long long)lane * CX;
-    // ---- A ----
+    // ---- A (records staged in ws.rec by the TMA; lane l reads its group's
+    //      16-byte chunks in the rotated order c = (m + l/2) mod 4, which
+    //      spreads 8 consecutive lanes over all 32 banks) ----
     uint32_t acc = 0, s0, n0, m0, i0;
     {
-        const uint4 *p = reinterpret_cast<const uint4 *>(P.skx + q0);
+        const uint4 *p = reinterpret_cast<const uint4 *>(ws.rec[0] + lane * CX);
+        const uint32_t r = ((uint32_t)lane >> 1) & 3u;
         uint4 v[CX / 4];
 #pragma unroll
-        for (int m = 0; m < CX / 4; m++) v[m] = __ldcs(p + m);
-        s0 = v[0].x;
-        acc = s0 & 0xffffu;   // transformation 0 first, so s0 + x == s0 ^ x
+        for (int m = 0; m < CX / 4; m++) v[m] = p[(m + r) & 3u];
+        // record 0's skx from the first chunk read: valid groups have
+        // skx[q] = s0 ^ q with (s0 & 0xffff) == 0 (transformation q at q)
+        s0 = v[0].x ^ (4u * r);
+        acc = s0 & 0xffffu;
 #pragma unroll
         for (int m = 0; m < CX / 4; m++) {
-            acc |= (v[m].x ^ s0) ^ (uint32_t)(4 * m + 0);
-            acc |= (v[m].y ^ s0) ^ (uint32_t)(4 * m + 1);
-            acc |= (v[m].z ^ s0) ^ (uint32_t)(4 * m + 2);
-            acc |= (v[m].w ^ s0) ^ (uint32_t)(4 * m + 3);
+            const uint32_t c4 = 4u * ((m + r) & 3u);
+            acc |= (v[m].x ^ s0) ^ (c4 + 0u);
+            acc |= (v[m].y ^ s0) ^ (c4 + 1u);
+            acc |= (v[m].z ^ s0) ^ (c4 + 2u);
+            acc |= (v[m].w ^ s0) ^ (c4 + 3u);
         }
     }
-    auto same = [&](const uint32_t *arr, uint32_t &first) {
-        const uint4 *p = reinterpret_cast<const uint4 *>(arr + q0);
+    auto same = [&](int arr, uint32_t &first) {
+        const uint4 *p = reinterpret_cast<const uint4 *>(ws.rec[arr] + lane * CX);
+        const uint32_t r = ((uint32_t)lane >> 1) & 3u;
         uint4 v[CX / 4];
 #pragma unroll
-        for (int m = 0; m < CX / 4; m++) v[m] = __ldcs(p + m);
+        for (int m = 0; m < CX / 4; m++) v[m] = p[(m + r) & 3u];
         first = v[0].x;
 #pragma unroll
         for (int m = 0; m < CX / 4; m++)
             acc |= (v[m].x ^ first) | (v[m].y ^ first) | (v[m].z ^ first) | (v[m].w ^ first);
     };
-    same(P.nx, n0);
-    same(P.ny, m0);
-    same(P.iters, i0);
+    same(1, n0);
+    same(2, m0);
+    same(3, i0);
+    // every read of ws.rec is consumed (acc): the buffer takes the next tile
+    __syncwarp();
+    if (lane == 0 && next_tb != ~0ull) issue_tile_copy(P, ws, next_tb);
     const uint32_t skel = s0 >> 16;
     const uint32_t skel_l0 = __shfl_sync(FULL, skel, 0);   // (every lane: no short-circuit)
     bool ok = acc == 0 && skel < S.n_skels && n0 - 1u < GROPHECY_MAX_DIM &&
@@ -1400,26 +1454,27 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
     ws.best_d[lane] = 0;
     const unsigned long long ntiles = (P.n + CTILE - 1) / CTILE;
     const unsigned long long wstride = (unsigned long long)gridDim.x * WARPS;
-    for (unsigned long long tile = (unsigned long long)blockIdx.x * WARPS + warp; tile < ntiles;
-         tile += wstride) {
-        const unsigned long long tb = tile * CTILE;
-        // warm L2 with the records of this warp's next tile
-        if (lane < 4) {
-            const unsigned long long nt = tile + wstride;
-            if (nt < ntiles && P.aligned) {
-                const unsigned long long nb = nt * CTILE;
-                const unsigned long long cnt = min((unsigned long long)CTILE, P.n - nb);
-                const uint32_t *base = lane == 0 ? P.skx : lane == 1 ? P.nx : lane == 2 ? P.ny : P.iters;
-                const uint32_t bytes = (uint32_t)(cnt * 4) & ~15u;
-                if (bytes)
-                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;"
-                                 :: "l"(base + nb), "r"(bytes) : "memory");
-            }
+    // full tiles of 16-byte aligned records are staged in shared memory by
+    // the TMA one tile ahead (the copy of the next tile overlaps phases B and
+    // C of this one); the others go to the general path directly
+    auto full = [&](unsigned long long t) { return P.aligned && (t + 1) * CTILE <= P.n; };
+    if (lane == 0) mbar_init(&ws.mbar, 1);
+    __syncwarp();
+    uint32_t phase = 0;
+    const unsigned long long t0 = (unsigned long long)blockIdx.x * WARPS + warp;
+    if (lane == 0 && t0 < ntiles && full(t0)) issue_tile_copy(P, ws, t0 * CTILE);
+    for (unsigned long long tile = t0; tile < ntiles; tile += wstride) {
+        const unsigned long long tb = tile * CTILE, nt = tile + wstride;
+        const unsigned long long next_tb = nt < ntiles && full(nt) ? nt * CTILE : ~0ull;
+        bool done = false;
+        if (full(tile)) {
+            mbar_wait(&ws.mbar, phase);
+            phase ^= 1u;
+            done = canon_tile<BEST>(P, ws, tb, next_tb, lane, best_t, best_i, cnt_val);
+        } else if (lane == 0 && next_tb != ~0ull) {
+            issue_tile_copy(P, ws, next_tb);   // the buffer is idle during this tile
         }
-        if (!(P.aligned && tb + CTILE <= P.n &&
-              canon_tile<BEST>(P, ws, tb, lane, best_t, best_i, cnt_val)) &&
-            lane == 0)
-            P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)tile;
+        if (!done && lane == 0) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)tile;
     }
     if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, 0u, cnt_val);
 }
