@@ -1344,24 +1344,27 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
 #pragma unroll
             for (int j = 0; j < CG; j++) to[j] = inf;
         }
-        // totals: run-once + iters x per-iteration + transfers
+        // totals: run-once + iters x per-iteration +
+        // transfers.  Without run-once kernels t_once = +0.0 and
+        // +0.0 + iters * t_iter = iters * t_iter exactly (both >= +0).
+        const bool once = pim != (K == 32 ? 0xffffffffu : (1u << K) - 1u) || (xf & XINF_ONCE);
+        double cm = __longlong_as_double(0x7ff0000000000000LL);
+        int cj = -1;
 #pragma unroll
         for (int j = 0; j < CG; j++) {
             const uint32_t g = 2u * (uint32_t)(i0g + j) + h;
-            const double tt = __dadd_rn(__dadd_rn(__dadd_rn(to[j], __dmul_rn(ws.it[g], ti[j])),
-                                                  ws.th[g]), ws.td[g]);
-            const unsigned long long r = tb + (unsigned long long)g * CX + x;
+            double tk = __dmul_rn(ws.it[g], ti[j]);
+            if (once) tk = __dadd_rn(to[j], tk);
+            const double tt = __dadd_rn(__dadd_rn(tk, ws.th[g]), ws.td[g]);
             if (BEST) {
-                // a lane meets its records in increasing index order (tiles,
-                // then groups): strict < keeps the lowest index among ties
-                const unsigned long long gi = P.base + r;
-                if (tt < best_t) {
-                    best_t = tt;
-                    best_i = gi;
-                    ws.best_h[lane] = ws.uh[g];
-                    ws.best_d[lane] = ws.ud[g];
+                // the lane's records come in increasing index order (tiles,
+                // chunks, j): strict < keeps the lowest index among ties
+                if (tt < cm) {
+                    cm = tt;
+                    cj = j;
                 }
             } else {
+                const unsigned long long r = tb + (unsigned long long)g * CX + x;
                 __stcs(P.h2d + r, ws.uh[g]);
                 __stcs(P.d2h + r, ws.ud[g]);
                 __stcs(P.t + r, tt);
@@ -1370,6 +1373,13 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
                 if (P.p_h2d) __stcs(P.p_h2d + r, ws.th[g]);
                 if (P.p_d2h) __stcs(P.p_d2h + r, ws.td[g]);
             }
+        }
+        if (BEST && cm < best_t) {
+            const uint32_t g = 2u * (uint32_t)(i0g + cj) + h;
+            best_t = cm;
+            best_i = P.base + tb + (unsigned long long)g * CX + x;
+            ws.best_h[lane] = ws.uh[g];
+            ws.best_d[lane] = ws.ud[g];
         }
     }
     if (BEST) cnt_val += CX;
