@@ -1132,6 +1132,54 @@ __device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsi
         }
 }
 
+// One design point's data usage from its residue class's byte polynomials
+// (plan.cpp; internal.h layout): per array, H2D and D2H bytes and their
+// Eq. (1) transfer times added in array order (N6).  AU arrays per step with
+// every coefficient load of the step issued first (independent loads instead
+// of one dependent round trip per array); polynomials that vanish in every
+// class (pm bit clear) are not loaded: their bytes are 0 and their transfer
+// adds +0.0 to a sum that is never -0.0, i.e. nothing (exact).
+template <bool BIQ, int AU>
+__device__ __forceinline__ void group_usage(const unsigned long long *pp, uint32_t stride,
+                                            uint32_t n_arrays, uint32_t pm, uint32_t a8,
+                                            uint32_t b8, const grophecy_pcie &pc, Usage &u)
+{
+    constexpr int NQ = BIQ ? 5 : 2;   // 16-byte coefficient pairs per polynomial
+    for (uint32_t a0 = 0; a0 < n_arrays; a0 += AU) {
+        ulonglong2 c[AU][2][NQ];
+#pragma unroll
+        for (int i = 0; i < AU; i++)
+#pragma unroll
+            for (int dir = 0; dir < 2; dir++) {
+                const uint32_t q = 2u * (a0 + (uint32_t)i) + (uint32_t)dir;
+                const bool on = a0 + (uint32_t)i < n_arrays && ((pm >> q) & 1u);
+                const ulonglong2 *src = reinterpret_cast<const ulonglong2 *>(pp + (size_t)q * stride);
+#pragma unroll
+                for (int m = 0; m < NQ; m++) c[i][dir][m] = on ? __ldg(src + m) : make_ulonglong2(0, 0);
+            }
+#pragma unroll
+        for (int i = 0; i < AU; i++) {
+            if (a0 + (uint32_t)i >= n_arrays) break;
+            unsigned long long v[2];
+#pragma unroll
+            for (int dir = 0; dir < 2; dir++) {
+                const ulonglong2 *k = c[i][dir];
+                unsigned long long e = k[0].x + k[0].y * a8 + (k[1].x + k[1].y * a8) * b8;
+                if (BIQ)
+                    e += (unsigned long long)a8 * (a8 * (k[2].x + b8 * (k[3].x + b8 * k[4].x))) +
+                         (unsigned long long)b8 * (b8 * (k[2].y + a8 * k[3].y));
+                v[dir] = e;
+            }
+            if (v[0]) u.th = __dadd_rn(u.th, __dadd_rn(pc.h2d.alpha_s,
+                                                       __dmul_rn(pc.h2d.beta_s_per_byte, __ull2double_rn(v[0]))));
+            if (v[1]) u.td = __dadd_rn(u.td, __dadd_rn(pc.d2h.alpha_s,
+                                                       __dmul_rn(pc.d2h.beta_s_per_byte, __ull2double_rn(v[1]))));
+            u.h += v[0];
+            u.d += v[1];
+        }
+    }
+}
+
 // ---- 1-D bulk copies (TMA) global -> shared with mbarrier completion ----
 __device__ __forceinline__ uint32_t smem_u32(const void *p)
 {
@@ -1261,21 +1309,8 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
         // skipped polynomials vanish in every class: their transfers add +0.0
         // to a sum that is never -0.0, i.e. nothing (exact)
         const uint32_t pm = I.poly_mask;
-        for (uint32_t a = 0; a < n_arrays; a++, pp += 2 * stride) {
-            unsigned long long h = 0, d = 0;
-            if ((pm >> (2 * a)) & 1u)
-                h = stride > 4 ? poly_eval<true>(pp, a8, b8) : poly_eval<false>(pp, a8, b8);
-            if ((pm >> (2 * a + 1)) & 1u)
-                d = stride > 4 ? poly_eval<true>(pp + stride, a8, b8)
-                               : poly_eval<false>(pp + stride, a8, b8);
-            // Eq. (1) per array, times added in array order (N6)
-            if (h) u.th = __dadd_rn(u.th, __dadd_rn(P.pc.h2d.alpha_s,
-                                                    __dmul_rn(P.pc.h2d.beta_s_per_byte, __ull2double_rn(h))));
-            if (d) u.td = __dadd_rn(u.td, __dadd_rn(P.pc.d2h.alpha_s,
-                                                    __dmul_rn(P.pc.d2h.beta_s_per_byte, __ull2double_rn(d))));
-            u.h += h;
-            u.d += d;
-        }
+        if (stride > 4) group_usage<true, 2>(pp, stride, n_arrays, pm, a8, b8, P.pc, u);
+        else group_usage<false, 4>(pp, stride, n_arrays, pm, a8, b8, P.pc, u);
         ws.th[lane] = u.th;
         ws.td[lane] = u.td;
         ws.uh[lane] = u.h;
