@@ -95,6 +95,7 @@ struct SkelPlanHost {
     uint32_t poly_stride = 0;
 };
 constexpr uint32_t POLY_CLASSES = 64;
+constexpr uint32_t POLY_ZERO_WORDS = 10;   // SpaceDev::poly[0..9] = 0 (one zero polynomial)
 constexpr uint32_t SMALL_GRID_MAX = 1024;   // tabulated small grids per (kernel, xform)
 #define GROPHECY_TILE_CAP (1u << 21)        // tiles of 512 records per projection pass
 

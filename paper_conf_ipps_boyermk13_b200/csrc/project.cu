@@ -22,6 +22,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <type_traits>
 #include <cmath>
 
 #include "grophecy.h"
@@ -1142,7 +1143,8 @@ __device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsi
 template <bool BIQ, int AU>
 __device__ __forceinline__ void group_usage(const unsigned long long *pp, uint32_t stride,
                                             uint32_t n_arrays, uint32_t pm, uint32_t a8,
-                                            uint32_t b8, const grophecy_pcie &pc, Usage &u)
+                                            uint32_t b8, const grophecy_pcie &pc,
+                                            const unsigned long long *zero, Usage &u)
 {
     constexpr int NQ = BIQ ? 5 : 2;   // 16-byte coefficient pairs per polynomial
     for (uint32_t a0 = 0; a0 < n_arrays; a0 += AU) {
@@ -1153,9 +1155,10 @@ __device__ __forceinline__ void group_usage(const unsigned long long *pp, uint32
             for (int dir = 0; dir < 2; dir++) {
                 const uint32_t q = 2u * (a0 + (uint32_t)i) + (uint32_t)dir;
                 const bool on = a0 + (uint32_t)i < n_arrays && ((pm >> q) & 1u);
-                const ulonglong2 *src = reinterpret_cast<const ulonglong2 *>(pp + (size_t)q * stride);
+                const ulonglong2 *src =
+                    reinterpret_cast<const ulonglong2 *>(on ? pp + (size_t)q * stride : zero);
 #pragma unroll
-                for (int m = 0; m < NQ; m++) c[i][dir][m] = on ? __ldg(src + m) : make_ulonglong2(0, 0);
+                for (int m = 0; m < NQ; m++) c[i][dir][m] = __ldg(src + m);
             }
 #pragma unroll
         for (int i = 0; i < AU; i++) {
@@ -1309,8 +1312,8 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
         // skipped polynomials vanish in every class: their transfers add +0.0
         // to a sum that is never -0.0, i.e. nothing (exact)
         const uint32_t pm = I.poly_mask;
-        if (stride > 4) group_usage<true, 2>(pp, stride, n_arrays, pm, a8, b8, P.pc, u);
-        else group_usage<false, 4>(pp, stride, n_arrays, pm, a8, b8, P.pc, u);
+        if (stride > 4) group_usage<true, 2>(pp, stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
+        else group_usage<false, 4>(pp, stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
         ws.th[lane] = u.th;
         ws.td[lane] = u.td;
         ws.uh[lane] = u.h;
@@ -1356,10 +1359,15 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
             if (any) {
                 // off the saturated path: the small-grid table (SKF_TABULATED:
                 // blocks < sat32 <= small_stride; infeasible pairs never get here)
-                const double *tab = S.small_t + (size_t)kxi * S.small_stride;
+                // this pair's table row (32-bit element offset, space.cpp), pinned
+                // in a register once instead of being rematerialised per record
+                unsigned long long row;
+                asm volatile("mad.wide.u32 %0, %1, 8, %2;"
+                             : "=l"(row)
+                             : "r"(kxi * S.small_stride), "l"(S.small_t));
 #pragma unroll
                 for (int j = 0; j < CG; j++)
-                    if (gen[j]) tk[j] = __ldg(tab + blocks[j]);
+                    if (gen[j]) tk[j] = __ldg(reinterpret_cast<const double *>(row) + blocks[j]);
             }
             if ((pim >> k) & 1u) {
 #pragma unroll
@@ -1385,30 +1393,34 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
         const bool once = pim != (K == 32 ? 0xffffffffu : (1u << K) - 1u) || (xf & XINF_ONCE);
         double cm = __longlong_as_double(0x7ff0000000000000LL);
         int cj = -1;
+        auto totals = [&](auto ONCE) {
 #pragma unroll
-        for (int j = 0; j < CG; j++) {
-            const uint32_t g = 2u * (uint32_t)(i0g + j) + h;
-            double tk = __dmul_rn(ws.it[g], ti[j]);
-            if (once) tk = __dadd_rn(to[j], tk);
-            const double tt = __dadd_rn(__dadd_rn(tk, ws.th[g]), ws.td[g]);
-            if (BEST) {
-                // the lane's records come in increasing index order (tiles,
-                // chunks, j): strict < keeps the lowest index among ties
-                if (tt < cm) {
-                    cm = tt;
-                    cj = j;
+            for (int j = 0; j < CG; j++) {
+                const uint32_t g = 2u * (uint32_t)(i0g + j) + h;
+                double tk = __dmul_rn(ws.it[g], ti[j]);
+                if constexpr (decltype(ONCE)::value) tk = __dadd_rn(to[j], tk);
+                const double tt = __dadd_rn(__dadd_rn(tk, ws.th[g]), ws.td[g]);
+                if (BEST) {
+                    // the lane's records come in increasing index order (tiles,
+                    // chunks, j): strict < keeps the lowest index among ties
+                    if (tt < cm) {
+                        cm = tt;
+                        cj = j;
+                    }
+                } else {
+                    const unsigned long long r = tb + (unsigned long long)g * CX + x;
+                    __stcs(P.h2d + r, ws.uh[g]);
+                    __stcs(P.d2h + r, ws.ud[g]);
+                    __stcs(P.t + r, tt);
+                    if (P.p_iter) __stcs(P.p_iter + r, ti[j]);
+                    if (P.p_once) __stcs(P.p_once + r, to[j]);
+                    if (P.p_h2d) __stcs(P.p_h2d + r, ws.th[g]);
+                    if (P.p_d2h) __stcs(P.p_d2h + r, ws.td[g]);
                 }
-            } else {
-                const unsigned long long r = tb + (unsigned long long)g * CX + x;
-                __stcs(P.h2d + r, ws.uh[g]);
-                __stcs(P.d2h + r, ws.ud[g]);
-                __stcs(P.t + r, tt);
-                if (P.p_iter) __stcs(P.p_iter + r, ti[j]);
-                if (P.p_once) __stcs(P.p_once + r, to[j]);
-                if (P.p_h2d) __stcs(P.p_h2d + r, ws.th[g]);
-                if (P.p_d2h) __stcs(P.p_d2h + r, ws.td[g]);
             }
-        }
+        };
+        if (once) totals(std::true_type{});
+        else totals(std::false_type{});
         if (BEST && cm < best_t) {
             const uint32_t g = 2u * (uint32_t)(i0g + cj) + h;
             best_t = cm;

@@ -311,7 +311,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxG> kg;
     std::vector<KxFast> kf;
     std::vector<uint32_t> xinf;   // per (skeleton, xform) at kx_base + x: XINF_* bits
-    std::vector<unsigned long long> poly;
+    // poly[0..9]: an all-zero polynomial (the device reads it instead of the
+    // polynomials that vanish in every class: unconditional loads)
+    std::vector<unsigned long long> poly(POLY_ZERO_WORDS, 0ull);
     auto a4 = [](const grophecy_affine8 &a) { return make_int4(a.c0, a.c1, a.c2, a.c3); };
     for (uint32_t s = 0; s < n_skels; s++) {
         const grophecy_skeleton_desc &S = skels[s];
@@ -459,8 +461,10 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             for (uint32_t b = 0; b < kxf_sat(kf[q]); b++)
                 small[q * small_stride + b] = small_grid_time(kj[q], kg[q], gpu->n_sm, gpu->freq_hz, b);
 
+    // the canonical kernel indexes the table with 32-bit element offsets
+    const bool small_idx32 = (uint64_t)kf.size() * small_stride < (1ull << 32);
     for (uint32_t s = 0; s < n_skels; s++) {
-        bool tab = true;
+        bool tab = small_idx32;
         const uint32_t nkx = skels[s].n_kernels * skels[s].n_xforms;
         for (uint32_t q = info[s].kx_base; q < info[s].kx_base + nkx; q++)
             tab = tab && kxf_sat(kf[q]) <= small_stride;
