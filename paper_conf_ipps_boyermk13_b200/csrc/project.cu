@@ -740,6 +740,9 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
 // groups per pass, so one (kernel, x) constant load serves CG records.
 constexpr int CX = 16;
 constexpr int CTILE = 32 * CX;
+#ifndef GROPHECY_PREF
+#define GROPHECY_PREF 0
+#endif
 #ifndef GROPHECY_CG
 #define GROPHECY_CG 8
 #endif
@@ -1333,11 +1336,17 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
         for (int j = 0; j < CG; j++) ti[j] = to[j] = 0.0;
         const KxFast *F = F0;
         uint32_t kxi = I.kx_base + x;
+#if GROPHECY_PREF
         KxFast fn = *F0;   // K >= 1; the next kernel's constants load one step ahead
+#endif
 #pragma unroll 1
         for (uint32_t k = 0; k < K; k++, F += X, kxi += X) {
+#if GROPHECY_PREF
             const KxFast f = fn;   // this lane's (kernel, transformation) constants
             if (k + 1 < K) fn = F[X];
+#else
+            const KxFast f = *F;   // this lane's (kernel, transformation) constants
+#endif
             const uint32_t sat = f.satsh & KXF_SAT_MASK, sh = f.satsh >> KXF_SAT_BITS;
             uint32_t w[CG];
 #pragma unroll
