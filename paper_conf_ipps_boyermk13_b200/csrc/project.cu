@@ -84,6 +84,11 @@ struct SweepScratch {
     unsigned pr_m[64];          // strided arrays: regions whose row lattice hits residue rho
     unsigned pc_m[64];
     unsigned upto[32];
+    // strided arrays: (slab, residue) units aggregated by coverage mask,
+    // [0] rows / [1] columns (open addressing, key 0 = empty)
+    unsigned agg_key[2][64];
+    unsigned long long agg_sum[2][64];
+    unsigned agg_over;
 };
 
 constexpr int MAX_SEG = 8;                   // keys per warp pass (plan path)
@@ -259,7 +264,82 @@ __device__ __forceinline__ void strided_cells(SweepScratch &ws, unsigned Lr, uns
         if (rho < Lc) ws.pc_m[rho] = mc;
     }
     __syncwarp();
-    const int Uc = Sc * (int)Lc;
+    // Aggregate the row units (slab i, residue rho) by coverage mask — their
+    // heights add up, the first-reader / first-writer rule only sees the mask —
+    // and the column units likewise; then classify each (row mask, column
+    // mask) pair once with area = (sum of heights) x (sum of widths).  Far
+    // fewer cells than the units' product; a table overflow (> 64 distinct
+    // masks in a dimension) falls back to the product.
+    for (int q = lane; q < 128; q += 32) {
+        ws.agg_key[q >> 6][q & 63] = 0u;
+        ws.agg_sum[q >> 6][q & 63] = 0ull;
+    }
+    if (lane == 0) ws.agg_over = 0u;
+    __syncwarp();
+    auto insert = [&](int dim, unsigned m, unsigned long long v) {
+        unsigned slot = (m * 0x9E3779B1u) >> 26;
+        for (int probe = 0; probe < 64; probe++, slot = (slot + 1) & 63u) {
+            const unsigned old = atomicCAS(&ws.agg_key[dim][slot], 0u, m);
+            if (old == 0u || old == m) {
+                atomicAdd(&ws.agg_sum[dim][slot], v);
+                return;
+            }
+        }
+        ws.agg_over = 1u;
+    };
+    const int Ur = Sr * (int)Lr, Uc = Sc * (int)Lc;
+    for (int u = lane; u < Ur; u += 32) {
+        const int i = u / (int)Lr;
+        const unsigned rho = (unsigned)(u - i * (int)Lr);
+        const unsigned m = ws.rs_m[i] & ws.pr_m[rho];
+        if (!m) continue;
+        const unsigned long long hg = count_residue(ws.rs_a[i], ws.rs_h[i], rho, Lr);
+        if (hg) insert(0, m, hg);
+    }
+    for (int u = lane; u < Uc; u += 32) {
+        const int j = u / (int)Lc;
+        const unsigned sig = (unsigned)(u - j * (int)Lc);
+        const unsigned m = ws.cs_m[j] & ws.pc_m[sig];
+        if (!m) continue;
+        const unsigned long long wd = count_residue(ws.cs_a[j], ws.cs_w[j], sig, Lc);
+        if (wd) insert(1, m, wd);
+    }
+    __syncwarp();
+    if (!ws.agg_over) {
+        // occupied slots as bit lists (ballots over the 64 slots)
+        const unsigned long long occ_r =
+            (unsigned long long)__ballot_sync(FULL, ws.agg_key[0][lane] != 0u) |
+            (unsigned long long)__ballot_sync(FULL, ws.agg_key[0][lane + 32] != 0u) << 32;
+        const unsigned long long occ_c =
+            (unsigned long long)__ballot_sync(FULL, ws.agg_key[1][lane] != 0u) |
+            (unsigned long long)__ballot_sync(FULL, ws.agg_key[1][lane + 32] != 0u) << 32;
+        // compact into the (now free) slab arrays: masks -> rs_m / cs_m,
+        // summed heights / widths -> rs_h / cs_w
+        const unsigned long long below = (1ull << lane) - 1ull;
+        const unsigned kr0 = ws.agg_key[0][lane], kr1 = ws.agg_key[0][lane + 32];
+        const unsigned kc0 = ws.agg_key[1][lane], kc1 = ws.agg_key[1][lane + 32];
+        const unsigned long long sr0 = ws.agg_sum[0][lane], sr1 = ws.agg_sum[0][lane + 32];
+        const unsigned long long sc0 = ws.agg_sum[1][lane], sc1 = ws.agg_sum[1][lane + 32];
+        __syncwarp();
+        if (kr0) { const int q = __popcll(occ_r & below); ws.rs_m[q] = kr0; ws.rs_h[q] = (long long)sr0; }
+        if (kr1) { const int q = __popcll(occ_r & (below << 32 | 0xffffffffull)); ws.rs_m[q] = kr1; ws.rs_h[q] = (long long)sr1; }
+        if (kc0) { const int q = __popcll(occ_c & below); ws.cs_m[q] = kc0; ws.cs_w[q] = (long long)sc0; }
+        if (kc1) { const int q = __popcll(occ_c & (below << 32 | 0xffffffffull)); ws.cs_m[q] = kc1; ws.cs_w[q] = (long long)sc1; }
+        __syncwarp();
+        const int nr = __popcll(occ_r), nc = __popcll(occ_c);
+        for (int p = lane; p < nr * nc; p += 32) {
+            const int i = p / nc, j = p - i * nc;
+            const unsigned m = ws.rs_m[i] & ws.cs_m[j];
+            if (m) {
+                const unsigned long long area =
+                    (unsigned long long)ws.rs_h[i] * (unsigned long long)ws.cs_w[j];
+                const unsigned mr = m & Rm, mw = m & Wm;
+                if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) h += area;
+                if (mw) d += area;
+            }
+        }
+        return;
+    }
     for (int i = 0; i < Sr; i++) {
         const unsigned sm = ws.rs_m[i];
         if (!sm) continue;
