@@ -1700,12 +1700,20 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
 {
     const unsigned long long cap = (unsigned long long)GROPHECY_TILE_CAP * CTILE;
     const unsigned long long n = P.n;
+    // canonical groups sit at global indices that are multiples of CX (the
+    // sweep layout); a batch starting inside a group (e.g. a shard boundary)
+    // projects its head on its own so the tiles of the rest stay aligned
+    const unsigned long long head = (CX - P.base % CX) % CX;
     unsigned long long off = 0;
     do {
         Params Q = P;
-        Q.n = std::min(cap, n - off);
+        Q.n = off == 0 && head ? std::min(head, n) : std::min(cap, n - off);
         Q.skx += off; Q.nx += off; Q.ny += off; Q.iters += off;
         Q.base += off;
+        {
+            const uintptr_t m = (uintptr_t)Q.skx | (uintptr_t)Q.nx | (uintptr_t)Q.ny | (uintptr_t)Q.iters;
+            Q.aligned = (m & 15u) == 0;   // this chunk's records (vector loads, TMA)
+        }
         if (!BEST) {
             Q.h2d += off; Q.d2h += off; Q.t += off;
             if (Q.p_iter) Q.p_iter += off;

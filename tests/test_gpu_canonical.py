@@ -112,3 +112,24 @@ def test_canonical_tiles_with_invalid_record(G, O):
     orc, ob = P.best(rec)
     assert rc == G.EBADCAND and (b.index, b.n_invalid) == (ob.index, ob.n_invalid) == (ob.index, 1)
     space.close()
+
+
+@pytest.mark.parametrize("start", [333_333_333, 125_000_003])
+def test_shard_starting_inside_a_group(G, O, start):
+    """A shard boundary inside a design point (P = 3 shards of 10^9): the
+    head up to the next multiple of 16 is projected on its own, the rest in
+    canonical tiles; eval and best (global indices) match the oracle."""
+    c = R.config("c4")
+    rec = records_slice(c, np.arange(start, start + 3 * 512 + 40, dtype=np.uint64))
+    space = G.Space(c["skeletons"], S.FX5600)
+    pc = paper_pcie(G)
+    P = oracle_problem(O, c["skeletons"])
+    h, d, t = space.eval(pc, G.Records.from_numpy(rec), index_base=start)
+    torch.cuda.synchronize()
+    assert_same((h.cpu().numpy().view(np.uint64), d.cpu().numpy().view(np.uint64),
+                 t.cpu().numpy()), P.eval(rec))
+    rc, b = space.best(pc, G.Records.from_numpy(rec), index_base=start)
+    orc, ob = P.best(rec, index_base=start)
+    assert (b.index, b.n_valid) == (ob.index, ob.n_valid)
+    assert _bits([b.t_total_s]) == _bits([ob.t_total_s])
+    space.close()
