@@ -339,6 +339,60 @@ int grophecy_measure_transfer(int device, int direction, uint64_t bytes, int rep
 int grophecy_calibrate(int device, int reps, uint64_t large_bytes, grophecy_pcie *out);
 
 /* ---------------------------------------------------------------------- */
+/* Pinned vs pageable memory ("we may extend  */
+/* our framework to automatically explore the tradeoff between the two types */
+/* of memory", "account for the overhead of memory allocation";       */
+/* DESIGN.md reading 17)                                                    */
+/* ---------------------------------------------------------------------- */
+
+enum { GROPHECY_MEM_PINNED = 0, GROPHECY_MEM_PAGEABLE = 1 };
+
+/* grophecy_measure_transfer with the host buffer's memory type: PINNED
+ * (cudaHostAlloc, as grophecy_measure_transfer) or PAGEABLE (malloc'd,
+ * touched before timing).  Same protocol, outputs and limits. */
+int grophecy_measure_transfer_mem(int device, int direction, int memory, uint64_t bytes,
+                                  int reps, int warmup, double *mean_wall_s,
+                                  double *mean_event_s);
+
+/* Mean host steady-clock time of cudaHostAlloc(bytes) (mean_alloc_s) and of
+ * the matching cudaFreeHost (mean_free_s, may be NULL) over `reps` pairs
+ * after three discarded pairs; the buffer is not touched.  1 <= bytes <= 2^34. */
+int grophecy_measure_pin_alloc(int device, uint64_t bytes, int reps, double *mean_alloc_s,
+                               double *mean_free_s);
+
+/* The memory model: Eq. (1) links per direction for pinned and for pageable
+ * host memory, and the pinned allocation overhead in the same two-parameter
+ * form, A(F) = alpha + beta * F for a pinned buffer of F bytes (allocation +
+ * release; F = 0 -> 0). */
+typedef struct {
+    grophecy_pcie pinned, pageable;
+    grophecy_link pin_alloc;
+} grophecy_memory_model;
+
+/* Automatic calibration of the whole model with the paper's protocol
+ * (P:L113): per direction and memory type t_S (1 byte) and t_L (large_bytes),
+ * each the mean of `reps` transfers; A from a one-page and a large_bytes
+ * pinned allocation (alloc + free), alpha = t(4096), beta = t(large) / large. */
+int grophecy_calibrate_memory(int device, int reps, uint64_t large_bytes,
+                              grophecy_memory_model *out);
+
+/* The per-array choice (reading 17): with h2d / d2h the array's transfer
+ * bytes and footprint its full host buffer,
+ *   pinned   = (A(footprint) if h2d + d2h > 0 else 0) + T_pin,h2d(h2d) + T_pin,d2h(d2h)
+ *   pageable = T_page,h2d(h2d) + T_page,d2h(d2h)
+ * (sums left to right, Eq. (1) with T(0) = 0); memory = PINNED iff
+ * pinned <= pageable.  Pure host function.  EINVAL on NULL arguments or
+ * footprint < max(h2d, d2h). */
+typedef struct {
+    double t_pinned_s, t_pageable_s;
+    int32_t memory;
+    int32_t reserved;
+} grophecy_memory_choice;
+int grophecy_choose_memory(const grophecy_memory_model *model, uint64_t h2d_bytes,
+                           uint64_t d2h_bytes, uint64_t footprint_bytes,
+                           grophecy_memory_choice *out);
+
+/* ---------------------------------------------------------------------- */
 /* Synthetic workloads (bench / tests) — not part of the method             */
 /* ---------------------------------------------------------------------- */
 

@@ -39,6 +39,31 @@ double oracle_pcie_time(const or_link *l, uint64_t bytes)
     return l->alpha + l->beta * (double)bytes;
 }
 
+/* Pinned vs pageable (NEXT-4, reading 17): the paper's future work
+ * "explore the tradeoff between the two types of memory" and
+ * "account for the overhead of memory allocation".  Written out:
+ * both candidates priced with Eq. (1), the allocation of the whole host
+ * buffer in the same linear form, the cheaper one chosen (pinned on ties). */
+int oracle_choose_memory(const or_link *pin_h2d, const or_link *pin_d2h,
+                         const or_link *page_h2d, const or_link *page_d2h,
+                         const or_link *pin_alloc, uint64_t h2d, uint64_t d2h,
+                         uint64_t footprint, double *t_pinned, double *t_pageable,
+                         int *memory)
+{
+    if (footprint < h2d || footprint < d2h) return -1;
+    double alloc = 0.0;
+    if (h2d > 0 || d2h > 0) alloc = oracle_pcie_time(pin_alloc, footprint);
+    double pinned = alloc;
+    pinned = pinned + oracle_pcie_time(pin_h2d, h2d);
+    pinned = pinned + oracle_pcie_time(pin_d2h, d2h);
+    double pageable = oracle_pcie_time(page_h2d, h2d);
+    pageable = pageable + oracle_pcie_time(page_d2h, d2h);
+    *t_pinned = pinned;
+    *t_pageable = pageable;
+    *memory = pinned <= pageable ? 0 : 1;
+    return 0;
+}
+
 /* Size-affine value (N2): c0 + floor((c1 nx + c2 ny + c3 nx ny) / 8). */
 int64_t oracle_affine8(const or_affine8 *a, int64_t nx, int64_t ny)
 {

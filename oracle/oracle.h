@@ -25,6 +25,10 @@
  *                                           ("parity unpinned" by the paper itself)
  *   oracle_eval_one / oracle_best ........ pinned (composition identities, brute-force min)
  *   validation helpers ................... pinned (Table II arithmetic)
+ *   oracle_choose_memory ................. pinned to closed forms of OUR reading 17
+ *                                           (pinned vs pageable + allocation, NEXT-4);
+ *                                           the paper only names the tradeoff (P:L93,
+ *                                           L296): "parity unpinned" by the paper
  */
 #ifndef GROPHECY_ORACLE_H
 #define GROPHECY_ORACLE_H
@@ -70,6 +74,16 @@ typedef struct { double alpha, beta; } or_link;
 /* §III-C, Eq. (1) and P:L113 */
 int     oracle_fit_pcie(double t_small, double t_large, uint64_t large_bytes, or_link *out);
 double  oracle_pcie_time(const or_link *l, uint64_t bytes);
+
+/* NEXT-4 (reading 17): per-array pinned vs pageable
+ * choice.  pinned = (A(footprint) if any transfer else 0) + T_pin,h2d(h) +
+ * T_pin,d2h(d); pageable = T_page,h2d(h) + T_page,d2h(d); *memory = 0 (pinned)
+ * iff pinned <= pageable.  Returns -1 if footprint < max(h, d). */
+int oracle_choose_memory(const or_link *pin_h2d, const or_link *pin_d2h,
+                         const or_link *page_h2d, const or_link *page_d2h,
+                         const or_link *pin_alloc, uint64_t h2d, uint64_t d2h,
+                         uint64_t footprint, double *t_pinned, double *t_pageable,
+                         int *memory);
 
 int64_t oracle_affine8(const or_affine8 *a, int64_t nx, int64_t ny);
 

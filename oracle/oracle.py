@@ -91,6 +91,10 @@ def lib():
         L.oracle_fit_pcie.argtypes = [C.c_double, C.c_double, C.c_uint64, C.POINTER(Link)]
         L.oracle_pcie_time.argtypes = [C.POINTER(Link), C.c_uint64]
         L.oracle_pcie_time.restype = C.c_double
+        LP = C.POINTER(Link)
+        L.oracle_choose_memory.argtypes = [LP, LP, LP, LP, LP, C.c_uint64, C.c_uint64, C.c_uint64,
+                                           C.POINTER(C.c_double), C.POINTER(C.c_double),
+                                           C.POINTER(C.c_int)]
         L.oracle_affine8.argtypes = [C.POINTER(Affine8), C.c_int64, C.c_int64]
         L.oracle_affine8.restype = C.c_int64
         L.oracle_usage.argtypes = [SK, C.c_int64, C.c_int64, u64p, u64p]
@@ -179,6 +183,15 @@ def fit_pcie(t_small, t_large, large_bytes):
 
 def pcie_time(link, nbytes):
     return lib().oracle_pcie_time(C.byref(link), nbytes)
+
+
+def choose_memory(pin_h2d, pin_d2h, page_h2d, page_d2h, pin_alloc, h2d, d2h, footprint):
+    """NEXT-4 reading 17 -> (rc, t_pinned, t_pageable, memory: 0 pinned / 1 pageable)."""
+    tp, tg, m = C.c_double(), C.c_double(), C.c_int()
+    rc = lib().oracle_choose_memory(*[C.byref(x) for x in (pin_h2d, pin_d2h, page_h2d, page_d2h,
+                                                            pin_alloc)],
+                                    h2d, d2h, footprint, C.byref(tp), C.byref(tg), C.byref(m))
+    return rc, tp.value, tg.value, m.value
 
 
 def affine8(coef, nx, ny):

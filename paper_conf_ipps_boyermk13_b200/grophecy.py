@@ -44,6 +44,16 @@ class PCIe(C.Structure):
     _fields_ = [("h2d", Link), ("d2h", Link)]
 
 
+class MemoryModel(C.Structure):
+    """grophecy_memory_model (NEXT-4): pinned / pageable links + pinned allocation."""
+    _fields_ = [("pinned", PCIe), ("pageable", PCIe), ("pin_alloc", Link)]
+
+
+class MemoryChoice(C.Structure):
+    _fields_ = [("t_pinned_s", C.c_double), ("t_pageable_s", C.c_double),
+                ("memory", C.c_int32), ("reserved", C.c_int32)]
+
+
 class Affine8(C.Structure):
     _fields_ = [("c0", C.c_int32), ("c1", C.c_int32), ("c2", C.c_int32), ("c3", C.c_int32)]
 
@@ -150,6 +160,14 @@ _sig = {
     "grophecy_measure_transfer": (C.c_int, [C.c_int, C.c_int, C.c_uint64, C.c_int, C.c_int,
                                             C.POINTER(C.c_double), C.POINTER(C.c_double)]),
     "grophecy_calibrate": (C.c_int, [C.c_int, C.c_int, C.c_uint64, C.POINTER(PCIe)]),
+    "grophecy_measure_transfer_mem": (C.c_int, [C.c_int, C.c_int, C.c_int, C.c_uint64, C.c_int,
+                                                C.c_int, C.POINTER(C.c_double),
+                                                C.POINTER(C.c_double)]),
+    "grophecy_measure_pin_alloc": (C.c_int, [C.c_int, C.c_uint64, C.c_int, C.POINTER(C.c_double),
+                                             C.POINTER(C.c_double)]),
+    "grophecy_calibrate_memory": (C.c_int, [C.c_int, C.c_int, C.c_uint64, C.POINTER(MemoryModel)]),
+    "grophecy_choose_memory": (C.c_int, [C.POINTER(MemoryModel), C.c_uint64, C.c_uint64,
+                                         C.c_uint64, C.POINTER(MemoryChoice)]),
     "grophecy_synth_records": (C.c_int, [C.POINTER(SynthRule), C.c_uint32, C.c_uint64, C.c_uint32,
                                          C.c_uint64, C.c_uint64, C.c_uint64, _vp, _vp, _vp, _vp,
                                          _vp]),
@@ -443,6 +461,37 @@ def measure_transfer(device, direction, nbytes, reps=10, warmup=2):
 def calibrate(device=0, reps=10, large_bytes=1 << 29):
     out = PCIe()
     _check(_L.grophecy_calibrate(device, reps, large_bytes, C.byref(out)), "calibrate")
+    return out
+
+
+MEM_PINNED, MEM_PAGEABLE = 0, 1
+
+
+def measure_transfer_mem(device, direction, memory, nbytes, reps=10, warmup=2):
+    wall, ev = C.c_double(), C.c_double()
+    _check(_L.grophecy_measure_transfer_mem(device, direction, memory, nbytes, reps, warmup,
+                                            C.byref(wall), C.byref(ev)), "measure_transfer_mem")
+    return wall.value, ev.value
+
+
+def measure_pin_alloc(device, nbytes, reps=10):
+    a, f = C.c_double(), C.c_double()
+    _check(_L.grophecy_measure_pin_alloc(device, nbytes, reps, C.byref(a), C.byref(f)),
+           "measure_pin_alloc")
+    return a.value, f.value
+
+
+def calibrate_memory(device=0, reps=10, large_bytes=1 << 29):
+    out = MemoryModel()
+    _check(_L.grophecy_calibrate_memory(device, reps, large_bytes, C.byref(out)),
+           "calibrate_memory")
+    return out
+
+
+def choose_memory(model, h2d_bytes, d2h_bytes, footprint_bytes):
+    out = MemoryChoice()
+    _check(_L.grophecy_choose_memory(C.byref(model), h2d_bytes, d2h_bytes, footprint_bytes,
+                                     C.byref(out)), "choose_memory")
     return out
 
 

@@ -35,11 +35,12 @@ def default_sizes(lo_exp=10, hi_exp=30, include_one=True):
     return ([1] if include_one else []) + [1 << e for e in range(lo_exp, hi_exp + 1)]
 
 
-def sweep(device, sizes, reps=10, warmup=2):
+def sweep(device, sizes, reps=10, warmup=2, memory=G.MEM_PINNED):
     """{direction: [(bytes, mean_wall_s, mean_event_s)]} for one device."""
     out = {}
     for name, d in DIRS:
-        out[name] = [(s, *G.measure_transfer(device, d, s, reps, warmup)) for s in sizes]
+        out[name] = [(s, *G.measure_transfer_mem(device, d, memory, s, reps, warmup))
+                     for s in sizes]
     return out
 
 
@@ -123,3 +124,68 @@ def validate(devices, sizes=None, reps=10, warmup=2, large=1 << 29, concurrent=T
 
 def calibrate(device=0, reps=10, large=1 << 29):
     return G.calibrate(device, reps, large)
+
+
+def memory_tradeoff(device, sizes=None, reps=10, warmup=2, large=1 << 29,
+                    alloc_sizes=None):
+    """NEXT-4 (reading 17): the pageable sweep with
+    its own two-point fit and validation errors, the speedup of pinned over
+    pageable per size and direction (the paper's Fig. 3), the pinned
+    allocation overhead line A(F) = alpha + beta F (fit at 4 KiB and `large`,
+    checked on a size sweep), and where the per-array choice flips for an
+    array whose footprint equals its transfer size."""
+    sizes = sizes or default_sizes()
+    if large not in sizes:
+        sizes = sorted(set(sizes) | {large})
+    pin = sweep(device, sizes, reps, warmup, G.MEM_PINNED)
+    page = sweep(device, sizes, reps, warmup, G.MEM_PAGEABLE)
+    pin_links, page_links = fit_from_sweep(pin, large), fit_from_sweep(page, large)
+    speed = {}
+    for name, _ in DIRS:
+        speed[name] = [{"bytes": a[0], "pinned_s": a[1], "pageable_s": b[1],
+                        "pinned_speedup": b[1] / a[1]} for a, b in zip(pin[name], page[name])]
+    # piecewise-linear alternative for the pageable links (footnote 4: pageable
+    # transfers are "slightly more non-linear"): knots at 2^0, 2^12, 2^16,
+    # 2^20, 2^24 and `large`, linear in d between knots, the last slope beyond
+    knots = [k for k in (1, 1 << 12, 1 << 16, 1 << 20, 1 << 24, large) if k in sizes]
+    piecewise = {}
+    for name, _ in DIRS:
+        t = {s_: w for s_, w, _ in page[name]}
+        kt = [(k, t[k]) for k in knots]
+
+        def pred(d, kt=kt):
+            for (x0, y0), (x1, y1) in zip(kt, kt[1:]):
+                if d <= x1 or (x1, y1) == kt[-1]:
+                    return y0 + (y1 - y0) * (d - x0) / (x1 - x0)
+            return kt[-1][1]
+        errs = [error_magnitude(pred(s_), w) for s_, w, _ in page[name]]
+        piecewise[name] = {"knots": knots, "mean_error": mean(errs), "max_error": max(errs)}
+    alloc_sizes = alloc_sizes or [1 << e for e in range(12, 31, 2)]
+    if 4096 not in alloc_sizes or large not in alloc_sizes:
+        alloc_sizes = sorted(set(alloc_sizes) | {4096, large})
+    at = {s: sum(G.measure_pin_alloc(device, s, reps)) for s in alloc_sizes}
+    alloc_link = G.fit_pcie(at[4096], at[large], large)
+    alloc_rows = [{"bytes": s, "measured_s": t, "predicted_s": G.pcie_time(alloc_link, s),
+                   "error": error_magnitude(G.pcie_time(alloc_link, s), t)} for s, t in at.items()]
+    model = G.MemoryModel()
+    model.pinned.h2d, model.pinned.d2h = pin_links["h2d"], pin_links["d2h"]
+    model.pageable.h2d, model.pageable.d2h = page_links["h2d"], page_links["d2h"]
+    model.pin_alloc = alloc_link
+    choice = {}
+    for name, _ in DIRS:
+        rows = []
+        for s in sizes:
+            c = G.choose_memory(model, s if name == "h2d" else 0, s if name == "d2h" else 0, s)
+            rows.append({"bytes": s, "t_pinned_s": c.t_pinned_s, "t_pageable_s": c.t_pageable_s,
+                         "memory": "pinned" if c.memory == G.MEM_PINNED else "pageable"})
+        choice[name] = rows
+    return {"device": device, "sizes": sizes, "reps": reps,
+            "pageable_fit": {k: _link_dict(v) for k, v in page_links.items()},
+            "pinned_fit": {k: _link_dict(v) for k, v in pin_links.items()},
+            "pageable_errors": score(page, page_links),
+            "pageable_piecewise": piecewise,
+            "pinned_speedup": speed,
+            "pin_alloc_fit": {"alpha_s": alloc_link.alpha_s,
+                              "beta_s_per_byte": alloc_link.beta_s_per_byte},
+            "pin_alloc": alloc_rows,
+            "choice_single_transfer_arrays": choice}

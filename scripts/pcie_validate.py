@@ -22,6 +22,8 @@ def main():
     devs = list(range(torch.cuda.device_count()))
     rep = pcie.validate(devs, reps=reps)
     rep["gpus"] = [torch.cuda.get_device_name(d) for d in devs]
+    if not os.environ.get("NO_MEMORY_TRADEOFF"):
+        rep["memory_tradeoff"] = [pcie.memory_tradeoff(d, reps=reps) for d in devs[:1]]
     os.makedirs(os.path.dirname(out) or ".", exist_ok=True)
     json.dump(rep, open(out, "w"), indent=1)
     for r in rep["single"]:
@@ -30,6 +32,20 @@ def main():
             print(f"gpu{r['device']} {d}: alpha={f['alpha_s']*1e6:.2f}us "
                   f"1/beta={f['bandwidth_GBps']:.2f}GB/s mean_err={100*e['mean_error']:.2f}% "
                   f"max_err={100*e['max_error']:.2f}% noise_floor={100*nf['mean_error']:.2f}%")
+    for r in rep.get("memory_tradeoff", []):
+        for d in ("h2d", "d2h"):
+            f, e = r["pageable_fit"][d], r["pageable_errors"][d]
+            sp = r["pinned_speedup"][d]
+            flips = [x["bytes"] for x in r["choice_single_transfer_arrays"][d]
+                     if x["memory"] == "pageable"]
+            print(f"gpu{r['device']} pageable {d}: alpha={f['alpha_s']*1e6:.2f}us "
+                  f"1/beta={f['bandwidth_GBps']:.2f}GB/s mean_err={100*e['mean_error']:.2f}% "
+                  f"pinned speedup {min(x['pinned_speedup'] for x in sp):.2f}-"
+                  f"{max(x['pinned_speedup'] for x in sp):.2f}x; pageable chosen at {flips[:6]}; "
+                  f"piecewise mean_err={100*r['pageable_piecewise'][d]['mean_error']:.2f}%")
+        a = r["pin_alloc_fit"]
+        print(f"gpu{r['device']} pinned alloc: alpha={a['alpha_s']*1e6:.1f}us "
+              f"beta={a['beta_s_per_byte']*1e12:.2f}ps/B")
 
 
 if __name__ == "__main__":

@@ -43,3 +43,22 @@ def test_measure_rejects_bad_args(G):
         G.measure_transfer(0, 5, 1024)
     with pytest.raises(G.GrophecyError):
         G.measure_transfer(0, 0, 0)
+
+
+def test_memory_model_calibration(G):
+    """NEXT-4: pageable links and the pinned allocation line come out of the
+    same two-point protocol with physical magnitudes; large transfers are
+    faster from pinned memory (Fig. 3); the choice is consistent with
+    the calibrated model."""
+    m = G.calibrate_memory(0, reps=3, large_bytes=1 << 26)
+    for l in (m.pinned.h2d, m.pinned.d2h, m.pageable.h2d, m.pageable.d2h):
+        assert 1e-7 < l.alpha_s < 1e-2
+        assert 1e8 < 1.0 / l.beta_s_per_byte < 1e12
+    assert m.pin_alloc.alpha_s > 0 and m.pin_alloc.beta_s_per_byte > 0
+    pin, _ = G.measure_transfer_mem(0, G.DIR_H2D, G.MEM_PINNED, 1 << 26, reps=3)
+    page, _ = G.measure_transfer_mem(0, G.DIR_H2D, G.MEM_PAGEABLE, 1 << 26, reps=3)
+    assert pin < page
+    c = G.choose_memory(m, 1 << 26, 0, 1 << 26)
+    assert c.memory == (G.MEM_PINNED if c.t_pinned_s <= c.t_pageable_s else G.MEM_PAGEABLE)
+    a, f = G.measure_pin_alloc(0, 1 << 20, reps=3)
+    assert a > 0 and f > 0
