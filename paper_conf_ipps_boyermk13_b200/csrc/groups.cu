@@ -230,6 +230,7 @@ extern "C" int grophecy_group_best(grophecy_space *s, const grophecy_pcie *pc,
     }
     *n_groups = 0;
     if (b->n == 0) return GROPHECY_OK;
+    DeviceGuard guard(s->device);
     cudaStream_t st = (cudaStream_t)stream;
     const unsigned long long n = b->n;
     const unsigned long long nb = (n + G_BLOCK - 1) / G_BLOCK;

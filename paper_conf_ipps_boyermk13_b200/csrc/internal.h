@@ -171,6 +171,20 @@ struct grophecy_space {
 };
 
 namespace grophecy {
+// Makes the space's device current for one ABI call (and restores the
+// caller's): launches, streams and the per-device kernel attributes match.
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int device)
+    {
+        if (cudaGetDevice(&prev) == cudaSuccess && prev != device) cudaSetDevice(device);
+        else prev = -1;
+    }
+    ~DeviceGuard()
+    {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
 bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out);
 void set_error(const std::string &msg);
 int cuda_fail(cudaError_t e, const char *what);

@@ -1663,7 +1663,11 @@ __global__ void combine_kernel(const grophecy_best_result *in, uint32_t count,
 
 static void set_smem_attrs()
 {
-    static bool done = false;
+    // per device: the attributes belong to the current device's context
+    static bool done_dev[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    bool &done = done_dev[dev & 63];
     if (done) return;
     const int sm = (int)sizeof(CtaSmem), cs = (int)sizeof(CanonCtaSmem);
     cudaFuncSetAttribute(canon_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
@@ -1780,6 +1784,7 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
 int launch_best(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
                 grophecy_best_result *dout, int accumulate, cudaStream_t st)
 {
+    DeviceGuard guard(s->device);
     Params P = make_params(s, pc, b);
     P.out = dout;
     P.accumulate = accumulate;
@@ -1807,6 +1812,7 @@ int grophecy_eval_parts(const grophecy_space *s, const grophecy_pcie *pc, const 
     P.h2d = (unsigned long long *)h2d;
     P.d2h = (unsigned long long *)d2h;
     P.t = t;
+    DeviceGuard guard(s->device);
     if (parts) {
         P.p_iter = parts->t_iter_s;
         P.p_once = parts->t_once_s;
@@ -1858,6 +1864,7 @@ int grophecy_best(grophecy_space *s, const grophecy_pcie *pc, const grophecy_bat
     }
     cudaStream_t st = (cudaStream_t)stream;
     // the result slot lives in the space's scratch, after the partials
+    DeviceGuard guard(s->device);
     grophecy_best_result *dres = s->partials + (s->max_partials - 1);
     rc = launch_best(s, pc, b, dres, 0, st);
     if (rc) return rc;
@@ -1895,6 +1902,7 @@ int grophecy_best_host(grophecy_space *s, const grophecy_pcie *pc, const uint32_
     }
     cudaStream_t st = (cudaStream_t)stream;
     cudaError_t e;
+    DeviceGuard guard(s->device);
     const uint64_t CHUNK = 1ull << 23;   // records per chunk (128 MiB of records)
     const size_t need = (size_t)CHUNK * 16;
     if (!s->copy_stream) {
