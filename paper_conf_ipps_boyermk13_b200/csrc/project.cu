@@ -820,9 +820,6 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
 // groups per pass, so one (kernel, x) constant load serves CG records.
 constexpr int CX = 16;
 constexpr int CTILE = 32 * CX;
-#ifndef GROPHECY_PREF
-#define GROPHECY_PREF 0
-#endif
 #ifndef GROPHECY_CG
 #define GROPHECY_CG 8
 #endif
@@ -1326,7 +1323,6 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
                                            unsigned long long &best_i, uint32_t &cnt_val)
 {
     const SpaceDev &S = P.S;
-    const unsigned long long q0 = tb + (unsigned long long)lane * CX;
     // ---- A (records staged in ws.rec by the TMA; lane l reads its group's
     //      16-byte chunks in the rotated order c = (m + l/2) mod 4, which
     //      spreads 8 consecutive lanes over all 32 banks) ----
@@ -1414,58 +1410,52 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
         double ti[CG], to[CG];
 #pragma unroll
         for (int j = 0; j < CG; j++) ti[j] = to[j] = 0.0;
-        const KxFast *F = F0;
-        uint32_t kxi = I.kx_base + x;
-#if GROPHECY_PREF
-        KxFast fn = *F0;   // K >= 1; the next kernel's constants load one step ahead
-#endif
+        // the kernels of one sum (bit k of `mask`) in ascending k: this lane's
+        // (kernel, transformation) constants, the 8 groups' work counts, the
+        // saturated model, small grids from the table, the sum (N6)
+        auto kernel_sum = [&](uint32_t mask, double (&acc)[CG]) {
 #pragma unroll 1
-        for (uint32_t k = 0; k < K; k++, F += X, kxi += X) {
-#if GROPHECY_PREF
-            const KxFast f = fn;   // this lane's (kernel, transformation) constants
-            if (k + 1 < K) fn = F[X];
-#else
-            const KxFast f = *F;   // this lane's (kernel, transformation) constants
-#endif
-            const uint32_t sat = f.satsh & KXF_SAT_MASK, sh = f.satsh >> KXF_SAT_BITS;
-            uint32_t w[CG];
+            for (; mask; mask &= mask - 1u) {
+                const uint32_t k = (uint32_t)__ffs(mask) - 1u;
+                const uint32_t kxi = I.kx_base + x + k * X;
+                const KxFast f = F0[(size_t)k * X];
+                const uint32_t sat = f.satsh & KXF_SAT_MASK, sh = f.satsh >> KXF_SAT_BITS;
+                uint32_t w[CG];
 #pragma unroll
-            for (int j = 0; j < CG; j += 4) {
-                const uint4 v = *reinterpret_cast<const uint4 *>(&ws.cw[k][h][i0g + j]);
-                w[j] = v.x;
-                w[j + 1] = v.y;
-                w[j + 2] = v.z;
-                w[j + 3] = v.w;
+                for (int j = 0; j < CG; j += 4) {
+                    const uint4 v = *reinterpret_cast<const uint4 *>(&ws.cw[k][h][i0g + j]);
+                    w[j] = v.x;
+                    w[j + 1] = v.y;
+                    w[j + 2] = v.z;
+                    w[j + 3] = v.w;
+                }
+                double tk[CG];
+                bool gen[CG], any = false;
+                uint32_t blocks[CG];
+#pragma unroll
+                for (int j = 0; j < CG; j++) {
+                    tk[j] = fast_time(f, sat, sh, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
+                    any |= gen[j];
+                }
+                if (any) {
+                    // off the saturated path: the small-grid table (SKF_TABULATED:
+                    // blocks < sat <= small_stride; infeasible pairs never get
+                    // here); this pair's table row (32-bit element offset) once
+                    unsigned long long row;
+                    asm volatile("mad.wide.u32 %0, %1, 8, %2;"
+                                 : "=l"(row)
+                                 : "r"(kxi * S.small_stride), "l"(S.small_t));
+#pragma unroll
+                    for (int j = 0; j < CG; j++)
+                        if (gen[j]) tk[j] = __ldg(reinterpret_cast<const double *>(row) + blocks[j]);
+                }
+#pragma unroll
+                for (int j = 0; j < CG; j++) acc[j] = __dadd_rn(acc[j], tk[j]);
             }
-            double tk[CG];
-            bool gen[CG], any = false;
-            uint32_t blocks[CG];
-#pragma unroll
-            for (int j = 0; j < CG; j++) {
-                tk[j] = fast_time(f, sat, sh, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
-                any |= gen[j];
-            }
-            if (any) {
-                // off the saturated path: the small-grid table (SKF_TABULATED:
-                // blocks < sat32 <= small_stride; infeasible pairs never get here)
-                // this pair's table row (32-bit element offset, space.cpp), pinned
-                // in a register once instead of being rematerialised per record
-                unsigned long long row;
-                asm volatile("mad.wide.u32 %0, %1, 8, %2;"
-                             : "=l"(row)
-                             : "r"(kxi * S.small_stride), "l"(S.small_t));
-#pragma unroll
-                for (int j = 0; j < CG; j++)
-                    if (gen[j]) tk[j] = __ldg(reinterpret_cast<const double *>(row) + blocks[j]);
-            }
-            if ((pim >> k) & 1u) {
-#pragma unroll
-                for (int j = 0; j < CG; j++) ti[j] = __dadd_rn(ti[j], tk[j]);
-            } else {
-#pragma unroll
-                for (int j = 0; j < CG; j++) to[j] = __dadd_rn(to[j], tk[j]);
-            }
-        }
+        };
+        const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
+        kernel_sum(pim & kmask, ti);                       // t_iter
+        if (~pim & kmask) kernel_sum(~pim & kmask, to);    // t_once
         // infeasible kernels: that sum is +inf (exact, see xinf)
         const double inf = __longlong_as_double(0x7ff0000000000000LL);
         if (xf & XINF_ITER) {
