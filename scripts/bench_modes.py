@@ -91,6 +91,19 @@ def main():
                           "bytes_per_candidate": bpc, "hbm_GBps": gbs, "hbm_frac": gbs / peak,
                           "timer": "cuda events" if ev else "host clock (synchronous call)"}),
               flush=True)
+    # the general (pass-2) kernel alone: the same records with the
+    # transformations of every design point in reverse order, so no tile is
+    # canonical (keys and their runs unchanged)
+    idx = torch.arange(n, device="cuda")
+    idx = (idx // 16) * 16 + 15 - (idx % 16)
+    grec = G.Records(*[getattr(rec, f)[idx].contiguous() for f in ("skx", "nx", "ny", "iters")])
+    gb = grec.batch()
+    sec = timed(lambda: space.best_async(pc, gb, out), reps, True)
+    gbs = 16 * n / sec / 1e9
+    print(json.dumps({"mode": "best_general_path", "n": n, "cand_per_s": n / sec,
+                      "ms": sec * 1e3, "bytes_per_candidate": 16, "hbm_GBps": gbs,
+                      "hbm_frac": gbs / peak, "timer": "cuda events"}), flush=True)
+    del grec, gb, idx
     # next-row workloads: crossover (NEXT-2) on eval_parts outputs
     ti, to, th, td = parts
     sec = timed(lambda: G.crossover(ti, to, th, td, 1e-3), reps, True)
