@@ -1413,45 +1413,48 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
         // the kernels of one sum (bit k of `mask`) in ascending k: this lane's
         // (kernel, transformation) constants, the 8 groups' work counts, the
         // saturated model, small grids from the table, the sum (N6)
+        auto one_kernel = [&](uint32_t k, double (&acc)[CG]) {
+            const uint32_t kxi = I.kx_base + x + k * X;
+            const KxFast f = F0[(size_t)k * X];
+            const uint32_t sat = f.satsh & KXF_SAT_MASK, sh = f.satsh >> KXF_SAT_BITS;
+            uint32_t w[CG];
+#pragma unroll
+            for (int j = 0; j < CG; j += 4) {
+                const uint4 v = *reinterpret_cast<const uint4 *>(&ws.cw[k][h][i0g + j]);
+                w[j] = v.x;
+                w[j + 1] = v.y;
+                w[j + 2] = v.z;
+                w[j + 3] = v.w;
+            }
+            double tk[CG];
+            bool gen[CG], any = false;
+            uint32_t blocks[CG];
+#pragma unroll
+            for (int j = 0; j < CG; j++) {
+                tk[j] = fast_time(f, sat, sh, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
+                any |= gen[j];
+            }
+            if (any) {
+                // off the saturated path: the small-grid table (SKF_TABULATED:
+                // blocks < sat <= small_stride; infeasible pairs never get
+                // here); this pair's table row (32-bit element offset) once
+                unsigned long long row;
+                asm volatile("mad.wide.u32 %0, %1, 8, %2;"
+                             : "=l"(row)
+                             : "r"(kxi * S.small_stride), "l"(S.small_t));
+#pragma unroll
+                for (int j = 0; j < CG; j++)
+                    if (gen[j]) tk[j] = __ldg(reinterpret_cast<const double *>(row) + blocks[j]);
+            }
+#pragma unroll
+            for (int j = 0; j < CG; j++) acc[j] = __dadd_rn(acc[j], tk[j]);
+        };
+        // the kernels of one sum (bit k of `mask`) in ascending k: this lane's
+        // (kernel, transformation) constants, the 8 groups' work counts, the
+        // saturated model, small grids from the table, the sum (N6)
         auto kernel_sum = [&](uint32_t mask, double (&acc)[CG]) {
 #pragma unroll 1
-            for (; mask; mask &= mask - 1u) {
-                const uint32_t k = (uint32_t)__ffs(mask) - 1u;
-                const uint32_t kxi = I.kx_base + x + k * X;
-                const KxFast f = F0[(size_t)k * X];
-                const uint32_t sat = f.satsh & KXF_SAT_MASK, sh = f.satsh >> KXF_SAT_BITS;
-                uint32_t w[CG];
-#pragma unroll
-                for (int j = 0; j < CG; j += 4) {
-                    const uint4 v = *reinterpret_cast<const uint4 *>(&ws.cw[k][h][i0g + j]);
-                    w[j] = v.x;
-                    w[j + 1] = v.y;
-                    w[j + 2] = v.z;
-                    w[j + 3] = v.w;
-                }
-                double tk[CG];
-                bool gen[CG], any = false;
-                uint32_t blocks[CG];
-#pragma unroll
-                for (int j = 0; j < CG; j++) {
-                    tk[j] = fast_time(f, sat, sh, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
-                    any |= gen[j];
-                }
-                if (any) {
-                    // off the saturated path: the small-grid table (SKF_TABULATED:
-                    // blocks < sat <= small_stride; infeasible pairs never get
-                    // here); this pair's table row (32-bit element offset) once
-                    unsigned long long row;
-                    asm volatile("mad.wide.u32 %0, %1, 8, %2;"
-                                 : "=l"(row)
-                                 : "r"(kxi * S.small_stride), "l"(S.small_t));
-#pragma unroll
-                    for (int j = 0; j < CG; j++)
-                        if (gen[j]) tk[j] = __ldg(reinterpret_cast<const double *>(row) + blocks[j]);
-                }
-#pragma unroll
-                for (int j = 0; j < CG; j++) acc[j] = __dadd_rn(acc[j], tk[j]);
-            }
+            for (; mask; mask &= mask - 1u) one_kernel((uint32_t)__ffs(mask) - 1u, acc);
         };
         const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
         kernel_sum(pim & kmask, ti);                       // t_iter
