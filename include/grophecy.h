@@ -424,7 +424,9 @@ int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int64_t nx, int
 /* Diagnostic: size of the usage plan compiled for `skel`: stats[0] =
  * expressions, [1] = program words, [2] = terms, [3] = terms, [4] = max terms
  * of one array program, [5] = max words of one program, [6] = coefficients
- * per byte polynomial (4 bilinear, 10 otherwise).  `stats` holds 7 entries.
+ * per byte polynomial (4 bilinear, 10 otherwise), [7] = distinct residue
+ * classes among the 64 polynomial sets, [8] = polynomial table bytes.
+ * `stats` holds 9 entries.
  * ELIMIT if the skeleton has no plan.  Pure host function. */
 int grophecy_plan_stats(const grophecy_skeleton_desc *skel, uint32_t *stats);
 

@@ -60,7 +60,11 @@ struct SkelInfo {
     uint32_t plan_tx, plan_ty, poly_base, poly_stride;
     uint32_t per_iter_mask;   // bit k = kernel k per-iteration
     uint32_t poly_mask;       // bit 2a + dir: byte polynomial not zero in every size class
-    uint32_t pad2, pad3;
+    // compact copy of a bilinear table whose coefficients all fit int32:
+    // poly[poly32_base + 2 * (c * n_polys + p)] holds int4 {c0, c1, c2, c3}
+    // (sign-extended they are the u64 coefficients); POLY32_NONE if absent
+    uint32_t poly32_base;
+    uint32_t pad3;
 };
 
 struct ArrayDev {
@@ -96,6 +100,7 @@ struct SkelPlanHost {
 };
 constexpr uint32_t POLY_CLASSES = 64;
 constexpr uint32_t POLY_ZERO_WORDS = 10;   // SpaceDev::poly[0..9] = 0 (one zero polynomial)
+constexpr uint32_t POLY32_NONE = 0xffffffffu;
 constexpr uint32_t SMALL_GRID_MAX = 1024;   // tabulated small grids per (kernel, xform)
 #define GROPHECY_TILE_CAP (1u << 21)        // tiles of 512 records per projection pass
 

@@ -434,5 +434,17 @@ extern "C" int grophecy_plan_stats(const grophecy_skeleton_desc *skel, uint32_t 
     stats[4] = maxb;
     stats[5] = maxw;
     stats[6] = P.poly_stride;
+    // distinct residue classes among the 64 byte-polynomial sets
+    const size_t blk = 2 * (size_t)skel->n_arrays * P.poly_stride;
+    uint32_t distinct = 0;
+    for (size_t c = 0; c < POLY_CLASSES; c++) {
+        bool seen = false;
+        for (size_t e = 0; e < c && !seen; e++)
+            seen = std::equal(P.poly.begin() + c * blk, P.poly.begin() + (c + 1) * blk,
+                              P.poly.begin() + e * blk);
+        distinct += !seen;
+    }
+    stats[7] = distinct;
+    stats[8] = (uint32_t)(P.poly.size() * sizeof(uint64_t));
     return GROPHECY_OK;
 }

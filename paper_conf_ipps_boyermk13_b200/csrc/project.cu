@@ -820,6 +820,9 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
 // groups per pass, so one (kernel, x) constant load serves CG records.
 constexpr int CX = 16;
 constexpr int CTILE = 32 * CX;
+#ifndef GROPHECY_AU32
+#define GROPHECY_AU32 4
+#endif
 #ifndef GROPHECY_CG
 #define GROPHECY_CG 8
 #endif
@@ -1263,6 +1266,46 @@ __device__ __forceinline__ void group_usage(const unsigned long long *pp, uint32
     }
 }
 
+// group_usage over the compact table (SkelInfo::poly32_base): one 16-byte
+// load {c0, c1, c2, c3} (int32, the u64 coefficients sign-extended) per
+// polynomial; evaluated with wrapping 64-bit arithmetic like the u64 table
+// (the same residues mod 2^64, hence the same bytes).
+template <int AU>
+__device__ __forceinline__ void group_usage32(const int4 *pp, uint32_t n_arrays, uint32_t pm,
+                                              uint32_t a8, uint32_t b8, const grophecy_pcie &pc,
+                                              const int4 *zero, Usage &u)
+{
+    const long long a = (long long)a8, b = (long long)b8;
+    for (uint32_t a0 = 0; a0 < n_arrays; a0 += AU) {
+        int4 c[AU][2];
+#pragma unroll
+        for (int i = 0; i < AU; i++)
+#pragma unroll
+            for (int dir = 0; dir < 2; dir++) {
+                const uint32_t q = 2u * (a0 + (uint32_t)i) + (uint32_t)dir;
+                const bool on = a0 + (uint32_t)i < n_arrays && ((pm >> q) & 1u);
+                c[i][dir] = __ldg(on ? pp + q : zero);
+            }
+#pragma unroll
+        for (int i = 0; i < AU; i++) {
+            if (a0 + (uint32_t)i >= n_arrays) break;
+            unsigned long long v[2];
+#pragma unroll
+            for (int dir = 0; dir < 2; dir++) {
+                const int4 k = c[i][dir];
+                const unsigned long long t = (unsigned long long)((long long)k.w * a + (long long)k.z);
+                v[dir] = (unsigned long long)((long long)k.y * a + (long long)k.x) + t * (unsigned long long)b;
+            }
+            if (v[0]) u.th = __dadd_rn(u.th, __dadd_rn(pc.h2d.alpha_s,
+                                                       __dmul_rn(pc.h2d.beta_s_per_byte, __ull2double_rn(v[0]))));
+            if (v[1]) u.td = __dadd_rn(u.td, __dadd_rn(pc.d2h.alpha_s,
+                                                       __dmul_rn(pc.d2h.beta_s_per_byte, __ull2double_rn(v[1]))));
+            u.h += v[0];
+            u.d += v[1];
+        }
+    }
+}
+
 // ---- 1-D bulk copies (TMA) global -> shared with mbarrier completion ----
 __device__ __forceinline__ uint32_t smem_u32(const void *p)
 {
@@ -1391,7 +1434,12 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
         // skipped polynomials vanish in every class: their transfers add +0.0
         // to a sum that is never -0.0, i.e. nothing (exact)
         const uint32_t pm = I.poly_mask;
-        if (stride > 4) group_usage<true, 2>(pp, stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
+        if (I.poly32_base != POLY32_NONE)
+            group_usage32<GROPHECY_AU32>(reinterpret_cast<const int4 *>(S.poly + I.poly32_base) +
+                                             (size_t)((n0 & 7u) * 8u + (m0 & 7u)) * (2u * n_arrays),
+                                         n_arrays, pm, a8, b8, P.pc,
+                                         reinterpret_cast<const int4 *>(S.poly), u);
+        else if (stride > 4) group_usage<true, 2>(pp, stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
         else group_usage<false, 4>(pp, stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
         ws.th[lane] = u.th;
         ws.td[lane] = u.td;

@@ -10,6 +10,7 @@
 #include <atomic>
 #include <cmath>
 #include <cstdio>
+#include <climits>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -348,12 +349,32 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 for (size_t q = 0; q < np; q++)
                     for (size_t m = 0; m < st; m++)
                         if (plan.poly[(c * np + q) * st + m]) I.poly_mask |= 1u << q;
+            // compact int32 copy (bilinear tables whose coefficients, read as
+            // two's-complement int64, all fit int32): half the bytes per load
+            I.poly32_base = POLY32_NONE;
+            bool fits = st == 4;
+            for (size_t i = 0; fits && i < plan.poly.size(); i++) {
+                const int64_t v = (int64_t)plan.poly[i];
+                fits = v >= INT32_MIN && v <= INT32_MAX;
+            }
+            if (fits) {
+                I.poly32_base = (uint32_t)poly.size();   // even: 16-byte aligned
+                for (size_t i = 0; i < plan.poly.size(); i += 4) {
+                    uint64_t w[2];
+                    const uint32_t c[4] = {(uint32_t)plan.poly[i], (uint32_t)plan.poly[i + 1],
+                                           (uint32_t)plan.poly[i + 2], (uint32_t)plan.poly[i + 3]};
+                    std::memcpy(w, c, sizeof w);
+                    poly.push_back(w[0]);
+                    poly.push_back(w[1]);
+                }
+            }
         } else {
             I.plan_tx = I.plan_ty = 0xffffffffu;   // never applicable
             I.poly_base = I.poly_stride = 0;
             I.poly_mask = 0;
+            I.poly32_base = POLY32_NONE;
         }
-        I.per_iter_mask = I.pad2 = I.pad3 = 0;
+        I.per_iter_mask = I.pad3 = 0;
         for (uint32_t k = 0; k < S.n_kernels; k++)
             if (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) I.per_iter_mask |= 1u << k;
         for (uint32_t k = 0; k < S.n_kernels; k++) {

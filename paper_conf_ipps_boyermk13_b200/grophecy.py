@@ -509,7 +509,7 @@ def plan_usage_host(skel, nx, ny):
 
 def plan_stats(skel):
     sd = Skeletons([skel])
-    st = (C.c_uint32 * 7)()
+    st = (C.c_uint32 * 9)()
     rc = _L.grophecy_plan_stats(sd.arr, st)
     return rc, list(st)
 
