@@ -165,6 +165,8 @@ struct grophecy_space {
     unsigned long long *invalid_counter;
     uint32_t max_partials;
     int grid_best, grid_eval;            // persistent grid sizes
+    uint32_t max_kernels;                // largest kernel count of the space's skeletons
+    int occ_canon;                       // pass-1 CTAs per SM (0 = not yet queried)
     // group_best scratch (grown on demand)
     void *gscratch;
     size_t gscratch_bytes;

@@ -847,19 +847,23 @@ struct WarpSmem {
 // ... and of the canonical kernel.  Per group g (= lane of phase A/B):
 // work counts at cw[k][g & 1][g >> 1] (a phase-C lane of half h reads its
 // groups h, h + 2, ... as consecutive words), usage and iterations at [g].
-struct CanonSmem {
+// The work counts follow the struct in the warp's slice, sized by the
+// space's largest kernel count (canon_warp_bytes): shared memory left to L1,
+// which the usage polynomials and the constants live in.
+struct alignas(128) CanonSmem {
     alignas(128) uint32_t rec[4][CTILE];        // the tile's SoA records (TMA bulk copies)
-    alignas(16) uint32_t cw[MAXK][2][16];       // work counts (w_store)
     double th[32], td[32], it[32];              // transfer times, (double) iters
     unsigned long long uh[32], ud[32];          // transfer bytes
     unsigned long long best_h[32], best_d[32];
     unsigned long long mbar;                    // completion of the rec copies
 };
+constexpr uint32_t CW_BYTES_PER_KERNEL = 2 * 16 * sizeof(uint32_t);   // cw[k][2][16] (w_store)
+__host__ __device__ constexpr uint32_t canon_warp_bytes(uint32_t kmax)
+{
+    return (uint32_t)((sizeof(CanonSmem) + kmax * CW_BYTES_PER_KERNEL + 127) / 128 * 128);
+}
 struct CtaSmem {
     WarpSmem w[WARPS];
-};
-struct CanonCtaSmem {
-    CanonSmem w[WARPS];
 };
 
 // Saturated-grid kernel time (DESIGN.md §3 N5, saturated reduction) of one
@@ -978,6 +982,7 @@ struct Params {
     int aligned;    // record arrays 16-byte aligned -> vector loads
     uint32_t *tile_list;      // pass 1 -> pass 2: tiles left to the general path
     unsigned int *tile_count;
+    uint32_t canon_warp_bytes; // pass 1: shared memory per warp (canon_warp_bytes(kmax))
 };
 
 // Record validity (include/grophecy.h) and its usage key (skeleton, nx, ny).
@@ -1361,7 +1366,8 @@ __device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, 
 //      (the constants of (kernel, xform) are warp-uniform: one broadcast
 //      load serves 32 records), then writes outputs / keeps its argmin.
 template <bool BEST>
-__device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsigned long long tb,
+__device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint32_t *cw,
+                                           unsigned long long tb,
                                            unsigned long long next_tb, int lane, double &best_t,
                                            unsigned long long &best_i, uint32_t &cnt_val)
 {
@@ -1420,7 +1426,7 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
     bool huge = false;
     for (uint32_t k = 0; k < K; k++) {
         const uint32_t w = w_store(aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny));
-        ws.cw[k][lane & 1][lane >> 1] = w;
+        cw[k * 32 + (lane & 1) * 16 + (lane >> 1)] = w;
         huge |= w == W_HUGE;
     }
     if (__any_sync(FULL, huge)) return false;   // (nothing written yet)
@@ -1468,7 +1474,7 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, unsig
             uint32_t w[CG];
 #pragma unroll
             for (int j = 0; j < CG; j += 4) {
-                const uint4 v = *reinterpret_cast<const uint4 *>(&ws.cw[k][h][i0g + j]);
+                const uint4 v = *reinterpret_cast<const uint4 *>(&cw[k * 32 + h * 16 + i0g + j]);
                 w[j] = v.x;
                 w[j + 1] = v.y;
                 w[j + 2] = v.z;
@@ -1631,7 +1637,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    CanonSmem &ws = reinterpret_cast<CanonCtaSmem *>(smem_raw)->w[warp];
+    unsigned char *wbase = smem_raw + (size_t)warp * P.canon_warp_bytes;
+    CanonSmem &ws = *reinterpret_cast<CanonSmem *>(wbase);
+    uint32_t *cw = reinterpret_cast<uint32_t *>(wbase + sizeof(CanonSmem));
     // running argmin kept lean in registers: (t, index) + counters; the
     // winner's byte counts go to shared memory (rarely updated)
     double best_t = __longlong_as_double(0x7ff0000000000000LL);
@@ -1657,7 +1665,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
         if (full(tile)) {
             mbar_wait(&ws.mbar, phase);
             phase ^= 1u;
-            done = canon_tile<BEST>(P, ws, tb, next_tb, lane, best_t, best_i, cnt_val);
+            done = canon_tile<BEST>(P, ws, cw, tb, next_tb, lane, best_t, best_i, cnt_val);
         } else if (lane == 0 && next_tb != ~0ull) {
             issue_tile_copy(P, ws, next_tb);   // the buffer is idle during this tile
         }
@@ -1710,7 +1718,7 @@ static void set_smem_attrs()
     cudaGetDevice(&dev);
     bool &done = done_dev[dev & 63];
     if (done) return;
-    const int sm = (int)sizeof(CtaSmem), cs = (int)sizeof(CanonCtaSmem);
+    const int sm = (int)sizeof(CtaSmem), cs = (int)(WARPS * canon_warp_bytes(MAXK));
     cudaFuncSetAttribute(canon_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
     cudaFuncSetAttribute(canon_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
     cudaFuncSetAttribute(general_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
@@ -1720,19 +1728,28 @@ static void set_smem_attrs()
 
 static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_cap, bool canon)
 {
-    static int occ[2] = {0, 0};
+    static int occ_general = 0;
     set_smem_attrs();
-    if (!occ[canon]) {
-        if (canon)
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[1], canon_kernel<true>, THREADS,
-                                                          sizeof(CanonCtaSmem));
-        else
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[0], general_kernel<true>, THREADS,
+    int occ = 0;
+    if (canon) {
+        // per space: its dynamic shared memory depends on its kernel count
+        if (!s->occ_canon) {
+            int o = 0;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, canon_kernel<true>, THREADS,
+                                                          WARPS * canon_warp_bytes(s->max_kernels));
+            const_cast<grophecy_space *>(s)->occ_canon = o < 1 ? 1 : o;
+        }
+        occ = s->occ_canon;
+    } else {
+        if (!occ_general) {
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_general, general_kernel<true>, THREADS,
                                                           sizeof(CtaSmem));
-        if (occ[canon] < 1) occ[canon] = 1;
+            if (occ_general < 1) occ_general = 1;
+        }
+        occ = occ_general;
     }
     const unsigned long long want = (n + (unsigned long long)CTILE * WARPS - 1) / ((unsigned long long)CTILE * WARPS);
-    unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ[canon], per_sm_cap);
+    unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ, per_sm_cap);
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
 }
@@ -1771,7 +1788,8 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, sizeof(unsigned int), st);
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(tile count)");
         const int grid = grid_for(s, Q.n, 32, false), grid_c = grid_for(s, Q.n, 32, true);
-        canon_kernel<BEST><<<grid_c, THREADS, sizeof(CanonCtaSmem), st>>>(Q);
+        Q.canon_warp_bytes = canon_warp_bytes(s->max_kernels);
+        canon_kernel<BEST><<<grid_c, THREADS, WARPS * Q.canon_warp_bytes, st>>>(Q);
         Q.accumulate = BEST ? 1 : 0;   // pass 2 merges into pass 1's result
         general_kernel<BEST><<<grid, THREADS, sizeof(CtaSmem), st>>>(Q);
         count_launch(2);
@@ -1817,6 +1835,7 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
     P.accumulate = 0;
     P.tile_list = s->tile_list;
     P.tile_count = s->tile_count;
+    P.canon_warp_bytes = canon_warp_bytes(s->max_kernels);
     const uintptr_t m = (uintptr_t)b->skx | (uintptr_t)b->nx | (uintptr_t)b->ny | (uintptr_t)b->iters;
     P.aligned = (m & 15u) == 0;
     return P;

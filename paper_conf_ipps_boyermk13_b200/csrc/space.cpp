@@ -580,6 +580,10 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     if ((e = cudaMemcpy(sp->dev_copy, &D, sizeof D, cudaMemcpyHostToDevice)) != cudaSuccess)
         return bail(e, "cudaMemcpy(space header)");
     sp->grid_best = nsm;
+    sp->max_kernels = 1;
+    for (uint32_t q = 0; q < n_skels; q++)
+        sp->max_kernels = std::max(sp->max_kernels, skels[q].n_kernels);
+    sp->occ_canon = 0;
     sp->grid_eval = nsm;
     cudaSetDevice(prev);
     *out = sp;
