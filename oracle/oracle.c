@@ -91,6 +91,18 @@ static void region_box(const or_region *g, int64_t R, int64_t C, int64_t nx, int
     *c1 = imin64(imax64(oracle_affine8(&g->c1, nx, ny), 0), C);
 }
 
+/* The region's plane range (rank-3 arrays, N4r), clamped to [0, P). */
+static void region_pbox(const or_region *g, int64_t P, int64_t nx, int64_t ny, int64_t *p0,
+                        int64_t *p1)
+{
+    if (g->whole) {
+        *p0 = 0; *p1 = P;
+        return;
+    }
+    *p0 = imin64(imax64(oracle_affine8(&g->p0, nx, ny), 0), P);
+    *p1 = imin64(imax64(oracle_affine8(&g->p1, nx, ny), 0), P);
+}
+
 /* Strides of a region (whole regions are dense). */
 static int64_t row_step(const or_region *g) { return (!g->whole && g->r_step > 1) ? g->r_step : 1; }
 static int64_t col_step(const or_region *g) { return (!g->whole && g->c_step > 1) ? g->c_step : 1; }
@@ -171,30 +183,39 @@ void oracle_usage(const or_skeleton *s, int64_t nx, int64_t ny,
     int nreg = (int)s->n_regions;
     int64_t *rb = (int64_t *)malloc(sizeof(int64_t) * (size_t)(2 * nreg + 2));
     int64_t *cb = (int64_t *)malloc(sizeof(int64_t) * (size_t)(2 * nreg + 2));
-    int64_t *box = (int64_t *)malloc(sizeof(int64_t) * (size_t)(6 * nreg + 6));
+    int64_t *pb = (int64_t *)malloc(sizeof(int64_t) * (size_t)(2 * nreg + 2));
+    int64_t *box = (int64_t *)malloc(sizeof(int64_t) * (size_t)(8 * nreg + 8));
     for (uint32_t a = 0; a < s->n_arrays; a++) {
         const or_array *A = &s->arrays[a];
         int64_t R = imax64(0, oracle_affine8(&A->rows, nx, ny));
         int64_t C = imax64(0, oracle_affine8(&A->cols, nx, ny));
-        int nr = 0, nc = 0;
+        int64_t Pl = imax64(0, oracle_affine8(&A->planes, nx, ny));
+        int nr = 0, nc = 0, np = 0;
         int64_t Lr = 1, Lc = 1;
         rb[nr++] = 0; rb[nr++] = R;
         cb[nc++] = 0; cb[nc++] = C;
+        pb[np++] = 0; pb[np++] = Pl;
         for (int j = 0; j < nreg; j++) {
             const or_region *g = &s->regions[j];
             if (g->array != a) continue;
-            int64_t *b = &box[6 * j];
+            int64_t *b = &box[8 * j];
             region_box(g, R, C, nx, ny, &b[0], &b[1], &b[2], &b[3]);
             b[4] = row_anchor(g, nx, ny);
             b[5] = col_anchor(g, nx, ny);
+            region_pbox(g, Pl, nx, ny, &b[6], &b[7]);
             rb[nr++] = b[0]; rb[nr++] = b[1];
             cb[nc++] = b[2]; cb[nc++] = b[3];
+            pb[np++] = b[6]; pb[np++] = b[7];
             Lr = Lr / gcd64(Lr, row_step(g)) * row_step(g);
             Lc = Lc / gcd64(Lc, col_step(g)) * col_step(g);
         }
         nr = sort_unique(rb, nr);
         nc = sort_unique(cb, nc);
+        np = sort_unique(pb, np);
         uint64_t h = 0, d = 0;
+        /* rank-3: the plane breakpoints cut the planes into slabs as well */
+        for (int k = 0; k + 1 < np; k++) {
+        int64_t z0 = pb[k], z1 = pb[k + 1];
         for (int i = 0; i + 1 < nr; i++)
             for (int64_t rho = 0; rho < Lr; rho++) {
                 int64_t y0 = rb[i], y1 = rb[i + 1];
@@ -209,8 +230,9 @@ void oracle_usage(const or_skeleton *s, int64_t nx, int64_t ny,
                         for (int j = 0; j < nreg; j++) {
                             const or_region *g = &s->regions[j];
                             if (g->array != a) continue;
-                            const int64_t *b = &box[6 * j];
-                            if (b[0] <= y0 && y1 <= b[1] && b[2] <= x0 && x1 <= b[3] &&
+                            const int64_t *b = &box[8 * j];
+                            if (b[6] <= z0 && z1 <= b[7] &&
+                                b[0] <= y0 && y1 <= b[1] && b[2] <= x0 && x1 <= b[3] &&
                                 pmod(rho - b[4], row_step(g)) == 0 &&
                                 pmod(sig - b[5], col_step(g)) == 0) {
                                 uint32_t m = eff_mode(g);
@@ -218,15 +240,16 @@ void oracle_usage(const or_skeleton *s, int64_t nx, int64_t ny,
                                 if ((m & 2u) && (int)g->kernel < fw) fw = (int)g->kernel;
                             }
                         }
-                        uint64_t area = (uint64_t)hgt * (uint64_t)wid;
+                        uint64_t area = (uint64_t)(z1 - z0) * (uint64_t)hgt * (uint64_t)wid;
                         if (fr != OR_INF_K && fr <= fw) h += area;
                         if (fw != OR_INF_K) d += area;
                     }
             }
+        }
         h2d_per_array[a] = h * A->elem_bytes;
         d2h_per_array[a] = A->liveout ? d * A->elem_bytes : 0;
     }
-    free(rb); free(cb); free(box);
+    free(rb); free(cb); free(pb); free(box);
 }
 
 /* The literal per-element definition (test-only; R*C <= 2^20 per array). */
@@ -237,17 +260,20 @@ int oracle_bitmap_usage(const or_skeleton *s, int64_t nx, int64_t ny,
         const or_array *A = &s->arrays[a];
         int64_t R = imax64(0, oracle_affine8(&A->rows, nx, ny));
         int64_t C = imax64(0, oracle_affine8(&A->cols, nx, ny));
-        if (R * C > (1 << 20)) return -1;
+        int64_t Pl = imax64(0, oracle_affine8(&A->planes, nx, ny));
+        if (R * C * Pl > (1 << 20)) return -1;
         uint64_t h = 0, d = 0;
+        for (int64_t p = 0; p < Pl; p++)
         for (int64_t r = 0; r < R; r++) {
             for (int64_t c = 0; c < C; c++) {
                 int fr = OR_INF_K, fw = OR_INF_K;
                 for (uint32_t j = 0; j < s->n_regions; j++) {
                     const or_region *g = &s->regions[j];
                     if (g->array != a) continue;
-                    int64_t r0, r1, c0, c1;
+                    int64_t r0, r1, c0, c1, p0, p1;
                     region_box(g, R, C, nx, ny, &r0, &r1, &c0, &c1);
-                    if (r0 <= r && r < r1 && c0 <= c && c < c1 &&
+                    region_pbox(g, Pl, nx, ny, &p0, &p1);
+                    if (p0 <= p && p < p1 && r0 <= r && r < r1 && c0 <= c && c < c1 &&
                         pmod(r - row_anchor(g, nx, ny), row_step(g)) == 0 &&
                         pmod(c - col_anchor(g, nx, ny), col_step(g)) == 0) {
                         uint32_t m = eff_mode(g);
@@ -272,8 +298,8 @@ int oracle_bitmap_usage(const or_skeleton *s, int64_t nx, int64_t ny,
 
 /* One dimension of a section: {l, l+s, ..., u}; s == 0 iff l == u; empty iff l > u. */
 typedef struct { int64_t l, u, s; } or_sec1;
-/* A 2-D section (rows x columns); empty iff either dimension is. */
-typedef struct { or_sec1 r, c; } or_sec;
+/* A section (planes x rows x columns); empty iff any dimension is. */
+typedef struct { or_sec1 r, c, p; } or_sec;
 
 static int sec1_empty(or_sec1 a) { return a.l > a.u; }
 
@@ -317,13 +343,13 @@ static uint64_t sec1_count(or_sec1 a)
     return a.s == 0 ? 1 : (uint64_t)((a.u - a.l) / a.s) + 1;
 }
 
-static int sec_empty(or_sec x) { return sec1_empty(x.r) || sec1_empty(x.c); }
+static int sec_empty(or_sec x) { return sec1_empty(x.r) || sec1_empty(x.c) || sec1_empty(x.p); }
 
 static or_sec sec_union(or_sec a, or_sec b)
 {
     if (sec_empty(a)) return b;
     if (sec_empty(b)) return a;
-    or_sec v = {sec1_union(a.r, b.r), sec1_union(a.c, b.c)};
+    or_sec v = {sec1_union(a.r, b.r), sec1_union(a.c, b.c), sec1_union(a.p, b.p)};
     return v;
 }
 
@@ -331,20 +357,23 @@ static int sec_contains(or_sec w, or_sec x)
 {
     if (sec_empty(x)) return 1;
     if (sec_empty(w)) return 0;
-    return sec1_contains(w.r, x.r) && sec1_contains(w.c, x.c);
+    return sec1_contains(w.r, x.r) && sec1_contains(w.c, x.c) && sec1_contains(w.p, x.p);
 }
 
 static uint64_t sec_count(or_sec a)
 {
-    return sec_empty(a) ? 0 : sec1_count(a.r) * sec1_count(a.c);
+    return sec_empty(a) ? 0 : sec1_count(a.r) * sec1_count(a.c) * sec1_count(a.p);
 }
 
-static or_sec region_sec(const or_region *g, int64_t R, int64_t C, int64_t nx, int64_t ny)
+static or_sec region_sec(const or_region *g, int64_t R, int64_t C, int64_t Pl, int64_t nx,
+                         int64_t ny)
 {
-    int64_t r0, r1, c0, c1;
+    int64_t r0, r1, c0, c1, p0, p1;
     region_box(g, R, C, nx, ny, &r0, &r1, &c0, &c1);
+    region_pbox(g, Pl, nx, ny, &p0, &p1);
     or_sec v = {sec1_make(r0, r1, row_anchor(g, nx, ny), row_step(g)),
-                sec1_make(c0, c1, col_anchor(g, nx, ny), col_step(g))};
+                sec1_make(c0, c1, col_anchor(g, nx, ny), col_step(g)),
+                sec1_make(p0, p1, p0, 1)};
     return v;
 }
 
@@ -365,13 +394,14 @@ void oracle_usage_hull(const or_skeleton *s, int64_t nx, int64_t ny,
         const or_array *A = &s->arrays[a];
         int64_t R = imax64(0, oracle_affine8(&A->rows, nx, ny));
         int64_t C = imax64(0, oracle_affine8(&A->cols, nx, ny));
-        or_sec hr = {{1, 0, 0}, {1, 0, 0}}, hw = {{1, 0, 0}, {1, 0, 0}};
+        int64_t Pl = imax64(0, oracle_affine8(&A->planes, nx, ny));
+        or_sec hr = {{1, 0, 0}, {1, 0, 0}, {1, 0, 0}}, hw = {{1, 0, 0}, {1, 0, 0}, {1, 0, 0}};
         int nw = 0;                                   /* writes of kernels < k */
         for (uint32_t k = 0; k < s->n_kernels; k++) {
             for (uint32_t j = 0; j < s->n_regions; j++) {   /* reads of kernel k */
                 const or_region *g = &s->regions[j];
                 if (g->array != a || g->kernel != k || !(eff_mode(g) & 1u)) continue;
-                or_sec x = region_sec(g, R, C, nx, ny);
+                or_sec x = region_sec(g, R, C, Pl, nx, ny);
                 if (sec_empty(x)) continue;
                 int written = 0;
                 for (int q = 0; q < nw; q++)
@@ -381,7 +411,7 @@ void oracle_usage_hull(const or_skeleton *s, int64_t nx, int64_t ny,
             for (uint32_t j = 0; j < s->n_regions; j++) {   /* then its writes */
                 const or_region *g = &s->regions[j];
                 if (g->array != a || g->kernel != k || !(eff_mode(g) & 2u)) continue;
-                or_sec x = region_sec(g, R, C, nx, ny);
+                or_sec x = region_sec(g, R, C, Pl, nx, ny);
                 if (sec_empty(x)) continue;
                 wl[nw++] = x;
                 hw = sec_union(hw, x);

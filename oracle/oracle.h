@@ -40,7 +40,9 @@ extern "C" {
 
 typedef struct { int32_t c0, c1, c2, c3; } or_affine8;   /* c0 + floor((c1 nx + c2 ny + c3 nx ny)/8) */
 
-typedef struct { or_affine8 rows, cols; uint32_t elem_bytes, liveout; } or_array;
+/* planes: extent of a leading third dimension (rank-3 arrays, SURVEY §8(f)
+ * NEXT-3; N4r); 1 for the 2-D arrays of the paper's workloads. */
+typedef struct { or_affine8 rows, cols; uint32_t elem_bytes, liveout; or_affine8 planes; } or_array;
 /* mode: bit0 = read, bit1 = write.  whole != 0: irregular access, the whole
  * array may be referenced; an irregular write is a "may-write" and
  * counts as read + write of the whole array (reading 10).
@@ -51,6 +53,7 @@ typedef struct {
     uint32_t kernel, array, mode, whole;
     or_affine8 r0, r1, c0, c1;
     uint32_t r_step, c_step;
+    or_affine8 p0, p1;             /* planes [p0, p1) (dense); whole: all planes */
 } or_region;
 typedef struct { or_affine8 work; uint32_t per_iter; } or_kernel;
 typedef struct {

@@ -32,13 +32,14 @@ class Affine8(C.Structure):
 
 class Array(C.Structure):
     _fields_ = [("rows", Affine8), ("cols", Affine8), ("elem_bytes", C.c_uint32),
-                ("liveout", C.c_uint32)]
+                ("liveout", C.c_uint32), ("planes", Affine8)]
 
 
 class Region(C.Structure):
     _fields_ = [("kernel", C.c_uint32), ("array", C.c_uint32), ("mode", C.c_uint32),
                 ("whole", C.c_uint32), ("r0", Affine8), ("r1", Affine8), ("c0", Affine8),
-                ("c1", Affine8), ("r_step", C.c_uint32), ("c_step", C.c_uint32)]
+                ("c1", Affine8), ("r_step", C.c_uint32), ("c_step", C.c_uint32),
+                ("p0", Affine8), ("p1", Affine8)]
 
 
 class Kernel(C.Structure):
@@ -148,12 +149,16 @@ class SkeletonSet:
             ks = (Kernel * len(s["kernels"]))(*[Kernel(_a8(k["work"]), int(k["per_iter"]))
                                                for k in s["kernels"]])
             ars = (Array * len(s["arrays"]))(*[Array(_a8(a["rows"]), _a8(a["cols"]),
-                                                     a["elem_bytes"], int(a["liveout"]))
+                                                     a["elem_bytes"], int(a["liveout"]),
+                                                     _a8(a.get("planes", (1, 0, 0, 0))))
                                                for a in s["arrays"]])
+            # planes of a region: [p0, p1), default every plane of its array
             rs = (Region * max(1, len(s["regions"])))(*[
                 Region(r["kernel"], r["array"], _MODES[r["mode"]], int(r["whole"]),
                        _a8(r["r0"]), _a8(r["r1"]), _a8(r["c0"]), _a8(r["c1"]),
-                       int(r.get("r_step", 1)), int(r.get("c_step", 1)))
+                       int(r.get("r_step", 1)), int(r.get("c_step", 1)),
+                       _a8(r.get("p0", (0, 0, 0, 0))),
+                       _a8(r.get("p1", s["arrays"][r["array"]].get("planes", (1, 0, 0, 0)))))
                 for r in s["regions"]])
             flat = [c for row in s["kx"] for c in row]
             kx = (KX * len(flat))(*[KX(c["tpb"], c["ipt"], c["regs"], c["smem"], c["total"],

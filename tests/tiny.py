@@ -16,9 +16,11 @@ def _a8_const(v):
 
 
 def random_tiny_skeleton(rng, n_xforms=1, max_kernels=8, max_arrays=3, max_regions=12,
-                         strided=False, maywrite=False, hull=False):
+                         strided=False, maywrite=False, hull=False, rank3=False):
     """strided: BRS strides in {1, 2, 3, 4, 6} per dimension (lcm <= 12);
-    maywrite: irregular (WHOLE) writes too; hull: the approximate-UNION mode."""
+    maywrite: irregular (WHOLE) writes too; hull: the approximate-UNION mode;
+    rank3: arrays get 1-5 (possibly size-dependent) planes and regions plane
+    ranges (N4r)."""
     nx = int(rng.integers(1, 13))
     ny = int(rng.integers(1, 13))
     n_arr = int(rng.integers(1, max_arrays + 1))
@@ -35,6 +37,12 @@ def random_tiny_skeleton(rng, n_xforms=1, max_kernels=8, max_arrays=3, max_regio
         arrays.append({"name": "a", "rows": rows, "cols": cols,
                        "elem_bytes": int(rng.choice([1, 4, 8, 16])),
                        "liveout": bool(rng.integers(0, 2))})
+        if rank3:
+            arrays[-1]["planes"] = ((int(rng.integers(1, 6)), 0, 0, 0) if rng.random() < 0.6
+                                    else (int(rng.integers(0, 2)), 2, 0, 0))   # c0 + nx/4
+            if kind == 1:
+                arrays[-1]["rows"] = (1, 0, 0, 0)
+                arrays[-1]["cols"] = (int(rng.integers(0, 3)), 8, 0, 0)   # keep P*R*C small
     K = int(rng.integers(1, max_kernels + 1))
     kernels = [{"name": f"k{k}", "work": (0, 0, 0, 8), "per_iter": True} for k in range(K)]
     regions = []
@@ -56,6 +64,9 @@ def random_tiny_skeleton(rng, n_xforms=1, max_kernels=8, max_arrays=3, max_regio
         if strided:
             reg["r_step"] = int(rng.choice([1, 1, 2, 3, 4, 6]))
             reg["c_step"] = int(rng.choice([1, 1, 2, 3, 4, 6]))
+        if rank3 and rng.random() < 0.7:
+            reg["p0"] = (int(rng.integers(-1, 4)), int(rng.integers(0, 3)) if rng.random() < 0.3 else 0, 0, 0)
+            reg["p1"] = (int(rng.integers(0, 6)), int(rng.integers(0, 3)) if rng.random() < 0.3 else 0, 0, 0)
         regions.append(reg)
     kx = [[DUMMY_KX] * K] * n_xforms
     sk = {"name": "tiny", "arrays": arrays, "kernels": kernels, "regions": regions, "kx": kx}
