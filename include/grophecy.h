@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define GROPHECY_ABI_VERSION 2
+#define GROPHECY_ABI_VERSION 3
 
 typedef enum {
     GROPHECY_OK = 0,
@@ -87,8 +87,15 @@ enum { GROPHECY_REGION_WHOLE = 1u };    /* irregular access: the whole array may
                                            + write (reading 10) */
 enum { GROPHECY_KERNEL_PER_ITER = 1u }; /* runs every iteration; else once */
 
-/* A 2-D array of rows x cols elements (row-major), extents clamped at 0. */
-typedef struct { grophecy_affine8 rows, cols; uint32_t elem_bytes, flags; } grophecy_array_desc;
+/* An array of planes x rows x cols elements (row-major), extents clamped at
+ * 0.  planes = {1, 0, 0, 0} for the 2-D arrays of the paper's workloads;
+ * rank-3 arrays (N4r) have any other planes
+ * expression.  56 bytes. */
+typedef struct {
+    grophecy_affine8 rows, cols;
+    uint32_t elem_bytes, flags;
+    grophecy_affine8 planes;
+} grophecy_array_desc;
 
 /* A bounded regular section (Havlak-Kennedy [5]) of `array` accessed
  * by `kernel` (program order index): rows r0, r0 + r_step, ... and columns
@@ -96,12 +103,14 @@ typedef struct { grophecy_affine8 rows, cols; uint32_t elem_bytes, flags; } grop
  * array (the lattice stays anchored at the unclamped r0 / c0; lo >= hi is
  * empty).  r_step / c_step: 0 or 1 = dense, else <= GROPHECY_MAX_STEP and the
  * least common multiple of one array's row (column) steps must be
- * <= GROPHECY_MAX_STEP_LCM.  WHOLE regions ignore the box and the steps.
- * 72 bytes. */
+ * <= GROPHECY_MAX_STEP_LCM.  Planes [p0, p1) (dense, clamped to the array's
+ * planes; 2-D arrays: {0,0,0,0} and {1,0,0,0}).  WHOLE regions ignore the box,
+ * the planes and the steps.  104 bytes. */
 typedef struct {
     uint8_t kernel, array, mode, flags;
     grophecy_affine8 r0, r1, c0, c1;
     uint16_t r_step, c_step;
+    grophecy_affine8 p0, p1;
 } grophecy_region_desc;
 
 typedef struct { grophecy_affine8 work_items; uint32_t flags; } grophecy_kernel_desc;

@@ -135,6 +135,12 @@ def lib():
 _MODES = {"R": 1, "W": 2, "RW": 3}
 
 
+def _planes_of(skel, a):
+    """The planes expression of array a (a region's default upper plane)."""
+    arrs = skel["arrays"]
+    return arrs[a].get("planes", (1, 0, 0, 0)) if 0 <= a < len(arrs) else (1, 0, 0, 0)
+
+
 def _a8(t):
     return Affine8(*[int(v) for v in t])
 
@@ -158,7 +164,7 @@ class SkeletonSet:
                        _a8(r["r0"]), _a8(r["r1"]), _a8(r["c0"]), _a8(r["c1"]),
                        int(r.get("r_step", 1)), int(r.get("c_step", 1)),
                        _a8(r.get("p0", (0, 0, 0, 0))),
-                       _a8(r.get("p1", s["arrays"][r["array"]].get("planes", (1, 0, 0, 0)))))
+                       _a8(r.get("p1", _planes_of(s, r["array"]))))
                 for r in s["regions"]])
             flat = [c for row in s["kx"] for c in row]
             kx = (KX * len(flat))(*[KX(c["tpb"], c["ipt"], c["regs"], c["smem"], c["total"],

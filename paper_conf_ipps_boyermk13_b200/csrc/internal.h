@@ -71,12 +71,15 @@ struct ArrayDev {
     int4 rows, cols;
     uint32_t elem_bytes, liveout, r_base, r_count;   // regions [r_base, r_base+r_count)
     uint32_t lr, lc;    // lcm of the regions' row / column steps (1 = dense array)
-    uint32_t pad0, pad1;
+    uint32_t rank3;     // planes != 1 or a region's plane range != [0, 1) (N4r)
+    uint32_t pad1;
+    int4 planes;
 };
 enum : uint32_t {
     SKF_STRIDED = 1u << 16,     // some region has a step > 1
     SKF_TABULATED = 1u << 17,   // every (kernel, xform) off the saturated path is in the
                                 // small-grid table or infeasible (canonical kernel eligible)
+    SKF_RANK3 = 1u << 18,       // some array is rank-3 (no usage plan: general sweep)
 };
 
 constexpr uint32_t PLAN_MAX_EXPR = 128;   // < 256: programs pack u8 indices
@@ -122,6 +125,7 @@ struct RegionDev {
     int4 r0, r1, c0, c1;
     uint32_t mode, whole, upto, kernel;
     uint32_t rs, cs, pad0, pad1;
+    int4 p0, p1;        // plane range (rank-3 arrays)
 };
 
 struct SpaceDev {
@@ -178,6 +182,23 @@ struct grophecy_space {
 };
 
 namespace grophecy {
+// The affine value is the constant v (c1 = c2 = c3 = 0).
+inline bool affine_is(const grophecy_affine8 &a, int32_t v)
+{
+    return a.c0 == v && a.c1 == 0 && a.c2 == 0 && a.c3 == 0;
+}
+// Some array of the skeleton is rank-3 (N4r): planes != 1, or a
+// (non-whole) region's plane range is not [0, 1).
+inline bool skeleton_rank3(const grophecy_skeleton_desc &S)
+{
+    for (uint32_t a = 0; a < S.n_arrays; a++)
+        if (!affine_is(S.arrays[a].planes, 1)) return true;
+    for (uint32_t j = 0; j < S.n_regions; j++)
+        if (!(S.regions[j].flags & GROPHECY_REGION_WHOLE) &&
+            !(affine_is(S.regions[j].p0, 0) && affine_is(S.regions[j].p1, 1)))
+            return true;
+    return false;
+}
 // Makes the space's device current for one ABI call (and restores the
 // caller's): launches, streams and the per-device kernel attributes match.
 struct DeviceGuard {

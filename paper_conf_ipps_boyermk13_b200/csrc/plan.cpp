@@ -282,8 +282,10 @@ void compile_polys(const grophecy_skeleton_desc &S, const std::vector<Ex> &table
 bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out)
 {
     out = SkelPlanHost();
-    // the approximate (hull) mode and strided sections take the general path
+    // the approximate (hull) mode, strided sections and rank-3 arrays take
+    // the general path
     if (S.flags & GROPHECY_SKEL_HULL) return false;
+    if (skeleton_rank3(S)) return false;
     for (uint32_t j = 0; j < S.n_regions; j++)
         if (!(S.regions[j].flags & GROPHECY_REGION_WHOLE) &&
             (S.regions[j].r_step > 1 || S.regions[j].c_step > 1))

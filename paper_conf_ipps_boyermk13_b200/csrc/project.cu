@@ -240,6 +240,28 @@ __device__ __forceinline__ unsigned long long count_residue(long long a, long lo
     return first < b ? (unsigned long long)((b - 1 - first) / L) + 1ull : 0ull;
 }
 
+// Rank-3 arrays (N4r): the planes [0, P) are cut into slabs at
+// every region's plane bounds; f(pm, depth) is called per slab with the mask
+// of the (valid) regions covering it.  2-D arrays: one slab [0, 1).
+template <class F>
+__device__ __forceinline__ void plane_slabs(bool valid, long long p0, long long p1, long long P, F &&f)
+{
+    long long z = 0;
+    while (z < P) {
+        long long c = P;
+        if (valid && p0 > z && p0 < c) c = p0;
+        if (valid && p1 > z && p1 < c) c = p1;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const long long t = __shfl_xor_sync(FULL, c, o);
+            c = t < c ? t : c;
+        }
+        const unsigned pm = __ballot_sync(FULL, valid && p0 <= z && c <= p1);
+        if (pm) f(pm, (unsigned long long)(c - z));
+        z = c;
+    }
+}
+
 // Strided arrays (BRS [l:u:s]): the slabs of the sweep
 // are split by row residue rho mod Lr and column residue sigma mod Lc (Lr, Lc
 // = lcm of the array's steps); a region covers a (slab, residue) unit iff it
@@ -247,7 +269,8 @@ __device__ __forceinline__ unsigned long long count_residue(long long a, long lo
 // The first-reader / first-writer rule per cell is the dense sweep's.
 __device__ __forceinline__ void strided_cells(SweepScratch &ws, unsigned Lr, unsigned Lc, int Sr, int Sc, int n,
                               long long ar, long long ac, unsigned rs, unsigned cs, unsigned Rm,
-                              unsigned Wm, int lane, unsigned long long &h, unsigned long long &d)
+                              unsigned Wm, int lane, unsigned long long &h, unsigned long long &d,
+                              bool valid, long long pl0, long long pl1, long long P)
 {
     // residue masks: lanes over residues, regions' phases by shuffle
     const unsigned pr = (unsigned)pmodll(ar, rs), pcp = (unsigned)pmodll(ac, cs);
@@ -327,19 +350,28 @@ __device__ __forceinline__ void strided_cells(SweepScratch &ws, unsigned Lr, uns
         if (kc1) { const int q = __popcll(occ_c & (below << 32 | 0xffffffffull)); ws.cs_m[q] = kc1; ws.cs_w[q] = (long long)sc1; }
         __syncwarp();
         const int nr = __popcll(occ_r), nc = __popcll(occ_c);
-        for (int p = lane; p < nr * nc; p += 32) {
-            const int i = p / nc, j = p - i * nc;
-            const unsigned m = ws.rs_m[i] & ws.cs_m[j];
-            if (m) {
-                const unsigned long long area =
-                    (unsigned long long)ws.rs_h[i] * (unsigned long long)ws.cs_w[j];
-                const unsigned mr = m & Rm, mw = m & Wm;
-                if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) h += area;
-                if (mw) d += area;
+        plane_slabs(valid, pl0, pl1, P, [&](unsigned pm, unsigned long long depth) {
+            const unsigned Rp = Rm & pm, Wp = Wm & pm;
+            unsigned long long hs = 0, ds = 0;
+            for (int p = lane; p < nr * nc; p += 32) {
+                const int i = p / nc, j = p - i * nc;
+                const unsigned m = ws.rs_m[i] & ws.cs_m[j];
+                if (m) {
+                    const unsigned long long area =
+                        (unsigned long long)ws.rs_h[i] * (unsigned long long)ws.cs_w[j];
+                    const unsigned mr = m & Rp, mw = m & Wp;
+                    if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) hs += area;
+                    if (mw) ds += area;
+                }
             }
-        }
+            h += depth * hs;
+            d += depth * ds;
+        });
         return;
     }
+    plane_slabs(valid, pl0, pl1, P, [&](unsigned pm, unsigned long long depth) {
+    const unsigned Rp = Rm & pm, Wp = Wm & pm;
+    unsigned long long hs = 0, ds = 0;
     for (int i = 0; i < Sr; i++) {
         const unsigned sm = ws.rs_m[i];
         if (!sm) continue;
@@ -356,13 +388,16 @@ __device__ __forceinline__ void strided_cells(SweepScratch &ws, unsigned Lr, uns
                 if (m) {
                     const unsigned long long area =
                         hg * count_residue(ws.cs_a[j], ws.cs_w[j], sig, Lc);
-                    const unsigned mr = m & Rm, mw = m & Wm;
-                    if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) h += area;
-                    if (mw) d += area;
+                    const unsigned mr = m & Rp, mw = m & Wp;
+                    if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) hs += area;
+                    if (mw) ds += area;
                 }
             }
         }
     }
+    h += depth * hs;
+    d += depth * ds;
+    });
 }
 
 // Data usage of one (skeleton, nx, ny) key by the general coordinate-compressed
@@ -381,10 +416,15 @@ __device__ __forceinline__ Usage warp_usage_sweep(const SpaceDev &S, const SkelI
         long long C = aff8(A.cols, nx, ny);
         R = R > 0 ? R : 0;
         C = C > 0 ? C : 0;
+        long long P = 1;                       // planes (rank-3 arrays, N4r)
+        if (A.rank3) {
+            P = aff8(A.planes, nx, ny);
+            P = P > 0 ? P : 0;
+        }
         const int n = (int)A.r_count;
         unsigned long long h = 0, d = 0;
-        if (n > 0 && R > 0 && C > 0) {
-            long long r0 = 0, r1 = 0, c0 = 0, c1 = 0;
+        if (n > 0 && R > 0 && C > 0 && P > 0) {
+            long long r0 = 0, r1 = 0, c0 = 0, c1 = 0, p0 = 0, p1 = 0;
             long long ar = 0, ac = 0;          // lattice anchors (unclamped lower bounds)
             bool valid = false;
             unsigned mode = 0, up = 0, rs = 1, cs = 1;
@@ -393,6 +433,7 @@ __device__ __forceinline__ Usage warp_usage_sweep(const SpaceDev &S, const SkelI
                 if (g.whole) {
                     r1 = R;
                     c1 = C;
+                    p1 = P;
                 } else {
                     ar = aff8(g.r0, nx, ny);
                     ac = aff8(g.c0, nx, ny);
@@ -400,8 +441,14 @@ __device__ __forceinline__ Usage warp_usage_sweep(const SpaceDev &S, const SkelI
                     r1 = clampll(aff8(g.r1, nx, ny), R);
                     c0 = clampll(ac, C);
                     c1 = clampll(aff8(g.c1, nx, ny), C);
+                    if (A.rank3) {
+                        p0 = clampll(aff8(g.p0, nx, ny), P);
+                        p1 = clampll(aff8(g.p1, nx, ny), P);
+                    } else {
+                        p1 = 1;
+                    }
                 }
-                valid = r0 < r1 && c0 < c1;
+                valid = r0 < r1 && c0 < c1 && p0 < p1;
                 mode = g.mode;
                 up = g.upto;
                 rs = g.rs;
@@ -413,13 +460,14 @@ __device__ __forceinline__ Usage warp_usage_sweep(const SpaceDev &S, const SkelI
             const unsigned Wm = __ballot_sync(FULL, valid && (mode & GROPHECY_W));
             if (vm) {
                 const bool full = valid && r0 == 0 && r1 == R && c0 == 0 && c1 == C && rs == 1 &&
-                                  cs == 1;
+                                  cs == 1 && p0 == 0 && p1 == P;
                 const unsigned fm = __ballot_sync(FULL, full);
                 if (fm == vm) {
                     // every access covers the whole array: one cell
                     const int fwl = Wm ? __ffs(Wm) - 1 : 0;
                     const unsigned upw = __shfl_sync(FULL, up, fwl);
-                    const unsigned long long area = (unsigned long long)R * (unsigned long long)C;
+                    const unsigned long long area =
+                        (unsigned long long)P * (unsigned long long)R * (unsigned long long)C;
                     if (Rm && (!Wm || (Rm & upw))) h = area;
                     if (Wm) d = area;
                 } else {
@@ -495,22 +543,29 @@ __device__ __forceinline__ Usage warp_usage_sweep(const SpaceDev &S, const SkelI
                     const int Sr = __popc(br0) + __popc(br1);
                     const int Sc = __popc(bc0) + __popc(bc1);
                     if (strided) {
-                        strided_cells(ws, A.lr, A.lc, Sr, Sc, n, ar, ac, rs, cs, Rm, Wm, lane, h, d);
+                        strided_cells(ws, A.lr, A.lc, Sr, Sc, n, ar, ac, rs, cs, Rm, Wm, lane, h, d,
+                                      valid, p0, p1, P);
                     } else
-                    for (int i = 0; i < Sr; i++) {
-                        const unsigned rm = ws.rs_m[i];
-                        if (!rm) continue;
-                        const unsigned long long hg = (unsigned long long)ws.rs_h[i];
-                        for (int j = lane; j < Sc; j += 32) {
-                            const unsigned m = rm & ws.cs_m[j];
-                            if (m) {
-                                const unsigned mr = m & Rm, mw = m & Wm;
-                                const unsigned long long area = hg * (unsigned long long)ws.cs_w[j];
-                                if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) h += area;
-                                if (mw) d += area;
+                    plane_slabs(valid, p0, p1, P, [&](unsigned pm, unsigned long long depth) {
+                        const unsigned Rp = Rm & pm, Wp = Wm & pm;
+                        unsigned long long hs = 0, ds = 0;
+                        for (int i = 0; i < Sr; i++) {
+                            const unsigned rm = ws.rs_m[i] & pm;
+                            if (!rm) continue;
+                            const unsigned long long hg = (unsigned long long)ws.rs_h[i];
+                            for (int j = lane; j < Sc; j += 32) {
+                                const unsigned m = rm & ws.cs_m[j];
+                                if (m) {
+                                    const unsigned mr = m & Rp, mw = m & Wp;
+                                    const unsigned long long area = hg * (unsigned long long)ws.cs_w[j];
+                                    if (mr && (!mw || (mr & ws.upto[__ffs(mw) - 1]))) hs += area;
+                                    if (mw) ds += area;
+                                }
                             }
                         }
-                    }
+                        h += depth * hs;
+                        d += depth * ds;
+                    });
                     h = warp_sum_u64(h);
                     d = warp_sum_u64(d);
                     __syncwarp();
@@ -582,9 +637,14 @@ __device__ __forceinline__ unsigned long long sec1_count(const Sec1 &a)
 
 // One dimension (rows: dim 0, columns: dim 1) of a region's section.
 __device__ __forceinline__ Sec1 region_sec1(const RegionDev &g, int dim, long long nx, long long ny,
-                                            long long E)
+                                            long long E, bool rank3 = false)
 {
     if (g.whole) return sec1_make(0, E, 0, 1);
+    if (dim == 2) {   // planes (rank-3 arrays, N4r): dense [p0, p1); 2-D arrays [0, 1)
+        if (!rank3) return sec1_make(0, E, 0, 1);
+        const long long q0 = clampll(aff8(g.p0, nx, ny), E);
+        return sec1_make(q0, clampll(aff8(g.p1, nx, ny), E), q0, 1);
+    }
     const int4 lo = dim ? g.c0 : g.r0, hi = dim ? g.c1 : g.r1;
     const long long an = aff8(lo, nx, ny);
     return sec1_make(clampll(an, E), clampll(aff8(hi, nx, ny), E), an, dim ? g.cs : g.rs);
@@ -602,16 +662,20 @@ __device__ __forceinline__ Usage warp_usage_hull(const SpaceDev &S, const SkelIn
     unsigned long long h = 0, d = 0;
     if ((uint32_t)lane < I.n_arrays) {
         const ArrayDev &A = S.arrays[I.a_base + lane];
-        long long E[2] = {aff8(A.rows, nx, ny), aff8(A.cols, nx, ny)};
+        long long E[3] = {aff8(A.rows, nx, ny), aff8(A.cols, nx, ny),
+                          A.rank3 ? aff8(A.planes, nx, ny) : 1};
         E[0] = E[0] > 0 ? E[0] : 0;
         E[1] = E[1] > 0 ? E[1] : 0;
+        E[2] = E[2] > 0 ? E[2] : 0;
+        const bool r3 = A.rank3 != 0;
         const RegionDev *G = S.regions + A.r_base;
         const uint32_t n = A.r_count;
         uint32_t nonempty = 0, keep = 0, wmask = 0;
         for (uint32_t j = 0; j < n; j++) {
             const Sec1 xr = region_sec1(G[j], 0, nx, ny, E[0]);
             const Sec1 xc = region_sec1(G[j], 1, nx, ny, E[1]);
-            if (sec1_empty(xr) || sec1_empty(xc)) continue;
+            const Sec1 xp = region_sec1(G[j], 2, nx, ny, E[2], r3);
+            if (sec1_empty(xr) || sec1_empty(xc) || sec1_empty(xp)) continue;
             nonempty |= 1u << j;
             if (G[j].mode & GROPHECY_W) wmask |= 1u << j;
             if (!(G[j].mode & GROPHECY_R)) continue;
@@ -619,16 +683,17 @@ __device__ __forceinline__ Usage warp_usage_hull(const SpaceDev &S, const SkelIn
             for (uint32_t q = 0; q < j && !written; q++) {
                 if (!((wmask >> q) & 1u) || G[q].kernel >= G[j].kernel) continue;
                 written = sec1_contains(region_sec1(G[q], 0, nx, ny, E[0]), xr) &&
-                          sec1_contains(region_sec1(G[q], 1, nx, ny, E[1]), xc);
+                          sec1_contains(region_sec1(G[q], 1, nx, ny, E[1]), xc) &&
+                          sec1_contains(region_sec1(G[q], 2, nx, ny, E[2], r3), xp);
             }
             if (!written) keep |= 1u << j;
         }
         unsigned long long cr = 1, cw = 1;
-        for (int dim = 0; dim < 2; dim++) {
+        for (int dim = 0; dim < 3; dim++) {
             Sec1 hr = {1, 0, 0}, hw = {1, 0, 0};
             for (uint32_t j = 0; j < n; j++) {
                 if (!((nonempty >> j) & 1u)) continue;
-                const Sec1 x = region_sec1(G[j], dim, nx, ny, E[dim]);
+                const Sec1 x = region_sec1(G[j], dim, nx, ny, E[dim], r3);
                 if ((keep >> j) & 1u) hr = sec1_union(hr, x);
                 if ((wmask >> j) & 1u) hw = sec1_union(hw, x);
             }

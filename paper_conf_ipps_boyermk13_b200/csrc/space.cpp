@@ -89,7 +89,8 @@ static int validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             if (!coef_ok(S.kernels[k].work_items))
                 return fail(GROPHECY_ELIMIT, std::string(where) + "work coefficient out of range");
         for (uint32_t a = 0; a < S.n_arrays; a++) {
-            if (!coef_ok(S.arrays[a].rows) || !coef_ok(S.arrays[a].cols))
+            if (!coef_ok(S.arrays[a].rows) || !coef_ok(S.arrays[a].cols) ||
+                !coef_ok(S.arrays[a].planes))
                 return fail(GROPHECY_ELIMIT, std::string(where) + "extent coefficient out of range");
             if (S.arrays[a].elem_bytes < 1)
                 return fail(GROPHECY_EINVAL, std::string(where) + "elem_bytes must be >= 1");
@@ -103,7 +104,8 @@ static int validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 return fail(GROPHECY_EINVAL, std::string(where) + "region mode must be R, W or R|W");
             if (r.r_step > GROPHECY_MAX_STEP || r.c_step > GROPHECY_MAX_STEP)
                 return fail(GROPHECY_ELIMIT, std::string(where) + "region step > 64");
-            if (!coef_ok(r.r0) || !coef_ok(r.r1) || !coef_ok(r.c0) || !coef_ok(r.c1))
+            if (!coef_ok(r.r0) || !coef_ok(r.r1) || !coef_ok(r.c0) || !coef_ok(r.c1) ||
+                !coef_ok(r.p0) || !coef_ok(r.p1))
                 return fail(GROPHECY_ELIMIT, std::string(where) + "region coefficient out of range");
             if (++per_array[r.array] > GROPHECY_MAX_REGIONS_PER_ARRAY)
                 return fail(GROPHECY_ELIMIT, std::string(where) + "more than 32 regions on one array");
@@ -332,6 +334,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             if (!(S.regions[j].flags & GROPHECY_REGION_WHOLE) &&
                 (S.regions[j].r_step > 1 || S.regions[j].c_step > 1))
                 I.flags |= SKF_STRIDED;
+        if (skeleton_rank3(S)) I.flags |= SKF_RANK3;
         SkelPlanHost plan;
         if (compile_plan(S, plan)) {
             I.plan_tx = plan.tx;
@@ -389,7 +392,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             A.liveout = (S.arrays[a].flags & GROPHECY_ARRAY_LIVEOUT) ? 1u : 0u;
             A.r_base = (uint32_t)regions.size();
             A.lr = A.lc = 1;
-            A.pad0 = A.pad1 = 0;
+            A.planes = a4(S.arrays[a].planes);
+            A.rank3 = !affine_is(S.arrays[a].planes, 1);
+            A.pad1 = 0;
             // regions of this array, stably sorted by kernel (order within a
             // kernel is irrelevant: usage does not depend on region order)
             std::vector<const grophecy_region_desc *> rs;
@@ -411,6 +416,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 R.rs = (!R.whole && rs[j]->r_step > 1) ? rs[j]->r_step : 1u;
                 R.cs = (!R.whole && rs[j]->c_step > 1) ? rs[j]->c_step : 1u;
                 R.pad0 = R.pad1 = 0;
+                R.p0 = a4(rs[j]->p0);
+                R.p1 = a4(rs[j]->p1);
+                if (!R.whole && !(affine_is(rs[j]->p0, 0) && affine_is(rs[j]->p1, 1))) A.rank3 = 1;
                 A.lr = (uint32_t)lcm_step(A.lr, R.rs);
                 A.lc = (uint32_t)lcm_step(A.lc, R.cs);
                 R.kernel = rs[j]->kernel;

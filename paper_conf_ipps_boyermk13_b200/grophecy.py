@@ -60,13 +60,14 @@ class Affine8(C.Structure):
 
 class ArrayDesc(C.Structure):
     _fields_ = [("rows", Affine8), ("cols", Affine8), ("elem_bytes", C.c_uint32),
-                ("flags", C.c_uint32)]
+                ("flags", C.c_uint32), ("planes", Affine8)]
 
 
 class RegionDesc(C.Structure):
     _fields_ = [("kernel", C.c_uint8), ("array", C.c_uint8), ("mode", C.c_uint8),
                 ("flags", C.c_uint8), ("r0", Affine8), ("r1", Affine8), ("c0", Affine8),
-                ("c1", Affine8), ("r_step", C.c_uint16), ("c_step", C.c_uint16)]
+                ("c1", Affine8), ("r_step", C.c_uint16), ("c_step", C.c_uint16),
+                ("p0", Affine8), ("p1", Affine8)]
 
 
 class KernelDesc(C.Structure):
@@ -111,7 +112,7 @@ class BestResult(C.Structure):
                 self.n_valid)
 
 
-assert C.sizeof(BestResult) == 48 and C.sizeof(RegionDesc) == 72 and C.sizeof(KxDesc) == 64
+assert C.sizeof(BestResult) == 48 and C.sizeof(RegionDesc) == 104 and C.sizeof(ArrayDesc) == 56 and C.sizeof(KxDesc) == 64
 assert C.sizeof(SkeletonDesc) == 56
 
 
@@ -216,6 +217,12 @@ def pcie(h2d, d2h=None):
 _MODES = {"R": R, "W": W, "RW": R | W}
 
 
+def _planes_of(skel, a):
+    """The planes expression of array a (a region's default upper plane)."""
+    arrs = skel["arrays"]
+    return arrs[a].get("planes", (1, 0, 0, 0)) if 0 <= a < len(arrs) else (1, 0, 0, 0)
+
+
 def _a8(t):
     return Affine8(*[int(v) for v in t])
 
@@ -233,12 +240,16 @@ class Skeletons:
                 for k in s["kernels"]])
             ars = (ArrayDesc * max(1, len(s["arrays"])))(*[
                 ArrayDesc(_a8(a["rows"]), _a8(a["cols"]), a["elem_bytes"],
-                          ARRAY_LIVEOUT if a["liveout"] else 0) for a in s["arrays"]])
+                          ARRAY_LIVEOUT if a["liveout"] else 0,
+                          _a8(a.get("planes", (1, 0, 0, 0)))) for a in s["arrays"]])
+            # planes of a region: [p0, p1), default every plane of its array
             rs = (RegionDesc * max(1, len(s["regions"])))(*[
                 RegionDesc(r["kernel"], r["array"], _MODES[r["mode"]],
                            REGION_WHOLE if r["whole"] else 0, _a8(r["r0"]), _a8(r["r1"]),
                            _a8(r["c0"]), _a8(r["c1"]), int(r.get("r_step", 1)),
-                           int(r.get("c_step", 1))) for r in s["regions"]])
+                           int(r.get("c_step", 1)), _a8(r.get("p0", (0, 0, 0, 0))),
+                           _a8(r.get("p1", _planes_of(s, r["array"]))))
+                for r in s["regions"]])
             flat = [c for row in s["kx"] for c in row]
             kx = (KxDesc * len(flat))(*[
                 KxDesc(c["tpb"], c["ipt"], c["regs"], c["smem"], c["total"], c["coal"],

@@ -39,7 +39,7 @@ def test_every_declared_symbol_is_exported(G):
 
 
 def test_abi_version(G):
-    assert G.lib().grophecy_abi_version() == 2
+    assert G.lib().grophecy_abi_version() == 3
 
 
 def test_fit_pcie_matches_oracle_bitwise(G, O):
@@ -230,3 +230,21 @@ def test_strided_and_hull_skeletons_have_no_plan(G):
         rc, h, d, tx, ty = G.plan_usage_host(dict(s, hull=True), 64, 64)
         assert rc == G.ELIMIT and tx == 0xFFFFFFFF
     assert n_str > 20
+
+
+def test_rank3_skeletons_have_no_plan_and_validate(G):
+    """Rank-3 arrays (N4r) take the general sweep: no usage plan; the space
+    validation accepts them and rejects out-of-range plane coefficients."""
+    from tests.tiny import random_tiny_skeleton, rng
+    r = rng(9900)
+    for _ in range(50):
+        sk, nx, ny = random_tiny_skeleton(r, rank3=True)
+        if not any(a.get("planes", (1, 0, 0, 0)) != (1, 0, 0, 0) for a in sk["arrays"]) and \
+                not any(g.get("p0", (0, 0, 0, 0)) != (0, 0, 0, 0) for g in sk["regions"]):
+            continue
+        rc = G.plan_stats(sk)[0]
+        assert rc == G.ELIMIT
+    sk, _, _ = random_tiny_skeleton(r, rank3=True)
+    sk["arrays"][0]["planes"] = (0, 1 << 16, 0, 0)
+    from synth import skeletons as S
+    assert G.validate([sk], S.FX5600) == G.ELIMIT
