@@ -401,6 +401,21 @@ int grophecy_choose_memory(const grophecy_memory_model *model, uint64_t h2d_byte
                            uint64_t d2h_bytes, uint64_t footprint_bytes,
                            grophecy_memory_choice *out);
 
+/* The batched projection with the per-array memory choice (reading 17):
+ * grophecy_eval_parts / grophecy_best where every array with a transfer is
+ * priced pinned — t_h2d gets A(footprint) + T_pin,h2d, t_d2h gets T_pin,d2h —
+ * or pageable — T_page,h2d / T_page,d2h — whichever grophecy_choose_memory
+ * picks for it (footprint = planes * rows * cols * elem_bytes at the
+ * candidate's size).  Bytes, kernel times and everything else as in
+ * grophecy_eval / grophecy_best; same layouts, ownership and errors (parts
+ * may be NULL).  Runs on the general projection path. */
+int grophecy_eval_mem(const grophecy_space *space, const grophecy_memory_model *model,
+                      const grophecy_batch *batch, uint64_t *h2d_bytes, uint64_t *d2h_bytes,
+                      double *t_total_s, const grophecy_parts *parts, void *cuda_stream);
+int grophecy_best_mem(grophecy_space *space, const grophecy_memory_model *model,
+                      const grophecy_batch *batch, grophecy_best_result *host_out,
+                      void *cuda_stream);
+
 /* ---------------------------------------------------------------------- */
 /* Synthetic workloads (bench / tests) — not part of the method             */
 /* ---------------------------------------------------------------------- */

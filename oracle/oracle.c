@@ -539,6 +539,65 @@ int oracle_eval_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
     return 1;
 }
 
+/* The projection with the per-array memory choice (NEXT-4, DESIGN.md
+ * reading 17): every array with a transfer is priced as pinned (its
+ * allocation A(footprint) + pinned transfers) or pageable, whichever
+ * oracle_choose_memory picks; the pinned H2D term carries the allocation.
+ * footprint = planes * rows * cols * elem_bytes (the whole host buffer). */
+int oracle_eval_mem_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                        const or_link *pin_h2d, const or_link *pin_d2h,
+                        const or_link *page_h2d, const or_link *page_d2h,
+                        const or_link *pin_alloc,
+                        uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters,
+                        uint64_t *h2d, uint64_t *d2h, double *t, double *t_h2d, double *t_d2h)
+{
+    uint32_t skel = skx >> 16, xform = skx & 0xffffu;
+    if (skel >= n_skels || xform >= skels[skel].n_xforms || nx < 1 || nx > (1u << 20) ||
+        ny < 1 || ny > (1u << 20) || iters < 1) {
+        *h2d = 0; *d2h = 0; *t = NAN; *t_h2d = NAN; *t_d2h = NAN;
+        return 0;
+    }
+    const or_skeleton *s = &skels[skel];
+    uint64_t hpa[64], dpa[64];
+    oracle_usage(s, nx, ny, hpa, dpa);
+    double t_iter = 0.0, t_once = 0.0;
+    for (uint32_t k = 0; k < s->n_kernels; k++) {
+        double tk = oracle_kernel_time(s, g, xform, k, nx, ny, NULL);
+        if (s->kernels[k].per_iter) t_iter = t_iter + tk;
+        else t_once = t_once + tk;
+    }
+    double t_kern = t_once + (double)iters * t_iter;
+    double t_h = 0.0, t_d = 0.0;
+    uint64_t H = 0, D = 0;
+    for (uint32_t a = 0; a < s->n_arrays; a++) {
+        const or_array *A = &s->arrays[a];
+        H += hpa[a];
+        D += dpa[a];
+        if (hpa[a] == 0 && dpa[a] == 0) continue;
+        uint64_t P = (uint64_t)imax64(0, oracle_affine8(&A->planes, nx, ny));
+        uint64_t R = (uint64_t)imax64(0, oracle_affine8(&A->rows, nx, ny));
+        uint64_t C = (uint64_t)imax64(0, oracle_affine8(&A->cols, nx, ny));
+        uint64_t F = P * R * C * A->elem_bytes;
+        double tp, tg;
+        int m;
+        oracle_choose_memory(pin_h2d, pin_d2h, page_h2d, page_d2h, pin_alloc, hpa[a], dpa[a], F,
+                             &tp, &tg, &m);
+        if (m == 0) {
+            t_h = t_h + (oracle_pcie_time(pin_alloc, F) + oracle_pcie_time(pin_h2d, hpa[a]));
+            t_d = t_d + oracle_pcie_time(pin_d2h, dpa[a]);
+        } else {
+            t_h = t_h + oracle_pcie_time(page_h2d, hpa[a]);
+            t_d = t_d + oracle_pcie_time(page_d2h, dpa[a]);
+        }
+    }
+    *h2d = H;
+    *d2h = D;
+    *t_h2d = t_h;
+    *t_d2h = t_d;
+    *t = (t_kern + t_h) + t_d;
+    return 1;
+}
+
 /* The same computation, returning the four components. */
 int oracle_eval_parts_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
                           const or_link *h2d_link, const or_link *d2h_link,

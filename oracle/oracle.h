@@ -109,6 +109,15 @@ double oracle_kernel_time(const or_skeleton *s, const or_gpu *g, uint32_t xform,
 /* Components of one candidate's time:
  * t = ((t_once + iters * t_iter) + t_h2d) + t_d2h.  Returns 1 if valid
  * (else all components NaN). */
+/* NEXT-4: one candidate with the per-array pinned / pageable choice
+ * (reading 17); also returns the two transfer components. */
+int oracle_eval_mem_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                        const or_link *pin_h2d, const or_link *pin_d2h,
+                        const or_link *page_h2d, const or_link *page_d2h,
+                        const or_link *pin_alloc,
+                        uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters,
+                        uint64_t *h2d, uint64_t *d2h, double *t, double *t_h2d, double *t_d2h);
+
 int oracle_eval_parts_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
                           const or_link *h2d_link, const or_link *d2h_link,
                           uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters,

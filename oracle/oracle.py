@@ -117,6 +117,11 @@ def lib():
         L.oracle_eval_parts_one.argtypes = [SK, C.c_uint32, C.POINTER(GPU), C.POINTER(Link),
                                             C.POINTER(Link), C.c_uint32, C.c_uint32, C.c_uint32,
                                             C.c_uint32] + [C.POINTER(C.c_double)] * 4
+        LPm = C.POINTER(Link)
+        L.oracle_eval_mem_one.argtypes = [SK, C.c_uint32, C.POINTER(GPU), LPm, LPm, LPm, LPm, LPm,
+                                          C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32,
+                                          C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)] + \
+            [C.POINTER(C.c_double)] * 3
         L.oracle_group_best.argtypes = [SK, C.c_uint32, C.POINTER(GPU), C.POINTER(Link),
                                         C.POINTER(Link), u32p, u32p, u32p, u32p, C.c_uint64,
                                         C.c_uint64, C.c_uint64, u64p, u64p, u64p, f64p]
@@ -257,6 +262,16 @@ class Problem:
         lib().oracle_eval(self.ss.arr, self.ss.n, C.byref(self.gpu), C.byref(self.hl),
                           C.byref(self.dl), *a, n, nthreads, h, d, t)
         return h, d, t
+
+    def eval_mem_one(self, links, skx, nx, ny, iters):
+        """links = (pin_h2d, pin_d2h, page_h2d, page_d2h, pin_alloc) as Link;
+        -> (ok, h2d, d2h, t, t_h2d, t_d2h) with the per-array memory choice."""
+        h, d = C.c_uint64(), C.c_uint64()
+        t, th, td = C.c_double(), C.c_double(), C.c_double()
+        ok = lib().oracle_eval_mem_one(self.ss.arr, self.ss.n, C.byref(self.gpu),
+                                       *[C.byref(x) for x in links], skx, nx, ny, iters,
+                                       C.byref(h), C.byref(d), C.byref(t), C.byref(th), C.byref(td))
+        return bool(ok), h.value, d.value, t.value, th.value, td.value
 
     def eval_parts_one(self, skx, nx, ny, iters):
         v = [C.c_double() for _ in range(4)]

@@ -22,6 +22,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cstring>
 #include <type_traits>
 #include <cmath>
 
@@ -114,17 +115,72 @@ __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v)
     return v;
 }
 
+// How transfers are priced: the pinned links of `pc` (the paper's model), or
+// with mem set the per-array pinned / pageable choice of DESIGN.md reading 17
+// (NEXT-4, grophecy_choose_memory's rule; general path only).
+struct Price {
+    grophecy_pcie pc;
+    grophecy_memory_model mm;
+    int mem;
+};
+
+__device__ __forceinline__ double link_time(const grophecy_link &l, unsigned long long b)
+{
+    return b ? __dadd_rn(l.alpha_s, __dmul_rn(l.beta_s_per_byte, __ull2double_rn(b))) : 0.0;
+}
+
+// Reading 17 for one array with transfer bytes (h, d) and host footprint F:
+// the H2D / D2H terms it adds (the pinned H2D term carries the allocation).
+__device__ __forceinline__ void mem_terms(const grophecy_memory_model &m, unsigned long long h,
+                                          unsigned long long d, unsigned long long F, double &th,
+                                          double &td)
+{
+    th = td = 0.0;
+    if (!h && !d) return;
+    const double a = link_time(m.pin_alloc, F);
+    const double ph = __dadd_rn(a, link_time(m.pinned.h2d, h)), pd = link_time(m.pinned.d2h, d);
+    const double gh = link_time(m.pageable.h2d, h), gd = link_time(m.pageable.d2h, d);
+    if (__dadd_rn(ph, pd) <= __dadd_rn(gh, gd)) {
+        th = ph;
+        td = pd;
+    } else {
+        th = gh;
+        td = gd;
+    }
+}
+
+// Host footprint of an array at (nx, ny): planes * rows * cols * elem_bytes.
+__device__ __forceinline__ unsigned long long footprint(const ArrayDev &A, long long nx, long long ny)
+{
+    long long R = aff8(A.rows, nx, ny), C = aff8(A.cols, nx, ny);
+    long long Pl = A.rank3 ? aff8(A.planes, nx, ny) : 1;
+    R = R > 0 ? R : 0;
+    C = C > 0 ? C : 0;
+    Pl = Pl > 0 ? Pl : 0;
+    return (unsigned long long)Pl * (unsigned long long)R * (unsigned long long)C *
+           (unsigned long long)A.elem_bytes;
+}
+
 // Per-array byte counts -> totals and per-array PCIe times in array order
 // (Eq. (1), one transfer per array).  Warp-uniform.
 __device__ __forceinline__ void add_array(Usage &o, const ArrayDev &A, unsigned long long h,
-                                          unsigned long long d, const grophecy_pcie &pc)
+                                          unsigned long long d, const Price &pr, long long nx,
+                                          long long ny)
 {
     const unsigned long long ha = h * (unsigned long long)A.elem_bytes;
     const unsigned long long da = A.liveout ? d * (unsigned long long)A.elem_bytes : 0ull;
-    if (ha) o.th = __dadd_rn(o.th, __dadd_rn(pc.h2d.alpha_s,
-                                             __dmul_rn(pc.h2d.beta_s_per_byte, (double)ha)));
-    if (da) o.td = __dadd_rn(o.td, __dadd_rn(pc.d2h.alpha_s,
-                                             __dmul_rn(pc.d2h.beta_s_per_byte, (double)da)));
+    if (pr.mem) {
+        double th, td;
+        mem_terms(pr.mm, ha, da, footprint(A, nx, ny), th, td);
+        o.th = __dadd_rn(o.th, th);
+        o.td = __dadd_rn(o.td, td);
+    } else {
+        const grophecy_pcie &pc = pr.pc;
+        if (ha) o.th = __dadd_rn(o.th, __dadd_rn(pc.h2d.alpha_s,
+                                                 __dmul_rn(pc.h2d.beta_s_per_byte, (double)ha)));
+        if (da) o.td = __dadd_rn(o.td, __dadd_rn(pc.d2h.alpha_s,
+                                                 __dmul_rn(pc.d2h.beta_s_per_byte, (double)da)));
+    }
     o.h += ha;
     o.d += da;
 }
@@ -165,15 +221,17 @@ __device__ __forceinline__ unsigned long long poly_eval(const unsigned long long
 // the segment's lane 0 adds the transfer times in array order (N6).  The
 // kernels' work-item counts go to w_out.  Results: *res (segment lane 0).
 __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsigned long long key,
-                                           const grophecy_pcie &pc, double *T, int sl, int L,
+                                           const Price &pr, double *T, int sl, int L,
                                            Usage *res, uint32_t *w_out)
 {
-    uint32_t n_arrays = 0, K = 0, kb = 0, stride = 4;
+    const grophecy_pcie &pc = pr.pc;
+    uint32_t n_arrays = 0, K = 0, kb = 0, stride = 4, a_base = 0;
     uint32_t nx = 0, ny = 0;
     const unsigned long long *P = S.poly;
     if (active) {
         const SkelInfo &I = S.skel[(uint32_t)(key >> 42)];
         n_arrays = I.n_arrays;
+        a_base = I.a_base;
         K = I.n_kernels;
         kb = I.k_base;
         stride = I.poly_stride;
@@ -194,6 +252,13 @@ __device__ __forceinline__ void plan_usage(const SpaceDev &S, bool active, unsig
                                                                     __ull2double_rn(bytes)))
                                    : 0.0;
             if (dir) ds += bytes; else hs += bytes;
+        }
+        if (pr.mem) {   // reading 17: this array's pinned / pageable terms
+            const unsigned long long *c = P + (2 * a) * stride;
+            const unsigned long long bh = stride > 4 ? poly_eval<true>(c, a8, b8) : poly_eval<false>(c, a8, b8);
+            const unsigned long long bd = stride > 4 ? poly_eval<true>(c + stride, a8, b8)
+                                                     : poly_eval<false>(c + stride, a8, b8);
+            mem_terms(pr.mm, bh, bd, footprint(S.arrays[a_base + a], nx, ny), T[2 * a], T[2 * a + 1]);
         }
     }
     {
@@ -405,7 +470,7 @@ __device__ __forceinline__ void strided_cells(SweepScratch &ws, unsigned Lr, uns
 // the per-array PCIe transfer times in array order.  Used for keys outside
 // their skeleton's plan domain.
 __device__ __forceinline__ Usage warp_usage_sweep(const SpaceDev &S, const SkelInfo &I, long long nx, long long ny,
-                                  const grophecy_pcie &pc, WarpScratch &wsu, int lane)
+                                  const Price &pc, WarpScratch &wsu, int lane)
 {
     SweepScratch &ws = wsu.sw;
     Usage o = {0ull, 0ull, 0.0, 0.0};
@@ -572,7 +637,7 @@ __device__ __forceinline__ Usage warp_usage_sweep(const SpaceDev &S, const SkelI
                 }
             }
         }
-        add_array(o, A, h, d, pc);
+        add_array(o, A, h, d, pc, nx, ny);
     }
     return o;
 }
@@ -657,7 +722,7 @@ __device__ __forceinline__ Sec1 region_sec1(const RegionDev &g, int dim, long lo
 // dimensions); the hulls are then built one dimension at a time (the HK
 // UNION works per dimension), which keeps the live state small.
 __device__ __forceinline__ Usage warp_usage_hull(const SpaceDev &S, const SkelInfo &I, long long nx,
-                                                 long long ny, const grophecy_pcie &pc, int lane)
+                                                 long long ny, const Price &pc, int lane)
 {
     unsigned long long h = 0, d = 0;
     if ((uint32_t)lane < I.n_arrays) {
@@ -706,14 +771,14 @@ __device__ __forceinline__ Usage warp_usage_hull(const SpaceDev &S, const SkelIn
     Usage o = {0ull, 0ull, 0.0, 0.0};
     for (uint32_t a = 0; a < I.n_arrays; a++) {   // transfer times in array order
         const unsigned long long ha = __shfl_sync(FULL, h, a), da = __shfl_sync(FULL, d, a);
-        add_array(o, S.arrays[I.a_base + a], ha, da, pc);
+        add_array(o, S.arrays[I.a_base + a], ha, da, pc, nx, ny);
     }
     return o;
 }
 
 // Usage of one key off the plan path (outside the plan's domain, strided
 // sections, the hull mode) and its kernels' work counts, by the whole warp.
-__device__ __forceinline__ void slow_usage(const SpaceDev *gS, unsigned long long k, grophecy_pcie pc,
+__device__ __forceinline__ void slow_usage(const SpaceDev *gS, unsigned long long k, const Price &pc,
                                         WarpScratch *scr, Usage *res, uint32_t *w_out, int lane)
 {
     const SpaceDev &S = *gS;
@@ -1034,6 +1099,7 @@ struct Params {
     SpaceDev S;
     const SpaceDev *gS;   // device copy of S (out-of-line paths)
     grophecy_pcie pc;
+    Price pr;             // general path pricing (pc, or the memory choice)
     const uint32_t *skx, *nx, *ny, *iters;
     unsigned long long n, base;
     unsigned long long *h2d;
@@ -1173,14 +1239,14 @@ __device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsi
                     const unsigned pos = act ? ws.plan_pos[p0 + seg] : 0u;
                     const unsigned long long k = __shfl_sync(FULL, mk, pos);
                     const unsigned ls = g0 - c0 + pos;
-                    plan_usage(S, act, k, P.pc, ws.scratch.pl.T[seg], sl, L, &ws.res[ls],
+                    plan_usage(S, act, k, P.pr, ws.scratch.pl.T[seg], sl, L, &ws.res[ls],
                                ws.slot_w[ls]);
                     __syncwarp();
                 }
                 while (sweep) {
                     const int pos = __ffs(sweep) - 1;
                     const unsigned long long k = __shfl_sync(FULL, mk, pos);
-                    slow_usage(P.gS, k, P.pc, &ws.scratch, &ws.res[g0 - c0 + pos],
+                    slow_usage(P.gS, k, P.pr, &ws.scratch, &ws.res[g0 - c0 + pos],
                                ws.slot_w[g0 - c0 + pos], lane);
                     sweep &= sweep - 1;
                     __syncwarp();
@@ -1722,12 +1788,14 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
     __syncwarp();
     uint32_t phase = 0;
     const unsigned long long t0 = (unsigned long long)blockIdx.x * WARPS + warp;
-    if (lane == 0 && t0 < ntiles && full(t0)) issue_tile_copy(P, ws, t0 * CTILE);
+    if (lane == 0 && t0 < ntiles && full(t0) && !P.pr.mem) issue_tile_copy(P, ws, t0 * CTILE);
     for (unsigned long long tile = t0; tile < ntiles; tile += wstride) {
         const unsigned long long tb = tile * CTILE, nt = tile + wstride;
-        const unsigned long long next_tb = nt < ntiles && full(nt) ? nt * CTILE : ~0ull;
+        const unsigned long long next_tb = nt < ntiles && full(nt) && !P.pr.mem ? nt * CTILE : ~0ull;
         bool done = false;
-        if (full(tile)) {
+        if (P.pr.mem) {
+            // the memory choice is priced by the general path only
+        } else if (full(tile)) {
             mbar_wait(&ws.mbar, phase);
             phase ^= 1u;
             done = canon_tile<BEST>(P, ws, cw, tb, next_tb, lane, best_t, best_i, cnt_val);
@@ -1884,6 +1952,9 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
     P.S = s->dev;
     P.gS = s->dev_copy;
     P.pc = *pc;
+    P.pr.pc = *pc;
+    P.pr.mem = 0;
+    memset(&P.pr.mm, 0, sizeof P.pr.mm);
     P.skx = b->skx;
     P.nx = b->nx;
     P.ny = b->ny;
@@ -1951,6 +2022,73 @@ int grophecy_eval(const grophecy_space *s, const grophecy_pcie *pc, const grophe
                   uint64_t *h2d, uint64_t *d2h, double *t, void *stream)
 {
     return grophecy_eval_parts(s, pc, b, h2d, d2h, t, nullptr, stream);
+}
+
+static int status_of(const grophecy_best_result &r);
+
+// NEXT-4 (reading 17): the projection with every array's pinned /
+// pageable choice; the general path prices it (mem_terms).
+static int mem_params(const grophecy_space *s, const grophecy_memory_model *m,
+                      const grophecy_batch *b, Params &P)
+{
+    if (!m) {
+        set_error("null memory model");
+        return GROPHECY_EINVAL;
+    }
+    int rc = check_batch(s, &m->pinned, b);
+    if (rc) return rc;
+    P = make_params(s, &m->pinned, b);
+    P.pr.mm = *m;
+    P.pr.mem = 1;
+    return GROPHECY_OK;
+}
+
+int grophecy_eval_mem(const grophecy_space *s, const grophecy_memory_model *m,
+                      const grophecy_batch *b, uint64_t *h2d, uint64_t *d2h, double *t,
+                      const grophecy_parts *parts, void *stream)
+{
+    Params P;
+    int rc = mem_params(s, m, b, P);
+    if (rc) return rc;
+    if (b->n == 0) return GROPHECY_OK;
+    if (!h2d || !d2h || !t) {
+        set_error("null output array");
+        return GROPHECY_EINVAL;
+    }
+    DeviceGuard guard(s->device);
+    P.h2d = (unsigned long long *)h2d;
+    P.d2h = (unsigned long long *)d2h;
+    P.t = t;
+    if (parts) {
+        P.p_iter = parts->t_iter_s;
+        P.p_once = parts->t_once_s;
+        P.p_h2d = parts->t_h2d_s;
+        P.p_d2h = parts->t_d2h_s;
+    }
+    return launch_passes<false>(s, P, (cudaStream_t)stream);
+}
+
+int grophecy_best_mem(grophecy_space *s, const grophecy_memory_model *m, const grophecy_batch *b,
+                      grophecy_best_result *host_out, void *stream)
+{
+    Params P;
+    int rc = mem_params(s, m, b, P);
+    if (rc) return rc;
+    if (!host_out) {
+        set_error("null host_out");
+        return GROPHECY_EINVAL;
+    }
+    DeviceGuard guard(s->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    grophecy_best_result *dres = s->partials + (s->max_partials - 1);
+    P.out = dres;
+    P.accumulate = 0;
+    rc = launch_passes<true>(s, P, st);
+    if (rc) return rc;
+    cudaError_t e = cudaMemcpyAsync(host_out, dres, sizeof *host_out, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_fail(e, "grophecy_best_mem");
+    return status_of(*host_out);
 }
 
 int grophecy_best_async(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,

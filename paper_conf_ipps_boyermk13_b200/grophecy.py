@@ -141,6 +141,10 @@ _sig = {
     "grophecy_space_destroy": (None, [_vp]),
     "grophecy_eval": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, _vp, _vp, _vp]),
     "grophecy_invalid_count": (C.c_int, [_vp, C.POINTER(C.c_uint64), _vp]),
+    "grophecy_eval_mem": (C.c_int, [_vp, C.POINTER(MemoryModel), C.POINTER(Batch), _vp, _vp, _vp,
+                                    _vp, _vp]),
+    "grophecy_best_mem": (C.c_int, [_vp, C.POINTER(MemoryModel), C.POINTER(Batch),
+                                    C.POINTER(BestResult), _vp]),
     "grophecy_eval_parts": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, _vp, _vp,
                                       C.POINTER(Parts), _vp]),
     "grophecy_group_best": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, C.c_uint64,
@@ -387,6 +391,28 @@ class Space:
                                       _ptr(ts[0]), C.byref(parts), _stream_ptr(stream)),
                "eval_parts")
         return (h, d, *ts)
+
+    def eval_mem(self, model, rec, index_base=0, stream=None):
+        """NEXT-4: (h2d, d2h, t, t_iter, t_once, t_h2d, t_d2h) with the per-array
+        pinned / pageable choice of `model` (MemoryModel)."""
+        torch = _torch()
+        n, dev = rec.n, rec.skx.device
+        h = torch.empty(n, dtype=torch.int64, device=dev)
+        d = torch.empty(n, dtype=torch.int64, device=dev)
+        ts = [torch.empty(n, dtype=torch.float64, device=dev) for _ in range(5)]
+        parts = Parts(*[t.data_ptr() for t in ts[1:]])
+        b = rec.batch(index_base)
+        _check(_L.grophecy_eval_mem(self.h, C.byref(model), C.byref(b), _ptr(h), _ptr(d),
+                                    _ptr(ts[0]), C.byref(parts), _stream_ptr(stream)), "eval_mem")
+        return (h, d, *ts)
+
+    def best_mem(self, model, rec, index_base=0, stream=None):
+        r = BestResult()
+        b = rec.batch(index_base)
+        rc = _L.grophecy_best_mem(self.h, C.byref(model), C.byref(b), C.byref(r),
+                                  _stream_ptr(stream))
+        _check(rc, "best_mem", ok=(OK, ENOFEASIBLE, EBADCAND))
+        return rc, r
 
     def group_best(self, pc, rec, index_base=0, capacity=None, stream=None, out=None,
                    as_tensor=False):

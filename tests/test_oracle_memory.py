@@ -97,3 +97,70 @@ def test_library_matches_oracle_bitwise(O):
         assert rc == 0
         assert (c.t_pinned_s, c.t_pageable_s, c.memory) == (tp, tg, mm)
         assert not math.isnan(tp) and not math.isnan(tg)
+
+
+def _problem(O, skels):
+    from synth import skeletons as S
+    return O.Problem(skels, S.FX5600, O.fit_pcie(1e-5, 1.0, 1 << 20)[1])
+
+
+def test_eval_mem_reduces_to_the_paper_model(O):
+    """Pageable links equal to the pinned ones and a free allocation: every
+    array ties, stays pinned, and the projection is the paper's one with the
+    pinned links — bitwise."""
+    from synth import records as R
+    c = R.config("c4")
+    idx = np.arange(0, 10**9, 10**9 // 3000, dtype=np.uint64)
+    rec = R.gen_records_at(c, idx)
+    pin = L(O, 1.0e-5, 4.0e-10)
+    P = _problem(O, c["skeletons"])
+    P.hl = pin
+    P.dl = pin
+    for k in range(len(idx)):
+        a = [int(rec[f][k]) for f in ("skx", "nx", "ny", "iters")]
+        ok, h, d, t, th, td = P.eval_mem_one((pin, pin, pin, pin, L(O, 0.0, 0.0)), *a)
+        ok2, h2, d2, t2 = P.eval_one(*a)
+        assert (ok, h, d) == (ok2, h2, d2)
+        assert np.float64(t).view(np.uint64) == np.float64(t2).view(np.uint64)
+
+
+def test_eval_mem_expensive_allocation_is_all_pageable(O):
+    """A prohibitive allocation: every array pageable, i.e. the paper's model
+    with the pageable links."""
+    from synth import records as R
+    c = R.config("c3")
+    rec = R.gen_records(c, 0, 2000)
+    pin, page = L(O, 1.0e-5, 2.0e-11), L(O, 2.0e-5, 9.0e-11)
+    P = _problem(O, c["skeletons"])
+    P.hl = page
+    P.dl = page
+    for k in range(0, 2000, 3):
+        a = [int(rec[f][k]) for f in ("skx", "nx", "ny", "iters")]
+        ok, h, d, t, th, td = P.eval_mem_one((pin, pin, page, page, L(O, 1e3, 0.0)), *a)
+        assert (ok, h, d, t) == P.eval_one(*a)
+
+
+def test_eval_mem_hand_case(O):
+    """One array read (4 MiB, footprint 4 MiB) and written back: the chosen
+    memory and the two terms follow reading 17 by hand."""
+    from tests.tiny import DUMMY_KX
+    sk = {"name": "h", "arrays": [{"name": "a", "rows": (1, 0, 0, 0), "cols": (0, 8, 0, 0),
+                                   "elem_bytes": 4, "liveout": True}],
+          "kernels": [{"name": "k", "work": (0, 0, 0, 0), "per_iter": True}],
+          "regions": [{"kernel": 0, "array": 0, "mode": "RW", "whole": False, "r0": (0, 0, 0, 0),
+                       "r1": (1, 0, 0, 0), "c0": (0, 0, 0, 0), "c1": (0, 8, 0, 0)}],
+          "kx": [[DUMMY_KX]]}
+    n = 1 << 20
+    B = 4 * n
+    pin, page = L(O, 1e-5, 1e-10), L(O, 1e-5, 4e-10)
+    P = _problem(O, [sk])
+    for alloc, want in ((L(O, 1e-4, 0.0), 0), (L(O, 1e-2, 0.0), 1)):
+        ok, h, d, t, th, td = P.eval_mem_one((pin, pin, page, page, alloc), 0, n, 1, 1)
+        assert ok and (h, d) == (B, B)
+        pinned = (alloc.alpha + (1e-5 + 1e-10 * B)) + (1e-5 + 1e-10 * B)
+        pageable = (1e-5 + 4e-10 * B) + (1e-5 + 4e-10 * B)
+        assert (pinned <= pageable) == (want == 0)
+        if want == 0:
+            assert th == alloc.alpha + (1e-5 + 1e-10 * B) and td == 1e-5 + 1e-10 * B
+        else:
+            assert th == 1e-5 + 4e-10 * B and td == 1e-5 + 4e-10 * B
