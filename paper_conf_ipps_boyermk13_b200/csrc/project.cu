@@ -1705,7 +1705,8 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
 __device__ __forceinline__ void finish_best(const Params &P, const unsigned long long *best_h,
                                             const unsigned long long *best_d, int lane, int warp,
                                             double best_t, unsigned long long best_i,
-                                            uint32_t cnt_inv, uint32_t cnt_val)
+                                            uint32_t cnt_inv, uint32_t cnt_val,
+                                            unsigned nblocks)   // blocks taking part
 {
     __shared__ Best wbest[WARPS];
     __shared__ bool am_last;
@@ -1727,7 +1728,7 @@ __device__ __forceinline__ void finish_best(const Params &P, const unsigned long
             to_result(P.partials[blockIdx.x], b);
             __threadfence();
             const unsigned prev = atomicAdd(P.ticket, 1u);
-            am_last = prev == gridDim.x - 1;
+            am_last = prev == nblocks - 1;
         }
     }
     __syncthreads();
@@ -1735,7 +1736,7 @@ __device__ __forceinline__ void finish_best(const Params &P, const unsigned long
     __threadfence();
     if (warp == 0) {
         Best b = none_best();
-        for (unsigned j = lane; j < gridDim.x; j += 32) {
+        for (unsigned j = lane; j < nblocks; j += 32) {
             grophecy_best_result r;
             const volatile grophecy_best_result *pr = P.partials + j;
             r.t_total_s = pr->t_total_s;
@@ -1804,7 +1805,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
         }
         if (!done && lane == 0) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)tile;
     }
-    if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, 0u, cnt_val);
+    if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, 0u, cnt_val, gridDim.x);
 }
 
 // Pass 2: the listed tiles as general 128-record tiles (any layout).
@@ -1821,6 +1822,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
     ws.best_h[lane] = 0;
     ws.best_d[lane] = 0;
     const unsigned count = *(volatile unsigned *)P.tile_count;
+    // only the blocks with listed tiles take part (none: pass 1's result and
+    // outputs are final)
+    const unsigned nblocks = min(gridDim.x, (count + WARPS - 1) / WARPS);
+    if (blockIdx.x >= nblocks) return;
     const unsigned wstride = gridDim.x * WARPS;
     for (unsigned e = blockIdx.x * WARPS + warp; e < count; e += wstride) {
         const unsigned long long tb = (unsigned long long)P.tile_list[e] * CTILE;
@@ -1830,7 +1835,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
             if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
         }
     }
-    if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, cnt_inv, cnt_val);
+    if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, cnt_inv, cnt_val, nblocks);
 }
 
 __global__ void combine_kernel(const grophecy_best_result *in, uint32_t count,
