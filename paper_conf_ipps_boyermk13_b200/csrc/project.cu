@@ -1379,9 +1379,9 @@ __device__ __forceinline__ void group_usage(const unsigned long long *pp, uint32
 #pragma unroll
                 for (int m = 0; m < NQ; m++) c[i][dir][m] = __ldg(src + m);
             }
+        // arrays past n_arrays read the zero polynomial: 0 bytes, no term
 #pragma unroll
         for (int i = 0; i < AU; i++) {
-            if (a0 + (uint32_t)i >= n_arrays) break;
             unsigned long long v[2];
 #pragma unroll
             for (int dir = 0; dir < 2; dir++) {
@@ -1422,9 +1422,10 @@ __device__ __forceinline__ void group_usage32(const int4 *pp, uint32_t n_arrays,
                 const bool on = a0 + (uint32_t)i < n_arrays && ((pm >> q) & 1u);
                 c[i][dir] = __ldg(on ? pp + q : zero);
             }
+        // arrays past n_arrays read the zero polynomial: 0 bytes, no term
+        // (no early exit, so every load of the step is issued up front)
 #pragma unroll
         for (int i = 0; i < AU; i++) {
-            if (a0 + (uint32_t)i >= n_arrays) break;
             unsigned long long v[2];
 #pragma unroll
             for (int dir = 0; dir < 2; dir++) {
