@@ -1,20 +1,26 @@
-// The projection hot path for sm_100a: grophecy_eval / grophecy_best[_async]
-// / grophecy_best_combine / grophecy_best_host.
+// The projection hot path for sm_100a: grophecy_eval[_parts|_mem] /
+// grophecy_best[_async|_mem|_host] / grophecy_best_combine.
 //
-// One fused, persistent kernel per call.  A CTA (256 threads) takes a tile of
-// 1024 consecutive candidate records: each thread loads 4 records with one
-// 16-byte load per SoA array.  Data usage depends only on the key
-// (skeleton, nx, ny) (reading 11), so the CTA finds the runs of equal
-// keys with a block scan, computes the usage of every distinct key ONCE — from
-// the skeleton's compiled usage plan (plan.cpp) with several keys per warp, or
-// with the general coordinate-compressed sweep for keys outside the plan
-// domain — and keeps the results in shared memory.  The kernel-time model then
-// runs per candidate from per-(kernel, transformation) constants the host
-// precomputed in the definition's operation order; on saturated grids the two
-// remaining IEEE divisions use Markstein's correction
-// (q = a*rb; r = fma(-q, b, a); q' = fma(r, rb, q)), correctly rounded when
-// rb = RN(1/b), i.e. bitwise a / b.  Best mode fuses the argmin
-// (thread -> warp -> CTA -> grid, last-block pattern).
+// Two persistent launches per call.  Pass 1 (canon_kernel): every warp works
+// alone on canonical tiles of 512 records = 32 design points x 16
+// transformations of one skeleton, staged in shared memory by 1-D TMA bulk
+// copies one tile ahead; lane = design point computes the kernels' work
+// counts and the data usage once per design point from the skeleton's
+// residue-class byte polynomials (plan.cpp; usage depends only on the key
+// (skeleton, nx, ny), reading 11); then lane = (transformation,
+// half) models 8 design points per pass with one constant load per kernel.
+// Tiles that are not canonical (any other layout, ragged tails, invalid
+// records, keys off the polynomial domain, strided / hull / rank-3
+// skeletons, huge work counts) go to a list for pass 2 (general_kernel):
+// 128-record warp tiles, runs of equal keys, usage per distinct key (plans,
+// else the warp-cooperative coordinate-compressed sweep or the HK hull), the
+// model per record.  The kernel-time model runs from per-(kernel,
+// transformation) constants the host precomputed in the definition's
+// operation order; on saturated grids the two remaining IEEE divisions use
+// Markstein's correction (q = a*rb; r = fma(-q, b, a); q' = fma(r, rb, q)),
+// correctly rounded when rb = RN(1/b), i.e. bitwise a / b; small grids come
+// from a table computed step by step at space creation.  Best mode fuses the
+// argmin (lane -> warp -> CTA -> grid, last-block pattern).
 //
 // Compiled with -fmad=false: no contraction anywhere; FMAs appear only as the
 // explicit __fma_rn of the Markstein step.
