@@ -44,6 +44,7 @@ typedef enum {
     GROPHECY_EINVAL = -1,       /* bad argument / malformed descriptor */
     GROPHECY_ELIMIT = -2,       /* a documented size limit is exceeded */
     GROPHECY_ECUDA = -3,        /* CUDA runtime error (message has details) */
+    GROPHECY_ENCCL = -4,        /* NCCL missing or an NCCL call failed */
     GROPHECY_ENOFEASIBLE = -5,  /* best: no valid candidate with finite time */
     GROPHECY_EBADCAND = -6,     /* some records were invalid (see n_invalid) */
     GROPHECY_EINTERNAL = -7     /* internal consistency check failed (a bug) */
@@ -259,6 +260,24 @@ int grophecy_best_combine(const grophecy_best_result *device_in, uint32_t count,
 /* The same combine on the host (pure C, no CUDA). */
 int grophecy_best_combine_host(const grophecy_best_result *in, uint32_t count,
                                grophecy_best_result *out);
+
+/* Cross-GPU min-loc: every rank calls this with
+ * its shard (batch.index_base = the global index of its first record) and
+ * an ncclComm_t of the ranks (one rank per GPU); the fused best kernel runs
+ * on the shard, the ranks' results are all-gathered by NCCL on cuda_stream,
+ * and every rank receives the global best (lexicographic min of (t, global
+ * index)) in host_out.  Synchronises the stream.  NCCL is resolved at run
+ * time (libnccl.so.2, or the path in GROPHECY_NCCL_LIB): ENCCL if missing or
+ * on an NCCL error; status otherwise as grophecy_best for the global result. */
+int grophecy_best_allreduce(grophecy_space *space, const grophecy_pcie *pcie,
+                            const grophecy_batch *batch, void *nccl_comm,
+                            grophecy_best_result *host_out, void *cuda_stream);
+/* Communicator helpers (same run-time NCCL): a 128-byte ncclUniqueId for rank
+ * 0 to broadcast; ncclCommInitRank on `device` (comm_out: ncclComm_t);
+ * ncclCommDestroy. */
+int grophecy_nccl_unique_id(void *id_out);
+int grophecy_nccl_comm_init(int nranks, int rank, const void *id, int device, void **comm_out);
+int grophecy_nccl_comm_destroy(void *comm);
 
 /* Best transformation per projection point (the predicted kernel time
  * "is the predicted time of the best-performing version").  A group is a

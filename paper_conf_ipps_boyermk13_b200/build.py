@@ -16,7 +16,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(HERE, "libgrophecy.so")
-SOURCES = ["space.cpp", "plan.cpp", "project.cu", "groups.cu", "synth.cu", "pcie.cu"]
+SOURCES = ["space.cpp", "plan.cpp", "project.cu", "groups.cu", "synth.cu", "pcie.cu", "nccl.cpp"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -50,7 +50,7 @@ def build(force=False, verbose=False):
             cmd += [f"-D{m}={int(os.environ[m])}"]
     if os.environ.get("GROPHECY_MINB"):
         cmd += [f"-DGROPHECY_MINB={int(os.environ['GROPHECY_MINB'])}"]
-    cmd += [os.path.join(CSRC, f) for f in SOURCES]
+    cmd += [os.path.join(CSRC, f) for f in SOURCES] + ["-ldl"]
     subprocess.check_call(cmd)
     return LIB
 

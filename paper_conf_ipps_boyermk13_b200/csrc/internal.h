@@ -174,6 +174,9 @@ struct grophecy_space {
     // group_best scratch (grown on demand)
     void *gscratch;
     size_t gscratch_bytes;
+    // best_allreduce: gathered results + the combined one (grown on demand)
+    void *mscratch;
+    size_t mscratch_bytes;
     // e2e host path staging
     void *stage[2];
     size_t stage_bytes;

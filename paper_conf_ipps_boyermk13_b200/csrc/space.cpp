@@ -615,6 +615,7 @@ void grophecy_space_destroy(grophecy_space *sp)
     for (int i = 0; i < 2; i++)
         if (sp->stage[i]) cudaFree(sp->stage[i]);
     if (sp->gscratch) cudaFree(sp->gscratch);
+    if (sp->mscratch) cudaFree(sp->mscratch);
     if (sp->blob) cudaFree(sp->blob);
     cudaSetDevice(prev);
     delete sp;

@@ -141,6 +141,11 @@ _sig = {
     "grophecy_space_destroy": (None, [_vp]),
     "grophecy_eval": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, _vp, _vp, _vp]),
     "grophecy_invalid_count": (C.c_int, [_vp, C.POINTER(C.c_uint64), _vp]),
+    "grophecy_best_allreduce": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp,
+                                          C.POINTER(BestResult), _vp]),
+    "grophecy_nccl_unique_id": (C.c_int, [_vp]),
+    "grophecy_nccl_comm_init": (C.c_int, [C.c_int, C.c_int, _vp, C.c_int, C.POINTER(_vp)]),
+    "grophecy_nccl_comm_destroy": (C.c_int, [_vp]),
     "grophecy_eval_mem": (C.c_int, [_vp, C.POINTER(MemoryModel), C.POINTER(Batch), _vp, _vp, _vp,
                                     _vp, _vp]),
     "grophecy_best_mem": (C.c_int, [_vp, C.POINTER(MemoryModel), C.POINTER(Batch),
@@ -406,6 +411,16 @@ class Space:
                                     _ptr(ts[0]), C.byref(parts), _stream_ptr(stream)), "eval_mem")
         return (h, d, *ts)
 
+    def best_allreduce(self, pc, rec, comm, index_base=0, stream=None, batch=None):
+        """Global best over the ranks of NCCL communicator `comm` (NcclComm):
+        this rank's shard `rec` with global index_base."""
+        r = BestResult()
+        b = batch if batch is not None else rec.batch(index_base)
+        rc = _L.grophecy_best_allreduce(self.h, C.byref(pc), C.byref(b), comm.handle, C.byref(r),
+                                        _stream_ptr(stream))
+        _check(rc, "best_allreduce", ok=(OK, ENOFEASIBLE, EBADCAND))
+        return rc, r
+
     def best_mem(self, model, rec, index_base=0, stream=None):
         r = BestResult()
         b = rec.batch(index_base)
@@ -462,6 +477,31 @@ class Space:
                                    _stream_ptr(stream))
         _check(rc, "best_host", ok=(OK, ENOFEASIBLE, EBADCAND))
         return rc, r
+
+
+ENCCL = -4
+
+
+def nccl_unique_id():
+    """128-byte ncclUniqueId (rank 0 creates, all ranks receive it)."""
+    buf = (C.c_char * 128)()
+    _check(_L.grophecy_nccl_unique_id(buf), "nccl_unique_id")
+    return bytes(buf)
+
+
+class NcclComm:
+    """An ncclComm_t for grophecy_best_allreduce (one rank per GPU)."""
+
+    def __init__(self, nranks, rank, uid, device=0):
+        self.handle = C.c_void_p()
+        buf = (C.c_char * 128).from_buffer_copy(uid)
+        _check(_L.grophecy_nccl_comm_init(nranks, rank, buf, device, C.byref(self.handle)),
+               "nccl_comm_init")
+
+    def close(self):
+        if self.handle:
+            _L.grophecy_nccl_comm_destroy(self.handle)
+            self.handle = C.c_void_p()
 
 
 def best_result_tensor(n=1, device="cuda"):
