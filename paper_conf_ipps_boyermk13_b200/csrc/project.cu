@@ -988,7 +988,9 @@ struct WarpSmem {
 // which the usage polynomials and the constants live in.
 struct alignas(128) CanonSmem {
     alignas(128) uint32_t rec[4][CTILE];        // the tile's SoA records (TMA bulk copies)
-    double th[32], td[32], it[32];              // transfer times, (double) iters
+    // per group g at index (g & 1) * 16 + (g >> 1): a phase-C lane's groups
+    // (h, h + 2, ...) are consecutive (vector loads)
+    alignas(16) double th[32], td[32], it[32];  // transfer times, (double) iters
     unsigned long long uh[32], ud[32];          // transfer bytes
     unsigned long long best_h[32], best_d[32];
     unsigned long long mbar;                    // completion of the rec copies
@@ -1585,11 +1587,12 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
                                          reinterpret_cast<const int4 *>(S.poly), u);
         else if (stride > 4) group_usage<true, 2>(pp, stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
         else group_usage<false, 4>(pp, stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
-        ws.th[lane] = u.th;
-        ws.td[lane] = u.td;
-        ws.uh[lane] = u.h;
-        ws.ud[lane] = u.d;
-        ws.it[lane] = (double)i0;
+        const int q = (lane & 1) * 16 + (lane >> 1);
+        ws.th[q] = u.th;
+        ws.td[q] = u.td;
+        ws.uh[q] = u.h;
+        ws.ud[q] = u.d;
+        ws.it[q] = (double)i0;
     }
     __syncwarp();
     // ---- C: lane = (transformation x, half h); groups g = 2 i + h ----
@@ -1667,13 +1670,25 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
         const bool once = pim != (K == 32 ? 0xffffffffu : (1u << K) - 1u) || (xf & XINF_ONCE);
         double cm = __longlong_as_double(0x7ff0000000000000LL);
         int cj = -1;
+        // this chunk's per-group values: consecutive in the permuted layout
+        const int q0 = (int)h * 16 + i0g;
+        double itv[CG], thv[CG], tdv[CG];
+#pragma unroll
+        for (int j = 0; j < CG; j += 2) {
+            const double2 a = *reinterpret_cast<const double2 *>(&ws.it[q0 + j]);
+            const double2 b = *reinterpret_cast<const double2 *>(&ws.th[q0 + j]);
+            const double2 c = *reinterpret_cast<const double2 *>(&ws.td[q0 + j]);
+            itv[j] = a.x; itv[j + 1] = a.y;
+            thv[j] = b.x; thv[j + 1] = b.y;
+            tdv[j] = c.x; tdv[j + 1] = c.y;
+        }
         auto totals = [&](auto ONCE) {
 #pragma unroll
             for (int j = 0; j < CG; j++) {
                 const uint32_t g = 2u * (uint32_t)(i0g + j) + h;
-                double tk = __dmul_rn(ws.it[g], ti[j]);
+                double tk = __dmul_rn(itv[j], ti[j]);
                 if constexpr (decltype(ONCE)::value) tk = __dadd_rn(to[j], tk);
-                const double tt = __dadd_rn(__dadd_rn(tk, ws.th[g]), ws.td[g]);
+                const double tt = __dadd_rn(__dadd_rn(tk, thv[j]), tdv[j]);
                 if (BEST) {
                     // the lane's records come in increasing index order (tiles,
                     // chunks, j): strict < keeps the lowest index among ties
@@ -1683,13 +1698,13 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
                     }
                 } else {
                     const unsigned long long r = tb + (unsigned long long)g * CX + x;
-                    __stcs(P.h2d + r, ws.uh[g]);
-                    __stcs(P.d2h + r, ws.ud[g]);
+                    __stcs(P.h2d + r, ws.uh[q0 + j]);
+                    __stcs(P.d2h + r, ws.ud[q0 + j]);
                     __stcs(P.t + r, tt);
                     if (P.p_iter) __stcs(P.p_iter + r, ti[j]);
                     if (P.p_once) __stcs(P.p_once + r, to[j]);
-                    if (P.p_h2d) __stcs(P.p_h2d + r, ws.th[g]);
-                    if (P.p_d2h) __stcs(P.p_d2h + r, ws.td[g]);
+                    if (P.p_h2d) __stcs(P.p_h2d + r, thv[j]);
+                    if (P.p_d2h) __stcs(P.p_d2h + r, tdv[j]);
                 }
             }
         };
@@ -1699,8 +1714,8 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
             const uint32_t g = 2u * (uint32_t)(i0g + cj) + h;
             best_t = cm;
             best_i = P.base + tb + (unsigned long long)g * CX + x;
-            ws.best_h[lane] = ws.uh[g];
-            ws.best_d[lane] = ws.ud[g];
+            ws.best_h[lane] = ws.uh[q0 + cj];
+            ws.best_d[lane] = ws.ud[q0 + cj];
         }
     }
     if (BEST) cnt_val += CX;
