@@ -755,12 +755,12 @@ __device__ __forceinline__ Usage warp_usage_hull(const SpaceDev &S, const SkelIn
                 if (!((wmask >> q) & 1u) || G[q].kernel >= G[j].kernel) continue;
                 written = sec1_contains(region_sec1(G[q], 0, nx, ny, E[0]), xr) &&
                           sec1_contains(region_sec1(G[q], 1, nx, ny, E[1]), xc) &&
-                          sec1_contains(region_sec1(G[q], 2, nx, ny, E[2], r3), xp);
+                          (!r3 || sec1_contains(region_sec1(G[q], 2, nx, ny, E[2], r3), xp));
             }
             if (!written) keep |= 1u << j;
         }
         unsigned long long cr = 1, cw = 1;
-        for (int dim = 0; dim < 3; dim++) {
+        for (int dim = 0; dim < (r3 ? 3 : 2); dim++) {   // 2-D arrays: one plane
             Sec1 hr = {1, 0, 0}, hw = {1, 0, 0};
             for (uint32_t j = 0; j < n; j++) {
                 if (!((nonempty >> j) & 1u)) continue;
@@ -1476,12 +1476,14 @@ __device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t phas
 // Lane 0 of a warp: copy the CTILE records of the tile at tb (full, 16-byte
 // aligned) into ws.rec, completing on ws.mbar.  Earlier generic-proxy reads of
 // ws.rec are ordered before the async-proxy writes by the fence.
-__device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, unsigned long long tb)
+__device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, unsigned long long tb,
+                                                uint32_t ng)   // design points (<= 32)
 {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     const uint32_t bar = smem_u32(&ws.mbar);
+    const uint32_t bytes = ng * CX * (uint32_t)sizeof(uint32_t);   // per SoA array
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
-                 "r"((uint32_t)(4 * CTILE * sizeof(uint32_t)))
+                 "r"(4 * bytes)
                  : "memory");
     const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
 #pragma unroll
@@ -1489,7 +1491,7 @@ __device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, 
         asm volatile(
             "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                 smem_u32(ws.rec[a])),
-            "l"(src[a] + tb), "r"((uint32_t)(CTILE * sizeof(uint32_t))), "r"(bar)
+            "l"(src[a] + tb), "r"(bytes), "r"(bar)
             : "memory");
 }
 
@@ -1507,9 +1509,10 @@ __device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, 
 //      load serves 32 records), then writes outputs / keeps its argmin.
 template <bool BEST>
 __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint32_t *cw,
-                                           unsigned long long tb,
-                                           unsigned long long next_tb, int lane, double &best_t,
-                                           unsigned long long &best_i, uint32_t &cnt_val)
+                                           unsigned long long tb, uint32_t ng,
+                                           unsigned long long next_tb, uint32_t next_ng, int lane,
+                                           double &best_t, unsigned long long &best_i,
+                                           uint32_t &cnt_val)
 {
     const SpaceDev &S = P.S;
     // ---- A (records staged in ws.rec by the TMA; lane l reads its group's
@@ -1551,7 +1554,21 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
     same(3, i0);
     // every read of ws.rec is consumed (acc): the buffer takes the next tile
     __syncwarp();
-    if (lane == 0 && next_tb != ~0ull) issue_tile_copy(P, ws, next_tb);
+    if (lane == 0 && next_tb != ~0ull) issue_tile_copy(P, ws, next_tb, next_ng);
+    // a partial tile (the batch's last ng < 32 design points): lanes past it
+    // stand in for design point 0 in the warp-wide steps and output nothing
+    {
+        const uint32_t s00 = __shfl_sync(FULL, s0, 0), n00 = __shfl_sync(FULL, n0, 0);
+        const uint32_t m00 = __shfl_sync(FULL, m0, 0), i00 = __shfl_sync(FULL, i0, 0);
+        const uint32_t a00 = __shfl_sync(FULL, acc, 0);
+        if ((uint32_t)lane >= ng) {
+            s0 = s00;
+            n0 = n00;
+            m0 = m00;
+            i0 = i00;
+            acc = a00;
+        }
+    }
     const uint32_t skel = s0 >> 16;
     const uint32_t skel_l0 = __shfl_sync(FULL, skel, 0);   // (every lane: no short-circuit)
     bool ok = acc == 0 && skel < S.n_skels && n0 - 1u < GROPHECY_MAX_DIM &&
@@ -1689,6 +1706,7 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
                 double tk = __dmul_rn(itv[j], ti[j]);
                 if constexpr (decltype(ONCE)::value) tk = __dadd_rn(to[j], tk);
                 const double tt = __dadd_rn(__dadd_rn(tk, thv[j]), tdv[j]);
+                if (g >= ng) continue;   // past a partial tile
                 if (BEST) {
                     // the lane's records come in increasing index order (tiles,
                     // chunks, j): strict < keeps the lowest index among ties
@@ -1718,7 +1736,7 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
             ws.best_d[lane] = ws.ud[q0 + cj];
         }
     }
-    if (BEST) cnt_val += CX;
+    if (BEST && (uint32_t)lane < ng) cnt_val += CX;
     __syncwarp();
     return true;
 }
@@ -1806,24 +1824,32 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
     // full tiles of 16-byte aligned records are staged in shared memory by
     // the TMA one tile ahead (the copy of the next tile overlaps phases B and
     // C of this one); the others go to the general path directly
-    auto full = [&](unsigned long long t) { return P.aligned && (t + 1) * CTILE <= P.n; };
+    // design points a tile stages: 32, or the batch's last ng whole design
+    // points (n - tb a multiple of 16); 0 = not for pass 1
+    auto groups = [&](unsigned long long t) -> uint32_t {
+        if (!P.aligned || P.pr.mem) return 0u;
+        const unsigned long long tb = t * CTILE;
+        if (tb + CTILE <= P.n) return (uint32_t)(CTILE / CX);
+        const unsigned long long rest = P.n - tb;
+        return rest % CX == 0 ? (uint32_t)(rest / CX) : 0u;
+    };
     if (lane == 0) mbar_init(&ws.mbar, 1);
     __syncwarp();
     uint32_t phase = 0;
     const unsigned long long t0 = (unsigned long long)blockIdx.x * WARPS + warp;
-    if (lane == 0 && t0 < ntiles && full(t0) && !P.pr.mem) issue_tile_copy(P, ws, t0 * CTILE);
+    if (lane == 0 && t0 < ntiles && groups(t0)) issue_tile_copy(P, ws, t0 * CTILE, groups(t0));
     for (unsigned long long tile = t0; tile < ntiles; tile += wstride) {
         const unsigned long long tb = tile * CTILE, nt = tile + wstride;
-        const unsigned long long next_tb = nt < ntiles && full(nt) && !P.pr.mem ? nt * CTILE : ~0ull;
+        const uint32_t ng = groups(tile), next_ng = nt < ntiles ? groups(nt) : 0u;
+        const unsigned long long next_tb = next_ng ? nt * CTILE : ~0ull;
         bool done = false;
-        if (P.pr.mem) {
-            // the memory choice is priced by the general path only
-        } else if (full(tile)) {
+        if (ng) {   // (the memory choice, P.pr.mem, is priced by the general path only)
             mbar_wait(&ws.mbar, phase);
             phase ^= 1u;
-            done = canon_tile<BEST>(P, ws, cw, tb, next_tb, lane, best_t, best_i, cnt_val);
+            done = canon_tile<BEST>(P, ws, cw, tb, ng, next_tb, next_ng, lane, best_t, best_i,
+                                    cnt_val);
         } else if (lane == 0 && next_tb != ~0ull) {
-            issue_tile_copy(P, ws, next_tb);   // the buffer is idle during this tile
+            issue_tile_copy(P, ws, next_tb, next_ng);   // the buffer is idle during this tile
         }
         if (!done && lane == 0) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)tile;
     }
@@ -1846,14 +1872,21 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
     const unsigned count = *(volatile unsigned *)P.tile_count;
     // only the blocks with listed tiles take part (none: pass 1's result and
     // outputs are final)
-    const unsigned nblocks = min(gridDim.x, (count + WARPS - 1) / WARPS);
-    if (blockIdx.x >= nblocks) return;
+    // units of work: whole listed tiles per warp, or — when they are few
+    // (skeleton boundaries, a ragged tail) — their 128-record sub-tiles, so
+    // that as many warps share them instead of one warp per tile
+    constexpr unsigned SUBS = CTILE / WTILE;
     const unsigned wstride = gridDim.x * WARPS;
-    for (unsigned e = blockIdx.x * WARPS + warp; e < count; e += wstride) {
-        const unsigned long long tb = (unsigned long long)P.tile_list[e] * CTILE;
+    const unsigned per = count * SUBS <= wstride ? 1u : SUBS;   // sub-tiles per unit
+    const unsigned units = count * (SUBS / per);
+    const unsigned nblocks = min(gridDim.x, (units + WARPS - 1) / WARPS);
+    if (blockIdx.x >= nblocks) return;
+    for (unsigned u = blockIdx.x * WARPS + warp; u < units; u += wstride) {
+        const unsigned first = u * per;   // sub-tile index over the list
 #pragma unroll 1
-        for (int sub = 0; sub < CTILE / WTILE; sub++) {
-            const unsigned long long t0 = tb + (unsigned long long)sub * WTILE;
+        for (unsigned q = first; q < first + per; q++) {
+            const unsigned long long t0 = (unsigned long long)P.tile_list[q / SUBS] * CTILE +
+                                          (unsigned long long)(q % SUBS) * WTILE;
             if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
         }
     }

@@ -133,3 +133,13 @@ def test_shard_starting_inside_a_group(G, O, start):
     assert (b.index, b.n_valid) == (ob.index, ob.n_valid)
     assert _bits([b.t_total_s]) == _bits([ob.t_total_s])
     space.close()
+
+
+@pytest.mark.parametrize("n", [16, 160, 512 + 48, 3 * 512 + 496])
+def test_partial_canonical_tail(G, O, n):
+    """A batch ending in whole design points short of a full tile: the last
+    tile is canonical with fewer than 32 design points (lanes past them stand
+    in for the first and output nothing)."""
+    c = R.config("c4")
+    for s in (1, 4, 9):
+        _parts_parity(G, O, c["skeletons"], _segment(c, s, n))
