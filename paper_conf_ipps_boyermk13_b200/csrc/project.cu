@@ -317,6 +317,11 @@ __device__ __forceinline__ unsigned long long count_residue(long long a, long lo
 template <class F>
 __device__ __forceinline__ void plane_slabs(bool valid, long long p0, long long p1, long long P, F &&f)
 {
+    if (P == 1) {   // 2-D arrays (and one-plane rank-3 ones): every valid region
+        const unsigned pm = __ballot_sync(FULL, valid);
+        if (pm) f(pm, 1ull);
+        return;
+    }
     long long z = 0;
     while (z < P) {
         long long c = P;
