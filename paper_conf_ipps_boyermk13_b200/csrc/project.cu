@@ -348,19 +348,21 @@ __device__ __forceinline__ void strided_cells(SweepScratch &ws, unsigned Lr, uns
                               unsigned Wm, int lane, unsigned long long &h, unsigned long long &d,
                               bool valid, long long pl0, long long pl1, long long P)
 {
-    // residue masks: lanes over residues, regions' phases by shuffle
-    const unsigned pr = (unsigned)pmodll(ar, rs), pcp = (unsigned)pmodll(ac, cs);
-    for (unsigned rho0 = 0; rho0 < 64; rho0 += 32) {
-        const unsigned rho = rho0 + lane;
-        unsigned mr = 0, mc = 0;
-        for (int q = 0; q < n; q++) {
-            const unsigned sq = __shfl_sync(FULL, rs, q), phq = __shfl_sync(FULL, pr, q);
-            const unsigned tq = __shfl_sync(FULL, cs, q), pcq = __shfl_sync(FULL, pcp, q);
-            if (rho < Lr && (rho + sq - phq) % sq == 0) mr |= 1u << q;
-            if (rho < Lc && (rho + tq - pcq) % tq == 0) mc |= 1u << q;
-        }
-        if (rho < Lr) ws.pr_m[rho] = mr;
-        if (rho < Lc) ws.pc_m[rho] = mc;
+    // residue masks: lane q marks the residues its lattice hits (phase,
+    // phase + step, ... < L), then one ballot per residue transposes them
+    // into pr_m[rho] / pc_m[sigma] = the regions hitting that residue
+    unsigned long long rbits = 0, cbits = 0;
+    if (lane < n) {
+        for (unsigned r = (unsigned)pmodll(ar, rs); r < Lr; r += rs) rbits |= 1ull << r;
+        for (unsigned c = (unsigned)pmodll(ac, cs); c < Lc; c += cs) cbits |= 1ull << c;
+    }
+    for (unsigned rho = 0; rho < Lr; rho++) {
+        const unsigned m = __ballot_sync(FULL, (rbits >> rho) & 1ull);
+        if (lane == 0) ws.pr_m[rho] = m;
+    }
+    for (unsigned sig = 0; sig < Lc; sig++) {
+        const unsigned m = __ballot_sync(FULL, (cbits >> sig) & 1ull);
+        if (lane == 0) ws.pc_m[sig] = m;
     }
     __syncwarp();
     // Aggregate the row units (slab i, residue rho) by coverage mask — their
