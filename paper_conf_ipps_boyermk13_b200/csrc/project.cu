@@ -306,6 +306,11 @@ __device__ __forceinline__ unsigned long long count_residue(long long a, long lo
                                                            unsigned L)
 {
     if (L == 1) return (unsigned long long)len;
+    if (((unsigned long long)a | (unsigned long long)(a + len)) < (1ull << 31)) {   // 32-bit
+        const unsigned ua = (unsigned)a, ub = (unsigned)(a + len);
+        const unsigned first = ua + (rho + L - ua % L) % L;
+        return first < ub ? (unsigned long long)((ub - 1u - first) / L) + 1ull : 0ull;
+    }
     const long long first = a + pmodll((long long)rho - a, L);
     const long long b = a + len;
     return first < b ? (unsigned long long)((b - 1 - first) / L) + 1ull : 0ull;
