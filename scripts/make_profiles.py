@@ -93,6 +93,12 @@ def main(tag):
                    "warp_inst_per_launch": winst,
                    "source": f"profiles/{tag}_ncu_best.txt"},
                   open(os.path.join(PROF, "ncu_best_summary.json"), "w"), indent=1)
+    # stall / pipe breakdown and the hottest source lines of the same capture
+    for src, dst in (("best_summary.txt", f"{tag}_ncu_best_stalls.txt"),
+                     ("best_lines.txt", f"{tag}_ncu_best_lines.txt")):
+        p = os.path.join(OUT, src)
+        if os.path.exists(p) and os.path.getsize(p) > 0:
+            shutil.copy(p, os.path.join(PROF, dst))
     pj = os.path.join(OUT, "pcie.json")
     if os.path.exists(pj):
         shutil.copy(pj, os.path.join(PROF, f"{tag}_pcie.json"))
