@@ -1884,23 +1884,25 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
     const unsigned count = *(volatile unsigned *)P.tile_count;
     // only the blocks with listed tiles take part (none: pass 1's result and
     // outputs are final)
-    // units of work: whole listed tiles per warp, or — when they are few
-    // (skeleton boundaries, a ragged tail) — their 128-record sub-tiles, so
-    // that as many warps share them instead of one warp per tile
+    // units of work: the listed tiles' 128-record sub-tiles, claimed one at a
+    // time from a counter (P.tile_count[1], zeroed with the tile count before
+    // pass 1): the per-tile cost of the general sweep varies by orders of
+    // magnitude, so a static split leaves warps idle at the end.  One warp's
+    // claims increase, so its records still come in increasing index order.
     constexpr unsigned SUBS = CTILE / WTILE;
-    const unsigned wstride = gridDim.x * WARPS;
-    const unsigned per = count * SUBS <= wstride ? 1u : SUBS;   // sub-tiles per unit
-    const unsigned units = count * (SUBS / per);
+    const unsigned units = count * SUBS;
     const unsigned nblocks = min(gridDim.x, (units + WARPS - 1) / WARPS);
     if (blockIdx.x >= nblocks) return;
-    for (unsigned u = blockIdx.x * WARPS + warp; u < units; u += wstride) {
-        const unsigned first = u * per;   // sub-tile index over the list
+    unsigned *next = P.tile_count + 1;
 #pragma unroll 1
-        for (unsigned q = first; q < first + per; q++) {
-            const unsigned long long t0 = (unsigned long long)P.tile_list[q / SUBS] * CTILE +
-                                          (unsigned long long)(q % SUBS) * WTILE;
-            if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
-        }
+    for (;;) {
+        unsigned q = 0;
+        if (lane == 0) q = atomicAdd(next, 1u);
+        q = __shfl_sync(FULL, q, 0);
+        if (q >= units) break;
+        const unsigned long long t0 = (unsigned long long)P.tile_list[q / SUBS] * CTILE +
+                                      (unsigned long long)(q % SUBS) * WTILE;
+        if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
     }
     if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, cnt_inv, cnt_val, nblocks);
 }
@@ -1990,7 +1992,7 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         } else if (off) {
             Q.accumulate = 1;
         }
-        cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, sizeof(unsigned int), st);
+        cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, 2 * sizeof(unsigned int), st);   // count + pass-2 claim counter
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(tile count)");
         const int grid = grid_for(s, Q.n, 32, false), grid_c = grid_for(s, Q.n, 32, true);
         Q.canon_warp_bytes = canon_warp_bytes(s->max_kernels);
