@@ -966,6 +966,10 @@ __device__ __forceinline__ void to_result(grophecy_best_result &r, const Best &b
 // group per lane in phases A/B).  Phase C maps lane = (transformation x,
 // half h): the lane models transformation x of groups h, h + 2, ..., CG
 // groups per pass, so one (kernel, x) constant load serves CG records.
+// Work counters after P.tile_count (the space's 128-byte counter block):
+// the pass-1 and pass-2 tile claims.  (Separate 32-byte sectors, with the
+// pass-1 claim issued a tile further ahead, measured 2 % slower on C4.)
+constexpr int CLAIM1 = 2, CLAIM2 = 1;
 constexpr int CX = 16;
 constexpr int CTILE = 32 * CX;
 #ifndef GROPHECY_AU32
@@ -1848,10 +1852,22 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
     if (lane == 0) mbar_init(&ws.mbar, 1);
     __syncwarp();
     uint32_t phase = 0;
+    // first tile: blockIdx.x * WARPS + warp; then each warp claims its next
+    // tile from a counter (P.tile_count[CLAIM1], zeroed before the launch) one
+    // tile ahead, so that the TMA copy still overlaps this tile's phases B
+    // and C and the warps finish together although tile costs differ by
+    // skeleton.  One warp's claims increase (argmin tie order, see totals).
+    unsigned *claim = P.tile_count + CLAIM1;
     const unsigned long long t0 = (unsigned long long)blockIdx.x * WARPS + warp;
     if (lane == 0 && t0 < ntiles && groups(t0)) issue_tile_copy(P, ws, t0 * CTILE, groups(t0));
-    for (unsigned long long tile = t0; tile < ntiles; tile += wstride) {
-        const unsigned long long tb = tile * CTILE, nt = tile + wstride;
+#pragma unroll 1
+    for (unsigned long long tile = t0, nt; tile < ntiles; tile = nt) {
+        {
+            unsigned long long v = 0;
+            if (lane == 0) v = (unsigned long long)atomicAdd(claim, 1u) + wstride;
+            nt = __shfl_sync(FULL, v, 0);
+        }
+        const unsigned long long tb = tile * CTILE;
         const uint32_t ng = groups(tile), next_ng = nt < ntiles ? groups(nt) : 0u;
         const unsigned long long next_tb = next_ng ? nt * CTILE : ~0ull;
         bool done = false;
@@ -1885,15 +1901,15 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
     // only the blocks with listed tiles take part (none: pass 1's result and
     // outputs are final)
     // units of work: the listed tiles' 128-record sub-tiles, claimed one at a
-    // time from a counter (P.tile_count[1], zeroed with the tile count before
-    // pass 1): the per-tile cost of the general sweep varies by orders of
+    // time from a counter (P.tile_count[CLAIM2], zeroed with the tile count
+    // before pass 1): the per-tile cost of the general sweep varies by orders of
     // magnitude, so a static split leaves warps idle at the end.  One warp's
     // claims increase, so its records still come in increasing index order.
     constexpr unsigned SUBS = CTILE / WTILE;
     const unsigned units = count * SUBS;
     const unsigned nblocks = min(gridDim.x, (units + WARPS - 1) / WARPS);
     if (blockIdx.x >= nblocks) return;
-    unsigned *next = P.tile_count + 1;
+    unsigned *next = P.tile_count + CLAIM2;
 #pragma unroll 1
     for (;;) {
         unsigned q = 0;
@@ -1992,7 +2008,7 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         } else if (off) {
             Q.accumulate = 1;
         }
-        cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, 2 * sizeof(unsigned int), st);   // count + pass-2 claim counter
+        cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, (std::max(CLAIM1, CLAIM2) + 1) * sizeof(unsigned int), st);   // count + claim counters
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(tile count)");
         const int grid = grid_for(s, Q.n, 32, false), grid_c = grid_for(s, Q.n, 32, true);
         Q.canon_warp_bytes = canon_warp_bytes(s->max_kernels);

@@ -559,7 +559,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     unsigned char *ctr = base + scratch_off + align_up(part_bytes, 256);
     sp->ticket = (unsigned int *)ctr;
     sp->invalid_counter = (unsigned long long *)(ctr + 64);
-    sp->tile_count = (unsigned int *)(ctr + 128);
+    sp->tile_count = (unsigned int *)(ctr + 128);   // + the tile-claim counters (project.cu CLAIM1/2)
     sp->tile_list = (uint32_t *)(ctr + 256 + align_up(sizeof(SpaceDev), 256));
     if ((e = cudaMemset(ctr, 0, 256)) != cudaSuccess) return bail(e, "cudaMemset(space)");
 
