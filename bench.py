@@ -42,6 +42,8 @@ def parse():
     p.add_argument("--impl", default="grophecy", choices=["grophecy", "reference"])
     p.add_argument("--config", default="c4")
     p.add_argument("--n", type=int, default=None, help="override candidate count")
+    p.add_argument("--stripes", type=int, default=16,
+                   help="chunks per rank when N > 1 (strided over the workload)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -223,13 +225,24 @@ def main():
     if args.n:
         cfg = R.with_n(cfg, args.n)
     N = cfg["n"]
-    lo, hi = D.shard_range(N, rank, world)
-    n_local = hi - lo
+    # N > 1: the rank's shard is `stripes` tile-aligned chunks strided over
+    # the workload (chunk r + P k), so every rank gets the same skeleton mix
+    # (per-skeleton costs differ 4x; contiguous shards would leave the ranks
+    # with cheap skeletons idle).  N = 1: one contiguous launch.
+    chunks = D.striped_chunks(N, rank, world, args.stripes if world > 1 else 1)
+    lo = chunks[0][0]
+    n_local = sum(b - a for a, b in chunks)
     pc = G.pcie(G.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL))
     space = G.Space(cfg["skeletons"], S.FX5600)
     stream = torch.cuda.current_stream()
-    rec = G.synth_records(cfg, lo, n_local)          # shard generated in its own HBM
-    batch = rec.batch(index_base=lo)
+    rec = G.Records.empty(n_local)                   # shard generated in its own HBM
+    batches, off = [], 0
+    for a, b in chunks:
+        part = G.Records(rec.skx[off:off + b - a], rec.nx[off:off + b - a],
+                         rec.ny[off:off + b - a], rec.iters[off:off + b - a])
+        G.synth_records(cfg, a, b - a, out=part)
+        batches.append(part.batch(index_base=a))
+        off += b - a
     minloc = D.MinLoc(world, backend=backend)
     host_res = torch.empty(6, dtype=torch.int64, pin_memory=True)
     torch.cuda.synchronize()
@@ -240,7 +253,8 @@ def main():
     def step(i=None):
         if i is not None:
             ev_k[i][0].record(stream)
-        space.best_async(pc, batch, minloc.local)
+        for k, batch in enumerate(batches):
+            space.best_async(pc, batch, minloc.local, accumulate=k > 0)
         if i is not None:
             ev_k[i][1].record(stream)
         minloc.combine()                              # all-gather + combine kernel (N>1)
@@ -282,7 +296,8 @@ def main():
     # ---- end-to-end: host records through the public C-ABI call ----
     e2e = None
     if not args.no_e2e:
-        e2e = run_e2e(G, torch, dist, space, pc, rec, lo, n_local, N, world, args, minloc)
+        e2e = run_e2e(G, torch, dist, space, pc, rec, lo, chunks[0][1] - chunks[0][0], N, world,
+                      args, minloc)   # the first chunk (contiguous host records)
     if world > 1:
         dist.barrier()
     if rank != 0:

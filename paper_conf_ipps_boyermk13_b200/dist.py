@@ -20,6 +20,26 @@ def shard_range(n, rank, world):
     return (n * rank) // world, (n * (rank + 1)) // world
 
 
+def striped_chunks(n, rank, world, stripes, align=512):
+    """Rank r's records as ``stripes`` chunks j = r + P k (k < stripes) of the
+    P * stripes equal parts of [0, n), bounds rounded down to ``align`` (whole
+    512-record tiles) except the end.  Global indices are unchanged (each
+    chunk is projected with index_base = its start), so ties resolve
+    globally and the union over ranks is [0, n) exactly once."""
+    parts = world * stripes
+
+    def bound(j):
+        return n if j >= parts else (n * j // parts) // align * align
+
+    out = []
+    for k in range(stripes):
+        j = rank + world * k
+        a, b = bound(j), bound(j + 1)
+        if b > a:
+            out.append((a, b))
+    return out or [(0, 0)]
+
+
 class MinLoc:
     """Device buffers for one query: ``local`` (this rank's result, written by
     grophecy_best_async), ``result`` (the global best after combine()).

@@ -207,3 +207,23 @@ def test_group_fixup_over_gloo(O, world):
     for r in range(world):
         got += res[r]
     assert got == want
+
+
+@pytest.mark.parametrize("n,world,stripes", [(10**9, 8, 16), (10**9, 2, 16), (1000, 4, 16),
+                                             (10**6, 3, 5), (0, 2, 4)])
+def test_striped_chunks_partition(n, world, stripes):
+    """bench.py's N > 1 shards: every record exactly once, tile-aligned
+    chunk starts, every rank's chunks in increasing order."""
+    from paper_conf_ipps_boyermk13_b200 import dist as D
+    chunks = []
+    for r in range(world):
+        mine = [c for c in D.striped_chunks(n, r, world, stripes) if c[1] > c[0]]
+        assert all(a < b for a, b in mine)
+        assert all(mine[i][1] <= mine[i + 1][0] for i in range(len(mine) - 1))
+        assert all(a % 512 == 0 for a, _ in mine)
+        chunks += mine
+    pos = 0
+    for a, b in sorted(chunks):
+        assert a == pos
+        pos = b
+    assert pos == n
