@@ -42,13 +42,8 @@ def test_fit_rejects_invalid(O, args):
     assert rc != 0
 
 
-def test_linear_in_bytes(O, paper_link):
-    # Eq. (1) is affine: T(2d) - T(d) == T(d) - T(0+) - ... check slope exactly
-    # at power-of-two sizes where beta*d is an exact scaling of beta.
-    a = paper_link.alpha
-    for e in range(0, 30):
-        d = 1 << e
-        assert O.pcie_time(paper_link, d) == a + paper_link.beta * d
+# Eq. (1) itself is pinned against exact rational arithmetic in
+# tests/test_oracle_golden.py::test_pcie_time_exact_rational.
 
 
 def test_regimes_match_paper_magnitudes(O, paper_link):
