@@ -37,12 +37,32 @@ enum : uint32_t { XINF_ITER = 1u, XINF_ONCE = 2u };
 // Infeasible (occupancy 0): E = S = 0, sat = 0 (a finite 0 from the fast
 // path, replaced by +inf through SpaceDev::xinf).
 constexpr uint32_t KXF_SAT_BITS = 27, KXF_SAT_MASK = (1u << KXF_SAT_BITS) - 1u;
+// rep = RN(blocks / D) = RN(blocks * rDh + RN(blocks * rDl)) with rDh = RN(1/D),
+// rDl = RN(1/D - rDh) (one DMUL + one DFMA, exact for integer blocks and
+// integer D < 2^50: DESIGN.md §5 "two-product division"); t = cyc / freq the
+// same way with SpaceDev::rfh / rfl.
 struct __align__(16) KxFast {
     uint32_t m, satsh;        // first: the chain starts with blocks
     uint64_t cc;
-    double D, rD, E, S;
+    double rDl, rDh, E, S;
 };
 inline uint32_t kxf_sat(const KxFast &f) { return f.satsh & KXF_SAT_MASK; }
+
+// Class-specialised saturated constants (sweep kernel).  With
+// b = blocks (an integer), rep = RN(b / D) and cyc = RN(RN(E rep) + RN(S rep)):
+//   P2S0  D a power of two, S = 0:  cyc = RN(b E')            c = {E' = E / D}
+//   P2S   D a power of two:         cyc = RN(RN(b E') + RN(b S'))   c = {E', S'}
+//   NS0   S = 0:                    cyc = RN(E rep)          c = {rDh, rDl, E}
+//   NS    otherwise:                the full form            c = {rDh, rDl, E, S}
+// (b / D = b 2^-k is exact when D = 2^k, and E 2^-k, S 2^-k are exact scalings,
+// so RN(E rep) = RN(b E'); S = 0 makes RN(S rep) = +0.0, which adds nothing.)
+// m / satsh / cc as in KxFast.
+enum : uint32_t { KXC_P2S0 = 0u, KXC_P2S = 1u, KXC_NS0 = 2u, KXC_NS = 3u };
+struct __align__(16) KxCls {
+    uint32_t m, satsh;
+    uint64_t cc;
+    double c[4];
+};
 
 // General-grid constants (small grids / huge W), read only off the fast path.
 struct KxG {
@@ -64,8 +84,13 @@ struct SkelInfo {
     // poly[poly32_base + 2 * (c * n_polys + p)] holds int4 {c0, c1, c2, c3}
     // (sign-extended they are the u64 coefficients); POLY32_NONE if absent
     uint32_t poly32_base;
-    uint32_t pad3;
+    // the compact table padded for the sweep kernel: poly[polyf_base + 2 * (p
+    // * 64 + c)] holds int4 {c0, c1, c2, c3} of polynomial p in size class c,
+    // p < 2 * n_arrays rounded up to 2 * POLYF_AU (zero polynomials past
+    // n_arrays); POLY32_NONE if absent (staged whole into shared memory)
+    uint32_t polyf_base;
 };
+constexpr uint32_t POLYF_AU = 4;   // arrays per step of the fp64 usage evaluation
 
 struct ArrayDev {
     int4 rows, cols;
@@ -140,6 +165,10 @@ struct SpaceDev {
     const KxJ *kx_j;
     const KxG *kx_g;
     const KxFast *kx_f;
+    const KxCls *kx_c;          // class-specialised saturated constants (sweep kernel)
+    // per (skeleton, xform) at kx_base + x: kernel bit masks {infeasible,
+    // P2S0, P2S, NS0} (a feasible kernel in none of the three is NS)
+    const uint4 *xcls;
     const unsigned long long *poly;   // usage byte polynomials (all skeletons)
     // small-grid kernel times: small_t[kxi * small_stride + blocks] for
     // blocks < sat32 when sat32 <= small_stride (space.cpp small_grid_time)
@@ -147,10 +176,19 @@ struct SpaceDev {
     // per (skeleton, xform), at kx_base + x: some per-iteration (XINF_ITER) /
     // run-once (XINF_ONCE) kernel is infeasible, so that sum is +inf
     const uint32_t *xinf;
+    // sweep kernel: per (skeleton, kernel) at k_base + k, the smallest work
+    // count w for which every transformation's grid is saturated (blocks >=
+    // sat for all x); per (skeleton, unit u) at kx_base + u, the
+    // transformation of phase-C unit u (descending estimated cost)
+    const uint32_t *kern_wsat;
+    const uint32_t *xorder;
     uint32_t small_stride;
     uint32_t n_skels;
     uint32_t n_sm;
     double freq, rfreq;
+    // 1/freq as an unevaluated sum rfh + rfl (fast path: t = RN(cyc * rfh +
+    // RN(cyc * rfl)) = RN(cyc / freq) when freq's odd significand < 2^50)
+    double rfh, rfl;
     unsigned long long *invalid_counter;
 };
 
@@ -171,6 +209,8 @@ struct grophecy_space {
     int grid_best, grid_eval;            // persistent grid sizes
     uint32_t max_kernels;                // largest kernel count of the space's skeletons
     int occ_canon;                       // pass-1 CTAs per SM (0 = not yet queried)
+    int occ_sweep;                       // sweep-kernel CTAs per SM (0 = not yet queried)
+    uint32_t usage_tbl_bytes;            // largest padded usage table (sweep shared memory)
     // group_best scratch (grown on demand)
     void *gscratch;
     size_t gscratch_bytes;

@@ -1024,21 +1024,20 @@ struct CtaSmem {
 // (record, kernel) from the packed constants (sat, sh = satsh fields) and
 // the stored work count w (w_store, < 2^30 here): blocks = ceil(w / ipb) by
 // one 32x32+64 multiply-add and a shift, cyc = E rep + S rep, rep = blocks /
-// D, t = cyc / freq, both divisions by Markstein's correction (bitwise the
-// IEEE quotients).  gen is set when the grid is not saturated — the returned
-// value is then meaningless and the general branch decides.
+// D, t = cyc / freq, both divisions by the two-product method (x * zh +
+// RN(x * zl) with zh + zl = 1/divisor; one DMUL + one DFMA, bitwise the IEEE
+// quotient: DESIGN.md §5).  gen is set when the grid is not saturated — the
+// returned value is then meaningless and the general branch decides.
 __device__ __forceinline__ double fast_time(const KxFast &f, uint32_t sat, uint32_t sh, uint32_t w,
-                                            double freq, double rfreq, bool &gen, uint32_t &blocks)
+                                            double rfh, double rfl, bool &gen, uint32_t &blocks)
 {
     const unsigned long long p = (unsigned long long)w * f.m + f.cc;
     blocks = (uint32_t)(p >> 32) >> sh;
     gen = blocks < sat;
     const double bb = __uint2double_rn(blocks);
-    const double q = __dmul_rn(bb, f.rD);
-    const double rep = __fma_rn(__fma_rn(-q, f.D, bb), f.rD, q);
+    const double rep = __fma_rn(bb, f.rDh, __dmul_rn(bb, f.rDl));
     const double cyc = __dadd_rn(__dmul_rn(f.E, rep), __dmul_rn(f.S, rep));
-    const double q2 = __dmul_rn(cyc, rfreq);
-    return __fma_rn(__fma_rn(-q2, freq, cyc), rfreq, q2);
+    return __fma_rn(cyc, rfh, __dmul_rn(cyc, rfl));
 }
 
 // Kernel time off the saturated path: the small-grid table when the pair is
@@ -1081,7 +1080,7 @@ __device__ __forceinline__ void model_n(const SpaceDev &S, uint32_t s, const uin
             const KxFast F = SAMEX ? F0 : S.kx_f[kb + x[j]];
             w[j] = ws.slot_w[ls[j]][k];
             sat[j] = F.satsh & KXF_SAT_MASK;
-            tk[j] = fast_time(F, sat[j], F.satsh >> KXF_SAT_BITS, w[j], S.freq, S.rfreq, gen[j],
+            tk[j] = fast_time(F, sat[j], F.satsh >> KXF_SAT_BITS, w[j], S.rfh, S.rfl, gen[j],
                               blocks[j]);
             gen[j] |= w[j] == W_HUGE;
             E[j] = F.E;
@@ -1138,6 +1137,7 @@ struct Params {
     uint32_t *tile_list;      // pass 1 -> pass 2: tiles left to the general path
     unsigned int *tile_count;
     uint32_t canon_warp_bytes; // pass 1: shared memory per warp (canon_warp_bytes(kmax))
+    uint32_t sweep_kmax;       // sweep kernel: the space's largest kernel count (smem layout)
 };
 
 // Record validity (include/grophecy.h) and its usage key (skeleton, nx, ny).
@@ -1492,11 +1492,12 @@ __device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t phas
 // Lane 0 of a warp: copy the CTILE records of the tile at tb (full, 16-byte
 // aligned) into ws.rec, completing on ws.mbar.  Earlier generic-proxy reads of
 // ws.rec are ordered before the async-proxy writes by the fence.
-__device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, unsigned long long tb,
-                                                uint32_t ng)   // design points (<= 32)
+__device__ __forceinline__ void issue_copy(const Params &P, uint32_t (*rec)[CTILE],
+                                           unsigned long long *mbar, unsigned long long tb,
+                                           uint32_t ng)   // design points (<= 32)
 {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    const uint32_t bar = smem_u32(&ws.mbar);
+    const uint32_t bar = smem_u32(mbar);
     const uint32_t bytes = ng * CX * (uint32_t)sizeof(uint32_t);   // per SoA array
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
                  "r"(4 * bytes)
@@ -1506,9 +1507,14 @@ __device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, 
     for (int a = 0; a < 4; a++)
         asm volatile(
             "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                smem_u32(ws.rec[a])),
+                smem_u32(rec[a])),
             "l"(src[a] + tb), "r"(bytes), "r"(bar)
             : "memory");
+}
+__device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, unsigned long long tb,
+                                                uint32_t ng)
+{
+    issue_copy(P, ws.rec, &ws.mbar, tb, ng);
 }
 
 // One canonical tile: CTILE records from tb where every group of CX
@@ -1659,7 +1665,7 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
             uint32_t blocks[CG];
 #pragma unroll
             for (int j = 0; j < CG; j++) {
-                tk[j] = fast_time(f, sat, sh, w[j], S.freq, S.rfreq, gen[j], blocks[j]);
+                tk[j] = fast_time(f, sat, sh, w[j], S.rfh, S.rfl, gen[j], blocks[j]);
                 any |= gen[j];
             }
             if (any) {
@@ -1884,6 +1890,433 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
     if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, 0u, cnt_val, gridDim.x);
 }
 
+// ---- Sweep tiles: pass 1 of best mode ----
+// A CTA tile is WARPS canonical warp tiles of one skeleton: 32 * WARPS design
+// points x CX transformations (4096 records).  Phases A/B run per warp with
+// lane = design point (as canon_tile: TMA-staged records, checks, work
+// counts, byte polynomials, Eq. (1) pricing) and leave each design point's
+// work counts and transfer terms in CTA shared memory; after a barrier, phase
+// C is CTA-wide: a warp claims a transformation x and its lanes model x for
+// NCH design points each (groups 32 j + lane), so the (kernel, x) constants
+// and their class (internal.h KxCls) are warp-uniform and every lane runs
+// NCH independent chains of the class-specialised saturated model:
+// infeasible kernels are skipped (their sum is +inf through xinf), power-of-
+// two denominators and S = 0 drop their multiplications, and both divisions
+// take the two-product form.  CTA tiles that are not uniform (a skeleton
+// boundary, any other layout) and the batch's tail go to pass 2.
+constexpr int SW_GROUPS = 32 * WARPS;                               // design points per CTA tile
+constexpr unsigned long long SW_TILE = (unsigned long long)SW_GROUPS * CX;   // records per CTA tile
+#ifndef GROPHECY_NCH
+#define GROPHECY_NCH 8
+#endif
+constexpr int NCH = GROPHECY_NCH;                                   // chains per lane (divides WARPS)
+constexpr int SW_UNITS = CX * (WARPS / NCH);                        // phase-C units (x, chain block)
+constexpr uint32_t SW_BAD = 0xffffffffu;
+
+struct alignas(128) SweepSmem {
+    alignas(128) uint32_t rec[WARPS][4][CTILE];   // per warp: its warp tile (TMA bulk copies)
+    unsigned long long mbar[WARPS];
+    unsigned long long tbar;     // completion of the usage-table copy
+    // per design point g = 32 * (warp of phase B) + lane, natural order
+    alignas(16) double it[SW_GROUPS], th[SW_GROUPS], td[SW_GROUPS];
+    unsigned long long uh[SW_GROUPS], ud[SW_GROUPS];
+    unsigned long long best_h[THREADS], best_d[THREADS];   // bytes of each lane's running best
+    uint32_t smallk[SW_GROUPS];  // per design point: kernels whose grid may be unsaturated
+    uint32_t askel[WARPS];       // phase A result per warp: its skeleton, or SW_BAD
+    uint32_t wstat[WARPS];       // phase B result per warp: its skeleton, or SW_BAD
+    uint32_t next_tile;          // the CTA's next tile (claimed by thread 0)
+    uint32_t unit;               // phase-C unit counter
+    uint32_t tbl_skel;           // skeleton whose usage table is staged (SW_BAD: none)
+    uint32_t tbl_wait;           // this tile: parity to wait for on tbar, or SW_BAD (no copy)
+    uint32_t tbl_phase;          // parity of the next tbar completion
+};
+// followed by the work counts cw[k][lane][8] (uint32, w_store; design point
+// g = 32 j + lane at chunk (j / 4) ^ ((lane / 4) & 1), so a phase-C lane reads
+// its chains with two conflict-free 16-byte loads), sized by the space's
+// largest kernel count, then the staged usage table (SkelInfo::polyf_base)
+__host__ __device__ constexpr uint32_t sweep_cw_offset() { return (uint32_t)((sizeof(SweepSmem) + 127) / 128 * 128); }
+__host__ __device__ constexpr uint32_t sweep_tbl_offset(uint32_t kmax)
+{
+    return sweep_cw_offset() + kmax * (uint32_t)SW_GROUPS * (uint32_t)sizeof(uint32_t);
+}
+__host__ __device__ constexpr uint32_t sweep_smem_bytes(uint32_t kmax, uint32_t tbl_bytes)
+{
+    return sweep_tbl_offset(kmax) + tbl_bytes;
+}
+__device__ __forceinline__ uint32_t cw_index(uint32_t k, uint32_t lane, uint32_t j)
+{
+    return k * (uint32_t)SW_GROUPS + lane * 8u + ((((j >> 2) ^ (lane >> 2)) & 1u) << 2) + (j & 3u);
+}
+
+// group_usage over the staged padded table (shared memory, [q][class]):
+// per polynomial one 16-byte load {c0, c1, c2, c3} (int32: the u64
+// coefficients sign-extended; zero polynomials past n_arrays), bytes = c0 +
+// c1 a + c2 b + (c3 a) b in wrapping 64-bit arithmetic (the same residue mod
+// 2^64 as the u64 table, hence the same bytes), priced by Eq. (1) in array
+// order.
+__device__ __forceinline__ void group_usage_s(const int4 *pp, uint32_t n_arrays, uint32_t a8,
+                                              uint32_t b8, const grophecy_pcie &pc, Usage &u)
+{
+    const int a = (int)a8, b = (int)b8;
+    for (uint32_t a0 = 0; a0 < n_arrays; a0 += POLYF_AU, pp += 2 * POLYF_AU * POLY_CLASSES) {
+        int4 c[2 * POLYF_AU];
+#pragma unroll
+        for (int q = 0; q < 2 * (int)POLYF_AU; q++) c[q] = pp[q * POLY_CLASSES];
+#pragma unroll
+        for (int i = 0; i < (int)POLYF_AU; i++) {
+            unsigned long long v[2];
+#pragma unroll
+            for (int dir = 0; dir < 2; dir++) {
+                const int4 k = c[2 * i + dir];
+                const long long s1 = (long long)k.y * a + (long long)k.x + (long long)k.z * b;
+                const unsigned long long t = (unsigned long long)((long long)k.w * a);
+                v[dir] = (unsigned long long)s1 + t * (unsigned long long)(unsigned)b;
+            }
+            if (v[0]) u.th = __dadd_rn(u.th, __dadd_rn(pc.h2d.alpha_s,
+                                                       __dmul_rn(pc.h2d.beta_s_per_byte, __ull2double_rn(v[0]))));
+            if (v[1]) u.td = __dadd_rn(u.td, __dadd_rn(pc.d2h.alpha_s,
+                                                       __dmul_rn(pc.d2h.beta_s_per_byte, __ull2double_rn(v[1]))));
+            u.h += v[0];
+            u.d += v[1];
+        }
+    }
+}
+
+// Phase A of one warp tile staged at rec (full: 32 design points): lane l
+// reads its design point's 16 records (rotated 16-byte chunks, conflict-free)
+// and checks the canonical layout (skx = s0 ^ q, equal nx, ny, iters) and
+// validity; warp-uniform result.
+__device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*rec)[CTILE], int lane,
+                                              uint32_t &s0, uint32_t &n0, uint32_t &m0, uint32_t &i0)
+{
+    uint32_t acc;
+    const uint32_t r = ((uint32_t)lane >> 1) & 3u;
+    {
+        const uint4 *p = reinterpret_cast<const uint4 *>(rec[0] + lane * CX);
+        uint4 v[CX / 4];
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++) v[m] = p[(m + r) & 3u];
+        s0 = v[0].x ^ (4u * r);
+        acc = s0 & 0xffffu;
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++) {
+            const uint32_t c4 = 4u * ((m + r) & 3u);
+            acc |= (v[m].x ^ s0) ^ (c4 + 0u);
+            acc |= (v[m].y ^ s0) ^ (c4 + 1u);
+            acc |= (v[m].z ^ s0) ^ (c4 + 2u);
+            acc |= (v[m].w ^ s0) ^ (c4 + 3u);
+        }
+    }
+    auto same = [&](int arr, uint32_t &first) {
+        const uint4 *p = reinterpret_cast<const uint4 *>(rec[arr] + lane * CX);
+        uint4 v[CX / 4];
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++) v[m] = p[(m + r) & 3u];
+        first = v[0].x;
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++)
+            acc |= (v[m].x ^ first) | (v[m].y ^ first) | (v[m].z ^ first) | (v[m].w ^ first);
+    };
+    same(1, n0);
+    same(2, m0);
+    same(3, i0);
+    const uint32_t skel = s0 >> 16;
+    const uint32_t skel_l0 = __shfl_sync(FULL, skel, 0);
+    bool ok = acc == 0 && skel < S.n_skels && n0 - 1u < GROPHECY_MAX_DIM &&
+              m0 - 1u < GROPHECY_MAX_DIM && i0 >= 1 && skel == skel_l0;
+    if (ok) ok = S.skel[skel].n_xforms >= (uint32_t)CX && (S.skel[skel].flags & SKF_TABULATED);
+    return __all_sync(FULL, ok);
+}
+
+// Saturated kernel times of NCH records of one (kernel, x) pair of class C
+// (internal.h KxCls) from their block counts; t = cyc / freq by the
+// two-product division.
+template <uint32_t C>
+__device__ __forceinline__ void cls_times(const double2 c01, const double2 c23, const uint32_t (&blocks)[NCH],
+                                          double rfh, double rfl, double (&tk)[NCH])
+{
+#pragma unroll
+    for (int j = 0; j < NCH; j++) {
+        const double bb = __uint2double_rn(blocks[j]);
+        double cyc;
+        if (C == KXC_P2S0) {
+            cyc = __dmul_rn(bb, c01.x);
+        } else if (C == KXC_P2S) {
+            cyc = __dadd_rn(__dmul_rn(bb, c01.x), __dmul_rn(bb, c01.y));
+        } else {
+            const double rep = __fma_rn(bb, c01.x, __dmul_rn(bb, c01.y));
+            cyc = __dmul_rn(c23.x, rep);
+            if (C == KXC_NS) cyc = __dadd_rn(cyc, __dmul_rn(c23.y, rep));
+        }
+        tk[j] = __fma_rn(cyc, rfh, __dmul_rn(cyc, rfl));
+    }
+}
+
+// One (kernel, transformation) record of KxCls loaded whole (the next
+// kernel's is loaded while the current one is modelled).
+struct KC {
+    uint4 hd;
+    double2 c01, c23;
+};
+__device__ __forceinline__ KC load_kc(const KxCls *cp)
+{
+    const uint4 *q = reinterpret_cast<const uint4 *>(cp);
+    KC r;
+    r.hd = __ldg(q);
+    r.c01 = __ldg(reinterpret_cast<const double2 *>(q + 1));
+    r.c23 = __ldg(reinterpret_cast<const double2 *>(q + 2));
+    return r;
+}
+
+template <bool BEST>
+__global__ void __launch_bounds__(THREADS, 2) sweep_kernel(const Params P)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    SweepSmem &sm = *reinterpret_cast<SweepSmem *>(smem_raw);
+    uint32_t *cw = reinterpret_cast<uint32_t *>(smem_raw + sweep_cw_offset());
+    const int4 *tbl = reinterpret_cast<const int4 *>(smem_raw + sweep_tbl_offset(P.sweep_kmax));
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const SpaceDev &S = P.S;
+    double best_t = __longlong_as_double(0x7ff0000000000000LL);
+    unsigned long long best_i = ~0ull;
+    uint32_t cnt_val = 0;
+    sm.best_h[tid] = 0;
+    sm.best_d[tid] = 0;
+    // full CTA tiles of 16-byte aligned records (the TMA's alignment)
+    const unsigned long long ntiles = (P.aligned && !P.pr.mem) ? P.n / SW_TILE : 0ull;
+    // everything past them goes to pass 2 as warp tiles (warp-aggregated list appends)
+    {
+        const unsigned long long nsub = (P.n + CTILE - 1) / CTILE;
+        for (unsigned long long b0 = ntiles * WARPS + (unsigned long long)blockIdx.x * THREADS;
+             b0 < nsub; b0 += (unsigned long long)gridDim.x * THREADS) {
+            const unsigned long long sub = b0 + tid;
+            const bool mine = sub < nsub;
+            const unsigned bal = __ballot_sync(FULL, mine);
+            unsigned base = 0;
+            if (lane == 0 && bal) base = atomicAdd(P.tile_count, (unsigned)__popc(bal));
+            base = __shfl_sync(FULL, base, 0);
+            if (mine) P.tile_list[base + __popc(bal & ((1u << lane) - 1u))] = (uint32_t)sub;
+        }
+    }
+    if (lane == 0) mbar_init(&sm.mbar[warp], 1);
+    if (tid == 0) {
+        mbar_init(&sm.tbar, 1);
+        sm.tbl_skel = SW_BAD;
+        sm.tbl_phase = 0;
+    }
+    unsigned *claim = P.tile_count + CLAIM1;
+    unsigned long long tile = blockIdx.x;
+    __syncthreads();
+    if (lane == 0 && tile < ntiles) issue_copy(P, sm.rec[warp], &sm.mbar[warp], tile * SW_TILE + (unsigned long long)warp * CTILE, 32u);
+    uint32_t phase = 0;
+    const double rfh = S.rfh, rfl = S.rfl;
+#pragma unroll 1
+    while (tile < ntiles) {
+        // ---- A (this warp's tile) ----
+        mbar_wait(&sm.mbar[warp], phase);
+        phase ^= 1u;
+        uint32_t s0, n0, m0, i0;
+        bool ok = sweep_phase_a(S, sm.rec[warp], lane, s0, n0, m0, i0);
+        const uint32_t skel = s0 >> 16;
+        if (tid == 0) {
+            // warp 0's skeleton decides the tile's usage table: stage it in
+            // shared memory when it changes (every reader of the previous one
+            // passed the previous tile's barriers)
+            const uint32_t ts = ok ? skel : SW_BAD;
+            sm.tbl_wait = SW_BAD;
+            if (ts != SW_BAD && ts != sm.tbl_skel && S.skel[ts].polyf_base != POLY32_NONE) {
+                const SkelInfo &I0 = S.skel[ts];
+                const uint32_t bytes = 2u * ((I0.n_arrays + POLYF_AU - 1) / POLYF_AU) * POLYF_AU * POLY_CLASSES * 16u;
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                const uint32_t bar = smem_u32(&sm.tbar);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+                asm volatile(
+                    "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                        smem_u32(tbl)),
+                    "l"(S.poly + I0.polyf_base), "r"(bytes), "r"(bar)
+                    : "memory");
+                sm.tbl_skel = ts;
+                sm.tbl_wait = sm.tbl_phase;
+                sm.tbl_phase ^= 1u;
+            }
+        }
+        __syncthreads();   // the previous tile's phase C is done with the per-design-point arrays
+        if (tid == 0) {
+            sm.next_tile = atomicAdd(claim, 1u) + gridDim.x;
+            sm.unit = 0;
+        }
+        const uint32_t tw = sm.tbl_wait;
+        if (tw != SW_BAD) mbar_wait(&sm.tbar, tw);
+        // ---- B: work counts and usage of design point g ----
+        const int g = warp * 32 + lane;
+        if (ok) {
+            const SkelInfo &I = S.skel[skel];   // warp-uniform
+            const uint32_t K = I.n_kernels, n_arrays = I.n_arrays;
+            const long long nxny = (long long)((unsigned long long)n0 * m0);
+            bool huge = false;
+            uint32_t small = 0;
+            for (uint32_t k = 0; k < K; k++) {
+                const uint32_t w = w_store(aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny));
+                cw[cw_index(k, (uint32_t)lane, (uint32_t)warp)] = w;
+                huge |= w == W_HUGE;
+                small |= (w < __ldg(&S.kern_wsat[I.k_base + k]) ? 1u : 0u) << k;
+            }
+            sm.smallk[g] = small;
+            ok = !__any_sync(FULL, huge) && __all_sync(FULL, n0 >= I.plan_tx && m0 >= I.plan_ty);
+            if (ok) {
+                Usage u = {0ull, 0ull, 0.0, 0.0};
+                const uint32_t stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
+                const uint32_t cls = (n0 & 7u) * 8u + (m0 & 7u);
+                const uint32_t pm = I.poly_mask;
+                if (I.polyf_base != POLY32_NONE) {
+                    // the staged table is warp 0's skeleton: another skeleton
+                    // makes the tile non-uniform (pass 2) anyway
+                    ok = skel == sm.tbl_skel;
+                    if (ok) group_usage_s(tbl + cls, n_arrays, a8, b8, P.pc, u);
+                } else if (I.poly32_base != POLY32_NONE) {
+                    group_usage32<GROPHECY_AU32>(reinterpret_cast<const int4 *>(S.poly + I.poly32_base) +
+                                                     (size_t)cls * (2u * n_arrays),
+                                                 n_arrays, pm, a8, b8, P.pc,
+                                                 reinterpret_cast<const int4 *>(S.poly), u);
+                } else if (stride > 4) {
+                    group_usage<true, 2>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride), stride,
+                                         n_arrays, pm, a8, b8, P.pc, S.poly, u);
+                } else {
+                    group_usage<false, 4>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride), stride,
+                                          n_arrays, pm, a8, b8, P.pc, S.poly, u);
+                }
+                sm.th[g] = u.th;
+                sm.td[g] = u.td;
+                sm.uh[g] = u.h;
+                sm.ud[g] = u.d;
+                sm.it[g] = (double)i0;
+            }
+        }
+        if (lane == 0) sm.wstat[warp] = ok ? skel : SW_BAD;
+        __syncthreads();
+        const unsigned long long nt = sm.next_tile;
+        // every read of this warp's staged tile is done (phase A): it takes the next one
+        if (lane == 0 && nt < ntiles)
+            issue_copy(P, sm.rec[warp], &sm.mbar[warp], nt * SW_TILE + (unsigned long long)warp * CTILE, 32u);
+        const uint32_t s_all = sm.wstat[0];
+        bool uni = s_all != SW_BAD;
+#pragma unroll
+        for (int w = 1; w < WARPS; w++) uni &= sm.wstat[w] == s_all;
+        if (!uni) {
+            if (lane == 0) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * WARPS + warp);
+            tile = nt;
+            continue;
+        }
+        // ---- C: CTA-wide; unit = (transformation x, chain block) ----
+        const SkelInfo &I = S.skel[s_all];
+        const uint32_t K = I.n_kernels, X = I.n_xforms, pim = I.per_iter_mask;
+        const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
+        const unsigned long long tbase = P.base + tile * SW_TILE;
+#pragma unroll 1
+        for (;;) {
+            unsigned u = 0;
+            if (lane == 0) u = atomicAdd(&sm.unit, 1u);
+            u = __shfl_sync(FULL, u, 0);
+            if (u >= (unsigned)SW_UNITS) break;
+            const uint32_t x = __ldg(&S.xorder[I.kx_base + u % CX]), jb = u / CX;
+            const uint4 cm = __ldg(&S.xcls[I.kx_base + x]);
+            const uint32_t xf = __ldg(&S.xinf[I.kx_base + x]);
+            // kernels whose grid may be unsaturated for one of the warp's design points
+            uint32_t gk = 0;
+#pragma unroll
+            for (int j = 0; j < NCH; j++) gk |= sm.smallk[32 * ((int)jb * NCH + j) + lane];
+            gk = __reduce_or_sync(FULL, gk);
+            double ti[NCH], to[NCH];
+#pragma unroll
+            for (int j = 0; j < NCH; j++) ti[j] = to[j] = 0.0;
+            const KxCls *cbase = S.kx_c + I.kx_base + x;
+            auto one_kernel = [&](uint32_t k, double (&acc)[NCH]) {
+                const KC kc = load_kc(cbase + k * X);
+                const uint32_t sat = kc.hd.y & KXF_SAT_MASK, sh = kc.hd.y >> KXF_SAT_BITS;
+                const unsigned long long cc = ((unsigned long long)kc.hd.w << 32) | kc.hd.z;
+                uint32_t blocks[NCH];
+#pragma unroll
+                for (int j = 0; j < NCH; j += 4) {
+                    const uint4 w4 = *reinterpret_cast<const uint4 *>(
+                        cw + cw_index(k, (uint32_t)lane, (uint32_t)((int)jb * NCH + j)));
+                    const uint32_t w[4] = {w4.x, w4.y, w4.z, w4.w};
+#pragma unroll
+                    for (int q = 0; q < 4; q++)
+                        blocks[j + q] = (uint32_t)(((unsigned long long)w[q] * kc.hd.x + cc) >> 32) >> sh;
+                }
+                double tk[NCH];
+                const uint32_t bit = 1u << k;
+                if (cm.y & bit) cls_times<KXC_P2S0>(kc.c01, kc.c23, blocks, rfh, rfl, tk);
+                else if (cm.z & bit) cls_times<KXC_P2S>(kc.c01, kc.c23, blocks, rfh, rfl, tk);
+                else if (cm.w & bit) cls_times<KXC_NS0>(kc.c01, kc.c23, blocks, rfh, rfl, tk);
+                else cls_times<KXC_NS>(kc.c01, kc.c23, blocks, rfh, rfl, tk);
+                if (gk & bit) {
+                    // off the saturated path: the small-grid table (SKF_TABULATED)
+                    bool any = false;
+#pragma unroll
+                    for (int j = 0; j < NCH; j++) any |= blocks[j] < sat;
+                    if (any) {
+                        const double *row = S.small_t + (size_t)(I.kx_base + k * X + x) * S.small_stride;
+#pragma unroll
+                        for (int j = 0; j < NCH; j++)
+                            if (blocks[j] < sat) tk[j] = __ldg(row + blocks[j]);
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < NCH; j++) acc[j] = __dadd_rn(acc[j], tk[j]);
+            };
+            // sums in ascending kernel order (N6); infeasible kernels skipped:
+            // their sum is +inf (xinf), whatever the others add
+#pragma unroll 1
+            for (uint32_t mask = pim & kmask & ~cm.x; mask; mask &= mask - 1u)
+                one_kernel((uint32_t)__ffs(mask) - 1u, ti);
+#pragma unroll 1
+            for (uint32_t mask = ~pim & kmask & ~cm.x; mask; mask &= mask - 1u)
+                one_kernel((uint32_t)__ffs(mask) - 1u, to);
+            const double inf = __longlong_as_double(0x7ff0000000000000LL);
+            if (xf & XINF_ITER) {
+#pragma unroll
+                for (int j = 0; j < NCH; j++) ti[j] = inf;
+            }
+            if (xf & XINF_ONCE) {
+#pragma unroll
+                for (int j = 0; j < NCH; j++) to[j] = inf;
+            }
+            // totals; without run-once kernels t_once =
+            // +0.0 and +0.0 + iters * t_iter = iters * t_iter exactly
+            const bool once = (pim & kmask) != kmask || (xf & XINF_ONCE);
+            double cmin = inf;
+            int cj = -1;
+#pragma unroll
+            for (int j = 0; j < NCH; j++) {
+                const int gj = 32 * ((int)jb * NCH + j) + lane;
+                double tk = __dmul_rn(sm.it[gj], ti[j]);
+                if (once) tk = __dadd_rn(to[j], tk);
+                const double tt = __dadd_rn(__dadd_rn(tk, sm.th[gj]), sm.td[gj]);
+                // chains in increasing record index: strict < keeps the lowest
+                if (tt < cmin) {
+                    cmin = tt;
+                    cj = j;
+                }
+            }
+            if (cj >= 0) {
+                const int gj = 32 * ((int)jb * NCH + cj) + lane;
+                const unsigned long long idx = tbase + (unsigned long long)gj * CX + x;
+                if (better(cmin, idx, best_t, best_i)) {
+                    best_t = cmin;
+                    best_i = idx;
+                    sm.best_h[tid] = sm.uh[gj];
+                    sm.best_d[tid] = sm.ud[gj];
+                }
+            }
+        }
+        if (lane == 0) cnt_val += (uint32_t)CTILE;
+        tile = nt;
+    }
+    if (BEST) finish_best(P, sm.best_h + warp * 32, sm.best_d + warp * 32, lane, warp, best_t, best_i, 0u,
+                          cnt_val, gridDim.x);
+}
+
 // Pass 2: the listed tiles as general 128-record tiles (any layout).
 template <bool BEST>
 __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const Params P)
@@ -1946,6 +2379,8 @@ static void set_smem_attrs()
     cudaFuncSetAttribute(canon_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
     cudaFuncSetAttribute(general_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     cudaFuncSetAttribute(general_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+    cudaFuncSetAttribute(sweep_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)sweep_smem_bytes(MAXK, 2u * GROPHECY_MAX_ARRAYS * POLY_CLASSES * 16u));
     done = true;
 }
 
@@ -1975,6 +2410,24 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)std::min(occ, per_sm_cap);
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
+}
+
+// Persistent grid of the sweep kernel: every SM full (occupancy per space:
+// its dynamic shared memory depends on the largest kernel count), at most one
+// CTA per CTA tile (at least one: it lists the tail for pass 2).
+static int sweep_grid(const grophecy_space *s, unsigned long long n)
+{
+    set_smem_attrs();
+    if (!s->occ_sweep) {
+        int o = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, sweep_kernel<true>, THREADS,
+                                                      sweep_smem_bytes(s->max_kernels, s->usage_tbl_bytes));
+        const_cast<grophecy_space *>(s)->occ_sweep = o < 1 ? 1 : o;
+    }
+    const unsigned long long want = std::max<unsigned long long>(1ull, n / SW_TILE);
+    unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)s->occ_sweep;
+    if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
+    return (int)std::min(want, cap);
 }
 
 // One projection = per chunk of at most GROPHECY_TILE_CAP tiles: reset the
@@ -2010,9 +2463,17 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         }
         cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, (std::max(CLAIM1, CLAIM2) + 1) * sizeof(unsigned int), st);   // count + claim counters
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(tile count)");
-        const int grid = grid_for(s, Q.n, 32, false), grid_c = grid_for(s, Q.n, 32, true);
+        const int grid = grid_for(s, Q.n, 32, false);
         Q.canon_warp_bytes = canon_warp_bytes(s->max_kernels);
-        canon_kernel<BEST><<<grid_c, THREADS, WARPS * Q.canon_warp_bytes, st>>>(Q);
+        if (BEST) {
+            // pass 1: CTA sweep tiles (canonical layouts, one skeleton per tile)
+            const int grid_s = sweep_grid(s, Q.n);
+            Q.sweep_kmax = s->max_kernels;
+            sweep_kernel<true><<<grid_s, THREADS, sweep_smem_bytes(s->max_kernels, s->usage_tbl_bytes), st>>>(Q);
+        } else {
+            const int grid_c = grid_for(s, Q.n, 32, true);
+            canon_kernel<BEST><<<grid_c, THREADS, WARPS * Q.canon_warp_bytes, st>>>(Q);
+        }
         Q.accumulate = BEST ? 1 : 0;   // pass 2 merges into pass 1's result
         general_kernel<BEST><<<grid, THREADS, sizeof(CtaSmem), st>>>(Q);
         count_launch(2);

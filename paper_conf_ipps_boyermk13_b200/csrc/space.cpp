@@ -215,6 +215,29 @@ static void precompute(const grophecy_kx_desc &c, const grophecy_gpu_model &g, K
     es.S = gg.dd * (mwp - 1.0) * c.synch_insts * (double)occ;
 }
 
+// The two-product division x / v = RN(x * hi + RN(x * lo)), hi = RN(1/v),
+// lo = RN(1/v - hi) (the residual 1 - v * hi is exact by FMA), is bitwise the
+// IEEE quotient for every double x (normal operands) when the odd part of v's
+// significand is below 2^50: x / v then lies at least ulp / (2 * odd) from
+// every rounding midpoint while the unevaluated sum errs by at most
+// ulp * 2^-52.  div2_ok checks the condition.
+static bool div2_ok(double v)
+{
+    if (!(v > 0.0) || !std::isfinite(v)) return false;
+    int e = 0;
+    uint64_t M = (uint64_t)std::ldexp(std::frexp(v, &e), 53);   // exact 53-bit significand
+    while (!(M & 1u)) M >>= 1;
+    return M < (1ull << 50);
+}
+static void split_recip(double v, double &hi, double &lo)
+{
+    hi = 1.0 / v;
+    lo = std::fma(-v, hi, 1.0) / v;
+}
+// Saturated constants usable by the fast path: zero or normal and far from
+// overflow, so every product of the two-product divisions stays normal.
+static bool fast_const_ok(double c) { return c == 0.0 || (c >= 0x1p-900 && c <= 0x1p+900); }
+
 // Kernel time on a grid of `blocks` < sat_blocks blocks: the general branch of
 // DESIGN.md §3 N5 step by step, in the definition's operation order (the same
 // order as the device's kernel_time and the oracle).  Tabulated at space
@@ -313,7 +336,15 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxJ> kj;
     std::vector<KxG> kg;
     std::vector<KxFast> kf;
+    std::vector<KxCls> kc;
+    std::vector<uint4> xcls;      // per (skeleton, xform) at kx_base + x: class masks
+    std::vector<uint32_t> kwsat;  // per (skeleton, kernel): work count saturating every xform
+    std::vector<uint32_t> xord;   // per (skeleton, unit) at kx_base + u: phase-C order
     std::vector<uint32_t> xinf;   // per (skeleton, xform) at kx_base + x: XINF_* bits
+    // the fast path divides by freq with the two-product method: without it
+    // (a frequency whose odd significand is >= 2^50) every pair takes the
+    // general path's step-by-step definition
+    const bool freq_ok = div2_ok(gpu->freq_hz);
     // poly[0..9]: an all-zero polynomial (the device reads it instead of the
     // polynomials that vanish in every class: unconditional loads)
     std::vector<unsigned long long> poly(POLY_ZERO_WORDS, 0ull);
@@ -377,7 +408,27 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             I.poly_mask = 0;
             I.poly32_base = POLY32_NONE;
         }
-        I.per_iter_mask = I.pad3 = 0;
+        // padded int32 copy of the bilinear table for the sweep kernel, laid
+        // out polynomial-major ([q][class]: lanes of different size classes
+        // read different shared-memory banks): 2 * n_arrays polynomials
+        // rounded up to 2 * POLYF_AU (zero polynomials past n_arrays)
+        I.polyf_base = POLY32_NONE;
+        if (I.poly32_base != POLY32_NONE) {
+            const size_t np = 2 * (size_t)S.n_arrays;
+            const size_t npf = 2 * ((S.n_arrays + POLYF_AU - 1) / POLYF_AU) * POLYF_AU;
+            I.polyf_base = (uint32_t)poly.size();   // even: 16-byte aligned
+            for (size_t q = 0; q < npf; q++)
+                for (size_t c = 0; c < POLY_CLASSES; c++) {
+                    uint32_t w4[4] = {0u, 0u, 0u, 0u};
+                    if (q < np)
+                        for (int m = 0; m < 4; m++) w4[m] = (uint32_t)plan.poly[(c * np + q) * 4 + m];
+                    uint64_t w[2];
+                    std::memcpy(w, w4, sizeof w);
+                    poly.push_back(w[0]);
+                    poly.push_back(w[1]);
+                }
+        }
+        I.per_iter_mask = 0;
         for (uint32_t k = 0; k < S.n_kernels; k++)
             if (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) I.per_iter_mask |= 1u << k;
         for (uint32_t k = 0; k < S.n_kernels; k++) {
@@ -431,7 +482,11 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             arrays.push_back(A);
         }
         const size_t kx0 = kf.size();   // this skeleton's kx_base
+        kwsat.resize(kwork.size(), 0u);
+        xord.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, 0u);
+        std::vector<double> xcost(S.n_xforms, 0.0);
         xinf.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, 0u);
+        xcls.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, make_uint4(0u, 0u, 0u, 0u));
         for (uint32_t k = 0; k < S.n_kernels; k++)
             for (uint32_t x = 0; x < S.n_xforms; x++) {
                 KxES es; KxD d; KxI i; KxJ j; KxG g;
@@ -464,19 +519,59 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                     // path yields a finite 0 here (sat = 0, never the general
                     // branch) and the record's sum is set to +inf from xinf
                     // (+inf + finite = +inf in any order: exact)
-                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; sat = 0;
+                    f.E = 0.0; f.S = 0.0; f.rDh = 1.0; f.rDl = 0.0; sat = 0;
                     xinf[kx0 + x] |= (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) ? XINF_ITER : XINF_ONCE;
-                } else if (dv > (1u << 30) || i.sat_blocks >= KXF_SAT_MASK) {
-                    f.E = 0.0; f.S = 0.0; f.D = 1.0; f.rD = 1.0; sat = KXF_SAT_MASK;
+                } else if (dv > (1u << 30) || i.sat_blocks >= KXF_SAT_MASK || !freq_ok ||
+                           !div2_ok(d.D) || !fast_const_ok(es.E) || !fast_const_ok(es.S)) {
+                    f.E = 0.0; f.S = 0.0; f.rDh = 1.0; f.rDl = 0.0; sat = KXF_SAT_MASK;
                     f.m = 0;
                     f.cc = 0;
                 } else {
-                    f.E = es.E; f.S = es.S; f.D = d.D; f.rD = d.rD;
+                    f.E = es.E; f.S = es.S;
+                    split_recip(d.D, f.rDh, f.rDl);
                     sat = (uint32_t)i.sat_blocks;
                 }
                 f.satsh = sat | sh << KXF_SAT_BITS;
                 kf.push_back(f);
+                // the sweep kernel's class record (internal.h KxCls)
+                KxCls c;
+                std::memset(&c, 0, sizeof c);
+                c.m = f.m;
+                c.satsh = f.satsh;
+                c.cc = f.cc;
+                uint4 &cm = xcls[kx0 + x];
+                if (j.flags & KXF_INFEASIBLE) {
+                    cm.x |= 1u << k;
+                } else if (sat != KXF_SAT_MASK) {
+                    const bool p2 = f.rDl == 0.0, s0 = f.S == 0.0;
+                    // blocks < sat <=> w <= (sat - 1) * ipb
+                    const uint64_t ws = (uint64_t)(sat - 1) * dv + 1;
+                    uint32_t &kw = kwsat[I.k_base + k];
+                    kw = (uint32_t)std::max<uint64_t>(kw, std::min<uint64_t>(ws, 1ull << 30));
+                    xcost[x] += 5.0 + (p2 ? (s0 ? 4.0 : 6.0) : (s0 ? 6.0 : 8.0));
+                    if (p2) {
+                        c.c[0] = f.E * f.rDh;   // exact: rDh = 2^-k, E normal (fast_const_ok)
+                        c.c[1] = f.S * f.rDh;
+                        (s0 ? cm.y : cm.z) |= 1u << k;
+                    } else {
+                        c.c[0] = f.rDh;
+                        c.c[1] = f.rDl;
+                        c.c[2] = f.E;
+                        c.c[3] = f.S;
+                        if (s0) cm.w |= 1u << k;
+                    }
+                }
+                kc.push_back(c);
             }
+        // phase-C units in descending estimated cost (longest first: the
+        // CTA's warps finish together)
+        {
+            std::vector<uint32_t> ord(S.n_xforms);
+            for (uint32_t x = 0; x < S.n_xforms; x++) ord[x] = x;
+            std::stable_sort(ord.begin(), ord.end(),
+                             [&](uint32_t a, uint32_t b) { return xcost[a] > xcost[b]; });
+            for (uint32_t x = 0; x < S.n_xforms; x++) xord[kx0 + x] = ord[x];
+        }
     }
 
     // ---- small-grid table: t(kernel, xform, blocks) for blocks < sat32 ----
@@ -517,6 +612,10 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {kf.data(), kf.size() * sizeof(KxFast), 0},
         {small.data(), small.size() * sizeof(double), 0},
         {xinf.data(), xinf.size() * sizeof(uint32_t), 0},
+        {kc.data(), kc.size() * sizeof(KxCls), 0},
+        {xcls.data(), xcls.size() * sizeof(uint4), 0},
+        {kwsat.data(), kwsat.size() * sizeof(uint32_t), 0},
+        {xord.data(), xord.size() * sizeof(uint32_t), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -578,16 +677,27 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.kx_f = (const KxFast *)(base + parts[11].off);
     D.small_t = (const double *)(base + parts[12].off);
     D.xinf = (const uint32_t *)(base + parts[13].off);
+    D.kx_c = (const KxCls *)(base + parts[14].off);
+    D.xcls = (const uint4 *)(base + parts[15].off);
+    D.kern_wsat = (const uint32_t *)(base + parts[16].off);
+    D.xorder = (const uint32_t *)(base + parts[17].off);
     D.small_stride = small_stride;
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;
     D.freq = gpu->freq_hz;
     D.rfreq = 1.0 / gpu->freq_hz;
+    split_recip(gpu->freq_hz, D.rfh, D.rfl);
     D.invalid_counter = sp->invalid_counter;
     sp->dev_copy = (SpaceDev *)(ctr + 256);
     if ((e = cudaMemcpy(sp->dev_copy, &D, sizeof D, cudaMemcpyHostToDevice)) != cudaSuccess)
         return bail(e, "cudaMemcpy(space header)");
     sp->grid_best = nsm;
+    sp->usage_tbl_bytes = 0;
+    for (uint32_t q = 0; q < n_skels; q++)
+        if (info[q].polyf_base != POLY32_NONE)
+            sp->usage_tbl_bytes = std::max<uint32_t>(
+                sp->usage_tbl_bytes,
+                (uint32_t)(2 * ((skels[q].n_arrays + POLYF_AU - 1) / POLYF_AU) * POLYF_AU * POLY_CLASSES * 16));
     sp->max_kernels = 1;
     for (uint32_t q = 0; q < n_skels; q++)
         sp->max_kernels = std::max(sp->max_kernels, skels[q].n_kernels);
