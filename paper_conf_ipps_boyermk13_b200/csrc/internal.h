@@ -57,10 +57,14 @@ inline uint32_t kxf_sat(const KxFast &f) { return f.satsh & KXF_SAT_MASK; }
 // (b / D = b 2^-k is exact when D = 2^k, and E 2^-k, S 2^-k are exact scalings,
 // so RN(E rep) = RN(b E'); S = 0 makes RN(S rep) = +0.0, which adds nothing.)
 // m / satsh / cc as in KxFast.
-enum : uint32_t { KXC_P2S0 = 0u, KXC_P2S = 1u, KXC_NS0 = 2u, KXC_NS = 3u };
-struct __align__(16) KxCls {
-    uint32_t m, satsh;
+// A transformation's program (sweep kernel): its feasible kernels' entries in
+// summation order (per-iteration kernels, then run-once ones, each ascending;
+// infeasible kernels are left out: their sum is +inf through xinf).
+enum : uint32_t { KXC_P2S0 = 0u, KXC_P2S = 1u, KXC_NS0 = 2u, KXC_NS = 3u, KXC_NONE = 4u };
+struct __align__(16) KxProg {
+    uint32_t m, satsh;      // as KxFast
     uint64_t cc;
+    uint32_t k, cls, pad0, pad1;
     double c[4];
 };
 
@@ -165,10 +169,11 @@ struct SpaceDev {
     const KxJ *kx_j;
     const KxG *kx_g;
     const KxFast *kx_f;
-    const KxCls *kx_c;          // class-specialised saturated constants (sweep kernel)
-    // per (skeleton, xform) at kx_base + x: kernel bit masks {infeasible,
-    // P2S0, P2S, NS0} (a feasible kernel in none of the three is NS)
-    const uint4 *xcls;
+    // sweep kernel: per (skeleton, unit u) at kx_base + u (units in
+    // descending estimated cost) {x, first program entry, n_iter | n_once <<
+    // 16, xinf bits}; the programs' entries
+    const uint4 *xhdr;
+    const KxProg *xprog;
     const unsigned long long *poly;   // usage byte polynomials (all skeletons)
     // small-grid kernel times: small_t[kxi * small_stride + blocks] for
     // blocks < sat32 when sat32 <= small_stride (space.cpp small_grid_time)
@@ -178,10 +183,8 @@ struct SpaceDev {
     const uint32_t *xinf;
     // sweep kernel: per (skeleton, kernel) at k_base + k, the smallest work
     // count w for which every transformation's grid is saturated (blocks >=
-    // sat for all x); per (skeleton, unit u) at kx_base + u, the
-    // transformation of phase-C unit u (descending estimated cost)
+    // sat for all x)
     const uint32_t *kern_wsat;
-    const uint32_t *xorder;
     uint32_t small_stride;
     uint32_t n_skels;
     uint32_t n_sm;

@@ -1516,7 +1516,6 @@ __device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, 
 {
     issue_copy(P, ws.rec, &ws.mbar, tb, ng);
 }
-
 // One canonical tile: CTILE records from tb where every group of CX
 // consecutive records (lane l: records tb + CX l ...) is one design point
 // (same skeleton, nx, ny, iters; xform = position in the group, the layout
@@ -1912,6 +1911,9 @@ constexpr unsigned long long SW_TILE = (unsigned long long)SW_GROUPS * CX;   // 
 constexpr int NCH = GROPHECY_NCH;                                   // chains per lane (divides WARPS)
 constexpr int SW_UNITS = CX * (WARPS / NCH);                        // phase-C units (x, chain block)
 constexpr uint32_t SW_BAD = 0xffffffffu;
+#ifndef GROPHECY_SMINB
+#define GROPHECY_SMINB 2
+#endif
 
 struct alignas(128) SweepSmem {
     alignas(128) uint32_t rec[WARPS][4][CTILE];   // per warp: its warp tile (TMA bulk copies)
@@ -2029,7 +2031,7 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
 }
 
 // Saturated kernel times of NCH records of one (kernel, x) pair of class C
-// (internal.h KxCls) from their block counts; t = cyc / freq by the
+// (internal.h KxProg) from their block counts; t = cyc / freq by the
 // two-product division.
 template <uint32_t C>
 __device__ __forceinline__ void cls_times(const double2 c01, const double2 c23, const uint32_t (&blocks)[NCH],
@@ -2052,24 +2054,8 @@ __device__ __forceinline__ void cls_times(const double2 c01, const double2 c23, 
     }
 }
 
-// One (kernel, transformation) record of KxCls loaded whole (the next
-// kernel's is loaded while the current one is modelled).
-struct KC {
-    uint4 hd;
-    double2 c01, c23;
-};
-__device__ __forceinline__ KC load_kc(const KxCls *cp)
-{
-    const uint4 *q = reinterpret_cast<const uint4 *>(cp);
-    KC r;
-    r.hd = __ldg(q);
-    r.c01 = __ldg(reinterpret_cast<const double2 *>(q + 1));
-    r.c23 = __ldg(reinterpret_cast<const double2 *>(q + 2));
-    return r;
-}
-
 template <bool BEST>
-__global__ void __launch_bounds__(THREADS, 2) sweep_kernel(const Params P)
+__global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Params P)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SweepSmem &sm = *reinterpret_cast<SweepSmem *>(smem_raw);
@@ -2118,7 +2104,8 @@ __global__ void __launch_bounds__(THREADS, 2) sweep_kernel(const Params P)
         uint32_t s0, n0, m0, i0;
         bool ok = sweep_phase_a(S, sm.rec[warp], lane, s0, n0, m0, i0);
         const uint32_t skel = s0 >> 16;
-        if (tid == 0) {
+        if (lane == 0) mbar_init(&sm.mbar[warp], 1);
+    if (tid == 0) {
             // warp 0's skeleton decides the tile's usage table: stage it in
             // shared memory when it changes (every reader of the previous one
             // passed the previous tile's barriers)
@@ -2141,7 +2128,8 @@ __global__ void __launch_bounds__(THREADS, 2) sweep_kernel(const Params P)
             }
         }
         __syncthreads();   // the previous tile's phase C is done with the per-design-point arrays
-        if (tid == 0) {
+        if (lane == 0) mbar_init(&sm.mbar[warp], 1);
+    if (tid == 0) {
             sm.next_tile = atomicAdd(claim, 1u) + gridDim.x;
             sm.unit = 0;
         }
@@ -2218,9 +2206,11 @@ __global__ void __launch_bounds__(THREADS, 2) sweep_kernel(const Params P)
             if (lane == 0) u = atomicAdd(&sm.unit, 1u);
             u = __shfl_sync(FULL, u, 0);
             if (u >= (unsigned)SW_UNITS) break;
-            const uint32_t x = __ldg(&S.xorder[I.kx_base + u % CX]), jb = u / CX;
-            const uint4 cm = __ldg(&S.xcls[I.kx_base + x]);
-            const uint32_t xf = __ldg(&S.xinf[I.kx_base + x]);
+            // the unit's transformation and its program (header in unit order)
+            const uint4 hdr = __ldg(&S.xhdr[I.kx_base + u % CX]);
+            const uint32_t x = hdr.x, jb = u / CX, xf = hdr.w;
+            const KxProg *pe = S.xprog + hdr.y;
+            const uint32_t n_it = hdr.z & 0xffffu, n_all = n_it + (hdr.z >> 16);
             // kernels whose grid may be unsaturated for one of the warp's design points
             uint32_t gk = 0;
 #pragma unroll
@@ -2229,11 +2219,14 @@ __global__ void __launch_bounds__(THREADS, 2) sweep_kernel(const Params P)
             double ti[NCH], to[NCH];
 #pragma unroll
             for (int j = 0; j < NCH; j++) ti[j] = to[j] = 0.0;
-            const KxCls *cbase = S.kx_c + I.kx_base + x;
-            auto one_kernel = [&](uint32_t k, double (&acc)[NCH]) {
-                const KC kc = load_kc(cbase + k * X);
-                const uint32_t sat = kc.hd.y & KXF_SAT_MASK, sh = kc.hd.y >> KXF_SAT_BITS;
-                const unsigned long long cc = ((unsigned long long)kc.hd.w << 32) | kc.hd.z;
+            auto one_kernel = [&](const KxProg *e, double (&acc)[NCH]) {
+                const uint4 *q = reinterpret_cast<const uint4 *>(e);
+                const uint4 hd = __ldg(q), kk = __ldg(q + 1);
+                const double2 c01 = __ldg(reinterpret_cast<const double2 *>(q + 2));
+                const double2 c23 = __ldg(reinterpret_cast<const double2 *>(q + 3));
+                const uint32_t k = kk.x, cls = kk.y;
+                const uint32_t sat = hd.y & KXF_SAT_MASK, sh = hd.y >> KXF_SAT_BITS;
+                const unsigned long long cc = ((unsigned long long)hd.w << 32) | hd.z;
                 uint32_t blocks[NCH];
 #pragma unroll
                 for (int j = 0; j < NCH; j += 4) {
@@ -2242,15 +2235,14 @@ __global__ void __launch_bounds__(THREADS, 2) sweep_kernel(const Params P)
                     const uint32_t w[4] = {w4.x, w4.y, w4.z, w4.w};
 #pragma unroll
                     for (int q = 0; q < 4; q++)
-                        blocks[j + q] = (uint32_t)(((unsigned long long)w[q] * kc.hd.x + cc) >> 32) >> sh;
+                        blocks[j + q] = (uint32_t)(((unsigned long long)w[q] * hd.x + cc) >> 32) >> sh;
                 }
                 double tk[NCH];
-                const uint32_t bit = 1u << k;
-                if (cm.y & bit) cls_times<KXC_P2S0>(kc.c01, kc.c23, blocks, rfh, rfl, tk);
-                else if (cm.z & bit) cls_times<KXC_P2S>(kc.c01, kc.c23, blocks, rfh, rfl, tk);
-                else if (cm.w & bit) cls_times<KXC_NS0>(kc.c01, kc.c23, blocks, rfh, rfl, tk);
-                else cls_times<KXC_NS>(kc.c01, kc.c23, blocks, rfh, rfl, tk);
-                if (gk & bit) {
+                if (cls == KXC_P2S0) cls_times<KXC_P2S0>(c01, c23, blocks, rfh, rfl, tk);
+                else if (cls == KXC_P2S) cls_times<KXC_P2S>(c01, c23, blocks, rfh, rfl, tk);
+                else if (cls == KXC_NS0) cls_times<KXC_NS0>(c01, c23, blocks, rfh, rfl, tk);
+                else cls_times<KXC_NS>(c01, c23, blocks, rfh, rfl, tk);
+                if ((gk >> k) & 1u) {
                     // off the saturated path: the small-grid table (SKF_TABULATED)
                     bool any = false;
 #pragma unroll
@@ -2265,14 +2257,14 @@ __global__ void __launch_bounds__(THREADS, 2) sweep_kernel(const Params P)
 #pragma unroll
                 for (int j = 0; j < NCH; j++) acc[j] = __dadd_rn(acc[j], tk[j]);
             };
-            // sums in ascending kernel order (N6); infeasible kernels skipped:
-            // their sum is +inf (xinf), whatever the others add
+            // sums in ascending kernel order (N6): the program lists the
+            // per-iteration kernels, then the run-once ones; infeasible
+            // kernels are not listed (their sum is +inf through xinf)
+            uint32_t e = 0;
 #pragma unroll 1
-            for (uint32_t mask = pim & kmask & ~cm.x; mask; mask &= mask - 1u)
-                one_kernel((uint32_t)__ffs(mask) - 1u, ti);
+            for (; e < n_it; e++) one_kernel(pe + e, ti);
 #pragma unroll 1
-            for (uint32_t mask = ~pim & kmask & ~cm.x; mask; mask &= mask - 1u)
-                one_kernel((uint32_t)__ffs(mask) - 1u, to);
+            for (; e < n_all; e++) one_kernel(pe + e, to);
             const double inf = __longlong_as_double(0x7ff0000000000000LL);
             if (xf & XINF_ITER) {
 #pragma unroll

@@ -336,10 +336,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxJ> kj;
     std::vector<KxG> kg;
     std::vector<KxFast> kf;
-    std::vector<KxCls> kc;
-    std::vector<uint4> xcls;      // per (skeleton, xform) at kx_base + x: class masks
+    std::vector<KxProg> kprog;    // sweep-kernel programs (all skeletons)
+    std::vector<uint4> xhdr;      // per (skeleton, unit) at kx_base + u: program header
     std::vector<uint32_t> kwsat;  // per (skeleton, kernel): work count saturating every xform
-    std::vector<uint32_t> xord;   // per (skeleton, unit) at kx_base + u: phase-C order
     std::vector<uint32_t> xinf;   // per (skeleton, xform) at kx_base + x: XINF_* bits
     // the fast path divides by freq with the two-product method: without it
     // (a frequency whose odd significand is >= 2^50) every pair takes the
@@ -483,10 +482,10 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         }
         const size_t kx0 = kf.size();   // this skeleton's kx_base
         kwsat.resize(kwork.size(), 0u);
-        xord.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, 0u);
         std::vector<double> xcost(S.n_xforms, 0.0);
         xinf.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, 0u);
-        xcls.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, make_uint4(0u, 0u, 0u, 0u));
+        xhdr.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, make_uint4(0u, 0u, 0u, 0u));
+        std::vector<KxProg> pair_prog((size_t)S.n_kernels * S.n_xforms);
         for (uint32_t k = 0; k < S.n_kernels; k++)
             for (uint32_t x = 0; x < S.n_xforms; x++) {
                 KxES es; KxD d; KxI i; KxJ j; KxG g;
@@ -533,16 +532,15 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 }
                 f.satsh = sat | sh << KXF_SAT_BITS;
                 kf.push_back(f);
-                // the sweep kernel's class record (internal.h KxCls)
-                KxCls c;
+                // the sweep kernel's program entry (internal.h KxProg)
+                KxProg c;
                 std::memset(&c, 0, sizeof c);
                 c.m = f.m;
                 c.satsh = f.satsh;
                 c.cc = f.cc;
-                uint4 &cm = xcls[kx0 + x];
-                if (j.flags & KXF_INFEASIBLE) {
-                    cm.x |= 1u << k;
-                } else if (sat != KXF_SAT_MASK) {
+                c.k = k;
+                c.cls = KXC_NONE;
+                if (!(j.flags & KXF_INFEASIBLE) && sat != KXF_SAT_MASK) {
                     const bool p2 = f.rDl == 0.0, s0 = f.S == 0.0;
                     // blocks < sat <=> w <= (sat - 1) * ipb
                     const uint64_t ws = (uint64_t)(sat - 1) * dv + 1;
@@ -552,16 +550,16 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                     if (p2) {
                         c.c[0] = f.E * f.rDh;   // exact: rDh = 2^-k, E normal (fast_const_ok)
                         c.c[1] = f.S * f.rDh;
-                        (s0 ? cm.y : cm.z) |= 1u << k;
+                        c.cls = s0 ? KXC_P2S0 : KXC_P2S;
                     } else {
                         c.c[0] = f.rDh;
                         c.c[1] = f.rDl;
                         c.c[2] = f.E;
                         c.c[3] = f.S;
-                        if (s0) cm.w |= 1u << k;
+                        c.cls = s0 ? KXC_NS0 : KXC_NS;
                     }
                 }
-                kc.push_back(c);
+                pair_prog[(size_t)x * S.n_kernels + k] = c;
             }
         // phase-C units in descending estimated cost (longest first: the
         // CTA's warps finish together)
@@ -570,7 +568,23 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             for (uint32_t x = 0; x < S.n_xforms; x++) ord[x] = x;
             std::stable_sort(ord.begin(), ord.end(),
                              [&](uint32_t a, uint32_t b) { return xcost[a] > xcost[b]; });
-            for (uint32_t x = 0; x < S.n_xforms; x++) xord[kx0 + x] = ord[x];
+            // per unit: the header and the program of its transformation
+            // (feasible saturated-capable kernels, per-iteration ones then
+            // run-once ones, each in ascending kernel order: N6)
+            for (uint32_t u = 0; u < S.n_xforms; u++) {
+                const uint32_t x = ord[u];
+                const uint32_t first = (uint32_t)kprog.size();
+                uint32_t n_it = 0, n_on = 0;
+                for (int pass = 0; pass < 2; pass++)
+                    for (uint32_t k = 0; k < S.n_kernels; k++) {
+                        const bool per = (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) != 0;
+                        const KxProg &e = pair_prog[(size_t)x * S.n_kernels + k];
+                        if (per != (pass == 0) || e.cls == KXC_NONE) continue;
+                        kprog.push_back(e);
+                        (pass == 0 ? n_it : n_on)++;
+                    }
+                xhdr[kx0 + u] = make_uint4(x, first, n_it | n_on << 16, xinf[kx0 + x]);
+            }
         }
     }
 
@@ -612,10 +626,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {kf.data(), kf.size() * sizeof(KxFast), 0},
         {small.data(), small.size() * sizeof(double), 0},
         {xinf.data(), xinf.size() * sizeof(uint32_t), 0},
-        {kc.data(), kc.size() * sizeof(KxCls), 0},
-        {xcls.data(), xcls.size() * sizeof(uint4), 0},
+        {kprog.data(), kprog.size() * sizeof(KxProg), 0},
+        {xhdr.data(), xhdr.size() * sizeof(uint4), 0},
         {kwsat.data(), kwsat.size() * sizeof(uint32_t), 0},
-        {xord.data(), xord.size() * sizeof(uint32_t), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -677,10 +690,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.kx_f = (const KxFast *)(base + parts[11].off);
     D.small_t = (const double *)(base + parts[12].off);
     D.xinf = (const uint32_t *)(base + parts[13].off);
-    D.kx_c = (const KxCls *)(base + parts[14].off);
-    D.xcls = (const uint4 *)(base + parts[15].off);
+    D.xprog = (const KxProg *)(base + parts[14].off);
+    D.xhdr = (const uint4 *)(base + parts[15].off);
     D.kern_wsat = (const uint32_t *)(base + parts[16].off);
-    D.xorder = (const uint32_t *)(base + parts[17].off);
     D.small_stride = small_stride;
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;
