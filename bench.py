@@ -6,11 +6,13 @@
 
 Workload (BASELINE.json configs[3], the one the metric is quoted on): the full
 design-space sweep of 10^9 candidates (16 skeletons x 16 transformations x
-problem sizes), sharded contiguously over the ranks (strong scaling); the
-global best is a min-loc over ranks (16-byte-class all-gather over NCCL +
-the library's combine kernel).  One step = one fused projection + argmin
-launch over the rank's shard (inputs resident in HBM), the cross-rank
-min-loc, and the 48-byte result read back to the host.
+problem sizes), sharded over the ranks (strong scaling) as back-to-back
+stripes + a contiguous tail per rank (dist.stripe_layout); the global best is
+a min-loc over ranks (grophecy_best_allreduce_result: the library's NCCL
+all-gather of 48-byte results + combine kernel).  One step = the fused
+projection + argmin launches over the rank's share (inputs resident in HBM;
+two launch pairs at N > 1, one at N = 1, whatever --stripes is), the
+cross-rank min-loc, and the 48-byte result read back to the host.
 
 Rank 0 prints ONE JSON line.  See DESIGN.md §6 for every field.
 """
@@ -43,7 +45,7 @@ def parse():
     p.add_argument("--config", default="c4")
     p.add_argument("--n", type=int, default=None, help="override candidate count")
     p.add_argument("--stripes", type=int, default=16,
-                   help="chunks per rank when N > 1 (strided over the workload)")
+                   help="stripes per rank when N > 1 (strided over the workload, one launch)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -225,30 +227,40 @@ def main():
     if args.n:
         cfg = R.with_n(cfg, args.n)
     N = cfg["n"]
-    # N > 1: the rank's shard is `stripes` tile-aligned chunks strided over
-    # the workload (chunk r + P k), so every rank gets the same skeleton mix
-    # (per-skeleton costs differ 4x; contiguous shards would leave the ranks
-    # with cheap skeletons idle).  N = 1: one contiguous launch.
-    chunks = D.striped_chunks(N, rank, world, args.stripes if world > 1 else 1)
-    lo = chunks[0][0]
-    n_local = sum(b - a for a, b in chunks)
+    # N > 1: the rank's share is `stripes` sweep-tile-aligned stripes strided
+    # over the workload, stored back to back and projected by ONE launch with
+    # grophecy_batch's stripe map (every rank gets the same skeleton mix:
+    # per-skeleton costs differ 4x), plus a contiguous piece of the remainder
+    # (dist.stripe_layout).  N = 1: one contiguous launch.
+    if world > 1:
+        L, n_main, (t_lo, t_hi) = D.stripe_layout(N, rank, world, args.stripes)
+    else:
+        L, n_main, (t_lo, t_hi) = 0, 0, (0, N)
+    n_tail = t_hi - t_lo
+    n_local = n_main + n_tail
     pc = G.pcie(G.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL))
     space = G.Space(cfg["skeletons"], S.FX5600)
     stream = torch.cuda.current_stream()
     rec = G.Records.empty(n_local)                   # shard generated in its own HBM
-    batches, off = [], 0
-    for a, b in chunks:
-        part = G.Records(rec.skx[off:off + b - a], rec.nx[off:off + b - a],
-                         rec.ny[off:off + b - a], rec.iters[off:off + b - a])
-        G.synth_records(cfg, a, b - a, out=part)
-        batches.append(part.batch(index_base=a))
-        off += b - a
-    minloc = D.MinLoc(world, backend=backend)
+    for k in range(n_main // L if L else 0):
+        part = G.Records(*[t[k * L:(k + 1) * L] for t in (rec.skx, rec.nx, rec.ny, rec.iters)])
+        G.synth_records(cfg, rank * L + k * world * L, L, out=part)
+    if n_tail:
+        part = G.Records(*[t[n_main:] for t in (rec.skx, rec.nx, rec.ny, rec.iters)])
+        G.synth_records(cfg, t_lo, n_tail, out=part)
+    batches = []
+    if n_main:
+        batches.append(rec.batch(index_base=rank * L, start=0, stop=n_main, stripe_len=L,
+                                 stripe_stride=world * L))
+    if n_tail or not batches:
+        batches.append(rec.batch(index_base=t_lo, start=n_main, stop=n_local))
+    minloc = D.MinLoc(world, backend=backend, space=space)
     host_res = torch.empty(6, dtype=torch.int64, pin_memory=True)
     torch.cuda.synchronize()
 
     ev_k = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
             for _ in range(args.steps)]
+    last = {}
 
     def step(i=None):
         if i is not None:
@@ -257,8 +269,11 @@ def main():
             space.best_async(pc, batch, minloc.local, accumulate=k > 0)
         if i is not None:
             ev_k[i][1].record(stream)
-        minloc.combine()                              # all-gather + combine kernel (N>1)
-        host_res.copy_(minloc.result, non_blocking=True)
+        if minloc.comm is not None:                   # library NCCL min-loc (N > 1)
+            last["r"] = minloc.allreduce()
+        else:
+            minloc.combine()                          # gloo fallback / N = 1
+            host_res.copy_(minloc.result, non_blocking=True)
 
     for _ in range(max(3, args.warmup)):
         step()
@@ -291,13 +306,12 @@ def main():
     if world > 1:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
     ms_max, kern_avg_max = float(ms_t[0]), float(ms_t[1])
-    best = G.result_from_tensor(host_res)
+    best = last["r"] if "r" in last else G.result_from_tensor(host_res)
 
     # ---- end-to-end: host records through the public C-ABI call ----
     e2e = None
     if not args.no_e2e:
-        e2e = run_e2e(G, torch, dist, space, pc, rec, lo, chunks[0][1] - chunks[0][0], N, world,
-                      args, minloc)   # the first chunk (contiguous host records)
+        e2e = run_e2e(G, torch, dist, space, pc, rec, batches, n_local, world, args, minloc)
     if world > 1:
         dist.barrier()
     if rank != 0:
@@ -371,10 +385,12 @@ def main():
         dist.destroy_process_group()
 
 
-def run_e2e(G, torch, dist, space, pc, rec, lo, n_local, N, world, args, minloc):
-    """Same metric through grophecy_best_host: pinned host records, chunked
-    H2D copies inside the timed region, 48-byte result D2H; with N > 1 ranks
-    the global min-loc of the ranks' results (all-gather + combine) per step."""
+def run_e2e(G, torch, dist, space, pc, rec, batches, n_local, world, args, minloc):
+    """Same metric through grophecy_best_host: each rank's whole share (the
+    same batches as the device-resident timing, stripe map included) in
+    pinned host memory, chunked H2D copies inside the timed region, 48-byte
+    result per batch back to the host; with N > 1 the global min-loc over the
+    ranks (grophecy_best_allreduce_result) every step."""
     avail = 0
     try:
         for ln in open("/proc/meminfo"):
@@ -382,46 +398,56 @@ def run_e2e(G, torch, dist, space, pc, rec, lo, n_local, N, world, args, minloc)
                 avail = int(ln.split()[1]) * 1024
     except Exception:
         pass
-    budget = avail // (3 * max(1, world))
-    n_e2e = min(n_local, max(1 << 20, budget // 16))
+    if 16 * n_local * world > avail // 2:
+        return {"skipped": f"host memory: {avail >> 30} GiB available < 2 x {16 * n_local * world >> 30} GiB of pinned records"}
     host = {}
     for k, t in zip(("skx", "nx", "ny", "iters"), (rec.skx, rec.nx, rec.ny, rec.iters)):
-        h = torch.empty(n_e2e, dtype=torch.int32, pin_memory=True)
-        h.copy_(t[:n_e2e])
+        h = torch.empty(n_local, dtype=torch.int32, pin_memory=True)
+        h.copy_(t[:n_local])
         host[k] = h
     torch.cuda.synchronize()
     steps = max(1, min(args.steps, 5))
-    space.best_host(pc, host, index_base=lo)
+    hb = []
+    off = 0
+    for b in batches:
+        hb.append(({k: v[off:off + b.n] for k, v in host.items()}, b.index_base, b.stripe_len,
+                   b.stripe_stride))
+        off += b.n
+    dres = torch.empty(6, dtype=torch.int64, device="cuda")
+
+    def one():
+        res = [space.best_host(pc, h, index_base=ib, stripe_len=sl, stripe_stride=ss)[1]
+               for h, ib, sl, ss in hb]
+        r = G.best_combine_host(res)
+        if world > 1:   # global best over the ranks' shares
+            if minloc.comm is not None:
+                dres.copy_(torch.frombuffer(bytearray(bytes(r)), dtype=torch.int64))
+                r = minloc.space.allreduce_result(dres, minloc.comm)[1]
+            else:
+                from paper_conf_ipps_boyermk13_b200 import dist as D
+                r = D.minloc_host(r)
+        return r
+
+    one()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    res_h = torch.empty(6, dtype=torch.int64, pin_memory=True)
-
-    def one():
-        rc, r = space.best_host(pc, host, index_base=lo)
-        if world > 1:   # global best over the ranks' shards
-            res_h.copy_(torch.frombuffer(bytearray(bytes(r)), dtype=torch.int64))
-            minloc.local.copy_(res_h, non_blocking=True)
-            minloc.combine()
-            res_h.copy_(minloc.result)
-        return r
-
     t0 = time.perf_counter()
     for _ in range(steps):
-        one()
+        r = one()
     dt = time.perf_counter() - t0
     dt_t = torch.tensor([dt], dtype=torch.float64,
                         device="cuda" if dist.is_initialized() and dist.get_backend() == "nccl" else "cpu")
     if world > 1:
         dist.all_reduce(dt_t, op=dist.ReduceOp.MAX)
     dt = float(dt_t[0])
-    total = n_e2e * world * steps
-    return {"value": total / dt, "unit": UNIT, "h2d_bytes_per_step": 16 * n_e2e * world,
-            "d2h_bytes_per_step": 48 * world, "steps": steps,
-            "records_per_gpu": n_e2e,
-            "path": "grophecy_best_host (pinned host SoA records -> chunked cudaMemcpyAsync "
-                    "overlapped with the fused kernel -> 48 B result; N > 1: all-gather + "
-                    "combine of the ranks' results)",
+    total = n_local * world * steps
+    return {"value": total / dt, "unit": UNIT, "h2d_bytes_per_step": 16 * n_local * world,
+            "d2h_bytes_per_step": 48 * len(batches) * world, "steps": steps,
+            "records_per_gpu": n_local, "best_index": r.index,
+            "path": "grophecy_best_host per batch (pinned host SoA records -> chunked cudaMemcpyAsync "
+                    "overlapped with the fused kernel -> 48 B result) + host combine; N > 1: "
+                    "grophecy_best_allreduce_result over the ranks",
             "timer": "host wall clock, max over ranks"}
 
 

@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define GROPHECY_ABI_VERSION 3
+#define GROPHECY_ABI_VERSION 4
 
 typedef enum {
     GROPHECY_OK = 0,
@@ -194,12 +194,19 @@ void grophecy_space_destroy(grophecy_space *space);
 
 /* Struct-of-arrays candidate records, DEVICE pointers, length n, 16-byte
  * aligned.  skx = (skeleton << 16) | transformation.  Global index of
- * record i is index_base + i (used for tie-breaking and reported by best).
+ * record i (used for tie-breaking and reported by best): index_base + i when
+ * stripe_len == 0; otherwise the batch is a rank's stripes of a larger
+ * workload stored back to back and record i is
+ *   index_base + (i / stripe_len) * stripe_stride + i % stripe_len
+ * (stripe_stride >= stripe_len, else EINVAL; an increasing map, so ties still
+ * resolve to the lowest global index).  The map only changes reported
+ * indices: eval outputs stay positional, group_best rejects striped batches.
  * A record is valid iff skeleton < n_skels, transformation < that
  * skeleton's n_xforms, 1 <= nx, ny <= 2^20 and iters >= 1. */
 typedef struct {
     const uint32_t *skx, *nx, *ny, *iters;
     uint64_t n, index_base;
+    uint64_t stripe_len, stripe_stride;   /* 0, 0: contiguous */
 } grophecy_batch;
 
 /* Project every candidate.  Outputs are DEVICE arrays of length n owned by
@@ -272,6 +279,13 @@ int grophecy_best_combine_host(const grophecy_best_result *in, uint32_t count,
 int grophecy_best_allreduce(grophecy_space *space, const grophecy_pcie *pcie,
                             const grophecy_batch *batch, void *nccl_comm,
                             grophecy_best_result *host_out, void *cuda_stream);
+/* The same min-loc for a result already in DEVICE memory (e.g. accumulated
+ * by several grophecy_best_async launches over a rank's batches): NCCL
+ * all-gather of the ranks' device_in on cuda_stream, combine, global best to
+ * host_out on every rank.  Synchronises the stream; errors as above. */
+int grophecy_best_allreduce_result(grophecy_space *space, const grophecy_best_result *device_in,
+                                   void *nccl_comm, grophecy_best_result *host_out,
+                                   void *cuda_stream);
 /* Communicator helpers (same run-time NCCL): a 128-byte ncclUniqueId for rank
  * 0 to broadcast; ncclCommInitRank on `device` (comm_out: ncclComm_t);
  * ncclCommDestroy. */
@@ -338,14 +352,14 @@ double grophecy_speedup(double t_cpu_s, double t_gpu_s);
  * it to predicted vs measured speedups).  Pure host functions. */
 double grophecy_error_magnitude(double predicted, double measured);
 
-/* End-to-end entry point with HOST record arrays (pinned for full speed):
- * streams the records to the device in chunks, overlapping copies with the
- * fused projection + argmin, and returns the result in host memory.
- * Synchronous.  Same status rules as grophecy_best. */
+/* End-to-end entry point: host_batch's record arrays are HOST memory
+ * (pinned for full speed; index_base / stripes as in grophecy_batch).  The
+ * records stream to the device in chunks, copies overlapped with the fused
+ * projection + argmin, and the result returns in host memory.  Synchronous.
+ * Same status rules as grophecy_best. */
 int grophecy_best_host(grophecy_space *space, const grophecy_pcie *pcie,
-                       const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
-                       const uint32_t *iters, uint64_t n, uint64_t index_base,
-                       grophecy_best_result *host_out, void *cuda_stream);
+                       const grophecy_batch *host_batch, grophecy_best_result *host_out,
+                       void *cuda_stream);
 
 /* ---------------------------------------------------------------------- */
 /* PCIe calibration / validation subsystem      */

@@ -229,6 +229,10 @@ extern "C" int grophecy_group_best(grophecy_space *s, const grophecy_pcie *pc,
         return GROPHECY_EINVAL;
     }
     *n_groups = 0;
+    if (b->stripe_len) {
+        set_error("grophecy_group_best: striped batches are not supported (groups need contiguous indices)");
+        return GROPHECY_EINVAL;
+    }
     if (b->n == 0) return GROPHECY_OK;
     DeviceGuard guard(s->device);
     cudaStream_t st = (cudaStream_t)stream;

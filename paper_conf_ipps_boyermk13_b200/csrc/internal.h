@@ -263,6 +263,8 @@ bool compile_plan(const grophecy_skeleton_desc &S, SkelPlanHost &out);
 void set_error(const std::string &msg);
 int cuda_fail(cudaError_t e, const char *what);
 void count_launch(uint64_t n = 1);
+// local_off: for a striped batch, the batch-local index of its record 0
+// (chunked host batches)
 int launch_best(grophecy_space *s, const grophecy_pcie *pcie, const grophecy_batch *b,
-                grophecy_best_result *dout, int accumulate, cudaStream_t st);
+                grophecy_best_result *dout, int accumulate, cudaStream_t st, uint64_t local_off = 0);
 }  // namespace grophecy

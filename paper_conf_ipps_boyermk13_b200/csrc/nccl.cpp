@@ -123,23 +123,14 @@ int grophecy_nccl_comm_destroy(void *comm)
     return GROPHECY_OK;
 }
 
-int grophecy_best_allreduce(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
-                            void *nccl_comm, grophecy_best_result *host_out, void *stream)
+// All-gather of the ranks' device results + combine + D2H (every rank gets
+// the global best).  The shared tail of both allreduce entry points.
+static int allreduce_device(grophecy_space *s, const Nccl *n, const grophecy_best_result *local,
+                            void *nccl_comm, grophecy_best_result *host_out, cudaStream_t st)
 {
-    if (!s || !pc || !b || !nccl_comm || !host_out) {
-        set_error("grophecy_best_allreduce: null argument");
-        return GROPHECY_EINVAL;
-    }
-    const Nccl *n = nccl();
-    if (!n) {
-        set_error("NCCL (libnccl.so.2) not available");
-        return GROPHECY_ENCCL;
-    }
     int nranks = 0;
     int r = n->comm_count(nccl_comm, &nranks);
     if (r) return nccl_fail(n, r, "ncclCommCount");
-    DeviceGuard guard(s->device);
-    cudaStream_t st = (cudaStream_t)stream;
     cudaError_t e;
     const size_t need = sizeof(grophecy_best_result) * ((size_t)nranks + 1);
     if (s->mscratch_bytes < need) {   // gathered results + the combined one
@@ -149,14 +140,11 @@ int grophecy_best_allreduce(grophecy_space *s, const grophecy_pcie *pc, const gr
         if ((e = cudaMalloc(&s->mscratch, need)) != cudaSuccess) return cuda_fail(e, "cudaMalloc(minloc)");
         s->mscratch_bytes = need;
     }
-    grophecy_best_result *local = s->partials + (s->max_partials - 1);
     grophecy_best_result *gathered = (grophecy_best_result *)s->mscratch;
     grophecy_best_result *result = gathered + nranks;
-    int rc = launch_best(s, pc, b, local, 0, st);
-    if (rc) return rc;
     r = n->all_gather(local, gathered, sizeof(grophecy_best_result), NCCL_INT8, nccl_comm, st);
     if (r) return nccl_fail(n, r, "ncclAllGather");
-    rc = grophecy_best_combine(gathered, (uint32_t)nranks, result, stream);
+    int rc = grophecy_best_combine(gathered, (uint32_t)nranks, result, st);
     if (rc) return rc;
     e = cudaMemcpyAsync(host_out, result, sizeof *host_out, cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -170,6 +158,42 @@ int grophecy_best_allreduce(grophecy_space *s, const grophecy_pcie *pc, const gr
         return GROPHECY_EBADCAND;
     }
     return GROPHECY_OK;
+}
+
+int grophecy_best_allreduce(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
+                            void *nccl_comm, grophecy_best_result *host_out, void *stream)
+{
+    if (!s || !pc || !b || !nccl_comm || !host_out) {
+        set_error("grophecy_best_allreduce: null argument");
+        return GROPHECY_EINVAL;
+    }
+    const Nccl *n = nccl();
+    if (!n) {
+        set_error("NCCL (libnccl.so.2) not available");
+        return GROPHECY_ENCCL;
+    }
+    DeviceGuard guard(s->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    grophecy_best_result *local = s->partials + (s->max_partials - 1);
+    const int rc = launch_best(s, pc, b, local, 0, st);
+    if (rc) return rc;
+    return allreduce_device(s, n, local, nccl_comm, host_out, st);
+}
+
+int grophecy_best_allreduce_result(grophecy_space *s, const grophecy_best_result *device_in,
+                                   void *nccl_comm, grophecy_best_result *host_out, void *stream)
+{
+    if (!s || !device_in || !nccl_comm || !host_out) {
+        set_error("grophecy_best_allreduce_result: null argument");
+        return GROPHECY_EINVAL;
+    }
+    const Nccl *n = nccl();
+    if (!n) {
+        set_error("NCCL (libnccl.so.2) not available");
+        return GROPHECY_ENCCL;
+    }
+    DeviceGuard guard(s->device);
+    return allreduce_device(s, n, device_in, nccl_comm, host_out, (cudaStream_t)stream);
 }
 
 }  // extern "C"

@@ -1138,6 +1138,10 @@ struct Params {
     unsigned int *tile_count;
     uint32_t canon_warp_bytes; // pass 1: shared memory per warp (canon_warp_bytes(kmax))
     uint32_t sweep_kmax;       // sweep kernel: the space's largest kernel count (smem layout)
+    // striped batches (grophecy_batch.stripe_len != 0): kernels work with
+    // batch-local indices (base = the launch's local offset) and the final
+    // best index is mapped to map_base + (i / map_len) * map_stride + i % map_len
+    unsigned long long map_len, map_stride, map_base;
 };
 
 // Record validity (include/grophecy.h) and its usage key (skeleton, nx, ny).
@@ -1516,6 +1520,7 @@ __device__ __forceinline__ void issue_tile_copy(const Params &P, CanonSmem &ws, 
 {
     issue_copy(P, ws.rec, &ws.mbar, tb, ng);
 }
+
 // One canonical tile: CTILE records from tb where every group of CX
 // consecutive records (lane l: records tb + CX l ...) is one design point
 // (same skeleton, nx, ny, iters; xform = position in the group, the layout
@@ -1810,6 +1815,8 @@ __device__ __forceinline__ void finish_best(const Params &P, const unsigned long
         }
         b = warp_best(b);
         if (lane == 0) {
+            if (P.map_len && b.i != ~0ull)   // striped batch: local -> global index
+                b.i = P.map_base + (b.i / P.map_len) * P.map_stride + b.i % P.map_len;
             if (P.accumulate) {
                 Best prev = from_result(*P.out);
                 merge(prev, b);
@@ -2104,8 +2111,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         uint32_t s0, n0, m0, i0;
         bool ok = sweep_phase_a(S, sm.rec[warp], lane, s0, n0, m0, i0);
         const uint32_t skel = s0 >> 16;
-        if (lane == 0) mbar_init(&sm.mbar[warp], 1);
-    if (tid == 0) {
+        if (tid == 0) {
             // warp 0's skeleton decides the tile's usage table: stage it in
             // shared memory when it changes (every reader of the previous one
             // passed the previous tile's barriers)
@@ -2128,8 +2134,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             }
         }
         __syncthreads();   // the previous tile's phase C is done with the per-design-point arrays
-        if (lane == 0) mbar_init(&sm.mbar[warp], 1);
-    if (tid == 0) {
+        if (tid == 0) {
             sm.next_tile = atomicAdd(claim, 1u) + gridDim.x;
             sm.unit = 0;
         }
@@ -2486,6 +2491,10 @@ static int check_batch(const grophecy_space *s, const grophecy_pcie *pc, const g
         set_error("null record array");
         return GROPHECY_EINVAL;
     }
+    if (b->stripe_len && b->stripe_stride < b->stripe_len) {
+        set_error("stripe_stride < stripe_len");
+        return GROPHECY_EINVAL;
+    }
     return GROPHECY_OK;
 }
 
@@ -2504,6 +2513,10 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
     P.iters = b->iters;
     P.n = b->n;
     P.base = b->index_base;
+    P.map_len = b->stripe_len;
+    P.map_stride = b->stripe_stride;
+    P.map_base = b->index_base;
+    if (b->stripe_len) P.base = 0;   // batch-local indices (launch_best adds the local offset)
     P.h2d = nullptr;
     P.d2h = nullptr;
     P.t = nullptr;
@@ -2521,10 +2534,11 @@ static Params make_params(const grophecy_space *s, const grophecy_pcie *pc, cons
 }
 
 int launch_best(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *b,
-                grophecy_best_result *dout, int accumulate, cudaStream_t st)
+                grophecy_best_result *dout, int accumulate, cudaStream_t st, uint64_t local_off)
 {
     DeviceGuard guard(s->device);
     Params P = make_params(s, pc, b);
+    if (P.map_len) P.base = local_off;
     P.out = dout;
     P.accumulate = accumulate;
     return launch_passes<true>(s, P, st);
@@ -2697,15 +2711,19 @@ int grophecy_best_combine(const grophecy_best_result *din, uint32_t count,
 // End-to-end path with host records: chunked H2D copies on a copy stream,
 // double-buffered, overlapped with the fused kernel on the caller's stream;
 // one accumulating result slot; one D2H of 48 bytes at the end.
-int grophecy_best_host(grophecy_space *s, const grophecy_pcie *pc, const uint32_t *skx,
-                       const uint32_t *nx, const uint32_t *ny, const uint32_t *iters,
-                       uint64_t n, uint64_t index_base, grophecy_best_result *host_out,
-                       void *stream)
+int grophecy_best_host(grophecy_space *s, const grophecy_pcie *pc, const grophecy_batch *hb,
+                       grophecy_best_result *host_out, void *stream)
 {
-    if (!s || !pc || !host_out || (n && (!skx || !nx || !ny || !iters))) {
+    if (!s || !pc || !hb || !host_out || (hb->n && (!hb->skx || !hb->nx || !hb->ny || !hb->iters))) {
         set_error("null argument");
         return GROPHECY_EINVAL;
     }
+    if (hb->stripe_len && hb->stripe_stride < hb->stripe_len) {
+        set_error("stripe_stride < stripe_len");
+        return GROPHECY_EINVAL;
+    }
+    const uint32_t *skx = hb->skx, *nx = hb->nx, *ny = hb->ny, *iters = hb->iters;
+    const uint64_t n = hb->n;
     cudaStream_t st = (cudaStream_t)stream;
     cudaError_t e;
     DeviceGuard guard(s->device);
@@ -2748,8 +2766,12 @@ int grophecy_best_host(grophecy_space *s, const grophecy_pcie *pc, const uint32_
         }
         cudaEventRecord(s->ev_copied[slot], s->copy_stream);
         cudaStreamWaitEvent(st, s->ev_copied[slot], 0);
-        grophecy_batch b = {buf, buf + CHUNK, buf + 2 * CHUNK, buf + 3 * CHUNK, m, index_base + off};
-        int rc = launch_best(s, pc, &b, dres, 1, st);
+        // the chunk is records [off, off + m) of the host batch: same index
+        // map, local offset off
+        grophecy_batch b = {buf, buf + CHUNK, buf + 2 * CHUNK, buf + 3 * CHUNK, m,
+                            hb->index_base, hb->stripe_len, hb->stripe_stride};
+        if (!hb->stripe_len) b.index_base = hb->index_base + off;
+        int rc = launch_best(s, pc, &b, dres, 1, st, hb->stripe_len ? off : 0);
         if (rc) return rc;
         cudaEventRecord(s->ev_done[slot], st);
     }

@@ -40,6 +40,29 @@ def striped_chunks(n, rank, world, stripes, align=512):
     return out or [(0, 0)]
 
 
+def stripe_layout(n, rank, world, stripes, align=4096):
+    """Rank r's share of [0, n) as ONE batch of back-to-back stripes plus a
+    contiguous tail.  The first world * stripes * L records
+    (L = n / (world * stripes) rounded down to ``align``, whole sweep tiles)
+    are cut into stripes of L; rank r holds stripes j = r + world * k
+    (k < stripes), stored contiguously, so its local record i has global index
+    r * L + (i // L) * (world * L) + i % L: grophecy_batch's stripe map with
+    index_base = r * L, stripe_len = L, stripe_stride = world * L (one launch
+    per rank whatever ``stripes`` is; every rank gets a slice of every
+    skeleton of a skeleton-major workload).  The rest [world * stripes * L, n)
+    is split contiguously (shard_range).  Returns (L, main_count, (tail_lo,
+    tail_hi)); L = 0 (everything in the tail) when n is too small."""
+    L = (n // (world * stripes)) // align * align
+    main_end = world * stripes * L
+    t_lo, t_hi = shard_range(n - main_end, rank, world)
+    return L, stripes * L, (main_end + t_lo, main_end + t_hi)
+
+
+def stripe_global_index(i, rank, world, L):
+    """Global index of batch-local record i of the main stripe batch."""
+    return rank * L + (i // L) * (world * L) + i % L
+
+
 class MinLoc:
     """Device buffers for one query: ``local`` (this rank's result, written by
     grophecy_best_async), ``result`` (the global best after combine()).
@@ -49,12 +72,19 @@ class MinLoc:
     gloo process group (CPU collectives; used to exercise the multi-rank path
     on a single GPU) the gather goes through host memory."""
 
-    def __init__(self, world, device="cuda", backend=None):
+    def __init__(self, world, device="cuda", backend=None, space=None):
         from . import grophecy as G
         self.G = G
         self.world = world
         self.backend = backend or (dist.get_backend() if world > 1 else "nccl")
         self.local = torch.empty(RESULT_WORDS, dtype=torch.int64, device=device)
+        # NCCL: the library's own communicator and grophecy_best_allreduce_result
+        # (the product path); its unique id travels over the torch process group
+        self.space, self.comm, self.host = space, None, None
+        if world > 1 and self.backend == "nccl" and space is not None:
+            uid = [G.nccl_unique_id() if dist.get_rank() == 0 else None]
+            dist.broadcast_object_list(uid, src=0)
+            self.comm = G.NcclComm(world, dist.get_rank(), uid[0], torch.cuda.current_device())
         if world > 1:
             self.gathered = torch.empty(RESULT_WORDS * world, dtype=torch.int64, device=device)
             self.result = torch.empty(RESULT_WORDS, dtype=torch.int64, device=device)
@@ -63,6 +93,12 @@ class MinLoc:
                 self.h_gathered = torch.empty(RESULT_WORDS * world, dtype=torch.int64)
         else:
             self.result = self.local
+
+    def allreduce(self):
+        """Global best on the host via grophecy_best_allreduce_result (NCCL
+        all-gather + combine kernel + 48-byte D2H; synchronises)."""
+        rc, r = self.space.allreduce_result(self.local, self.comm)
+        return r
 
     def combine(self):
         if self.world == 1:

@@ -100,7 +100,8 @@ class GpuModel(C.Structure):
 
 class Batch(C.Structure):
     _fields_ = [("skx", C.c_void_p), ("nx", C.c_void_p), ("ny", C.c_void_p),
-                ("iters", C.c_void_p), ("n", C.c_uint64), ("index_base", C.c_uint64)]
+                ("iters", C.c_void_p), ("n", C.c_uint64), ("index_base", C.c_uint64),
+                ("stripe_len", C.c_uint64), ("stripe_stride", C.c_uint64)]
 
 
 class BestResult(C.Structure):
@@ -165,8 +166,9 @@ _sig = {
     "grophecy_best_async": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, C.c_int, _vp]),
     "grophecy_best_combine": (C.c_int, [_vp, C.c_uint32, _vp, _vp]),
     "grophecy_best_combine_host": (C.c_int, [C.POINTER(BestResult), C.c_uint32, C.POINTER(BestResult)]),
-    "grophecy_best_host": (C.c_int, [_vp, C.POINTER(PCIe), _vp, _vp, _vp, _vp, C.c_uint64,
-                                     C.c_uint64, C.POINTER(BestResult), _vp]),
+    "grophecy_best_host": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), C.POINTER(BestResult),
+                                     _vp]),
+    "grophecy_best_allreduce_result": (C.c_int, [_vp, _vp, _vp, C.POINTER(BestResult), _vp]),
     "grophecy_measure_transfer": (C.c_int, [C.c_int, C.c_int, C.c_uint64, C.c_int, C.c_int,
                                             C.POINTER(C.c_double), C.POINTER(C.c_double)]),
     "grophecy_calibrate": (C.c_int, [C.c_int, C.c_int, C.c_uint64, C.POINTER(PCIe)]),
@@ -195,6 +197,11 @@ for _name, (_res, _args) in _sig.items():
     _f.argtypes = _args
 
 EXPORTED = tuple(_sig)
+
+# the struct layouts above are ABI version 4 (include/grophecy.h)
+ABI_VERSION = 4
+if _L.grophecy_abi_version() != ABI_VERSION:
+    raise ImportError(f"libgrophecy.so ABI {_L.grophecy_abi_version()} != binding ABI {ABI_VERSION}: rebuild")
 
 
 def lib():
@@ -320,12 +327,15 @@ class Records:
         return cls(*[torch.empty(max(n, 1), dtype=torch.int32, device=device)[:n]
                      for _ in range(4)])
 
-    def batch(self, index_base=0, start=0, stop=None):
+    def batch(self, index_base=0, start=0, stop=None, stripe_len=0, stripe_stride=0):
+        """Records [start, stop) as a grophecy_batch; with stripe_len the
+        batch-local record i has global index index_base + (i // stripe_len)
+        * stripe_stride + i % stripe_len (include/grophecy.h)."""
         stop = self.n if stop is None else stop
         off = start * 4
         return Batch(self.skx.data_ptr() + off, self.nx.data_ptr() + off,
                      self.ny.data_ptr() + off, self.iters.data_ptr() + off, stop - start,
-                     index_base)
+                     index_base, stripe_len, stripe_stride)
 
 
 def synth_rules(cfg):
@@ -465,21 +475,27 @@ class Space:
         _check(_L.grophecy_best_async(self.h, C.byref(pc), C.byref(batch), _ptr(dout),
                                       int(bool(accumulate)), _stream_ptr(stream)), "best_async")
 
-    def best_host(self, pc, rec_host, index_base=0, stream=None):
+    def best_host(self, pc, rec_host, index_base=0, stream=None, stripe_len=0, stripe_stride=0):
         """rec_host: dict of four uint32 arrays (numpy or pinned torch CPU tensors)."""
         ptrs = []
         for k in ("skx", "nx", "ny", "iters"):
             a = rec_host[k]
-            ptrs.append(C.c_void_p(a.data_ptr() if hasattr(a, "data_ptr") else a.ctypes.data))
+            ptrs.append(a.data_ptr() if hasattr(a, "data_ptr") else a.ctypes.data)
         n = len(rec_host["skx"])
+        hb = Batch(*ptrs, n, index_base, stripe_len, stripe_stride)
         r = BestResult()
-        rc = _L.grophecy_best_host(self.h, C.byref(pc), *ptrs, n, index_base, C.byref(r),
-                                   _stream_ptr(stream))
+        rc = _L.grophecy_best_host(self.h, C.byref(pc), C.byref(hb), C.byref(r), _stream_ptr(stream))
         _check(rc, "best_host", ok=(OK, ENOFEASIBLE, EBADCAND))
         return rc, r
 
-
-ENCCL = -4
+    def allreduce_result(self, dres, comm, stream=None):
+        """Global best over the ranks of `comm` of a device result tensor
+        (grophecy_best_allreduce_result)."""
+        r = BestResult()
+        rc = _L.grophecy_best_allreduce_result(self.h, _ptr(dres), comm.handle, C.byref(r),
+                                               _stream_ptr(stream))
+        _check(rc, "best_allreduce_result", ok=(OK, ENOFEASIBLE, EBADCAND))
+        return rc, r
 
 
 def nccl_unique_id():

@@ -5,9 +5,9 @@ mkdir -p gpurun_out
 nvidia-smi -L > gpurun_out/gpu.txt 2>&1
 nproc >> gpurun_out/gpu.txt; free -g >> gpurun_out/gpu.txt; lscpu | head -20 >> gpurun_out/gpu.txt
 python -m paper_conf_ipps_boyermk13_b200.build --force --verbose > gpurun_out/build.log 2>&1 || { echo BUILD FAILED; tail -30 gpurun_out/build.log; exit 1; }
-timeout ${PYTEST_TIMEOUT:-1500} python -m pytest tests -m gpu -q --timeout 900 ${PYTEST_ARGS} > gpurun_out/pytest_gpu.log 2>&1
+timeout ${PYTEST_TIMEOUT:-1200} python -m pytest tests -m gpu -q --timeout 300 --durations=15 ${PYTEST_ARGS} > gpurun_out/pytest_gpu.log 2>&1
 echo "pytest rc=$?"; tail -25 gpurun_out/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -3 gpurun_out/smoke.log
 if [ -z "$NO_BENCH" ]; then
-timeout 900 python bench.py ${BENCH_ARGS} > gpurun_out/bench.log 2>&1; echo "bench rc=$?"; tail -3 gpurun_out/bench.log
+timeout 600 python bench.py ${BENCH_ARGS} > gpurun_out/bench.log 2>&1; echo "bench rc=$?"; tail -3 gpurun_out/bench.log
 fi

@@ -39,7 +39,7 @@ def test_every_declared_symbol_is_exported(G):
 
 
 def test_abi_version(G):
-    assert G.lib().grophecy_abi_version() == 3
+    assert G.lib().grophecy_abi_version() == G.ABI_VERSION == 4
 
 
 def test_fit_pcie_matches_oracle_bitwise(G, O):

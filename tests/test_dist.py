@@ -227,3 +227,36 @@ def test_striped_chunks_partition(n, world, stripes):
         assert a == pos
         pos = b
     assert pos == n
+
+
+@pytest.mark.parametrize("n,world,stripes", [(10**9, 8, 16), (10**9, 2, 16), (10**7, 3, 5),
+                                             (5000, 4, 16), (0, 2, 4), (123457, 7, 3)])
+def test_stripe_layout_partition(n, world, stripes):
+    """dist.stripe_layout: the ranks' stripe batches + tails cover [0, n)
+    exactly once, and the local -> global map of the stripe batch is the one
+    grophecy_batch documents (increasing, so ties stay lowest-index)."""
+    import numpy as np
+    from paper_conf_ipps_boyermk13_b200 import dist as D
+    total = 0
+    pieces = []
+    for r in range(world):
+        L, n_main, (t_lo, t_hi) = D.stripe_layout(n, r, world, stripes)
+        assert L % 4096 == 0 and n_main == (stripes * L)
+        total += n_main + t_hi - t_lo
+        for k in range(stripes if L else 0):
+            g0 = D.stripe_global_index(k * L, r, world, L)
+            assert g0 == (r + world * k) * L
+            pieces.append((g0, g0 + L))
+        if t_hi > t_lo:
+            pieces.append((t_lo, t_hi))
+        if L:
+            i = np.array([0, L - 1, L, n_main - 1])
+            g = [D.stripe_global_index(int(v), r, world, L) for v in i]
+            assert g == sorted(g)
+    assert total == n
+    pieces.sort()
+    pos = 0
+    for a, b in pieces:
+        assert a == pos
+        pos = b
+    assert pos == n
