@@ -126,12 +126,52 @@ def measured_peaks():
 
 
 def profile_summary():
-    """Per-launch DRAM traffic and executed warp instructions of the best
-    kernel from the committed ncu capture (profiles/ncu_best_summary.json)."""
+    """Per-launch DRAM traffic of the best kernel from the committed ncu
+    capture (profiles/ncu_best_summary.json)."""
     p = os.path.join(ROOT, "profiles", "ncu_best_summary.json")
     if not os.path.exists(p):
         return {}
     return json.load(open(p))
+
+
+def op_roofline(config_name, value, hbm_peak_gbs):
+    """The op-bound half of the roofline: the
+    oracle's algorithmic op tally per candidate (profiles/op_tally.json,
+    scripts/op_tally.py) against the microbenchmarked pipe peaks
+    (profiles/peaks.json, scripts/micro/peaks.cu); each op class bounds the
+    rate at peak / tally, the HBM bound is peak bandwidth / 16 B, and the
+    binding bound is the smallest."""
+    try:
+        tally = json.load(open(os.path.join(ROOT, "profiles", "op_tally.json")))[config_name]
+        peaks = json.load(open(os.path.join(ROOT, "profiles", "peaks.json")))
+    except (OSError, KeyError, ValueError):
+        return None
+    classes = {"fp64": ("fp64", peaks["fp64_ops_per_s"]),
+               "int": ("int", peaks["int_imad_ops_per_s"]),
+               "cvt": ("cvt", peaks["i2f_f64_ops_per_s"])}
+    bounds = {"hbm": hbm_peak_gbs * 1e9 / 16.0}
+    for name, (key, peak) in classes.items():
+        if tally.get(key):
+            bounds[name] = peak / tally[key]
+    binding = min(bounds, key=bounds.get)
+    op = min((k for k in bounds if k != "hbm"), key=bounds.get)
+    return {"bound": op, "achieved": value * tally[classes[op][0]], "peak": classes[op][1],
+            "unit": f"{op} op/s", "frac": value * tally[classes[op][0]] / classes[op][1],
+            "tally_per_candidate": {k: tally[k] for k in ("fp64", "int", "cvt")},
+            "bounds_candidates_per_s": bounds, "binding": binding,
+            "frac_of_binding": value / bounds[binding],
+            "source": "profiles/op_tally.json (oracle tally, scripts/op_tally.py) / profiles/peaks.json "
+                      "(scripts/micro/peaks.cu, measured on a B200)"}
+
+
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 # ---------------------------------------------------------------- oracle legs
@@ -327,27 +367,14 @@ def main():
         traffic = traffic * n_local / prof_n
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": achieved / peak, "traffic": traffic,
-            "kernel": "canon_kernel<best> + general_kernel<best> (fused projection + argmin; pass 1 is >99% of the step, profiles/)",
+            "kernel": "sweep_kernel<best> + general_kernel<best> (fused projection + argmin; pass 1 is >99% of the step, profiles/)",
             "algorithmic_bytes_per_launch": 16 * n_local,
             "kernel_ms_avg": kern_avg_max, "peak_source": peak_src,
             "note": "16 B/candidate record read (DESIGN.md §5); kernel duration from CUDA "
                     "events around each launch on its stream"}
-    # the binding resource: instruction issue (executed warp instructions per
-    # candidate from the committed ncu capture x this run's candidates / time)
-    roof_issue = None
-    if prof.get("warp_inst_per_launch") and prof_n:
-        sm_mhz = (clocks or {}).get("sm_mhz") or 1965.0
-        props = torch.cuda.get_device_properties(local_dev)
-        peak_issue = props.multi_processor_count * 4 * sm_mhz * 1e6
-        ach = prof["warp_inst_per_launch"] / prof_n * n_local / (kern_avg_max * 1e-3)
-        if ach > 1.02 * peak_issue:   # committed capture is stale for this build
-            ach = None
-        roof_issue = None if ach is None else {"bound": "alu", "achieved": ach, "peak": peak_issue,
-                      "unit": "warp-inst/s", "frac": ach / peak_issue,
-                      "warp_inst_per_candidate": prof["warp_inst_per_launch"] / prof_n,
-                      "note": "executed (not algorithmic) warp instructions from "
-                              + prof.get("source", "profiles/") + "; peak = SMs x 4 "
-                              "schedulers x 1 inst/clk x measured SM clock"}
+    roof_op = op_roofline(args.config, value, peak)
+    if roof_op:
+        roof["binding"] = roof_op["binding"]
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         threads = cpu_cores()
@@ -356,6 +383,9 @@ def main():
         P.best(srec, nthreads=threads)
         dt = time.perf_counter() - t_a
         cpu = {"value": m / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
+               "cpu_model": cpu_model(),
+               "full_configs": "profiles/cpu_baseline.json (scripts/cpu_baseline.py: C1-C3 in full, "
+                               "1 thread and all cores, on the GPU box's host)",
                "sample": f"{m} records: 16 equal slices at offsets k*N/16 of the workload "
                          f"(every skeleton), one oracle_best pass, {dt:.1f} s"}
         # the same oracle on one core (1 thread and all cores)
@@ -376,7 +406,7 @@ def main():
                        "gpu_model": "Quadro FX 5600 preset (paper's GPU, P:L149)",
                        "pcie": "alpha=1e-5 s, 1/beta=2.5 GB/s (paper magnitudes, P:L111)",
                        "l2": "inputs 16 B x shard >> 126 MB L2; no flush needed"},
-            "roofline": roof, "roofline_issue": roof_issue, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "roofline": roof, "roofline_op": roof_op, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
             "gpu_launches": launches,
             "best": {"index": best.index, "t_total_s": best.t_total_s,
                      "h2d_bytes": best.h2d_bytes, "d2h_bytes": best.d2h_bytes}}

@@ -351,6 +351,9 @@ double grophecy_speedup(double t_cpu_s, double t_gpu_s);
 /* Error magnitude |predicted - measured| / measured (Table II applies
  * it to predicted vs measured speedups).  Pure host functions. */
 double grophecy_error_magnitude(double predicted, double measured);
+/* Arithmetic mean of n values, summed in order (the paper's averages of
+ * error magnitudes).  NaN for n = 0.  Pure host. */
+double grophecy_mean(const double *values, uint64_t n);
 
 /* End-to-end entry point: host_batch's record arrays are HOST memory
  * (pinned for full speed; index_base / stripes as in grophecy_batch).  The

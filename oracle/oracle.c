@@ -539,6 +539,122 @@ int oracle_eval_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
     return 1;
 }
 
+/* ------------------------------------------------------------------------ */
+/* Algorithmic op tally of one candidate (DESIGN.md §6,     */
+/* "op-bound roofline").  Counts the arithmetic the definition N4-N6 needs   */
+/* per candidate under the stated amortisation rule:                         */
+/*  R1  size-independent quantities are computed once per design space and   */
+/*      charge nothing per candidate: N5 part A, the saturated-grid          */
+/*      constants (E, S, D: on a saturated grid #Active_SMs = n_sm and        */
+/*      active blocks/SM = occupancy, so MWP, CWP, the H&K case and the       */
+/*      synch factor are fixed) and the times of the finitely many grids     */
+/*      below saturation (blocks < sat: a per-(kernel, transformation)       */
+/*      table);                                                               */
+/*  R2  data usage depends only on (skeleton, nx, ny) (N4, reading 11): it is */
+/*      charged once per design point of X transformations, 1/X per record:   */
+/*      per kernel its work count (affine8: 3 mul + 2 add + 1 shift = 6 int), */
+/*      per array and direction its byte count (a bilinear form: 6 int) and,  */
+/*      when the bytes are non-zero, Eq. (1) priced and summed (1 int->fp64   */
+/*      conversion, 1 mul, 2 add);                                           */
+/*  R3  exact identities cost nothing: a product with an exact zero (S = 0),  */
+/*      a division by a power of two (rep = blocks * 2^-k folds into E), and  */
+/*      a kernel with zero occupancy (its sum is +inf).                       */
+/* Per (candidate, kernel) on a saturated grid: blocks = ceil(W / ipb) by a  */
+/* multiply-high and a shift (2 int), 1 conversion, rep = blocks / D (a      */
+/* division), cyc = E rep (+ S rep: mul + add), t = cyc / freq (a division),  */
+/* the running sum (1 add); below saturation 2 int + the running sum.  Per   */
+/* candidate: iters * t_iter (mul), + t_once (add, when the skeleton has     */
+/* run-once kernels), + t_h2d, + t_d2h (2 add), the argmin compare (1).       */
+/* fp64 counts each add / mul / compare as 1 and each division by a space    */
+/* constant as 2 (its cheapest exact evaluation, x*zh + RN(x*zl): the        */
+/* two-product form).  Returns 1 for a valid record (0: all counts 0).        */
+int oracle_op_tally_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                        uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters, uint32_t X,
+                        double *fp64, double *ints, double *cvt)
+{
+    uint32_t skel = skx >> 16, xform = skx & 0xffffu;
+    *fp64 = *ints = *cvt = 0.0;
+    if (skel >= n_skels || xform >= skels[skel].n_xforms || nx < 1 || nx > (1u << 20) ||
+        ny < 1 || ny > (1u << 20) || iters < 1 || X < 1)
+        return 0;
+    const or_skeleton *s = &skels[skel];
+    double f = 0.0, in = 0.0, cv = 0.0;
+    int has_once = 0;
+    for (uint32_t k = 0; k < s->n_kernels; k++) {
+        const or_kx *c = &s->kx[(size_t)xform * s->n_kernels + k];
+        if (!s->kernels[k].per_iter) has_once = 1;
+        uint64_t occ;
+        if (c->tpb > g->max_tpb) {
+            occ = 0;
+        } else {
+            occ = umin64(g->max_bps, g->max_tps / c->tpb);
+            if (c->regs > 0) occ = umin64(occ, g->regs_sm / ((uint64_t)c->regs * c->tpb));
+            if (c->smem > 0) occ = umin64(occ, g->smem_sm / c->smem);
+        }
+        in += 6.0 / X;                                   /* work count (R2) */
+        if (occ == 0) continue;                          /* R3: sum is +inf */
+        uint64_t ipb = (uint64_t)c->tpb * c->ipt;
+        int64_t Wi = oracle_affine8(&s->kernels[k].work, nx, ny);
+        uint64_t W = Wi > 0 ? (uint64_t)Wi : 0;
+        uint64_t blocks = W / ipb + (W % ipb != 0);
+        in += 2.0;                                       /* ceil division */
+        f += 1.0;                                        /* running sum */
+        uint64_t asm_ = umin64(g->n_sm, blocks ? blocks : 1);
+        uint64_t abps = blocks ? umin64(occ, blocks / asm_ + (blocks % asm_ != 0)) : 0;
+        if (!(asm_ == g->n_sm && abps == occ)) continue; /* below saturation: tabulated (R1) */
+        cv += 1.0;
+        uint64_t D = occ * g->n_sm;
+        if (D & (D - 1)) f += 2.0;                       /* rep = blocks / D */
+        f += 1.0;                                        /* E * rep */
+        /* S = Departure_delay * (MWP - 1) * #synch * occupancy at saturation */
+        double mem = c->coal + c->uncoal, S = 0.0;
+        if (mem != 0.0) {
+            double mlu = g->mem_ld + (c->upm - 1.0) * g->dd_uncoal, mlc = g->mem_ld;
+            double wu = c->uncoal / mem, wc = c->coal / mem;
+            double ml = mlu * wu + mlc * wc;
+            double dd = (g->dd_uncoal * c->upm) * wu + g->dd_coal * wc;
+            double bwr = g->mem_bw / (g->freq * c->lbpw / ml);
+            double N = (double)(occ * (c->tpb / g->warp_size + (c->tpb % g->warp_size != 0)));
+            double mwp = dmin(dmin(ml / dd, bwr / (double)g->n_sm), N);
+            S = dd * (mwp - 1.0) * c->synch * (double)occ;
+        }
+        if (S != 0.0) f += 2.0;                          /* + S * rep */
+        f += 2.0;                                        /* / freq */
+    }
+    /* usage of the design point (R2) */
+    uint64_t hpa[64], dpa[64];
+    oracle_usage(s, nx, ny, hpa, dpa);
+    for (uint32_t a = 0; a < s->n_arrays; a++) {
+        in += 12.0 / X;
+        if (hpa[a]) { f += 3.0 / X; cv += 1.0 / X; }
+        if (dpa[a]) { f += 3.0 / X; cv += 1.0 / X; }
+    }
+    f += 1.0 + (has_once ? 1.0 : 0.0) + 2.0 + 1.0;      /* totals + argmin */
+    *fp64 = f;
+    *ints = in;
+    *cvt = cv;
+    return 1;
+}
+
+/* Mean tally over a batch (single thread).  Returns the valid record count. */
+uint64_t oracle_op_tally(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                         const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                         const uint32_t *iters, uint64_t n, uint32_t X, double *mean3)
+{
+    double sf = 0.0, si = 0.0, sc = 0.0;
+    uint64_t v = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        double f, in, cv;
+        if (oracle_op_tally_one(skels, n_skels, g, skx[i], nx[i], ny[i], iters[i], X, &f, &in, &cv)) {
+            sf += f; si += in; sc += cv; v++;
+        }
+    }
+    mean3[0] = v ? sf / (double)v : 0.0;
+    mean3[1] = v ? si / (double)v : 0.0;
+    mean3[2] = v ? sc / (double)v : 0.0;
+    return v;
+}
+
 /* The projection with the per-array memory choice (NEXT-4, DESIGN.md
  * reading 17): every array with a transfer is priced as pinned (its
  * allocation A(footprint) + pinned transfers) or pageable, whichever

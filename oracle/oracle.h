@@ -25,6 +25,9 @@
  *                                           ("parity unpinned" by the paper itself)
  *   oracle_eval_one / oracle_best ........ pinned (composition identities, brute-force min)
  *   validation helpers ................... pinned (Table II arithmetic)
+ *   oracle_op_tally[_one] ................ pinned to hand counts of its own stated
+ *                                           rule: a measurement
+ *                                           convention, not a paper quantity
  *   oracle_choose_memory ................. pinned to closed forms of OUR reading 17
  *                                           (pinned vs pageable + allocation, NEXT-4);
  *                                           the paper only names the tradeoff (P:L93,
@@ -159,6 +162,19 @@ int oracle_best(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
                 const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
                 const uint32_t *iters, uint64_t n, uint64_t index_base,
                 int nthreads, or_best *out);
+
+/* Algorithmic op tally of one candidate under the amortisation rule of
+ * DESIGN.md §6 (oracle.c states it in full): fp64 operations (a division by a
+ * space constant counts 2), integer operations and int->fp64 conversions per
+ * record, usage charged once per design point of X records.  Returns 1 if the
+ * record is valid.  oracle_op_tally: means over a batch (mean3 = {fp64, int,
+ * cvt}), returns the number of valid records. */
+int oracle_op_tally_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                        uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters, uint32_t X,
+                        double *fp64, double *ints, double *cvt);
+uint64_t oracle_op_tally(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
+                         const uint32_t *skx, const uint32_t *nx, const uint32_t *ny,
+                         const uint32_t *iters, uint64_t n, uint32_t X, double *mean3);
 
 /* Validation helpers (Table II). */
 double oracle_error_magnitude(double predicted, double measured);

@@ -131,6 +131,12 @@ def lib():
             getattr(L, name).restype = C.c_double
         L.oracle_crossover.argtypes = [C.c_double] * 5 + [C.POINTER(C.c_double),
                                                           C.POINTER(C.c_uint64)]
+        L.oracle_op_tally_one.argtypes = [SK, C.c_uint32, C.POINTER(GPU), C.c_uint32, C.c_uint32,
+                                          C.c_uint32, C.c_uint32, C.c_uint32] + \
+            [C.POINTER(C.c_double)] * 3
+        L.oracle_op_tally.argtypes = [SK, C.c_uint32, C.POINTER(GPU), u32p, u32p, u32p, u32p,
+                                      C.c_uint64, C.c_uint32, f64p]
+        L.oracle_op_tally.restype = C.c_uint64
         L.oracle_mean.argtypes = [f64p, C.c_uint64]
         L.oracle_mean.restype = C.c_double
         _lib = L
@@ -291,6 +297,20 @@ class Problem:
         ng = lib().oracle_group_best(self.ss.arr, self.ss.n, C.byref(self.gpu), C.byref(self.hl),
                                      C.byref(self.dl), *a, n, index_base, cap, first, count, bi, bt)
         return first[:ng], count[:ng], bi[:ng], bt[:ng]
+
+    def op_tally_one(self, skx, nx, ny, iters, X=16):
+        """(ok, fp64, int, cvt) algorithmic ops of one candidate (oracle.c)."""
+        v = [C.c_double() for _ in range(3)]
+        ok = lib().oracle_op_tally_one(self.ss.arr, self.ss.n, C.byref(self.gpu), skx, nx, ny,
+                                       iters, X, *[C.byref(x) for x in v])
+        return bool(ok), v[0].value, v[1].value, v[2].value
+
+    def op_tally(self, rec, X=16):
+        """Mean {fp64, int, cvt} ops per valid record of a batch."""
+        m = np.zeros(3, np.float64)
+        a = [np.ascontiguousarray(rec[k], dtype=np.uint32) for k in ("skx", "nx", "ny", "iters")]
+        nv = lib().oracle_op_tally(self.ss.arr, self.ss.n, C.byref(self.gpu), *a, len(a[0]), X, m)
+        return {"fp64": float(m[0]), "int": float(m[1]), "cvt": float(m[2]), "n_valid": int(nv)}
 
     def best(self, rec, index_base=0, nthreads=None):
         n = len(rec["skx"])

@@ -308,6 +308,14 @@ double grophecy_error_magnitude(double predicted, double measured)
     return std::fabs(predicted - measured) / measured;
 }
 
+double grophecy_mean(const double *values, uint64_t n)
+{
+    if (!values || n == 0) return NAN;
+    double s = 0.0;
+    for (uint64_t i = 0; i < n; i++) s += values[i];
+    return s / (double)n;
+}
+
 int grophecy_space_validate(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                             const grophecy_gpu_model *gpu)
 {

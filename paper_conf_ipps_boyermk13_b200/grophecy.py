@@ -162,6 +162,7 @@ _sig = {
                                      _vp]),
     "grophecy_speedup": (C.c_double, [C.c_double, C.c_double]),
     "grophecy_error_magnitude": (C.c_double, [C.c_double, C.c_double]),
+    "grophecy_mean": (C.c_double, [C.POINTER(C.c_double), C.c_uint64]),
     "grophecy_best": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), C.POINTER(BestResult), _vp]),
     "grophecy_best_async": (C.c_int, [_vp, C.POINTER(PCIe), C.POINTER(Batch), _vp, C.c_int, _vp]),
     "grophecy_best_combine": (C.c_int, [_vp, C.c_uint32, _vp, _vp]),
@@ -644,6 +645,13 @@ def crossover(t_iter, t_once, t_h2d, t_d2h, t_cpu_iter, stream=None):
 
 def speedup(t_cpu, t_gpu):
     return _L.grophecy_speedup(t_cpu, t_gpu)
+
+
+def mean(values):
+    """grophecy_mean: arithmetic mean summed in order."""
+    v = list(values)
+    arr = (C.c_double * max(1, len(v)))(*v)
+    return _L.grophecy_mean(arr, len(v))
 
 
 def error_magnitude(pred, meas):

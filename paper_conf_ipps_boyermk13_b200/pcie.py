@@ -8,10 +8,12 @@
   magnitude |pred - meas| / meas per size, its mean and max per direction,
   and the run-to-run noise floor (a second sweep predicted from the first).
   Modes: "single" (one GPU at a time) and "concurrent" (all GPUs at once,
-  barrier-aligned), the latter also scored against the single-mode fit.
+  a barrier before every size and direction), the latter also scored
+  against the single-mode fit.
 
-Every transfer is measured by the CUDA library (grophecy_measure_transfer);
-this module only orchestrates and does the bookkeeping arithmetic.
+Every transfer is measured by the CUDA library (grophecy_measure_transfer)
+and every error magnitude and mean is computed by the library's helpers
+(grophecy_error_magnitude, grophecy_mean); this module only orchestrates.
 """
 import threading
 
@@ -19,15 +21,8 @@ from . import grophecy as G
 
 DIRS = (("h2d", G.DIR_H2D), ("d2h", G.DIR_D2H))
 
-
-def error_magnitude(pred, meas):
-    """|pred - meas| / meas (as a fraction)."""
-    return abs(pred - meas) / meas
-
-
-def mean(v):
-    v = list(v)
-    return sum(v) / len(v)
+error_magnitude = G.error_magnitude   # |pred - meas| / meas
+mean = G.mean                         # arithmetic mean
 
 
 def default_sizes(lo_exp=10, hi_exp=30, include_one=True):
@@ -35,12 +30,19 @@ def default_sizes(lo_exp=10, hi_exp=30, include_one=True):
     return ([1] if include_one else []) + [1 << e for e in range(lo_exp, hi_exp + 1)]
 
 
-def sweep(device, sizes, reps=10, warmup=2, memory=G.MEM_PINNED):
-    """{direction: [(bytes, mean_wall_s, mean_event_s)]} for one device."""
+def sweep(device, sizes, reps=10, warmup=2, memory=G.MEM_PINNED, barrier=None):
+    """{direction: [(bytes, mean_wall_s, mean_event_s)]} for one device.
+    With a barrier (concurrent mode) every (direction, size) measurement
+    starts together on all devices, so each size is measured under the
+    contention of all of them."""
     out = {}
     for name, d in DIRS:
-        out[name] = [(s, *G.measure_transfer_mem(device, d, memory, s, reps, warmup))
-                     for s in sizes]
+        rows = []
+        for s in sizes:
+            if barrier is not None:
+                barrier.wait()
+            rows.append((s, *G.measure_transfer_mem(device, d, memory, s, reps, warmup)))
+        out[name] = rows
     return out
 
 
@@ -104,9 +106,8 @@ def validate(devices, sizes=None, reps=10, warmup=2, large=1 << 29, concurrent=T
         barrier = threading.Barrier(len(devices))
         results = {}
 
-        def run(d):
-            barrier.wait()
-            results[d] = sweep(d, sizes, reps, warmup)
+        def run(d):   # one host thread per GPU, aligned at every size
+            results[d] = sweep(d, sizes, reps, warmup, barrier=barrier)
 
         th = [threading.Thread(target=run, args=(d,)) for d in devices]
         for t in th:
