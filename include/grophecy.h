@@ -490,6 +490,12 @@ int grophecy_plan_usage_host(const grophecy_skeleton_desc *skel, int64_t nx, int
  * ELIMIT if the skeleton has no plan.  Pure host function. */
 int grophecy_plan_stats(const grophecy_skeleton_desc *skel, uint32_t *stats);
 
+/* Diagnostic: per-phase warp-cycle sums of the sweep kernel (8 entries:
+ * waiting for staged records, phase A, barrier, phase B, barrier, phase C),
+ * copied to HOST out8 and reset.  Only in builds with GROPHECY_PHASE_TIMING=1
+ * (scripts/phase_timing.py); EINVAL otherwise. */
+int grophecy_debug_phase_cycles(uint64_t *out8);
+
 /* Number of CUDA kernel launches issued by this library since load (for
  * the bench's gpu_launches count). */
 uint64_t grophecy_launch_count(void);

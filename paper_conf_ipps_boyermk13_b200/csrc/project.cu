@@ -1921,10 +1921,42 @@ constexpr uint32_t SW_BAD = 0xffffffffu;
 #ifndef GROPHECY_SMINB
 #define GROPHECY_SMINB 2
 #endif
+#ifndef GROPHECY_I2F_MAGIC
+#define GROPHECY_I2F_MAGIC 0
+#endif
+#ifndef GROPHECY_EUNROLL
+#define GROPHECY_EUNROLL 1
+#endif
+#ifndef GROPHECY_LDGSTS
+#define GROPHECY_LDGSTS 0
+#endif
+#ifndef GROPHECY_DIAG_NOLOAD
+#define GROPHECY_DIAG_NOLOAD 0
+#endif
+#ifndef GROPHECY_PF
+#define GROPHECY_PF 0
+#endif
+// GROPHECY_PHASE_TIMING=1 (diagnostic builds only): per-warp clock64 time per
+// phase of the sweep kernel, summed into g_phase_cycles and read back by
+// grophecy_debug_phase_cycles (scripts/phase_timing.py)
+#ifndef GROPHECY_PHASE_TIMING
+#define GROPHECY_PHASE_TIMING 0
+#endif
+#if GROPHECY_PHASE_TIMING
+__device__ unsigned long long g_phase_cycles[8];
+#define PT_MARK(slot)                                                              \
+    do {                                                                           \
+        const long long t_ = clock64();                                            \
+        if (lane == 0) atomicAdd(&g_phase_cycles[slot], (unsigned long long)(t_ - pt_last)); \
+        pt_last = t_;                                                              \
+    } while (0)
+#else
+#define PT_MARK(slot) do { } while (0)
+#endif
 
 struct alignas(128) SweepSmem {
-    alignas(128) uint32_t rec[WARPS][4][CTILE];   // per warp: its warp tile (TMA bulk copies)
-    unsigned long long mbar[WARPS];
+    alignas(128) uint32_t rec[4][SW_TILE];   // the CTA tile's SoA records (4 TMA bulk copies)
+    unsigned long long rbar;     // completion of the record copies
     unsigned long long tbar;     // completion of the usage-table copy
     // per design point g = 32 * (warp of phase B) + lane, natural order
     alignas(16) double it[SW_GROUPS], th[SW_GROUPS], td[SW_GROUPS];
@@ -1933,7 +1965,8 @@ struct alignas(128) SweepSmem {
     uint32_t smallk[SW_GROUPS];  // per design point: kernels whose grid may be unsaturated
     uint32_t askel[WARPS];       // phase A result per warp: its skeleton, or SW_BAD
     uint32_t wstat[WARPS];       // phase B result per warp: its skeleton, or SW_BAD
-    uint32_t next_tile;          // the CTA's next tile (claimed by thread 0)
+    uint32_t next0;              // the CTA's second tile (claimed by thread 0 before the loop)
+    uint32_t next_tile;          // the tile after the next one (claimed by thread 0 each tile)
     uint32_t unit;               // phase-C unit counter
     uint32_t tbl_skel;           // skeleton whose usage table is staged (SW_BAD: none)
     uint32_t tbl_wait;           // this tile: parity to wait for on tbar, or SW_BAD (no copy)
@@ -1991,13 +2024,56 @@ __device__ __forceinline__ void group_usage_s(const int4 *pp, uint32_t n_arrays,
     }
 }
 
+// CTA tile copy (thread 0): the 4 SoA arrays' SW_TILE records from tb into
+// sm.rec, completing on sm.rbar.  Every generic-proxy read of sm.rec by the
+// CTA happened before the caller's barrier; the fence orders them before the
+// async-proxy writes.
+__device__ __forceinline__ void issue_cta_copy(const Params &P, uint32_t (*rec)[SW_TILE],
+                                               unsigned long long *rbar, unsigned long long tb)
+{
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    const uint32_t bar = smem_u32(rbar);
+    const uint32_t bytes = (uint32_t)(SW_TILE * sizeof(uint32_t));
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(4 * bytes)
+                 : "memory");
+    const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
+#pragma unroll
+    for (int a = 0; a < 4; a++)
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                smem_u32(rec[a])),
+            "l"(src[a] + tb), "r"(bytes), "r"(bar)
+            : "memory");
+}
+
+// The same CTA tile copy issued by every thread as 16-byte cp.async
+// (LDGSTS through L1) whose completions arrive on sm.rbar (initialised with
+// THREADS arrivals): many requests in flight per SM instead of 4 bulk copies.
+__device__ __forceinline__ void issue_cta_copy_async(const Params &P, uint32_t (*rec)[SW_TILE],
+                                                     unsigned long long *rbar, unsigned long long tb,
+                                                     int tid)
+{
+    const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
+    constexpr int CHUNKS = (int)(SW_TILE / 4);   // 16-byte chunks per array
+#pragma unroll
+    for (int a = 0; a < 4; a++)
+#pragma unroll
+        for (int c = tid; c < CHUNKS; c += THREADS)
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(rec[a] + 4 * c)),
+                         "l"(src[a] + tb + 4 * c)
+                         : "memory");
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(rbar)) : "memory");
+}
+
 // Phase A of one warp tile staged at rec (full: 32 design points): lane l
 // reads its design point's 16 records (rotated 16-byte chunks, conflict-free)
 // and checks the canonical layout (skx = s0 ^ q, equal nx, ny, iters) and
 // validity; warp-uniform result.
-__device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*rec)[CTILE], int lane,
-                                              uint32_t &s0, uint32_t &n0, uint32_t &m0, uint32_t &i0)
+__device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*recs)[SW_TILE], int warp,
+                                              int lane, uint32_t &s0, uint32_t &n0, uint32_t &m0, uint32_t &i0)
 {
+    const uint32_t *rec[4] = {recs[0] + warp * CTILE, recs[1] + warp * CTILE, recs[2] + warp * CTILE,
+                              recs[3] + warp * CTILE};
     uint32_t acc;
     const uint32_t r = ((uint32_t)lane >> 1) & 3u;
     {
@@ -2046,7 +2122,12 @@ __device__ __forceinline__ void cls_times(const double2 c01, const double2 c23, 
 {
 #pragma unroll
     for (int j = 0; j < NCH; j++) {
+#if GROPHECY_I2F_MAGIC
+        // (2^52 + blocks) - 2^52 on the fp64 pipe: exact for blocks < 2^52
+        const double bb = __dadd_rn(__hiloint2double(0x43300000, (int)blocks[j]), -0x1p52);
+#else
         const double bb = __uint2double_rn(blocks[j]);
+#endif
         double cyc;
         if (C == KXC_P2S0) {
             cyc = __dmul_rn(bb, c01.x);
@@ -2091,25 +2172,51 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             if (mine) P.tile_list[base + __popc(bal & ((1u << lane) - 1u))] = (uint32_t)sub;
         }
     }
-    if (lane == 0) mbar_init(&sm.mbar[warp], 1);
     if (tid == 0) {
+        mbar_init(&sm.rbar, GROPHECY_LDGSTS ? THREADS : 1);
         mbar_init(&sm.tbar, 1);
         sm.tbl_skel = SW_BAD;
         sm.tbl_phase = 0;
     }
+    // tiles: the first is blockIdx.x, then claims from a counter two tiles
+    // ahead (tile, next nt, and the claim in flight), so a warp's TMA copy of
+    // its part of the next tile starts as soon as phase A has consumed the
+    // current one and overlaps phases B and C
     unsigned *claim = P.tile_count + CLAIM1;
     unsigned long long tile = blockIdx.x;
+    if (tid == 0) sm.next0 = atomicAdd(claim, 1u) + gridDim.x;
     __syncthreads();
-    if (lane == 0 && tile < ntiles) issue_copy(P, sm.rec[warp], &sm.mbar[warp], tile * SW_TILE + (unsigned long long)warp * CTILE, 32u);
+    unsigned long long nt = sm.next0;
+#if GROPHECY_LDGSTS
+    if (tile < ntiles) issue_cta_copy_async(P, sm.rec, &sm.rbar, tile * SW_TILE, tid);
+#elif GROPHECY_DIAG_NOLOAD
+    // diagnostic: representative tiles per CTA (spread over the batch)
+    if (tid == 0 && tile < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, (blockIdx.x * (ntiles / gridDim.x)) * SW_TILE);
+#else
+    if (tid == 0 && tile < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, tile * SW_TILE);
+#endif
     uint32_t phase = 0;
     const double rfh = S.rfh, rfl = S.rfl;
+#if GROPHECY_PHASE_TIMING
+    long long pt_last = clock64();
+#endif
 #pragma unroll 1
     while (tile < ntiles) {
+        // the tile after nt: claimed now, its value is needed only after
+        // phase A (the atomic's latency overlaps the record wait and phase A)
+        unsigned claimed = 0;
+        if (tid == 0) claimed = atomicAdd(claim, 1u);
         // ---- A (this warp's tile) ----
-        mbar_wait(&sm.mbar[warp], phase);
+#if GROPHECY_DIAG_NOLOAD == 1   // diagnostic only (wrong results): records of the first tile reused
+        if (phase == 0) mbar_wait(&sm.rbar, 0);
+        phase = 1;
+#else
+        mbar_wait(&sm.rbar, phase);
         phase ^= 1u;
+#endif
+        PT_MARK(0);   // waiting for the staged records
         uint32_t s0, n0, m0, i0;
-        bool ok = sweep_phase_a(S, sm.rec[warp], lane, s0, n0, m0, i0);
+        bool ok = sweep_phase_a(S, sm.rec, warp, lane, s0, n0, m0, i0);
         const uint32_t skel = s0 >> 16;
         if (tid == 0) {
             // warp 0's skeleton decides the tile's usage table: stage it in
@@ -2132,12 +2239,49 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 sm.tbl_wait = sm.tbl_phase;
                 sm.tbl_phase ^= 1u;
             }
+            sm.next_tile = claimed + gridDim.x;   // the tile after nt
         }
+        PT_MARK(1);   // phase A (+ table check)
         __syncthreads();   // the previous tile's phase C is done with the per-design-point arrays
-        if (tid == 0) {
-            sm.next_tile = atomicAdd(claim, 1u) + gridDim.x;
-            sm.unit = 0;
+        PT_MARK(2);   // barrier 0
+        // every read of the staged tile is done (phase A): it takes the next
+        // one, and the tile after that is prefetched into L2
+        const unsigned long long nnt = sm.next_tile;
+#if GROPHECY_LDGSTS
+        if (nt < ntiles) issue_cta_copy_async(P, sm.rec, &sm.rbar, nt * SW_TILE, tid);
+#endif
+#if GROPHECY_PF == 2
+        // the tile after next into L2: one 128-byte line per thread and array half
+        if (nnt < ntiles) {
+            const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
+#pragma unroll
+            for (int a = 0; a < 4; a++)
+#pragma unroll
+                for (int l = tid; l < (int)(SW_TILE * 4 / 128); l += THREADS)
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(src[a] + nnt * SW_TILE + 32 * l) : "memory");
         }
+#endif
+        if (tid == 0) {
+#if GROPHECY_DIAG_NOLOAD == 2   // diagnostic: the same representative tile copied again (L2 hits)
+            if (nt < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, (blockIdx.x * (ntiles / gridDim.x)) * SW_TILE);
+#elif GROPHECY_DIAG_NOLOAD == 3   // diagnostic: 4 representative tiles in rotation (L2-resident, new data)
+            if (nt < ntiles)
+                issue_cta_copy(P, sm.rec, &sm.rbar, (blockIdx.x * (ntiles / gridDim.x) + (nt & 3u)) * SW_TILE);
+#elif !GROPHECY_LDGSTS && !GROPHECY_DIAG_NOLOAD
+            if (nt < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, nt * SW_TILE);
+#endif
+#if GROPHECY_PF == 1
+            if (nnt < ntiles) {
+                const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
+#pragma unroll
+                for (int a = 0; a < 4; a++)
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src[a] + nnt * SW_TILE),
+                                 "r"((uint32_t)(SW_TILE * sizeof(uint32_t)))
+                                 : "memory");
+            }
+#endif
+        }
+        if (tid == 0) sm.unit = 0;
         const uint32_t tw = sm.tbl_wait;
         if (tw != SW_BAD) mbar_wait(&sm.tbar, tw);
         // ---- B: work counts and usage of design point g ----
@@ -2186,11 +2330,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             }
         }
         if (lane == 0) sm.wstat[warp] = ok ? skel : SW_BAD;
+        PT_MARK(3);   // phase B (work counts, usage)
         __syncthreads();
-        const unsigned long long nt = sm.next_tile;
-        // every read of this warp's staged tile is done (phase A): it takes the next one
-        if (lane == 0 && nt < ntiles)
-            issue_copy(P, sm.rec[warp], &sm.mbar[warp], nt * SW_TILE + (unsigned long long)warp * CTILE, 32u);
+        PT_MARK(4);   // barrier 1
         const uint32_t s_all = sm.wstat[0];
         bool uni = s_all != SW_BAD;
 #pragma unroll
@@ -2198,6 +2340,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         if (!uni) {
             if (lane == 0) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * WARPS + warp);
             tile = nt;
+            nt = nnt;
             continue;
         }
         // ---- C: CTA-wide; unit = (transformation x, chain block) ----
@@ -2224,29 +2367,48 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             double ti[NCH], to[NCH];
 #pragma unroll
             for (int j = 0; j < NCH; j++) ti[j] = to[j] = 0.0;
-            auto one_kernel = [&](const KxProg *e, double (&acc)[NCH]) {
-                const uint4 *q = reinterpret_cast<const uint4 *>(e);
-                const uint4 hd = __ldg(q), kk = __ldg(q + 1);
-                const double2 c01 = __ldg(reinterpret_cast<const double2 *>(q + 2));
-                const double2 c23 = __ldg(reinterpret_cast<const double2 *>(q + 3));
-                const uint32_t k = kk.x, cls = kk.y;
-                const uint32_t sat = hd.y & KXF_SAT_MASK, sh = hd.y >> KXF_SAT_BITS;
-                const unsigned long long cc = ((unsigned long long)hd.w << 32) | hd.z;
-                uint32_t blocks[NCH];
+            // this lane's work-count chunks (cw_index for chains jb*NCH + 4q)
+            const uint32_t *cwl = cw + lane * (SW_GROUPS / 32);
+            uint32_t cwo[NCH / 4];
 #pragma unroll
-                for (int j = 0; j < NCH; j += 4) {
-                    const uint4 w4 = *reinterpret_cast<const uint4 *>(
-                        cw + cw_index(k, (uint32_t)lane, (uint32_t)((int)jb * NCH + j)));
+            for (int q = 0; q < NCH / 4; q++)
+                cwo[q] = ((((jb * NCH) / 4 + (uint32_t)q) ^ ((uint32_t)lane >> 2)) & 1u) << 2;
+            struct Ent {
+                uint4 hd;
+                double2 c01, c23;
+            };
+            auto load_ent = [&](const KxProg *e) {
+                const uint4 *q = reinterpret_cast<const uint4 *>(e);
+                Ent r;
+                r.hd = __ldg(q);
+                r.c01 = __ldg(reinterpret_cast<const double2 *>(q + 1));
+                r.c23 = __ldg(reinterpret_cast<const double2 *>(q + 2));
+                return r;
+            };
+            auto one_kernel = [&](const Ent &en, double (&acc)[NCH]) {
+                const uint32_t code = en.hd.y;
+                const uint32_t k = (code >> KXP_K_SHIFT) & 31u, cls = code >> KXP_CLS_SHIFT;
+                const uint32_t sat = code & KXP_SAT_MASK, sh = (code >> KXP_SH_SHIFT) & 31u;
+                const unsigned long long cc = ((unsigned long long)en.hd.w << 32) | en.hd.z;
+                uint32_t blocks[NCH];
+                const uint32_t *cwk = cwl + k * SW_GROUPS;
+#pragma unroll
+                for (int q = 0; q < NCH / 4; q++) {
+                    const uint4 w4 = *reinterpret_cast<const uint4 *>(cwk + cwo[q]);
                     const uint32_t w[4] = {w4.x, w4.y, w4.z, w4.w};
 #pragma unroll
-                    for (int q = 0; q < 4; q++)
-                        blocks[j + q] = (uint32_t)(((unsigned long long)w[q] * hd.x + cc) >> 32) >> sh;
+                    for (int t = 0; t < 4; t++)
+                        blocks[4 * q + t] = (uint32_t)(((unsigned long long)w[t] * en.hd.x + cc) >> 32);
+                }
+                if (sh) {   // (power-of-two ipb: none)
+#pragma unroll
+                    for (int j = 0; j < NCH; j++) blocks[j] >>= sh;
                 }
                 double tk[NCH];
-                if (cls == KXC_P2S0) cls_times<KXC_P2S0>(c01, c23, blocks, rfh, rfl, tk);
-                else if (cls == KXC_P2S) cls_times<KXC_P2S>(c01, c23, blocks, rfh, rfl, tk);
-                else if (cls == KXC_NS0) cls_times<KXC_NS0>(c01, c23, blocks, rfh, rfl, tk);
-                else cls_times<KXC_NS>(c01, c23, blocks, rfh, rfl, tk);
+                if (cls == KXC_P2S0) cls_times<KXC_P2S0>(en.c01, en.c23, blocks, rfh, rfl, tk);
+                else if (cls == KXC_P2S) cls_times<KXC_P2S>(en.c01, en.c23, blocks, rfh, rfl, tk);
+                else if (cls == KXC_NS0) cls_times<KXC_NS0>(en.c01, en.c23, blocks, rfh, rfl, tk);
+                else cls_times<KXC_NS>(en.c01, en.c23, blocks, rfh, rfl, tk);
                 if ((gk >> k) & 1u) {
                     // off the saturated path: the small-grid table (SKF_TABULATED)
                     bool any = false;
@@ -2264,12 +2426,23 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             };
             // sums in ascending kernel order (N6): the program lists the
             // per-iteration kernels, then the run-once ones; infeasible
-            // kernels are not listed (their sum is +inf through xinf)
-            uint32_t e = 0;
+            // kernels are not listed (their sum is +inf through xinf).  Two
+            // entries per step: the second's loads overlap the first's model.
+            auto run = [&](uint32_t e0, uint32_t e1, double (&acc)[NCH]) {
+                uint32_t e = e0;
+#if GROPHECY_EUNROLL == 2
 #pragma unroll 1
-            for (; e < n_it; e++) one_kernel(pe + e, ti);
+                for (; e + 1 < e1; e += 2) {
+                    const Ent a = load_ent(pe + e), b = load_ent(pe + e + 1);
+                    one_kernel(a, acc);
+                    one_kernel(b, acc);
+                }
+#endif
 #pragma unroll 1
-            for (; e < n_all; e++) one_kernel(pe + e, to);
+                for (; e < e1; e++) one_kernel(load_ent(pe + e), acc);
+            };
+            run(0, n_it, ti);
+            run(n_it, n_all, to);
             const double inf = __longlong_as_double(0x7ff0000000000000LL);
             if (xf & XINF_ITER) {
 #pragma unroll
@@ -2308,7 +2481,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             }
         }
         if (lane == 0) cnt_val += (uint32_t)CTILE;
+        PT_MARK(5);   // phase C (model, totals, argmin)
         tile = nt;
+        nt = nnt;
     }
     if (BEST) finish_best(P, sm.best_h + warp * 32, sm.best_d + warp * 32, lane, warp, best_t, best_i, 0u,
                           cnt_val, gridDim.x);
@@ -2692,6 +2867,25 @@ int grophecy_best(grophecy_space *s, const grophecy_pcie *pc, const grophecy_bat
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     if (e != cudaSuccess) return cuda_fail(e, "grophecy_best");
     return status_of(*host_out);
+}
+
+// Diagnostic builds (GROPHECY_PHASE_TIMING=1): copy out and reset the sweep
+// kernel's per-phase cycle sums (warp-cycles); ENOTSUP-like EINVAL otherwise.
+int grophecy_debug_phase_cycles(uint64_t *out8)
+{
+#if GROPHECY_PHASE_TIMING
+    if (!out8) return GROPHECY_EINVAL;
+    cudaError_t e = cudaMemcpyFromSymbol(out8, g_phase_cycles, 8 * sizeof(uint64_t));
+    if (e == cudaSuccess) {
+        static const unsigned long long zero[8] = {};
+        e = cudaMemcpyToSymbol(g_phase_cycles, zero, sizeof zero);
+    }
+    return e == cudaSuccess ? GROPHECY_OK : cuda_fail(e, "phase cycles");
+#else
+    (void)out8;
+    set_error("built without GROPHECY_PHASE_TIMING");
+    return GROPHECY_EINVAL;
+#endif
 }
 
 int grophecy_best_combine(const grophecy_best_result *din, uint32_t count,

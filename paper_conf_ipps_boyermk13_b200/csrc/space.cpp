@@ -543,12 +543,23 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 // the sweep kernel's program entry (internal.h KxProg)
                 KxProg c;
                 std::memset(&c, 0, sizeof c);
-                c.m = f.m;
-                c.satsh = f.satsh;
-                c.cc = f.cc;
-                c.k = k;
-                c.cls = KXC_NONE;
-                if (!(j.flags & KXF_INFEASIBLE) && sat != KXF_SAT_MASK) {
+                uint32_t pcls = KXC_NONE;
+                {
+                    // power-of-two ipb: no post-shift (m = 2^(32 - l))
+                    uint32_t psh = sh, pm = f.m;
+                    uint64_t pcc = f.cc;
+                    if (dv >= 2 && dv <= (1u << 30) && (dv & (dv - 1)) == 0) {
+                        uint32_t l = 0;
+                        while ((1u << l) < dv) l++;
+                        pm = 1u << (32 - l);
+                        pcc = (uint64_t)(dv - 1) * pm;
+                        psh = 0;
+                    }
+                    c.m = pm;
+                    c.cc = pcc;
+                    c.code = (sat & KXP_SAT_MASK) | psh << KXP_SH_SHIFT | k << KXP_K_SHIFT;
+                }
+                if (!(j.flags & KXF_INFEASIBLE) && sat != KXF_SAT_MASK && sat <= KXP_SAT_MASK) {
                     const bool p2 = f.rDl == 0.0, s0 = f.S == 0.0;
                     // blocks < sat <=> w <= (sat - 1) * ipb
                     const uint64_t ws = (uint64_t)(sat - 1) * dv + 1;
@@ -558,15 +569,16 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                     if (p2) {
                         c.c[0] = f.E * f.rDh;   // exact: rDh = 2^-k, E normal (fast_const_ok)
                         c.c[1] = f.S * f.rDh;
-                        c.cls = s0 ? KXC_P2S0 : KXC_P2S;
+                        pcls = s0 ? KXC_P2S0 : KXC_P2S;
                     } else {
                         c.c[0] = f.rDh;
                         c.c[1] = f.rDl;
                         c.c[2] = f.E;
                         c.c[3] = f.S;
-                        c.cls = s0 ? KXC_NS0 : KXC_NS;
+                        pcls = s0 ? KXC_NS0 : KXC_NS;
                     }
                 }
+                c.code |= (pcls & 7u) << KXP_CLS_SHIFT;
                 pair_prog[(size_t)x * S.n_kernels + k] = c;
             }
         // phase-C units in descending estimated cost (longest first: the
@@ -587,7 +599,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                     for (uint32_t k = 0; k < S.n_kernels; k++) {
                         const bool per = (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) != 0;
                         const KxProg &e = pair_prog[(size_t)x * S.n_kernels + k];
-                        if (per != (pass == 0) || e.cls == KXC_NONE) continue;
+                        if (per != (pass == 0) || (e.code >> KXP_CLS_SHIFT) == KXC_NONE) continue;
                         kprog.push_back(e);
                         (pass == 0 ? n_it : n_on)++;
                     }

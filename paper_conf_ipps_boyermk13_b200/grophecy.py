@@ -189,6 +189,7 @@ _sig = {
                                            C.POINTER(C.c_uint32), C.POINTER(C.c_uint32)]),
     "grophecy_plan_stats": (C.c_int, [C.POINTER(SkeletonDesc), C.POINTER(C.c_uint32)]),
     "grophecy_launch_count": (C.c_uint64, []),
+    "grophecy_debug_phase_cycles": (C.c_int, [C.POINTER(C.c_uint64)]),
     "grophecy_last_error": (C.c_char_p, []),
     "grophecy_abi_version": (C.c_int, []),
 }

@@ -1,0 +1,33 @@
+"""Per-phase time of the sweep kernel on C4 (diagnostic build with
+GROPHECY_PHASE_TIMING=1): warp-cycles per phase, summed over warps, as
+fractions.  usage: GROPHECY_PHASE_TIMING=1 python -m ...build --force;
+python scripts/phase_timing.py"""
+import ctypes as C
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import torch  # noqa: E402
+
+from paper_conf_ipps_boyermk13_b200 import grophecy as G  # noqa: E402
+from synth import records as R  # noqa: E402
+from synth import skeletons as S  # noqa: E402
+
+name = sys.argv[1] if len(sys.argv) > 1 else "c4"
+cfg = R.config(name)
+pc = G.pcie(G.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL))
+space = G.Space(cfg["skeletons"], S.FX5600)
+rec = G.synth_records(cfg)
+space.best(pc, rec)
+fn = G.lib().grophecy_debug_phase_cycles
+fn.argtypes = [C.POINTER(C.c_uint64)]
+out = (C.c_uint64 * 8)()
+fn(out)
+space.best(pc, rec)
+torch.cuda.synchronize()
+fn(out)
+names = ["wait records (TMA)", "phase A", "barrier 0", "phase B", "barrier 1", "phase C"]
+tot = sum(out[i] for i in range(6))
+for i, nm in enumerate(names):
+    print(f"{nm:22s} {100 * out[i] / tot:6.2f} %")
