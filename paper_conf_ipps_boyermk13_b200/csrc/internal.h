@@ -217,6 +217,7 @@ struct grophecy_space {
     int occ_canon;                       // pass-1 CTAs per SM (0 = not yet queried)
     int occ_sweep;                       // sweep-kernel CTAs per SM (0 = not yet queried)
     uint32_t usage_tbl_bytes;            // largest padded usage table (sweep shared memory)
+    bool counters_clean;                 // tile counters known zero (after a best projection)
     // group_best scratch (grown on demand)
     void *gscratch;
     size_t gscratch_bytes;

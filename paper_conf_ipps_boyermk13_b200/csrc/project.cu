@@ -24,6 +24,7 @@
 //
 // Compiled with -fmad=false: no contraction anywhere; FMAs appear only as the
 // explicit __fma_rn of the Markstein step.
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -1138,6 +1139,9 @@ struct Params {
     unsigned int *tile_count;
     uint32_t canon_warp_bytes; // pass 1: shared memory per warp (canon_warp_bytes(kmax))
     uint32_t sweep_kmax;       // sweep kernel: the space's largest kernel count (smem layout)
+    int direct;                // pass 2 takes every warp tile of the batch (no pass 1, no list)
+    int reset_counters;        // best mode: pass 2 leaves the tile counters zeroed for the next call
+    int fused;                 // best mode: the sweep kernel runs pass 2 itself (cooperative launch)
     // striped batches (grophecy_batch.stripe_len != 0): kernels work with
     // batch-local indices (base = the launch's local offset) and the final
     // best index is mapped to map_base + (i / map_len) * map_stride + i % map_len
@@ -1824,6 +1828,11 @@ __device__ __forceinline__ void finish_best(const Params &P, const unsigned long
             }
             to_result(*P.out, b);
             *P.ticket = 0u;
+            if (P.reset_counters) {   // pass 2 of best mode: every claim is done
+                P.tile_count[0] = 0u;
+                P.tile_count[CLAIM1] = 0u;
+                P.tile_count[CLAIM2] = 0u;
+            }
         }
     }
 }
@@ -1917,7 +1926,7 @@ constexpr unsigned long long SW_TILE = (unsigned long long)SW_GROUPS * CX;   // 
 #endif
 constexpr int NCH = GROPHECY_NCH;                                   // chains per lane (divides WARPS)
 constexpr int SW_UNITS = CX * (WARPS / NCH);                        // phase-C units (x, chain block)
-constexpr uint32_t SW_BAD = 0xffffffffu;
+constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_SMINB
 #define GROPHECY_SMINB 2
 #endif
@@ -1935,6 +1944,9 @@ constexpr uint32_t SW_BAD = 0xffffffffu;
 #endif
 #ifndef GROPHECY_PF
 #define GROPHECY_PF 0
+#endif
+#ifndef GROPHECY_FUSED
+#define GROPHECY_FUSED 1
 #endif
 // GROPHECY_PHASE_TIMING=1 (diagnostic builds only): per-warp clock64 time per
 // phase of the sweep kernel, summed into g_phase_cycles and read back by
@@ -2033,7 +2045,9 @@ __device__ __forceinline__ void issue_cta_copy(const Params &P, uint32_t (*rec)[
 {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     const uint32_t bar = smem_u32(rbar);
-    const uint32_t bytes = (uint32_t)(SW_TILE * sizeof(uint32_t));
+    // a full tile, or the batch's last one (a whole number of design points)
+    const unsigned long long nrec = P.n - tb < SW_TILE ? P.n - tb : SW_TILE;
+    const uint32_t bytes = (uint32_t)(nrec * sizeof(uint32_t));
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(4 * bytes)
                  : "memory");
     const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
@@ -2070,7 +2084,8 @@ __device__ __forceinline__ void issue_cta_copy_async(const Params &P, uint32_t (
 // and checks the canonical layout (skx = s0 ^ q, equal nx, ny, iters) and
 // validity; warp-uniform result.
 __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*recs)[SW_TILE], int warp,
-                                              int lane, uint32_t &s0, uint32_t &n0, uint32_t &m0, uint32_t &i0)
+                                              int lane, uint32_t gw, uint32_t &s0, uint32_t &n0, uint32_t &m0,
+                                              uint32_t &i0)
 {
     const uint32_t *rec[4] = {recs[0] + warp * CTILE, recs[1] + warp * CTILE, recs[2] + warp * CTILE,
                               recs[3] + warp * CTILE};
@@ -2105,6 +2120,20 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
     same(1, n0);
     same(2, m0);
     same(3, i0);
+    // the batch's last warp tile may hold gw < 32 design points: lanes past
+    // it stand in for design point 0 (their results are never used)
+    {
+        const uint32_t a0 = __shfl_sync(FULL, acc, 0), s00 = __shfl_sync(FULL, s0, 0);
+        const uint32_t n00 = __shfl_sync(FULL, n0, 0), m00 = __shfl_sync(FULL, m0, 0);
+        const uint32_t i00 = __shfl_sync(FULL, i0, 0);
+        if ((uint32_t)lane >= gw) {
+            acc = a0;
+            s0 = s00;
+            n0 = n00;
+            m0 = m00;
+            i0 = i00;
+        }
+    }
     const uint32_t skel = s0 >> 16;
     const uint32_t skel_l0 = __shfl_sync(FULL, skel, 0);
     bool ok = acc == 0 && skel < S.n_skels && n0 - 1u < GROPHECY_MAX_DIM &&
@@ -2156,8 +2185,15 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
     uint32_t cnt_val = 0;
     sm.best_h[tid] = 0;
     sm.best_d[tid] = 0;
+    // pass 2 may be scheduled now (it waits for this grid's completion)
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     // full CTA tiles of 16-byte aligned records (the TMA's alignment)
-    const unsigned long long ntiles = (P.aligned && !P.pr.mem) ? P.n / SW_TILE : 0ull;
+    // CTA tiles of 16-byte aligned records (the TMA's alignment): the full
+    // ones, plus the batch's last partial one when the batch is a whole
+    // number of design points (its missing warp tiles are empty)
+    const bool sweepable = P.aligned && !P.pr.mem;
+    const unsigned long long ntiles =
+        sweepable ? P.n / SW_TILE + ((P.n % SW_TILE) && (P.n % CX) == 0 ? 1ull : 0ull) : 0ull;
     // everything past them goes to pass 2 as warp tiles (warp-aggregated list appends)
     {
         const unsigned long long nsub = (P.n + CTILE - 1) / CTILE;
@@ -2215,8 +2251,12 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         phase ^= 1u;
 #endif
         PT_MARK(0);   // waiting for the staged records
-        uint32_t s0, n0, m0, i0;
-        bool ok = sweep_phase_a(S, sm.rec, warp, lane, s0, n0, m0, i0);
+        // design points of this tile, and of this warp's part of it
+        const uint32_t ngt = (uint32_t)((P.n - tile * SW_TILE < SW_TILE ? P.n - tile * SW_TILE : SW_TILE) / CX);
+        const int gwi = (int)ngt - 32 * warp;
+        const uint32_t gw = gwi <= 0 ? 0u : (gwi >= 32 ? 32u : (uint32_t)gwi);
+        uint32_t s0 = 0, n0 = 0, m0 = 0, i0 = 0;
+        bool ok = gw ? sweep_phase_a(S, sm.rec, warp, lane, gw, s0, n0, m0, i0) : false;
         const uint32_t skel = s0 >> 16;
         if (tid == 0) {
             // warp 0's skeleton decides the tile's usage table: stage it in
@@ -2329,16 +2369,17 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 sm.it[g] = (double)i0;
             }
         }
-        if (lane == 0) sm.wstat[warp] = ok ? skel : SW_BAD;
+        if (lane == 0) sm.wstat[warp] = gw == 0 ? SW_EMPTY : (ok ? skel : SW_BAD);
         PT_MARK(3);   // phase B (work counts, usage)
         __syncthreads();
         PT_MARK(4);   // barrier 1
+        // uniform: every non-empty warp tile canonical, of one skeleton
         const uint32_t s_all = sm.wstat[0];
-        bool uni = s_all != SW_BAD;
+        bool uni = s_all != SW_BAD && s_all != SW_EMPTY;
 #pragma unroll
-        for (int w = 1; w < WARPS; w++) uni &= sm.wstat[w] == s_all;
+        for (int w = 1; w < WARPS; w++) uni &= sm.wstat[w] == s_all || sm.wstat[w] == SW_EMPTY;
         if (!uni) {
-            if (lane == 0) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * WARPS + warp);
+            if (lane == 0 && gw) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * WARPS + warp);
             tile = nt;
             nt = nnt;
             continue;
@@ -2464,7 +2505,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 if (once) tk = __dadd_rn(to[j], tk);
                 const double tt = __dadd_rn(__dadd_rn(tk, sm.th[gj]), sm.td[gj]);
                 // chains in increasing record index: strict < keeps the lowest
-                if (tt < cmin) {
+                // (design points past a partial tile's end take no part)
+                if (tt < cmin && (uint32_t)gj < ngt) {
                     cmin = tt;
                     cj = j;
                 }
@@ -2480,13 +2522,41 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 }
             }
         }
-        if (lane == 0) cnt_val += (uint32_t)CTILE;
+        if (lane == 0) cnt_val += gw * (uint32_t)CX;
         PT_MARK(5);   // phase C (model, totals, argmin)
         tile = nt;
         nt = nnt;
     }
-    if (BEST) finish_best(P, sm.best_h + warp * 32, sm.best_d + warp * 32, lane, warp, best_t, best_i, 0u,
-                          cnt_val, gridDim.x);
+    if (!P.fused) {
+        if (BEST) finish_best(P, sm.best_h + warp * 32, sm.best_d + warp * 32, lane, warp, best_t, best_i, 0u,
+                              cnt_val, gridDim.x);
+        return;
+    }
+    // ---- pass 2 in the same (cooperative) launch: once every CTA has
+    // listed its tiles, the CTAs drain the list with the general 128-record
+    // tiles (claims from a counter), each lane's running best continuing ----
+    __syncthreads();
+    cooperative_groups::this_grid().sync();
+    const unsigned long long keep_h = sm.best_h[tid], keep_d = sm.best_d[tid];
+    __syncthreads();   // the sweep's shared memory becomes the general tiles'
+    WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
+    ws.best_h[lane] = keep_h;
+    ws.best_d[lane] = keep_d;
+    constexpr unsigned SUBS = CTILE / WTILE;
+    const unsigned units = *(volatile unsigned *)P.tile_count * SUBS;
+    unsigned *next = P.tile_count + CLAIM2;
+    uint32_t cnt_inv = 0;
+#pragma unroll 1
+    for (;;) {
+        unsigned q = 0;
+        if (lane == 0) q = atomicAdd(next, 1u);
+        q = __shfl_sync(FULL, q, 0);
+        if (q >= units) break;
+        const unsigned long long t0 = (unsigned long long)P.tile_list[q / SUBS] * CTILE +
+                                      (unsigned long long)(q % SUBS) * WTILE;
+        if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
+    }
+    if (BEST) finish_best(P, ws.best_h, ws.best_d, lane, warp, best_t, best_i, cnt_inv, cnt_val, gridDim.x);
 }
 
 // Pass 2: the listed tiles as general 128-record tiles (any layout).
@@ -2502,7 +2572,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
     uint32_t cnt_inv = 0, cnt_val = 0;
     ws.best_h[lane] = 0;
     ws.best_d[lane] = 0;
-    const unsigned count = *(volatile unsigned *)P.tile_count;
+    // launched programmatically dependent on pass 1 (best mode): wait until
+    // pass 1 has completed and its list / result are visible
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    const unsigned count = P.direct ? (unsigned)((P.n + CTILE - 1) / CTILE) : *(volatile unsigned *)P.tile_count;
     // only the blocks with listed tiles take part (none: pass 1's result and
     // outputs are final)
     // units of work: the listed tiles' 128-record sub-tiles, claimed one at a
@@ -2513,7 +2586,15 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
     constexpr unsigned SUBS = CTILE / WTILE;
     const unsigned units = count * SUBS;
     const unsigned nblocks = min(gridDim.x, (units + WARPS - 1) / WARPS);
-    if (blockIdx.x >= nblocks) return;
+    if (blockIdx.x >= nblocks) {
+        if (nblocks == 0 && blockIdx.x == 0 && threadIdx.x == 0) {
+            // nothing listed: pass 1 used only its tile claims; zero them here
+            if (P.reset_counters) P.tile_count[CLAIM1] = 0u;
+            // an empty direct batch: its (empty) result, unless merging
+            if (BEST && P.direct && !P.accumulate) to_result(*P.out, none_best());
+        }
+        return;
+    }
     unsigned *next = P.tile_count + CLAIM2;
 #pragma unroll 1
     for (;;) {
@@ -2521,7 +2602,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
         if (lane == 0) q = atomicAdd(next, 1u);
         q = __shfl_sync(FULL, q, 0);
         if (q >= units) break;
-        const unsigned long long t0 = (unsigned long long)P.tile_list[q / SUBS] * CTILE +
+        const unsigned long long t0 = (unsigned long long)(P.direct ? q / SUBS : P.tile_list[q / SUBS]) * CTILE +
                                       (unsigned long long)(q % SUBS) * WTILE;
         if (t0 < P.n) general_tile<BEST>(P, ws, t0, lane, best_t, best_i, cnt_inv, cnt_val);
     }
@@ -2552,7 +2633,8 @@ static void set_smem_attrs()
     cudaFuncSetAttribute(general_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     cudaFuncSetAttribute(general_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     cudaFuncSetAttribute(sweep_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)sweep_smem_bytes(MAXK, 2u * GROPHECY_MAX_ARRAYS * POLY_CLASSES * 16u));
+                         (int)std::max<uint32_t>(sweep_smem_bytes(MAXK, 2u * GROPHECY_MAX_ARRAYS * POLY_CLASSES * 16u),
+                                                 (uint32_t)sizeof(CtaSmem)));
     done = true;
 }
 
@@ -2584,6 +2666,13 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
 }
 
+// Dynamic shared memory of the (fused) sweep launch: its own layout, or the
+// general tiles' one after the grid barrier, whichever is larger.
+static uint32_t sweep_launch_smem(const grophecy_space *s)
+{
+    return std::max<uint32_t>(sweep_smem_bytes(s->max_kernels, s->usage_tbl_bytes), (uint32_t)sizeof(CtaSmem));
+}
+
 // Persistent grid of the sweep kernel: every SM full (occupancy per space:
 // its dynamic shared memory depends on the largest kernel count), at most one
 // CTA per CTA tile (at least one: it lists the tail for pass 2).
@@ -2592,11 +2681,10 @@ static int sweep_grid(const grophecy_space *s, unsigned long long n)
     set_smem_attrs();
     if (!s->occ_sweep) {
         int o = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, sweep_kernel<true>, THREADS,
-                                                      sweep_smem_bytes(s->max_kernels, s->usage_tbl_bytes));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, sweep_kernel<true>, THREADS, sweep_launch_smem(s));
         const_cast<grophecy_space *>(s)->occ_sweep = o < 1 ? 1 : o;
     }
-    const unsigned long long want = std::max<unsigned long long>(1ull, n / SW_TILE);
+    const unsigned long long want = std::max<unsigned long long>(1ull, (n + SW_TILE - 1) / SW_TILE);
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)s->occ_sweep;
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::min(want, cap);
@@ -2633,22 +2721,79 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         } else if (off) {
             Q.accumulate = 1;
         }
-        cudaError_t e = cudaMemsetAsync(Q.tile_count, 0, (std::max(CLAIM1, CLAIM2) + 1) * sizeof(unsigned int), st);   // count + claim counters
-        if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(tile count)");
+        // count + claim counters: zero after space creation and after every
+        // best projection (its pass 2 resets them); eval leaves them dirty
+        grophecy_space *sm_ = const_cast<grophecy_space *>(s);
+        cudaError_t e = cudaSuccess;
+        if (!BEST || !sm_->counters_clean) {
+            e = cudaMemsetAsync(Q.tile_count, 0, (std::max(CLAIM1, CLAIM2) + 1) * sizeof(unsigned int), st);
+            if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(tile count)");
+        }
         const int grid = grid_for(s, Q.n, 32, false);
         Q.canon_warp_bytes = canon_warp_bytes(s->max_kernels);
-        if (BEST) {
-            // pass 1: CTA sweep tiles (canonical layouts, one skeleton per tile)
+        Q.reset_counters = 0;   // (pass 2 only, below: pass 1's list must survive pass 1)
+        // batches the sweep takes nothing of (unaligned, the memory choice) and
+        // batches smaller than one tile (pass 2 alone is quicker) go to pass 2 whole
+        Q.direct = BEST && !(Q.aligned && !Q.pr.mem && Q.n >= SW_TILE);
+        int launches = 1;
+        Q.fused = 0;
+        if (BEST && !Q.direct && GROPHECY_FUSED) {
+            // passes 1 and 2 in one cooperative launch: CTA sweep tiles
+            // (canonical layouts, one skeleton per tile), a grid barrier, then
+            // the listed tiles on the general path
             const int grid_s = sweep_grid(s, Q.n);
             Q.sweep_kmax = s->max_kernels;
-            sweep_kernel<true><<<grid_s, THREADS, sweep_smem_bytes(s->max_kernels, s->usage_tbl_bytes), st>>>(Q);
-        } else {
+            Q.fused = 1;
+            Q.reset_counters = 1;
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(grid_s);
+            cfg.blockDim = dim3(THREADS);
+            cfg.dynamicSmemBytes = sweep_launch_smem(s);
+            cfg.stream = st;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeCooperative;
+            attr[0].val.cooperative = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            e = cudaLaunchKernelEx(&cfg, sweep_kernel<true>, Q);
+            if (e != cudaSuccess) return cuda_fail(e, "projection (best) sweep launch");
+            sm_->counters_clean = true;
+            count_launch(1);
+            off += Q.n;
+            continue;
+        } else if (BEST && !Q.direct) {
+            // pass 1 alone (pass 2 launched below, programmatically dependent)
+            const int grid_s = sweep_grid(s, Q.n);
+            Q.sweep_kmax = s->max_kernels;
+            sweep_kernel<true><<<grid_s, THREADS, sweep_launch_smem(s), st>>>(Q);
+            launches++;
+        } else if (!BEST) {
             const int grid_c = grid_for(s, Q.n, 32, true);
             canon_kernel<BEST><<<grid_c, THREADS, WARPS * Q.canon_warp_bytes, st>>>(Q);
+            launches++;
         }
-        Q.accumulate = BEST ? 1 : 0;   // pass 2 merges into pass 1's result
-        general_kernel<BEST><<<grid, THREADS, sizeof(CtaSmem), st>>>(Q);
-        count_launch(2);
+        if (!(BEST && Q.direct)) Q.accumulate = BEST ? 1 : 0;   // pass 2 merges into pass 1's result
+        if (BEST) {
+            Q.reset_counters = 1;
+            // programmatic dependent launch: pass 2's launch overlaps pass 1
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(grid);
+            cfg.blockDim = dim3(THREADS);
+            cfg.dynamicSmemBytes = sizeof(CtaSmem);
+            cfg.stream = st;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            attr[0].val.programmaticStreamSerializationAllowed = Q.direct ? 0 : 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            e = cudaLaunchKernelEx(&cfg, general_kernel<true>, Q);
+            if (e != cudaSuccess) return cuda_fail(e, "projection (best) pass 2 launch");
+            sm_->counters_clean = true;
+        } else {
+            general_kernel<BEST><<<grid, THREADS, sizeof(CtaSmem), st>>>(Q);
+            sm_->counters_clean = false;
+        }
+        count_launch(launches);
         e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_fail(e, BEST ? "projection (best) launch" : "projection (eval) launch");
         off += Q.n;

@@ -51,8 +51,30 @@ def timed(fn, reps, events=True):
     return (time.perf_counter() - t0) / reps
 
 
+def latency(pc, reps=200):
+    """Per-query time of small batches (C1: 16 records, C2: 10^6): the fused
+    best into device memory (CUDA events, back to back) and the synchronous
+    grophecy_best (host clock, result on the host)."""
+    out = torch.empty(6, dtype=torch.int64, device="cuda")
+    for wname in ("c1", "c2"):
+        wc = R.config(wname)
+        wsp = G.Space(wc["skeletons"], S.FX5600)
+        wrec = G.synth_records(wc)
+        wb = wrec.batch()
+        sec = timed(lambda: wsp.best_async(pc, wb, out), reps, True)
+        sec_sync = timed(lambda: wsp.best(pc, wrec), reps, False)
+        print(json.dumps({"mode": "latency", "workload": wname, "n": wrec.n,
+                          "us_per_query_async": sec * 1e6, "us_per_query_sync": sec_sync * 1e6,
+                          "cand_per_s": wrec.n / sec,
+                          "launches_per_query": None}), flush=True)
+        wsp.close()
+
+
 def main():
     n = int(sys.argv[1]) if len(sys.argv) > 1 else 1 << 27
+    if os.environ.get("LATENCY_ONLY"):
+        latency(G.pcie(G.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL)))
+        return
     reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
     cfg = R.config("c4")
     space = G.Space(cfg["skeletons"], S.FX5600)
