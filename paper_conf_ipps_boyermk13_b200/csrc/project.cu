@@ -1,29 +1,33 @@
 // The projection hot path for sm_100a: grophecy_eval[_parts|_mem] /
 // grophecy_best[_async|_mem|_host] / grophecy_best_combine.
 //
-// Two persistent launches per call.  Pass 1 (canon_kernel): every warp works
-// alone on canonical tiles of 512 records = 32 design points x 16
-// transformations of one skeleton, staged in shared memory by 1-D TMA bulk
-// copies one tile ahead; lane = design point computes the kernels' work
-// counts and the data usage once per design point from the skeleton's
-// residue-class byte polynomials (plan.cpp; usage depends only on the key
-// (skeleton, nx, ny), reading 11); then lane = (transformation,
-// half) models 8 design points per pass with one constant load per kernel.
-// Tiles that are not canonical (any other layout, ragged tails, invalid
-// records, keys off the polynomial domain, strided / hull / rank-3
-// skeletons, huge work counts) go to a list for pass 2 (general_kernel):
-// 128-record warp tiles, runs of equal keys, usage per distinct key (plans,
-// else the warp-cooperative coordinate-compressed sweep or the HK hull), the
-// model per record.  The kernel-time model runs from per-(kernel,
-// transformation) constants the host precomputed in the definition's
-// operation order; on saturated grids the two remaining IEEE divisions use
-// Markstein's correction (q = a*rb; r = fma(-q, b, a); q' = fma(r, rb, q)),
-// correctly rounded when rb = RN(1/b), i.e. bitwise a / b; small grids come
-// from a table computed step by step at space creation.  Best mode fuses the
-// argmin (lane -> warp -> CTA -> grid, last-block pattern).
+// Best mode: one cooperative launch of sweep_kernel.  CTA sweep tiles of
+// 4096 records = 256 design points x 16 transformations of one skeleton are
+// staged in shared memory by TMA bulk copies one tile ahead; per warp (lane =
+// design point) phase A checks the canonical layout, phase B computes the
+// kernels' work counts and the data usage from the skeleton's residue-class
+// byte polynomials (plan.cpp; usage depends only on (skeleton, nx, ny),
+// DESIGN.md reading 11) staged in shared memory; then CTA-wide phase C: a
+// warp takes a transformation and its lanes run its program (the feasible
+// kernels in summation order, each with its class of the saturated model) on
+// 8 design points each, so every (kernel, transformation) record and code
+// path is warp-uniform.  Tiles that are not canonical (any other layout,
+// mixed skeletons, keys off the polynomial domain, strided / hull / rank-3
+// skeletons, huge work counts) are listed and, after a grid barrier, drained
+// by the same CTAs with general_tile: 128-record warp tiles, runs of equal
+// keys, usage per distinct key (plans, else the warp-cooperative
+// coordinate-compressed sweep or the HK hull), the model per record.  Eval
+// mode: canon_kernel (warp tiles, lane = (transformation, half), coalesced
+// stores) then general_kernel over the list.  The kernel-time model runs from
+// per-(kernel, transformation) constants the host precomputed in the
+// definition's operation order; on saturated grids the two remaining IEEE
+// divisions use the two-product method (x * zh + RN(x * zl), exact for the
+// divisors used: space.cpp div2_ok), small grids come from a table computed
+// step by step at space creation.  Best mode fuses the argmin (lane -> warp
+// -> CTA -> grid, last-block pattern).
 //
 // Compiled with -fmad=false: no contraction anywhere; FMAs appear only as the
-// explicit __fma_rn of the Markstein step.
+// explicit __fma_rn of the divisions.
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -2581,8 +2585,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_MINB) general_kernel(const P
     // units of work: the listed tiles' 128-record sub-tiles, claimed one at a
     // time from a counter (P.tile_count[CLAIM2], zeroed with the tile count
     // before pass 1): the per-tile cost of the general sweep varies by orders of
-    // magnitude, so a static split leaves warps idle at the end.  One warp's
-    // claims increase, so its records still come in increasing index order.
+    // magnitude, so a static split leaves warps idle at the end.  The list
+    // is appended in any order (atomics across CTAs), so a warp meets its
+    // records in arbitrary index order: general_tile's running best must (and
+    // does) compare (t, index) lexicographically, never by t alone.
     constexpr unsigned SUBS = CTILE / WTILE;
     const unsigned units = count * SUBS;
     const unsigned nblocks = min(gridDim.x, (units + WARPS - 1) / WARPS);
@@ -2628,7 +2634,6 @@ static void set_smem_attrs()
     bool &done = done_dev[dev & 63];
     if (done) return;
     const int sm = (int)sizeof(CtaSmem), cs = (int)(WARPS * canon_warp_bytes(MAXK));
-    cudaFuncSetAttribute(canon_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
     cudaFuncSetAttribute(canon_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
     cudaFuncSetAttribute(general_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     cudaFuncSetAttribute(general_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
@@ -2647,7 +2652,7 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
         // per space: its dynamic shared memory depends on its kernel count
         if (!s->occ_canon) {
             int o = 0;
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, canon_kernel<true>, THREADS,
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, canon_kernel<false>, THREADS,
                                                           WARPS * canon_warp_bytes(s->max_kernels));
             const_cast<grophecy_space *>(s)->occ_canon = o < 1 ? 1 : o;
         }
@@ -2769,7 +2774,7 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
             launches++;
         } else if (!BEST) {
             const int grid_c = grid_for(s, Q.n, 32, true);
-            canon_kernel<BEST><<<grid_c, THREADS, WARPS * Q.canon_warp_bytes, st>>>(Q);
+            canon_kernel<false><<<grid_c, THREADS, WARPS * Q.canon_warp_bytes, st>>>(Q);
             launches++;
         }
         if (!(BEST && Q.direct)) Q.accumulate = BEST ? 1 : 0;   // pass 2 merges into pass 1's result
