@@ -172,11 +172,13 @@ struct SpaceDev {
     const KxJ *kx_j;
     const KxG *kx_g;
     const KxFast *kx_f;
-    // sweep kernel: per (skeleton, unit u) at kx_base + u (units in
-    // descending estimated cost) {x, first program entry, n_iter | n_once <<
-    // 16, xinf bits}; the programs' entries
+    // sweep kernel: per (skeleton, xform x) at kx_base + x the program
+    // header {x, first entry, n_iter | n_once << 16, xinf bits | cost << 8}
+    // (cost: estimated work, for the phase-C claim order); the programs
     const uint4 *xhdr;
     const KxProg *xprog;
+    const uint32_t *xord;       // per (skeleton, unit u) at kx_base + u: xforms by descending cost
+    const uint4 *xhdru;         // xhdr in that order (one load per unit in the identity layout)
     const unsigned long long *poly;   // usage byte polynomials (all skeletons)
     // small-grid kernel times: small_t[kxi * small_stride + blocks] for
     // blocks < sat32 when sat32 <= small_stride (space.cpp small_grid_time)

@@ -1952,6 +1952,9 @@ constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_FUSED
 #define GROPHECY_FUSED 1
 #endif
+#ifndef GROPHECY_PERM
+#define GROPHECY_PERM 1
+#endif
 // GROPHECY_PHASE_TIMING=1 (diagnostic builds only): per-warp clock64 time per
 // phase of the sweep kernel, summed into g_phase_cycles and read back by
 // grophecy_debug_phase_cycles (scripts/phase_timing.py)
@@ -1987,6 +1990,9 @@ struct alignas(128) SweepSmem {
     uint32_t tbl_skel;           // skeleton whose usage table is staged (SW_BAD: none)
     uint32_t tbl_wait;           // this tile: parity to wait for on tbar, or SW_BAD (no copy)
     uint32_t tbl_phase;          // parity of the next tbar completion
+    uint32_t perm[CX];           // this tile's skx at each position of a design point (its first one's)
+    uint32_t perm_ident;         // perm is the identity (claims follow the cost order)
+    uint32_t perm_ok;            // the tile's first design point is consistent (one skeleton, valid xforms)
 };
 // followed by the work counts cw[k][lane][8] (uint32, w_store; design point
 // g = 32 j + lane at chunk (j / 4) ^ ((lane / 4) & 1), so a phase-C lane reads
@@ -2083,10 +2089,13 @@ __device__ __forceinline__ void issue_cta_copy_async(const Params &P, uint32_t (
     asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(rbar)) : "memory");
 }
 
-// Phase A of one warp tile staged at rec (full: 32 design points): lane l
-// reads its design point's 16 records (rotated 16-byte chunks, conflict-free)
-// and checks the canonical layout (skx = s0 ^ q, equal nx, ny, iters) and
-// validity; warp-uniform result.
+// Phase A of one warp tile of the CTA tile staged at recs: lane l reads its
+// design point's 16 records (rotated 16-byte chunks, conflict-free) and
+// checks the layout of a sweep: every design point of the CTA tile holds 16
+// records of one skeleton with equal nx, ny, iters, and the transformations
+// in the same order as the tile's first design point (any fixed order of
+// valid transformations); warp-uniform result.  The batch's last warp tile
+// may hold gw < 32 design points: lanes past it stand in for design point 0.
 __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*recs)[SW_TILE], int warp,
                                               int lane, uint32_t gw, uint32_t &s0, uint32_t &n0, uint32_t &m0,
                                               uint32_t &i0)
@@ -2097,6 +2106,23 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
     const uint32_t r = ((uint32_t)lane >> 1) & 3u;
     {
         const uint4 *p = reinterpret_cast<const uint4 *>(rec[0] + lane * CX);
+#if GROPHECY_PERM
+        const uint4 *g = reinterpret_cast<const uint4 *>(recs[0]);   // the tile's first design point
+        uint4 v[CX / 4], w[CX / 4];
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++) {
+            v[m] = p[(m + r) & 3u];
+            w[m] = g[(m + r) & 3u];
+        }
+        s0 = v[0].x;
+        acc = 0;
+        // equal to the tile's first design point record by record (whose own
+        // consistency — one skeleton, valid transformations — warp 0 checks
+        // once per tile: SweepSmem::perm_ok)
+#pragma unroll
+        for (int m = 0; m < CX / 4; m++)
+            acc |= (v[m].x ^ w[m].x) | (v[m].y ^ w[m].y) | (v[m].z ^ w[m].z) | (v[m].w ^ w[m].w);
+#else
         uint4 v[CX / 4];
 #pragma unroll
         for (int m = 0; m < CX / 4; m++) v[m] = p[(m + r) & 3u];
@@ -2110,6 +2136,7 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
             acc |= (v[m].z ^ s0) ^ (c4 + 2u);
             acc |= (v[m].w ^ s0) ^ (c4 + 3u);
         }
+#endif
     }
     auto same = [&](int arr, uint32_t &first) {
         const uint4 *p = reinterpret_cast<const uint4 *>(rec[arr] + lane * CX);
@@ -2124,8 +2151,6 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
     same(1, n0);
     same(2, m0);
     same(3, i0);
-    // the batch's last warp tile may hold gw < 32 design points: lanes past
-    // it stand in for design point 0 (their results are never used)
     {
         const uint32_t a0 = __shfl_sync(FULL, acc, 0), s00 = __shfl_sync(FULL, s0, 0);
         const uint32_t n00 = __shfl_sync(FULL, n0, 0), m00 = __shfl_sync(FULL, m0, 0);
@@ -2142,7 +2167,7 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
     const uint32_t skel_l0 = __shfl_sync(FULL, skel, 0);
     bool ok = acc == 0 && skel < S.n_skels && n0 - 1u < GROPHECY_MAX_DIM &&
               m0 - 1u < GROPHECY_MAX_DIM && i0 >= 1 && skel == skel_l0;
-    if (ok) ok = S.skel[skel].n_xforms >= (uint32_t)CX && (S.skel[skel].flags & SKF_TABULATED);
+    if (ok) ok = (S.skel[skel].flags & SKF_TABULATED) != 0;
     return __all_sync(FULL, ok);
 }
 
@@ -2291,6 +2316,16 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         // every read of the staged tile is done (phase A): it takes the next
         // one, and the tile after that is prefetched into L2
         const unsigned long long nnt = sm.next_tile;
+        uint32_t sq = 0;
+        if (tid < CX) {
+            // the tile's transformation order (its first design point's skx),
+            // read before the buffer is refilled (checked in phase B: perm_ok)
+            sq = sm.rec[0][tid];
+            sm.perm[tid] = sq;
+            const unsigned bad = __ballot_sync(0xffffu, (sq & 0xffffu) != (uint32_t)tid);
+            if (tid == 0) sm.perm_ident = bad == 0u;
+        }
+        __syncwarp();
 #if GROPHECY_LDGSTS
         if (nt < ntiles) issue_cta_copy_async(P, sm.rec, &sm.rbar, nt * SW_TILE, tid);
 #endif
@@ -2343,6 +2378,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 small |= (w < __ldg(&S.kern_wsat[I.k_base + k]) ? 1u : 0u) << k;
             }
             sm.smallk[g] = small;
+            if (warp == 0) {
+                // the tile's first design point (lane 0's) is itself consistent:
+                // one skeleton, every transformation < n_xforms
+                const bool okq = (uint32_t)lane >= CX || ((sq >> 16) == skel && (sq & 0xffffu) < I.n_xforms);
+                const bool all = __all_sync(FULL, okq);
+                if (lane == 0) sm.perm_ok = all;
+            }
             ok = !__any_sync(FULL, huge) && __all_sync(FULL, n0 >= I.plan_tx && m0 >= I.plan_ty);
             if (ok) {
                 Usage u = {0ull, 0ull, 0.0, 0.0};
@@ -2374,12 +2416,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             }
         }
         if (lane == 0) sm.wstat[warp] = gw == 0 ? SW_EMPTY : (ok ? skel : SW_BAD);
+        if (tid == 0 && !ok) sm.perm_ok = 0u;   // (warp 0 skipped its check; the tile is not uniform)
         PT_MARK(3);   // phase B (work counts, usage)
         __syncthreads();
         PT_MARK(4);   // barrier 1
         // uniform: every non-empty warp tile canonical, of one skeleton
         const uint32_t s_all = sm.wstat[0];
-        bool uni = s_all != SW_BAD && s_all != SW_EMPTY;
+        bool uni = s_all != SW_BAD && s_all != SW_EMPTY && sm.perm_ok;
 #pragma unroll
         for (int w = 1; w < WARPS; w++) uni &= sm.wstat[w] == s_all || sm.wstat[w] == SW_EMPTY;
         if (!uni) {
@@ -2399,9 +2442,19 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             if (lane == 0) u = atomicAdd(&sm.unit, 1u);
             u = __shfl_sync(FULL, u, 0);
             if (u >= (unsigned)SW_UNITS) break;
-            // the unit's transformation and its program (header in unit order)
-            const uint4 hdr = __ldg(&S.xhdr[I.kx_base + u % CX]);
-            const uint32_t x = hdr.x, jb = u / CX, xf = hdr.w;
+            // the unit's position in the design points and its transformation:
+            // in the identity layout by descending cost, else in position order
+            uint4 hdr;
+            uint32_t pos;
+            if (sm.perm_ident) {
+                hdr = __ldg(&S.xhdru[I.kx_base + u % CX]);
+                pos = hdr.x;
+            } else {
+                pos = u % CX;
+                hdr = __ldg(&S.xhdr[I.kx_base + (sm.perm[pos] & 0xffffu)]);
+            }
+            const uint32_t x = hdr.x;
+            const uint32_t jb = u / CX, xf = hdr.w & 0xffu;
             const KxProg *pe = S.xprog + hdr.y;
             const uint32_t n_it = hdr.z & 0xffffu, n_all = n_it + (hdr.z >> 16);
             // kernels whose grid may be unsaturated for one of the warp's design points
@@ -2517,7 +2570,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             }
             if (cj >= 0) {
                 const int gj = 32 * ((int)jb * NCH + cj) + lane;
-                const unsigned long long idx = tbase + (unsigned long long)gj * CX + x;
+                const unsigned long long idx = tbase + (unsigned long long)gj * CX + pos;
                 if (better(cmin, idx, best_t, best_i)) {
                     best_t = cmin;
                     best_i = idx;

@@ -345,7 +345,9 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<KxG> kg;
     std::vector<KxFast> kf;
     std::vector<KxProg> kprog;    // sweep-kernel programs (all skeletons)
-    std::vector<uint4> xhdr;      // per (skeleton, unit) at kx_base + u: program header
+    std::vector<uint4> xhdr;      // per (skeleton, xform) at kx_base + x: program header
+    std::vector<uint32_t> xord;   // per (skeleton, unit) at kx_base + u: xforms by descending cost
+    std::vector<uint4> xhdru;     // the headers in that order
     std::vector<uint32_t> kwsat;  // per (skeleton, kernel): work count saturating every xform
     std::vector<uint32_t> xinf;   // per (skeleton, xform) at kx_base + x: XINF_* bits
     // the fast path divides by freq with the two-product method: without it
@@ -493,6 +495,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         std::vector<double> xcost(S.n_xforms, 0.0);
         xinf.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, 0u);
         xhdr.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, make_uint4(0u, 0u, 0u, 0u));
+        xord.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, 0u);
+        xhdru.resize(kx0 + (size_t)S.n_kernels * S.n_xforms, make_uint4(0u, 0u, 0u, 0u));
         std::vector<KxProg> pair_prog((size_t)S.n_kernels * S.n_xforms);
         for (uint32_t k = 0; k < S.n_kernels; k++)
             for (uint32_t x = 0; x < S.n_xforms; x++) {
@@ -581,29 +585,34 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 c.code |= (pcls & 7u) << KXP_CLS_SHIFT;
                 pair_prog[(size_t)x * S.n_kernels + k] = c;
             }
-        // phase-C units in descending estimated cost (longest first: the
-        // CTA's warps finish together)
+        // per transformation: its program header (at kx_base + x) and program
+        // (feasible saturated-capable kernels, per-iteration ones then run-once
+        // ones, each in ascending kernel order: N6); the header carries an
+        // estimated cost for the phase-C claim order (longest first)
+        for (uint32_t x = 0; x < S.n_xforms; x++) {
+            const uint32_t first = (uint32_t)kprog.size();
+            uint32_t n_it = 0, n_on = 0;
+            for (int pass = 0; pass < 2; pass++)
+                for (uint32_t k = 0; k < S.n_kernels; k++) {
+                    const bool per = (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) != 0;
+                    const KxProg &e = pair_prog[(size_t)x * S.n_kernels + k];
+                    if (per != (pass == 0) || (e.code >> KXP_CLS_SHIFT) == KXC_NONE) continue;
+                    kprog.push_back(e);
+                    (pass == 0 ? n_it : n_on)++;
+                }
+            const uint32_t cost = (uint32_t)std::min(xcost[x], 16777215.0);
+            xhdr[kx0 + x] = make_uint4(x, first, n_it | n_on << 16, xinf[kx0 + x] | cost << 8);
+        }
+        // phase-C claim order of the transformations (longest first: the CTA's
+        // warps finish together)
         {
             std::vector<uint32_t> ord(S.n_xforms);
             for (uint32_t x = 0; x < S.n_xforms; x++) ord[x] = x;
             std::stable_sort(ord.begin(), ord.end(),
                              [&](uint32_t a, uint32_t b) { return xcost[a] > xcost[b]; });
-            // per unit: the header and the program of its transformation
-            // (feasible saturated-capable kernels, per-iteration ones then
-            // run-once ones, each in ascending kernel order: N6)
             for (uint32_t u = 0; u < S.n_xforms; u++) {
-                const uint32_t x = ord[u];
-                const uint32_t first = (uint32_t)kprog.size();
-                uint32_t n_it = 0, n_on = 0;
-                for (int pass = 0; pass < 2; pass++)
-                    for (uint32_t k = 0; k < S.n_kernels; k++) {
-                        const bool per = (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) != 0;
-                        const KxProg &e = pair_prog[(size_t)x * S.n_kernels + k];
-                        if (per != (pass == 0) || (e.code >> KXP_CLS_SHIFT) == KXC_NONE) continue;
-                        kprog.push_back(e);
-                        (pass == 0 ? n_it : n_on)++;
-                    }
-                xhdr[kx0 + u] = make_uint4(x, first, n_it | n_on << 16, xinf[kx0 + x]);
+                xord[kx0 + u] = ord[u];
+                xhdru[kx0 + u] = xhdr[kx0 + ord[u]];
             }
         }
     }
@@ -649,6 +658,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {kprog.data(), kprog.size() * sizeof(KxProg), 0},
         {xhdr.data(), xhdr.size() * sizeof(uint4), 0},
         {kwsat.data(), kwsat.size() * sizeof(uint32_t), 0},
+        {xord.data(), xord.size() * sizeof(uint32_t), 0},
+        {xhdru.data(), xhdru.size() * sizeof(uint4), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -713,6 +724,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.xprog = (const KxProg *)(base + parts[14].off);
     D.xhdr = (const uint4 *)(base + parts[15].off);
     D.kern_wsat = (const uint32_t *)(base + parts[16].off);
+    D.xord = (const uint32_t *)(base + parts[17].off);
+    D.xhdru = (const uint4 *)(base + parts[18].off);
     D.small_stride = small_stride;
     D.n_skels = n_skels;
     D.n_sm = gpu->n_sm;

@@ -11,7 +11,9 @@ import os
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libgrophecy.so")
+# GROPHECY_LIB: an alternative in-tree build of the same library (A/B
+# measurements of build variants, scripts/ab_lib.sh)
+LIB_PATH = os.environ.get("GROPHECY_LIB") or os.path.join(HERE, "libgrophecy.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

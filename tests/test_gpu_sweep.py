@@ -1,0 +1,77 @@
+"""The sweep path's layout cases: design points of 16 records
+in any fixed transformation order, the batch's last partial tile, mixed
+orders (the tile falls back to the general path), all against the oracle.
+Best and eval are compared record by record / by argmin; index_base and
+ragged sizes exercised."""
+import numpy as np
+import pytest
+
+from synth import records as R
+from synth import skeletons as S
+from tests.gpu_helpers import assert_same, gpu_eval, oracle_problem, paper_pcie
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def G():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_boyermk13_b200 import build
+    build.build()
+    from paper_conf_ipps_boyermk13_b200 import grophecy
+    torch.cuda.set_device(0)
+    return grophecy
+
+
+def check(G, O, skels, rec, index_base=0):
+    pc = paper_pcie(G)
+    space = G.Space(skels, S.FX5600)
+    P = oracle_problem(O, skels)
+    assert_same(gpu_eval(G, space, pc, rec, index_base), P.eval(rec))
+    rc, b = space.best(pc, G.Records.from_numpy(rec), index_base=index_base)
+    orc, ob = P.best(rec, index_base=index_base)
+    assert (b.index, b.n_valid, b.n_invalid) == (ob.index, ob.n_valid, ob.n_invalid)
+    assert b.t_total_s == ob.t_total_s and (b.h2d_bytes, b.d2h_bytes) == (ob.h2d_bytes, ob.d2h_bytes)
+    space.close()
+
+
+def permuted(rec, perm):
+    """Reorder the 16 records of every design point by `perm` (positions)."""
+    n = len(rec["skx"])
+    idx = (np.arange(n) // 16) * 16 + np.asarray(perm)[np.arange(n) % 16]
+    return {k: v[idx] for k, v in rec.items()}
+
+
+@pytest.mark.parametrize("order", ["reversed", "random", "repeat"])
+def test_fixed_transformation_order(G, O, order):
+    c = R.config("c4")
+    n = 3 * 4096 + 16 * 37            # three full CTA tiles and a partial one
+    base = 16 * 1000
+    rec = R.gen_records(c, base, base + n)
+    rng = np.random.default_rng(17)
+    perm = {"reversed": np.arange(16)[::-1], "random": rng.permutation(16),
+            "repeat": np.array([0, 3, 3, 1, 15, 2, 7, 7, 4, 5, 6, 8, 9, 10, 11, 12])}[order]
+    check(G, O, c["skeletons"], permuted(rec, perm), index_base=base)
+
+
+def test_mixed_orders_fall_back(G, O):
+    """One design point in a different order: its CTA tile is not a sweep
+    tile (general path); the others still are."""
+    c = R.config("c4")
+    n = 4 * 4096
+    rec = R.gen_records(c, 0, n)
+    rec = permuted(rec, np.arange(16)[::-1])
+    i = 4096 + 16 * 5                  # one design point of tile 1 in natural order
+    for k in rec:
+        rec[k][i:i + 16] = rec[k][i:i + 16][::-1]
+    check(G, O, c["skeletons"], rec)
+
+
+@pytest.mark.parametrize("n", [4096 + 16, 8192 - 16, 4096 * 5 + 16 * 255, 4096 * 2 + 7])
+def test_partial_last_tile(G, O, n):
+    c = R.config("c4")
+    start = 16 * 62_500_000 // 16     # inside the skeleton-major ranges
+    rec = R.gen_records(c, start, start + n)
+    check(G, O, c["skeletons"], rec, index_base=start)
