@@ -62,14 +62,17 @@ inline uint32_t kxf_sat(const KxFast &f) { return f.satsh & KXF_SAT_MASK; }
 // infeasible kernels are left out: their sum is +inf through xinf).
 enum : uint32_t { KXC_P2S0 = 0u, KXC_P2S = 1u, KXC_NS0 = 2u, KXC_NS = 3u, KXC_NONE = 4u };
 // blocks = hi32(w m + cc) >> sh (as KxFast; a power-of-two ipb = 2^l uses
-// m = 2^(32 - l), cc = (ipb - 1) m, sh = 0); code = sat | sh << 11 | k << 16
-// | cls << 21 (sat <= SMALL_GRID_MAX: the sweep path requires tabulated pairs).
+// m = 2^(32 - l), cc = (ipb - 1) m, sh = 0); the kernel as its work-count
+// offset cwoff = k * 256 (sweep shared memory) and its bit kbit = 1 << k;
+// sat <= SMALL_GRID_MAX (the sweep path requires tabulated pairs).  Fields
+// unpacked: 64 bytes, four 16-byte loads, no decoding.
 struct __align__(16) KxProg {
-    uint32_t m, code;
+    uint32_t m, sat;
     uint64_t cc;
+    uint32_t cwoff, sh, kbit, cls;
     double c[4];
 };
-constexpr uint32_t KXP_SAT_MASK = 0x7ffu, KXP_SH_SHIFT = 11, KXP_K_SHIFT = 16, KXP_CLS_SHIFT = 21;
+constexpr uint32_t KXP_SAT_MAX = 0x7ffu;
 
 // General-grid constants (small grids / huge W), read only off the fast path.
 struct KxG {

@@ -1937,9 +1937,6 @@ constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_I2F_MAGIC
 #define GROPHECY_I2F_MAGIC 0
 #endif
-#ifndef GROPHECY_EUNROLL
-#define GROPHECY_EUNROLL 1
-#endif
 #ifndef GROPHECY_LDGSTS
 #define GROPHECY_LDGSTS 0
 #endif
@@ -2471,25 +2468,26 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
 #pragma unroll
             for (int q = 0; q < NCH / 4; q++)
                 cwo[q] = ((((jb * NCH) / 4 + (uint32_t)q) ^ ((uint32_t)lane >> 2)) & 1u) << 2;
+            static_assert(SW_GROUPS == 256, "KxProg::cwoff = k * 256");
             struct Ent {
-                uint4 hd;
+                uint4 hd, kw;
                 double2 c01, c23;
             };
             auto load_ent = [&](const KxProg *e) {
                 const uint4 *q = reinterpret_cast<const uint4 *>(e);
                 Ent r;
                 r.hd = __ldg(q);
-                r.c01 = __ldg(reinterpret_cast<const double2 *>(q + 1));
-                r.c23 = __ldg(reinterpret_cast<const double2 *>(q + 2));
+                r.kw = __ldg(q + 1);
+                r.c01 = __ldg(reinterpret_cast<const double2 *>(q + 2));
+                r.c23 = __ldg(reinterpret_cast<const double2 *>(q + 3));
                 return r;
             };
             auto one_kernel = [&](const Ent &en, double (&acc)[NCH]) {
-                const uint32_t code = en.hd.y;
-                const uint32_t k = (code >> KXP_K_SHIFT) & 31u, cls = code >> KXP_CLS_SHIFT;
-                const uint32_t sat = code & KXP_SAT_MASK, sh = (code >> KXP_SH_SHIFT) & 31u;
+                // hd = {m, sat, cc lo, cc hi}, kw = {cwoff, sh, kbit, cls}
+                const uint32_t sat = en.hd.y, sh = en.kw.y;
                 const unsigned long long cc = ((unsigned long long)en.hd.w << 32) | en.hd.z;
                 uint32_t blocks[NCH];
-                const uint32_t *cwk = cwl + k * SW_GROUPS;
+                const uint32_t *cwk = cwl + en.kw.x;
 #pragma unroll
                 for (int q = 0; q < NCH / 4; q++) {
                     const uint4 w4 = *reinterpret_cast<const uint4 *>(cwk + cwo[q]);
@@ -2503,16 +2501,19 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     for (int j = 0; j < NCH; j++) blocks[j] >>= sh;
                 }
                 double tk[NCH];
-                if (cls == KXC_P2S0) cls_times<KXC_P2S0>(en.c01, en.c23, blocks, rfh, rfl, tk);
-                else if (cls == KXC_P2S) cls_times<KXC_P2S>(en.c01, en.c23, blocks, rfh, rfl, tk);
-                else if (cls == KXC_NS0) cls_times<KXC_NS0>(en.c01, en.c23, blocks, rfh, rfl, tk);
-                else cls_times<KXC_NS>(en.c01, en.c23, blocks, rfh, rfl, tk);
-                if ((gk >> k) & 1u) {
+                switch (en.kw.w) {
+                case KXC_P2S0: cls_times<KXC_P2S0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                case KXC_P2S: cls_times<KXC_P2S>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                case KXC_NS0: cls_times<KXC_NS0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                default: cls_times<KXC_NS>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                }
+                if (gk & en.kw.z) {
                     // off the saturated path: the small-grid table (SKF_TABULATED)
                     bool any = false;
 #pragma unroll
                     for (int j = 0; j < NCH; j++) any |= blocks[j] < sat;
                     if (any) {
+                        const uint32_t k = en.kw.x / SW_GROUPS;
                         const double *row = S.small_t + (size_t)(I.kx_base + k * X + x) * S.small_stride;
 #pragma unroll
                         for (int j = 0; j < NCH; j++)
@@ -2524,23 +2525,14 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             };
             // sums in ascending kernel order (N6): the program lists the
             // per-iteration kernels, then the run-once ones; infeasible
-            // kernels are not listed (their sum is +inf through xinf).  Two
-            // entries per step: the second's loads overlap the first's model.
-            auto run = [&](uint32_t e0, uint32_t e1, double (&acc)[NCH]) {
-                uint32_t e = e0;
-#if GROPHECY_EUNROLL == 2
+            // kernels are not listed (their sum is +inf through xinf)
+            {
+                const KxProg *e = pe, *const e_it = pe + n_it, *const e_all = pe + n_all;
 #pragma unroll 1
-                for (; e + 1 < e1; e += 2) {
-                    const Ent a = load_ent(pe + e), b = load_ent(pe + e + 1);
-                    one_kernel(a, acc);
-                    one_kernel(b, acc);
-                }
-#endif
+                for (; e != e_it; ++e) one_kernel(load_ent(e), ti);
 #pragma unroll 1
-                for (; e < e1; e++) one_kernel(load_ent(pe + e), acc);
-            };
-            run(0, n_it, ti);
-            run(n_it, n_all, to);
+                for (; e != e_all; ++e) one_kernel(load_ent(e), to);
+            }
             const double inf = __longlong_as_double(0x7ff0000000000000LL);
             if (xf & XINF_ITER) {
 #pragma unroll

@@ -561,9 +561,12 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                     }
                     c.m = pm;
                     c.cc = pcc;
-                    c.code = (sat & KXP_SAT_MASK) | psh << KXP_SH_SHIFT | k << KXP_K_SHIFT;
+                    c.sat = sat;
+                    c.sh = psh;
+                    c.cwoff = k * 256u;   // = k * SW_GROUPS (project.cu)
+                    c.kbit = 1u << k;
                 }
-                if (!(j.flags & KXF_INFEASIBLE) && sat != KXF_SAT_MASK && sat <= KXP_SAT_MASK) {
+                if (!(j.flags & KXF_INFEASIBLE) && sat != KXF_SAT_MASK && sat <= KXP_SAT_MAX) {
                     const bool p2 = f.rDl == 0.0, s0 = f.S == 0.0;
                     // blocks < sat <=> w <= (sat - 1) * ipb
                     const uint64_t ws = (uint64_t)(sat - 1) * dv + 1;
@@ -582,7 +585,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                         pcls = s0 ? KXC_NS0 : KXC_NS;
                     }
                 }
-                c.code |= (pcls & 7u) << KXP_CLS_SHIFT;
+                c.cls = pcls;
                 pair_prog[(size_t)x * S.n_kernels + k] = c;
             }
         // per transformation: its program header (at kx_base + x) and program
@@ -596,7 +599,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 for (uint32_t k = 0; k < S.n_kernels; k++) {
                     const bool per = (S.kernels[k].flags & GROPHECY_KERNEL_PER_ITER) != 0;
                     const KxProg &e = pair_prog[(size_t)x * S.n_kernels + k];
-                    if (per != (pass == 0) || (e.code >> KXP_CLS_SHIFT) == KXC_NONE) continue;
+                    if (per != (pass == 0) || e.cls == KXC_NONE) continue;
                     kprog.push_back(e);
                     (pass == 0 ? n_it : n_on)++;
                 }
