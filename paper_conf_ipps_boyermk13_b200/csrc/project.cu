@@ -1776,13 +1776,14 @@ __device__ __forceinline__ bool canon_tile(const Params &P, CanonSmem &ws, uint3
 }
 // Block-level epilogue of best mode: warp -> CTA -> grid argmin (last-block
 // pattern; the last block also resets the ticket for reuse).
+template <int NW = WARPS>   // warps per CTA
 __device__ __forceinline__ void finish_best(const Params &P, const unsigned long long *best_h,
                                             const unsigned long long *best_d, int lane, int warp,
                                             double best_t, unsigned long long best_i,
                                             uint32_t cnt_inv, uint32_t cnt_val,
                                             unsigned nblocks)   // blocks taking part
 {
-    __shared__ Best wbest[WARPS];
+    __shared__ Best wbest[NW];
     __shared__ bool am_last;
     // ---- argmin: warp -> CTA -> grid (last-block pattern) ----
     Best mine;
@@ -1796,7 +1797,7 @@ __device__ __forceinline__ void finish_best(const Params &P, const unsigned long
     if (lane == 0) wbest[warp] = mine;
     __syncthreads();
     if (warp == 0) {
-        Best b = lane < WARPS ? wbest[lane] : none_best();
+        Best b = lane < NW ? wbest[lane] : none_best();
         b = warp_best(b);
         if (lane == 0) {
             to_result(P.partials[blockIdx.x], b);
@@ -2093,7 +2094,8 @@ __device__ __forceinline__ void issue_cta_copy_async(const Params &P, uint32_t (
 // in the same order as the tile's first design point (any fixed order of
 // valid transformations); warp-uniform result.  The batch's last warp tile
 // may hold gw < 32 design points: lanes past it stand in for design point 0.
-__device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*recs)[SW_TILE], int warp,
+template <unsigned long long ROW>   // staged array length (a CTA tile, or one warp tile)
+__device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*recs)[ROW], int warp,
                                               int lane, uint32_t gw, uint32_t &s0, uint32_t &n0, uint32_t &m0,
                                               uint32_t &i0)
 {
@@ -2791,20 +2793,19 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
             // passes 1 and 2 in one cooperative launch: CTA sweep tiles
             // (canonical layouts, one skeleton per tile), a grid barrier, then
             // the listed tiles on the general path
-            const int grid_s = sweep_grid(s, Q.n);
             Q.sweep_kmax = s->max_kernels;
             Q.fused = 1;
             Q.reset_counters = 1;
             cudaLaunchConfig_t cfg = {};
-            cfg.gridDim = dim3(grid_s);
             cfg.blockDim = dim3(THREADS);
-            cfg.dynamicSmemBytes = sweep_launch_smem(s);
             cfg.stream = st;
             cudaLaunchAttribute attr[1];
             attr[0].id = cudaLaunchAttributeCooperative;
             attr[0].val.cooperative = 1;
             cfg.attrs = attr;
             cfg.numAttrs = 1;
+            cfg.gridDim = dim3(sweep_grid(s, Q.n));
+            cfg.dynamicSmemBytes = sweep_launch_smem(s);
             e = cudaLaunchKernelEx(&cfg, sweep_kernel<true>, Q);
             if (e != cudaSuccess) return cuda_fail(e, "projection (best) sweep launch");
             sm_->counters_clean = true;
