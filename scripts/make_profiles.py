@@ -76,8 +76,8 @@ def main(tag):
                 "smsp__inst_executed.sum", "dram__throughput.avg.pct_of_peak_sustained_elapsed"]
         summ = {}
         with open(os.path.join(PROF, f"{tag}_ncu_best.txt"), "w") as f:
-            f.write("ncu --set full --clock-control none -k regex:canon_kernel (bench config, "
-                    "pass 1 of one 10^9-candidate best projection)\n")
+            f.write("ncu --set full --clock-control none -k regex:sweep_kernel (bench config, "
+                    "the fused best projection of 10^9 candidates)\n")
             for k in want:
                 if k in r:
                     f.write(f"{k:70s} {r[k]} {units.get(k, '')}\n")
@@ -95,7 +95,8 @@ def main(tag):
                   open(os.path.join(PROF, "ncu_best_summary.json"), "w"), indent=1)
     # stall / pipe breakdown and the hottest source lines of the same capture
     for src, dst in (("best_summary.txt", f"{tag}_ncu_best_stalls.txt"),
-                     ("best_lines.txt", f"{tag}_ncu_best_lines.txt")):
+                     ("best_lines.txt", f"{tag}_ncu_best_lines.txt"),
+                     ("best_groups.txt", f"{tag}_ncu_best_phases.txt")):
         p = os.path.join(OUT, src)
         if os.path.exists(p) and os.path.getsize(p) > 0:
             shutil.copy(p, os.path.join(PROF, dst))
