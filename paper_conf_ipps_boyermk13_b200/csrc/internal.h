@@ -94,11 +94,14 @@ struct SkelInfo {
     // poly[poly32_base + 2 * (c * n_polys + p)] holds int4 {c0, c1, c2, c3}
     // (sign-extended they are the u64 coefficients); POLY32_NONE if absent
     uint32_t poly32_base;
-    // the compact table padded for the sweep kernel: poly[polyf_base + 2 * (p
-    // * 64 + c)] holds int4 {c0, c1, c2, c3} of polynomial p in size class c,
-    // p < 2 * n_arrays rounded up to 2 * POLYF_AU (zero polynomials past
-    // n_arrays); POLY32_NONE if absent (staged whole into shared memory)
+    // the sweep kernel's table: poly[polyf_base + 2 * (q * 64 + c)] holds
+    // int4 {c0, c1, c2, c3} of list entry q in size class c; the entries are
+    // the H2D polynomials not zero in every class (array order), padded with
+    // zero ones to a multiple of POLYF_AU, then the D2H ones likewise;
+    // polyf_nhd = (padded H2D count) | (padded D2H count) << 16.
+    // POLY32_NONE if absent (staged whole into shared memory)
     uint32_t polyf_base;
+    uint32_t polyf_nhd;
 };
 constexpr uint32_t POLYF_AU = 4;   // arrays per step of the fp64 usage evaluation
 

@@ -2010,38 +2010,35 @@ __device__ __forceinline__ uint32_t cw_index(uint32_t k, uint32_t lane, uint32_t
     return k * (uint32_t)SW_GROUPS + lane * 8u + ((((j >> 2) ^ (lane >> 2)) & 1u) << 2) + (j & 3u);
 }
 
-// group_usage over the staged padded table (shared memory, [q][class]):
-// per polynomial one 16-byte load {c0, c1, c2, c3} (int32: the u64
-// coefficients sign-extended; zero polynomials past n_arrays), bytes = c0 +
-// c1 a + c2 b + (c3 a) b in wrapping 64-bit arithmetic (the same residue mod
-// 2^64 as the u64 table, hence the same bytes), priced by Eq. (1) in array
-// order.
-__device__ __forceinline__ void group_usage_s(const int4 *pp, uint32_t n_arrays, uint32_t a8,
-                                              uint32_t b8, const grophecy_pcie &pc, Usage &u)
+// group_usage over the staged table (shared memory, [q][class]; SkelInfo::
+// polyf_base): the non-zero H2D polynomials in array order, then the D2H
+// ones, per polynomial one 16-byte load {c0, c1, c2, c3} (int32: the u64
+// coefficients sign-extended), bytes = c0 + c1 a + c2 b + (c3 a) b in wrapping
+// 64-bit arithmetic (the same residue mod 2^64 as the u64 table, hence the
+// same bytes), priced by Eq. (1) and summed in array order per direction
+// (the skipped polynomials are zero: they price and add nothing).
+__device__ __forceinline__ void group_usage_s(const int4 *pp, uint32_t nhd, uint32_t a8, uint32_t b8,
+                                              const grophecy_pcie &pc, Usage &u)
 {
     const int a = (int)a8, b = (int)b8;
-    for (uint32_t a0 = 0; a0 < n_arrays; a0 += POLYF_AU, pp += 2 * POLYF_AU * POLY_CLASSES) {
-        int4 c[2 * POLYF_AU];
+    auto run = [&](uint32_t n, const grophecy_link &lk, double &tsum, unsigned long long &bsum) {
+        for (uint32_t q0 = 0; q0 < n; q0 += POLYF_AU, pp += POLYF_AU * POLY_CLASSES) {
+            int4 c[POLYF_AU];
 #pragma unroll
-        for (int q = 0; q < 2 * (int)POLYF_AU; q++) c[q] = pp[q * POLY_CLASSES];
+            for (int q = 0; q < (int)POLYF_AU; q++) c[q] = pp[q * POLY_CLASSES];
 #pragma unroll
-        for (int i = 0; i < (int)POLYF_AU; i++) {
-            unsigned long long v[2];
-#pragma unroll
-            for (int dir = 0; dir < 2; dir++) {
-                const int4 k = c[2 * i + dir];
+            for (int q = 0; q < (int)POLYF_AU; q++) {
+                const int4 k = c[q];
                 const long long s1 = (long long)k.y * a + (long long)k.x + (long long)k.z * b;
                 const unsigned long long t = (unsigned long long)((long long)k.w * a);
-                v[dir] = (unsigned long long)s1 + t * (unsigned long long)(unsigned)b;
+                const unsigned long long v = (unsigned long long)s1 + t * (unsigned long long)(unsigned)b;
+                if (v) tsum = __dadd_rn(tsum, __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte, __ull2double_rn(v))));
+                bsum += v;
             }
-            if (v[0]) u.th = __dadd_rn(u.th, __dadd_rn(pc.h2d.alpha_s,
-                                                       __dmul_rn(pc.h2d.beta_s_per_byte, __ull2double_rn(v[0]))));
-            if (v[1]) u.td = __dadd_rn(u.td, __dadd_rn(pc.d2h.alpha_s,
-                                                       __dmul_rn(pc.d2h.beta_s_per_byte, __ull2double_rn(v[1]))));
-            u.h += v[0];
-            u.d += v[1];
         }
-    }
+    };
+    run(nhd & 0xffffu, pc.h2d, u.th, u.h);
+    run(nhd >> 16, pc.d2h, u.td, u.d);
 }
 
 // CTA tile copy (thread 0): the 4 SoA arrays' SW_TILE records from tb into
@@ -2294,18 +2291,21 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             sm.tbl_wait = SW_BAD;
             if (ts != SW_BAD && ts != sm.tbl_skel && S.skel[ts].polyf_base != POLY32_NONE) {
                 const SkelInfo &I0 = S.skel[ts];
-                const uint32_t bytes = 2u * ((I0.n_arrays + POLYF_AU - 1) / POLYF_AU) * POLYF_AU * POLY_CLASSES * 16u;
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                const uint32_t bar = smem_u32(&sm.tbar);
-                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-                asm volatile(
-                    "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                        smem_u32(tbl)),
-                    "l"(S.poly + I0.polyf_base), "r"(bytes), "r"(bar)
-                    : "memory");
+                const uint32_t bytes = ((I0.polyf_nhd & 0xffffu) + (I0.polyf_nhd >> 16)) * POLY_CLASSES * 16u;
                 sm.tbl_skel = ts;
-                sm.tbl_wait = sm.tbl_phase;
-                sm.tbl_phase ^= 1u;
+                if (bytes) {   // (no transfer at all: nothing to stage)
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    const uint32_t bar = smem_u32(&sm.tbar);
+                    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
+                                 : "memory");
+                    asm volatile(
+                        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                            smem_u32(tbl)),
+                        "l"(S.poly + I0.polyf_base), "r"(bytes), "r"(bar)
+                        : "memory");
+                    sm.tbl_wait = sm.tbl_phase;
+                    sm.tbl_phase ^= 1u;
+                }
             }
             sm.next_tile = claimed + gridDim.x;   // the tile after nt
         }
@@ -2394,7 +2394,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     // the staged table is warp 0's skeleton: another skeleton
                     // makes the tile non-uniform (pass 2) anyway
                     ok = skel == sm.tbl_skel;
-                    if (ok) group_usage_s(tbl + cls, n_arrays, a8, b8, P.pc, u);
+                    if (ok) group_usage_s(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
                 } else if (I.poly32_base != POLY32_NONE) {
                     group_usage32<GROPHECY_AU32>(reinterpret_cast<const int4 *>(S.poly + I.poly32_base) +
                                                      (size_t)cls * (2u * n_arrays),

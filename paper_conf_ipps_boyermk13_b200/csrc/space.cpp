@@ -417,25 +417,34 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             I.poly_mask = 0;
             I.poly32_base = POLY32_NONE;
         }
-        // padded int32 copy of the bilinear table for the sweep kernel, laid
-        // out polynomial-major ([q][class]: lanes of different size classes
-        // read different shared-memory banks): 2 * n_arrays polynomials
-        // rounded up to 2 * POLYF_AU (zero polynomials past n_arrays)
+        // the sweep kernel's copy of the bilinear int32 table, laid out
+        // polynomial-major ([q][class]: lanes of different size classes read
+        // different shared-memory banks): the H2D polynomials that are not
+        // zero in every class, in array order, then the D2H ones, each list
+        // padded with zero polynomials to a multiple of POLYF_AU (zero
+        // polynomials price nothing: Eq. (1) is applied to non-zero bytes only)
         I.polyf_base = POLY32_NONE;
+        I.polyf_nhd = 0;
         if (I.poly32_base != POLY32_NONE) {
             const size_t np = 2 * (size_t)S.n_arrays;
-            const size_t npf = 2 * ((S.n_arrays + POLYF_AU - 1) / POLYF_AU) * POLYF_AU;
+            std::vector<size_t> lists[2];
+            for (size_t q = 0; q < np; q++)
+                if ((I.poly_mask >> q) & 1u) lists[q & 1].push_back(q);
+            size_t nl[2];
+            for (int d = 0; d < 2; d++) nl[d] = (lists[d].size() + POLYF_AU - 1) / POLYF_AU * POLYF_AU;
+            I.polyf_nhd = (uint32_t)nl[0] | (uint32_t)nl[1] << 16;
             I.polyf_base = (uint32_t)poly.size();   // even: 16-byte aligned
-            for (size_t q = 0; q < npf; q++)
-                for (size_t c = 0; c < POLY_CLASSES; c++) {
-                    uint32_t w4[4] = {0u, 0u, 0u, 0u};
-                    if (q < np)
-                        for (int m = 0; m < 4; m++) w4[m] = (uint32_t)plan.poly[(c * np + q) * 4 + m];
-                    uint64_t w[2];
-                    std::memcpy(w, w4, sizeof w);
-                    poly.push_back(w[0]);
-                    poly.push_back(w[1]);
-                }
+            for (int d = 0; d < 2; d++)
+                for (size_t i = 0; i < nl[d]; i++)
+                    for (size_t c = 0; c < POLY_CLASSES; c++) {
+                        uint32_t w4[4] = {0u, 0u, 0u, 0u};
+                        if (i < lists[d].size())
+                            for (int m = 0; m < 4; m++) w4[m] = (uint32_t)plan.poly[(c * np + lists[d][i]) * 4 + m];
+                        uint64_t w[2];
+                        std::memcpy(w, w4, sizeof w);
+                        poly.push_back(w[0]);
+                        poly.push_back(w[1]);
+                    }
         }
         I.per_iter_mask = 0;
         for (uint32_t k = 0; k < S.n_kernels; k++)
@@ -745,7 +754,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         if (info[q].polyf_base != POLY32_NONE)
             sp->usage_tbl_bytes = std::max<uint32_t>(
                 sp->usage_tbl_bytes,
-                (uint32_t)(2 * ((skels[q].n_arrays + POLYF_AU - 1) / POLYF_AU) * POLYF_AU * POLY_CLASSES * 16));
+                ((info[q].polyf_nhd & 0xffffu) + (info[q].polyf_nhd >> 16)) * POLY_CLASSES * 16u);
     sp->max_kernels = 1;
     for (uint32_t q = 0; q < n_skels; q++)
         sp->max_kernels = std::max(sp->max_kernels, skels[q].n_kernels);
