@@ -1976,7 +1976,8 @@ struct alignas(128) SweepSmem {
     unsigned long long rbar;     // completion of the record copies
     unsigned long long tbar;     // completion of the usage-table copy
     // per design point g = 32 * (warp of phase B) + lane, natural order
-    alignas(16) double it[SW_GROUPS], th[SW_GROUPS], td[SW_GROUPS];
+    alignas(16) double it[SW_GROUPS];
+    double2 thd[SW_GROUPS];      // {t_h2d, t_d2h}: one 16-byte read in the totals
     unsigned long long uh[SW_GROUPS], ud[SW_GROUPS];
     unsigned long long best_h[THREADS], best_d[THREADS];   // bytes of each lane's running best
     uint32_t smallk[SW_GROUPS];  // per design point: kernels whose grid may be unsaturated
@@ -2407,8 +2408,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     group_usage<false, 4>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride), stride,
                                           n_arrays, pm, a8, b8, P.pc, S.poly, u);
                 }
-                sm.th[g] = u.th;
-                sm.td[g] = u.td;
+                sm.thd[g] = make_double2(u.th, u.td);
                 sm.uh[g] = u.h;
                 sm.ud[g] = u.d;
                 sm.it[g] = (double)i0;
@@ -2554,7 +2554,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 const int gj = 32 * ((int)jb * NCH + j) + lane;
                 double tk = __dmul_rn(sm.it[gj], ti[j]);
                 if (once) tk = __dadd_rn(to[j], tk);
-                const double tt = __dadd_rn(__dadd_rn(tk, sm.th[gj]), sm.td[gj]);
+                const double2 thd = sm.thd[gj];
+                const double tt = __dadd_rn(__dadd_rn(tk, thd.x), thd.y);
                 // chains in increasing record index: strict < keeps the lowest
                 // (design points past a partial tile's end take no part)
                 if (tt < cmin && (uint32_t)gj < ngt) {
