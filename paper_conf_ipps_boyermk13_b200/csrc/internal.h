@@ -102,6 +102,11 @@ struct SkelInfo {
     // POLY32_NONE if absent (staged whole into shared memory)
     uint32_t polyf_base;
     uint32_t polyf_nhd;
+    // bound of |coefficient m| over the sweep table's polynomials (saturated
+    // at 2^32 - 1): when cmax0 + cmax1 a + cmax2 b + cmax3 a b < 2^32 every
+    // partial sum of a polynomial is below 2^32, so its 32-bit wrapping
+    // evaluation is the exact byte count
+    uint32_t polyf_cmax[4];
 };
 constexpr uint32_t POLYF_AU = 4;   // arrays per step of the fp64 usage evaluation
 

@@ -2018,10 +2018,12 @@ __device__ __forceinline__ uint32_t cw_index(uint32_t k, uint32_t lane, uint32_t
 // 64-bit arithmetic (the same residue mod 2^64 as the u64 table, hence the
 // same bytes), priced by Eq. (1) and summed in array order per direction
 // (the skipped polynomials are zero: they price and add nothing).
+template <bool U32>   // every partial sum below 2^32: 32-bit wrapping evaluation (exact)
 __device__ __forceinline__ void group_usage_s(const int4 *pp, uint32_t nhd, uint32_t a8, uint32_t b8,
                                               const grophecy_pcie &pc, Usage &u)
 {
     const int a = (int)a8, b = (int)b8;
+    const uint32_t ab = a8 * b8;
     auto run = [&](uint32_t n, const grophecy_link &lk, double &tsum, unsigned long long &bsum) {
         for (uint32_t q0 = 0; q0 < n; q0 += POLYF_AU, pp += POLYF_AU * POLY_CLASSES) {
             int4 c[POLYF_AU];
@@ -2030,11 +2032,17 @@ __device__ __forceinline__ void group_usage_s(const int4 *pp, uint32_t nhd, uint
 #pragma unroll
             for (int q = 0; q < (int)POLYF_AU; q++) {
                 const int4 k = c[q];
-                const long long s1 = (long long)k.y * a + (long long)k.x + (long long)k.z * b;
-                const unsigned long long t = (unsigned long long)((long long)k.w * a);
-                const unsigned long long v = (unsigned long long)s1 + t * (unsigned long long)(unsigned)b;
-                if (v) tsum = __dadd_rn(tsum, __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte, __ull2double_rn(v))));
-                bsum += v;
+                if (U32) {
+                    const uint32_t v = (uint32_t)k.x + (uint32_t)k.y * a8 + (uint32_t)k.z * b8 + (uint32_t)k.w * ab;
+                    if (v) tsum = __dadd_rn(tsum, __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte, __uint2double_rn(v))));
+                    bsum += v;
+                } else {
+                    const long long s1 = (long long)k.y * a + (long long)k.x + (long long)k.z * b;
+                    const unsigned long long t = (unsigned long long)((long long)k.w * a);
+                    const unsigned long long v = (unsigned long long)s1 + t * (unsigned long long)(unsigned)b;
+                    if (v) tsum = __dadd_rn(tsum, __dadd_rn(lk.alpha_s, __dmul_rn(lk.beta_s_per_byte, __ull2double_rn(v))));
+                    bsum += v;
+                }
             }
         }
     };
@@ -2395,7 +2403,16 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     // the staged table is warp 0's skeleton: another skeleton
                     // makes the tile non-uniform (pass 2) anyway
                     ok = skel == sm.tbl_skel;
-                    if (ok) group_usage_s(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
+                    if (ok) {
+                        const unsigned long long bnd =
+                            (unsigned long long)I.polyf_cmax[0] + (unsigned long long)I.polyf_cmax[1] * a8 +
+                            (unsigned long long)I.polyf_cmax[2] * b8 +
+                            (unsigned long long)I.polyf_cmax[3] * ((unsigned long long)a8 * b8);
+                        if (__all_sync(FULL, bnd < (1ull << 32)))
+                            group_usage_s<true>(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
+                        else
+                            group_usage_s<false>(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
+                    }
                 } else if (I.poly32_base != POLY32_NONE) {
                     group_usage32<GROPHECY_AU32>(reinterpret_cast<const int4 *>(S.poly + I.poly32_base) +
                                                      (size_t)cls * (2u * n_arrays),
@@ -2529,11 +2546,11 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             // per-iteration kernels, then the run-once ones; infeasible
             // kernels are not listed (their sum is +inf through xinf)
             {
-                const KxProg *e = pe, *const e_it = pe + n_it, *const e_all = pe + n_all;
+                const KxProg *e = pe;
 #pragma unroll 1
-                for (; e != e_it; ++e) one_kernel(load_ent(e), ti);
+                for (int i = (int)n_it; i > 0; i--, ++e) one_kernel(load_ent(e), ti);
 #pragma unroll 1
-                for (; e != e_all; ++e) one_kernel(load_ent(e), to);
+                for (int i = (int)(n_all - n_it); i > 0; i--, ++e) one_kernel(load_ent(e), to);
             }
             const double inf = __longlong_as_double(0x7ff0000000000000LL);
             if (xf & XINF_ITER) {
@@ -2549,20 +2566,24 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             const bool once = (pim & kmask) != kmask || (xf & XINF_ONCE);
             double cmin = inf;
             int cj = -1;
+            auto totals = [&](auto ONCE) {
 #pragma unroll
-            for (int j = 0; j < NCH; j++) {
-                const int gj = 32 * ((int)jb * NCH + j) + lane;
-                double tk = __dmul_rn(sm.it[gj], ti[j]);
-                if (once) tk = __dadd_rn(to[j], tk);
-                const double2 thd = sm.thd[gj];
-                const double tt = __dadd_rn(__dadd_rn(tk, thd.x), thd.y);
-                // chains in increasing record index: strict < keeps the lowest
-                // (design points past a partial tile's end take no part)
-                if (tt < cmin && (uint32_t)gj < ngt) {
-                    cmin = tt;
-                    cj = j;
+                for (int j = 0; j < NCH; j++) {
+                    const int gj = 32 * ((int)jb * NCH + j) + lane;
+                    double tk = __dmul_rn(sm.it[gj], ti[j]);
+                    if constexpr (decltype(ONCE)::value) tk = __dadd_rn(to[j], tk);
+                    const double2 thd = sm.thd[gj];
+                    const double tt = __dadd_rn(__dadd_rn(tk, thd.x), thd.y);
+                    // chains in increasing record index: strict < keeps the lowest
+                    // (design points past a partial tile's end take no part)
+                    if (tt < cmin && (uint32_t)gj < ngt) {
+                        cmin = tt;
+                        cj = j;
+                    }
                 }
-            }
+            };
+            if (once) totals(std::true_type{});
+            else totals(std::false_type{});
             if (cj >= 0) {
                 const int gj = 32 * ((int)jb * NCH + cj) + lane;
                 const unsigned long long idx = tbase + (unsigned long long)gj * CX + pos;

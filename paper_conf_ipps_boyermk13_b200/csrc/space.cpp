@@ -425,6 +425,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         // polynomials price nothing: Eq. (1) is applied to non-zero bytes only)
         I.polyf_base = POLY32_NONE;
         I.polyf_nhd = 0;
+        for (int m = 0; m < 4; m++) I.polyf_cmax[m] = 0xffffffffu;
         if (I.poly32_base != POLY32_NONE) {
             const size_t np = 2 * (size_t)S.n_arrays;
             std::vector<size_t> lists[2];
@@ -433,6 +434,16 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             size_t nl[2];
             for (int d = 0; d < 2; d++) nl[d] = (lists[d].size() + POLYF_AU - 1) / POLYF_AU * POLYF_AU;
             I.polyf_nhd = (uint32_t)nl[0] | (uint32_t)nl[1] << 16;
+            for (int m = 0; m < 4; m++) {
+                uint64_t mx = 0;
+                for (int d = 0; d < 2; d++)
+                    for (size_t q : lists[d])
+                        for (size_t c = 0; c < POLY_CLASSES; c++) {
+                            const int64_t v = (int32_t)(uint32_t)plan.poly[(c * np + q) * 4 + m];
+                            mx = std::max<uint64_t>(mx, (uint64_t)(v < 0 ? -v : v));
+                        }
+                I.polyf_cmax[m] = (uint32_t)std::min<uint64_t>(mx, 0xffffffffull);
+            }
             I.polyf_base = (uint32_t)poly.size();   // even: 16-byte aligned
             for (int d = 0; d < 2; d++)
                 for (size_t i = 0; i < nl[d]; i++)
