@@ -75,3 +75,24 @@ def test_partial_last_tile(G, O, n):
     start = 16 * 62_500_000 // 16     # inside the skeleton-major ranges
     rec = R.gen_records(c, start, start + n)
     check(G, O, c["skeletons"], rec, index_base=start)
+
+
+def test_large_counts_u64_usage(G, O):
+    """Sweep tiles whose byte counts exceed 2^32 (random multi-kernel
+    skeletons at nx, ny around 2^15, 8-byte elements: counts up to 2^33, work
+    counts still below the fast path's 2^30): the usage takes the 64-bit
+    evaluation (the 32-bit one only when a per-skeleton bound proves every
+    count < 2^32); a tile mixing both kinds of sizes, against the oracle."""
+    c = R.config("c3")
+    n = 2 * 4096
+    rec = R.gen_records(c, 0, n)
+    rng = np.random.default_rng(99)
+    g = n // 16
+    big = rng.integers(30000, 32768, g).astype(np.uint32)
+    small = rng.integers(256, 2048, g).astype(np.uint32)
+    pick = rng.random(g) < 0.7
+    nx = np.where(pick, big, small)
+    ny = np.where(pick, big[::-1], small[::-1])
+    rec["nx"] = np.repeat(nx, 16)
+    rec["ny"] = np.repeat(ny, 16)
+    check(G, O, c["skeletons"], rec)
