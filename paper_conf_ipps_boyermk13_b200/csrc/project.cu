@@ -2438,9 +2438,12 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         PT_MARK(4);   // barrier 1
         // uniform: every non-empty warp tile canonical, of one skeleton
         const uint32_t s_all = sm.wstat[0];
-        bool uni = s_all != SW_BAD && s_all != SW_EMPTY && sm.perm_ok;
-#pragma unroll
-        for (int w = 1; w < WARPS; w++) uni &= sm.wstat[w] == s_all || sm.wstat[w] == SW_EMPTY;
+        bool uni;
+        {   // lanes < WARPS read one warp tile's status each
+            const uint32_t st = sm.wstat[lane & (WARPS - 1)];
+            uni = __all_sync(FULL, st == s_all || st == SW_EMPTY) && s_all != SW_BAD && s_all != SW_EMPTY &&
+                  sm.perm_ok;
+        }
         if (!uni) {
             if (lane == 0 && gw) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * WARPS + warp);
             tile = nt;
