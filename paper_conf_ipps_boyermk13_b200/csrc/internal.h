@@ -60,7 +60,7 @@ inline uint32_t kxf_sat(const KxFast &f) { return f.satsh & KXF_SAT_MASK; }
 // A transformation's program (sweep kernel): its feasible kernels' entries in
 // summation order (per-iteration kernels, then run-once ones, each ascending;
 // infeasible kernels are left out: their sum is +inf through xinf).
-enum : uint32_t { KXC_P2S0 = 0u, KXC_P2S = 1u, KXC_NS0 = 2u, KXC_NS = 3u, KXC_NONE = 4u };
+enum : uint32_t { KXC_P2S0 = 0u, KXC_P2S = 1u, KXC_NS0 = 2u, KXC_NS = 3u, KXC_SHIFT = 4u, KXC_NONE = 8u };
 // blocks = hi32(w m + cc) >> sh (as KxFast; a power-of-two ipb = 2^l uses
 // m = 2^(32 - l), cc = (ipb - 1) m, sh = 0); the kernel as its work-count
 // offset cwoff = k * 256 (sweep shared memory) and its bit kbit = 1 << k;

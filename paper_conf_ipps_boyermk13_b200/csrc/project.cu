@@ -1935,6 +1935,9 @@ constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_SMINB
 #define GROPHECY_SMINB 2
 #endif
+#ifndef GROPHECY_STATIC_UNITS
+#define GROPHECY_STATIC_UNITS 1
+#endif
 #ifndef GROPHECY_I2F_MAGIC
 #define GROPHECY_I2F_MAGIC 0
 #endif
@@ -2455,12 +2458,23 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         const uint32_t K = I.n_kernels, X = I.n_xforms, pim = I.per_iter_mask;
         const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
         const unsigned long long tbase = P.base + tile * SW_TILE;
+#if GROPHECY_STATIC_UNITS
+        // warp w takes units w and SW_UNITS-1-w: in the identity layout the
+        // costliest transformation pairs with the cheapest (the longest-first
+        // claim order's outcome for warps that start together, without the
+        // per-claim atomic)
+        static_assert(SW_UNITS == 2 * WARPS, "two units per warp");
+#pragma unroll 1
+        for (int r = 0; r < 2; r++) {
+            const unsigned u = r ? (unsigned)(SW_UNITS - 1 - warp) : (unsigned)warp;
+#else
 #pragma unroll 1
         for (;;) {
             unsigned u = 0;
             if (lane == 0) u = atomicAdd(&sm.unit, 1u);
             u = __shfl_sync(FULL, u, 0);
             if (u >= (unsigned)SW_UNITS) break;
+#endif
             // the unit's position in the design points and its transformation:
             // in the identity layout by descending cost, else in position order
             uint4 hdr;
@@ -2518,15 +2532,22 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     for (int t = 0; t < 4; t++)
                         blocks[4 * q + t] = (uint32_t)(((unsigned long long)w[t] * en.hd.x + cc) >> 32);
                 }
-                if (sh) {   // (power-of-two ipb: none)
+                // the post-shift (power-of-two ipb: none) is a case of its own
+                // falling through into the class, so that no unshifted entry
+                // issues it predicated off
+                auto shift = [&] {
 #pragma unroll
                     for (int j = 0; j < NCH; j++) blocks[j] >>= sh;
-                }
+                };
                 double tk[NCH];
                 switch (en.kw.w) {
+                case KXC_P2S0 | KXC_SHIFT: shift(); [[fallthrough]];
                 case KXC_P2S0: cls_times<KXC_P2S0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                case KXC_P2S | KXC_SHIFT: shift(); [[fallthrough]];
                 case KXC_P2S: cls_times<KXC_P2S>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                case KXC_NS0 | KXC_SHIFT: shift(); [[fallthrough]];
                 case KXC_NS0: cls_times<KXC_NS0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                case KXC_NS | KXC_SHIFT: shift(); [[fallthrough]];
                 default: cls_times<KXC_NS>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
                 }
                 if (gk & en.kw.z) {

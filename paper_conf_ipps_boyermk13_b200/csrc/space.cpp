@@ -605,7 +605,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                         pcls = s0 ? KXC_NS0 : KXC_NS;
                     }
                 }
-                c.cls = pcls;
+                // KXC_SHIFT: the class's program post-shifts the block counts
+                c.cls = pcls | (pcls != KXC_NONE && c.sh ? KXC_SHIFT : 0u);
                 pair_prog[(size_t)x * S.n_kernels + k] = c;
             }
         // per transformation: its program header (at kx_base + x) and program
