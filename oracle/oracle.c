@@ -558,7 +558,10 @@ int oracle_eval_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
 /*      conversion, 1 mul, 2 add);                                           */
 /*  R3  exact identities cost nothing: a product with an exact zero (S = 0),  */
 /*      a division by a power of two (rep = blocks * 2^-k folds into E), and  */
-/*      a kernel with zero occupancy (its sum is +inf).                       */
+/*      a kernel with zero occupancy (its sum is +inf);                       */
+/*  R4  a candidate whose transformation has a zero-occupancy kernel has a    */
+/*      non-finite total and takes no part in the argmin (N7): beyond its     */
+/*      share of the design point's work (R2) it costs nothing.               */
 /* Per (candidate, kernel) on a saturated grid: blocks = ceil(W / ipb) by a  */
 /* multiply-high and a shift (2 int), 1 conversion, rep = blocks / D (a      */
 /* division), cyc = E rep (+ S rep: mul + add), t = cyc / freq (a division),  */
@@ -568,6 +571,15 @@ int oracle_eval_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
 /* fp64 counts each add / mul / compare as 1 and each division by a space    */
 /* constant as 2 (its cheapest exact evaluation, x*zh + RN(x*zl): the        */
 /* two-product form).  Returns 1 for a valid record (0: all counts 0).        */
+static uint64_t occupancy_of(const or_gpu *g, const or_kx *c)
+{
+    if (c->tpb > g->max_tpb) return 0;
+    uint64_t occ = umin64(g->max_bps, g->max_tps / c->tpb);
+    if (c->regs > 0) occ = umin64(occ, g->regs_sm / ((uint64_t)c->regs * c->tpb));
+    if (c->smem > 0) occ = umin64(occ, g->smem_sm / c->smem);
+    return occ;
+}
+
 int oracle_op_tally_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu *g,
                         uint32_t skx, uint32_t nx, uint32_t ny, uint32_t iters, uint32_t X,
                         double *fp64, double *ints, double *cvt)
@@ -579,20 +591,17 @@ int oracle_op_tally_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu
         return 0;
     const or_skeleton *s = &skels[skel];
     double f = 0.0, in = 0.0, cv = 0.0;
-    int has_once = 0;
+    int has_once = 0, feasible = 1;
+    for (uint32_t k = 0; k < s->n_kernels; k++) {
+        const or_kx *c = &s->kx[(size_t)xform * s->n_kernels + k];
+        if (occupancy_of(g, c) == 0) feasible = 0;
+    }
     for (uint32_t k = 0; k < s->n_kernels; k++) {
         const or_kx *c = &s->kx[(size_t)xform * s->n_kernels + k];
         if (!s->kernels[k].per_iter) has_once = 1;
-        uint64_t occ;
-        if (c->tpb > g->max_tpb) {
-            occ = 0;
-        } else {
-            occ = umin64(g->max_bps, g->max_tps / c->tpb);
-            if (c->regs > 0) occ = umin64(occ, g->regs_sm / ((uint64_t)c->regs * c->tpb));
-            if (c->smem > 0) occ = umin64(occ, g->smem_sm / c->smem);
-        }
         in += 6.0 / X;                                   /* work count (R2) */
-        if (occ == 0) continue;                          /* R3: sum is +inf */
+        if (!feasible) continue;                         /* R3, R4 */
+        const uint64_t occ = occupancy_of(g, c);
         uint64_t ipb = (uint64_t)c->tpb * c->ipt;
         int64_t Wi = oracle_affine8(&s->kernels[k].work, nx, ny);
         uint64_t W = Wi > 0 ? (uint64_t)Wi : 0;
@@ -629,7 +638,7 @@ int oracle_op_tally_one(const or_skeleton *skels, uint32_t n_skels, const or_gpu
         if (hpa[a]) { f += 3.0 / X; cv += 1.0 / X; }
         if (dpa[a]) { f += 3.0 / X; cv += 1.0 / X; }
     }
-    f += 1.0 + (has_once ? 1.0 : 0.0) + 2.0 + 1.0;      /* totals + argmin */
+    if (feasible) f += 1.0 + (has_once ? 1.0 : 0.0) + 2.0 + 1.0;   /* totals + argmin */
     *fp64 = f;
     *ints = in;
     *cvt = cv;

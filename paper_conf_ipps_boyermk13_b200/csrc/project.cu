@@ -1935,6 +1935,9 @@ constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_SMINB
 #define GROPHECY_SMINB 2
 #endif
+#ifndef GROPHECY_XINF_SKIP
+#define GROPHECY_XINF_SKIP 1
+#endif
 #ifndef GROPHECY_STATIC_UNITS
 #define GROPHECY_STATIC_UNITS 1
 #endif
@@ -2488,6 +2491,12 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             }
             const uint32_t x = hdr.x;
             const uint32_t jb = u / CX, xf = hdr.w & 0xffu;
+#if GROPHECY_XINF_SKIP
+            // an infeasible kernel makes every total of the unit +inf (or NaN
+            // at iters = 0): none takes part in the argmin (non-finite totals
+            // never win), so the unit has nothing to compute
+            if (xf & (XINF_ITER | XINF_ONCE)) continue;
+#endif
             const KxProg *pe = S.xprog + hdr.y;
             const uint32_t n_it = hdr.z & 0xffffu, n_all = n_it + (hdr.z >> 16);
             // kernels whose grid may be unsaturated for one of the warp's design points
@@ -2577,6 +2586,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 for (int i = (int)(n_all - n_it); i > 0; i--, ++e) one_kernel(load_ent(e), to);
             }
             const double inf = __longlong_as_double(0x7ff0000000000000LL);
+#if !GROPHECY_XINF_SKIP
             if (xf & XINF_ITER) {
 #pragma unroll
                 for (int j = 0; j < NCH; j++) ti[j] = inf;
@@ -2585,6 +2595,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
 #pragma unroll
                 for (int j = 0; j < NCH; j++) to[j] = inf;
             }
+#endif
             // totals; without run-once kernels t_once =
             // +0.0 and +0.0 + iters * t_iter = iters * t_iter exactly
             const bool once = (pim & kmask) != kmask || (xf & XINF_ONCE);

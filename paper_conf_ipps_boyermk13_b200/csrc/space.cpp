@@ -614,6 +614,7 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         // ones, each in ascending kernel order: N6); the header carries an
         // estimated cost for the phase-C claim order (longest first)
         for (uint32_t x = 0; x < S.n_xforms; x++) {
+            if (xinf[kx0 + x]) xcost[x] = 0.0;   // the sweep skips the unit (no finite total)
             const uint32_t first = (uint32_t)kprog.size();
             uint32_t n_it = 0, n_on = 0;
             for (int pass = 0; pass < 2; pass++)

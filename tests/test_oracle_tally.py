@@ -6,7 +6,8 @@ workloads.  The tally is a measurement convention for the op-bound roofline
 Rule recap: per (candidate, kernel) on a saturated grid 2 int (ceil
 division) + 1 conversion + fp64 {rep: 2 unless D is a power of two; E rep:
 1; S rep + add: 2 unless S = 0; / freq: 2; running sum: 1}; below saturation
-2 int + 1 fp64 (table + running sum); infeasible kernels nothing.  Per
+2 int + 1 fp64 (table + running sum); a transformation with an infeasible
+kernel nothing per kernel and no totals (R4: its total is +inf, N7).  Per
 candidate: fp64 iters*t_iter (1) + t_once (1, run-once kernels only) + t_h2d
 + t_d2h (2) + argmin compare (1).  Per design point (/X = /16 per record):
 6 int per kernel (work count), 12 int per array (two byte counts), 3 fp64 +
@@ -43,9 +44,10 @@ def test_hotspot_1024(O, sk):
     f, i, c = tally(O, sk, s, 4, 1024, 10)
     assert f == 6 + 4 + 9 / 16
     # x = 14 (tpb 512, coarse2: regs 20 * 512 > 8192): infeasible -> no
-    # kernel arithmetic, no conversion of its block count
+    # kernel arithmetic, no conversion of its block count, and (R4: its total
+    # is +inf, outside the argmin, N7) no totals: only the design point's share
     f, i, c = tally(O, sk, s, 14, 1024, 10)
-    assert f == 4 + 9 / 16
+    assert f == 9 / 16
     assert i == 6 / 16 + 36 / 16
     assert c == 3 / 16
 
@@ -62,7 +64,7 @@ def test_stencil_64_below_saturation(O, sk):
     assert c == 3 / 16
     # x = 14 infeasible: nothing per kernel
     f, i, c = tally(O, sk, s, 14, 64, 1)
-    assert f == 4 + 9 / 16 and i == 2 * 6 / 16 + 24 / 16
+    assert f == 9 / 16 and i == 2 * 6 / 16 + 24 / 16
 
 
 def test_run_once_kernel_adds_t_once(O, sk):
@@ -95,4 +97,4 @@ def test_invalid_and_batch_mean(O, sk):
            "ny": np.full(3, 1024, np.uint32), "iters": np.full(3, 10, np.uint32)}
     m = P.op_tally(rec)
     assert m["n_valid"] == 2
-    assert m["fp64"] == ((8 + 9 / 16) + (4 + 9 / 16)) / 2
+    assert m["fp64"] == ((8 + 9 / 16) + 9 / 16) / 2
