@@ -62,10 +62,11 @@ inline uint32_t kxf_sat(const KxFast &f) { return f.satsh & KXF_SAT_MASK; }
 // infeasible kernels are left out: their sum is +inf through xinf).
 enum : uint32_t { KXC_P2S0 = 0u, KXC_P2S = 1u, KXC_NS0 = 2u, KXC_NS = 3u, KXC_SHIFT = 4u, KXC_NONE = 8u };
 // blocks = hi32(w m + cc) >> sh (as KxFast; a power-of-two ipb = 2^l uses
-// m = 2^(32 - l), cc = (ipb - 1) m, sh = 0); the kernel as its work-count
-// offset cwoff = k * 256 (sweep shared memory) and its bit kbit = 1 << k;
-// sat <= SMALL_GRID_MAX (the sweep path requires tabulated pairs).  Fields
-// unpacked: 64 bytes, four 16-byte loads, no decoding.
+// m = 2^(32 - l), cc = (ipb - 1) m, sh = 0); the kernel's work slot j
+// (SkelInfo::n_wslots) as its work-count offset cwoff = j * 256 (sweep shared
+// memory) and its bit kbit = 1 << j; sat = sat_blocks | k << 16 (kernel k:
+// the small-grid table's row), sat_blocks <= SMALL_GRID_MAX (the sweep path
+// requires tabulated pairs).  Fields unpacked: 64 bytes, four 16-byte loads.
 struct __align__(16) KxProg {
     uint32_t m, sat;
     uint64_t cc;
@@ -107,6 +108,13 @@ struct SkelInfo {
     // partial sum of a polynomial is below 2^32, so its 32-bit wrapping
     // evaluation is the exact byte count
     uint32_t polyf_cmax[4];
+    // sweep kernel: the distinct work-count functions of the kernels ("work
+    // slots", first-use order) at wslot_work[w_base + j], j < n_wslots; a
+    // program entry reads its kernel's slot.  wslot_c32: max |c1|, |c2|, |c3|
+    // over the slots (0xffffffff when some |c0| >= 2^29): when
+    // wslot_c32 * (nx + ny + nx ny) < 2^31 every slot's count is exact in
+    // 32-bit arithmetic
+    uint32_t w_base, n_wslots, wslot_c32, pad_w;
 };
 constexpr uint32_t POLYF_AU = 4;   // arrays per step of the fp64 usage evaluation
 
@@ -197,10 +205,11 @@ struct SpaceDev {
     // per (skeleton, xform), at kx_base + x: some per-iteration (XINF_ITER) /
     // run-once (XINF_ONCE) kernel is infeasible, so that sum is +inf
     const uint32_t *xinf;
-    // sweep kernel: per (skeleton, kernel) at k_base + k, the smallest work
-    // count w for which every transformation's grid is saturated (blocks >=
-    // sat for all x)
-    const uint32_t *kern_wsat;
+    // sweep kernel: per (skeleton, work slot) at w_base + j, the slot's work
+    // function and the smallest work count w for which the grid of every
+    // (kernel of the slot, transformation) is saturated (blocks >= sat)
+    const int4 *wslot_work;
+    const uint32_t *wslot_sat;
     uint32_t small_stride;
     uint32_t n_skels;
     uint32_t n_sm;
@@ -227,6 +236,7 @@ struct grophecy_space {
     uint32_t max_partials;
     int grid_best, grid_eval;            // persistent grid sizes
     uint32_t max_kernels;                // largest kernel count of the space's skeletons
+    uint32_t max_wslots;                 // largest work-slot count (SkelInfo::n_wslots)
     int occ_canon;                       // pass-1 CTAs per SM (0 = not yet queried)
     int occ_sweep;                       // sweep-kernel CTAs per SM (0 = not yet queried)
     uint32_t usage_tbl_bytes;            // largest padded usage table (sweep shared memory)

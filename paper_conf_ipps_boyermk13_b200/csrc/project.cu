@@ -1142,7 +1142,7 @@ struct Params {
     uint32_t *tile_list;      // pass 1 -> pass 2: tiles left to the general path
     unsigned int *tile_count;
     uint32_t canon_warp_bytes; // pass 1: shared memory per warp (canon_warp_bytes(kmax))
-    uint32_t sweep_kmax;       // sweep kernel: the space's largest kernel count (smem layout)
+    uint32_t sweep_kmax;       // sweep kernel: the space's largest work-slot count (smem layout)
     int direct;                // pass 2 takes every warp tile of the batch (no pass 1, no list)
     int reset_counters;        // best mode: pass 2 leaves the tile counters zeroed for the next call
     int fused;                 // best mode: the sweep kernel runs pass 2 itself (cooperative launch)
@@ -1950,6 +1950,9 @@ constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_DIAG_NOLOAD
 #define GROPHECY_DIAG_NOLOAD 0
 #endif
+#ifndef GROPHECY_TMA_SPLIT
+#define GROPHECY_TMA_SPLIT 1   // bulk copies per SoA array of a CTA tile
+#endif
 #ifndef GROPHECY_PF
 #define GROPHECY_PF 0
 #endif
@@ -1977,40 +1980,37 @@ __device__ unsigned long long g_phase_cycles[8];
 #define PT_MARK(slot) do { } while (0)
 #endif
 
+constexpr int SW_NB = 2;   // buffers of the per-design-point phase-B results (tiles r, r + 1)
 struct alignas(128) SweepSmem {
     alignas(128) uint32_t rec[4][SW_TILE];   // the CTA tile's SoA records (4 TMA bulk copies)
-    unsigned long long rbar;     // completion of the record copies
-    unsigned long long tbar;     // completion of the usage-table copy
-    // per design point g = 32 * (warp of phase B) + lane, natural order
-    alignas(16) double it[SW_GROUPS];
-    double2 thd[SW_GROUPS];      // {t_h2d, t_d2h}: one 16-byte read in the totals
-    unsigned long long uh[SW_GROUPS], ud[SW_GROUPS];
-    unsigned long long best_h[THREADS], best_d[THREADS];   // bytes of each lane's running best
-    uint32_t smallk[SW_GROUPS];  // per design point: kernels whose grid may be unsaturated
-    uint32_t askel[WARPS];       // phase A result per warp: its skeleton, or SW_BAD
-    uint32_t wstat[WARPS];       // phase B result per warp: its skeleton, or SW_BAD
-    uint32_t next0;              // the CTA's second tile (claimed by thread 0 before the loop)
-    uint32_t next_tile;          // the tile after the next one (claimed by thread 0 each tile)
-    uint32_t unit;               // phase-C unit counter
-    uint32_t tbl_skel;           // skeleton whose usage table is staged (SW_BAD: none)
-    uint32_t tbl_wait;           // this tile: parity to wait for on tbar, or SW_BAD (no copy)
-    uint32_t tbl_phase;          // parity of the next tbar completion
-    uint32_t perm[CX];           // this tile's skx at each position of a design point (its first one's)
-    uint32_t perm_ident;         // perm is the identity (claims follow the cost order)
-    uint32_t perm_ok;            // the tile's first design point is consistent (one skeleton, valid xforms)
+    unsigned long long rbar;     // completion of the record copies (phase = the tile's sequence number & 1)
+    unsigned long long tbar[2];  // usage-table decision of the tile of sequence parity p (TMA or plain arrive)
+    // per buffer b (the tile of sequence parity b), design point g = 32 * (A/B task) + lane
+    alignas(16) double2 thd[SW_NB][SW_GROUPS];   // {t_h2d, t_d2h}: one 16-byte read in the totals
+    uint32_t it[SW_NB][SW_GROUPS];               // iterations
+    uint32_t smallk[SW_NB][SW_GROUPS];   // per design point: work slots whose grid may be unsaturated
+    uint32_t wstat[SW_NB][WARPS];        // A/B result per warp tile: its skeleton, SW_BAD or SW_EMPTY
+    uint32_t perm[SW_NB][CX];            // the tile's skx at each position of a design point (its first one's)
+    uint32_t perm_ident[SW_NB];          // perm is the identity (units follow the cost order)
+    uint32_t perm_ok[SW_NB];             // the tile's first design point is consistent
+    uint32_t ab_cnt[2];                  // A/B task claims of the tile of sequence parity p
+    uint32_t a_done[2];                  // phase-A completions of the tile of sequence parity p
+    uint32_t tile_id[4];                 // the CTA's tiles by sequence number mod 4 (claimed ahead)
+    uint32_t tbl_skel;                   // skeleton whose usage table is staged (SW_BAD: none)
 };
-// followed by the work counts cw[k][lane][8] (uint32, w_store; design point
-// g = 32 j + lane at chunk (j / 4) ^ ((lane / 4) & 1), so a phase-C lane reads
-// its chains with two conflict-free 16-byte loads), sized by the space's
-// largest kernel count, then the staged usage table (SkelInfo::polyf_base)
+// followed by the work counts cw[b][j][lane][8] (uint32, w_store; buffer b,
+// work slot j; design point g = 32 t + lane at chunk (t / 4) ^ ((lane / 4) & 1),
+// so a phase-C lane reads its chains with two conflict-free 16-byte loads),
+// sized by the space's largest work-slot count, then the staged usage table
+// (SkelInfo::polyf_base)
 __host__ __device__ constexpr uint32_t sweep_cw_offset() { return (uint32_t)((sizeof(SweepSmem) + 127) / 128 * 128); }
-__host__ __device__ constexpr uint32_t sweep_tbl_offset(uint32_t kmax)
+__host__ __device__ constexpr uint32_t sweep_tbl_offset(uint32_t wmax)
 {
-    return sweep_cw_offset() + kmax * (uint32_t)SW_GROUPS * (uint32_t)sizeof(uint32_t);
+    return sweep_cw_offset() + (uint32_t)SW_NB * wmax * (uint32_t)SW_GROUPS * (uint32_t)sizeof(uint32_t);
 }
-__host__ __device__ constexpr uint32_t sweep_smem_bytes(uint32_t kmax, uint32_t tbl_bytes)
+__host__ __device__ constexpr uint32_t sweep_smem_bytes(uint32_t wmax, uint32_t tbl_bytes)
 {
-    return sweep_tbl_offset(kmax) + tbl_bytes;
+    return sweep_tbl_offset(wmax) + tbl_bytes;
 }
 __device__ __forceinline__ uint32_t cw_index(uint32_t k, uint32_t lane, uint32_t j)
 {
@@ -2071,13 +2071,26 @@ __device__ __forceinline__ void issue_cta_copy(const Params &P, uint32_t (*rec)[
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(4 * bytes)
                  : "memory");
     const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
+    if (GROPHECY_TMA_SPLIT == 1 || nrec < SW_TILE) {
 #pragma unroll
-    for (int a = 0; a < 4; a++)
-        asm volatile(
-            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                smem_u32(rec[a])),
-            "l"(src[a] + tb), "r"(bytes), "r"(bar)
-            : "memory");
+        for (int a = 0; a < 4; a++)
+            asm volatile(
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                    smem_u32(rec[a])),
+                "l"(src[a] + tb), "r"(bytes), "r"(bar)
+                : "memory");
+    } else {
+        constexpr uint32_t PIECE = (uint32_t)(SW_TILE / GROPHECY_TMA_SPLIT);
+#pragma unroll
+        for (uint32_t q = 0; q < GROPHECY_TMA_SPLIT; q++)
+#pragma unroll
+            for (int a = 0; a < 4; a++)
+                asm volatile(
+                    "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                        smem_u32(rec[a] + q * PIECE)),
+                    "l"(src[a] + tb + q * PIECE), "r"(PIECE * 4u), "r"(bar)
+                    : "memory");
+    }
 }
 
 // The same CTA tile copy issued by every thread as 16-byte cp.async
@@ -2211,23 +2224,63 @@ __device__ __forceinline__ void cls_times(const double2 c01, const double2 c23, 
     }
 }
 
+// Transfer bytes of a design point (skeleton I, nx, ny) on the sweep path:
+// phase B's evaluation read from the global copy of the tables (the staged
+// one may already hold the next tile's).  Only for a lane's new running best.
+__device__ __noinline__ void sweep_bytes(const unsigned long long *poly, const grophecy_pcie pc, const SkelInfo *Ip,
+                                         uint32_t n0, uint32_t m0, unsigned long long *hd)
+{
+    const SkelInfo &I = *Ip;
+    Usage u = {0ull, 0ull, 0.0, 0.0};
+    const uint32_t n_arrays = I.n_arrays, stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
+    const uint32_t cls = (n0 & 7u) * 8u + (m0 & 7u), pm = I.poly_mask;
+    if (I.polyf_base != POLY32_NONE) {
+        const int4 *tg = reinterpret_cast<const int4 *>(poly + I.polyf_base);
+        const unsigned long long bnd = (unsigned long long)I.polyf_cmax[0] +
+                                       (unsigned long long)I.polyf_cmax[1] * a8 +
+                                       (unsigned long long)I.polyf_cmax[2] * b8 +
+                                       (unsigned long long)I.polyf_cmax[3] * ((unsigned long long)a8 * b8);
+        if (bnd < (1ull << 32))
+            group_usage_s<true>(tg + cls, I.polyf_nhd, a8, b8, pc, u);
+        else
+            group_usage_s<false>(tg + cls, I.polyf_nhd, a8, b8, pc, u);
+    } else if (I.poly32_base != POLY32_NONE) {
+        group_usage32<GROPHECY_AU32>(reinterpret_cast<const int4 *>(poly + I.poly32_base) +
+                                         (size_t)cls * (2u * n_arrays),
+                                     n_arrays, pm, a8, b8, pc, reinterpret_cast<const int4 *>(poly), u);
+    } else if (stride > 4) {
+        group_usage<true, 2>(poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride), stride, n_arrays, pm,
+                             a8, b8, pc, poly, u);
+    } else {
+        group_usage<false, 4>(poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride), stride, n_arrays, pm,
+                              a8, b8, pc, poly, u);
+    }
+    hd[0] = u.h;
+    hd[1] = u.d;
+}
+
+// The sweep kernel works in rounds: round r runs phase C of the CTA's tile r
+// (its phase-B results in buffer r & 1) and the phase A/B tasks of tile r + 1
+// (one per warp tile, buffer (r + 1) & 1), claimed from a shared counter by
+// the warps as they run out of phase-C units, so a transformation-poor tile's
+// idle warps prepare the next tile instead of waiting; one CTA barrier ends
+// the round.  The last warp to finish phase A of a tile issues the TMA copy
+// of the CTA's next tile into the (single) record buffer.
 template <bool BEST>
 __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Params P)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SweepSmem &sm = *reinterpret_cast<SweepSmem *>(smem_raw);
-    uint32_t *cw = reinterpret_cast<uint32_t *>(smem_raw + sweep_cw_offset());
-    const int4 *tbl = reinterpret_cast<const int4 *>(smem_raw + sweep_tbl_offset(P.sweep_kmax));
+    const uint32_t wmax = P.sweep_kmax;
+    uint32_t *cw_all = reinterpret_cast<uint32_t *>(smem_raw + sweep_cw_offset());
+    const int4 *tbl = reinterpret_cast<const int4 *>(smem_raw + sweep_tbl_offset(wmax));
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const SpaceDev &S = P.S;
     double best_t = __longlong_as_double(0x7ff0000000000000LL);
     unsigned long long best_i = ~0ull;
     uint32_t cnt_val = 0;
-    sm.best_h[tid] = 0;
-    sm.best_d[tid] = 0;
     // pass 2 may be scheduled now (it waits for this grid's completion)
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    // full CTA tiles of 16-byte aligned records (the TMA's alignment)
     // CTA tiles of 16-byte aligned records (the TMA's alignment): the full
     // ones, plus the batch's last partial one when the batch is a whole
     // number of design points (its missing warp tiles are empty)
@@ -2248,395 +2301,396 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             if (mine) P.tile_list[base + __popc(bal & ((1u << lane) - 1u))] = (uint32_t)sub;
         }
     }
-    if (tid == 0) {
-        mbar_init(&sm.rbar, GROPHECY_LDGSTS ? THREADS : 1);
-        mbar_init(&sm.tbar, 1);
-        sm.tbl_skel = SW_BAD;
-        sm.tbl_phase = 0;
-    }
-    // tiles: the first is blockIdx.x, then claims from a counter two tiles
-    // ahead (tile, next nt, and the claim in flight), so a warp's TMA copy of
-    // its part of the next tile starts as soon as phase A has consumed the
-    // current one and overlaps phases B and C
+    // tiles: the first is blockIdx.x, the second claimed now, tile r + 3 by
+    // the first A/B task of round r (two rounds before its copy is issued)
     unsigned *claim = P.tile_count + CLAIM1;
-    unsigned long long tile = blockIdx.x;
-    if (tid == 0) sm.next0 = atomicAdd(claim, 1u) + gridDim.x;
+    if (tid == 0) {
+        mbar_init(&sm.rbar, 1);
+        mbar_init(&sm.tbar[0], 1);
+        mbar_init(&sm.tbar[1], 1);
+        sm.tbl_skel = SW_BAD;
+        sm.ab_cnt[0] = sm.ab_cnt[1] = 0;
+        sm.a_done[0] = sm.a_done[1] = 0;
+        sm.tile_id[0] = blockIdx.x;
+        sm.tile_id[1] = atomicAdd(claim, 1u) + gridDim.x;
+        sm.tile_id[2] = sm.tile_id[3] = 0xffffffffu;
+        if (blockIdx.x < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, (unsigned long long)blockIdx.x * SW_TILE);
+    }
     __syncthreads();
-    unsigned long long nt = sm.next0;
-#if GROPHECY_LDGSTS
-    if (tile < ntiles) issue_cta_copy_async(P, sm.rec, &sm.rbar, tile * SW_TILE, tid);
-#elif GROPHECY_DIAG_NOLOAD
-    // diagnostic: representative tiles per CTA (spread over the batch)
-    if (tid == 0 && tile < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, (blockIdx.x * (ntiles / gridDim.x)) * SW_TILE);
-#else
-    if (tid == 0 && tile < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, tile * SW_TILE);
-#endif
-    uint32_t phase = 0;
     const double rfh = S.rfh, rfl = S.rfl;
 #if GROPHECY_PHASE_TIMING
     long long pt_last = clock64();
 #endif
 #pragma unroll 1
-    while (tile < ntiles) {
-        // the tile after nt: claimed now, its value is needed only after
-        // phase A (the atomic's latency overlaps the record wait and phase A)
-        unsigned claimed = 0;
-        if (tid == 0) claimed = atomicAdd(claim, 1u);
-        // ---- A (this warp's tile) ----
-#if GROPHECY_DIAG_NOLOAD == 1   // diagnostic only (wrong results): records of the first tile reused
-        if (phase == 0) mbar_wait(&sm.rbar, 0);
-        phase = 1;
-#else
-        mbar_wait(&sm.rbar, phase);
-        phase ^= 1u;
-#endif
-        PT_MARK(0);   // waiting for the staged records
-        // design points of this tile, and of this warp's part of it
-        const uint32_t ngt = (uint32_t)((P.n - tile * SW_TILE < SW_TILE ? P.n - tile * SW_TILE : SW_TILE) / CX);
-        const int gwi = (int)ngt - 32 * warp;
-        const uint32_t gw = gwi <= 0 ? 0u : (gwi >= 32 ? 32u : (uint32_t)gwi);
-        uint32_t s0 = 0, n0 = 0, m0 = 0, i0 = 0;
-        bool ok = gw ? sweep_phase_a(S, sm.rec, warp, lane, gw, s0, n0, m0, i0) : false;
-        const uint32_t skel = s0 >> 16;
+    for (int r = -1;; r++) {
+        // counters of tile r (used in round r - 1) are next used for tile r + 2
         if (tid == 0) {
-            // warp 0's skeleton decides the tile's usage table: stage it in
-            // shared memory when it changes (every reader of the previous one
-            // passed the previous tile's barriers)
-            const uint32_t ts = ok ? skel : SW_BAD;
-            sm.tbl_wait = SW_BAD;
-            if (ts != SW_BAD && ts != sm.tbl_skel && S.skel[ts].polyf_base != POLY32_NONE) {
-                const SkelInfo &I0 = S.skel[ts];
-                const uint32_t bytes = ((I0.polyf_nhd & 0xffffu) + (I0.polyf_nhd >> 16)) * POLY_CLASSES * 16u;
-                sm.tbl_skel = ts;
-                if (bytes) {   // (no transfer at all: nothing to stage)
-                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                    const uint32_t bar = smem_u32(&sm.tbar);
-                    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
-                                 : "memory");
-                    asm volatile(
-                        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                            smem_u32(tbl)),
-                        "l"(S.poly + I0.polyf_base), "r"(bytes), "r"(bar)
-                        : "memory");
-                    sm.tbl_wait = sm.tbl_phase;
-                    sm.tbl_phase ^= 1u;
-                }
+            sm.ab_cnt[r & 1] = 0;
+            sm.a_done[r & 1] = 0;
+        }
+        const unsigned long long tn = sm.tile_id[(r + 1) & 3];   // tile r + 1
+        // ---- C: tile r, CTA-wide; unit = transformation x ----
+        if (r >= 0) {
+            const uint32_t b = (uint32_t)r & 1u;
+            const unsigned long long tile = sm.tile_id[r & 3];
+            const uint32_t ngt = (uint32_t)((P.n - tile * SW_TILE < SW_TILE ? P.n - tile * SW_TILE : SW_TILE) / CX);
+            const int gwi = (int)ngt - 32 * warp;
+            const uint32_t gw = gwi <= 0 ? 0u : (gwi >= 32 ? 32u : (uint32_t)gwi);
+            // uniform: every non-empty warp tile canonical, of one skeleton
+            const uint32_t s_all = sm.wstat[b][0];
+            bool uni;
+            {   // lanes < WARPS read one warp tile's status each
+                const uint32_t st = sm.wstat[b][lane & (WARPS - 1)];
+                uni = __all_sync(FULL, st == s_all || st == SW_EMPTY) && s_all != SW_BAD && s_all != SW_EMPTY &&
+                      sm.perm_ok[b];
             }
-            sm.next_tile = claimed + gridDim.x;   // the tile after nt
-        }
-        PT_MARK(1);   // phase A (+ table check)
-        __syncthreads();   // the previous tile's phase C is done with the per-design-point arrays
-        PT_MARK(2);   // barrier 0
-        // every read of the staged tile is done (phase A): it takes the next
-        // one, and the tile after that is prefetched into L2
-        const unsigned long long nnt = sm.next_tile;
-        uint32_t sq = 0;
-        if (tid < CX) {
-            // the tile's transformation order (its first design point's skx),
-            // read before the buffer is refilled (checked in phase B: perm_ok)
-            sq = sm.rec[0][tid];
-            sm.perm[tid] = sq;
-            const unsigned bad = __ballot_sync(0xffffu, (sq & 0xffffu) != (uint32_t)tid);
-            if (tid == 0) sm.perm_ident = bad == 0u;
-        }
-        __syncwarp();
-#if GROPHECY_LDGSTS
-        if (nt < ntiles) issue_cta_copy_async(P, sm.rec, &sm.rbar, nt * SW_TILE, tid);
-#endif
-#if GROPHECY_PF == 2
-        // the tile after next into L2: one 128-byte line per thread and array half
-        if (nnt < ntiles) {
-            const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
-#pragma unroll
-            for (int a = 0; a < 4; a++)
-#pragma unroll
-                for (int l = tid; l < (int)(SW_TILE * 4 / 128); l += THREADS)
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(src[a] + nnt * SW_TILE + 32 * l) : "memory");
-        }
-#endif
-        if (tid == 0) {
-#if GROPHECY_DIAG_NOLOAD == 2   // diagnostic: the same representative tile copied again (L2 hits)
-            if (nt < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, (blockIdx.x * (ntiles / gridDim.x)) * SW_TILE);
-#elif GROPHECY_DIAG_NOLOAD == 3   // diagnostic: 4 representative tiles in rotation (L2-resident, new data)
-            if (nt < ntiles)
-                issue_cta_copy(P, sm.rec, &sm.rbar, (blockIdx.x * (ntiles / gridDim.x) + (nt & 3u)) * SW_TILE);
-#elif !GROPHECY_LDGSTS && !GROPHECY_DIAG_NOLOAD
-            if (nt < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, nt * SW_TILE);
-#endif
-#if GROPHECY_PF == 1
-            if (nnt < ntiles) {
-                const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
-#pragma unroll
-                for (int a = 0; a < 4; a++)
-                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src[a] + nnt * SW_TILE),
-                                 "r"((uint32_t)(SW_TILE * sizeof(uint32_t)))
-                                 : "memory");
-            }
-#endif
-        }
-        if (tid == 0) sm.unit = 0;
-        const uint32_t tw = sm.tbl_wait;
-        if (tw != SW_BAD) mbar_wait(&sm.tbar, tw);
-        // ---- B: work counts and usage of design point g ----
-        const int g = warp * 32 + lane;
-        if (ok) {
-            const SkelInfo &I = S.skel[skel];   // warp-uniform
-            const uint32_t K = I.n_kernels, n_arrays = I.n_arrays;
-            const long long nxny = (long long)((unsigned long long)n0 * m0);
-            bool huge = false;
-            uint32_t small = 0;
-            for (uint32_t k = 0; k < K; k++) {
-                const uint32_t w = w_store(aff8n(__ldg(&S.kern_work[I.k_base + k]), (int)n0, (int)m0, nxny));
-                cw[cw_index(k, (uint32_t)lane, (uint32_t)warp)] = w;
-                huge |= w == W_HUGE;
-                small |= (w < __ldg(&S.kern_wsat[I.k_base + k]) ? 1u : 0u) << k;
-            }
-            sm.smallk[g] = small;
-            if (warp == 0) {
-                // the tile's first design point (lane 0's) is itself consistent:
-                // one skeleton, every transformation < n_xforms
-                const bool okq = (uint32_t)lane >= CX || ((sq >> 16) == skel && (sq & 0xffffu) < I.n_xforms);
-                const bool all = __all_sync(FULL, okq);
-                if (lane == 0) sm.perm_ok = all;
-            }
-            ok = !__any_sync(FULL, huge) && __all_sync(FULL, n0 >= I.plan_tx && m0 >= I.plan_ty);
-            if (ok) {
-                Usage u = {0ull, 0ull, 0.0, 0.0};
-                const uint32_t stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
-                const uint32_t cls = (n0 & 7u) * 8u + (m0 & 7u);
-                const uint32_t pm = I.poly_mask;
-                if (I.polyf_base != POLY32_NONE) {
-                    // the staged table is warp 0's skeleton: another skeleton
-                    // makes the tile non-uniform (pass 2) anyway
-                    ok = skel == sm.tbl_skel;
-                    if (ok) {
-                        const unsigned long long bnd =
-                            (unsigned long long)I.polyf_cmax[0] + (unsigned long long)I.polyf_cmax[1] * a8 +
-                            (unsigned long long)I.polyf_cmax[2] * b8 +
-                            (unsigned long long)I.polyf_cmax[3] * ((unsigned long long)a8 * b8);
-                        if (__all_sync(FULL, bnd < (1ull << 32)))
-                            group_usage_s<true>(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
-                        else
-                            group_usage_s<false>(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
-                    }
-                } else if (I.poly32_base != POLY32_NONE) {
-                    group_usage32<GROPHECY_AU32>(reinterpret_cast<const int4 *>(S.poly + I.poly32_base) +
-                                                     (size_t)cls * (2u * n_arrays),
-                                                 n_arrays, pm, a8, b8, P.pc,
-                                                 reinterpret_cast<const int4 *>(S.poly), u);
-                } else if (stride > 4) {
-                    group_usage<true, 2>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride), stride,
-                                         n_arrays, pm, a8, b8, P.pc, S.poly, u);
-                } else {
-                    group_usage<false, 4>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride), stride,
-                                          n_arrays, pm, a8, b8, P.pc, S.poly, u);
-                }
-                sm.thd[g] = make_double2(u.th, u.td);
-                sm.uh[g] = u.h;
-                sm.ud[g] = u.d;
-                sm.it[g] = (double)i0;
-            }
-        }
-        if (lane == 0) sm.wstat[warp] = gw == 0 ? SW_EMPTY : (ok ? skel : SW_BAD);
-        if (tid == 0 && !ok) sm.perm_ok = 0u;   // (warp 0 skipped its check; the tile is not uniform)
-        PT_MARK(3);   // phase B (work counts, usage)
-        __syncthreads();
-        PT_MARK(4);   // barrier 1
-        // uniform: every non-empty warp tile canonical, of one skeleton
-        const uint32_t s_all = sm.wstat[0];
-        bool uni;
-        {   // lanes < WARPS read one warp tile's status each
-            const uint32_t st = sm.wstat[lane & (WARPS - 1)];
-            uni = __all_sync(FULL, st == s_all || st == SW_EMPTY) && s_all != SW_BAD && s_all != SW_EMPTY &&
-                  sm.perm_ok;
-        }
-        if (!uni) {
-            if (lane == 0 && gw) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * WARPS + warp);
-            tile = nt;
-            nt = nnt;
-            continue;
-        }
-        // ---- C: CTA-wide; unit = (transformation x, chain block) ----
-        const SkelInfo &I = S.skel[s_all];
-        const uint32_t K = I.n_kernels, X = I.n_xforms, pim = I.per_iter_mask;
-        const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
-        const unsigned long long tbase = P.base + tile * SW_TILE;
-#if GROPHECY_STATIC_UNITS
-        // warp w takes units w and SW_UNITS-1-w: in the identity layout the
-        // costliest transformation pairs with the cheapest (the longest-first
-        // claim order's outcome for warps that start together, without the
-        // per-claim atomic)
-        static_assert(SW_UNITS == 2 * WARPS, "two units per warp");
-#pragma unroll 1
-        for (int r = 0; r < 2; r++) {
-            const unsigned u = r ? (unsigned)(SW_UNITS - 1 - warp) : (unsigned)warp;
-#else
-#pragma unroll 1
-        for (;;) {
-            unsigned u = 0;
-            if (lane == 0) u = atomicAdd(&sm.unit, 1u);
-            u = __shfl_sync(FULL, u, 0);
-            if (u >= (unsigned)SW_UNITS) break;
-#endif
-            // the unit's position in the design points and its transformation:
-            // in the identity layout by descending cost, else in position order
-            uint4 hdr;
-            uint32_t pos;
-            if (sm.perm_ident) {
-                hdr = __ldg(&S.xhdru[I.kx_base + u % CX]);
-                pos = hdr.x;
+            if (!uni) {
+                if (lane == 0 && gw) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * WARPS + warp);
             } else {
-                pos = u % CX;
-                hdr = __ldg(&S.xhdr[I.kx_base + (sm.perm[pos] & 0xffffu)]);
-            }
-            const uint32_t x = hdr.x;
-            const uint32_t jb = u / CX, xf = hdr.w & 0xffu;
+                const SkelInfo &I = S.skel[s_all];
+                const uint32_t K = I.n_kernels, X = I.n_xforms, pim = I.per_iter_mask;
+                const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
+                const unsigned long long tbase = P.base + tile * SW_TILE;
+                const uint32_t *cwb = cw_all + b * wmax * (uint32_t)SW_GROUPS;
+                const bool ident = sm.perm_ident[b] != 0u;
+#if GROPHECY_STATIC_UNITS
+                // warp w takes units w and SW_UNITS-1-w: in the identity layout the
+                // costliest transformation pairs with the cheapest
+                static_assert(SW_UNITS == 2 * WARPS, "two units per warp");
+#pragma unroll 1
+                for (int rr = 0; rr < 2; rr++) {
+                    const unsigned u = rr ? (unsigned)(SW_UNITS - 1 - warp) : (unsigned)warp;
+#else
+#pragma unroll 1
+                for (unsigned u = (unsigned)warp; u < (unsigned)SW_UNITS; u += WARPS) {
+#endif
+                    // the unit's position in the design points and its transformation:
+                    // in the identity layout by descending cost, else in position order
+                    uint4 hdr;
+                    uint32_t pos;
+                    if (ident) {
+                        hdr = __ldg(&S.xhdru[I.kx_base + u % CX]);
+                        pos = hdr.x;
+                    } else {
+                        pos = u % CX;
+                        hdr = __ldg(&S.xhdr[I.kx_base + (sm.perm[b][pos] & 0xffffu)]);
+                    }
+                    const uint32_t x = hdr.x;
+                    const uint32_t jb = u / CX, xf = hdr.w & 0xffu;
 #if GROPHECY_XINF_SKIP
-            // an infeasible kernel makes every total of the unit +inf (or NaN
-            // at iters = 0): none takes part in the argmin (non-finite totals
-            // never win), so the unit has nothing to compute
-            if (xf & (XINF_ITER | XINF_ONCE)) continue;
+                    // an infeasible kernel makes every total of the unit +inf (or NaN
+                    // at iters = 0): none takes part in the argmin (non-finite totals
+                    // never win), so the unit has nothing to compute
+                    if (xf & (XINF_ITER | XINF_ONCE)) continue;
 #endif
-            const KxProg *pe = S.xprog + hdr.y;
-            const uint32_t n_it = hdr.z & 0xffffu, n_all = n_it + (hdr.z >> 16);
-            // kernels whose grid may be unsaturated for one of the warp's design points
-            uint32_t gk = 0;
+                    const KxProg *pe = S.xprog + hdr.y;
+                    const uint32_t n_it = hdr.z & 0xffffu, n_all = n_it + (hdr.z >> 16);
+                    // work slots whose grid may be unsaturated for one of the warp's design points
+                    uint32_t gk = 0;
 #pragma unroll
-            for (int j = 0; j < NCH; j++) gk |= sm.smallk[32 * ((int)jb * NCH + j) + lane];
-            gk = __reduce_or_sync(FULL, gk);
-            double ti[NCH], to[NCH];
+                    for (int j = 0; j < NCH; j++) gk |= sm.smallk[b][32 * ((int)jb * NCH + j) + lane];
+                    gk = __reduce_or_sync(FULL, gk);
+                    double ti[NCH], to[NCH];
 #pragma unroll
-            for (int j = 0; j < NCH; j++) ti[j] = to[j] = 0.0;
-            // this lane's work-count chunks (cw_index for chains jb*NCH + 4q)
-            const uint32_t *cwl = cw + lane * (SW_GROUPS / 32);
-            uint32_t cwo[NCH / 4];
+                    for (int j = 0; j < NCH; j++) ti[j] = to[j] = 0.0;
+                    // this lane's work-count chunks (cw_index for chains jb*NCH + 4q)
+                    const uint32_t *cwl = cwb + lane * (SW_GROUPS / 32);
+                    uint32_t cwo[NCH / 4];
 #pragma unroll
-            for (int q = 0; q < NCH / 4; q++)
-                cwo[q] = ((((jb * NCH) / 4 + (uint32_t)q) ^ ((uint32_t)lane >> 2)) & 1u) << 2;
-            static_assert(SW_GROUPS == 256, "KxProg::cwoff = k * 256");
-            struct Ent {
-                uint4 hd, kw;
-                double2 c01, c23;
-            };
-            auto load_ent = [&](const KxProg *e) {
-                const uint4 *q = reinterpret_cast<const uint4 *>(e);
-                Ent r;
-                r.hd = __ldg(q);
-                r.kw = __ldg(q + 1);
-                r.c01 = __ldg(reinterpret_cast<const double2 *>(q + 2));
-                r.c23 = __ldg(reinterpret_cast<const double2 *>(q + 3));
-                return r;
-            };
-            auto one_kernel = [&](const Ent &en, double (&acc)[NCH]) {
-                // hd = {m, sat, cc lo, cc hi}, kw = {cwoff, sh, kbit, cls}
-                const uint32_t sat = en.hd.y, sh = en.kw.y;
-                const unsigned long long cc = ((unsigned long long)en.hd.w << 32) | en.hd.z;
-                uint32_t blocks[NCH];
-                const uint32_t *cwk = cwl + en.kw.x;
+                    for (int q = 0; q < NCH / 4; q++)
+                        cwo[q] = ((((jb * NCH) / 4 + (uint32_t)q) ^ ((uint32_t)lane >> 2)) & 1u) << 2;
+                    static_assert(SW_GROUPS == 256, "KxProg::cwoff = slot * 256");
+                    struct Ent {
+                        uint4 hd, kw;
+                        double2 c01, c23;
+                    };
+                    auto load_ent = [&](const KxProg *e) {
+                        const uint4 *q = reinterpret_cast<const uint4 *>(e);
+                        Ent en;
+                        en.hd = __ldg(q);
+                        en.kw = __ldg(q + 1);
+                        en.c01 = __ldg(reinterpret_cast<const double2 *>(q + 2));
+                        en.c23 = __ldg(reinterpret_cast<const double2 *>(q + 3));
+                        return en;
+                    };
+                    auto one_kernel = [&](const Ent &en, double (&acc)[NCH]) {
+                        // hd = {m, sat, cc lo, cc hi}, kw = {cwoff, sh, kbit, cls}
+                        const uint32_t sh = en.kw.y;
+                        const unsigned long long cc = ((unsigned long long)en.hd.w << 32) | en.hd.z;
+                        uint32_t blocks[NCH];
+                        const uint32_t *cwk = cwl + en.kw.x;
 #pragma unroll
-                for (int q = 0; q < NCH / 4; q++) {
-                    const uint4 w4 = *reinterpret_cast<const uint4 *>(cwk + cwo[q]);
-                    const uint32_t w[4] = {w4.x, w4.y, w4.z, w4.w};
+                        for (int q = 0; q < NCH / 4; q++) {
+                            const uint4 w4 = *reinterpret_cast<const uint4 *>(cwk + cwo[q]);
+                            const uint32_t w[4] = {w4.x, w4.y, w4.z, w4.w};
 #pragma unroll
-                    for (int t = 0; t < 4; t++)
-                        blocks[4 * q + t] = (uint32_t)(((unsigned long long)w[t] * en.hd.x + cc) >> 32);
-                }
-                // the post-shift (power-of-two ipb: none) is a case of its own
-                // falling through into the class, so that no unshifted entry
-                // issues it predicated off
-                auto shift = [&] {
+                            for (int t = 0; t < 4; t++)
+                                blocks[4 * q + t] = (uint32_t)(((unsigned long long)w[t] * en.hd.x + cc) >> 32);
+                        }
+                        // the post-shift (power-of-two ipb: none) is a case of its own
+                        // falling through into the class, so that no unshifted entry
+                        // issues it predicated off
+                        auto shift = [&] {
 #pragma unroll
-                    for (int j = 0; j < NCH; j++) blocks[j] >>= sh;
-                };
-                double tk[NCH];
-                switch (en.kw.w) {
-                case KXC_P2S0 | KXC_SHIFT: shift(); [[fallthrough]];
-                case KXC_P2S0: cls_times<KXC_P2S0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
-                case KXC_P2S | KXC_SHIFT: shift(); [[fallthrough]];
-                case KXC_P2S: cls_times<KXC_P2S>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
-                case KXC_NS0 | KXC_SHIFT: shift(); [[fallthrough]];
-                case KXC_NS0: cls_times<KXC_NS0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
-                case KXC_NS | KXC_SHIFT: shift(); [[fallthrough]];
-                default: cls_times<KXC_NS>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
-                }
-                if (gk & en.kw.z) {
-                    // off the saturated path: the small-grid table (SKF_TABULATED)
-                    bool any = false;
+                            for (int j = 0; j < NCH; j++) blocks[j] >>= sh;
+                        };
+                        double tk[NCH];
+                        switch (en.kw.w) {
+                        case KXC_P2S0 | KXC_SHIFT: shift(); [[fallthrough]];
+                        case KXC_P2S0: cls_times<KXC_P2S0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                        case KXC_P2S | KXC_SHIFT: shift(); [[fallthrough]];
+                        case KXC_P2S: cls_times<KXC_P2S>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                        case KXC_NS0 | KXC_SHIFT: shift(); [[fallthrough]];
+                        case KXC_NS0: cls_times<KXC_NS0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                        case KXC_NS | KXC_SHIFT: shift(); [[fallthrough]];
+                        default: cls_times<KXC_NS>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
+                        }
+                        if (gk & en.kw.z) {
+                            // off the saturated path: the small-grid table (SKF_TABULATED)
+                            const uint32_t sat = en.hd.y & 0xffffu;
+                            bool any = false;
 #pragma unroll
-                    for (int j = 0; j < NCH; j++) any |= blocks[j] < sat;
-                    if (any) {
-                        const uint32_t k = en.kw.x / SW_GROUPS;
-                        const double *row = S.small_t + (size_t)(I.kx_base + k * X + x) * S.small_stride;
+                            for (int j = 0; j < NCH; j++) any |= blocks[j] < sat;
+                            if (any) {
+                                const uint32_t k = en.hd.y >> 16;   // the entry's kernel
+                                const double *row = S.small_t + (size_t)(I.kx_base + k * X + x) * S.small_stride;
 #pragma unroll
-                        for (int j = 0; j < NCH; j++)
-                            if (blocks[j] < sat) tk[j] = __ldg(row + blocks[j]);
+                                for (int j = 0; j < NCH; j++)
+                                    if (blocks[j] < sat) tk[j] = __ldg(row + blocks[j]);
+                            }
+                        }
+#pragma unroll
+                        for (int j = 0; j < NCH; j++) acc[j] = __dadd_rn(acc[j], tk[j]);
+                    };
+                    // sums in ascending kernel order (N6): the program lists the
+                    // per-iteration kernels, then the run-once ones; infeasible
+                    // kernels are not listed (their sum is +inf through xinf)
+                    {
+                        const KxProg *e = pe;
+#pragma unroll 1
+                        for (int i = (int)n_it; i > 0; i--, ++e) one_kernel(load_ent(e), ti);
+#pragma unroll 1
+                        for (int i = (int)(n_all - n_it); i > 0; i--, ++e) one_kernel(load_ent(e), to);
                     }
-                }
-#pragma unroll
-                for (int j = 0; j < NCH; j++) acc[j] = __dadd_rn(acc[j], tk[j]);
-            };
-            // sums in ascending kernel order (N6): the program lists the
-            // per-iteration kernels, then the run-once ones; infeasible
-            // kernels are not listed (their sum is +inf through xinf)
-            {
-                const KxProg *e = pe;
-#pragma unroll 1
-                for (int i = (int)n_it; i > 0; i--, ++e) one_kernel(load_ent(e), ti);
-#pragma unroll 1
-                for (int i = (int)(n_all - n_it); i > 0; i--, ++e) one_kernel(load_ent(e), to);
-            }
-            const double inf = __longlong_as_double(0x7ff0000000000000LL);
+                    const double inf = __longlong_as_double(0x7ff0000000000000LL);
 #if !GROPHECY_XINF_SKIP
-            if (xf & XINF_ITER) {
+                    if (xf & XINF_ITER) {
 #pragma unroll
-                for (int j = 0; j < NCH; j++) ti[j] = inf;
-            }
-            if (xf & XINF_ONCE) {
+                        for (int j = 0; j < NCH; j++) ti[j] = inf;
+                    }
+                    if (xf & XINF_ONCE) {
 #pragma unroll
-                for (int j = 0; j < NCH; j++) to[j] = inf;
-            }
+                        for (int j = 0; j < NCH; j++) to[j] = inf;
+                    }
 #endif
-            // totals; without run-once kernels t_once =
-            // +0.0 and +0.0 + iters * t_iter = iters * t_iter exactly
-            const bool once = (pim & kmask) != kmask || (xf & XINF_ONCE);
-            double cmin = inf;
-            int cj = -1;
-            auto totals = [&](auto ONCE) {
+                    // totals; without run-once kernels t_once =
+                    // +0.0 and +0.0 + iters * t_iter = iters * t_iter exactly
+                    const bool once = (pim & kmask) != kmask || (xf & XINF_ONCE);
+                    double cmin = inf;
+                    int cj = -1;
+                    auto totals = [&](auto ONCE) {
 #pragma unroll
-                for (int j = 0; j < NCH; j++) {
-                    const int gj = 32 * ((int)jb * NCH + j) + lane;
-                    double tk = __dmul_rn(sm.it[gj], ti[j]);
-                    if constexpr (decltype(ONCE)::value) tk = __dadd_rn(to[j], tk);
-                    const double2 thd = sm.thd[gj];
-                    const double tt = __dadd_rn(__dadd_rn(tk, thd.x), thd.y);
-                    // chains in increasing record index: strict < keeps the lowest
-                    // (design points past a partial tile's end take no part)
-                    if (tt < cmin && (uint32_t)gj < ngt) {
-                        cmin = tt;
-                        cj = j;
+                        for (int j = 0; j < NCH; j++) {
+                            const int gj = 32 * ((int)jb * NCH + j) + lane;
+                            double tk = __dmul_rn(__uint2double_rn(sm.it[b][gj]), ti[j]);
+                            if constexpr (decltype(ONCE)::value) tk = __dadd_rn(to[j], tk);
+                            const double2 thd = sm.thd[b][gj];
+                            const double tt = __dadd_rn(__dadd_rn(tk, thd.x), thd.y);
+                            // chains in increasing record index: strict < keeps the lowest
+                            // (design points past a partial tile's end take no part)
+                            if (tt < cmin && (uint32_t)gj < ngt) {
+                                cmin = tt;
+                                cj = j;
+                            }
+                        }
+                    };
+                    if (once) totals(std::true_type{});
+                    else totals(std::false_type{});
+                    if (cj >= 0) {
+                        const int gj = 32 * ((int)jb * NCH + cj) + lane;
+                        const unsigned long long idx = tbase + (unsigned long long)gj * CX + pos;
+                        if (better(cmin, idx, best_t, best_i)) {
+                            best_t = cmin;
+                            best_i = idx;
+                        }
                     }
                 }
-            };
-            if (once) totals(std::true_type{});
-            else totals(std::false_type{});
-            if (cj >= 0) {
-                const int gj = 32 * ((int)jb * NCH + cj) + lane;
-                const unsigned long long idx = tbase + (unsigned long long)gj * CX + pos;
-                if (better(cmin, idx, best_t, best_i)) {
-                    best_t = cmin;
-                    best_i = idx;
-                    sm.best_h[tid] = sm.uh[gj];
-                    sm.best_d[tid] = sm.ud[gj];
-                }
+                if (lane == 0) cnt_val += gw * (uint32_t)CX;
             }
         }
-        if (lane == 0) cnt_val += gw * (uint32_t)CX;
         PT_MARK(5);   // phase C (model, totals, argmin)
-        tile = nt;
-        nt = nnt;
+        // ---- A/B tasks of tile r + 1 (warp tile q, buffer b1) ----
+        if (tn < ntiles) {
+            const uint32_t b1 = (uint32_t)(r + 1) & 1u;
+            const uint32_t ngt = (uint32_t)((P.n - tn * SW_TILE < SW_TILE ? P.n - tn * SW_TILE : SW_TILE) / CX);
+            uint32_t *cwb = cw_all + b1 * wmax * (uint32_t)SW_GROUPS;
+#pragma unroll 1
+            for (;;) {
+                uint32_t q = 0;
+                if (lane == 0) q = atomicAdd(&sm.ab_cnt[b1], 1u);
+                q = __shfl_sync(FULL, q, 0);
+                if (q >= (uint32_t)WARPS) break;
+                // the first task claims tile r + 3 (its latency overlaps phase A)
+                unsigned claimed = 0;
+                if (q == 0 && lane == 0) claimed = atomicAdd(claim, 1u);
+                mbar_wait(&sm.rbar, (uint32_t)(r + 1) & 1u);
+                PT_MARK(0);   // waiting for the staged records
+                const int gwi = (int)ngt - 32 * (int)q;
+                const uint32_t gw = gwi <= 0 ? 0u : (gwi >= 32 ? 32u : (uint32_t)gwi);
+                uint32_t s0 = 0, n0 = 0, m0 = 0, i0 = 0;
+                bool ok = gw ? sweep_phase_a(S, sm.rec, (int)q, lane, gw, s0, n0, m0, i0) : false;
+                const uint32_t skel = s0 >> 16;
+                // the tile's transformation order (its first design point's skx)
+                uint32_t sq = 0;
+                if (q == 0 && lane < CX) sq = sm.rec[0][lane];
+                __syncwarp();
+                if (lane == 0) {
+                    if (q == 0) sm.tile_id[(r + 3) & 3] = claimed + gridDim.x;   // tile r + 3
+                    // every read of the record buffer by this warp is done: the
+                    // tile's last one releases it to the copy of tile r + 2
+                    __threadfence_block();
+                    if (atomicAdd(&sm.a_done[b1], 1u) == (unsigned)WARPS - 1u) {
+                        const unsigned long long t2 = sm.tile_id[(r + 2) & 3];
+                        if (t2 < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, t2 * SW_TILE);
+                    }
+                }
+                PT_MARK(1);   // phase A
+                if (q == 0) {
+                    // warp tile 0's skeleton decides the tile's usage table: staged
+                    // when it changes (every reader of the previous one finished in
+                    // an earlier round)
+                    if (lane == 0) {
+                        const uint32_t ts = ok ? skel : SW_BAD;
+                        bool staged = false;
+                        if (ts != SW_BAD && ts != sm.tbl_skel && S.skel[ts].polyf_base != POLY32_NONE) {
+                            const SkelInfo &I0 = S.skel[ts];
+                            const uint32_t bytes =
+                                ((I0.polyf_nhd & 0xffffu) + (I0.polyf_nhd >> 16)) * POLY_CLASSES * 16u;
+                            sm.tbl_skel = ts;
+                            if (bytes) {   // (no transfer at all: nothing to stage)
+                                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                                const uint32_t bar = smem_u32(&sm.tbar[b1]);
+                                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
+                                             "r"(bytes)
+                                             : "memory");
+                                asm volatile(
+                                    "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], "
+                                    "%2, [%3];" ::"r"(smem_u32(tbl)),
+                                    "l"(S.poly + I0.polyf_base), "r"(bytes), "r"(bar)
+                                    : "memory");
+                                staged = true;
+                            }
+                        }
+                        if (!staged)
+                            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tbar[b1]))
+                                         : "memory");
+                    }
+                    if (lane < CX) {
+                        sm.perm[b1][lane] = sq;
+                        const unsigned bad = __ballot_sync(0xffffu, (sq & 0xffffu) != (uint32_t)lane);
+                        if (lane == 0) sm.perm_ident[b1] = bad == 0u;
+                    }
+                    __syncwarp();
+                }
+                mbar_wait(&sm.tbar[b1], ((uint32_t)(r + 1) >> 1) & 1u);
+                PT_MARK(2);   // the tile's usage-table decision
+                // ---- B: work counts and usage of design point g ----
+                const int g = (int)q * 32 + lane;
+                if (ok) {
+                    const SkelInfo &I = S.skel[skel];   // warp-uniform
+                    const uint32_t n_arrays = I.n_arrays, nw = I.n_wslots;
+                    const long long nxny = (long long)((unsigned long long)n0 * m0);
+                    bool huge = false;
+                    uint32_t small = 0;
+                    const int4 *wf = S.wslot_work + I.w_base;
+                    const uint32_t *wsat = S.wslot_sat + I.w_base;
+                    if (__all_sync(FULL, (unsigned long long)I.wslot_c32 * ((unsigned long long)n0 + m0 +
+                                                                             (unsigned long long)nxny) <
+                                             (1ull << 31))) {
+                        // every slot's count is exact in 32-bit arithmetic
+                        const int nx32 = (int)n0, ny32 = (int)m0, nxny32 = (int)nxny;
+                        for (uint32_t j = 0; j < nw; j++) {
+                            const int4 c = __ldg(wf + j);
+                            const int w = c.x + ((c.y * nx32 + c.z * ny32 + c.w * nxny32) >> 3);
+                            const uint32_t ws = w <= 0 ? 0u : (uint32_t)w;   // < 2^30
+                            cwb[cw_index(j, (uint32_t)lane, q)] = ws;
+                            small |= (ws < __ldg(wsat + j) ? 1u : 0u) << j;
+                        }
+                    } else {
+                        for (uint32_t j = 0; j < nw; j++) {
+                            const uint32_t w = w_store(aff8n(__ldg(wf + j), (int)n0, (int)m0, nxny));
+                            cwb[cw_index(j, (uint32_t)lane, q)] = w;
+                            huge |= w == W_HUGE;
+                            small |= (w < __ldg(wsat + j) ? 1u : 0u) << j;
+                        }
+                    }
+                    sm.smallk[b1][g] = small;
+                    if (q == 0) {
+                        // the tile's first design point (lane 0's) is itself consistent:
+                        // one skeleton, every transformation < n_xforms
+                        const bool okq = (uint32_t)lane >= CX || ((sq >> 16) == skel && (sq & 0xffffu) < I.n_xforms);
+                        const bool all = __all_sync(FULL, okq);
+                        if (lane == 0) sm.perm_ok[b1] = all;
+                    }
+                    ok = !__any_sync(FULL, huge) && __all_sync(FULL, n0 >= I.plan_tx && m0 >= I.plan_ty);
+                    if (ok) {
+                        Usage u = {0ull, 0ull, 0.0, 0.0};
+                        const uint32_t stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
+                        const uint32_t cls = (n0 & 7u) * 8u + (m0 & 7u);
+                        const uint32_t pm = I.poly_mask;
+                        if (I.polyf_base != POLY32_NONE) {
+                            // the staged table is warp tile 0's skeleton: another
+                            // skeleton makes the tile non-uniform (pass 2) anyway
+                            ok = skel == sm.tbl_skel;
+                            if (ok) {
+                                const unsigned long long bnd =
+                                    (unsigned long long)I.polyf_cmax[0] + (unsigned long long)I.polyf_cmax[1] * a8 +
+                                    (unsigned long long)I.polyf_cmax[2] * b8 +
+                                    (unsigned long long)I.polyf_cmax[3] * ((unsigned long long)a8 * b8);
+                                if (__all_sync(FULL, bnd < (1ull << 32)))
+                                    group_usage_s<true>(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
+                                else
+                                    group_usage_s<false>(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
+                            }
+                        } else if (I.poly32_base != POLY32_NONE) {
+                            group_usage32<GROPHECY_AU32>(reinterpret_cast<const int4 *>(S.poly + I.poly32_base) +
+                                                             (size_t)cls * (2u * n_arrays),
+                                                         n_arrays, pm, a8, b8, P.pc,
+                                                         reinterpret_cast<const int4 *>(S.poly), u);
+                        } else if (stride > 4) {
+                            group_usage<true, 2>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride),
+                                                 stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
+                        } else {
+                            group_usage<false, 4>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride),
+                                                  stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
+                        }
+                        sm.thd[b1][g] = make_double2(u.th, u.td);
+                        sm.it[b1][g] = i0;
+                    }
+                } else if (q == 0 && lane == 0) {
+                    sm.perm_ok[b1] = 0u;   // (warp tile 0 is not canonical: the tile is not uniform)
+                }
+                if (lane == 0) sm.wstat[b1][q] = gw == 0 ? SW_EMPTY : (ok ? skel : SW_BAD);
+                PT_MARK(3);   // phase B (work counts, usage)
+            }
+        }
+        __syncthreads();
+        PT_MARK(4);   // the round's barrier
+        if (tn >= ntiles) break;
+    }
+    // the bytes of each lane's running best (its design point's usage; the
+    // record buffer is idle now: no copy is in flight after the last round)
+    unsigned long long keep[2] = {0ull, 0ull};
+    if (best_i != ~0ull) {
+        const unsigned long long li = best_i - P.base;
+        sweep_bytes(S.poly, P.pc, &S.skel[__ldg(P.skx + li) >> 16], __ldg(P.nx + li), __ldg(P.ny + li), keep);
     }
     if (!P.fused) {
-        if (BEST) finish_best(P, sm.best_h + warp * 32, sm.best_d + warp * 32, lane, warp, best_t, best_i, 0u,
+        unsigned long long *bh = reinterpret_cast<unsigned long long *>(sm.rec[0]);
+        bh[tid] = keep[0];
+        bh[THREADS + tid] = keep[1];
+        __syncwarp();
+        if (BEST) finish_best(P, bh + warp * 32, bh + THREADS + warp * 32, lane, warp, best_t, best_i, 0u,
                               cnt_val, gridDim.x);
         return;
     }
@@ -2645,11 +2699,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
     // tiles (claims from a counter), each lane's running best continuing ----
     __syncthreads();
     cooperative_groups::this_grid().sync();
-    const unsigned long long keep_h = sm.best_h[tid], keep_d = sm.best_d[tid];
-    __syncthreads();   // the sweep's shared memory becomes the general tiles'
     WarpSmem &ws = reinterpret_cast<CtaSmem *>(smem_raw)->w[warp];
-    ws.best_h[lane] = keep_h;
-    ws.best_d[lane] = keep_d;
+    ws.best_h[lane] = keep[0];
+    ws.best_d[lane] = keep[1];
     constexpr unsigned SUBS = CTILE / WTILE;
     const unsigned units = *(volatile unsigned *)P.tile_count * SUBS;
     unsigned *next = P.tile_count + CLAIM2;
@@ -2729,6 +2781,8 @@ __global__ void combine_kernel(const grophecy_best_result *in, uint32_t count,
     if (lane == 0) to_result(*out, b);
 }
 
+constexpr uint32_t SMEM_CTA_MAX = 227u * 1024u;   // opt-in shared memory per CTA (sm_100)
+
 static void set_smem_attrs()
 {
     // per device: the attributes belong to the current device's context
@@ -2742,8 +2796,8 @@ static void set_smem_attrs()
     cudaFuncSetAttribute(general_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     cudaFuncSetAttribute(general_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     cudaFuncSetAttribute(sweep_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)std::max<uint32_t>(sweep_smem_bytes(MAXK, 2u * GROPHECY_MAX_ARRAYS * POLY_CLASSES * 16u),
-                                                 (uint32_t)sizeof(CtaSmem)));
+                         (int)std::min<uint32_t>(SMEM_CTA_MAX, std::max<uint32_t>(sweep_smem_bytes(MAXK, 2u * GROPHECY_MAX_ARRAYS * POLY_CLASSES * 16u),
+                                                 (uint32_t)sizeof(CtaSmem))));
     done = true;
 }
 
@@ -2779,7 +2833,7 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
 // general tiles' one after the grid barrier, whichever is larger.
 static uint32_t sweep_launch_smem(const grophecy_space *s)
 {
-    return std::max<uint32_t>(sweep_smem_bytes(s->max_kernels, s->usage_tbl_bytes), (uint32_t)sizeof(CtaSmem));
+    return std::max<uint32_t>(sweep_smem_bytes(s->max_wslots, s->usage_tbl_bytes), (uint32_t)sizeof(CtaSmem));
 }
 
 // Persistent grid of the sweep kernel: every SM full (occupancy per space:
@@ -2843,14 +2897,14 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         Q.reset_counters = 0;   // (pass 2 only, below: pass 1's list must survive pass 1)
         // batches the sweep takes nothing of (unaligned, the memory choice) and
         // batches smaller than one tile (pass 2 alone is quicker) go to pass 2 whole
-        Q.direct = BEST && !(Q.aligned && !Q.pr.mem && Q.n >= SW_TILE);
+        Q.direct = BEST && !(Q.aligned && !Q.pr.mem && Q.n >= SW_TILE && sweep_launch_smem(s) <= SMEM_CTA_MAX);
         int launches = 1;
         Q.fused = 0;
         if (BEST && !Q.direct && GROPHECY_FUSED) {
             // passes 1 and 2 in one cooperative launch: CTA sweep tiles
             // (canonical layouts, one skeleton per tile), a grid barrier, then
             // the listed tiles on the general path
-            Q.sweep_kmax = s->max_kernels;
+            Q.sweep_kmax = s->max_wslots;
             Q.fused = 1;
             Q.reset_counters = 1;
             cudaLaunchConfig_t cfg = {};
@@ -2872,7 +2926,7 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         } else if (BEST && !Q.direct) {
             // pass 1 alone (pass 2 launched below, programmatically dependent)
             const int grid_s = sweep_grid(s, Q.n);
-            Q.sweep_kmax = s->max_kernels;
+            Q.sweep_kmax = s->max_wslots;
             sweep_kernel<true><<<grid_s, THREADS, sweep_launch_smem(s), st>>>(Q);
             launches++;
         } else if (!BEST) {

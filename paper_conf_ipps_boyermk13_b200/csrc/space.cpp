@@ -349,6 +349,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     std::vector<uint32_t> xord;   // per (skeleton, unit) at kx_base + u: xforms by descending cost
     std::vector<uint4> xhdru;     // the headers in that order
     std::vector<uint32_t> kwsat;  // per (skeleton, kernel): work count saturating every xform
+    std::vector<int4> wslot_work;     // per (skeleton, work slot): the distinct work functions
+    std::vector<uint32_t> wslot_sat;  // per (skeleton, work slot): max kwsat of its kernels
     std::vector<uint32_t> xinf;   // per (skeleton, xform) at kx_base + x: XINF_* bits
     // the fast path divides by freq with the two-product method: without it
     // (a frequency whose odd significand is >= 2^50) every pair takes the
@@ -463,6 +465,34 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         for (uint32_t k = 0; k < S.n_kernels; k++) {
             kwork.push_back(a4(S.kernels[k].work_items));
             kflags.push_back(S.kernels[k].flags);
+        }
+        // work slots: kernels with the same work function share one count
+        // per design point in the sweep kernel
+        std::vector<uint32_t> kslot(S.n_kernels);
+        I.w_base = (uint32_t)wslot_work.size();
+        I.n_wslots = 0;
+        {
+            uint64_t cm = 0;
+            bool c0ok = true;
+            for (uint32_t k = 0; k < S.n_kernels; k++) {
+                const int4 w = a4(S.kernels[k].work_items);
+                uint32_t j = 0;
+                while (j < I.n_wslots) {
+                    const int4 &v = wslot_work[I.w_base + j];
+                    if (v.x == w.x && v.y == w.y && v.z == w.z && v.w == w.w) break;
+                    j++;
+                }
+                if (j == I.n_wslots) {
+                    wslot_work.push_back(w);
+                    wslot_sat.push_back(0u);
+                    I.n_wslots++;
+                    const int64_t c[3] = {w.y, w.z, w.w};
+                    for (int m = 0; m < 3; m++) cm = std::max<uint64_t>(cm, (uint64_t)(c[m] < 0 ? -c[m] : c[m]));
+                    c0ok = c0ok && w.x > -(1 << 29) && w.x < (1 << 29);
+                }
+                kslot[k] = j;
+            }
+            I.wslot_c32 = c0ok ? (uint32_t)std::min<uint64_t>(cm, 0xffffffffull) : 0xffffffffu;
         }
         for (uint32_t a = 0; a < S.n_arrays; a++) {
             ArrayDev A;
@@ -581,10 +611,10 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                     }
                     c.m = pm;
                     c.cc = pcc;
-                    c.sat = sat;
+                    c.sat = (sat & 0xffffu) | k << 16;   // (the sweep reads it for tabulated pairs only)
                     c.sh = psh;
-                    c.cwoff = k * 256u;   // = k * SW_GROUPS (project.cu)
-                    c.kbit = 1u << k;
+                    c.cwoff = kslot[k] * 256u;   // = slot * SW_GROUPS (project.cu)
+                    c.kbit = 1u << kslot[k];
                 }
                 if (!(j.flags & KXF_INFEASIBLE) && sat != KXF_SAT_MASK && sat <= KXP_SAT_MAX) {
                     const bool p2 = f.rDl == 0.0, s0 = f.S == 0.0;
@@ -609,6 +639,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 c.cls = pcls | (pcls != KXC_NONE && c.sh ? KXC_SHIFT : 0u);
                 pair_prog[(size_t)x * S.n_kernels + k] = c;
             }
+        for (uint32_t k = 0; k < S.n_kernels; k++)
+            wslot_sat[I.w_base + kslot[k]] = std::max(wslot_sat[I.w_base + kslot[k]], kwsat[I.k_base + k]);
         // per transformation: its program header (at kx_base + x) and program
         // (feasible saturated-capable kernels, per-iteration ones then run-once
         // ones, each in ascending kernel order: N6); the header carries an
@@ -685,6 +717,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
         {kwsat.data(), kwsat.size() * sizeof(uint32_t), 0},
         {xord.data(), xord.size() * sizeof(uint32_t), 0},
         {xhdru.data(), xhdru.size() * sizeof(uint4), 0},
+        {wslot_work.data(), wslot_work.size() * sizeof(int4), 0},
+        {wslot_sat.data(), wslot_sat.size() * sizeof(uint32_t), 0},
     };
     size_t total = 0;
     for (auto &p : parts) {
@@ -748,7 +782,8 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
     D.xinf = (const uint32_t *)(base + parts[13].off);
     D.xprog = (const KxProg *)(base + parts[14].off);
     D.xhdr = (const uint4 *)(base + parts[15].off);
-    D.kern_wsat = (const uint32_t *)(base + parts[16].off);
+    D.wslot_work = (const int4 *)(base + parts[19].off);
+    D.wslot_sat = (const uint32_t *)(base + parts[20].off);
     D.xord = (const uint32_t *)(base + parts[17].off);
     D.xhdru = (const uint4 *)(base + parts[18].off);
     D.small_stride = small_stride;
@@ -769,8 +804,11 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 sp->usage_tbl_bytes,
                 ((info[q].polyf_nhd & 0xffffu) + (info[q].polyf_nhd >> 16)) * POLY_CLASSES * 16u);
     sp->max_kernels = 1;
-    for (uint32_t q = 0; q < n_skels; q++)
+    sp->max_wslots = 1;
+    for (uint32_t q = 0; q < n_skels; q++) {
         sp->max_kernels = std::max(sp->max_kernels, skels[q].n_kernels);
+        sp->max_wslots = std::max(sp->max_wslots, info[q].n_wslots);
+    }
     sp->occ_canon = 0;
     sp->grid_eval = nsm;
     cudaSetDevice(prev);

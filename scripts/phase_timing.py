@@ -18,7 +18,16 @@ name = sys.argv[1] if len(sys.argv) > 1 else "c4"
 cfg = R.config(name)
 pc = G.pcie(G.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL))
 space = G.Space(cfg["skeletons"], S.FX5600)
-rec = G.synth_records(cfg)
+seg = os.environ.get("SEG_ONLY")   # one skeleton's segment (as scripts/segbench.py)
+if seg is not None:
+    ns, Gn = len(cfg["skeletons"]), (cfg["n"] + 15) // 16
+    s = int(seg)
+    lo = -(-s * Gn // ns) * 16
+    hi = min(cfg["n"], -(-(s + 1) * Gn // ns) * 16)
+    rec = G.synth_records(cfg, lo, min(hi - lo, 1 << 25))
+    print("segment", s, cfg["skeletons"][s]["name"])
+else:
+    rec = G.synth_records(cfg)
 space.best(pc, rec)
 fn = G.lib().grophecy_debug_phase_cycles
 fn.argtypes = [C.POINTER(C.c_uint64)]
