@@ -1950,6 +1950,9 @@ constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_DIAG_NOLOAD
 #define GROPHECY_DIAG_NOLOAD 0
 #endif
+#ifndef GROPHECY_DISPATCH_TREE
+#define GROPHECY_DISPATCH_TREE 1   // class dispatch by uniform branches (0: switch)
+#endif
 #ifndef GROPHECY_TMA_SPLIT
 #define GROPHECY_TMA_SPLIT 1   // bulk copies per SoA array of a CTA tile
 #endif
@@ -2301,8 +2304,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             if (mine) P.tile_list[base + __popc(bal & ((1u << lane) - 1u))] = (uint32_t)sub;
         }
     }
-    // tiles: the first is blockIdx.x, the second claimed now, tile r + 3 by
-    // the first A/B task of round r (two rounds before its copy is issued)
+    // tiles: the first is blockIdx.x, the second claimed now, tile r + 3 in
+    // round r (one round before its copy is issued)
     unsigned *claim = P.tile_count + CLAIM1;
     if (tid == 0) {
         mbar_init(&sm.rbar, 1);
@@ -2329,6 +2332,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             sm.a_done[r & 1] = 0;
         }
         const unsigned long long tn = sm.tile_id[(r + 1) & 3];   // tile r + 1
+        // tile r + 3 (its copy is issued in round r + 1): claimed now, stored
+        // before the round's barrier (the atomic's latency overlaps the round)
+        unsigned claimed = 0;
+        if (tid == 0 && tn < ntiles) claimed = atomicAdd(claim, 1u);
         // ---- C: tile r, CTA-wide; unit = transformation x ----
         if (r >= 0) {
             const uint32_t b = (uint32_t)r & 1u;
@@ -2435,6 +2442,18 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                             for (int j = 0; j < NCH; j++) blocks[j] >>= sh;
                         };
                         double tk[NCH];
+#if GROPHECY_DISPATCH_TREE
+                        // warp-uniform branches on the class bits (no indirect jump)
+                        const uint32_t cl = en.kw.w;
+                        if (cl & KXC_SHIFT) shift();
+                        if (cl & 2u) {
+                            if (cl & 1u) cls_times<KXC_NS>(en.c01, en.c23, blocks, rfh, rfl, tk);
+                            else cls_times<KXC_NS0>(en.c01, en.c23, blocks, rfh, rfl, tk);
+                        } else {
+                            if (cl & 1u) cls_times<KXC_P2S>(en.c01, en.c23, blocks, rfh, rfl, tk);
+                            else cls_times<KXC_P2S0>(en.c01, en.c23, blocks, rfh, rfl, tk);
+                        }
+#else
                         switch (en.kw.w) {
                         case KXC_P2S0 | KXC_SHIFT: shift(); [[fallthrough]];
                         case KXC_P2S0: cls_times<KXC_P2S0>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
@@ -2445,6 +2464,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                         case KXC_NS | KXC_SHIFT: shift(); [[fallthrough]];
                         default: cls_times<KXC_NS>(en.c01, en.c23, blocks, rfh, rfl, tk); break;
                         }
+#endif
                         if (gk & en.kw.z) {
                             // off the saturated path: the small-grid table (SKF_TABULATED)
                             const uint32_t sat = en.hd.y & 0xffffu;
@@ -2530,9 +2550,6 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 if (lane == 0) q = atomicAdd(&sm.ab_cnt[b1], 1u);
                 q = __shfl_sync(FULL, q, 0);
                 if (q >= (uint32_t)WARPS) break;
-                // the first task claims tile r + 3 (its latency overlaps phase A)
-                unsigned claimed = 0;
-                if (q == 0 && lane == 0) claimed = atomicAdd(claim, 1u);
                 mbar_wait(&sm.rbar, (uint32_t)(r + 1) & 1u);
                 PT_MARK(0);   // waiting for the staged records
                 const int gwi = (int)ngt - 32 * (int)q;
@@ -2545,7 +2562,6 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 if (q == 0 && lane < CX) sq = sm.rec[0][lane];
                 __syncwarp();
                 if (lane == 0) {
-                    if (q == 0) sm.tile_id[(r + 3) & 3] = claimed + gridDim.x;   // tile r + 3
                     // every read of the record buffer by this warp is done: the
                     // tile's last one releases it to the copy of tile r + 2
                     __threadfence_block();
@@ -2674,6 +2690,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 PT_MARK(3);   // phase B (work counts, usage)
             }
         }
+        if (tid == 0 && tn < ntiles) sm.tile_id[(r + 3) & 3] = claimed + gridDim.x;
         __syncthreads();
         PT_MARK(4);   // the round's barrier
         if (tn >= ntiles) break;
