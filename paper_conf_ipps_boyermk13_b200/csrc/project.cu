@@ -1990,7 +1990,7 @@ struct alignas(128) SweepSmem {
     unsigned long long tbar[2];  // usage-table decision of the tile of sequence parity p (TMA or plain arrive)
     // per buffer b (the tile of sequence parity b), design point g = 32 * (A/B task) + lane
     alignas(16) double2 thd[SW_NB][SW_GROUPS];   // {t_h2d, t_d2h}: one 16-byte read in the totals
-    uint32_t it[SW_NB][SW_GROUPS];               // iterations
+    double it[SW_NB][SW_GROUPS];                 // iterations
     uint32_t smallk[SW_NB][SW_GROUPS];   // per design point: work slots whose grid may be unsaturated
     uint32_t wstat[SW_NB][WARPS];        // A/B result per warp tile: its skeleton, SW_BAD or SW_EMPTY
     uint32_t perm[SW_NB][CX];            // the tile's skx at each position of a design point (its first one's)
@@ -2336,6 +2336,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         // before the round's barrier (the atomic's latency overlaps the round)
         unsigned claimed = 0;
         if (tid == 0 && tn < ntiles) claimed = atomicAdd(claim, 1u);
+        // the round's tasks (GROPHECY_STATIC_UNITS=0): nC phase-C units, then
+        // the A/B tasks, claimed in that order from one counter
+        uint32_t nC = 0, pend = 0xffffffffu;
         // ---- C: tile r, CTA-wide; unit = transformation x ----
         if (r >= 0) {
             const uint32_t b = (uint32_t)r & 1u;
@@ -2368,8 +2371,17 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 for (int rr = 0; rr < 2; rr++) {
                     const unsigned u = rr ? (unsigned)(SW_UNITS - 1 - warp) : (unsigned)warp;
 #else
+                // units claimed in cost order (longest first), then the A/B tasks
+                nC = SW_UNITS;
 #pragma unroll 1
-                for (unsigned u = (unsigned)warp; u < (unsigned)SW_UNITS; u += WARPS) {
+                for (;;) {
+                    unsigned u = 0;
+                    if (lane == 0) u = atomicAdd(&sm.ab_cnt[(r + 1) & 1], 1u);
+                    u = __shfl_sync(FULL, u, 0);
+                    if (u >= (unsigned)SW_UNITS) {
+                        pend = u;   // (an A/B task, or none)
+                        break;
+                    }
 #endif
                     // the unit's position in the design points and its transformation:
                     // in the identity layout by descending cost, else in position order
@@ -2473,10 +2485,14 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                             for (int j = 0; j < NCH; j++) any |= blocks[j] < sat;
                             if (any) {
                                 const uint32_t k = en.hd.y >> 16;   // the entry's kernel
-                                const double *row = S.small_t + (size_t)(I.kx_base + k * X + x) * S.small_stride;
+                                const unsigned long long row =
+                                    reinterpret_cast<unsigned long long>(S.small_t) +
+                                    (unsigned long long)((I.kx_base + k * X + x) * S.small_stride) * sizeof(double);
 #pragma unroll
                                 for (int j = 0; j < NCH; j++)
-                                    if (blocks[j] < sat) tk[j] = __ldg(row + blocks[j]);
+                                    if (blocks[j] < sat)
+                                        tk[j] = __ldg(reinterpret_cast<const double *>(
+                                            row + (unsigned long long)blocks[j] * sizeof(double)));
                             }
                         }
 #pragma unroll
@@ -2512,13 +2528,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
 #pragma unroll
                         for (int j = 0; j < NCH; j++) {
                             const int gj = 32 * ((int)jb * NCH + j) + lane;
-                            double tk = __dmul_rn(__uint2double_rn(sm.it[b][gj]), ti[j]);
+                            double tk = __dmul_rn(sm.it[b][gj], ti[j]);
                             if constexpr (decltype(ONCE)::value) tk = __dadd_rn(to[j], tk);
                             const double2 thd = sm.thd[b][gj];
                             const double tt = __dadd_rn(__dadd_rn(tk, thd.x), thd.y);
                             // chains in increasing record index: strict < keeps the lowest
-                            // (design points past a partial tile's end take no part)
-                            if (tt < cmin && (uint32_t)gj < ngt) {
+                            // (design points past a partial tile's end have tt = +inf)
+                            if (tt < cmin) {
                                 cmin = tt;
                                 cj = j;
                             }
@@ -2546,9 +2562,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             uint32_t *cwb = cw_all + b1 * wmax * (uint32_t)SW_GROUPS;
 #pragma unroll 1
             for (;;) {
-                uint32_t q = 0;
-                if (lane == 0) q = atomicAdd(&sm.ab_cnt[b1], 1u);
-                q = __shfl_sync(FULL, q, 0);
+                uint32_t q = pend;
+                if (q == 0xffffffffu) {
+                    if (lane == 0) q = atomicAdd(&sm.ab_cnt[b1], 1u);
+                    q = __shfl_sync(FULL, q, 0);
+                }
+                pend = 0xffffffffu;
+                q -= nC;
                 if (q >= (uint32_t)WARPS) break;
                 mbar_wait(&sm.rbar, (uint32_t)(r + 1) & 1u);
                 PT_MARK(0);   // waiting for the staged records
@@ -2681,12 +2701,15 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                                                   stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
                         }
                         sm.thd[b1][g] = make_double2(u.th, u.td);
-                        sm.it[b1][g] = i0;
+                        sm.it[b1][g] = (double)i0;
                     }
                 } else if (q == 0 && lane == 0) {
                     sm.perm_ok[b1] = 0u;   // (warp tile 0 is not canonical: the tile is not uniform)
                 }
                 if (lane == 0) sm.wstat[b1][q] = gw == 0 ? SW_EMPTY : (ok ? skel : SW_BAD);
+                // design points past a partial tile's end: t_h2d = +inf makes their
+                // totals +inf (never below the running minimum in phase C)
+                if ((uint32_t)g >= ngt) sm.thd[b1][g] = make_double2(__longlong_as_double(0x7ff0000000000000LL), 0.0);
                 PT_MARK(3);   // phase B (work counts, usage)
             }
         }
