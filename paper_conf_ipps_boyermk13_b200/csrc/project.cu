@@ -1930,7 +1930,7 @@ constexpr unsigned long long SW_TILE = (unsigned long long)SW_GROUPS * CX;   // 
 #define GROPHECY_NCH 8
 #endif
 constexpr int NCH = GROPHECY_NCH;                                   // chains per lane (divides WARPS)
-constexpr int SW_UNITS = CX * (WARPS / NCH);                        // phase-C units (x, chain block)
+
 constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_SMINB
 #define GROPHECY_SMINB 2
@@ -2063,18 +2063,19 @@ __device__ __forceinline__ void group_usage_s(const int4 *pp, uint32_t nhd, uint
 // sm.rec, completing on sm.rbar.  Every generic-proxy read of sm.rec by the
 // CTA happened before the caller's barrier; the fence orders them before the
 // async-proxy writes.
+template <unsigned long long SWT>   // records per CTA tile
 __device__ __forceinline__ void issue_cta_copy(const Params &P, uint32_t (*rec)[SW_TILE],
                                                unsigned long long *rbar, unsigned long long tb)
 {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     const uint32_t bar = smem_u32(rbar);
     // a full tile, or the batch's last one (a whole number of design points)
-    const unsigned long long nrec = P.n - tb < SW_TILE ? P.n - tb : SW_TILE;
+    const unsigned long long nrec = P.n - tb < SWT ? P.n - tb : SWT;
     const uint32_t bytes = (uint32_t)(nrec * sizeof(uint32_t));
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(4 * bytes)
                  : "memory");
     const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
-    if (GROPHECY_TMA_SPLIT == 1 || nrec < SW_TILE) {
+    if (GROPHECY_TMA_SPLIT == 1 || nrec < SWT) {
 #pragma unroll
         for (int a = 0; a < 4; a++)
             asm volatile(
@@ -2083,7 +2084,7 @@ __device__ __forceinline__ void issue_cta_copy(const Params &P, uint32_t (*rec)[
                 "l"(src[a] + tb), "r"(bytes), "r"(bar)
                 : "memory");
     } else {
-        constexpr uint32_t PIECE = (uint32_t)(SW_TILE / GROPHECY_TMA_SPLIT);
+        constexpr uint32_t PIECE = (uint32_t)(SWT / GROPHECY_TMA_SPLIT);
 #pragma unroll
         for (uint32_t q = 0; q < GROPHECY_TMA_SPLIT; q++)
 #pragma unroll
@@ -2117,29 +2118,32 @@ __device__ __forceinline__ void issue_cta_copy_async(const Params &P, uint32_t (
 
 // Phase A of one warp tile of the CTA tile staged at recs: lane l reads its
 // design point's 16 records (rotated 16-byte chunks, conflict-free) and
-// checks the layout of a sweep: every design point of the CTA tile holds 16
+// checks the layout of a sweep: every design point of the CTA tile holds CXT
 // records of one skeleton with equal nx, ny, iters, and the transformations
 // in the same order as the tile's first design point (any fixed order of
 // valid transformations); warp-uniform result.  The batch's last warp tile
 // may hold gw < 32 design points: lanes past it stand in for design point 0.
-template <unsigned long long ROW>   // staged array length (a CTA tile, or one warp tile)
+template <int CXT, unsigned long long ROW>   // design-point size; staged array length
 __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*recs)[ROW], int warp,
                                               int lane, uint32_t gw, uint32_t &s0, uint32_t &n0, uint32_t &m0,
                                               uint32_t &i0)
 {
-    const uint32_t *rec[4] = {recs[0] + warp * CTILE, recs[1] + warp * CTILE, recs[2] + warp * CTILE,
-                              recs[3] + warp * CTILE};
+    constexpr int NCK = CXT / 4;                   // 16-byte chunks per design point and array
+    constexpr uint32_t CTW = 32u * (uint32_t)CXT;   // records per warp tile
+    const uint32_t *rec[4] = {recs[0] + warp * CTW, recs[1] + warp * CTW, recs[2] + warp * CTW,
+                              recs[3] + warp * CTW};
     uint32_t acc;
-    const uint32_t r = ((uint32_t)lane >> 1) & 3u;
+    // rotated chunk order: the 16-byte reads of a quarter warp hit distinct banks
+    const uint32_t r = NCK == 4 ? ((uint32_t)lane >> 1) & 3u : (NCK == 2 ? ((uint32_t)lane >> 2) & 1u : 0u);
     {
-        const uint4 *p = reinterpret_cast<const uint4 *>(rec[0] + lane * CX);
+        const uint4 *p = reinterpret_cast<const uint4 *>(rec[0] + lane * CXT);
 #if GROPHECY_PERM
         const uint4 *g = reinterpret_cast<const uint4 *>(recs[0]);   // the tile's first design point
-        uint4 v[CX / 4], w[CX / 4];
+        uint4 v[NCK], w[NCK];
 #pragma unroll
-        for (int m = 0; m < CX / 4; m++) {
-            v[m] = p[(m + r) & 3u];
-            w[m] = g[(m + r) & 3u];
+        for (int m = 0; m < NCK; m++) {
+            v[m] = p[(m + r) & (uint32_t)(NCK - 1)];
+            w[m] = g[(m + r) & (uint32_t)(NCK - 1)];
         }
         s0 = v[0].x;
         acc = 0;
@@ -2147,17 +2151,17 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
         // consistency — one skeleton, valid transformations — warp 0 checks
         // once per tile: SweepSmem::perm_ok)
 #pragma unroll
-        for (int m = 0; m < CX / 4; m++)
+        for (int m = 0; m < NCK; m++)
             acc |= (v[m].x ^ w[m].x) | (v[m].y ^ w[m].y) | (v[m].z ^ w[m].z) | (v[m].w ^ w[m].w);
 #else
-        uint4 v[CX / 4];
+        uint4 v[NCK];
 #pragma unroll
-        for (int m = 0; m < CX / 4; m++) v[m] = p[(m + r) & 3u];
+        for (int m = 0; m < NCK; m++) v[m] = p[(m + r) & (uint32_t)(NCK - 1)];
         s0 = v[0].x ^ (4u * r);
         acc = s0 & 0xffffu;
 #pragma unroll
-        for (int m = 0; m < CX / 4; m++) {
-            const uint32_t c4 = 4u * ((m + r) & 3u);
+        for (int m = 0; m < NCK; m++) {
+            const uint32_t c4 = 4u * ((m + r) & (uint32_t)(NCK - 1));
             acc |= (v[m].x ^ s0) ^ (c4 + 0u);
             acc |= (v[m].y ^ s0) ^ (c4 + 1u);
             acc |= (v[m].z ^ s0) ^ (c4 + 2u);
@@ -2166,13 +2170,13 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
 #endif
     }
     auto same = [&](int arr, uint32_t &first) {
-        const uint4 *p = reinterpret_cast<const uint4 *>(rec[arr] + lane * CX);
-        uint4 v[CX / 4];
+        const uint4 *p = reinterpret_cast<const uint4 *>(rec[arr] + lane * CXT);
+        uint4 v[NCK];
 #pragma unroll
-        for (int m = 0; m < CX / 4; m++) v[m] = p[(m + r) & 3u];
+        for (int m = 0; m < NCK; m++) v[m] = p[(m + r) & (uint32_t)(NCK - 1)];
         first = v[0].x;
 #pragma unroll
-        for (int m = 0; m < CX / 4; m++)
+        for (int m = 0; m < NCK; m++)
             acc |= (v[m].x ^ first) | (v[m].y ^ first) | (v[m].z ^ first) | (v[m].w ^ first);
     };
     same(1, n0);
@@ -2269,9 +2273,13 @@ __device__ __noinline__ void sweep_bytes(const unsigned long long *poly, const g
 // idle warps prepare the next tile instead of waiting; one CTA barrier ends
 // the round.  The last warp to finish phase A of a tile issues the TMA copy
 // of the CTA's next tile into the (single) record buffer.
-template <bool BEST>
+template <bool BEST, int CXT>   // CXT: records per design point (4, 8 or 16)
 __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Params P)
 {
+    static_assert(CXT == 4 || CXT == 8 || CXT == 16, "design-point sizes of the sweep");
+    constexpr unsigned long long SWT = (unsigned long long)SW_GROUPS * CXT;   // records per CTA tile
+    constexpr unsigned UNITS = (unsigned)CXT * (WARPS / NCH);                // phase-C units
+    constexpr unsigned CPT = (unsigned)(SWT / CTILE);                        // pass-2 chunks per CTA tile
     extern __shared__ __align__(16) unsigned char smem_raw[];
     SweepSmem &sm = *reinterpret_cast<SweepSmem *>(smem_raw);
     const uint32_t wmax = P.sweep_kmax;
@@ -2289,11 +2297,11 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
     // number of design points (its missing warp tiles are empty)
     const bool sweepable = P.aligned && !P.pr.mem;
     const unsigned long long ntiles =
-        sweepable ? P.n / SW_TILE + ((P.n % SW_TILE) && (P.n % CX) == 0 ? 1ull : 0ull) : 0ull;
+        sweepable ? P.n / SWT + ((P.n % SWT) && (P.n % CXT) == 0 ? 1ull : 0ull) : 0ull;
     // everything past them goes to pass 2 as warp tiles (warp-aggregated list appends)
     {
         const unsigned long long nsub = (P.n + CTILE - 1) / CTILE;
-        for (unsigned long long b0 = ntiles * WARPS + (unsigned long long)blockIdx.x * THREADS;
+        for (unsigned long long b0 = ntiles * CPT + (unsigned long long)blockIdx.x * THREADS;
              b0 < nsub; b0 += (unsigned long long)gridDim.x * THREADS) {
             const unsigned long long sub = b0 + tid;
             const bool mine = sub < nsub;
@@ -2317,7 +2325,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         sm.tile_id[0] = blockIdx.x;
         sm.tile_id[1] = atomicAdd(claim, 1u) + gridDim.x;
         sm.tile_id[2] = sm.tile_id[3] = 0xffffffffu;
-        if (blockIdx.x < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, (unsigned long long)blockIdx.x * SW_TILE);
+        if (blockIdx.x < ntiles) issue_cta_copy<SWT>(P, sm.rec, &sm.rbar, (unsigned long long)blockIdx.x * SWT);
     }
     __syncthreads();
     const double rfh = S.rfh, rfl = S.rfl;
@@ -2343,7 +2351,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         if (r >= 0) {
             const uint32_t b = (uint32_t)r & 1u;
             const unsigned long long tile = sm.tile_id[r & 3];
-            const uint32_t ngt = (uint32_t)((P.n - tile * SW_TILE < SW_TILE ? P.n - tile * SW_TILE : SW_TILE) / CX);
+            const uint32_t ngt = (uint32_t)((P.n - tile * SWT < SWT ? P.n - tile * SWT : SWT) / CXT);
             const int gwi = (int)ngt - 32 * warp;
             const uint32_t gw = gwi <= 0 ? 0u : (gwi >= 32 ? 32u : (uint32_t)gwi);
             // uniform: every non-empty warp tile canonical, of one skeleton
@@ -2355,30 +2363,33 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                       sm.perm_ok[b];
             }
             if (!uni) {
-                if (lane == 0 && gw) P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * WARPS + warp);
+                // its pass-2 chunks (CTILE records each), one per warp
+                if (lane == 0 && (unsigned)warp < CPT && (unsigned long long)warp * CTILE < (unsigned long long)ngt * CXT)
+                    P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * CPT + warp);
             } else {
                 const SkelInfo &I = S.skel[s_all];
                 const uint32_t K = I.n_kernels, X = I.n_xforms, pim = I.per_iter_mask;
                 const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
-                const unsigned long long tbase = P.base + tile * SW_TILE;
+                const unsigned long long tbase = P.base + tile * SWT;
                 const uint32_t *cwb = cw_all + b * wmax * (uint32_t)SW_GROUPS;
                 const bool ident = sm.perm_ident[b] != 0u;
 #if GROPHECY_STATIC_UNITS
-                // warp w takes units w and SW_UNITS-1-w: in the identity layout the
-                // costliest transformation pairs with the cheapest
-                static_assert(SW_UNITS == 2 * WARPS, "two units per warp");
+                // units in snake order over the warps (16 units: warp w takes w
+                // and 15 - w; in the identity layout the costliest transformation
+                // pairs with the cheapest)
 #pragma unroll 1
-                for (int rr = 0; rr < 2; rr++) {
-                    const unsigned u = rr ? (unsigned)(SW_UNITS - 1 - warp) : (unsigned)warp;
+                for (unsigned rr = 0; rr < (UNITS + WARPS - 1) / WARPS; rr++) {
+                    const unsigned u = (rr & 1u) ? (rr + 1u) * WARPS - 1u - (unsigned)warp : rr * WARPS + (unsigned)warp;
+                    if (u >= UNITS) continue;
 #else
                 // units claimed in cost order (longest first), then the A/B tasks
-                nC = SW_UNITS;
+                nC = UNITS;
 #pragma unroll 1
                 for (;;) {
                     unsigned u = 0;
                     if (lane == 0) u = atomicAdd(&sm.ab_cnt[(r + 1) & 1], 1u);
                     u = __shfl_sync(FULL, u, 0);
-                    if (u >= (unsigned)SW_UNITS) {
+                    if (u >= UNITS) {
                         pend = u;   // (an A/B task, or none)
                         break;
                     }
@@ -2388,14 +2399,14 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     uint4 hdr;
                     uint32_t pos;
                     if (ident) {
-                        hdr = __ldg(&S.xhdru[I.kx_base + u % CX]);
+                        hdr = __ldg(&S.xhdru[I.kx_base + u % CXT]);
                         pos = hdr.x;
                     } else {
-                        pos = u % CX;
+                        pos = u % CXT;
                         hdr = __ldg(&S.xhdr[I.kx_base + (sm.perm[b][pos] & 0xffffu)]);
                     }
                     const uint32_t x = hdr.x;
-                    const uint32_t jb = u / CX, xf = hdr.w & 0xffu;
+                    const uint32_t jb = u / CXT, xf = hdr.w & 0xffu;
 #if GROPHECY_XINF_SKIP
                     // an infeasible kernel makes every total of the unit +inf (or NaN
                     // at iters = 0): none takes part in the argmin (non-finite totals
@@ -2544,21 +2555,21 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     else totals(std::false_type{});
                     if (cj >= 0) {
                         const int gj = 32 * ((int)jb * NCH + cj) + lane;
-                        const unsigned long long idx = tbase + (unsigned long long)gj * CX + pos;
+                        const unsigned long long idx = tbase + (unsigned long long)gj * CXT + pos;
                         if (better(cmin, idx, best_t, best_i)) {
                             best_t = cmin;
                             best_i = idx;
                         }
                     }
                 }
-                if (lane == 0) cnt_val += gw * (uint32_t)CX;
+                if (lane == 0) cnt_val += gw * (uint32_t)CXT;
             }
         }
         PT_MARK(5);   // phase C (model, totals, argmin)
         // ---- A/B tasks of tile r + 1 (warp tile q, buffer b1) ----
         if (tn < ntiles) {
             const uint32_t b1 = (uint32_t)(r + 1) & 1u;
-            const uint32_t ngt = (uint32_t)((P.n - tn * SW_TILE < SW_TILE ? P.n - tn * SW_TILE : SW_TILE) / CX);
+            const uint32_t ngt = (uint32_t)((P.n - tn * SWT < SWT ? P.n - tn * SWT : SWT) / CXT);
             uint32_t *cwb = cw_all + b1 * wmax * (uint32_t)SW_GROUPS;
 #pragma unroll 1
             for (;;) {
@@ -2575,11 +2586,11 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 const int gwi = (int)ngt - 32 * (int)q;
                 const uint32_t gw = gwi <= 0 ? 0u : (gwi >= 32 ? 32u : (uint32_t)gwi);
                 uint32_t s0 = 0, n0 = 0, m0 = 0, i0 = 0;
-                bool ok = gw ? sweep_phase_a(S, sm.rec, (int)q, lane, gw, s0, n0, m0, i0) : false;
+                bool ok = gw ? sweep_phase_a<CXT>(S, sm.rec, (int)q, lane, gw, s0, n0, m0, i0) : false;
                 const uint32_t skel = s0 >> 16;
                 // the tile's transformation order (its first design point's skx)
                 uint32_t sq = 0;
-                if (q == 0 && lane < CX) sq = sm.rec[0][lane];
+                if (q == 0 && lane < CXT) sq = sm.rec[0][lane];
                 __syncwarp();
                 if (lane == 0) {
                     // every read of the record buffer by this warp is done: the
@@ -2587,7 +2598,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     __threadfence_block();
                     if (atomicAdd(&sm.a_done[b1], 1u) == (unsigned)WARPS - 1u) {
                         const unsigned long long t2 = sm.tile_id[(r + 2) & 3];
-                        if (t2 < ntiles) issue_cta_copy(P, sm.rec, &sm.rbar, t2 * SW_TILE);
+                        if (t2 < ntiles) issue_cta_copy<SWT>(P, sm.rec, &sm.rbar, t2 * SWT);
                     }
                 }
                 PT_MARK(1);   // phase A
@@ -2621,9 +2632,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                             asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.tbar[b1]))
                                          : "memory");
                     }
-                    if (lane < CX) {
+                    if (lane < CXT) {
                         sm.perm[b1][lane] = sq;
-                        const unsigned bad = __ballot_sync(0xffffu, (sq & 0xffffu) != (uint32_t)lane);
+                        const unsigned bad = __ballot_sync((1u << CXT) - 1u, (sq & 0xffffu) != (uint32_t)lane);
                         if (lane == 0) sm.perm_ident[b1] = bad == 0u;
                     }
                     __syncwarp();
@@ -2664,7 +2675,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     if (q == 0) {
                         // the tile's first design point (lane 0's) is itself consistent:
                         // one skeleton, every transformation < n_xforms
-                        const bool okq = (uint32_t)lane >= CX || ((sq >> 16) == skel && (sq & 0xffffu) < I.n_xforms);
+                        const bool okq = (uint32_t)lane >= CXT || ((sq >> 16) == skel && (sq & 0xffffu) < I.n_xforms);
                         const bool all = __all_sync(FULL, okq);
                         if (lane == 0) sm.perm_ok[b1] = all;
                     }
@@ -2835,9 +2846,12 @@ static void set_smem_attrs()
     cudaFuncSetAttribute(canon_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs);
     cudaFuncSetAttribute(general_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
     cudaFuncSetAttribute(general_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
-    cudaFuncSetAttribute(sweep_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)std::min<uint32_t>(SMEM_CTA_MAX, std::max<uint32_t>(sweep_smem_bytes(MAXK, 2u * GROPHECY_MAX_ARRAYS * POLY_CLASSES * 16u),
-                                                 (uint32_t)sizeof(CtaSmem))));
+    const int ss = (int)std::min<uint32_t>(
+        SMEM_CTA_MAX, std::max<uint32_t>(sweep_smem_bytes(MAXK, 2u * GROPHECY_MAX_ARRAYS * POLY_CLASSES * 16u),
+                                         (uint32_t)sizeof(CtaSmem)));
+    cudaFuncSetAttribute(sweep_kernel<true, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
+    cudaFuncSetAttribute(sweep_kernel<true, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
+    cudaFuncSetAttribute(sweep_kernel<true, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
     done = true;
 }
 
@@ -2869,6 +2883,13 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
     return (int)std::max<unsigned long long>(1ull, std::min(want, cap));
 }
 
+// The sweep kernel for the space's design-point size.
+using SweepFn = void (*)(Params);
+static SweepFn sweep_fn(const grophecy_space *s)
+{
+    return s->sweep_cx == 4 ? sweep_kernel<true, 4> : (s->sweep_cx == 8 ? sweep_kernel<true, 8> : sweep_kernel<true, 16>);
+}
+
 // Dynamic shared memory of the (fused) sweep launch: its own layout, or the
 // general tiles' one after the grid barrier, whichever is larger.
 static uint32_t sweep_launch_smem(const grophecy_space *s)
@@ -2884,10 +2905,11 @@ static int sweep_grid(const grophecy_space *s, unsigned long long n)
     set_smem_attrs();
     if (!s->occ_sweep) {
         int o = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, sweep_kernel<true>, THREADS, sweep_launch_smem(s));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, sweep_fn(s), THREADS, sweep_launch_smem(s));
         const_cast<grophecy_space *>(s)->occ_sweep = o < 1 ? 1 : o;
     }
-    const unsigned long long want = std::max<unsigned long long>(1ull, (n + SW_TILE - 1) / SW_TILE);
+    const unsigned long long swt = (unsigned long long)SW_GROUPS * s->sweep_cx;   // records per CTA tile
+    const unsigned long long want = std::max<unsigned long long>(1ull, (n + swt - 1) / swt);
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)s->occ_sweep;
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     return (int)std::min(want, cap);
@@ -2901,10 +2923,12 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
 {
     const unsigned long long cap = (unsigned long long)GROPHECY_TILE_CAP * CTILE;
     const unsigned long long n = P.n;
-    // canonical groups sit at global indices that are multiples of CX (the
-    // sweep layout); a batch starting inside a group (e.g. a shard boundary)
-    // projects its head on its own so the tiles of the rest stay aligned
-    const unsigned long long head = (CX - P.base % CX) % CX;
+    // canonical groups sit at global indices that are multiples of their
+    // size (CX = 16 for the eval kernel, the space's sweep_cx for best mode);
+    // a batch starting inside a group (e.g. a shard boundary) projects its
+    // head on its own so the tiles of the rest stay aligned
+    const unsigned long long gcx = BEST ? s->sweep_cx : (unsigned long long)CX;
+    const unsigned long long head = (gcx - P.base % gcx) % gcx;
     unsigned long long off = 0;
     do {
         Params Q = P;
@@ -2937,7 +2961,8 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
         Q.reset_counters = 0;   // (pass 2 only, below: pass 1's list must survive pass 1)
         // batches the sweep takes nothing of (unaligned, the memory choice) and
         // batches smaller than one tile (pass 2 alone is quicker) go to pass 2 whole
-        Q.direct = BEST && !(Q.aligned && !Q.pr.mem && Q.n >= SW_TILE && sweep_launch_smem(s) <= SMEM_CTA_MAX);
+        Q.direct = BEST && !(Q.aligned && !Q.pr.mem && Q.n >= (unsigned long long)SW_GROUPS * s->sweep_cx &&
+                             sweep_launch_smem(s) <= SMEM_CTA_MAX);
         int launches = 1;
         Q.fused = 0;
         if (BEST && !Q.direct && GROPHECY_FUSED) {
@@ -2957,7 +2982,7 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
             cfg.numAttrs = 1;
             cfg.gridDim = dim3(sweep_grid(s, Q.n));
             cfg.dynamicSmemBytes = sweep_launch_smem(s);
-            e = cudaLaunchKernelEx(&cfg, sweep_kernel<true>, Q);
+            e = cudaLaunchKernelEx(&cfg, sweep_fn(s), Q);
             if (e != cudaSuccess) return cuda_fail(e, "projection (best) sweep launch");
             sm_->counters_clean = true;
             count_launch(1);
@@ -2967,7 +2992,7 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
             // pass 1 alone (pass 2 launched below, programmatically dependent)
             const int grid_s = sweep_grid(s, Q.n);
             Q.sweep_kmax = s->max_wslots;
-            sweep_kernel<true><<<grid_s, THREADS, sweep_launch_smem(s), st>>>(Q);
+            sweep_fn(s)<<<grid_s, THREADS, sweep_launch_smem(s), st>>>(Q);
             launches++;
         } else if (!BEST) {
             const int grid_c = grid_for(s, Q.n, 32, true);

@@ -803,6 +803,15 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
             sp->usage_tbl_bytes = std::max<uint32_t>(
                 sp->usage_tbl_bytes,
                 ((info[q].polyf_nhd & 0xffffu) + (info[q].polyf_nhd >> 16)) * POLY_CLASSES * 16u);
+    // the sweep's design points: records of one (skeleton, nx, ny, iters) for
+    // every transformation, so their size is the skeletons' common n_xforms
+    sp->sweep_cx = 16;
+    {
+        bool same = true;
+        for (uint32_t q = 1; q < n_skels; q++) same = same && skels[q].n_xforms == skels[0].n_xforms;
+        const uint32_t x = skels[0].n_xforms;
+        if (same && (x == 4 || x == 8)) sp->sweep_cx = x;
+    }
     sp->max_kernels = 1;
     sp->max_wslots = 1;
     for (uint32_t q = 0; q < n_skels; q++) {

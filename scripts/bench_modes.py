@@ -113,19 +113,41 @@ def main():
                           "bytes_per_candidate": bpc, "hbm_GBps": gbs, "hbm_frac": gbs / peak,
                           "timer": "cuda events" if ev else "host clock (synchronous call)"}),
               flush=True)
-    # the general (pass-2) kernel alone: the same records with the
-    # transformations of every design point in reverse order, so no tile is
-    # canonical (keys and their runs unchanged)
-    idx = torch.arange(n, device="cuda")
-    idx = (idx // 16) * 16 + 15 - (idx % 16)
-    grec = G.Records(*[getattr(rec, f)[idx].contiguous() for f in ("skx", "nx", "ny", "iters")])
-    gb = grec.batch()
-    sec = timed(lambda: space.best_async(pc, gb, out), reps, True)
-    gbs = 16 * n / sec / 1e9
-    print(json.dumps({"mode": "best_general_path", "n": n, "cand_per_s": n / sec,
-                      "ms": sec * 1e3, "bytes_per_candidate": 16, "hbm_GBps": gbs,
-                      "hbm_frac": gbs / peak, "timer": "cuda events"}), flush=True)
+    # layouts other than the generator's: (1) the transformations of every
+    # design point in reverse order (still a sweep: any fixed order inside
+    # the design points), (2) the records of consecutive design point pairs
+    # interleaved, so no CTA tile is a sweep tile and everything takes the
+    # general (pass-2) path
+    layouts = {
+        "best_reversed_xforms": lambda i: (i // 16) * 16 + 15 - (i % 16),
+        "best_general_path": lambda i: (i // 32) * 32 + (i % 2) * 16 + (i % 32) // 2,
+    }
+    for lname, perm in layouts.items():
+        idx = perm(torch.arange(n, device="cuda"))
+        grec = G.Records(*[getattr(rec, f)[idx].contiguous() for f in ("skx", "nx", "ny", "iters")])
+        gb = grec.batch()
+        sec = timed(lambda: space.best_async(pc, gb, out), reps, True)
+        gbs = 16 * n / sec / 1e9
+        print(json.dumps({"mode": lname, "n": n, "cand_per_s": n / sec,
+                          "ms": sec * 1e3, "bytes_per_candidate": 16, "hbm_GBps": gbs,
+                          "hbm_frac": gbs / peak, "timer": "cuda events"}), flush=True)
     del grec, gb, idx
+    # spaces of skeletons with 8 / 4 transformations: the sweep's design
+    # points have that size (sweep_kernel<.., 8 / 4>)
+    for X in (8, 4):
+        xc = dict(cfg)
+        xc["skeletons"] = [dict(sk, kx=sk["kx"][:X]) for sk in cfg["skeletons"]]
+        xc["n_xforms"] = X
+        xsp = G.Space(xc["skeletons"], S.FX5600)
+        xrec = G.synth_records(dict(xc, n=n))
+        xb = xrec.batch()
+        sec = timed(lambda: xsp.best_async(pc, xb, out), reps, True)
+        gbs = 16 * n / sec / 1e9
+        print(json.dumps({"mode": f"best_x{X}", "n": n, "cand_per_s": n / sec,
+                          "ms": sec * 1e3, "bytes_per_candidate": 16, "hbm_GBps": gbs,
+                          "hbm_frac": gbs / peak, "timer": "cuda events"}), flush=True)
+        xsp.close()
+        del xrec, xb
     # next-row workloads: crossover (NEXT-2) on eval_parts outputs
     ti, to, th, td = parts
     sec = timed(lambda: G.crossover(ti, to, th, td, 1e-3), reps, True)

@@ -96,3 +96,40 @@ def test_large_counts_u64_usage(G, O):
     rec["nx"] = np.repeat(nx, 16)
     rec["ny"] = np.repeat(ny, 16)
     check(G, O, c["skeletons"], rec)
+
+
+def fewer_xforms(cfg, X):
+    """The config with every skeleton cut to its first X transformations
+    (design points of X records: the sweep's design-point size follows the
+    space)."""
+    c = dict(cfg)
+    c["skeletons"] = [dict(s, kx=s["kx"][:X]) for s in cfg["skeletons"]]
+    c["n_xforms"] = X
+    return c
+
+
+@pytest.mark.parametrize("X", [8, 4])
+def test_design_points_of_fewer_transformations(G, O, X):
+    """Spaces whose skeletons have 8 or 4 transformations run the sweep with
+    design points of that size: several full CTA tiles, a partial last one,
+    a reversed order (still a sweep), an index base inside the workload."""
+    c = fewer_xforms(R.config("c4"), X)
+    swt = 256 * X
+    n = 5 * swt + X * 37
+    base = X * 1_000_003
+    rec = R.gen_records(c, base, base + n)
+    check(G, O, c["skeletons"], rec, index_base=base)
+    rev = {k: v.reshape(-1, X)[:, ::-1].reshape(-1).copy() for k, v in rec.items()}
+    check(G, O, c["skeletons"], rev, index_base=base)
+
+
+@pytest.mark.parametrize("X", [8, 4])
+def test_fewer_transformations_bench_layout(G, O, X):
+    """C2-shaped spaces (three skeletons, skeleton boundaries inside CTA
+    tiles) with X transformations: eval record by record and the argmin vs
+    the oracle; the ragged batch end (not a whole design point) goes to the
+    general path."""
+    c = fewer_xforms(R.config("c2"), X)
+    n = 200_003
+    rec = R.gen_records(c, 0, n)
+    check(G, O, c["skeletons"], rec)
