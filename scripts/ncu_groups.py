@@ -26,33 +26,42 @@ for r in rows:
 src = open('paper_conf_ipps_boyermk13_b200/csrc/project.cu').read().splitlines()
 
 
-def find(pat):
+def find(pat, after=0):
     for i, l in enumerate(src):
-        if pat in l:
+        if i >= after and pat in l:
             return i + 1
     return 10 ** 9
 
 
-marks = [('phaseA', '__device__ __forceinline__ bool sweep_phase_a'),
-         ('cls_times', '__device__ __forceinline__ void cls_times'),
+# regions of project.cu in file order (each runs to the next mark)
+MARKS = [('helpers', '__device__ __forceinline__ long long aff8n'),
+         ('usage_fn', '__device__ __forceinline__ void group_usage('),
+         ('other', '// ---- 1-D bulk copies'),
+         ('usage_fn', 'template <bool U32>   // every partial sum below 2^32'),
+         ('other', '// CTA tile copy (thread 0)'),
+         ('phaseA', 'template <int CXT, unsigned long long ROW>'),
+         ('cls_times', '// Saturated kernel times of NCH'),
+         ('other', '// Transfer bytes of a design point'),
          ('prologue', 'sweep_kernel(const Params P)'),
+         ('phaseC', '// ---- C: tile r, CTA-wide'),
+         ('totals', '// totals (P:L77, L147, L167)'),
+         ('phaseA_task', '// ---- A/B tasks of tile r + 1'),
          ('phaseB', '// ---- B: work counts and usage of design point g'),
-         ('phaseC', '// ---- C: CTA-wide'),
-         ('totals', '// totals (P:L77, L147, L167); without run-once kernels t_once ='),
-         ('epilogue', 'if (lane == 0) cnt_val += (uint32_t)CTILE;')]
-marks = sorted([(find(p), n) for n, p in marks])
-gu = (find('__device__ __forceinline__ void group_usage('), find('// ---- 1-D bulk copies'))
+         ('round_end', 'PT_MARK(3);   // phase B'),
+         ('pass2', '// ---- pass 2 in the same (cooperative) launch'),
+         ('other', '// Pass 2: the listed tiles as general')]
+marks, pos = [], 0
+for n, p in MARKS:
+    pos = find(p, pos)
+    marks.append((pos, n))
 ti = sum(x[1] for x in L) or 1
 ts = sum(x[2] for x in L) or 1
 acc = {}
 for ln, i, s, rs in L:
     name = 'other'
-    if gu[0] <= ln < gu[1]:
-        name = 'usage_fn'
-    else:
-        for lo, n in marks:
-            if ln >= lo:
-                name = n
+    for lo, n in marks:
+        if ln >= lo:
+            name = n
     a = acc.setdefault(name, [0, 0, {k: 0 for k in REASONS}])
     a[0] += i
     a[1] += s
