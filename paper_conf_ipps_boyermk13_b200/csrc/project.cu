@@ -1938,9 +1938,6 @@ constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_XINF_SKIP
 #define GROPHECY_XINF_SKIP 1
 #endif
-#ifndef GROPHECY_STATIC_UNITS
-#define GROPHECY_STATIC_UNITS 1
-#endif
 #ifndef GROPHECY_I2F_MAGIC
 #define GROPHECY_I2F_MAGIC 0
 #endif
@@ -1988,6 +1985,8 @@ struct alignas(128) SweepSmem {
     alignas(128) uint32_t rec[4][SW_TILE];   // the CTA tile's SoA records (4 TMA bulk copies)
     unsigned long long rbar;     // completion of the record copies (phase = the tile's sequence number & 1)
     unsigned long long tbar[2];  // usage-table decision of the tile of sequence parity p (TMA or plain arrive)
+    unsigned long long abar[2];  // the WARPS A/B tasks of the tile of sequence parity p are done
+    unsigned long long cbar[2];  // every warp's phase C of the tile of sequence parity p is done
     // per buffer b (the tile of sequence parity b), design point g = 32 * (A/B task) + lane
     alignas(16) double2 thd[SW_NB][SW_GROUPS];   // {t_h2d, t_d2h}: one 16-byte read in the totals
     double it[SW_NB][SW_GROUPS];                 // iterations
@@ -1996,7 +1995,7 @@ struct alignas(128) SweepSmem {
     uint32_t perm[SW_NB][CX];            // the tile's skx at each position of a design point (its first one's)
     uint32_t perm_ident[SW_NB];          // perm is the identity (units follow the cost order)
     uint32_t perm_ok[SW_NB];             // the tile's first design point is consistent
-    uint32_t ab_cnt[2];                  // A/B task claims of the tile of sequence parity p
+    uint32_t ab_cnt[4];                  // A/B task claims of the tile of sequence number mod 4
     uint32_t a_done[2];                  // phase-A completions of the tile of sequence parity p
     uint32_t tile_id[4];                 // the CTA's tiles by sequence number mod 4 (claimed ahead)
     uint32_t tbl_skel;                   // skeleton whose usage table is staged (SW_BAD: none)
@@ -2319,8 +2318,12 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
         mbar_init(&sm.rbar, 1);
         mbar_init(&sm.tbar[0], 1);
         mbar_init(&sm.tbar[1], 1);
+        for (int i = 0; i < 2; i++) {
+            mbar_init(&sm.abar[i], WARPS);
+            mbar_init(&sm.cbar[i], WARPS);
+        }
         sm.tbl_skel = SW_BAD;
-        sm.ab_cnt[0] = sm.ab_cnt[1] = 0;
+        sm.ab_cnt[0] = sm.ab_cnt[1] = sm.ab_cnt[2] = sm.ab_cnt[3] = 0;
         sm.a_done[0] = sm.a_done[1] = 0;
         sm.tile_id[0] = blockIdx.x;
         sm.tile_id[1] = atomicAdd(claim, 1u) + gridDim.x;
@@ -2334,22 +2337,14 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
 #endif
 #pragma unroll 1
     for (int r = -1;; r++) {
-        // counters of tile r (used in round r - 1) are next used for tile r + 2
-        if (tid == 0) {
-            sm.ab_cnt[r & 1] = 0;
-            sm.a_done[r & 1] = 0;
-        }
-        const unsigned long long tn = sm.tile_id[(r + 1) & 3];   // tile r + 1
-        // tile r + 3 (its copy is issued in round r + 1): claimed now, stored
-        // before the round's barrier (the atomic's latency overlaps the round)
-        unsigned claimed = 0;
-        if (tid == 0 && tn < ntiles) claimed = atomicAdd(claim, 1u);
-        // the round's tasks (GROPHECY_STATIC_UNITS=0): nC phase-C units, then
-        // the A/B tasks, claimed in that order from one counter
-        uint32_t nC = 0, pend = 0xffffffffu;
+        // tile r + 1 (stored by the first A/B task of tile r - 1, which every
+        // warp has seen complete: the abar wait of its phase C of tile r - 1)
+        const unsigned long long tn = sm.tile_id[(r + 1) & 3];
         // ---- C: tile r, CTA-wide; unit = transformation x ----
         if (r >= 0) {
             const uint32_t b = (uint32_t)r & 1u;
+            mbar_wait(&sm.abar[b], ((uint32_t)r >> 1) & 1u);   // every A/B task of tile r
+            PT_MARK(4);   // waiting for tile r's A/B tasks
             const unsigned long long tile = sm.tile_id[r & 3];
             const uint32_t ngt = (uint32_t)((P.n - tile * SWT < SWT ? P.n - tile * SWT : SWT) / CXT);
             const int gwi = (int)ngt - 32 * warp;
@@ -2373,7 +2368,6 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 const unsigned long long tbase = P.base + tile * SWT;
                 const uint32_t *cwb = cw_all + b * wmax * (uint32_t)SW_GROUPS;
                 const bool ident = sm.perm_ident[b] != 0u;
-#if GROPHECY_STATIC_UNITS
                 // units in snake order over the warps (16 units: warp w takes w
                 // and 15 - w; in the identity layout the costliest transformation
                 // pairs with the cheapest)
@@ -2381,19 +2375,6 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 for (unsigned rr = 0; rr < (UNITS + WARPS - 1) / WARPS; rr++) {
                     const unsigned u = (rr & 1u) ? (rr + 1u) * WARPS - 1u - (unsigned)warp : rr * WARPS + (unsigned)warp;
                     if (u >= UNITS) continue;
-#else
-                // units claimed in cost order (longest first), then the A/B tasks
-                nC = UNITS;
-#pragma unroll 1
-                for (;;) {
-                    unsigned u = 0;
-                    if (lane == 0) u = atomicAdd(&sm.ab_cnt[(r + 1) & 1], 1u);
-                    u = __shfl_sync(FULL, u, 0);
-                    if (u >= UNITS) {
-                        pend = u;   // (an A/B task, or none)
-                        break;
-                    }
-#endif
                     // the unit's position in the design points and its transformation:
                     // in the identity layout by descending cost, else in position order
                     uint4 hdr;
@@ -2564,23 +2545,31 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 }
                 if (lane == 0) cnt_val += gw * (uint32_t)CXT;
             }
+            __syncwarp();
+            if (lane == 0)
+                asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.cbar[b])) : "memory");
         }
         PT_MARK(5);   // phase C (model, totals, argmin)
-        // ---- A/B tasks of tile r + 1 (warp tile q, buffer b1) ----
-        if (tn < ntiles) {
+        if (tn >= ntiles) break;
+        // ---- A/B tasks of tile r + 1 (warp tile q, buffer b1), claimed until
+        // none is left: every warp makes exactly one failing claim per tile, so
+        // the 2 WARPS-th claim is the tile's last and resets the counter ----
+        {
             const uint32_t b1 = (uint32_t)(r + 1) & 1u;
             const uint32_t ngt = (uint32_t)((P.n - tn * SWT < SWT ? P.n - tn * SWT : SWT) / CXT);
             uint32_t *cwb = cw_all + b1 * wmax * (uint32_t)SW_GROUPS;
 #pragma unroll 1
             for (;;) {
-                uint32_t q = pend;
-                if (q == 0xffffffffu) {
-                    if (lane == 0) q = atomicAdd(&sm.ab_cnt[b1], 1u);
-                    q = __shfl_sync(FULL, q, 0);
+                uint32_t q = 0;
+                if (lane == 0) {
+                    q = atomicAdd(&sm.ab_cnt[(r + 1) & 3], 1u);
+                    if (q == 2u * WARPS - 1u) sm.ab_cnt[(r + 1) & 3] = 0u;
                 }
-                pend = 0xffffffffu;
-                q -= nC;
+                q = __shfl_sync(FULL, q, 0);
                 if (q >= (uint32_t)WARPS) break;
+                // the first task claims tile r + 3 (stored at its end)
+                unsigned claimed = 0;
+                if (q == 0 && lane == 0) claimed = atomicAdd(claim, 1u);
                 mbar_wait(&sm.rbar, (uint32_t)(r + 1) & 1u);
                 PT_MARK(0);   // waiting for the staged records
                 const int gwi = (int)ngt - 32 * (int)q;
@@ -2597,11 +2586,15 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     // tile's last one releases it to the copy of tile r + 2
                     __threadfence_block();
                     if (atomicAdd(&sm.a_done[b1], 1u) == (unsigned)WARPS - 1u) {
+                        __threadfence_block();
+                        sm.a_done[b1] = 0u;   // (next used by tile r + 3)
                         const unsigned long long t2 = sm.tile_id[(r + 2) & 3];
                         if (t2 < ntiles) issue_cta_copy<SWT>(P, sm.rec, &sm.rbar, t2 * SWT);
                     }
                 }
                 PT_MARK(1);   // phase A
+                // buffer b1 was read by the phase C of tile r - 1
+                if (r >= 1) mbar_wait(&sm.cbar[b1], ((uint32_t)(r - 1) >> 1) & 1u);
                 if (q == 0) {
                     // warp tile 0's skeleton decides the tile's usage table: staged
                     // when it changes (every reader of the previous one finished in
@@ -2721,13 +2714,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 // design points past a partial tile's end: t_h2d = +inf makes their
                 // totals +inf (never below the running minimum in phase C)
                 if ((uint32_t)g >= ngt) sm.thd[b1][g] = make_double2(__longlong_as_double(0x7ff0000000000000LL), 0.0);
+                if (q == 0 && lane == 0) sm.tile_id[(r + 3) & 3] = claimed + gridDim.x;   // tile r + 3
+                __syncwarp();
+                if (lane == 0)
+                    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&sm.abar[b1])) : "memory");
                 PT_MARK(3);   // phase B (work counts, usage)
             }
         }
-        if (tid == 0 && tn < ntiles) sm.tile_id[(r + 3) & 3] = claimed + gridDim.x;
-        __syncthreads();
-        PT_MARK(4);   // the round's barrier
-        if (tn >= ntiles) break;
     }
     // the bytes of each lane's running best (its design point's usage; the
     // record buffer is idle now: no copy is in flight after the last round)
