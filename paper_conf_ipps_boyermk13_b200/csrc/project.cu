@@ -33,6 +33,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <type_traits>
 #include <cmath>
@@ -2905,6 +2906,11 @@ static int sweep_grid(const grophecy_space *s, unsigned long long n)
     const unsigned long long want = std::max<unsigned long long>(1ull, (n + swt - 1) / swt);
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)s->occ_sweep;
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
+    // test hook: a small grid makes every CTA run many tiles in sequence
+    if (const char *g = getenv("GROPHECY_SWEEP_GRID")) {
+        const long v = atol(g);
+        if (v > 0) cap = std::min<unsigned long long>(cap, (unsigned long long)v);
+    }
     return (int)std::min(want, cap);
 }
 

@@ -133,3 +133,22 @@ def test_fewer_transformations_bench_layout(G, O, X):
     n = 200_003
     rec = R.gen_records(c, 0, n)
     check(G, O, c["skeletons"], rec)
+
+
+@pytest.mark.parametrize("grid", [1, 3])
+def test_many_tiles_per_cta(G, O, monkeypatch, grid):
+    """A sweep grid of 1 or 3 CTAs (GROPHECY_SWEEP_GRID): every CTA runs
+    dozens of tiles back to back through its per-tile barriers and counters,
+    with the skeleton (the staged usage table) changing every 4 tiles,
+    non-uniform tiles (one design point in another order) between uniform
+    ones, and a partial last tile; eval and the argmin vs the oracle."""
+    c = R.config("c4")
+    c = dict(c, n=16 * 4 * 4096)       # 16 skeletons, a boundary every 4 tiles
+    n = c["n"] - 16 * 29               # partial last tile
+    rec = R.gen_records(c, 0, n)
+    for t in (5, 6, 17, 40):           # tiles with one design point reversed
+        i = t * 4096 + 16 * 7
+        for k in rec:
+            rec[k][i:i + 16] = rec[k][i:i + 16][::-1]
+    monkeypatch.setenv("GROPHECY_SWEEP_GRID", str(grid))
+    check(G, O, c["skeletons"], rec)
