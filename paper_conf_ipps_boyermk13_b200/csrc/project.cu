@@ -1187,8 +1187,8 @@ __device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsi
 {
     const SpaceDev &S = P.S;
     const unsigned lt = (1u << lane) - 1u;
-        // ---- A: records q = lane + 32 j (coalesced 32-bit loads), keys, run
-        //      heads (ballots) and slot ids in record order ----
+        // ---- A: records q = lane + 32 j (coalesced 32-bit loads), keys, one
+        //      slot per distinct key of each 32 records (match + ballots) ----
         uint32_t skx[RPT], nx[RPT], ny[RPT], it[RPT];
 #pragma unroll
         for (int j = 0; j < RPT; j++) {
@@ -1219,13 +1219,16 @@ __device__ __forceinline__ void general_tile(const Params &P, WarpSmem &ws, unsi
         const unsigned le = (2u << lane) - 1u;   // lanes <= this one
 #pragma unroll
         for (int j = 0; j < RPT; j++) {
-            // predecessor of record lane + 32 j is lane - 1 (same j) or lane 31 of j - 1
-            unsigned long long prev = __shfl_up_sync(FULL, key[j], 1);
-            const unsigned long long last_prev = j ? __shfl_sync(FULL, key[j > 0 ? j - 1 : 0], 31) : ~0ull;
-            if (lane == 0) prev = last_prev;
-            const bool head = key[j] != ~0ull && key[j] != prev;
+            // one slot per distinct key of the 32 records lane + 32 j (equal keys
+            // need not be adjacent: any order of a design point's records),
+            // its lowest lane the head; slots in head order
+            const unsigned mk = __match_any_sync(FULL, key[j]);
+            const int leader = __ffs(mk) - 1;
+            const bool head = key[j] != ~0ull && lane == leader;
             const unsigned hb = __ballot_sync(FULL, head);
-            const int slot = key[j] == ~0ull ? -1 : (int)(nslots + __popc(hb & le)) - 1;
+            const int hslot = (int)(nslots + __popc(hb & le)) - 1;
+            const int lslot = __shfl_sync(FULL, hslot, leader);   // (every lane: FULL mask)
+            const int slot = key[j] == ~0ull ? -1 : lslot;
             nslots += __popc(hb);
             const int q = lane + 32 * j;
             ws.rec_skx[q] = skx[j];

@@ -152,3 +152,17 @@ def test_many_tiles_per_cta(G, O, monkeypatch, grid):
             rec[k][i:i + 16] = rec[k][i:i + 16][::-1]
     monkeypatch.setenv("GROPHECY_SWEEP_GRID", str(grid))
     check(G, O, c["skeletons"], rec)
+
+
+def test_interleaved_design_points_general_path(G, O):
+    """The records of design point pairs interleaved record by record (equal
+    keys not adjacent): no sweep tile; the general path groups the equal keys
+    of each 32 records (one usage evaluation per key); vs the oracle."""
+    c = R.config("c4")
+    n = 6 * 4096 + 32 * 11 + 5
+    base = 16 * 3_000_000
+    rec = R.gen_records(c, base, base + n)
+    i = np.arange(n)
+    blk = (i // 32) * 32
+    idx = np.where(blk + 32 <= n, blk + (i % 2) * 16 + (i % 32) // 2, i)
+    check(G, O, c["skeletons"], {k: v[idx] for k, v in rec.items()}, index_base=base)
