@@ -1945,20 +1945,8 @@ constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_I2F_MAGIC
 #define GROPHECY_I2F_MAGIC 0
 #endif
-#ifndef GROPHECY_LDGSTS
-#define GROPHECY_LDGSTS 0
-#endif
-#ifndef GROPHECY_DIAG_NOLOAD
-#define GROPHECY_DIAG_NOLOAD 0
-#endif
 #ifndef GROPHECY_DISPATCH_TREE
 #define GROPHECY_DISPATCH_TREE 1   // class dispatch by uniform branches (0: switch)
-#endif
-#ifndef GROPHECY_TMA_SPLIT
-#define GROPHECY_TMA_SPLIT 1   // bulk copies per SoA array of a CTA tile
-#endif
-#ifndef GROPHECY_PF
-#define GROPHECY_PF 0
 #endif
 #ifndef GROPHECY_FUSED
 #define GROPHECY_FUSED 1
@@ -2078,45 +2066,13 @@ __device__ __forceinline__ void issue_cta_copy(const Params &P, uint32_t (*rec)[
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(4 * bytes)
                  : "memory");
     const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
-    if (GROPHECY_TMA_SPLIT == 1 || nrec < SWT) {
-#pragma unroll
-        for (int a = 0; a < 4; a++)
-            asm volatile(
-                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                    smem_u32(rec[a])),
-                "l"(src[a] + tb), "r"(bytes), "r"(bar)
-                : "memory");
-    } else {
-        constexpr uint32_t PIECE = (uint32_t)(SWT / GROPHECY_TMA_SPLIT);
-#pragma unroll
-        for (uint32_t q = 0; q < GROPHECY_TMA_SPLIT; q++)
-#pragma unroll
-            for (int a = 0; a < 4; a++)
-                asm volatile(
-                    "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                        smem_u32(rec[a] + q * PIECE)),
-                    "l"(src[a] + tb + q * PIECE), "r"(PIECE * 4u), "r"(bar)
-                    : "memory");
-    }
-}
-
-// The same CTA tile copy issued by every thread as 16-byte cp.async
-// (LDGSTS through L1) whose completions arrive on sm.rbar (initialised with
-// THREADS arrivals): many requests in flight per SM instead of 4 bulk copies.
-__device__ __forceinline__ void issue_cta_copy_async(const Params &P, uint32_t (*rec)[SW_TILE],
-                                                     unsigned long long *rbar, unsigned long long tb,
-                                                     int tid)
-{
-    const uint32_t *src[4] = {P.skx, P.nx, P.ny, P.iters};
-    constexpr int CHUNKS = (int)(SW_TILE / 4);   // 16-byte chunks per array
 #pragma unroll
     for (int a = 0; a < 4; a++)
-#pragma unroll
-        for (int c = tid; c < CHUNKS; c += THREADS)
-            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(rec[a] + 4 * c)),
-                         "l"(src[a] + tb + 4 * c)
-                         : "memory");
-    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(rbar)) : "memory");
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                smem_u32(rec[a])),
+            "l"(src[a] + tb), "r"(bytes), "r"(bar)
+            : "memory");
 }
 
 // Phase A of one warp tile of the CTA tile staged at recs: lane l reads its
