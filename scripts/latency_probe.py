@@ -34,7 +34,8 @@ def lat(space, pc, rec, reps=300):
 pc = G.pcie(G.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL))
 c2 = R.config("c2")
 one = dict(c2, skeletons=c2["skeletons"][:1], rules=c2["rules"][:1])
-for name, cfg, n in (("c2", c2, 10**6), ("c2_one_skeleton", one, 10**6), ("c2_one_tile", one, 4096),
+for name, cfg, n in (("c2", c2, 10**6), ("c2_tile_aligned", c2, 3 * 81 * 4096),
+                     ("c2_one_skeleton", one, 10**6), ("c2_one_tile", one, 4096),
                      ("c2_37_tiles", one, 37 * 4096), ("c1", R.config("c1"), 16)):
     sp = G.Space(cfg["skeletons"], S.FX5600)
     rec = G.synth_records(dict(cfg, n=n))
