@@ -2225,13 +2225,16 @@ __device__ __noinline__ void sweep_bytes(const unsigned long long *poly, const g
     hd[1] = u.d;
 }
 
-// The sweep kernel works in rounds: round r runs phase C of the CTA's tile r
-// (its phase-B results in buffer r & 1) and the phase A/B tasks of tile r + 1
-// (one per warp tile, buffer (r + 1) & 1), claimed from a shared counter by
-// the warps as they run out of phase-C units, so a transformation-poor tile's
-// idle warps prepare the next tile instead of waiting; one CTA barrier ends
-// the round.  The last warp to finish phase A of a tile issues the TMA copy
-// of the CTA's next tile into the (single) record buffer.
+// The sweep kernel works in rounds: in round r a warp runs its phase-C units
+// of the CTA's tile r (phase-B results in buffer r & 1), then claims phase
+// A/B tasks of tile r + 1 (one per warp tile, buffer (r + 1) & 1) from a
+// shared counter, so a transformation-poor tile's idle warps prepare the next
+// tile instead of waiting.  No CTA barrier: per-tile mbarriers order the
+// phases (abar: tile r's A/B tasks done -> its phase C; cbar: every warp's
+// phase C of tile r - 1 done -> the A/B tasks of tile r + 1 reuse its
+// buffer; rbar: records staged; tbar: usage-table decision).  The last warp
+// to finish phase A of a tile issues the TMA copy of the CTA's next tile
+// into the (single) record buffer.
 template <bool BEST, int CXT>   // CXT: records per design point (4, 8 or 16)
 __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Params P)
 {

@@ -36,7 +36,7 @@ fn(out)
 space.best(pc, rec)
 torch.cuda.synchronize()
 fn(out)
-names = ["wait records (TMA)", "phase A", "table decision", "phase B", "round barrier", "phase C"]
+names = ["wait records (TMA)", "phase A", "table decision", "phase B", "wait A/B tasks (abar)", "phase C"]
 tot = sum(out[i] for i in range(6))
 for i, nm in enumerate(names):
     print(f"{nm:22s} {100 * out[i] / tot:6.2f} %")
