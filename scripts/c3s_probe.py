@@ -17,6 +17,7 @@ from synth import skeletons as S  # noqa: E402
 name = sys.argv[1] if len(sys.argv) > 1 else "c3s"
 n = int(sys.argv[2]) if len(sys.argv) > 2 else 10**7
 cfg = R.config(name)
+cfg = dict(cfg, n=max(cfg["n"], n))   # (the same recipe at a larger size)
 pc = G.pcie(G.fit_pcie(S.PAPER_TS, S.PAPER_TL, S.PAPER_SL))
 space = G.Space(cfg["skeletons"], S.FX5600)
 rec = G.synth_records(cfg, 0, n)
