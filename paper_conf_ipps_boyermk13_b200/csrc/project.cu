@@ -2141,7 +2141,7 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
     same(1, n0);
     same(2, m0);
     same(3, i0);
-    {
+    if (gw < 32u) {   // (warp-uniform: the batch's last warp tile)
         const uint32_t a0 = __shfl_sync(FULL, acc, 0), s00 = __shfl_sync(FULL, s0, 0);
         const uint32_t n00 = __shfl_sync(FULL, n0, 0), m00 = __shfl_sync(FULL, m0, 0);
         const uint32_t i00 = __shfl_sync(FULL, i0, 0);
