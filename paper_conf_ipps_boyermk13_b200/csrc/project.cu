@@ -2153,10 +2153,11 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
             i0 = i00;
         }
     }
+    // (acc == 0 in every lane: every record equals the tile's first design
+    // point's in skx, so the warp tile has one skeleton)
     const uint32_t skel = s0 >> 16;
-    const uint32_t skel_l0 = __shfl_sync(FULL, skel, 0);
     bool ok = acc == 0 && skel < S.n_skels && n0 - 1u < GROPHECY_MAX_DIM &&
-              m0 - 1u < GROPHECY_MAX_DIM && i0 >= 1 && skel == skel_l0;
+              m0 - 1u < GROPHECY_MAX_DIM && i0 >= 1;
     if (ok) ok = (S.skel[skel].flags & SKF_TABULATED) != 0;
     return __all_sync(FULL, ok);
 }
@@ -2635,7 +2636,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                         const bool all = __all_sync(FULL, okq);
                         if (lane == 0) sm.perm_ok[b1] = all;
                     }
-                    ok = !__any_sync(FULL, huge) && __all_sync(FULL, n0 >= I.plan_tx && m0 >= I.plan_ty);
+                    ok = __all_sync(FULL, !huge && n0 >= I.plan_tx && m0 >= I.plan_ty);
                     if (ok) {
                         Usage u = {0ull, 0ull, 0.0, 0.0};
                         const uint32_t stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
