@@ -1987,6 +1987,8 @@ struct alignas(128) SweepSmem {
     uint32_t perm[SW_NB][CX];            // the tile's skx at each position of a design point (its first one's)
     uint32_t perm_ident[SW_NB];          // perm is the identity (units follow the cost order)
     uint32_t perm_ok[SW_NB];             // the tile's first design point is consistent
+    uint4 uhdr[SW_NB][CX];               // per phase-C unit: its program header (xhdr layout) ...
+    uint32_t upos[SW_NB][CX];            // ... and its position in the design points
     uint32_t ab_cnt[4];                  // A/B task claims of the tile of sequence number mod 4
     uint32_t a_done[2];                  // phase-A completions of the tile of sequence parity p
     uint32_t tile_id[4];                 // the CTA's tiles by sequence number mod 4 (claimed ahead)
@@ -2331,7 +2333,6 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
                 const unsigned long long tbase = P.base + tile * SWT;
                 const uint32_t *cwb = cw_all + b * wmax * (uint32_t)SW_GROUPS;
-                const bool ident = sm.perm_ident[b] != 0u;
                 // units in snake order over the warps (16 units: warp w takes w
                 // and 15 - w; in the identity layout the costliest transformation
                 // pairs with the cheapest)
@@ -2339,17 +2340,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 for (unsigned rr = 0; rr < (UNITS + WARPS - 1) / WARPS; rr++) {
                     const unsigned u = (rr & 1u) ? (rr + 1u) * WARPS - 1u - (unsigned)warp : rr * WARPS + (unsigned)warp;
                     if (u >= UNITS) continue;
-                    // the unit's position in the design points and its transformation:
-                    // in the identity layout by descending cost, else in position order
-                    uint4 hdr;
-                    uint32_t pos;
-                    if (ident) {
-                        hdr = __ldg(&S.xhdru[I.kx_base + u % CXT]);
-                        pos = hdr.x;
-                    } else {
-                        pos = u % CXT;
-                        hdr = __ldg(&S.xhdr[I.kx_base + (sm.perm[b][pos] & 0xffffu)]);
-                    }
+                    // the unit's transformation and position (set by the tile's first task)
+                    const uint4 hdr = sm.uhdr[b][u % CXT];
+                    const uint32_t pos = sm.upos[b][u % CXT];
                     const uint32_t x = hdr.x;
                     const uint32_t jb = u / CXT, xf = hdr.w & 0xffu;
 #if GROPHECY_XINF_SKIP
@@ -2635,6 +2628,22 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                         const bool okq = (uint32_t)lane >= CXT || ((sq >> 16) == skel && (sq & 0xffffu) < I.n_xforms);
                         const bool all = __all_sync(FULL, okq);
                         if (lane == 0) sm.perm_ok[b1] = all;
+                        // the units' headers for phase C: in the identity layout unit u
+                        // is the u-th costliest transformation (at its own position),
+                        // else the transformation at position u
+                        if (all && (uint32_t)lane < CXT) {
+                            uint4 h;
+                            uint32_t pos;
+                            if (sm.perm_ident[b1]) {
+                                h = __ldg(&S.xhdru[I.kx_base + lane]);
+                                pos = h.x;
+                            } else {
+                                h = __ldg(&S.xhdr[I.kx_base + (sq & 0xffffu)]);
+                                pos = (uint32_t)lane;
+                            }
+                            sm.uhdr[b1][lane] = h;
+                            sm.upos[b1][lane] = pos;
+                        }
                     }
                     ok = __all_sync(FULL, !huge && n0 >= I.plan_tx && m0 >= I.plan_ty);
                     if (ok) {
