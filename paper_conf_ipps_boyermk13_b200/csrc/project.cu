@@ -1982,7 +1982,7 @@ struct alignas(128) SweepSmem {
     // per buffer b (the tile of sequence parity b), design point g = 32 * (A/B task) + lane
     alignas(16) double2 thd[SW_NB][SW_GROUPS];   // {t_h2d, t_d2h}: one 16-byte read in the totals
     double it[SW_NB][SW_GROUPS];                 // iterations
-    uint32_t smallk[SW_NB][SW_GROUPS];   // per design point: work slots whose grid may be unsaturated
+    uint32_t smallw[SW_NB][WARPS];       // per warp tile: work slots whose grid may be unsaturated
     uint32_t wstat[SW_NB][WARPS];        // A/B result per warp tile: its skeleton, SW_BAD or SW_EMPTY
     uint32_t perm[SW_NB][CX];            // the tile's skx at each position of a design point (its first one's)
     uint32_t perm_ident[SW_NB];          // perm is the identity (units follow the cost order)
@@ -2333,6 +2333,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
                 const unsigned long long tbase = P.base + tile * SWT;
                 const uint32_t *cwb = cw_all + b * wmax * (uint32_t)SW_GROUPS;
+                // work slots whose grid may be unsaturated for one of the tile's
+                // design points (a unit covers all of them: its chains are the
+                // tile's warp tiles)
+                static_assert(UNITS == (unsigned)CXT, "one chain block per unit");
+                uint32_t gk = 0;
+#pragma unroll
+                for (int w = 0; w < WARPS; w++) gk |= sm.smallw[b][w];
                 // units in snake order over the warps (16 units: warp w takes w
                 // and 15 - w; in the identity layout the costliest transformation
                 // pairs with the cheapest)
@@ -2353,11 +2360,6 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
 #endif
                     const KxProg *pe = S.xprog + hdr.y;
                     const uint32_t n_it = hdr.z & 0xffffu, n_all = n_it + (hdr.z >> 16);
-                    // work slots whose grid may be unsaturated for one of the warp's design points
-                    uint32_t gk = 0;
-#pragma unroll
-                    for (int j = 0; j < NCH; j++) gk |= sm.smallk[b][32 * ((int)jb * NCH + j) + lane];
-                    gk = __reduce_or_sync(FULL, gk);
                     double ti[NCH], to[NCH];
 #pragma unroll
                     for (int j = 0; j < NCH; j++) ti[j] = to[j] = 0.0;
@@ -2593,6 +2595,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 PT_MARK(2);   // the tile's usage-table decision
                 // ---- B: work counts and usage of design point g ----
                 const int g = (int)q * 32 + lane;
+                uint32_t wsmall = 0;
                 if (ok) {
                     const SkelInfo &I = S.skel[skel];   // warp-uniform
                     const uint32_t n_arrays = I.n_arrays, nw = I.n_wslots;
@@ -2621,7 +2624,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                             small |= (w < __ldg(wsat + j) ? 1u : 0u) << j;
                         }
                     }
-                    sm.smallk[b1][g] = small;
+                    wsmall = __reduce_or_sync(FULL, small);
                     if (q == 0) {
                         // the tile's first design point (lane 0's) is itself consistent:
                         // one skeleton, every transformation < n_xforms
@@ -2683,7 +2686,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 } else if (q == 0 && lane == 0) {
                     sm.perm_ok[b1] = 0u;   // (warp tile 0 is not canonical: the tile is not uniform)
                 }
-                if (lane == 0) sm.wstat[b1][q] = gw == 0 ? SW_EMPTY : (ok ? skel : SW_BAD);
+                if (lane == 0) {
+                    sm.wstat[b1][q] = gw == 0 ? SW_EMPTY : (ok ? skel : SW_BAD);
+                    sm.smallw[b1][q] = wsmall;
+                }
                 // design points past a partial tile's end: t_h2d = +inf makes their
                 // totals +inf (never below the running minimum in phase C)
                 if ((uint32_t)g >= ngt) sm.thd[b1][g] = make_double2(__longlong_as_double(0x7ff0000000000000LL), 0.0);
