@@ -1989,6 +1989,7 @@ struct alignas(128) SweepSmem {
     uint32_t perm_ok[SW_NB];             // the tile's first design point is consistent
     uint4 uhdr[SW_NB][CX];               // per phase-C unit: its program header (xhdr layout) ...
     uint32_t upos[SW_NB][CX];            // ... and its position in the design points
+    uint4 tinf[SW_NB];                   // the tile's skeleton: {kx_base, n_xforms, has run-once kernels, -}
     uint32_t ab_cnt[4];                  // A/B task claims of the tile of sequence number mod 4
     uint32_t a_done[2];                  // phase-A completions of the tile of sequence parity p
     uint32_t tile_id[4];                 // the CTA's tiles by sequence number mod 4 (claimed ahead)
@@ -2328,9 +2329,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 if (lane == 0 && (unsigned)warp < CPT && (unsigned long long)warp * CTILE < (unsigned long long)ngt * CXT)
                     P.tile_list[atomicAdd(P.tile_count, 1u)] = (uint32_t)(tile * CPT + warp);
             } else {
-                const SkelInfo &I = S.skel[s_all];
-                const uint32_t K = I.n_kernels, X = I.n_xforms, pim = I.per_iter_mask;
-                const uint32_t kmask = K == 32 ? 0xffffffffu : (1u << K) - 1u;
+                // the tile's skeleton (set by its first task)
+                const uint4 ti4 = sm.tinf[b];
+                const uint32_t kx_base = ti4.x, X = ti4.y;
+                const bool has_once = ti4.z != 0u;
                 const unsigned long long tbase = P.base + tile * SWT;
                 const uint32_t *cwb = cw_all + b * wmax * (uint32_t)SW_GROUPS;
                 // work slots whose grid may be unsaturated for one of the tile's
@@ -2438,7 +2440,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                                 const uint32_t k = en.hd.y >> 16;   // the entry's kernel
                                 const unsigned long long row =
                                     reinterpret_cast<unsigned long long>(S.small_t) +
-                                    (unsigned long long)((I.kx_base + k * X + x) * S.small_stride) * sizeof(double);
+                                    (unsigned long long)((kx_base + k * X + x) * S.small_stride) * sizeof(double);
 #pragma unroll
                                 for (int j = 0; j < NCH; j++)
                                     if (blocks[j] < sat)
@@ -2472,7 +2474,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
 #endif
                     // totals; without run-once kernels t_once =
                     // +0.0 and +0.0 + iters * t_iter = iters * t_iter exactly
-                    const bool once = (pim & kmask) != kmask || (xf & XINF_ONCE);
+                    const bool once = has_once || (xf & XINF_ONCE);
                     double cmin = inf;
                     int cj = -1;
                     auto totals = [&](auto ONCE) {
@@ -2634,6 +2636,10 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                         // the units' headers for phase C: in the identity layout unit u
                         // is the u-th costliest transformation (at its own position),
                         // else the transformation at position u
+                        if (all && lane == 0) {
+                            const uint32_t km = I.n_kernels == 32 ? 0xffffffffu : (1u << I.n_kernels) - 1u;
+                            sm.tinf[b1] = make_uint4(I.kx_base, I.n_xforms, (I.per_iter_mask & km) != km, 0u);
+                        }
                         if (all && (uint32_t)lane < CXT) {
                             uint4 h;
                             uint32_t pos;
