@@ -1990,6 +1990,8 @@ struct alignas(128) SweepSmem {
     uint4 uhdr[SW_NB][CX];               // per phase-C unit: its program header (xhdr layout) ...
     uint32_t upos[SW_NB][CX];            // ... and its position in the design points
     uint4 tinf[SW_NB];                   // the tile's skeleton: {kx_base, n_xforms, has run-once kernels, -}
+    uint32_t wsk[SW_NB][WARPS];          // (TWO) per warp tile: its design points' other skeleton, or SW_BAD
+    uint8_t dsk[SW_NB][SW_GROUPS];       // (TWO) per design point: 1 = the tile's second skeleton
     uint32_t ab_cnt[4];                  // A/B task claims of the tile of sequence number mod 4
     uint32_t a_done[2];                  // phase-A completions of the tile of sequence parity p
     uint32_t tile_id[4];                 // the CTA's tiles by sequence number mod 4 (claimed ahead)
@@ -2085,7 +2087,24 @@ __device__ __forceinline__ void issue_cta_copy(const Params &P, uint32_t (*rec)[
 // in the same order as the tile's first design point (any fixed order of
 // valid transformations); warp-uniform result.  The batch's last warp tile
 // may hold gw < 32 design points: lanes past it stand in for design point 0.
-template <int CXT, unsigned long long ROW>   // design-point size; staged array length
+// A design point that differs from the tile's first in its skx: equal
+// transformations record by record and one skeleton for all its records
+// (which may be another than the first design point's: a tile's second
+// skeleton, sweep_kernel<.., TWO>).  Out of line: rare.
+template <int NCK>
+__device__ __noinline__ uint32_t skx_relaxed(const uint4 *p, const uint4 *g, uint32_t r)
+{
+    uint32_t acc = 0, D = 0;
+#pragma unroll
+    for (int m = 0; m < NCK; m++) {
+        const uint4 v = p[(m + r) & (uint32_t)(NCK - 1)], w = g[(m + r) & (uint32_t)(NCK - 1)];
+        if (m == 0) D = (v.x ^ w.x) & 0xffff0000u;
+        acc |= (v.x ^ w.x ^ D) | (v.y ^ w.y ^ D) | (v.z ^ w.z ^ D) | (v.w ^ w.w ^ D);
+    }
+    return acc;
+}
+
+template <int CXT, bool TWO, unsigned long long ROW>   // design-point size; two skeletons; staged length
 __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t (*recs)[ROW], int warp,
                                               int lane, uint32_t gw, uint32_t &s0, uint32_t &n0, uint32_t &m0,
                                               uint32_t &i0)
@@ -2115,6 +2134,7 @@ __device__ __forceinline__ bool sweep_phase_a(const SpaceDev &S, const uint32_t 
 #pragma unroll
         for (int m = 0; m < NCK; m++)
             acc |= (v[m].x ^ w[m].x) | (v[m].y ^ w[m].y) | (v[m].z ^ w[m].z) | (v[m].w ^ w[m].w);
+        if (TWO && acc) acc = skx_relaxed<NCK>(p, g, r);   // (a second skeleton's design point)
 #else
         uint4 v[NCK];
 #pragma unroll
@@ -2239,7 +2259,8 @@ __device__ __noinline__ void sweep_bytes(const unsigned long long *poly, const g
 // buffer; rbar: records staged; tbar: usage-table decision).  The last warp
 // to finish phase A of a tile issues the TMA copy of the CTA's next tile
 // into the (single) record buffer.
-template <bool BEST, int CXT>   // CXT: records per design point (4, 8 or 16)
+template <bool BEST, int CXT, bool TWO>   // CXT: records per design point (4, 8 or 16); TWO: a
+                                          // tile may hold two skeletons
 __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Params P)
 {
     static_assert(CXT == 4 || CXT == 8 || CXT == 16, "design-point sizes of the sweep");
@@ -2324,6 +2345,17 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 uni = __all_sync(FULL, st == s_all || st == SW_EMPTY) && s_all != SW_BAD && s_all != SW_EMPTY &&
                       sm.perm_ok[b];
             }
+            // (TWO) the tile's second skeleton: the same in every warp tile that has one
+            uint32_t skB = SW_BAD;
+            if constexpr (TWO) {
+                const uint32_t wo = sm.wsk[b][lane & (WARPS - 1)];
+                if (uni && __any_sync(FULL, wo != SW_BAD)) {
+                    skB = __reduce_min_sync(FULL, wo);
+                    uni = skB == __reduce_max_sync(FULL, wo == SW_BAD ? 0u : wo) &&
+                          __all_sync(FULL, (uint32_t)lane >= CXT ||
+                                               (sm.perm[b][lane] & 0xffffu) < S.skel[skB].n_xforms);
+                }
+            }
             if (!uni) {
                 // its pass-2 chunks (CTILE records each), one per warp
                 if (lane == 0 && (unsigned)warp < CPT && (unsigned long long)warp * CTILE < (unsigned long long)ngt * CXT)
@@ -2331,8 +2363,8 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
             } else {
                 // the tile's skeleton (set by its first task)
                 const uint4 ti4 = sm.tinf[b];
-                const uint32_t kx_base = ti4.x, X = ti4.y;
-                const bool has_once = ti4.z != 0u;
+                uint32_t kx_base = ti4.x, X = ti4.y;
+                bool has_once = ti4.z != 0u;
                 const unsigned long long tbase = P.base + tile * SWT;
                 const uint32_t *cwb = cw_all + b * wmax * (uint32_t)SW_GROUPS;
                 // work slots whose grid may be unsaturated for one of the tile's
@@ -2342,6 +2374,18 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 uint32_t gk = 0;
 #pragma unroll
                 for (int w = 0; w < WARPS; w++) gk |= sm.smallw[b][w];
+                const bool mixed = TWO && skB != SW_BAD;
+                // (TWO) the units of each skeleton; a design point takes part only
+                // in its own skeleton's (dsk)
+#pragma unroll 1
+                for (uint32_t si = 0; si < (mixed ? 2u : 1u); si++) {
+                if (si) {   // the second skeleton's constants (from global memory: rare)
+                    const SkelInfo &IB = S.skel[skB];
+                    const uint32_t km = IB.n_kernels == 32 ? 0xffffffffu : (1u << IB.n_kernels) - 1u;
+                    kx_base = IB.kx_base;
+                    X = IB.n_xforms;
+                    has_once = (IB.per_iter_mask & km) != km;
+                }
                 // units in snake order over the warps (16 units: warp w takes w
                 // and 15 - w; in the identity layout the costliest transformation
                 // pairs with the cheapest)
@@ -2350,8 +2394,17 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     const unsigned u = (rr & 1u) ? (rr + 1u) * WARPS - 1u - (unsigned)warp : rr * WARPS + (unsigned)warp;
                     if (u >= UNITS) continue;
                     // the unit's transformation and position (set by the tile's first task)
-                    const uint4 hdr = sm.uhdr[b][u % CXT];
-                    const uint32_t pos = sm.upos[b][u % CXT];
+                    uint4 hdr = sm.uhdr[b][u % CXT];
+                    uint32_t pos = sm.upos[b][u % CXT];
+                    if (TWO && si) {
+                        if (sm.perm_ident[b]) {
+                            hdr = __ldg(&S.xhdru[kx_base + u % CXT]);
+                            pos = hdr.x;
+                        } else {
+                            pos = u % CXT;
+                            hdr = __ldg(&S.xhdr[kx_base + (sm.perm[b][pos] & 0xffffu)]);
+                        }
+                    }
                     const uint32_t x = hdr.x;
                     const uint32_t jb = u / CXT, xf = hdr.w & 0xffu;
 #if GROPHECY_XINF_SKIP
@@ -2477,14 +2530,20 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     const bool once = has_once || (xf & XINF_ONCE);
                     double cmin = inf;
                     int cj = -1;
-                    auto totals = [&](auto ONCE) {
+                    auto totals = [&](auto ONCE, auto MIXED) {
 #pragma unroll
                         for (int j = 0; j < NCH; j++) {
                             const int gj = 32 * ((int)jb * NCH + j) + lane;
                             double tk = __dmul_rn(sm.it[b][gj], ti[j]);
                             if constexpr (decltype(ONCE)::value) tk = __dadd_rn(to[j], tk);
                             const double2 thd = sm.thd[b][gj];
-                            const double tt = __dadd_rn(__dadd_rn(tk, thd.x), thd.y);
+                            double tt = __dadd_rn(__dadd_rn(tk, thd.x), thd.y);
+                            if constexpr (decltype(MIXED)::value) {
+                                // the other skeleton's design point (chain j = warp tile
+                                // jb*NCH + j; dsk is written for warp tiles holding the second)
+                                const uint32_t d = sm.wsk[b][(int)jb * NCH + j] == SW_BAD ? 0u : sm.dsk[b][gj];
+                                if (d != si) tt = __longlong_as_double(0x7ff0000000000000LL);
+                            }
                             // chains in increasing record index: strict < keeps the lowest
                             // (design points past a partial tile's end have tt = +inf)
                             if (tt < cmin) {
@@ -2493,8 +2552,13 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                             }
                         }
                     };
-                    if (once) totals(std::true_type{});
-                    else totals(std::false_type{});
+                    if (TWO && mixed) {
+                        if (once) totals(std::true_type{}, std::integral_constant<bool, TWO>{});
+                        else totals(std::false_type{}, std::integral_constant<bool, TWO>{});
+                    } else {
+                        if (once) totals(std::true_type{}, std::false_type{});
+                        else totals(std::false_type{}, std::false_type{});
+                    }
                     if (cj >= 0) {
                         const int gj = 32 * ((int)jb * NCH + cj) + lane;
                         const unsigned long long idx = tbase + (unsigned long long)gj * CXT + pos;
@@ -2504,6 +2568,7 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                         }
                     }
                 }
+                }   // skeletons
                 if (lane == 0) cnt_val += gw * (uint32_t)CXT;
             }
             __syncwarp();
@@ -2536,11 +2601,23 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                 const int gwi = (int)ngt - 32 * (int)q;
                 const uint32_t gw = gwi <= 0 ? 0u : (gwi >= 32 ? 32u : (uint32_t)gwi);
                 uint32_t s0 = 0, n0 = 0, m0 = 0, i0 = 0;
-                bool ok = gw ? sweep_phase_a<CXT>(S, sm.rec, (int)q, lane, gw, s0, n0, m0, i0) : false;
+                bool ok = gw ? sweep_phase_a<CXT, TWO>(S, sm.rec, (int)q, lane, gw, s0, n0, m0, i0) : false;
                 const uint32_t skel = s0 >> 16;
                 // the tile's transformation order (its first design point's skx)
                 uint32_t sq = 0;
                 if (q == 0 && lane < CXT) sq = sm.rec[0][lane];
+                // (TWO) the tile's first skeleton; at most one other among its design points
+                uint32_t skA = 0, omin = SW_BAD;
+                bool anyoth = false;
+                if constexpr (TWO) {
+                    skA = sm.rec[0][0] >> 16;
+                    const bool oth = (uint32_t)lane < gw && skel != skA;
+                    anyoth = __any_sync(FULL, oth);
+                    if (anyoth) {
+                        omin = __reduce_min_sync(FULL, oth ? skel : SW_BAD);
+                        if (omin != __reduce_max_sync(FULL, oth ? skel : 0u)) ok = false;   // three: pass 2
+                    }
+                }
                 __syncwarp();
                 if (lane == 0) {
                     // every read of the record buffer by this warp is done: the
@@ -2630,24 +2707,27 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                     if (q == 0) {
                         // the tile's first design point (lane 0's) is itself consistent:
                         // one skeleton, every transformation < n_xforms
-                        const bool okq = (uint32_t)lane >= CXT || ((sq >> 16) == skel && (sq & 0xffffu) < I.n_xforms);
+                        const bool okq = TWO ? ((uint32_t)lane >= CXT ||
+                                                ((sq >> 16) == skA && (sq & 0xffffu) < S.skel[skA].n_xforms))
+                                             : ((uint32_t)lane >= CXT || ((sq >> 16) == skel && (sq & 0xffffu) < I.n_xforms));
                         const bool all = __all_sync(FULL, okq);
                         if (lane == 0) sm.perm_ok[b1] = all;
                         // the units' headers for phase C: in the identity layout unit u
                         // is the u-th costliest transformation (at its own position),
                         // else the transformation at position u
+                        const SkelInfo &IA = TWO ? S.skel[skA] : I;   // the tile's first skeleton
                         if (all && lane == 0) {
-                            const uint32_t km = I.n_kernels == 32 ? 0xffffffffu : (1u << I.n_kernels) - 1u;
-                            sm.tinf[b1] = make_uint4(I.kx_base, I.n_xforms, (I.per_iter_mask & km) != km, 0u);
+                            const uint32_t km = IA.n_kernels == 32 ? 0xffffffffu : (1u << IA.n_kernels) - 1u;
+                            sm.tinf[b1] = make_uint4(IA.kx_base, IA.n_xforms, (IA.per_iter_mask & km) != km, 0u);
                         }
                         if (all && (uint32_t)lane < CXT) {
                             uint4 h;
                             uint32_t pos;
                             if (sm.perm_ident[b1]) {
-                                h = __ldg(&S.xhdru[I.kx_base + lane]);
+                                h = __ldg(&S.xhdru[IA.kx_base + lane]);
                                 pos = h.x;
                             } else {
-                                h = __ldg(&S.xhdr[I.kx_base + (sq & 0xffffu)]);
+                                h = __ldg(&S.xhdr[IA.kx_base + (sq & 0xffffu)]);
                                 pos = (uint32_t)lane;
                             }
                             sm.uhdr[b1][lane] = h;
@@ -2660,7 +2740,35 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                         const uint32_t stride = I.poly_stride, a8 = n0 >> 3, b8 = m0 >> 3;
                         const uint32_t cls = (n0 & 7u) * 8u + (m0 & 7u);
                         const uint32_t pm = I.poly_mask;
-                        if (I.polyf_base != POLY32_NONE) {
+                        if (TWO && __any_sync(FULL, I.polyf_base != POLY32_NONE && skel != sm.tbl_skel)) {
+                            // (a second skeleton in this warp tile) collectives first,
+                            // then the staged table or its global copy per lane
+                            const bool pf = I.polyf_base != POLY32_NONE;
+                            const unsigned long long bnd =
+                                (unsigned long long)I.polyf_cmax[0] + (unsigned long long)I.polyf_cmax[1] * a8 +
+                                (unsigned long long)I.polyf_cmax[2] * b8 +
+                                (unsigned long long)I.polyf_cmax[3] * ((unsigned long long)a8 * b8);
+                            const bool u32 = __all_sync(FULL, !pf || bnd < (1ull << 32));
+                            if (pf && skel == sm.tbl_skel) {
+                                if (u32) group_usage_s<true>(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
+                                else group_usage_s<false>(tbl + cls, I.polyf_nhd, a8, b8, P.pc, u);
+                            } else if (pf) {
+                                const int4 *tg = reinterpret_cast<const int4 *>(S.poly + I.polyf_base) + cls;
+                                if (u32) group_usage_s<true>(tg, I.polyf_nhd, a8, b8, P.pc, u);
+                                else group_usage_s<false>(tg, I.polyf_nhd, a8, b8, P.pc, u);
+                            } else if (I.poly32_base != POLY32_NONE) {
+                                group_usage32<GROPHECY_AU32>(reinterpret_cast<const int4 *>(S.poly + I.poly32_base) +
+                                                                 (size_t)cls * (2u * n_arrays),
+                                                             n_arrays, pm, a8, b8, P.pc,
+                                                             reinterpret_cast<const int4 *>(S.poly), u);
+                            } else if (stride > 4) {
+                                group_usage<true, 2>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride),
+                                                     stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
+                            } else {
+                                group_usage<false, 4>(S.poly + I.poly_base + (size_t)cls * (2u * n_arrays * stride),
+                                                      stride, n_arrays, pm, a8, b8, P.pc, S.poly, u);
+                            }
+                        } else if (I.polyf_base != POLY32_NONE) {
                             // the staged table is warp tile 0's skeleton: another
                             // skeleton makes the tile non-uniform (pass 2) anyway
                             ok = skel == sm.tbl_skel;
@@ -2688,13 +2796,15 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_SMINB) sweep_kernel(const Pa
                         }
                         sm.thd[b1][g] = make_double2(u.th, u.td);
                         sm.it[b1][g] = (double)i0;
+                        if (TWO && anyoth) sm.dsk[b1][g] = skel != skA;   // (read for such warp tiles only)
                     }
                 } else if (q == 0 && lane == 0) {
                     sm.perm_ok[b1] = 0u;   // (warp tile 0 is not canonical: the tile is not uniform)
                 }
                 if (lane == 0) {
-                    sm.wstat[b1][q] = gw == 0 ? SW_EMPTY : (ok ? skel : SW_BAD);
+                    sm.wstat[b1][q] = gw == 0 ? SW_EMPTY : (ok ? (TWO ? skA : skel) : SW_BAD);
                     sm.smallw[b1][q] = wsmall;
+                    if (TWO) sm.wsk[b1][q] = omin;
                 }
                 // design points past a partial tile's end: t_h2d = +inf makes their
                 // totals +inf (never below the running minimum in phase C)
@@ -2827,9 +2937,12 @@ static void set_smem_attrs()
     const int ss = (int)std::min<uint32_t>(
         SMEM_CTA_MAX, std::max<uint32_t>(sweep_smem_bytes(MAXK, 2u * GROPHECY_MAX_ARRAYS * POLY_CLASSES * 16u),
                                          (uint32_t)sizeof(CtaSmem)));
-    cudaFuncSetAttribute(sweep_kernel<true, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
-    cudaFuncSetAttribute(sweep_kernel<true, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
-    cudaFuncSetAttribute(sweep_kernel<true, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
+    cudaFuncSetAttribute(sweep_kernel<true, 4, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
+    cudaFuncSetAttribute(sweep_kernel<true, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
+    cudaFuncSetAttribute(sweep_kernel<true, 16, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
+    cudaFuncSetAttribute(sweep_kernel<true, 4, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
+    cudaFuncSetAttribute(sweep_kernel<true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
+    cudaFuncSetAttribute(sweep_kernel<true, 16, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
     done = true;
 }
 
@@ -2863,9 +2976,24 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
 
 // The sweep kernel for the space's design-point size.
 using SweepFn = void (*)(Params);
-static SweepFn sweep_fn(const grophecy_space *s)
+static SweepFn sweep_fn(const grophecy_space *s, bool two)
 {
-    return s->sweep_cx == 4 ? sweep_kernel<true, 4> : (s->sweep_cx == 8 ? sweep_kernel<true, 8> : sweep_kernel<true, 16>);
+    if (two)
+        return s->sweep_cx == 4 ? sweep_kernel<true, 4, true>
+                                : (s->sweep_cx == 8 ? sweep_kernel<true, 8, true> : sweep_kernel<true, 16, true>);
+    return s->sweep_cx == 4 ? sweep_kernel<true, 4, false>
+                            : (s->sweep_cx == 8 ? sweep_kernel<true, 8, false> : sweep_kernel<true, 16, false>);
+}
+
+// Two-skeleton sweep tiles pay a little on every tile and save the general
+// path on the tiles that straddle a skeleton boundary: worth it when a batch
+// has few tiles per skeleton (the boundary tiles are a visible share of the
+// work or of the latency).
+static bool sweep_two(const grophecy_space *s, unsigned long long n)
+{
+    if (const char *e = getenv("GROPHECY_SWEEP_TWO")) return atoi(e) != 0;   // test hook
+    const unsigned long long tiles = n / ((unsigned long long)SW_GROUPS * s->sweep_cx) + 1;
+    return s->dev.n_skels > 1 && tiles < 128ull * s->dev.n_skels;
 }
 
 // Dynamic shared memory of the (fused) sweep launch: its own layout, or the
@@ -2883,7 +3011,7 @@ static int sweep_grid(const grophecy_space *s, unsigned long long n)
     set_smem_attrs();
     if (!s->occ_sweep) {
         int o = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, sweep_fn(s), THREADS, sweep_launch_smem(s));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, sweep_fn(s, false), THREADS, sweep_launch_smem(s));
         const_cast<grophecy_space *>(s)->occ_sweep = o < 1 ? 1 : o;
     }
     const unsigned long long swt = (unsigned long long)SW_GROUPS * s->sweep_cx;   // records per CTA tile
@@ -2965,7 +3093,7 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
             cfg.numAttrs = 1;
             cfg.gridDim = dim3(sweep_grid(s, Q.n));
             cfg.dynamicSmemBytes = sweep_launch_smem(s);
-            e = cudaLaunchKernelEx(&cfg, sweep_fn(s), Q);
+            e = cudaLaunchKernelEx(&cfg, sweep_fn(s, sweep_two(s, Q.n)), Q);
             if (e != cudaSuccess) return cuda_fail(e, "projection (best) sweep launch");
             sm_->counters_clean = true;
             count_launch(1);
@@ -2975,7 +3103,7 @@ static int launch_passes(const grophecy_space *s, Params P, cudaStream_t st)
             // pass 1 alone (pass 2 launched below, programmatically dependent)
             const int grid_s = sweep_grid(s, Q.n);
             Q.sweep_kmax = s->max_wslots;
-            sweep_fn(s)<<<grid_s, THREADS, sweep_launch_smem(s), st>>>(Q);
+            sweep_fn(s, sweep_two(s, Q.n))<<<grid_s, THREADS, sweep_launch_smem(s), st>>>(Q);
             launches++;
         } else if (!BEST) {
             const int grid_c = grid_for(s, Q.n, 32, true);

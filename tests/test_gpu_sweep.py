@@ -135,8 +135,9 @@ def test_fewer_transformations_bench_layout(G, O, X):
     check(G, O, c["skeletons"], rec)
 
 
+@pytest.mark.parametrize("two", ["0", "1"])
 @pytest.mark.parametrize("grid", [1, 3])
-def test_many_tiles_per_cta(G, O, monkeypatch, grid):
+def test_many_tiles_per_cta(G, O, monkeypatch, grid, two):
     """A sweep grid of 1 or 3 CTAs (GROPHECY_SWEEP_GRID): every CTA runs
     dozens of tiles back to back through its per-tile barriers and counters,
     with the skeleton (the staged usage table) changing every 4 tiles,
@@ -151,6 +152,7 @@ def test_many_tiles_per_cta(G, O, monkeypatch, grid):
         for k in rec:
             rec[k][i:i + 16] = rec[k][i:i + 16][::-1]
     monkeypatch.setenv("GROPHECY_SWEEP_GRID", str(grid))
+    monkeypatch.setenv("GROPHECY_SWEEP_TWO", two)   # one- and two-skeleton tiles
     check(G, O, c["skeletons"], rec)
 
 
@@ -166,3 +168,22 @@ def test_interleaved_design_points_general_path(G, O):
     blk = (i // 32) * 32
     idx = np.where(blk + 32 <= n, blk + (i % 2) * 16 + (i % 32) // 2, i)
     check(G, O, c["skeletons"], {k: v[idx] for k, v in rec.items()}, index_base=base)
+
+
+@pytest.mark.parametrize("two", ["0", "1"])
+@pytest.mark.parametrize("name", ["c2", "c3"])
+def test_skeleton_boundaries_inside_tiles(G, O, monkeypatch, name, two):
+    """Skeleton boundaries inside CTA tiles and inside warp tiles (C2 / C3
+    prefixes re-cut so that every few tiles hold two skeletons, one tile three),
+    with two-skeleton sweep tiles on and off (GROPHECY_SWEEP_TWO); vs the oracle."""
+    c = R.config(name)
+    k = len(c["skeletons"])
+    # records of consecutive skeleton ranges, cut at design points 4096*t + 16*(37 + 11 t)
+    parts, start = [], 0
+    for t in range(min(k, 6)):
+        lo = (t * c["n"] // k) // 16 * 16
+        n_t = 4096 + 16 * (37 + 11 * t) if t != 3 else 16 * 5   # (a 5-design-point run: 3 skeletons in a tile)
+        parts.append(R.gen_records(c, lo, lo + n_t))
+    rec = {f: np.concatenate([p[f] for p in parts]) for f in parts[0]}
+    monkeypatch.setenv("GROPHECY_SWEEP_TWO", two)
+    check(G, O, c["skeletons"], rec)
