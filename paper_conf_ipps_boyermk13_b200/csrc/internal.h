@@ -237,6 +237,8 @@ struct grophecy_space {
     int grid_best, grid_eval;            // persistent grid sizes
     uint32_t max_kernels;                // largest kernel count of the space's skeletons
     uint32_t max_wslots;                 // largest work-slot count (SkelInfo::n_wslots)
+    int sweep_two_env;                   // test hooks read at creation: GROPHECY_SWEEP_TWO (-1: unset)
+    uint32_t sweep_grid_env;             // ... and GROPHECY_SWEEP_GRID (0: unset)
     uint32_t sweep_cx;                   // sweep kernel's design-point size (4, 8 or 16: the
                                          // skeletons' common n_xforms, else 16)
     int occ_canon;                       // pass-1 CTAs per SM (0 = not yet queried)

@@ -2991,7 +2991,7 @@ static SweepFn sweep_fn(const grophecy_space *s, bool two)
 // work or of the latency).
 static bool sweep_two(const grophecy_space *s, unsigned long long n)
 {
-    if (const char *e = getenv("GROPHECY_SWEEP_TWO")) return atoi(e) != 0;   // test hook
+    if (s->sweep_two_env >= 0) return s->sweep_two_env != 0;   // test hook
     const unsigned long long tiles = n / ((unsigned long long)SW_GROUPS * s->sweep_cx) + 1;
     return s->dev.n_skels > 1 && tiles < 128ull * s->dev.n_skels;
 }
@@ -3019,10 +3019,7 @@ static int sweep_grid(const grophecy_space *s, unsigned long long n)
     unsigned long long cap = (unsigned long long)s->grid_best * (unsigned long long)s->occ_sweep;
     if (cap > s->max_partials - 1) cap = s->max_partials - 1;   // last slot = result
     // test hook: a small grid makes every CTA run many tiles in sequence
-    if (const char *g = getenv("GROPHECY_SWEEP_GRID")) {
-        const long v = atol(g);
-        if (v > 0) cap = std::min<unsigned long long>(cap, (unsigned long long)v);
-    }
+    if (s->sweep_grid_env) cap = std::min<unsigned long long>(cap, s->sweep_grid_env);
     return (int)std::min(want, cap);
 }
 

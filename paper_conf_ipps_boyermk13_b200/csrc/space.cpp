@@ -1,3 +1,4 @@
+#include <cstdlib>
 // Host side of the C ABI: PCIe fit, design-space validation, per-(kernel,
 // transformation) constant precompute and device upload.
 //
@@ -805,6 +806,11 @@ int grophecy_space_create(const grophecy_skeleton_desc *skels, uint32_t n_skels,
                 ((info[q].polyf_nhd & 0xffffu) + (info[q].polyf_nhd >> 16)) * POLY_CLASSES * 16u);
     // the sweep's design points: records of one (skeleton, nx, ny, iters) for
     // every transformation, so their size is the skeletons' common n_xforms
+    // test hooks (read once per space, not per launch)
+    sp->sweep_two_env = -1;
+    if (const char *e = getenv("GROPHECY_SWEEP_TWO")) sp->sweep_two_env = atoi(e) != 0;
+    sp->sweep_grid_env = 0;
+    if (const char *e = getenv("GROPHECY_SWEEP_GRID")) sp->sweep_grid_env = (uint32_t)std::max(0, atoi(e));
     sp->sweep_cx = 16;
     {
         bool same = true;
