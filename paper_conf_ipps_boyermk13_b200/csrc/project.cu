@@ -2940,8 +2940,6 @@ static void set_smem_attrs()
     cudaFuncSetAttribute(sweep_kernel<true, 4, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
     cudaFuncSetAttribute(sweep_kernel<true, 8, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
     cudaFuncSetAttribute(sweep_kernel<true, 16, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
-    cudaFuncSetAttribute(sweep_kernel<true, 4, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
-    cudaFuncSetAttribute(sweep_kernel<true, 8, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
     cudaFuncSetAttribute(sweep_kernel<true, 16, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ss);
     done = true;
 }
@@ -2978,9 +2976,7 @@ static int grid_for(const grophecy_space *s, unsigned long long n, int per_sm_ca
 using SweepFn = void (*)(Params);
 static SweepFn sweep_fn(const grophecy_space *s, bool two)
 {
-    if (two)
-        return s->sweep_cx == 4 ? sweep_kernel<true, 4, true>
-                                : (s->sweep_cx == 8 ? sweep_kernel<true, 8, true> : sweep_kernel<true, 16, true>);
+    if (two && s->sweep_cx == 16) return sweep_kernel<true, 16, true>;   // (design points of 16 only)
     return s->sweep_cx == 4 ? sweep_kernel<true, 4, false>
                             : (s->sweep_cx == 8 ? sweep_kernel<true, 8, false> : sweep_kernel<true, 16, false>);
 }
