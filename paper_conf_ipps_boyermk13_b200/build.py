@@ -45,7 +45,7 @@ def build(force=False, verbose=False):
         cmd += ["-Xptxas", "-v"]
     if os.environ.get("GROPHECY_THREADS"):
         cmd += [f"-DGROPHECY_THREADS={int(os.environ['GROPHECY_THREADS'])}"]
-    for m in ("GROPHECY_CG", "GROPHECY_CMINB", "GROPHECY_AU32", "GROPHECY_SMINB", "GROPHECY_NCH", "GROPHECY_I2F_MAGIC", "GROPHECY_PHASE_TIMING", "GROPHECY_FUSED", "GROPHECY_PERM", "GROPHECY_XINF_SKIP", "GROPHECY_DISPATCH_TREE"):
+    for m in ("GROPHECY_CG", "GROPHECY_CMINB", "GROPHECY_AU32", "GROPHECY_SMINB", "GROPHECY_I2F_MAGIC", "GROPHECY_PHASE_TIMING", "GROPHECY_FUSED", "GROPHECY_PERM", "GROPHECY_XINF_SKIP", "GROPHECY_DISPATCH_TREE"):
         if os.environ.get(m):
             cmd += [f"-D{m}={int(os.environ[m])}"]
     if os.environ.get("GROPHECY_MINB"):

@@ -1930,10 +1930,9 @@ __global__ void __launch_bounds__(THREADS, GROPHECY_CMINB) canon_kernel(const Pa
 // boundary, any other layout) and the batch's tail go to pass 2.
 constexpr int SW_GROUPS = 32 * WARPS;                               // design points per CTA tile
 constexpr unsigned long long SW_TILE = (unsigned long long)SW_GROUPS * CX;   // records per CTA tile
-#ifndef GROPHECY_NCH
-#define GROPHECY_NCH 8
-#endif
-constexpr int NCH = GROPHECY_NCH;                                   // chains per lane (divides WARPS)
+// chains per lane: a phase-C unit covers the tile's 256 design points (lane l,
+// chain j: design point 32 j + l, i.e. chain j = warp tile j)
+constexpr int NCH = WARPS;
 
 constexpr uint32_t SW_BAD = 0xffffffffu, SW_EMPTY = 0xfffffffeu;
 #ifndef GROPHECY_SMINB
